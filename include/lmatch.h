@@ -1,0 +1,159 @@
+/* lmatch.h -- C ABI of the B200-native pointer-based locally dominant matching library.
+ *
+ * Computes the 1/2-approximate maximum weight matching of Mandulak et al., "Efficient Weighted
+ * Graph Matching on GPUs" (SC'24): the maximal *locally dominant* matching (Def. II.1,
+ * PAPER.md:46; Lemma II.1) reached by the pointer-based iteration of Algorithm 1
+ * (LD-SEQ) / Algorithms 2-3 (LD-GPU): every round each
+ * unmatched vertex points to its heaviest unmatched neighbour, mutually pointing pairs are
+ * matched, and matched vertices are retired until no pointer changes.
+ *
+ * Edge order (R1): the paper's "greater or equal" is made strict: at a
+ * vertex u, neighbour v beats v' iff w(u,v) > w(u,v') or (w equal and v > v').  This is the
+ * restriction of one global strict order on edges, so the result is the UNIQUE maximal locally
+ * dominant matching (= the sequential greedy matching) and is bit-identical for every
+ * run, GPU count, tile size and streaming configuration.
+ *
+ * Graph input (CSR "separate vertex, edge, and value arrays"):
+ *   csr_offsets  int64[n+1]  row pointers; offsets[0] = 0, non-decreasing, offsets[n] = m
+ *   col_idx      int32[m]    neighbour ids in [0, n); each undirected edge appears in both rows
+ *   weights      float32[m]  edge weights, finite and > 0 ("w : E -> R>0");
+ *                            w(u,v) must equal w(v,u)
+ *   n < 2^31 vertices; m = number of DIRECTED entries (= 2 x undirected edges).
+ *   Self-loops are ignored (the paper assumes a simple graph).  Repeated entries
+ *   (u,v) with equal weights are harmless.  Rows need not be sorted.
+ *
+ * Output: mate int32[n]; mate[u] = v if {u,v} is matched, -1 if u is unmatched
+ *   (Alg. 1/2 "Output: ... matching in mate array").
+ *
+ * Errors: every function returns an lmatch_status (0 = OK, < 0 = error).  The library never
+ * aborts and no C++ exception crosses this ABI; lmatch_last_error() returns a thread-local
+ * human-readable detail of the last failure on the calling thread.
+ *
+ * Ownership: all input arrays are caller-owned and only read during the call that receives them.
+ * The handle owns every device allocation and stream it creates.  One handle must not be used
+ * from two threads at once; distinct handles are independent.
+ */
+#ifndef LMATCH_H_
+#define LMATCH_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define LMATCH_ABI_VERSION 1
+
+#if defined(__GNUC__)
+#define LMATCH_API __attribute__((visibility("default")))
+#else
+#define LMATCH_API
+#endif
+
+typedef enum lmatch_status {
+  LMATCH_OK = 0,
+  LMATCH_EINVAL = -1, /* malformed CSR: offsets[0] != 0, decreasing offsets, offsets[n] != m,
+                         col out of [0,n), weight NaN/inf/<= 0/-0.0, NULL pointer, or
+                         (validate_level 2) an asymmetric graph */
+  LMATCH_ERANGE = -2, /* n >= 2^31 or n < 0 or m < 0 */
+  LMATCH_ENOMEM = -3, /* device or pinned-host allocation failed */
+  LMATCH_ECUDA = -4,  /* CUDA runtime / kernel failure (detail in lmatch_last_error) */
+  LMATCH_ENCCL = -5,  /* reserved for the multi-GPU exchange */
+  LMATCH_ESTATE = -6  /* misuse: NULL handle, size mismatch on reload, ... */
+} lmatch_status;
+
+/* Opaque handle: one graph resident on one GPU (packed adjacency + per-vertex state). */
+typedef struct lmatch_graph lmatch_graph;
+
+/* Options for lmatch_create_ex / lmatch_create_device.  Zero-initialise, then set fields;
+ * every zero field means "default". */
+typedef struct lmatch_opts {
+  int32_t device;          /* CUDA device ordinal; default (0 with flag unset) = current device.
+                              Set use_device = 1 to honour `device`. */
+  int32_t use_device;
+  int32_t validate_level;  /* 0 = default (1); 1 = ranges + weights + offsets;
+                              2 = also symmetry (64-bit multiset hash of (u,v,w) vs (v,u,w));
+                              -1 = skip validation (caller guarantees a valid CSR) */
+  int32_t timing;          /* 1 = record CUDA events per phase into lmatch_stats */
+  int64_t max_rounds;      /* 0 = default: n/2 + 2 (the strict order bounds rounds by n/2+1) */
+  int64_t upload_chunk;    /* entries per host->device upload chunk (0 = default 2^25) */
+  int32_t reserved[16];
+} lmatch_opts;
+
+/* Filled by lmatch_run / lmatch_run_device when non-NULL. */
+typedef struct lmatch_stats {
+  int64_t rounds;            /* pointing phases executed (round 1 = full sweep) */
+  int64_t matched_vertices;  /* 2 x |M| */
+  int64_t cardinality;       /* |M| */
+  double weight;             /* w(M) = sum of matched edge weights, fp64 */
+  int64_t entries_swept;     /* adjacency entries scanned over all rounds */
+  int64_t frontier_total;    /* sum over rounds >= 2 of |F_r| (vertices re-pointed) */
+  double ms_total;           /* (timing=1) lmatch_run_device body, device time */
+  double ms_sweep;           /* (timing=1) round-1 pointer sweep kernel alone */
+  double ms_rounds;          /* (timing=1) rounds >= 2 (pointer + match + compaction) */
+  double ms_round1_rest;     /* (timing=1) round-1 match + compaction */
+  double ms_finish;          /* (timing=1) mate materialisation + weight reduction */
+  int64_t sweep_launches;    /* kernel launches of the round-1 sweep (1) */
+  int64_t kernel_launches;   /* all kernel launches issued by this run */
+  int64_t reserved[8];
+} lmatch_stats;
+
+/* Library / ABI identification.  Returns LMATCH_ABI_VERSION. */
+LMATCH_API int lmatch_abi_version(void);
+
+/* Build a handle from HOST CSR arrays (copied to the device in chunks, packed into 64-bit
+ * (weight-bits << 32 | neighbour) keys, validated, and indexed for the round-1 sweep).
+ * `out` receives the handle (NULL on failure).  Equivalent to lmatch_create_ex(..., NULL, out). */
+LMATCH_API int lmatch_create(const int64_t* csr_offsets, const int32_t* col_idx, const float* weights,
+                  int64_t n, int64_t m, lmatch_graph** out);
+
+LMATCH_API int lmatch_create_ex(const int64_t* csr_offsets, const int32_t* col_idx, const float* weights,
+                     int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** out);
+
+/* Same, but the three arrays are DEVICE pointers on the selected device (e.g. torch tensors'
+ * data_ptr()).  No host<->device copies; `stream` (cudaStream_t, may be NULL = legacy default)
+ * orders the reads of the caller's arrays. */
+LMATCH_API int lmatch_create_device(const int64_t* d_offsets, const int32_t* d_col, const float* d_weights,
+                         int64_t n, int64_t m, const lmatch_opts* opts, void* stream,
+                         lmatch_graph** out);
+
+/* Re-upload a graph with the SAME n and m from host arrays into an existing handle (reuses all
+ * device buffers; used for end-to-end timing).  ESTATE if sizes differ. */
+LMATCH_API int lmatch_reload(lmatch_graph* g, const int64_t* csr_offsets, const int32_t* col_idx,
+                  const float* weights);
+
+/* Compute the matching.  mate_out: HOST int32[n], caller-allocated (pinned memory gives the
+ * fastest copy).  stats may be NULL.  Returns after mate_out is complete. */
+LMATCH_API int lmatch_run(lmatch_graph* g, int32_t* mate_out, lmatch_stats* stats);
+
+/* Compute the matching into a DEVICE int32[n] buffer on `stream` (cudaStream_t; NULL = the
+ * handle's own stream).  Synchronises `stream` before returning (the round loop reads the
+ * frontier size each round). */
+LMATCH_API int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_stats* stats);
+
+/* w(M) = sum over pairs {u, mate[u]} of w(u, mate[u]) in fp64, for ANY mate[]
+ * (host int32[n]).  EINVAL if mate[] is not a symmetric set of edges of the graph. */
+LMATCH_API int lmatch_weight(lmatch_graph* g, const int32_t* mate, double* out_weight);
+
+/* Same with a DEVICE mate buffer, ordered on `stream` (NULL = handle stream); synchronises. */
+LMATCH_API int lmatch_weight_device(lmatch_graph* g, const int32_t* d_mate, void* stream,
+                         double* out_weight);
+
+/* Graph facts: n, m, non-empty rows, device bytes held by the handle. Any pointer may be NULL. */
+LMATCH_API int lmatch_info(const lmatch_graph* g, int64_t* n, int64_t* m, int64_t* nonempty_rows,
+                int64_t* device_bytes);
+
+/* Release everything the handle owns.  NULL-safe. */
+LMATCH_API void lmatch_destroy(lmatch_graph* g);
+
+/* Static string for a status code. */
+LMATCH_API const char* lmatch_strerror(int status);
+
+/* Thread-local detail of the last error on this thread ("" if none). */
+LMATCH_API const char* lmatch_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* LMATCH_H_ */

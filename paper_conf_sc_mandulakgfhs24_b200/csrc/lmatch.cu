@@ -1,0 +1,603 @@
+// lmatch.cu -- C ABI (include/lmatch.h) over the sm_100a kernels in kernels.cuh.
+//
+// Host-side structure:
+//   lmatch_create*   A1 ingest: chunked H2D (2 streams, double-buffered staging) + pack/validate,
+//                    offsets check, non-empty-row index, sweep tile index.   (untimed)
+//   lmatch_run*      reset -> A2 round-1 sweep -> A4 match-all -> A6 compact-all ->
+//                    { A2 frontier pointer (per degree bin) -> A4 match -> A6 compact }* ->
+//                    A10 mate + A9 weight.  The loop ends when the next frontier is empty
+//                    (termination; R6).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <climits>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+
+#include "../../include/lmatch.h"
+#include "kernels.cuh"
+
+namespace {
+
+thread_local char g_err[512] = "";
+
+void set_err(const char* fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(g_err, sizeof g_err, fmt, ap);
+  va_end(ap);
+}
+
+#define CK(call)                                                                        \
+  do {                                                                                  \
+    cudaError_t e_ = (call);                                                            \
+    if (e_ != cudaSuccess) {                                                            \
+      set_err("%s:%d %s: %s", __FILE__, __LINE__, #call, cudaGetErrorString(e_));       \
+      return (e_ == cudaErrorMemoryAllocation) ? LMATCH_ENOMEM : LMATCH_ECUDA;          \
+    }                                                                                   \
+  } while (0)
+#define CKL() CK(cudaGetLastError())
+#define TRY(x)                 \
+  do {                         \
+    int s_ = (x);              \
+    if (s_ != LMATCH_OK) return s_; \
+  } while (0)
+
+// Round-1 sweep configuration (tuned on B200).
+constexpr int kSweepThreads = 128;
+constexpr int kSweepPer = 8;
+constexpr int kSweepStages = 4;
+using Sweep = lm::SweepCfg<kSweepThreads, kSweepPer, kSweepStages>;
+constexpr int64_t kTile = Sweep::kTile;
+
+constexpr int kFinBlocks = 592;  // 4 x 148 SMs: fixed => deterministic fp64 summation order
+constexpr int kFinThreads = 256;
+constexpr int kNumCounters = 2 * 8;
+
+int num_sms_cached = 0;
+
+}  // namespace
+
+struct lmatch_graph {
+  int device = 0;
+  cudaStream_t stream = nullptr;   // handle stream
+  cudaStream_t up[2] = {nullptr, nullptr};
+  int64_t n = 0, m = 0, n_nz = 0, ntiles = 0;
+  int validate_level = 1;
+  int timing = 0;
+  int64_t max_rounds = 0;
+  int64_t upload_chunk = 1ll << 25;
+  int sweep_grid = 0;
+  int num_sms = 148;
+  // graph
+  int64_t* offs = nullptr;
+  uint64_t* adj = nullptr;
+  int64_t* noffs = nullptr;
+  int32_t* nzr = nullptr;
+  int32_t* tile_nz = nullptr;
+  // state
+  uint64_t* best = nullptr;
+  uint32_t* bits = nullptr;
+  int32_t* L[2] = {nullptr, nullptr};
+  int32_t* F[lm::kBins] = {};
+  unsigned long long* counters = nullptr;  // 2 sets of 8
+  unsigned long long* h_counters = nullptr;  // pinned mirror
+  double* pw = nullptr;
+  long long* pc = nullptr;
+  double* res_w = nullptr;
+  long long* res_c = nullptr;
+  double* h_res = nullptr;  // pinned: [0] = w, [1] = c (as double bits... stored separately)
+  long long* h_resc = nullptr;
+  int32_t* mate_tmp = nullptr;
+  lm::PackErr* perr = nullptr;
+  unsigned* werr = nullptr;
+  // upload staging
+  int32_t* st_col[2] = {nullptr, nullptr};
+  float* st_w[2] = {nullptr, nullptr};
+  cudaEvent_t ev[8] = {};
+  int64_t device_bytes = 0;
+};
+
+namespace {
+
+template <class T>
+int dmalloc(lmatch_graph* g, T** p, size_t count) {
+  size_t bytes = std::max<size_t>(count * sizeof(T), 16);
+  cudaError_t e = cudaMalloc(reinterpret_cast<void**>(p), bytes);
+  if (e != cudaSuccess) {
+    set_err("cudaMalloc(%zu bytes): %s", bytes, cudaGetErrorString(e));
+    *p = nullptr;
+    return e == cudaErrorMemoryAllocation ? LMATCH_ENOMEM : LMATCH_ECUDA;
+  }
+  g->device_bytes += (int64_t)bytes;
+  return LMATCH_OK;
+}
+
+int grid_for(int64_t work, int threads, int max_blocks) {
+  int64_t b = (work + threads - 1) / threads;
+  if (b < 1) b = 1;
+  if (b > max_blocks) b = max_blocks;
+  return (int)b;
+}
+
+int check_args(const void* a, const void* b, const void* c, int64_t n, int64_t m) {
+  if (n < 0 || m < 0) { set_err("negative n (%lld) or m (%lld)", (long long)n, (long long)m); return LMATCH_ERANGE; }
+  if (n >= (int64_t)1 << 31) { set_err("n = %lld >= 2^31 (vertex ids are int32)", (long long)n); return LMATCH_ERANGE; }
+  if (!a || (m > 0 && (!b || !c))) { set_err("NULL input array"); return LMATCH_EINVAL; }
+  if (n == 0 && m > 0) { set_err("n == 0 with m > 0"); return LMATCH_EINVAL; }
+  return LMATCH_OK;
+}
+
+int alloc_all(lmatch_graph* g) {
+  const int64_t n = g->n, m = g->m;
+  TRY(dmalloc(g, &g->offs, (size_t)n + 1));
+  TRY(dmalloc(g, &g->adj, (size_t)m + 2));
+  TRY(dmalloc(g, &g->noffs, (size_t)n + 5));
+  TRY(dmalloc(g, &g->nzr, (size_t)n + 8));
+  g->ntiles = (m + kTile - 1) / kTile;
+  TRY(dmalloc(g, &g->tile_nz, (size_t)g->ntiles + 2));
+  TRY(dmalloc(g, &g->best, (size_t)n + 1));
+  TRY(dmalloc(g, &g->bits, (size_t)((n + 31) / 32) + 1));
+  for (int i = 0; i < 2; ++i) TRY(dmalloc(g, &g->L[i], (size_t)n + 1));
+  for (int b = 0; b < lm::kBins; ++b) TRY(dmalloc(g, &g->F[b], (size_t)n + 1));
+  TRY(dmalloc(g, &g->counters, kNumCounters));
+  TRY(dmalloc(g, &g->pw, kFinBlocks));
+  TRY(dmalloc(g, &g->pc, kFinBlocks));
+  TRY(dmalloc(g, &g->res_w, 1));
+  TRY(dmalloc(g, &g->res_c, 1));
+  TRY(dmalloc(g, &g->perr, 1));
+  TRY(dmalloc(g, &g->werr, 1));
+  CK(cudaHostAlloc(reinterpret_cast<void**>(&g->h_counters), kNumCounters * 8, cudaHostAllocDefault));
+  CK(cudaHostAlloc(reinterpret_cast<void**>(&g->h_res), 16, cudaHostAllocDefault));
+  CK(cudaHostAlloc(reinterpret_cast<void**>(&g->h_resc), 16, cudaHostAllocDefault));
+  // best[] = 0 for every vertex: empty rows are never written again (their pointer stays none)
+  CK(cudaMemsetAsync(g->best, 0, ((size_t)n + 1) * 8, g->stream));
+  return LMATCH_OK;
+}
+
+// Sweep index: non-empty rows (noffs, nzr) + tile -> first row.  Also validates offsets.
+int build_index(lmatch_graph* g, cudaStream_t st) {
+  const int64_t n = g->n, m = g->m;
+  if (n == 0) { g->n_nz = 0; return LMATCH_OK; }
+  const int64_t nb = (n + lm::kScanBlock - 1) / lm::kScanBlock;
+  int64_t* bs = nullptr;
+  int64_t* tot = nullptr;
+  TRY(dmalloc(g, &bs, (size_t)nb + 1));
+  TRY(dmalloc(g, &tot, 1));
+  lm::k_nz_count<<<(unsigned)nb, lm::kScanThreads, 0, st>>>(g->offs, n, bs);
+  CKL();
+  lm::k_scan_blocksums<<<1, 1024, 0, st>>>(bs, nb, tot);
+  CKL();
+  lm::k_nz_scatter<<<(unsigned)nb, lm::kScanThreads, 0, st>>>(g->offs, n, bs, g->nzr, g->noffs);
+  CKL();
+  int64_t h_tot = 0;
+  CK(cudaMemcpyAsync(&h_tot, tot, 8, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  g->n_nz = h_tot;
+  CK(cudaMemcpyAsync(g->noffs + h_tot, &m, 8, cudaMemcpyHostToDevice, st));
+  CK(cudaStreamSynchronize(st));
+  if (g->ntiles > 0) {
+    lm::k_tile_rows<<<grid_for(g->ntiles + 1, 256, 4096), 256, 0, st>>>(g->noffs, g->n_nz, g->ntiles,
+                                                                        kTile, g->tile_nz);
+    CKL();
+  }
+  CK(cudaStreamSynchronize(st));
+  cudaFree(bs);
+  cudaFree(tot);
+  g->device_bytes -= (int64_t)(nb + 1 + 1) * 8;
+  return LMATCH_OK;
+}
+
+int check_offsets(lmatch_graph* g, cudaStream_t st) {
+  if (g->n == 0) return LMATCH_OK;
+  lm::k_check_offsets<<<grid_for(g->n, 256, 8192), 256, 0, st>>>(g->offs, g->n, g->m, g->perr);
+  CKL();
+  lm::PackErr h{};
+  CK(cudaMemcpyAsync(&h, g->perr, sizeof h, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  if (h.bad_offsets != ULLONG_MAX) {
+    set_err("invalid csr_offsets near row %llu (need offsets[0]=0, non-decreasing, offsets[n]=m)",
+            h.bad_offsets);
+    return LMATCH_EINVAL;
+  }
+  return LMATCH_OK;
+}
+
+int reset_err(lmatch_graph* g, cudaStream_t st) {
+  lm::PackErr h{ULLONG_MAX, ULLONG_MAX};
+  CK(cudaMemcpyAsync(g->perr, &h, sizeof h, cudaMemcpyHostToDevice, st));
+  CK(cudaStreamSynchronize(st));
+  return LMATCH_OK;
+}
+
+int check_pack(lmatch_graph* g, cudaStream_t st) {
+  lm::PackErr h{};
+  CK(cudaMemcpyAsync(&h, g->perr, sizeof h, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  if (h.first_bad != ULLONG_MAX && g->validate_level >= 0) {
+    set_err("invalid entry %llu: col out of [0,n) or weight not finite > 0", h.first_bad);
+    return LMATCH_EINVAL;
+  }
+  if (g->validate_level >= 2 && g->n > 0) {
+    unsigned long long* acc = nullptr;
+    TRY(dmalloc(g, &acc, 1));
+    CK(cudaMemsetAsync(acc, 0, 8, st));
+    lm::k_symhash<<<grid_for(g->n * 8, 256, 8192), 256, 0, st>>>(g->offs, g->adj, g->n, acc);
+    CKL();
+    unsigned long long hv = 0;
+    CK(cudaMemcpyAsync(&hv, acc, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    cudaFree(acc);
+    g->device_bytes -= 16;
+    if (hv != 0) {
+      set_err("graph is not symmetric: multiset of (u,v,w) differs from (v,u,w)");
+      return LMATCH_EINVAL;
+    }
+  }
+  return LMATCH_OK;
+}
+
+// Host arrays -> device: offsets in one copy; col/w in chunks through two staging buffers on two
+// streams so the PCIe copy of chunk k+1 overlaps packing chunk k (LOADBATCH double buffering,
+// Alg. 2 L4-5 P:115-116).
+int upload_host(lmatch_graph* g, const int64_t* offsets, const int32_t* col, const float* w) {
+  const int64_t n = g->n, m = g->m;
+  TRY(reset_err(g, g->stream));
+  CK(cudaMemcpyAsync(g->offs, offsets, ((size_t)n + 1) * 8, cudaMemcpyHostToDevice, g->stream));
+  CK(cudaStreamSynchronize(g->stream));
+  if (g->validate_level >= 0) TRY(check_offsets(g, g->stream));
+  const int64_t C = g->upload_chunk;
+  if (m > 0 && !g->st_col[0]) {
+    for (int i = 0; i < 2; ++i) {
+      TRY(dmalloc(g, &g->st_col[i], (size_t)std::min(C, m)));
+      TRY(dmalloc(g, &g->st_w[i], (size_t)std::min(C, m)));
+    }
+  }
+  for (int64_t base = 0, k = 0; base < m; base += C, ++k) {
+    const int64_t cnt = std::min(C, m - base);
+    const int i = (int)(k & 1);
+    cudaStream_t s = g->up[i];
+    CK(cudaMemcpyAsync(g->st_col[i], col + base, (size_t)cnt * 4, cudaMemcpyHostToDevice, s));
+    CK(cudaMemcpyAsync(g->st_w[i], w + base, (size_t)cnt * 4, cudaMemcpyHostToDevice, s));
+    lm::k_pack<<<grid_for(cnt, 256, 16384), 256, 0, s>>>(g->st_col[i], g->st_w[i], cnt, n,
+                                                          g->adj + base, base, g->perr);
+    CKL();
+  }
+  CK(cudaStreamSynchronize(g->up[0]));
+  CK(cudaStreamSynchronize(g->up[1]));
+  TRY(check_pack(g, g->stream));
+  return LMATCH_OK;
+}
+
+int upload_device(lmatch_graph* g, const int64_t* d_offsets, const int32_t* d_col,
+                  const float* d_w, cudaStream_t st) {
+  const int64_t n = g->n, m = g->m;
+  TRY(reset_err(g, st));
+  CK(cudaMemcpyAsync(g->offs, d_offsets, ((size_t)n + 1) * 8, cudaMemcpyDeviceToDevice, st));
+  if (g->validate_level >= 0) TRY(check_offsets(g, st));
+  if (m > 0) {
+    lm::k_pack<<<grid_for(m, 256, 65536), 256, 0, st>>>(d_col, d_w, m, n, g->adj, 0, g->perr);
+    CKL();
+  }
+  TRY(check_pack(g, st));
+  return LMATCH_OK;
+}
+
+int finish_create(lmatch_graph* g, cudaStream_t st) {
+  TRY(build_index(g, st));
+  if (g->ntiles > 0) {
+    CK(cudaFuncSetAttribute(lm::k_sweep<kSweepThreads, kSweepPer, kSweepStages>,
+                            cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Sweep::kSmem));
+    int occ = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+        &occ, lm::k_sweep<kSweepThreads, kSweepPer, kSweepStages>, kSweepThreads, Sweep::kSmem));
+    if (occ < 1) occ = 1;
+    g->sweep_grid = (int)std::min<int64_t>(g->ntiles, (int64_t)occ * g->num_sms);
+  }
+  CK(cudaStreamSynchronize(st));
+  return LMATCH_OK;
+}
+
+int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** out,
+                  lmatch_graph** gp) {
+  lmatch_graph* g = new (std::nothrow) lmatch_graph();
+  if (!g) { set_err("host allocation failed"); return LMATCH_ENOMEM; }
+  *gp = g;
+  g->n = n;
+  g->m = m;
+  if (opts) {
+    if (opts->use_device) CK(cudaSetDevice(opts->device));
+    if (opts->validate_level != 0) g->validate_level = opts->validate_level;
+    g->timing = opts->timing;
+    g->max_rounds = opts->max_rounds;
+    if (opts->upload_chunk > 0) g->upload_chunk = (opts->upload_chunk + 3) & ~3ll;
+  }
+  CK(cudaGetDevice(&g->device));
+  CK(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, g->device));
+  if (g->max_rounds <= 0) g->max_rounds = n / 2 + 2;
+  CK(cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking));
+  CK(cudaStreamCreateWithFlags(&g->up[0], cudaStreamNonBlocking));
+  CK(cudaStreamCreateWithFlags(&g->up[1], cudaStreamNonBlocking));
+  for (auto& e : g->ev) CK(cudaEventCreate(&e));
+  TRY(alloc_all(g));
+  (void)out;
+  return LMATCH_OK;
+}
+
+}  // namespace
+
+// ============================================================================ public ABI
+extern "C" {
+
+int lmatch_abi_version(void) { return LMATCH_ABI_VERSION; }
+
+const char* lmatch_strerror(int status) {
+  switch (status) {
+    case LMATCH_OK: return "ok";
+    case LMATCH_EINVAL: return "invalid argument / malformed graph";
+    case LMATCH_ERANGE: return "size out of range";
+    case LMATCH_ENOMEM: return "out of memory";
+    case LMATCH_ECUDA: return "CUDA error";
+    case LMATCH_ENCCL: return "NCCL error";
+    case LMATCH_ESTATE: return "invalid state";
+    default: return "unknown status";
+  }
+}
+
+const char* lmatch_last_error(void) { return g_err; }
+
+void lmatch_destroy(lmatch_graph* g) {
+  if (!g) return;
+  cudaSetDevice(g->device);
+  if (g->stream) cudaStreamSynchronize(g->stream);
+  void* dev[] = {g->offs, g->adj, g->noffs, g->nzr, g->tile_nz, g->best, g->bits, g->L[0], g->L[1],
+                 g->counters, g->pw, g->pc, g->res_w, g->res_c, g->mate_tmp, g->perr, g->werr,
+                 g->st_col[0], g->st_col[1], g->st_w[0], g->st_w[1]};
+  for (void* p : dev) if (p) cudaFree(p);
+  for (auto p : g->F) if (p) cudaFree(p);
+  if (g->h_counters) cudaFreeHost(g->h_counters);
+  if (g->h_res) cudaFreeHost(g->h_res);
+  if (g->h_resc) cudaFreeHost(g->h_resc);
+  for (auto e : g->ev) if (e) cudaEventDestroy(e);
+  if (g->stream) cudaStreamDestroy(g->stream);
+  for (auto s : g->up) if (s) cudaStreamDestroy(s);
+  delete g;
+}
+
+int lmatch_create_ex(const int64_t* csr_offsets, const int32_t* col_idx, const float* weights,
+                     int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** out) {
+  if (!out) { set_err("out == NULL"); return LMATCH_EINVAL; }
+  *out = nullptr;
+  g_err[0] = 0;
+  int s = check_args(csr_offsets, col_idx, weights, n, m);
+  if (s) return s;
+  lmatch_graph* g = nullptr;
+  s = create_common(n, m, opts, out, &g);
+  if (!s) s = upload_host(g, csr_offsets, col_idx, weights);
+  if (!s) s = finish_create(g, g->stream);
+  if (s) { lmatch_destroy(g); return s; }
+  *out = g;
+  return LMATCH_OK;
+}
+
+int lmatch_create(const int64_t* csr_offsets, const int32_t* col_idx, const float* weights,
+                  int64_t n, int64_t m, lmatch_graph** out) {
+  return lmatch_create_ex(csr_offsets, col_idx, weights, n, m, nullptr, out);
+}
+
+int lmatch_create_device(const int64_t* d_offsets, const int32_t* d_col, const float* d_weights,
+                         int64_t n, int64_t m, const lmatch_opts* opts, void* stream,
+                         lmatch_graph** out) {
+  if (!out) { set_err("out == NULL"); return LMATCH_EINVAL; }
+  *out = nullptr;
+  g_err[0] = 0;
+  int s = check_args(d_offsets, d_col, d_weights, n, m);
+  if (s) return s;
+  lmatch_graph* g = nullptr;
+  s = create_common(n, m, opts, out, &g);
+  cudaStream_t st = stream ? (cudaStream_t)stream : (g ? g->stream : nullptr);
+  if (!s) {
+    // order the caller's stream (which produced the arrays) before our reads
+    cudaError_t e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) { set_err("stream sync: %s", cudaGetErrorString(e)); s = LMATCH_ECUDA; }
+  }
+  if (!s) s = upload_device(g, d_offsets, d_col, d_weights, st);
+  if (!s) s = finish_create(g, st);
+  if (s) { lmatch_destroy(g); return s; }
+  *out = g;
+  return LMATCH_OK;
+}
+
+int lmatch_reload(lmatch_graph* g, const int64_t* csr_offsets, const int32_t* col_idx,
+                  const float* weights) {
+  if (!g) { set_err("NULL handle"); return LMATCH_ESTATE; }
+  g_err[0] = 0;
+  int s = check_args(csr_offsets, col_idx, weights, g->n, g->m);
+  if (s) return s;
+  CK(cudaSetDevice(g->device));
+  TRY(upload_host(g, csr_offsets, col_idx, weights));
+  TRY(finish_create(g, g->stream));
+  return LMATCH_OK;
+}
+
+int lmatch_info(const lmatch_graph* g, int64_t* n, int64_t* m, int64_t* nonempty_rows,
+                int64_t* device_bytes) {
+  if (!g) { set_err("NULL handle"); return LMATCH_ESTATE; }
+  if (n) *n = g->n;
+  if (m) *m = g->m;
+  if (nonempty_rows) *nonempty_rows = g->n_nz;
+  if (device_bytes) *device_bytes = g->device_bytes;
+  return LMATCH_OK;
+}
+
+int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_stats* stats) {
+  if (!g) { set_err("NULL handle"); return LMATCH_ESTATE; }
+  if (!d_mate && g->n > 0) { set_err("d_mate == NULL"); return LMATCH_EINVAL; }
+  g_err[0] = 0;
+  CK(cudaSetDevice(g->device));
+  cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
+  const int64_t n = g->n;
+  const bool tm = g->timing && stats;
+  int64_t launches = 0, rounds = 0, swept = 0, ftot_all = 0;
+  unsigned long long* cset[2] = {g->counters, g->counters + 8};
+
+  if (tm) CK(cudaEventRecord(g->ev[0], st));
+  // ---- reset (bitmap, counters, tile-crossing rows' best)
+  const int64_t nwords = (n + 31) / 32;
+  lm::k_reset<<<grid_for(std::max(nwords, g->ntiles), 256, 4096), 256, 0, st>>>(
+      g->bits, nwords, g->best, g->tile_nz, g->noffs, g->nzr, g->ntiles, kTile, g->counters,
+      kNumCounters);
+  CKL();
+  ++launches;
+  if (tm) CK(cudaEventRecord(g->ev[1], st));
+  if (g->ntiles > 0 && n > 0) {
+    // ---- round 1: A2 full sweep (no bitmap test), A4 match-all, A6 compact-all
+    lm::SweepArgs A{g->adj, g->noffs, g->nzr, g->tile_nz, g->best, g->m, g->ntiles};
+    lm::k_sweep<kSweepThreads, kSweepPer, kSweepStages>
+        <<<g->sweep_grid, kSweepThreads, Sweep::kSmem, st>>>(A);
+    CKL();
+    ++launches;
+    if (tm) CK(cudaEventRecord(g->ev[2], st));
+    rounds = 1;
+    swept = g->m;
+    lm::k_match_all<<<grid_for(nwords * 32, 256, 65536), 256, 0, st>>>(g->best, n, g->bits);
+    CKL();
+    lm::BinLists Fl{};
+    for (int b = 0; b < lm::kBins; ++b) Fl.list[b] = g->F[b];
+    lm::k_compact<true><<<grid_for(n, 256, 65536), 256, 0, st>>>(
+        nullptr, nullptr, n, g->best, g->bits, g->offs, g->L[0], Fl, cset[0]);
+    CKL();
+    launches += 2;
+    CK(cudaMemcpyAsync(g->h_counters, cset[0], 64, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (tm) CK(cudaEventRecord(g->ev[3], st));
+    int cur = 0;
+    for (;;) {
+      const unsigned long long* hc = g->h_counters + 8 * cur;
+      int64_t fb[lm::kBins], ftot = 0;
+      for (int b = 0; b < lm::kBins; ++b) { fb[b] = (int64_t)hc[1 + b]; ftot += fb[b]; }
+      const int64_t lcnt = (int64_t)hc[0];
+      if (ftot == 0 || rounds >= g->max_rounds) break;
+      ++rounds;
+      swept += (int64_t)hc[1 + lm::kBins];
+      ftot_all += ftot;
+      // A2 frontier pointer phase, one launch per non-empty degree bin
+      if (fb[0]) { lm::k_point_group<4><<<grid_for(fb[0] * 4, 256, 65536), 256, 0, st>>>(g->F[0], cset[cur] + 1, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }
+      if (fb[1]) { lm::k_point_group<16><<<grid_for(fb[1] * 16, 256, 65536), 256, 0, st>>>(g->F[1], cset[cur] + 2, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }
+      if (fb[2]) { lm::k_point_group<32><<<grid_for(fb[2] * 32, 256, 65536), 256, 0, st>>>(g->F[2], cset[cur] + 3, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }
+      if (fb[3]) { lm::k_point_cta<256><<<(unsigned)std::min<int64_t>(fb[3], 65536), 256, 0, st>>>(g->F[3], cset[cur] + 4, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }
+      // A4 match
+      lm::k_match_list<<<grid_for(ftot, 256, 65536), 256, 0, st>>>(Fl, cset[cur] + 1, g->best, g->bits);
+      CKL();
+      // A6 compaction of the live list
+      const int nxt = cur ^ 1;
+      CK(cudaMemsetAsync(cset[nxt], 0, 64, st));
+      lm::k_compact<false><<<grid_for(lcnt, 256, 65536), 256, 0, st>>>(
+          g->L[cur], cset[cur], n, g->best, g->bits, g->offs, g->L[nxt], Fl, cset[nxt]);
+      CKL();
+      launches += 2;
+      CK(cudaMemcpyAsync(g->h_counters + 8 * nxt, cset[nxt], 64, cudaMemcpyDeviceToHost, st));
+      CK(cudaStreamSynchronize(st));
+      cur = nxt;
+    }
+  } else if (tm) {
+    CK(cudaEventRecord(g->ev[2], st));
+    CK(cudaEventRecord(g->ev[3], st));
+  }
+  if (tm) CK(cudaEventRecord(g->ev[4], st));
+  // ---- A10 mate[] + A9 w(M)
+  if (n > 0) {
+    lm::k_materialize<kFinThreads><<<kFinBlocks, kFinThreads, 0, st>>>(g->best, g->bits, n, d_mate,
+                                                                       g->pw, g->pc);
+    CKL();
+    lm::k_final_sum<<<1, 32, 0, st>>>(g->pw, g->pc, kFinBlocks, g->res_w, g->res_c);
+    CKL();
+    launches += 2;
+    CK(cudaMemcpyAsync(g->h_res, g->res_w, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(g->h_resc, g->res_c, 8, cudaMemcpyDeviceToHost, st));
+  } else {
+    g->h_res[0] = 0.0;
+    g->h_resc[0] = 0;
+  }
+  if (tm) CK(cudaEventRecord(g->ev[5], st));
+  CK(cudaStreamSynchronize(st));
+  if (stats) {
+    std::memset(stats, 0, sizeof *stats);
+    stats->rounds = rounds;
+    stats->matched_vertices = g->h_resc[0];
+    stats->cardinality = g->h_resc[0] / 2;
+    stats->weight = g->h_res[0];
+    stats->entries_swept = swept;
+    stats->frontier_total = ftot_all;
+    stats->sweep_launches = (g->ntiles > 0 && n > 0) ? 1 : 0;
+    stats->kernel_launches = launches;
+    if (tm) {
+      float a = 0, b = 0, c = 0, d = 0, e = 0;
+      CK(cudaEventElapsedTime(&a, g->ev[0], g->ev[5]));
+      CK(cudaEventElapsedTime(&b, g->ev[1], g->ev[2]));
+      CK(cudaEventElapsedTime(&c, g->ev[2], g->ev[3]));
+      CK(cudaEventElapsedTime(&d, g->ev[3], g->ev[4]));
+      CK(cudaEventElapsedTime(&e, g->ev[4], g->ev[5]));
+      stats->ms_total = a;
+      stats->ms_sweep = b;
+      stats->ms_round1_rest = c;
+      stats->ms_rounds = d;
+      stats->ms_finish = e;
+    }
+  }
+  return LMATCH_OK;
+}
+
+int lmatch_run(lmatch_graph* g, int32_t* mate_out, lmatch_stats* stats) {
+  if (!g) { set_err("NULL handle"); return LMATCH_ESTATE; }
+  if (!mate_out && g->n > 0) { set_err("mate_out == NULL"); return LMATCH_EINVAL; }
+  CK(cudaSetDevice(g->device));
+  if (!g->mate_tmp) TRY(dmalloc(g, &g->mate_tmp, (size_t)g->n + 1));
+  TRY(lmatch_run_device(g, g->mate_tmp, g->stream, stats));
+  if (g->n > 0) {
+    CK(cudaMemcpyAsync(mate_out, g->mate_tmp, (size_t)g->n * 4, cudaMemcpyDeviceToHost, g->stream));
+    CK(cudaStreamSynchronize(g->stream));
+  }
+  return LMATCH_OK;
+}
+
+int lmatch_weight_device(lmatch_graph* g, const int32_t* d_mate, void* stream, double* out_weight) {
+  if (!g) { set_err("NULL handle"); return LMATCH_ESTATE; }
+  if (!out_weight || (!d_mate && g->n > 0)) { set_err("NULL argument"); return LMATCH_EINVAL; }
+  g_err[0] = 0;
+  CK(cudaSetDevice(g->device));
+  cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
+  if (g->n == 0) { *out_weight = 0.0; return LMATCH_OK; }
+  CK(cudaMemsetAsync(g->werr, 0, 4, st));
+  lm::k_weight_any<kFinThreads><<<kFinBlocks, kFinThreads, 0, st>>>(d_mate, g->n, g->offs, g->adj,
+                                                                    g->pw, g->pc, g->werr);
+  CKL();
+  lm::k_final_sum<<<1, 32, 0, st>>>(g->pw, g->pc, kFinBlocks, g->res_w, g->res_c);
+  CKL();
+  unsigned herr = 0;
+  CK(cudaMemcpyAsync(g->h_res, g->res_w, 8, cudaMemcpyDeviceToHost, st));
+  CK(cudaMemcpyAsync(&herr, g->werr, 4, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  if (herr) {
+    set_err("mate[] is not a matching of the graph (%s%s%s)", (herr & 1) ? "id out of range/self " : "",
+            (herr & 2) ? "asymmetric " : "", (herr & 4) ? "pair is not an edge" : "");
+    return LMATCH_EINVAL;
+  }
+  *out_weight = g->h_res[0];
+  return LMATCH_OK;
+}
+
+int lmatch_weight(lmatch_graph* g, const int32_t* mate, double* out_weight) {
+  if (!g) { set_err("NULL handle"); return LMATCH_ESTATE; }
+  if (!out_weight || (!mate && g->n > 0)) { set_err("NULL argument"); return LMATCH_EINVAL; }
+  CK(cudaSetDevice(g->device));
+  if (!g->mate_tmp) TRY(dmalloc(g, &g->mate_tmp, (size_t)g->n + 1));
+  if (g->n > 0)
+    CK(cudaMemcpyAsync(g->mate_tmp, mate, (size_t)g->n * 4, cudaMemcpyHostToDevice, g->stream));
+  return lmatch_weight_device(g, g->mate_tmp, g->stream, out_weight);
+}
+
+}  // extern "C"

@@ -1,0 +1,221 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the oracle, element by element.
+
+Bar: mate[] bit-exact (integer result); lmatch_stats.rounds equal to the
+frontier-driven Alg. 1 oracle's pointing phases; w(M) within 1e-9 relative of the oracle's fp64
+Neumaier sum (both sum exact fp32 values in fp64; only the summation order differs).
+"""
+import math
+
+import numpy as np
+import pytest
+
+import graphgen
+import oracle
+from helpers import golden_names, load_golden
+
+pytestmark = pytest.mark.gpu
+
+WTOL = 1e-9
+
+
+@pytest.fixture(scope="module")
+def lm():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_sc_mandulakgfhs24_b200 as p
+    return p
+
+
+def run_gpu(lm, g, **kw):
+    with lm.Matcher(g, **kw) as M:
+        mate, st = M.run()
+        return mate, st
+
+
+def check_parity(lm, g, rounds=True, **kw):
+    mate, st = run_gpu(lm, g, **kw)
+    ref = oracle.greedy(g)
+    bad = np.flatnonzero(mate != ref.mate)
+    assert bad.size == 0, f"{g.name}: {bad.size} mismatches, first {bad[:5]} gpu={mate[bad[:5]]} ref={ref.mate[bad[:5]]}"
+    assert st["cardinality"] == ref.cardinality
+    assert math.isclose(st["weight"], ref.weight, rel_tol=WTOL, abs_tol=1e-300)
+    if rounds:
+        _, ph, _ = oracle.ld_frontier(g)
+        assert st["rounds"] == ph, (st["rounds"], ph)
+    return mate, st
+
+
+@pytest.mark.parametrize("name", golden_names())
+def test_golden(lm, name):
+    g, mate, phases, weight = load_golden(name)
+    got, st = run_gpu(lm, g)
+    np.testing.assert_array_equal(got, mate)
+    assert st["rounds"] == phases
+    assert math.isclose(st["weight"], weight, rel_tol=1e-12)
+
+
+def test_empty_and_trivial(lm):
+    g = graphgen.from_edges(7, [])
+    mate, st = run_gpu(lm, g)
+    assert (mate == -1).all() and st["rounds"] == 0 and st["weight"] == 0
+    g = graphgen.from_edges(2, [(0, 1, 0.5)])
+    mate, st = run_gpu(lm, g)
+    assert list(mate) == [1, 0] and st["rounds"] == 1
+    g = graphgen.from_edges(3, [(1, 1, 0.5)])  # only a self-loop
+    mate, st = run_gpu(lm, g)
+    assert (mate == -1).all() and st["rounds"] == 1
+
+
+def test_random_tiny_many(lm):
+    rng = np.random.default_rng(17)
+    for _ in range(60):
+        n = int(rng.integers(2, 40))
+        g = graphgen.random_small(n, float(rng.choice([.1, .3, .7])), rng,
+                                  levels=int(rng.choice([0, 2, 5])) or None)
+        check_parity(lm, g)
+
+
+def test_increasing_path_rounds(lm):
+    for n in (2, 3, 17, 64, 301):
+        g = graphgen.from_edges(n, [(i, i + 1, float(i + 1)) for i in range(n - 1)])
+        _, st = check_parity(lm, g)
+        assert st["rounds"] == n // 2 + (n % 2)
+
+
+@pytest.mark.parametrize("maker", [
+    lambda: graphgen.er(1 << 16, 16.0, seed=1),                       # config 1 (PR1 ref)
+    lambda: graphgen.er(1 << 14, 16.0, seed=2, weights="paper"),      # 3-decimal ties
+    lambda: graphgen.er(5000, 30.0, seed=3, weights="ones"),          # ties only
+    lambda: graphgen.rmat(12, 16, seed=1),
+    lambda: graphgen.rmat(16, 16, seed=1),
+    lambda: graphgen.rmat(18, 16, seed=2),
+    lambda: graphgen.rmat(15, 16, seed=4, weights="paper"),
+    lambda: graphgen.mesh(256, seed=1),                                # uniform mesh
+    lambda: graphgen.mesh(300, keep=0.6, seed=1),                      # road-like
+    lambda: graphgen.mesh(64, seed=1, weights="gradient"),             # many rounds (~2*side)
+    lambda: graphgen.mesh(97, keep=0.6, seed=5, weights="ones"),
+])
+def test_synthetic_parity(lm, maker):
+    check_parity(lm, maker())
+
+
+def test_hub_rows_span_many_tiles(lm):
+    """Rows much longer than a sweep tile (merged with atomicMax across tiles), plus ragged
+    tails: a double star with 20k + 7k leaves and a sprinkling of random edges."""
+    rng = np.random.default_rng(3)
+    edges = [(0, v, float(np.float32(rng.random() * 0.5 + 0.25))) for v in range(2, 20002)]
+    edges += [(1, v, float(np.float32(rng.random()))) for v in range(15000, 22001)]
+    for _ in range(5000):
+        u, v = rng.integers(2, 22001, size=2)
+        if u != v:
+            edges.append((int(u), int(v), float(np.float32(1 - rng.random()))))
+    g = graphgen.from_edges(22001, edges)
+    check_parity(lm, g)
+    # a single hub with equal weights: the largest leaf id must win
+    g = graphgen.from_edges(9001, [(0, v, 1.0) for v in range(1, 9001)])
+    mate, _ = check_parity(lm, g)
+    assert mate[0] == 9000
+
+
+def test_chunked_upload_invariance(lm):
+    g = graphgen.rmat(14, 16, seed=7)
+    a, _ = run_gpu(lm, g)
+    b, _ = run_gpu(lm, g, upload_chunk=1000)
+    np.testing.assert_array_equal(a, b)
+    np.testing.assert_array_equal(a, oracle.greedy(g).mate)
+
+
+def test_repeat_runs_deterministic(lm):
+    g = graphgen.rmat(15, 16, seed=8)
+    with lm.Matcher(g) as M:
+        a, s1 = M.run()
+        b, s2 = M.run()
+    np.testing.assert_array_equal(a, b)
+    assert s1["weight"] == s2["weight"] and s1["rounds"] == s2["rounds"]
+
+
+def test_device_api_and_weight(lm):
+    import torch
+    g = graphgen.rmat(13, 16, seed=9)
+    dev = torch.device("cuda")
+    d_off = torch.from_numpy(g.offsets).to(dev)
+    d_col = torch.from_numpy(g.col).to(dev)
+    d_w = torch.from_numpy(g.w).to(dev)
+    M = lm.Matcher.from_device(d_off, d_col, d_w, g.n, g.m, stream=torch.cuda.current_stream())
+    d_mate = torch.empty(g.n, dtype=torch.int32, device=dev)
+    st = M.run_device(d_mate, stream=torch.cuda.current_stream())
+    ref = oracle.greedy(g)
+    np.testing.assert_array_equal(d_mate.cpu().numpy(), ref.mate)
+    assert math.isclose(st["weight"], ref.weight, rel_tol=WTOL)
+    # lmatch_weight on arbitrary mates: the oracle's, and an unmatched-everything mate
+    assert math.isclose(M.weight(ref.mate), ref.weight, rel_tol=WTOL)
+    assert M.weight(np.full(g.n, -1, np.int32)) == 0.0
+    assert math.isclose(lm.lmatch_weight_device(M.h, d_mate), ref.weight, rel_tol=WTOL)
+    # a different valid matching: drop one pair
+    other = ref.mate.copy()
+    u = int(np.flatnonzero(other >= 0)[0]); v = int(other[u])
+    other[u] = other[v] = -1
+    assert math.isclose(M.weight(other), oracle.weight(g, other), rel_tol=WTOL)
+    # invalid mates
+    bad = ref.mate.copy(); bad[u] = (v + 1) % g.n
+    with pytest.raises(lm.LMatchError):
+        M.weight(bad)
+    M.close()
+
+
+def test_reload(lm):
+    g1 = graphgen.er(4096, 8.0, seed=1)
+    g2 = graphgen.er(4096, 8.0, seed=1, wseed=99)  # same structure, new weights
+    with lm.Matcher(g1) as M:
+        a, _ = M.run()
+        M.reload(g2.offsets, g2.col, g2.w)
+        b, _ = M.run()
+    np.testing.assert_array_equal(a, oracle.greedy(g1).mate)
+    np.testing.assert_array_equal(b, oracle.greedy(g2).mate)
+
+
+def test_validation_errors(lm):
+    g, _, _, _ = load_golden("k4.txt")
+    o, c, w = g.offsets, g.col, g.w
+
+    def status(o, c, w, level=1, n=None, m=None):
+        try:
+            M = lm.Matcher(o, c, w, validate_level=level) if n is None else None
+            if M is None:
+                lm.lmatch_destroy(lm.lmatch_create(o, c, w, n, m))
+            else:
+                M.close()
+            return 0
+        except lm.LMatchError as e:
+            return e.status
+
+    assert status(o, c, w) == 0
+    o2 = o.copy(); o2[0] = 1
+    assert status(o2, c, w) == lm.LMATCH_EINVAL
+    o2 = o.copy(); o2[2] = o2[3] + 1
+    assert status(o2, c, w) == lm.LMATCH_EINVAL
+    c2 = c.copy(); c2[0] = 4
+    assert status(o, c2, w) == lm.LMATCH_EINVAL
+    for bad in (0.0, -0.0, -1.0, float("nan"), float("inf")):
+        w2 = w.copy(); w2[1] = bad
+        assert status(o, c, w2) == lm.LMATCH_EINVAL, bad
+    w2 = w.copy(); w2[0] = 0.123
+    assert status(o, c, w2, level=1) == 0
+    assert status(o, c, w2, level=2) == lm.LMATCH_EINVAL
+    assert status(o, c, w, level=2) == 0
+    # oracle agrees on every case above
+    assert oracle.validate(o, c, w2, 4, g.m, level=2)[0] == -1
+
+
+@pytest.mark.slow
+def test_full_size_rmat24_certificate(lm):
+    """configs[1] at full size: R-MAT scale 24, edge factor 16.  mate[] checked exactly with the
+    O(m) certificate (C(M) holds iff M is the unique LD matching) and w(M) against the oracle's
+    fp64 weight of the same mate[]."""
+    g = graphgen.rmat(24, 16, seed=1)
+    mate, st = run_gpu(lm, g)
+    code, bad = oracle.certificate(g, mate)
+    assert code == 0, (code, bad)
+    assert math.isclose(st["weight"], oracle.weight(g, mate), rel_tol=WTOL)
+    assert st["cardinality"] == int((mate >= 0).sum()) // 2
