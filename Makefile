@@ -9,7 +9,7 @@ LIB       := $(PKG)/liblmatch.so
 SRCS      := $(PKG)/csrc/lmatch.cu
 HDRS      := $(PKG)/csrc/kernels.cuh include/lmatch.h
 
-all: $(LIB) oracle/liboracle.so graphgen/libgraphgen.so
+all: $(LIB) oracle/liboracle.so graphgen/libgraphgen.so graphgen/libgraphgen_cuda.so
 
 $(LIB): $(SRCS) $(HDRS)
 	$(NVCC) $(NVFLAGS) -shared -Xlinker --exclude-libs=ALL $(SRCS) -o $@.tmp 2> $(PKG)/build.log || (cat $(PKG)/build.log; rm -f $@.tmp; exit 1)
@@ -19,8 +19,8 @@ $(LIB): $(SRCS) $(HDRS)
 oracle/liboracle.so: oracle/oracle.cpp
 	g++ -O2 -std=c++17 -fopenmp -fPIC -shared $< -o $@
 
-graphgen/libgraphgen.so: graphgen/graphgen.cpp
-	g++ -O3 -march=x86-64-v3 -std=c++17 -fopenmp -fPIC -shared $< -o $@
+graphgen/libgraphgen.so: graphgen/graphgen.cpp graphgen/gg_common.h
+	g++ -O3 -march=x86-64-v3 -ffp-contract=off -std=c++17 -fopenmp -fPIC -shared $< -o $@
 
 sass: $(LIB)
 	cuobjdump -sass $(LIB) > $(PKG)/liblmatch.sass
@@ -29,3 +29,6 @@ clean:
 	rm -f $(LIB) oracle/liboracle.so graphgen/libgraphgen.so $(PKG)/build.log
 
 .PHONY: all clean sass
+
+graphgen/libgraphgen_cuda.so: graphgen/graphgen_cuda.cu graphgen/gg_common.h
+	$(NVCC) -O3 -std=c++17 -fmad=false $(ARCH) -Xcompiler -fPIC -shared $< -o $@

@@ -1,0 +1,385 @@
+#!/usr/bin/env python
+"""bench.py -- matching edges/s (GTEPS) and % HBM roofline of the B200 LD-matching path.
+
+One step = one full matching (lmatch_run_device: reset, round-1 sweep, every frontier round,
+mate[] + w(M)) of a resident synthetic graph shaped like the paper's workloads (BASELINE.json
+configs; recipe in DESIGN.md).  GTEPS = undirected input edges m_u / step time / 1e9.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload rmat|er|mesh|road|gradient]
+                  [--scale S] [--impl ours|reference]
+
+N > 1 (torchrun, one rank per GPU): weak scaling over independent graph instances (rank r
+matches the seed+r instance of the same workload; no data-path collective).  The partitioned
+single-graph exchange is reported separately.
+
+--impl reference: the oracle (sequential greedy = the same unique matching) on the host cores,
+on a bounded sample of the workload (a smaller instance of the same generator recipe).
+Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "matching edges/s (GTEPS)"
+UNIT = "GTEPS"
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=20)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--workload", default="rmat", choices=["rmat", "er", "mesh", "road", "gradient"])
+    p.add_argument("--scale", type=int, default=None, help="log2(n) (rmat/er) or log2(n) of mesh")
+    p.add_argument("--edgefactor", type=int, default=16)
+    p.add_argument("--seed", type=int, default=1)
+    p.add_argument("--weights", default=None)
+    p.add_argument("--e2e-steps", type=int, default=3)
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-cpu", action="store_true")
+    p.add_argument("--cpu-scale", type=int, default=None)
+    p.add_argument("--gen", default="gpu", choices=["cpu", "gpu"])
+    return p.parse_args()
+
+
+DEFAULT_SCALE = {"rmat": 26, "er": 26, "mesh": 26, "road": 26, "gradient": 20}
+
+
+def make_graph_cpu(a, scale, seed):
+    import graphgen
+    wl = a.workload
+    if wl == "rmat":
+        return graphgen.rmat(scale, a.edgefactor, seed=seed, weights=a.weights or "uniform")
+    if wl == "er":
+        return graphgen.er(1 << scale, float(a.edgefactor), seed=seed, weights=a.weights or "uniform")
+    side = 1 << (scale // 2)
+    if wl == "mesh":
+        return graphgen.mesh(side, seed=seed, weights=a.weights or "uniform")
+    if wl == "road":
+        return graphgen.mesh(side, keep=0.6, seed=seed, weights=a.weights or "uniform")
+    return graphgen.mesh(side, seed=seed, weights="gradient")
+
+
+def make_graph_gpu(a, scale, seed, device):
+    import graphgen.gpu as gg
+    wl = a.workload
+    if wl == "rmat":
+        return gg.rmat(scale, a.edgefactor, seed=seed, weights=a.weights or "uniform", device=device)
+    if wl == "er":
+        return gg.er(1 << scale, float(a.edgefactor), seed=seed, weights=a.weights or "uniform",
+                     device=device)
+    side = 1 << (scale // 2)
+    if wl == "mesh":
+        return gg.mesh(side, seed=seed, weights=a.weights or "uniform", device=device)
+    if wl == "road":
+        return gg.mesh(side, keep=0.6, seed=seed, weights=a.weights or "uniform", device=device)
+    return gg.mesh(side, seed=seed, weights="gradient", device=device)
+
+
+def workload_config(a, scale, n, m):
+    cfg = {"workload": {"rmat": "R-MAT/Graph500 (A,B,C=.57,.19,.19), random relabel",
+                        "er": "Erdos-Renyi", "mesh": "2-D 4-neighbour mesh",
+                        "road": "road-like mesh (60% of grid edges kept)",
+                        "gradient": "2-D mesh, gradient weights (many rounds)"}[a.workload],
+           "scale": scale, "n": int(n), "m_directed": int(m), "m_undirected": int(m // 2),
+           "weights": a.weights or ("gradient" if a.workload == "gradient" else "uniform fp32 (2^24 levels)"),
+           "seed": a.seed}
+    if a.workload in ("rmat", "er"):
+        cfg["edgefactor"] = a.edgefactor
+    return cfg
+
+
+# ----------------------------------------------------------------------------- clocks (NVML)
+class ClockSampler:
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+               0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
+               0x100: "display_clock_setting"}
+
+    def __init__(self, device_index: int, period_s: float = 0.005):
+        self.ok = False
+        self.samples, self.reasons = [], 0
+        self.period = period_s
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # pragma: no cover
+            self.err = str(e)
+
+    def _loop(self):
+        nv = self.nv
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                self.reasons |= nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.ok:
+            self._stop = threading.Event()
+            self._t = threading.Thread(target=self._loop, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *exc):
+        if self.ok:
+            self._stop.set()
+            self._t.join()
+
+    def summary(self):
+        if not self.ok or not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
+        names = [v for k, v in self.REASONS.items() if self.reasons & k and v != "gpu_idle"]
+        return {"sm_mhz": float(statistics.median(self.samples)), "sm_max_mhz": int(self.max_mhz),
+                "reasons": names, "samples": len(self.samples)}
+
+
+def load_peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        d = json.load(open(path))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs: torch copy_ best of 10)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s; MEASURED_PEAKS.json absent)"
+
+
+def load_traffic(config_key: str):
+    """dram bytes per sweep launch from the committed ncu --set full summary, if it matches."""
+    path = os.path.join(ROOT, "profiles", "sweep_traffic.json")
+    try:
+        d = json.load(open(path))
+        e = d.get(config_key)
+        return None if e is None else float(e["dram_bytes_per_launch"])
+    except Exception:
+        return None
+
+
+# ------------------------------------------------------------------------------ cpu baseline
+def cpu_baseline(a, sample_scale):
+    """The oracle (sequential greedy, single thread) on a bounded sample: a smaller instance of
+    the same generator recipe.  Returns a dict in the bench's metric/unit."""
+    import oracle
+    g = make_graph_cpu(a, sample_scale, a.seed)
+    oracle.threads(1)
+    r = oracle.greedy(g)
+    t = r.sort_s + r.scan_s
+    return {"value": g.m_u / t / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"{a.workload} scale {sample_scale} (n={g.n}, m_u={g.m_u}) same recipe/seed; "
+                      f"greedy sort {r.sort_s:.2f}s + scan {r.scan_s:.2f}s, 1 thread, std::sort",
+            "seconds": t}
+
+
+def cpu_sample_scale(a):
+    if a.cpu_scale:
+        return a.cpu_scale
+    return {"rmat": 20, "er": 20, "mesh": 20, "road": 20, "gradient": 18}[a.workload]
+
+
+# ------------------------------------------------------------------------------ reference arm
+def run_reference(a, rank, world):
+    if rank != 0:
+        return 0
+    import oracle
+    scale = cpu_sample_scale(a)
+    g = make_graph_cpu(a, scale, a.seed)
+    oracle.threads(1)
+    for _ in range(a.warmup):
+        oracle.greedy(g)
+    t0 = time.perf_counter()
+    tt = 0.0
+    for _ in range(a.steps):
+        r = oracle.greedy(g)
+        tt += r.sort_s + r.scan_s
+    wall = time.perf_counter() - t0
+    val = g.m_u * a.steps / tt / 1e9
+    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": world,
+            "steps": a.steps, "warmup": a.warmup, "ms_per_step": tt / a.steps * 1e3,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32-compare",
+            "data": "synthetic",
+            "config": workload_config(a, scale, g.n, g.m) | {"sample_of_scale": a.scale or DEFAULT_SCALE[a.workload]},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": f"{a.workload} scale {scale} instance of the workload recipe"},
+            "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+            "wall_s": wall}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# -------------------------------------------------------------------------------- our arm
+def main():
+    a = parse()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", str(a.gpus)))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if a.impl == "reference":
+        return run_reference(a, rank, world)
+
+    import torch
+    import torch.distributed as dist
+    if not torch.cuda.is_available():
+        raise SystemExit("bench.py needs a CUDA device (no CPU fallback)")
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    import paper_conf_sc_mandulakgfhs24_b200 as lm
+
+    scale = a.scale or DEFAULT_SCALE[a.workload]
+    seed = a.seed + rank
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream(dev)
+    t0 = time.time()
+    if a.gen == "cpu":
+        g = make_graph_cpu(a, scale, seed)
+        d_off = torch.from_numpy(g.offsets).to(dev)
+        d_col = torch.from_numpy(g.col).to(dev)
+        d_w = torch.from_numpy(g.w).to(dev)
+        n, m, m_u = g.n, g.m, g.m_u
+    else:
+        dg = make_graph_gpu(a, scale, seed, dev)
+        d_off, d_col, d_w = dg.offsets, dg.col, dg.w
+        n, m, m_u = dg.n, dg.m, dg.m_u
+        g = None
+    gen_s = time.time() - t0
+
+    # resident inputs: CSR on the device, handle built from device pointers (create is untimed,
+    # P:179 excludes I/O, allocation, CSR construction and the initial transfer)
+    opts = lm.make_opts(validate_level=1, timing=1)
+    h = lm.lmatch_create_device(d_off, d_col, d_w, n, m, opts, stream)
+    if g is None and not a.no_e2e:  # host copies for the end-to-end leg
+        import graphgen
+        g = graphgen.Graph(d_off.cpu().numpy(), d_col.cpu().numpy(), d_w.cpu().numpy())
+    del d_off, d_col, d_w
+    dg = None
+    torch.cuda.empty_cache()
+    d_mate = torch.empty(n, dtype=torch.int32, device=dev)
+
+    for _ in range(a.warmup):
+        lm.lmatch_run_device(h, d_mate, stream)
+    torch.cuda.synchronize(dev)
+    if world > 1:
+        dist.barrier()
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    sweep_ms, launches, rounds = [], 0, []
+    with ClockSampler(local) as clk:
+        torch.cuda.synchronize(dev)
+        ev0.record(stream)
+        for _ in range(a.steps):
+            st = lm.lmatch_run_device(h, d_mate, stream)
+            sweep_ms.append(st.ms_sweep)
+            launches += st.kernel_launches
+            rounds.append(st.rounds)
+        ev1.record(stream)
+        torch.cuda.synchronize(dev)
+    ms = ev0.elapsed_time(ev1)
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+        tot = torch.tensor([m_u], dtype=torch.float64, device=dev)
+        dist.all_reduce(tot)
+        total_mu = float(tot.item())
+    else:
+        total_mu = float(m_u)
+    ms_per_step = ms / a.steps
+    value = total_mu * a.steps / (ms / 1e3) / 1e9
+    last = st.as_dict()
+
+    # roofline of the dominant kernel: the round-1 sweep (one launch per step)
+    info = lm.lmatch_info(h)
+    n_nz = info["nonempty_rows"]
+    tile = 1024
+    ntiles = (m + tile - 1) // tile
+    sweep_bytes = 8 * m + 16 * n_nz + 4 * (ntiles + 1)  # keys + (start lo32, id, best) per row + tile index
+    sweep_avg_ms = float(np.mean(sweep_ms))
+    peak, peak_src = load_peaks()
+    achieved = sweep_bytes / (sweep_avg_ms / 1e3) / 1e9
+    key = f"{a.workload}_s{scale}_ef{a.edgefactor}_seed{a.seed}"
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": achieved / peak, "traffic": load_traffic(key),
+                "kernel": "k_sweep (round-1 pointer sweep, TMA-staged)",
+                "algorithmic_bytes_per_launch": int(sweep_bytes), "launch_ms": sweep_avg_ms,
+                "share_of_step": sweep_avg_ms / ms_per_step, "peak_source": peak_src}
+
+    # end-to-end through the public C ABI with host buffers (pinned): reload + run + mate D2H
+    e2e = None
+    if not a.no_e2e and a.e2e_steps > 0:
+        cud = torch.cuda.cudart()
+        regs = []
+        for arr in (g.offsets, g.col, g.w):
+            if arr.nbytes:
+                cud.cudaHostRegister(arr.ctypes.data, arr.nbytes, 0)
+                regs.append(arr)
+        mate_h = torch.empty(n, dtype=torch.int32, pin_memory=True)
+        mate_np = mate_h.numpy()
+        lm.lmatch_reload(h, g.offsets, g.col, g.w)
+        lm.lmatch_run(h, mate_np)
+        torch.cuda.synchronize(dev)
+        if world > 1:
+            dist.barrier()
+        t1 = time.perf_counter()
+        for _ in range(a.e2e_steps):
+            lm.lmatch_reload(h, g.offsets, g.col, g.w)
+            lm.lmatch_run(h, mate_np)
+        el = time.perf_counter() - t1
+        if world > 1:
+            t = torch.tensor([el], dtype=torch.float64, device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            el = float(t.item())
+        for arr in regs:
+            cud.cudaHostUnregister(arr.ctypes.data)
+        e2e = {"value": total_mu * a.e2e_steps / el / 1e9, "unit": UNIT,
+               "h2d_bytes_per_step": int(g.offsets.nbytes + g.col.nbytes + g.w.nbytes),
+               "d2h_bytes_per_step": int(4 * n), "steps": a.e2e_steps,
+               "ms_per_step": el / a.e2e_steps * 1e3,
+               "includes": "lmatch_reload (H2D + pack + validate + index) + lmatch_run (+ mate D2H)"}
+
+    lm.lmatch_destroy(h)
+    del d_mate
+    torch.cuda.empty_cache()
+
+    cpu = None
+    if rank == 0 and world == 1 and not a.no_cpu:
+        cpu = cpu_baseline(a, cpu_sample_scale(a))
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps,
+                "warmup": a.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+                "data": "synthetic",
+                "config": workload_config(a, scale, n, m) | {
+                    "parallelism": "1 GPU" if world == 1 else f"{world} independent instances (seed+rank), no collective",
+                    "l2": f"inputs larger than L2 (adjacency {8 * m / 1e9:.1f} GB >> 126 MB); no flush",
+                    "gen_s": round(gen_s, 1)},
+                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+                "gpu_launches": int(launches), "clocks": clk.summary(),
+                "rounds": int(rounds[-1]), "cardinality": int(last["cardinality"]),
+                "matched_weight": last["weight"],
+                "phase_ms": {k: last[k] for k in ("ms_sweep", "ms_round1_rest", "ms_rounds",
+                                                  "ms_finish", "ms_total")}}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

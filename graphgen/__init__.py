@@ -18,6 +18,7 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SO = os.path.join(_HERE, "libgraphgen.so")
 _SRC = os.path.join(_HERE, "graphgen.cpp")
+_HDR = os.path.join(_HERE, "gg_common.h")
 _lib = None
 
 WEIGHT_MODES = {"uniform": 0, "paper": 1, "gradient": 2, "ones": 3}
@@ -25,8 +26,10 @@ WEIGHT_MODES = {"uniform": 0, "paper": 1, "gradient": 2, "ones": 3}
 
 def build(force: bool = False) -> str:
     """Compile libgraphgen.so (g++ -O3 -fopenmp)."""
-    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
-        cmd = ["g++", "-O3", "-march=x86-64-v3", "-std=c++17", "-fopenmp", "-fPIC", "-shared",
+    stale = not os.path.exists(_SO) or os.path.getmtime(_SO) < max(os.path.getmtime(_SRC),
+                                                                    os.path.getmtime(_HDR))
+    if force or stale:
+        cmd = ["g++", "-O3", "-march=x86-64-v3", "-ffp-contract=off", "-std=c++17", "-fopenmp", "-fPIC", "-shared",
                _SRC, "-o", _SO + ".tmp"]
         subprocess.check_call(cmd)
         os.replace(_SO + ".tmp", _SO)
@@ -50,8 +53,8 @@ def _load():
         lib.gg_mesh_csr.restype = i64
         lib.gg_weights.argtypes = [p, p, i64, u64, i32, i64, p]
         lib.gg_weights.restype = i32
-        lib.gg_hash2.argtypes = [u64, u64, u64]
-        lib.gg_hash2.restype = u64
+        lib.gg_hash.argtypes = [u64, u64, u64]
+        lib.gg_hash.restype = u64
         lib.gg_set_threads.argtypes = [i32]
         lib.gg_set_threads.restype = i32
         _lib = lib
@@ -183,7 +186,7 @@ def random_small(n: int, p: float, rng: np.random.Generator, levels: int | None 
 
 
 def hash2(seed: int, a: int, b: int) -> int:
-    return int(_load().gg_hash2(seed, a, b))
+    return int(_load().gg_hash(seed, a, b))
 
 
 def set_threads(t: int) -> int:

@@ -19,46 +19,12 @@
 #include <vector>
 #include <omp.h>
 
+#include "gg_common.h"
+
 namespace {
 
-inline uint64_t mix64(uint64_t x) {  // SplitMix64 finaliser
-  x += 0x9E3779B97F4A7C15ull;
-  x = (x ^ (x >> 30)) * 0xBF58476D1CE4E5B9ull;
-  x = (x ^ (x >> 27)) * 0x94D049BB133111EBull;
-  return x ^ (x >> 31);
-}
-inline uint64_t hash2(uint64_t seed, uint64_t a, uint64_t b) {
-  return mix64(mix64(mix64(seed) ^ a) ^ (b * 0xD6E8FEB86659FD93ull));
-}
-// Uniform integer in [0, n) from a 64-bit hash (multiply-high).
-inline uint64_t below(uint64_t h, uint64_t n) {
-  return (uint64_t)(((unsigned __int128)h * n) >> 64);
-}
-
-// Bijection on [0, 2^s): random relabelling of R-MAT ids without a table.
-struct Perm {
-  int s; uint64_t mask, k0, k1, c1, c2;
-  Perm(int s_, uint64_t seed) : s(s_) {
-    mask = (s >= 64) ? ~0ull : ((1ull << s) - 1);
-    k0 = mix64(seed ^ 0x1111) & mask;
-    k1 = mix64(seed ^ 0x2222) & mask;
-    c1 = mix64(seed ^ 0x3333) | 1ull;
-    c2 = mix64(seed ^ 0x4444) | 1ull;
-  }
-  uint64_t operator()(uint64_t x) const {
-    if (s <= 1) return x ^ (k0 & mask);
-    int h = (s + 1) / 2;
-    x = (x ^ k0) & mask;
-    x = (x * c1) & mask;
-    x ^= x >> h;
-    x = (x + k1) & mask;
-    x = (x * c2) & mask;
-    x ^= x >> (s / 2 > 0 ? s / 2 : 1);
-    x = (x * c1) & mask;
-    x ^= x >> h;
-    return x & mask;
-  }
-};
+inline uint64_t mix64(uint64_t x) { return gg_mix64(x); }
+inline uint64_t hash2(uint64_t seed, uint64_t a, uint64_t b) { return gg_hash2(seed, a, b); }
 
 // Builds a symmetric CSR from an edge generator gen(i, &u, &v) -> bool (false = skip),
 // i in [0, M).  Self-loops are dropped, rows are sorted ascending and deduplicated.
@@ -112,7 +78,7 @@ int64_t build_csr(int64_t n, int64_t M, Gen gen, int64_t* offsets, int32_t* col)
 
 extern "C" {
 
-uint64_t gg_hash2(uint64_t seed, uint64_t a, uint64_t b) { return hash2(seed, a, b); }
+uint64_t gg_hash(uint64_t seed, uint64_t a, uint64_t b) { return hash2(seed, a, b); }
 
 int gg_set_threads(int t) { if (t > 0) omp_set_num_threads(t); return omp_get_max_threads(); }
 
@@ -121,10 +87,9 @@ int64_t gg_er_csr(int64_t n, double avg_degree, uint64_t seed, int64_t* offsets,
                   int64_t cap) {
   int64_t M = (int64_t)std::llround((double)n * avg_degree / 2.0);
   if (2 * M > cap) return -1;
-  uint64_t s = mix64(seed ^ 0xE7u);
+  const GGEr er = gg_make_er(n, seed);
   auto gen = [=](int64_t i, int64_t* u, int64_t* v) {
-    *u = (int64_t)below(hash2(s, (uint64_t)i, 0), (uint64_t)n);
-    *v = (int64_t)below(hash2(s, (uint64_t)i, 1), (uint64_t)n);
+    er.edge(i, u, v);
     return true;
   };
   return build_csr(n, M, gen, offsets, col);
@@ -143,27 +108,9 @@ int64_t gg_rmat_csr(int scale, int64_t edgefactor, uint64_t seed, double a, doub
   int64_t n = (int64_t)1 << scale;
   int64_t M = edgefactor * n;
   if (2 * M > cap) return -1;
-  const uint32_t tA = (uint32_t)std::llround(a * 65536.0);
-  const uint32_t tAB = (uint32_t)std::llround((a + b) * 65536.0);
-  const uint32_t tABC = (uint32_t)std::llround((a + b + c) * 65536.0);
-  uint64_t s = mix64(seed ^ 0x5A7u);
-  Perm perm(scale, seed ^ 0xBEEFu);
+  const GGRmat rm = gg_make_rmat(scale, seed, a, b, c);
   auto gen = [=](int64_t i, int64_t* u, int64_t* v) {
-    uint64_t uu = 0, vv = 0, h = 0;
-    for (int l = 0; l < scale; ++l) {
-      if ((l & 3) == 0) h = hash2(s, (uint64_t)i, (uint64_t)(l >> 2));
-      uint32_t r = (uint32_t)(h & 0xFFFFu);
-      h >>= 16;
-      uint64_t bu, bv;
-      if (r < tA) { bu = 0; bv = 0; }
-      else if (r < tAB) { bu = 0; bv = 1; }
-      else if (r < tABC) { bu = 1; bv = 0; }
-      else { bu = 1; bv = 1; }
-      uu = (uu << 1) | bu;
-      vv = (vv << 1) | bv;
-    }
-    *u = (int64_t)perm(uu);
-    *v = (int64_t)perm(vv);
+    rm.edge(i, u, v);
     return true;
   };
   return build_csr(n, M, gen, offsets, col);
@@ -213,30 +160,10 @@ int64_t gg_mesh_csr(int64_t side, int keep_permille, uint64_t seed, int64_t* off
 //  mode 3: all weights 1.0 (pure tie-break by vertex id)
 int gg_weights(const int64_t* offsets, const int32_t* col, int64_t n, uint64_t seed, int mode,
                int64_t side, float* w) {
-  uint64_t s = mix64(seed ^ 0x77u);
+  const uint64_t ws = gg_mix64(seed ^ 0x77u);
 #pragma omp parallel for schedule(dynamic, 4096)
-  for (int64_t u = 0; u < n; ++u) {
-    for (int64_t j = offsets[u]; j < offsets[u + 1]; ++j) {
-      int64_t v = col[j];
-      uint64_t lo = (uint64_t)(u < v ? u : v), hi = (uint64_t)(u < v ? v : u);
-      uint64_t h = hash2(s, lo, hi);
-      float x;
-      switch (mode) {
-        case 1: x = (float)((double)(1 + h % 1000u) / 1000.0); break;
-        case 2: {
-          int64_t bx = (int64_t)hi % side, by = (int64_t)hi / side;
-          double U = (double)(h >> 11) * (1.0 / 9007199254740992.0);
-          double val = ((double)(bx + by) + 1e-3 * U) / (2.0 * (double)side);
-          x = (float)val;
-          if (!(x >= 5.9604644775390625e-08f)) x = 5.9604644775390625e-08f;
-          break;
-        }
-        case 3: x = 1.0f; break;
-        default: x = (float)(1 + (h & 0xFFFFFFu)) * 5.9604644775390625e-08f; break;
-      }
-      w[j] = x;
-    }
-  }
+  for (int64_t u = 0; u < n; ++u)
+    for (int64_t j = offsets[u]; j < offsets[u + 1]; ++j) w[j] = gg_weight(ws, mode, u, col[j], side);
   return 0;
 }
 

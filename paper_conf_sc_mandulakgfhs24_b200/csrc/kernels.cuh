@@ -274,40 +274,39 @@ __global__ void k_tile_rows(const int64_t* __restrict__ noffs, int64_t n_nz, int
 }
 
 // =============================================================================================
-// per-run reset: matched bitmap, counters, and best[] of rows that cross a sweep tile boundary
-// (those rows are merged with atomicMax by several tiles).
+// per-run reset: matched bitmap, counters, and best[] of the rows the sweep merges with
+// atomicMax (rows longer than one piece, or crossing a tile boundary; listed at create time).
 // =============================================================================================
 __global__ void k_reset(uint32_t* bits, int64_t nwords, uint64_t* best,
-                        const int32_t* __restrict__ tile_nz, const int64_t* __restrict__ noffs,
-                        const int32_t* __restrict__ nzr, int64_t ntiles, int64_t tile,
+                        const int32_t* __restrict__ atomic_rows, int64_t n_atomic,
                         unsigned long long* counters, int ncounters) {
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   for (int64_t i = tid; i < nwords; i += stride) bits[i] = 0u;
-  for (int64_t t = 1 + tid; t < ntiles; t += stride) {
-    const int32_t r = tile_nz[t];
-    if (noffs[r] < t * tile) best[nzr[r]] = 0ull;
-  }
+  for (int64_t i = tid; i < n_atomic; i += stride) best[atomic_rows[i]] = 0ull;
   if (tid < ncounters) counters[tid] = 0ull;
 }
 
 // =============================================================================================
 // A2 round-1 pointer sweep (SETPOINTERS over all vertices, Alg. 3 L1-9 P:141-151).
 //
-// Edge-centric: the adjacency is cut into fixed tiles of TILE entries regardless of row
+// Edge-centric tiles: the adjacency is cut into fixed tiles of TILE entries regardless of row
 // boundaries, so every CTA streams equal bytes (hub rows and degree-1 rows alike).  A persistent
-// CTA keeps STAGES tiles in flight with 1-D TMA bulk copies (keys, the tile's window of row
-// starts, and the window's vertex ids) completing on mbarriers.  Each thread then reduces PER
-// consecutive entries from shared memory, segmented by row:
-//   * a row lying wholly inside one thread's slice -> plain store of its max key;
-//   * a row split over threads of the tile -> smem atomicMax, then one store;
-//   * a row crossing a tile boundary -> global atomicMax (u64 max is order independent, so the
-//     result is identical to a single sequential scan; R5).
+// CTA keeps STAGES tiles in flight with 1-D TMA bulk copies (cp.async.bulk -> UBLKCP) completing
+// on mbarriers: the tile's packed keys, plus the window of its rows' start offsets (low 32 bits)
+// and vertex ids.  Per tile, entirely from shared memory:
+//   1. classify every row of the window by its in-tile length: short (< 32 entries) rows go to a
+//      thread-per-row list; long rows are cut into pieces of <= PIECE entries for a warp each;
+//   2. short rows: one thread scans the row;  pieces: a warp scans 32 consecutive keys per step
+//      (conflict-free) and reduces with two 32-bit __reduce_max_sync (packed-key max);
+//   3. a row wholly inside one unit (tile and piece) is stored; any other row is merged with a
+//      global atomicMax on its u64 key (max is order independent => identical to one sequential
+//      scan; the row was zeroed by k_reset).
 // Self-loops are skipped (simple graph).  No bitmap test: in round 1 nothing is matched.
 // =============================================================================================
 struct SweepArgs {
   const uint64_t* adj;
-  const int64_t* noffs;
+  const uint32_t* noffs_lo;  // low 32 bits of each non-empty row's start (+ m)
   const int32_t* nzr;
   const int32_t* tile_nz;
   uint64_t* best;
@@ -315,129 +314,201 @@ struct SweepArgs {
   int64_t ntiles;
 };
 
-template <int THREADS, int PER, int STAGES>
+template <int CONSUMER_WARPS, int STAGES>
 struct SweepCfg {
-  static constexpr int kTile = THREADS * PER;
+  static constexpr int kTile = 1024;
+  static constexpr int kPiece = 256;
+  static constexpr int kConsumers = CONSUMER_WARPS;
+  static constexpr int kThreads = 32 * (CONSUMER_WARPS + 1);  // warp 0 = TMA producer
   static constexpr int kKeys = kTile + 2;   // u64 slots per stage
-  static constexpr int kWin = kTile + 4;    // int64 row starts per stage
-  static constexpr int kIds = kTile + 8;    // int32 vertex ids per stage
-  static constexpr size_t kStageBytes = (size_t)kKeys * 8 + (size_t)kWin * 8 + (size_t)kIds * 4;
-  static constexpr size_t kSmem =
-      STAGES * kStageBytes + (size_t)(kTile + 2) * 8 + STAGES * 8 + STAGES * 8;
+  static constexpr int kWin = kTile + 8;    // u32 row starts per stage
+  static constexpr int kIds = kTile + 8;    // i32 vertex ids per stage
+  static constexpr int kMaxPieces = kTile / 32 + kTile / kPiece + 4;
+  static constexpr int kShort = kTile + 8;
+  static constexpr size_t kStageBytes = (size_t)kKeys * 8 + (size_t)kWin * 4 + (size_t)kIds * 4;
+  static constexpr size_t kSmem = STAGES * kStageBytes + 2 * (size_t)kShort * 2 +
+                                  2 * (size_t)kMaxPieces * 8 + 2 * STAGES * 8 + STAGES * 8 + 32;
 };
 
-template <int THREADS, int PER, int STAGES>
-__global__ void __launch_bounds__(THREADS) k_sweep(SweepArgs A) {
-  using C = SweepCfg<THREADS, PER, STAGES>;
-  constexpr int TILE = C::kTile;
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("{\n .reg .b64 st;\n mbarrier.arrive.shared::cta.b64 st, [%0];\n}\n" ::"r"(smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
+
+template <int CONSUMER_WARPS, int STAGES>
+__global__ void __launch_bounds__(32 * (CONSUMER_WARPS + 1)) k_sweep(SweepArgs A) {
+  using C = SweepCfg<CONSUMER_WARPS, STAGES>;
+  constexpr int TILE = C::kTile, PIECE = C::kPiece, NW = CONSUMER_WARPS, NCT = 32 * NW;
   extern __shared__ __align__(128) unsigned char smem[];
   uint64_t* keys = reinterpret_cast<uint64_t*>(smem);
-  int64_t* win = reinterpret_cast<int64_t*>(smem + (size_t)STAGES * C::kKeys * 8);
-  int32_t* ids = reinterpret_cast<int32_t*>(smem + (size_t)STAGES * (C::kKeys + C::kWin) * 8);
-  uint64_t* rowmax = reinterpret_cast<uint64_t*>(smem + (size_t)STAGES * C::kStageBytes);
-  uint64_t* bars = rowmax + (TILE + 2);
-  int32_t* meta = reinterpret_cast<int32_t*>(bars + STAGES);
+  uint32_t* win = reinterpret_cast<uint32_t*>(smem + (size_t)STAGES * C::kKeys * 8);
+  int32_t* ids = reinterpret_cast<int32_t*>(smem + (size_t)STAGES * (C::kKeys * 8 + C::kWin * 4));
+  int16_t* shortl = reinterpret_cast<int16_t*>(smem + (size_t)STAGES * C::kStageBytes);  // [2][kShort]
+  int2* pieces = reinterpret_cast<int2*>(shortl + 2 * C::kShort);  // [2][kMaxPieces] (row, a|b<<16)
+  uint64_t* full = reinterpret_cast<uint64_t*>(pieces + 2 * C::kMaxPieces);
+  uint64_t* empty = full + STAGES;
+  int32_t* meta = reinterpret_cast<int32_t*>(empty + STAGES);  // [STAGES][2]
+  int32_t* cnt = meta + 2 * STAGES;                              // [3][2]: short, pieces
 
-  const int tid = threadIdx.x;
-  for (int i = tid; i < TILE + 2; i += THREADS) rowmax[i] = 0ull;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  if (tid < 6) cnt[tid] = 0;
   if (tid == 0) {
-    for (int s = 0; s < STAGES; ++s) mbar_init(&bars[s], 1);
+    for (int s = 0; s < STAGES; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], NW);
+    }
     fence_mbar_init();
   }
   __syncthreads();
 
-  const uint64_t pol_stream = policy_evict_first();
-  auto issue = [&](int64_t k) {  // thread 0 only: load this CTA's k-th tile into stage k%STAGES
-    const int64_t t = (int64_t)blockIdx.x + k * gridDim.x;
-    if (t >= A.ntiles) return;
-    const int s = (int)(k % STAGES);
-    const int32_t a = A.tile_nz[t], bp = A.tile_nz[t + 1];
-    meta[2 * s] = a;
-    meta[2 * s + 1] = bp;
-    const int64_t e0 = t * TILE;
-    const int64_t len = min((int64_t)TILE, A.m - e0);
-    const uint32_t kbytes = (uint32_t)(((len + 1) & ~1ll) * 8);
-    const int64_t a2 = a & ~1ll;
-    const uint32_t wbytes = (uint32_t)((((int64_t)bp + 2 - a2 + 1) & ~1ll) * 8);
-    const int64_t a4 = a & ~3ll;
-    const uint32_t ibytes = (uint32_t)((((int64_t)bp + 1 - a4 + 3) & ~3ll) * 4);
-    fence_proxy_async_smem();
-    mbar_arrive_expect_tx(&bars[s], kbytes + wbytes + ibytes);
-    tma_bulk_g2s(keys + (size_t)s * C::kKeys, A.adj + e0, kbytes, &bars[s], pol_stream);
-    tma_bulk_g2s(win + (size_t)s * C::kWin, A.noffs + a2, wbytes, &bars[s], pol_stream);
-    tma_bulk_g2s(ids + (size_t)s * C::kIds, A.nzr + a4, ibytes, &bars[s], pol_stream);
-  };
-  if (tid == 0)
-    for (int k = 0; k < STAGES; ++k) issue(k);
+  if (warp == 0) {
+    // ---------------- producer: keep STAGES tiles in flight (1-D TMA bulk copies)
+    if (lane != 0) return;
+    const uint64_t pol = policy_evict_first();
+    int64_t t = blockIdx.x;
+    int32_t a = 0, bp = 0;
+    if (t < A.ntiles) { a = A.tile_nz[t]; bp = A.tile_nz[t + 1]; }
+    for (int64_t k = 0; t < A.ntiles; ++k) {
+      const int64_t tn = t + gridDim.x;  // prefetch the next tile's row range
+      int32_t an = 0, bpn = 0;
+      if (tn < A.ntiles) { an = A.tile_nz[tn]; bpn = A.tile_nz[tn + 1]; }
+      const int s = (int)(k % STAGES);
+      if (k >= STAGES)
+        while (!mbar_try_wait(&empty[s], (uint32_t)(((k / STAGES) - 1) & 1))) {
+        }
+      meta[2 * s] = a;
+      meta[2 * s + 1] = bp;
+      const int64_t e0 = t * TILE;
+      const int64_t len = min((int64_t)TILE, A.m - e0);
+      const uint32_t kbytes = (uint32_t)(((len + 1) & ~1ll) * 8);
+      const int64_t a4 = a & ~3ll;
+      const uint32_t wbytes = (uint32_t)((((int64_t)bp + 2 - a4 + 3) & ~3ll) * 4);
+      fence_proxy_async_smem();
+      mbar_arrive_expect_tx(&full[s], kbytes + 2 * wbytes);
+      tma_bulk_g2s(keys + (size_t)s * C::kKeys, A.adj + e0, kbytes, &full[s], pol);
+      tma_bulk_g2s(win + (size_t)s * C::kWin, A.noffs_lo + a4, wbytes, &full[s], pol);
+      tma_bulk_g2s(ids + (size_t)s * C::kIds, A.nzr + a4, wbytes, &full[s], pol);
+      t = tn; a = an; bp = bpn;
+    }
+    return;
+  }
 
+  // ------------------ consumers (warps 1..NW): one named barrier per tile
+  const int ctid = tid - 32, cwarp = warp - 1;
   for (int64_t k = 0;; ++k) {
     const int64_t t = (int64_t)blockIdx.x + k * gridDim.x;
     if (t >= A.ntiles) break;
     const int s = (int)(k % STAGES);
-    while (!mbar_try_wait(&bars[s], (uint32_t)((k / STAGES) & 1))) {
+    const int par = (int)(k & 1);
+    int32_t* ck = cnt + 2 * (int)(k % 3);
+    int16_t* SL = shortl + par * C::kShort;
+    int2* PL = pieces + par * C::kMaxPieces;
+    while (!mbar_try_wait(&full[s], (uint32_t)((k / STAGES) & 1))) {
     }
     const uint64_t* K = keys + (size_t)s * C::kKeys;
-    const int64_t* W = win + (size_t)s * C::kWin;
+    const uint32_t* W = win + (size_t)s * C::kWin;
     const int32_t* I = ids + (size_t)s * C::kIds;
     const int32_t a = meta[2 * s], bp = meta[2 * s + 1];
-    const int lo = a & 1;                   // window index of row a  (win base = a & ~1)
-    const int hi = bp - (a & ~1);           // window index of row bp
-    const int ioff = (a & 3) - lo;          // ids index = window index + ioff
+    const int lo = a & 3, hi = bp - (a & ~3);
     const int64_t ts = t * TILE;
-    const int64_t te = min(ts + (int64_t)TILE, A.m);
+    const int len = (int)min((int64_t)TILE, A.m - ts);
+    const uint32_t ts32 = (uint32_t)ts;
+    auto rel = [&](int r) { return (int32_t)(W[r] - ts32); };  // row start relative to tile
 
-    const int64_t i0 = ts + (int64_t)tid * PER;
-    if (i0 < te) {
-      const int64_t i1 = min(i0 + PER, te);
-      int l = lo, h = hi;  // last row r in [lo, hi] with W[r] <= i0
-      while (l < h) {
-        const int mid = (l + h + 1) >> 1;
-        if (W[mid] <= i0) l = mid; else h = mid - 1;
+    // ---- 1. classify the window's rows by in-tile length
+    for (int r0 = lo; r0 <= hi; r0 += NCT) {
+      const int r = r0 + ctid;
+      int L = 0, ra = 0, rb = 0;
+      if (r <= hi) {
+        ra = max(rel(r), 0);
+        rb = min(rel(r + 1), len);
+        L = rb - ra;
       }
-      int r = l;
-      int64_t rs = W[r], re = W[r + 1];
-      uint32_t vid = (uint32_t)I[r + ioff];
-      uint64_t cur = 0;
-      auto emit = [&]() {
-        if (rs >= i0 && re <= i1) A.best[vid] = cur;
-        else if (cur) atomicMax(reinterpret_cast<unsigned long long*>(&rowmax[r - lo]),
-                                (unsigned long long)cur);
-      };
-#pragma unroll
-      for (int q = 0; q < PER; ++q) {
-        const int64_t e = i0 + q;
-        if (e < i1) {
-          while (e >= re) {
-            emit();
-            ++r;
-            rs = re;
-            re = W[r + 1];
-            vid = (uint32_t)I[r + ioff];
-            cur = 0;
-          }
-          const uint64_t key = K[e - ts];
-          if ((uint32_t)key != vid && key > cur) cur = key;
+      const bool sh = L > 0 && L < 32;
+      const unsigned bs = __ballot_sync(0xffffffffu, sh);
+      if (bs) {
+        int base = 0;
+        const int leader = __ffs(bs) - 1;
+        if (lane == leader) base = atomicAdd(&ck[0], __popc(bs));
+        base = __shfl_sync(0xffffffffu, base, leader);
+        if (sh) SL[base + __popc(bs & lanemask_lt())] = (int16_t)r;
+      }
+      if (L >= 32) {
+        const int np = (L + PIECE - 1) / PIECE;
+        const int base = atomicAdd(&ck[1], np);
+        for (int q = 0; q < np; ++q) {
+          const int pa = ra + q * PIECE, pb = min(rb, pa + PIECE);
+          PL[base + q] = make_int2(r, pa | (pb << 16));
         }
       }
-      emit();
     }
-    __syncthreads();
-    // flush rows shared by several threads of this tile, or crossing its boundaries
-    for (int r = lo + tid; r <= hi; r += THREADS) {
-      const int64_t rs = W[r], re = W[r + 1];
-      if (re <= ts || rs >= te) continue;
-      const bool inside = rs >= ts && re <= te;
-      if (inside && ((rs - ts) / PER == (re - 1 - ts) / PER)) continue;  // single-thread row
-      const uint64_t v = rowmax[r - lo];
-      rowmax[r - lo] = 0ull;
-      const uint32_t vid = (uint32_t)I[r + ioff];
-      if (inside) A.best[vid] = v;
-      else if (v) atomicMax(reinterpret_cast<unsigned long long*>(&A.best[vid]),
-                            (unsigned long long)v);
+    named_bar_sync(1, NCT);
+    const int nshort = ck[0], npieces = ck[1];
+    if (ctid == 0) { int32_t* cz = cnt + 2 * (int)((k + 2) % 3); cz[0] = 0; cz[1] = 0; }
+    // ---- 2a. short rows: a thread per row
+    for (int i = ctid; i < nshort; i += NCT) {
+      const int r = SL[i];
+      const int32_t rs = rel(r), re = rel(r + 1);
+      const int ja = max(rs, 0), jb = min(re, len);
+      const uint32_t vid = (uint32_t)I[r];
+      uint64_t b = 0;
+      for (int j = ja; j < jb; ++j) {
+        const uint64_t key = K[j];
+        if ((uint32_t)key != vid && key > b) b = key;
+      }
+      if (rs >= 0 && re <= len) A.best[vid] = b;
+      else if (b) atomicMax(reinterpret_cast<unsigned long long*>(&A.best[vid]), (unsigned long long)b);
     }
-    __syncthreads();
-    if (tid == 0) issue(k + STAGES);
+    // ---- 2b. pieces of long rows: a warp per piece
+    for (int p = cwarp; p < npieces; p += NW) {
+      const int2 pc = PL[p];
+      const int r = pc.x, pa = pc.y & 0xffff, pb = pc.y >> 16;
+      const uint32_t vid = (uint32_t)I[r];
+      uint64_t b = 0;
+      for (int j = pa + lane; j < pb; j += 32) {
+        const uint64_t key = K[j];
+        if ((uint32_t)key != vid && key > b) b = key;
+      }
+      b = group_max_key(b, 0xffffffffu);
+      if (lane == 0) {
+        const int32_t rs = rel(r), re = rel(r + 1);
+        if (rs >= 0 && re <= len && re - rs <= PIECE) A.best[vid] = b;
+        else if (b) atomicMax(reinterpret_cast<unsigned long long*>(&A.best[vid]), (unsigned long long)b);
+      }
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[s]);  // this warp is done with stage s
   }
+}
+
+// rows the sweep merges with atomicMax: degree > PIECE, or crossing a tile boundary
+__global__ void k_atomic_rows(const int64_t* __restrict__ noffs, const int32_t* __restrict__ nzr,
+                              int64_t n_nz, const int32_t* __restrict__ tile_nz, int64_t ntiles,
+                              int64_t tile, int64_t piece, int32_t* out,
+                              unsigned long long* count) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t lim = ((n_nz > ntiles ? n_nz : ntiles) + 31) & ~31ll;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < lim; i += stride) {
+    const bool longrow = i < n_nz && noffs[i + 1] - noffs[i] > piece;
+    warp_append(longrow, longrow ? nzr[i] : 0, out, count);
+    bool cross = false;
+    int32_t v = 0;
+    if (i >= 1 && i < ntiles) {
+      const int32_t r = tile_nz[i];
+      cross = noffs[r] < i * tile && noffs[r + 1] - noffs[r] <= piece;  // long rows listed above
+      v = nzr[r];
+    }
+    warp_append(cross, v, out, count);
+  }
+}
+
+__global__ void k_low32(const int64_t* __restrict__ noffs, int64_t cnt, uint32_t* lo) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += stride)
+    lo[i] = (uint32_t)noffs[i];
 }
 
 // =============================================================================================
@@ -550,39 +621,73 @@ __global__ void k_match_list(BinLists F, const unsigned long long* cnt,
 //   L' = { u in L : !matched(u), best[u] != 0 }
 //   F' = { u in L' : matched(ptr u) }     binned by degree
 // counters layout: [0] |L'|, [1..kBins] |F'_b|, [kBins+1] sum of deg over F'
+// Each warp owns a chunk of 32*K items: pass 1 records the predicates in registers and counts,
+// ONE atomicAdd per list per warp reserves the output ranges, pass 2 writes -- so the global
+// counters see (items / 32K) atomics instead of one per 32 items.
 // =============================================================================================
-template <bool ALL>
+template <bool ALL, int K>
 __global__ void k_compact(const int32_t* __restrict__ L, const unsigned long long* Lcnt, int64_t n,
                           const uint64_t* __restrict__ best, const uint32_t* __restrict__ bits,
                           const int64_t* __restrict__ offs, int32_t* Lout, BinLists Fout,
                           unsigned long long* counters) {
   const int64_t cnt = ALL ? n : (int64_t)*Lcnt;
-  const int64_t cnt32 = (cnt + 31) & ~31ll;
-  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int lane = threadIdx.x & 31;
+  const int64_t warp0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const unsigned lt = lanemask_lt();
   unsigned long long degsum = 0;
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cnt32; i += stride) {
-    bool live = false, need = false;
-    int bin = -1;
-    uint32_t u = 0;
-    if (i < cnt) {
-      u = ALL ? (uint32_t)i : (uint32_t)L[i];
-      const uint64_t b = best[u];
-      live = b != 0 && !bit_test(bits, u);
-      if (live && bit_test(bits, (uint32_t)b)) {
-        need = true;
-        const int64_t d = offs[u + 1] - offs[u];
-        bin = bin_of(d);
-        degsum += (unsigned long long)d;
+  for (int64_t c0 = warp0 * 32 * K; c0 < cnt; c0 += nwarps * 32 * K) {
+    uint32_t live = 0, binb[kBins] = {0, 0, 0, 0};
+    uint32_t uu[K];
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+      const int64_t i = c0 + 32 * k + lane;
+      uu[k] = 0;
+      if (i < cnt) {
+        const uint32_t u = ALL ? (uint32_t)i : (uint32_t)L[i];
+        uu[k] = u;
+        const uint64_t b = best[u];
+        if (b != 0 && !bit_test(bits, u)) {
+          live |= 1u << k;
+          if (bit_test(bits, (uint32_t)b)) {
+            const int64_t d = offs[u + 1] - offs[u];
+            binb[bin_of(d)] |= 1u << k;
+            degsum += (unsigned long long)d;
+          }
+        }
       }
     }
-    warp_append(live, (int32_t)u, Lout, &counters[0]);
+    // reserve output ranges: one atomic per list per warp
+    unsigned long long base[1 + kBins];
+    {
+      unsigned tot[1 + kBins];
+      tot[0] = __reduce_add_sync(0xffffffffu, __popc(live));
 #pragma unroll
-    for (int bb = 0; bb < kBins; ++bb)
-      warp_append(need && bin == bb, (int32_t)u, const_cast<int32_t*>(Fout.list[bb]),
-                  &counters[1 + bb]);
+      for (int b = 0; b < kBins; ++b) tot[1 + b] = __reduce_add_sync(0xffffffffu, __popc(binb[b]));
+#pragma unroll
+      for (int q = 0; q < 1 + kBins; ++q) {
+        unsigned long long x = 0;
+        if (lane == q && tot[q]) x = atomicAdd(&counters[q], (unsigned long long)tot[q]);
+        base[q] = __shfl_sync(0xffffffffu, x, q);
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+      const bool pl = (live >> k) & 1u;
+      const unsigned bl = __ballot_sync(0xffffffffu, pl);
+      if (pl) Lout[base[0] + __popc(bl & lt)] = (int32_t)uu[k];
+      base[0] += __popc(bl);
+#pragma unroll
+      for (int b = 0; b < kBins; ++b) {
+        const bool pb = (binb[b] >> k) & 1u;
+        const unsigned bb = __ballot_sync(0xffffffffu, pb);
+        if (pb) const_cast<int32_t*>(Fout.list[b])[base[1 + b] + __popc(bb & lt)] = (int32_t)uu[k];
+        base[1 + b] += __popc(bb);
+      }
+    }
   }
   for (int o = 16; o; o >>= 1) degsum += __shfl_xor_sync(0xffffffffu, degsum, o);
-  if ((threadIdx.x & 31) == 0 && degsum) atomicAdd(&counters[1 + kBins], degsum);
+  if (lane == 0 && degsum) atomicAdd(&counters[1 + kBins], degsum);
 }
 
 // =============================================================================================

@@ -47,11 +47,12 @@ void set_err(const char* fmt, ...) {
   } while (0)
 
 // Round-1 sweep configuration (tuned on B200).
-constexpr int kSweepThreads = 128;
-constexpr int kSweepPer = 8;
+constexpr int kSweepConsumers = 4;  // consumer warps (+1 TMA producer warp)
 constexpr int kSweepStages = 4;
-using Sweep = lm::SweepCfg<kSweepThreads, kSweepPer, kSweepStages>;
+using Sweep = lm::SweepCfg<kSweepConsumers, kSweepStages>;
+constexpr int kSweepThreads = Sweep::kThreads;
 constexpr int64_t kTile = Sweep::kTile;
+constexpr int kCompactK = 16;  // items per lane per compaction chunk
 
 constexpr int kFinBlocks = 592;  // 4 x 148 SMs: fixed => deterministic fp64 summation order
 constexpr int kFinThreads = 256;
@@ -78,6 +79,9 @@ struct lmatch_graph {
   int64_t* noffs = nullptr;
   int32_t* nzr = nullptr;
   int32_t* tile_nz = nullptr;
+  uint32_t* noffs_lo = nullptr;
+  int32_t* atomic_rows = nullptr;
+  int64_t n_atomic = 0;
   // state
   uint64_t* best = nullptr;
   uint32_t* bits = nullptr;
@@ -139,6 +143,8 @@ int alloc_all(lmatch_graph* g) {
   TRY(dmalloc(g, &g->nzr, (size_t)n + 8));
   g->ntiles = (m + kTile - 1) / kTile;
   TRY(dmalloc(g, &g->tile_nz, (size_t)g->ntiles + 2));
+  TRY(dmalloc(g, &g->noffs_lo, (size_t)n + 9));
+  TRY(dmalloc(g, &g->atomic_rows, (size_t)n + (size_t)g->ntiles + 1));
   TRY(dmalloc(g, &g->best, (size_t)n + 1));
   TRY(dmalloc(g, &g->bits, (size_t)((n + 31) / 32) + 1));
   for (int i = 0; i < 2; ++i) TRY(dmalloc(g, &g->L[i], (size_t)n + 1));
@@ -183,6 +189,20 @@ int build_index(lmatch_graph* g, cudaStream_t st) {
     lm::k_tile_rows<<<grid_for(g->ntiles + 1, 256, 4096), 256, 0, st>>>(g->noffs, g->n_nz, g->ntiles,
                                                                         kTile, g->tile_nz);
     CKL();
+    lm::k_low32<<<grid_for(g->n_nz + 1, 256, 4096), 256, 0, st>>>(g->noffs, g->n_nz + 1, g->noffs_lo);
+    CKL();
+    unsigned long long* cnt = nullptr;
+    TRY(dmalloc(g, &cnt, 1));
+    CK(cudaMemsetAsync(cnt, 0, 8, st));
+    lm::k_atomic_rows<<<grid_for(std::max(g->n_nz, g->ntiles), 256, 4096), 256, 0, st>>>(
+        g->noffs, g->nzr, g->n_nz, g->tile_nz, g->ntiles, kTile, Sweep::kPiece, g->atomic_rows, cnt);
+    CKL();
+    unsigned long long h_cnt = 0;
+    CK(cudaMemcpyAsync(&h_cnt, cnt, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    g->n_atomic = (int64_t)h_cnt;
+    cudaFree(cnt);
+    g->device_bytes -= 16;
   }
   CK(cudaStreamSynchronize(st));
   cudaFree(bs);
@@ -289,11 +309,11 @@ int upload_device(lmatch_graph* g, const int64_t* d_offsets, const int32_t* d_co
 int finish_create(lmatch_graph* g, cudaStream_t st) {
   TRY(build_index(g, st));
   if (g->ntiles > 0) {
-    CK(cudaFuncSetAttribute(lm::k_sweep<kSweepThreads, kSweepPer, kSweepStages>,
+    CK(cudaFuncSetAttribute(lm::k_sweep<kSweepConsumers, kSweepStages>,
                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Sweep::kSmem));
     int occ = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-        &occ, lm::k_sweep<kSweepThreads, kSweepPer, kSweepStages>, kSweepThreads, Sweep::kSmem));
+        &occ, lm::k_sweep<kSweepConsumers, kSweepStages>, kSweepThreads, Sweep::kSmem));
     if (occ < 1) occ = 1;
     g->sweep_grid = (int)std::min<int64_t>(g->ntiles, (int64_t)occ * g->num_sms);
   }
@@ -353,7 +373,7 @@ void lmatch_destroy(lmatch_graph* g) {
   if (!g) return;
   cudaSetDevice(g->device);
   if (g->stream) cudaStreamSynchronize(g->stream);
-  void* dev[] = {g->offs, g->adj, g->noffs, g->nzr, g->tile_nz, g->best, g->bits, g->L[0], g->L[1],
+  void* dev[] = {g->offs, g->adj, g->noffs, g->nzr, g->tile_nz, g->noffs_lo, g->atomic_rows, g->best, g->bits, g->L[0], g->L[1],
                  g->counters, g->pw, g->pc, g->res_w, g->res_c, g->mate_tmp, g->perr, g->werr,
                  g->st_col[0], g->st_col[1], g->st_w[0], g->st_w[1]};
   for (void* p : dev) if (p) cudaFree(p);
@@ -447,16 +467,15 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
   if (tm) CK(cudaEventRecord(g->ev[0], st));
   // ---- reset (bitmap, counters, tile-crossing rows' best)
   const int64_t nwords = (n + 31) / 32;
-  lm::k_reset<<<grid_for(std::max(nwords, g->ntiles), 256, 4096), 256, 0, st>>>(
-      g->bits, nwords, g->best, g->tile_nz, g->noffs, g->nzr, g->ntiles, kTile, g->counters,
-      kNumCounters);
+  lm::k_reset<<<grid_for(std::max(nwords, g->n_atomic), 256, 4096), 256, 0, st>>>(
+      g->bits, nwords, g->best, g->atomic_rows, g->n_atomic, g->counters, kNumCounters);
   CKL();
   ++launches;
   if (tm) CK(cudaEventRecord(g->ev[1], st));
   if (g->ntiles > 0 && n > 0) {
     // ---- round 1: A2 full sweep (no bitmap test), A4 match-all, A6 compact-all
-    lm::SweepArgs A{g->adj, g->noffs, g->nzr, g->tile_nz, g->best, g->m, g->ntiles};
-    lm::k_sweep<kSweepThreads, kSweepPer, kSweepStages>
+    lm::SweepArgs A{g->adj, g->noffs_lo, g->nzr, g->tile_nz, g->best, g->m, g->ntiles};
+    lm::k_sweep<kSweepConsumers, kSweepStages>
         <<<g->sweep_grid, kSweepThreads, Sweep::kSmem, st>>>(A);
     CKL();
     ++launches;
@@ -467,7 +486,7 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
     CKL();
     lm::BinLists Fl{};
     for (int b = 0; b < lm::kBins; ++b) Fl.list[b] = g->F[b];
-    lm::k_compact<true><<<grid_for(n, 256, 65536), 256, 0, st>>>(
+    lm::k_compact<true, kCompactK><<<grid_for((n + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
         nullptr, nullptr, n, g->best, g->bits, g->offs, g->L[0], Fl, cset[0]);
     CKL();
     launches += 2;
@@ -495,7 +514,7 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
       // A6 compaction of the live list
       const int nxt = cur ^ 1;
       CK(cudaMemsetAsync(cset[nxt], 0, 64, st));
-      lm::k_compact<false><<<grid_for(lcnt, 256, 65536), 256, 0, st>>>(
+      lm::k_compact<false, kCompactK><<<grid_for((lcnt + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
           g->L[cur], cset[cur], n, g->best, g->bits, g->offs, g->L[nxt], Fl, cset[nxt]);
       CKL();
       launches += 2;
