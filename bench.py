@@ -306,7 +306,7 @@ def main():
     # roofline of the dominant kernel: the round-1 sweep (one launch per step)
     info = lm.lmatch_info(h)
     n_nz = info["nonempty_rows"]
-    tile = 1024
+    tile = info.get("sweep_tile", 512)
     ntiles = (m + tile - 1) // tile
     sweep_bytes = 8 * m + 16 * n_nz + 4 * (ntiles + 1)  # keys + (start lo32, id, best) per row + tile index
     sweep_avg_ms = float(np.mean(sweep_ms))
@@ -352,6 +352,7 @@ def main():
                "ms_per_step": el / a.e2e_steps * 1e3,
                "includes": "lmatch_reload (H2D + pack + validate + index) + lmatch_run (+ mate D2H)"}
 
+    round_log = lm.lmatch_round_log(h)
     lm.lmatch_destroy(h)
     del d_mate
     torch.cuda.empty_cache()
@@ -372,6 +373,8 @@ def main():
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
                 "gpu_launches": int(launches), "clocks": clk.summary(),
                 "rounds": int(rounds[-1]), "cardinality": int(last["cardinality"]),
+                "entries_swept": int(last["entries_swept"]), "frontier_total": int(last["frontier_total"]),
+                "round_log": round_log.tolist(),
                 "matched_weight": last["weight"],
                 "phase_ms": {k: last[k] for k in ("ms_sweep", "ms_round1_rest", "ms_rounds",
                                                   "ms_finish", "ms_total")}}

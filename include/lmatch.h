@@ -143,6 +143,12 @@ LMATCH_API int lmatch_weight_device(lmatch_graph* g, const int32_t* d_mate, void
 LMATCH_API int lmatch_info(const lmatch_graph* g, int64_t* n, int64_t* m, int64_t* nonempty_rows,
                 int64_t* device_bytes);
 
+/* Per-round log of the last lmatch_run*: for round r (0-based), out[3r] = |F_r| (vertices whose
+ * pointer was computed; round 0 = every non-empty row), out[3r+1] = |L_r| (live vertices scanned
+ * by the compaction), out[3r+2] = E(F_r) (adjacency entries scanned).  Writes at most `cap` rounds;
+ * *nrounds receives the number of rounds.  (Fig. 8 "edges accessed per iteration".) */
+LMATCH_API int lmatch_round_log(const lmatch_graph* g, int64_t* out, int64_t cap, int64_t* nrounds);
+
 /* Release everything the handle owns.  NULL-safe. */
 LMATCH_API void lmatch_destroy(lmatch_graph* g);
 

@@ -20,11 +20,12 @@ __all__ = [
     "LMatchError", "Opts", "Stats", "Matcher", "lib_path",
     "lmatch_abi_version", "lmatch_create", "lmatch_create_ex", "lmatch_create_device",
     "lmatch_reload", "lmatch_run", "lmatch_run_device", "lmatch_weight", "lmatch_weight_device",
-    "lmatch_info", "lmatch_destroy", "lmatch_strerror", "lmatch_last_error",
+    "lmatch_info", "lmatch_round_log", "lmatch_destroy", "lmatch_strerror", "lmatch_last_error",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-lib_path = os.path.join(_HERE, "liblmatch.so")
+# LMATCH_LIB may point at an alternative build of the same library (kernel-tuning variants).
+lib_path = os.environ.get("LMATCH_LIB") or os.path.join(_HERE, "liblmatch.so")
 if not os.path.exists(lib_path):
     raise ImportError(
         f"{lib_path} is missing: build it with `make` (or __graft_entry__.build()). "
@@ -76,6 +77,7 @@ _sig = {
     "lmatch_weight_device": ([_P, _P, _P, ctypes.POINTER(ctypes.c_double)], ctypes.c_int),
     "lmatch_info": ([_P, ctypes.POINTER(_I64), ctypes.POINTER(_I64), ctypes.POINTER(_I64),
                      ctypes.POINTER(_I64)], ctypes.c_int),
+    "lmatch_round_log": ([_P, _P, _I64, ctypes.POINTER(_I64)], ctypes.c_int),
     "lmatch_destroy": ([_P], None),
     "lmatch_strerror": ([ctypes.c_int], ctypes.c_char_p),
     "lmatch_last_error": ([], ctypes.c_char_p),
@@ -212,6 +214,15 @@ def lmatch_info(h: int) -> dict:
     _check(_lib.lmatch_info(h, ctypes.byref(n), ctypes.byref(m), ctypes.byref(nz),
                             ctypes.byref(db)), "lmatch_info")
     return dict(n=n.value, m=m.value, nonempty_rows=nz.value, device_bytes=db.value)
+
+
+def lmatch_round_log(h: int) -> np.ndarray:
+    """Per-round (|F_r|, |L_r|, E(F_r)) of the last run, shape (rounds, 3)."""
+    nr = _I64()
+    _check(_lib.lmatch_round_log(h, None, 0, ctypes.byref(nr)), "lmatch_round_log")
+    out = np.zeros((max(nr.value, 1), 3), dtype=np.int64)
+    _check(_lib.lmatch_round_log(h, out.ctypes.data, nr.value, ctypes.byref(nr)), "lmatch_round_log")
+    return out[: nr.value]
 
 
 def lmatch_destroy(h: int | None) -> None:

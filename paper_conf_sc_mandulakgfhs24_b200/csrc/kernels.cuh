@@ -18,6 +18,7 @@
 //   F[b]   int32[]           frontier (vertices whose target was matched), binned by degree
 #pragma once
 #include <cstdint>
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 namespace lm {
@@ -112,6 +113,7 @@ __device__ __forceinline__ uint64_t policy_evict_last() {
 }
 
 // =============================================================================================
+// =============================================================================================
 // A1 ingest: pack + validate  (adj[j] = bits(w[j]) << 32 | col[j]; PAPER.md:96 CSR arrays)
 // =============================================================================================
 struct PackErr {
@@ -131,6 +133,21 @@ __global__ void k_pack(const int32_t* __restrict__ col, const float* __restrict_
     if (!ok) atomicMin(&err->first_bad, (unsigned long long)(base + j));
     adj[j] = ((uint64_t)wb << 32) | (uint32_t)c;
   }
+}
+
+// Self-loops are ignored (simple graph): their keys become 0, which never wins a max, so
+// no kernel on the hot path needs a per-entry self test.  8 lanes per row.
+__global__ void k_zap_self_loops(const int64_t* __restrict__ offs, uint64_t* adj, int64_t n,
+                                 unsigned long long* count) {
+  const int lane8 = threadIdx.x & 7;
+  const int64_t g0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 3;
+  const int64_t gs = ((int64_t)gridDim.x * blockDim.x) >> 3;
+  unsigned long long c = 0;
+  for (int64_t u = g0; u < n; u += gs)
+    for (int64_t j = offs[u] + lane8; j < offs[u + 1]; j += 8)
+      if ((uint32_t)adj[j] == (uint32_t)u) { adj[j] = 0ull; ++c; }
+  for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+  if ((threadIdx.x & 31) == 0 && c) atomicAdd(count, c);
 }
 
 __global__ void k_check_offsets(const int64_t* __restrict__ offs, int64_t n, int64_t m,
@@ -161,6 +178,7 @@ __global__ void k_symhash(const int64_t* __restrict__ offs, const uint64_t* __re
   for (int64_t u = g0; u < n; u += gs) {
     for (int64_t j = offs[u] + lane8; j < offs[u + 1]; j += 8) {
       const uint64_t k = adj[j];
+      if (k == 0) continue;  // zeroed self-loop
       const uint64_t v = (uint32_t)k, wb = k >> 32;
       s += mix64(mix64((uint64_t)u * 0x100000001B3ull ^ v) ^ wb) -
            mix64(mix64(v * 0x100000001B3ull ^ (uint64_t)u) ^ wb);
@@ -274,8 +292,9 @@ __global__ void k_tile_rows(const int64_t* __restrict__ noffs, int64_t n_nz, int
 }
 
 // =============================================================================================
+// =============================================================================================
 // per-run reset: matched bitmap, counters, and best[] of the rows the sweep merges with
-// atomicMax (rows longer than one piece, or crossing a tile boundary; listed at create time).
+// atomicMax (rows crossing a sweep-tile boundary; listed at create time).
 // =============================================================================================
 __global__ void k_reset(uint32_t* bits, int64_t nwords, uint64_t* best,
                         const int32_t* __restrict__ atomic_rows, int64_t n_atomic,
@@ -290,20 +309,26 @@ __global__ void k_reset(uint32_t* bits, int64_t nwords, uint64_t* best,
 // =============================================================================================
 // A2 round-1 pointer sweep (SETPOINTERS over all vertices, Alg. 3 L1-9 P:141-151).
 //
-// Edge-centric tiles: the adjacency is cut into fixed tiles of TILE entries regardless of row
-// boundaries, so every CTA streams equal bytes (hub rows and degree-1 rows alike).  A persistent
-// CTA keeps STAGES tiles in flight with 1-D TMA bulk copies (cp.async.bulk -> UBLKCP) completing
-// on mbarriers: the tile's packed keys, plus the window of its rows' start offsets (low 32 bits)
-// and vertex ids.  Per tile, entirely from shared memory:
-//   1. classify every row of the window by its in-tile length: short (< 32 entries) rows go to a
-//      thread-per-row list; long rows are cut into pieces of <= PIECE entries for a warp each;
-//   2. short rows: one thread scans the row;  pieces: a warp scans 32 consecutive keys per step
-//      (conflict-free) and reduces with two 32-bit __reduce_max_sync (packed-key max);
-//   3. a row wholly inside one unit (tile and piece) is stored; any other row is merged with a
-//      global atomicMax on its u64 key (max is order independent => identical to one sequential
-//      scan; the row was zeroed by k_reset).
-// Self-loops are skipped (simple graph).  No bitmap test: in round 1 nothing is matched.
+// Edge-centric, warp-private tiles: the adjacency is cut into fixed tiles of TILE entries
+// regardless of row boundaries, so every warp streams equal bytes (hub rows and degree-1 rows
+// alike).  Each warp owns a ring of RING shared-memory stages; its lane 0 keeps RING-1 tiles in
+// flight with 1-D TMA bulk copies (cp.async.bulk -> UBLKCP) completing on the stage's mbarrier:
+// the tile's packed keys plus the window of its rows' start offsets (low 32 bits) and vertex ids.
+// No CTA-wide barrier anywhere: warps never wait for each other.  Per tile, from shared memory:
+//   * lane l takes row r0+l of the window; a row with fewer than 32 in-tile entries is scanned by
+//     its lane alone; longer rows are then scanned by the whole warp, one after the other
+//     (32 consecutive keys per step, conflict-free) and reduced across the warp;
+//   * a row wholly inside the tile stores its max key (the pointer); a row crossing a tile
+//     boundary merges its partial max with a global atomicMax on the u64 key (order independent
+//     => identical to one sequential scan; such rows are zeroed by k_reset).
+// Self-loop keys were zeroed at ingest (k_zap_self_loops).  No bitmap test in round 1.
 // =============================================================================================
+__device__ __forceinline__ uint64_t umax64(uint64_t a, uint64_t b) { return a > b ? a : b; }
+// max(b, key) unless key is the self-loop entry of vertex `self`
+__device__ __forceinline__ uint64_t umax_skip(uint64_t b, uint64_t key, uint32_t self) {
+  return ((uint32_t)key != self && key > b) ? key : b;
+}
+
 struct SweepArgs {
   const uint64_t* adj;
   const uint32_t* noffs_lo;  // low 32 bits of each non-empty row's start (+ m)
@@ -314,191 +339,400 @@ struct SweepArgs {
   int64_t ntiles;
 };
 
-template <int CONSUMER_WARPS, int STAGES>
+template <int TILE, int RING, int WARPS, int WCAP>
 struct SweepCfg {
-  static constexpr int kTile = 1024;
-  static constexpr int kPiece = 256;
-  static constexpr int kConsumers = CONSUMER_WARPS;
-  static constexpr int kThreads = 32 * (CONSUMER_WARPS + 1);  // warp 0 = TMA producer
-  static constexpr int kKeys = kTile + 2;   // u64 slots per stage
-  static constexpr int kWin = kTile + 8;    // u32 row starts per stage
-  static constexpr int kIds = kTile + 8;    // i32 vertex ids per stage
-  static constexpr int kMaxPieces = kTile / 32 + kTile / kPiece + 4;
-  static constexpr int kShort = kTile + 8;
-  static constexpr size_t kStageBytes = (size_t)kKeys * 8 + (size_t)kWin * 4 + (size_t)kIds * 4;
-  static constexpr size_t kSmem = STAGES * kStageBytes + 2 * (size_t)kShort * 2 +
-                                  2 * (size_t)kMaxPieces * 8 + 2 * STAGES * 8 + STAGES * 8 + 32;
+  static constexpr int kTile = TILE;
+  static constexpr int kRing = RING;
+  static constexpr int kWarps = WARPS;
+  static constexpr int kThreads = 32 * WARPS;
+  static constexpr int kKeys = TILE + 2;   // u64 slots per stage
+  static constexpr int kWin = WCAP;        // u32 row starts / ids staged per stage (rows beyond
+                                           // the cap are read from global memory)
+  static constexpr size_t kStageBytes = (size_t)kKeys * 8 + 2 * (size_t)kWin * 4;
+  static constexpr size_t kWarpBytes = RING * kStageBytes + ((RING * 8 + 8 + 15) / 16) * 16;
+  static constexpr size_t kSmem = WARPS * kWarpBytes;
+  static_assert(WCAP % 4 == 0, "window cap must be a multiple of 4 entries");
+  static_assert(kStageBytes % 16 == 0 && kWarpBytes % 16 == 0, "TMA needs 16-byte alignment");
 };
 
-__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
-  asm volatile("{\n .reg .b64 st;\n mbarrier.arrive.shared::cta.b64 st, [%0];\n}\n" ::"r"(smem_u32(bar))
-               : "memory");
-}
-__device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
-  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
-}
-
-template <int CONSUMER_WARPS, int STAGES>
-__global__ void __launch_bounds__(32 * (CONSUMER_WARPS + 1)) k_sweep(SweepArgs A) {
-  using C = SweepCfg<CONSUMER_WARPS, STAGES>;
-  constexpr int TILE = C::kTile, PIECE = C::kPiece, NW = CONSUMER_WARPS, NCT = 32 * NW;
+template <int TILE, int RING, int WARPS, int WCAP>
+__global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
+  using C = SweepCfg<TILE, RING, WARPS, WCAP>;
   extern __shared__ __align__(128) unsigned char smem[];
-  uint64_t* keys = reinterpret_cast<uint64_t*>(smem);
-  uint32_t* win = reinterpret_cast<uint32_t*>(smem + (size_t)STAGES * C::kKeys * 8);
-  int32_t* ids = reinterpret_cast<int32_t*>(smem + (size_t)STAGES * (C::kKeys * 8 + C::kWin * 4));
-  int16_t* shortl = reinterpret_cast<int16_t*>(smem + (size_t)STAGES * C::kStageBytes);  // [2][kShort]
-  int2* pieces = reinterpret_cast<int2*>(shortl + 2 * C::kShort);  // [2][kMaxPieces] (row, a|b<<16)
-  uint64_t* full = reinterpret_cast<uint64_t*>(pieces + 2 * C::kMaxPieces);
-  uint64_t* empty = full + STAGES;
-  int32_t* meta = reinterpret_cast<int32_t*>(empty + STAGES);  // [STAGES][2]
-  int32_t* cnt = meta + 2 * STAGES;                              // [3][2]: short, pieces
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  unsigned char* my = smem + (size_t)warp * C::kWarpBytes;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(my + RING * C::kStageBytes);
+  auto keys_of = [&](int s) { return reinterpret_cast<uint64_t*>(my + s * C::kStageBytes); };
+  auto win_of = [&](int s) {
+    return reinterpret_cast<uint32_t*>(my + s * C::kStageBytes + (size_t)C::kKeys * 8);
+  };
+  auto ids_of = [&](int s) {
+    return reinterpret_cast<int32_t*>(my + s * C::kStageBytes + (size_t)C::kKeys * 8 +
+                                      (size_t)C::kWin * 4);
+  };
+  (void)ids_of;
 
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  if (tid < 6) cnt[tid] = 0;
-  if (tid == 0) {
-    for (int s = 0; s < STAGES; ++s) {
-      mbar_init(&full[s], 1);
-      mbar_init(&empty[s], NW);
-    }
+  const int64_t gw = (int64_t)blockIdx.x * WARPS + warp;
+  const int64_t nwt = (int64_t)gridDim.x * WARPS;
+  if (lane == 0) {
+    for (int s = 0; s < RING; ++s) mbar_init(&bars[s], 1);
     fence_mbar_init();
   }
-  __syncthreads();
+  __syncwarp();
 
-  if (warp == 0) {
-    // ---------------- producer: keep STAGES tiles in flight (1-D TMA bulk copies)
-    if (lane != 0) return;
-    const uint64_t pol = policy_evict_first();
-    int64_t t = blockIdx.x;
-    int32_t a = 0, bp = 0;
-    if (t < A.ntiles) { a = A.tile_nz[t]; bp = A.tile_nz[t + 1]; }
-    for (int64_t k = 0; t < A.ntiles; ++k) {
-      const int64_t tn = t + gridDim.x;  // prefetch the next tile's row range
-      int32_t an = 0, bpn = 0;
-      if (tn < A.ntiles) { an = A.tile_nz[tn]; bpn = A.tile_nz[tn + 1]; }
-      const int s = (int)(k % STAGES);
-      if (k >= STAGES)
-        while (!mbar_try_wait(&empty[s], (uint32_t)(((k / STAGES) - 1) & 1))) {
-        }
-      meta[2 * s] = a;
-      meta[2 * s + 1] = bp;
-      const int64_t e0 = t * TILE;
-      const int64_t len = min((int64_t)TILE, A.m - e0);
-      const uint32_t kbytes = (uint32_t)(((len + 1) & ~1ll) * 8);
-      const int64_t a4 = a & ~3ll;
-      const uint32_t wbytes = (uint32_t)((((int64_t)bp + 2 - a4 + 3) & ~3ll) * 4);
-      fence_proxy_async_smem();
-      mbar_arrive_expect_tx(&full[s], kbytes + 2 * wbytes);
-      tma_bulk_g2s(keys + (size_t)s * C::kKeys, A.adj + e0, kbytes, &full[s], pol);
-      tma_bulk_g2s(win + (size_t)s * C::kWin, A.noffs_lo + a4, wbytes, &full[s], pol);
-      tma_bulk_g2s(ids + (size_t)s * C::kIds, A.nzr + a4, wbytes, &full[s], pol);
-      t = tn; a = an; bp = bpn;
-    }
-    return;
+  const uint64_t pol = policy_evict_first();
+  // lane 0 only: TMA-load tile t (row window [a, bp]) into stage s
+  auto issue = [&](int64_t t, int s, int32_t a, int32_t bp) {
+    const int64_t e0 = t * TILE;
+    const int64_t len = min((int64_t)TILE, A.m - e0);
+    const uint32_t kbytes = (uint32_t)(((len + 1) & ~1ll) * 8);
+    const int64_t a4 = a & ~3ll;
+    const int64_t wcnt = min((int64_t)bp + 2 - a4, (int64_t)WCAP);
+    const uint32_t wbytes = (uint32_t)(((wcnt + 3) & ~3ll) * 4);
+    fence_proxy_async_smem();
+    mbar_arrive_expect_tx(&bars[s], kbytes + 2 * wbytes);
+    tma_bulk_g2s(keys_of(s), A.adj + e0, kbytes, &bars[s], pol);
+    tma_bulk_g2s(win_of(s), A.noffs_lo + a4, wbytes, &bars[s], pol);
+    tma_bulk_g2s(ids_of(s), A.nzr + a4, wbytes, &bars[s], pol);
+  };
+  // lane s holds the row window of the tile now in stage s; lane 0 prefetches the next one
+  int32_t my_a = 0, my_bp = 0, nx_a = 0, nx_bp = 0;
+  if (lane < RING) {
+    const int64_t t = gw + (int64_t)lane * nwt;
+    if (t < A.ntiles) { my_a = A.tile_nz[t]; my_bp = A.tile_nz[t + 1]; }
+  }
+  __syncwarp();
+  for (int s = 0; s < RING; ++s) {
+    const int64_t t = gw + (int64_t)s * nwt;
+    const int32_t a = __shfl_sync(0xffffffffu, my_a, s), bp = __shfl_sync(0xffffffffu, my_bp, s);
+    if (lane == 0 && t < A.ntiles) issue(t, s, a, bp);
+  }
+  if (lane == 0) {
+    const int64_t t = gw + (int64_t)RING * nwt;
+    if (t < A.ntiles) { nx_a = A.tile_nz[t]; nx_bp = A.tile_nz[t + 1]; }
   }
 
-  // ------------------ consumers (warps 1..NW): one named barrier per tile
-  const int ctid = tid - 32, cwarp = warp - 1;
   for (int64_t k = 0;; ++k) {
-    const int64_t t = (int64_t)blockIdx.x + k * gridDim.x;
+    const int64_t t = gw + k * nwt;
     if (t >= A.ntiles) break;
-    const int s = (int)(k % STAGES);
-    const int par = (int)(k & 1);
-    int32_t* ck = cnt + 2 * (int)(k % 3);
-    int16_t* SL = shortl + par * C::kShort;
-    int2* PL = pieces + par * C::kMaxPieces;
-    while (!mbar_try_wait(&full[s], (uint32_t)((k / STAGES) & 1))) {
+    const int s = (int)(k % RING);
+    const int32_t a = __shfl_sync(0xffffffffu, my_a, s), bp = __shfl_sync(0xffffffffu, my_bp, s);
+    while (!mbar_try_wait(&bars[s], (uint32_t)((k / RING) & 1))) {
     }
-    const uint64_t* K = keys + (size_t)s * C::kKeys;
-    const uint32_t* W = win + (size_t)s * C::kWin;
-    const int32_t* I = ids + (size_t)s * C::kIds;
-    const int32_t a = meta[2 * s], bp = meta[2 * s + 1];
+    const uint64_t* K = keys_of(s);
+    const uint32_t* Ws = win_of(s);
+    const int32_t* Is = ids_of(s);
     const int lo = a & 3, hi = bp - (a & ~3);
+    const int64_t a4 = a & ~3ll;
     const int64_t ts = t * TILE;
     const int len = (int)min((int64_t)TILE, A.m - ts);
     const uint32_t ts32 = (uint32_t)ts;
-    auto rel = [&](int r) { return (int32_t)(W[r] - ts32); };  // row start relative to tile
+    // window accessors: staged entries from shared memory, the (rare) overflow from global
+    auto Wr = [&](int r) -> uint32_t { return r < WCAP ? Ws[r] : __ldg(A.noffs_lo + a4 + r); };
+    auto Ir = [&](int r) -> int32_t { return r < WCAP ? Is[r] : __ldg(A.nzr + a4 + r); };
 
-    // ---- 1. classify the window's rows by in-tile length
-    for (int r0 = lo; r0 <= hi; r0 += NCT) {
-      const int r = r0 + ctid;
-      int L = 0, ra = 0, rb = 0;
+    for (int r0 = lo; r0 <= hi; r0 += 32) {
+      const int r = r0 + lane;
+      int32_t rs = 0, re = 0;
+      int L = 0;
+      uint32_t vid = 0;
       if (r <= hi) {
-        ra = max(rel(r), 0);
-        rb = min(rel(r + 1), len);
-        L = rb - ra;
+        rs = (int32_t)(Wr(r) - ts32);
+        re = (int32_t)(Wr(r + 1) - ts32);
+        L = min(re, len) - max(rs, 0);
+        vid = (uint32_t)Ir(r);
       }
-      const bool sh = L > 0 && L < 32;
-      const unsigned bs = __ballot_sync(0xffffffffu, sh);
-      if (bs) {
-        int base = 0;
-        const int leader = __ffs(bs) - 1;
-        if (lane == leader) base = atomicAdd(&ck[0], __popc(bs));
-        base = __shfl_sync(0xffffffffu, base, leader);
-        if (sh) SL[base + __popc(bs & lanemask_lt())] = (int16_t)r;
+      const bool inside = rs >= 0 && re <= len;
+      // short rows: a lane each
+      if (L > 0 && L < 32) {
+        uint64_t b0 = 0, b1 = 0, b2 = 0, b3 = 0;  // 4 independent max chains
+        int j = max(rs, 0);
+        const int je = min(re, len);
+        for (; j + 3 < je; j += 4) {
+          b0 = umax64(b0, K[j]);
+          b1 = umax64(b1, K[j + 1]);
+          b2 = umax64(b2, K[j + 2]);
+          b3 = umax64(b3, K[j + 3]);
+        }
+        if (j < je) b0 = umax64(b0, K[j]);  // <= 3 left: independent, predicated
+        if (j + 1 < je) b1 = umax64(b1, K[j + 1]);
+        if (j + 2 < je) b2 = umax64(b2, K[j + 2]);
+        const uint64_t b = umax64(umax64(b0, b1), umax64(b2, b3));
+        if (inside) A.best[vid] = b;
+        else if (b) atomicMax(reinterpret_cast<unsigned long long*>(&A.best[vid]), (unsigned long long)b);
       }
-      if (L >= 32) {
-        const int np = (L + PIECE - 1) / PIECE;
-        const int base = atomicAdd(&ck[1], np);
-        for (int q = 0; q < np; ++q) {
-          const int pa = ra + q * PIECE, pb = min(rb, pa + PIECE);
-          PL[base + q] = make_int2(r, pa | (pb << 16));
+      // long rows: the whole warp, one row at a time
+      unsigned lm = __ballot_sync(0xffffffffu, L >= 32);
+      while (lm) {
+        const int l = __ffs(lm) - 1;
+        lm &= lm - 1;
+        const int32_t ja = __shfl_sync(0xffffffffu, max(rs, 0), l);
+        const int32_t jb = __shfl_sync(0xffffffffu, min(re, len), l);
+        const uint32_t v = __shfl_sync(0xffffffffu, vid, l);
+        const bool ins = __shfl_sync(0xffffffffu, (int)inside, l) != 0;
+        uint64_t b0 = 0, b1 = 0, b2 = 0, b3 = 0;  // 4 independent max chains
+        int j = ja + lane;
+        for (; j + 96 < jb; j += 128) {
+          b0 = umax64(b0, K[j]);
+          b1 = umax64(b1, K[j + 32]);
+          b2 = umax64(b2, K[j + 64]);
+          b3 = umax64(b3, K[j + 96]);
+        }
+        if (j < jb) b0 = umax64(b0, K[j]);  // <= 3 steps left: independent, predicated
+        if (j + 32 < jb) b1 = umax64(b1, K[j + 32]);
+        if (j + 64 < jb) b2 = umax64(b2, K[j + 64]);
+        const uint64_t b = group_max_key(umax64(umax64(b0, b1), umax64(b2, b3)), 0xffffffffu);
+        if (lane == 0) {
+          if (ins) A.best[v] = b;
+          else if (b) atomicMax(reinterpret_cast<unsigned long long*>(&A.best[v]), (unsigned long long)b);
         }
       }
     }
-    named_bar_sync(1, NCT);
-    const int nshort = ck[0], npieces = ck[1];
-    if (ctid == 0) { int32_t* cz = cnt + 2 * (int)((k + 2) % 3); cz[0] = 0; cz[1] = 0; }
-    // ---- 2a. short rows: a thread per row
-    for (int i = ctid; i < nshort; i += NCT) {
-      const int r = SL[i];
-      const int32_t rs = rel(r), re = rel(r + 1);
-      const int ja = max(rs, 0), jb = min(re, len);
-      const uint32_t vid = (uint32_t)I[r];
-      uint64_t b = 0;
-      for (int j = ja; j < jb; ++j) {
-        const uint64_t key = K[j];
-        if ((uint32_t)key != vid && key > b) b = key;
-      }
-      if (rs >= 0 && re <= len) A.best[vid] = b;
-      else if (b) atomicMax(reinterpret_cast<unsigned long long*>(&A.best[vid]), (unsigned long long)b);
-    }
-    // ---- 2b. pieces of long rows: a warp per piece
-    for (int p = cwarp; p < npieces; p += NW) {
-      const int2 pc = PL[p];
-      const int r = pc.x, pa = pc.y & 0xffff, pb = pc.y >> 16;
-      const uint32_t vid = (uint32_t)I[r];
-      uint64_t b = 0;
-      for (int j = pa + lane; j < pb; j += 32) {
-        const uint64_t key = K[j];
-        if ((uint32_t)key != vid && key > b) b = key;
-      }
-      b = group_max_key(b, 0xffffffffu);
-      if (lane == 0) {
-        const int32_t rs = rel(r), re = rel(r + 1);
-        if (rs >= 0 && re <= len && re - rs <= PIECE) A.best[vid] = b;
-        else if (b) atomicMax(reinterpret_cast<unsigned long long*>(&A.best[vid]), (unsigned long long)b);
-      }
-    }
     __syncwarp();
-    if (lane == 0) mbar_arrive(&empty[s]);  // this warp is done with stage s
+    // refill stage s with tile k + RING; prefetch the window of tile k + RING + 1
+    const int64_t tn = t + (int64_t)RING * nwt;
+    if (lane == 0 && tn < A.ntiles) issue(tn, s, nx_a, nx_bp);
+    {
+      const int32_t na = __shfl_sync(0xffffffffu, nx_a, 0), nbp = __shfl_sync(0xffffffffu, nx_bp, 0);
+      if (lane == s) { my_a = na; my_bp = nbp; }
+    }
+    if (lane == 0) {
+      const int64_t t2 = tn + nwt;
+      if (t2 < A.ntiles) { nx_a = A.tile_nz[t2]; nx_bp = A.tile_nz[t2 + 1]; }
+    }
   }
 }
 
-// rows the sweep merges with atomicMax: degree > PIECE, or crossing a tile boundary
+// =============================================================================================
+// A2 round-1 pointer sweep, v2: swizzled 2-D TMA tiles + merge-path style segmented reduction.
+//
+// The adjacency is viewed as a 2-D tensor [ceil(m/16)][16] of u64 keys (128-byte rows) and each
+// warp-private tile of TILE entries is fetched with ONE cp.async.bulk.tensor.2d (SASS UTMALDG)
+// using the 128-byte swizzle, so lane l can read its 16 CONTIGUOUS keys (one 128-B row) with
+// 8 conflict-free 16-byte shared loads (the swizzle spreads the lanes' chunks over all banks).
+// The tile's row window (row starts, vertex ids) comes with two 1-D bulk copies.
+// Each 512-entry pass: lane l walks entries [16l, 16l+16) of the pass in order, keeps the max key
+// of the current row segment, and stores every row that begins and ends inside its 16 entries;
+// rows spanning lanes are combined by ONE 5-step segmented max-scan over the lanes' open tail
+// segments; a row still open at the end of a pass is carried to the next pass in registers; a
+// row crossing the tile boundary is merged with a global atomicMax on its u64 key (zeroed by
+// k_reset).  u64 max is order independent => identical to one sequential scan of each row.
+// =============================================================================================
+struct Sweep2DArgs {
+  const uint32_t* noffs_lo;  // low 32 bits of each non-empty row's start (+ m)
+  const int32_t* nzr;
+  const int32_t* tile_nz;
+  uint64_t* best;
+  int64_t m;
+  int64_t ntiles;
+};
+
+template <int TILE, int RING, int WARPS, int WCAP>
+struct Sweep2DCfg {
+  static constexpr int kTile = TILE;
+  static constexpr int kThreads = 32 * WARPS;
+  static constexpr int kPasses = TILE / 512;
+  static constexpr size_t kKeyBytes = (size_t)TILE * 8;  // multiple of 1024 (swizzle atom)
+  static constexpr size_t kWinBytes = 2 * (size_t)WCAP * 4;
+  static constexpr size_t kWarpBytes =
+      ((RING * kKeyBytes + RING * kWinBytes + RING * 8 + 8 + 1023) / 1024) * 1024;
+  static constexpr size_t kSmem = WARPS * kWarpBytes + 1024;  // + runtime 1024-B alignment slack
+  static_assert(TILE % 512 == 0 && TILE / 16 <= 256, "tile = k*512 entries, box <= 256 rows");
+  static_assert(WCAP % 4 == 0, "window cap must be a multiple of 4 entries");
+};
+
+__device__ __forceinline__ void tma_tensor2d_g2s(void* dst, const void* tmap, int c0, int c1,
+                                                 uint64_t* bar, uint64_t policy) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+      " [%0], [%1, {%2, %3}], [%4], %5;" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(tmap)), "r"(c0), "r"(c1), "r"(smem_u32(bar)), "l"(policy)
+      : "memory");
+}
+
+template <int TILE, int RING, int WARPS, int WCAP>
+__global__ void __launch_bounds__(32 * WARPS)
+    k_sweep2d(const __grid_constant__ CUtensorMap tmap, Sweep2DArgs A) {
+  using C = Sweep2DCfg<TILE, RING, WARPS, WCAP>;
+  extern __shared__ unsigned char smem_raw[];
+  unsigned char* smem = reinterpret_cast<unsigned char*>(
+      (reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  unsigned char* my = smem + (size_t)warp * C::kWarpBytes;
+  unsigned char* keys0 = my;                                    // RING x kKeyBytes (1024-aligned)
+  unsigned char* wins0 = my + RING * C::kKeyBytes;              // RING x (starts[WCAP], ids[WCAP])
+  uint64_t* bars = reinterpret_cast<uint64_t*>(wins0 + RING * C::kWinBytes);
+
+  const int64_t gw = (int64_t)blockIdx.x * WARPS + warp;
+  const int64_t nwt = (int64_t)gridDim.x * WARPS;
+  if (lane == 0) {
+    for (int s = 0; s < RING; ++s) mbar_init(&bars[s], 1);
+    fence_mbar_init();
+  }
+  __syncwarp();
+
+  const uint64_t pol = policy_evict_first();
+  auto issue = [&](int64_t t, int s, int32_t a, int32_t bp) {  // lane 0 only
+    const int64_t a4 = a & ~3ll;
+    const int64_t wcnt = min((int64_t)bp + 2 - a4, (int64_t)WCAP);
+    const uint32_t wbytes = (uint32_t)(((wcnt + 3) & ~3ll) * 4);
+    unsigned char* w = wins0 + s * C::kWinBytes;
+    fence_proxy_async_smem();
+    mbar_arrive_expect_tx(&bars[s], (uint32_t)C::kKeyBytes + 2 * wbytes);
+    tma_tensor2d_g2s(keys0 + s * C::kKeyBytes, &tmap, 0, (int)(t * (TILE / 16)), &bars[s], pol);
+    tma_bulk_g2s(w, A.noffs_lo + a4, wbytes, &bars[s], pol);
+    tma_bulk_g2s(w + WCAP * 4, A.nzr + a4, wbytes, &bars[s], pol);
+  };
+  int32_t my_a = 0, my_bp = 0, nx_a = 0, nx_bp = 0;
+  if (lane < RING) {
+    const int64_t t = gw + (int64_t)lane * nwt;
+    if (t < A.ntiles) { my_a = A.tile_nz[t]; my_bp = A.tile_nz[t + 1]; }
+  }
+  __syncwarp();
+  for (int s = 0; s < RING; ++s) {
+    const int64_t t = gw + (int64_t)s * nwt;
+    const int32_t a = __shfl_sync(0xffffffffu, my_a, s), bp = __shfl_sync(0xffffffffu, my_bp, s);
+    if (lane == 0 && t < A.ntiles) issue(t, s, a, bp);
+  }
+  if (lane == 0) {
+    const int64_t t = gw + (int64_t)RING * nwt;
+    if (t < A.ntiles) { nx_a = A.tile_nz[t]; nx_bp = A.tile_nz[t + 1]; }
+  }
+
+  for (int64_t k = 0;; ++k) {
+    const int64_t t = gw + k * nwt;
+    if (t >= A.ntiles) break;
+    const int s = (int)(k % RING);
+    const int32_t a = __shfl_sync(0xffffffffu, my_a, s), bp = __shfl_sync(0xffffffffu, my_bp, s);
+    while (!mbar_try_wait(&bars[s], (uint32_t)((k / RING) & 1))) {
+    }
+    const unsigned char* K = keys0 + s * C::kKeyBytes;
+    const uint32_t* Ws = reinterpret_cast<const uint32_t*>(wins0 + s * C::kWinBytes);
+    const int32_t* Is = reinterpret_cast<const int32_t*>(wins0 + s * C::kWinBytes + WCAP * 4);
+    const int lo = a & 3, hi = bp - (a & ~3);
+    const int64_t a4 = a & ~3ll;
+    const int64_t ts = t * TILE;
+    const int len = (int)min((int64_t)TILE, A.m - ts);
+    const uint32_t ts32 = (uint32_t)ts;
+    auto rel = [&](int r) -> int32_t {
+      return (int32_t)((r < WCAP ? Ws[r] : __ldg(A.noffs_lo + a4 + r)) - ts32);
+    };
+    auto idr = [&](int r) -> uint32_t {
+      return (uint32_t)(r < WCAP ? Is[r] : __ldg(A.nzr + a4 + r));
+    };
+
+    int carryR = -1;        // row left open by the previous pass (window index), or -1
+    uint64_t carryV = 0;
+    int rlo = lo;           // search lower bound (rows before it ended in earlier passes)
+#pragma unroll 1
+    for (int p = 0; p < C::kPasses; ++p) {
+      const int pbase = p * 512;
+      if (pbase >= len) break;
+      const int e0 = pbase + lane * 16;
+      const int e1 = min(e0 + 16, len);
+      const bool has = e0 < len;
+      // row containing e0: last r in [rlo, hi] with rel(r) <= e0
+      int r = rlo;
+      if (has) {
+        int h = hi;
+        while (r < h) {
+          const int mid = (r + h + 1) >> 1;
+          if (rel(mid) <= e0) r = mid; else h = mid - 1;
+        }
+      }
+      int32_t rs = has ? rel(r) : 0, re = has ? rel(r + 1) : 0;
+      uint32_t vid = has ? idr(r) : 0;
+      // my 16 keys: one swizzled 128-byte row of the tile
+      ulonglong2 kv[8];
+      if (has) {
+        const int R = e0 >> 4;
+        const unsigned char* rowp = K + R * 128;
+#pragma unroll
+        for (int c = 0; c < 8; ++c)
+          kv[c] = *reinterpret_cast<const ulonglong2*>(rowp + ((c ^ (R & 7)) << 4));
+      }
+      const bool firstOpen = has && rs < e0;
+      const int firstR = r;
+      const int32_t f_rs = rs, f_re = re;
+      const uint32_t f_vid = vid;
+      bool firstClosed = false;
+      uint64_t firstVal = 0, b = 0;
+#pragma unroll
+      for (int q = 0; q < 16; ++q) {
+        const int e = e0 + q;
+        if (e < e1) {
+          if (e >= re) {  // the current row segment ends before e
+            if (r == firstR && firstOpen) { firstClosed = true; firstVal = b; }
+            else A.best[vid] = b;  // began and ended inside my 16 entries
+            ++r;
+            rs = re;
+            re = rel(r + 1);
+            vid = idr(r);
+            b = 0;
+          }
+          const uint64_t key = (q & 1) ? kv[q >> 1].y : kv[q >> 1].x;
+          b = umax64(b, key);
+        }
+      }
+      const bool lastOpen = has && re > e1;
+      if (has && !lastOpen) {  // the last segment ends exactly at e1
+        if (r == firstR && firstOpen) { firstClosed = true; firstVal = b; }
+        else A.best[vid] = b;
+      }
+      // segmented max-scan over the lanes' open tail segments
+      uint64_t T = lastOpen ? b : 0ull;
+      bool H = !(lastOpen && r == firstR && firstOpen);
+      if (lane == 0 && !H && carryR == r) T = umax64(T, carryV);
+#pragma unroll
+      for (int d = 1; d < 32; d <<= 1) {
+        const uint64_t tu = __shfl_up_sync(0xffffffffu, T, d);
+        const bool hu = __shfl_up_sync(0xffffffffu, (int)H, d) != 0;
+        if (lane >= d && !H) { T = umax64(T, tu); H = hu; }
+      }
+      const uint64_t Tprev = __shfl_up_sync(0xffffffffu, T, 1);
+      if (firstClosed) {
+        uint64_t tot = firstVal;
+        if (lane > 0) tot = umax64(tot, Tprev);
+        else if (carryR == firstR) tot = umax64(tot, carryV);
+        if (f_rs >= 0 && f_re <= len) A.best[f_vid] = tot;
+        else if (tot) atomicMax(reinterpret_cast<unsigned long long*>(&A.best[f_vid]),
+                                (unsigned long long)tot);
+      }
+      if (lastOpen && e1 == len && T)  // crosses the tile end
+        atomicMax(reinterpret_cast<unsigned long long*>(&A.best[vid]), (unsigned long long)T);
+      // carry the row left open at the end of this pass
+      const bool open31 = __shfl_sync(0xffffffffu, (int)(lastOpen && e1 < len), 31) != 0;
+      carryR = open31 ? __shfl_sync(0xffffffffu, r, 31) : -1;
+      carryV = __shfl_sync(0xffffffffu, T, 31);
+      rlo = __shfl_sync(0xffffffffu, r, 31);
+    }
+    __syncwarp();
+    const int64_t tn = t + (int64_t)RING * nwt;
+    if (lane == 0 && tn < A.ntiles) issue(tn, s, nx_a, nx_bp);
+    {
+      const int32_t na = __shfl_sync(0xffffffffu, nx_a, 0), nbp = __shfl_sync(0xffffffffu, nx_bp, 0);
+      if (lane == s) { my_a = na; my_bp = nbp; }
+    }
+    if (lane == 0) {
+      const int64_t t2 = tn + nwt;
+      if (t2 < A.ntiles) { nx_a = A.tile_nz[t2]; nx_bp = A.tile_nz[t2 + 1]; }
+    }
+  }
+}
+
+// rows the sweep merges with atomicMax: those crossing a tile boundary (one entry per boundary;
+// a row crossing several boundaries appears several times, which is harmless for zeroing)
 __global__ void k_atomic_rows(const int64_t* __restrict__ noffs, const int32_t* __restrict__ nzr,
-                              int64_t n_nz, const int32_t* __restrict__ tile_nz, int64_t ntiles,
-                              int64_t tile, int64_t piece, int32_t* out,
-                              unsigned long long* count) {
+                              const int32_t* __restrict__ tile_nz, int64_t ntiles, int64_t tile,
+                              int32_t* out, unsigned long long* count) {
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  const int64_t lim = ((n_nz > ntiles ? n_nz : ntiles) + 31) & ~31ll;
+  const int64_t lim = (ntiles + 31) & ~31ll;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < lim; i += stride) {
-    const bool longrow = i < n_nz && noffs[i + 1] - noffs[i] > piece;
-    warp_append(longrow, longrow ? nzr[i] : 0, out, count);
     bool cross = false;
     int32_t v = 0;
     if (i >= 1 && i < ntiles) {
       const int32_t r = tile_nz[i];
-      cross = noffs[r] < i * tile && noffs[r + 1] - noffs[r] <= piece;  // long rows listed above
+      cross = noffs[r] < i * tile;
       v = nzr[r];
     }
     warp_append(cross, v, out, count);
@@ -512,13 +746,64 @@ __global__ void k_low32(const int64_t* __restrict__ noffs, int64_t cnt, uint32_t
 }
 
 // =============================================================================================
-// A2 pointer phase on the frontier (rounds >= 2): G lanes per vertex, degree-binned.
-// best[u] = max{ adj[j] : j in row(u), col != u, !matched(col) }  (Alg. 3 L5-8).
+// Rounds >= 2.  Device counters (unsigned long long, RoundCounters layout, kNumCounters):
+//   [8 * set]               |S| of pair set `set` (stable live pairs)
+//   [8 * set + 1 + b]       |F_b| of frontier set `set`, degree bin b
+//   [16]                    adjacency entries of all frontiers produced so far (stats)
+// Lists: S = uint64 pairs (u | ptr u << 32); frontier bins = uint64 pairs (u | new ptr << 32):
+// the compaction writes (u, 0) and the pointer kernel overwrites the slot with its new pointer.
 // =============================================================================================
-template <int G>
-__global__ void k_point_group(const int32_t* __restrict__ list, const unsigned long long* cnt_ptr,
-                              const int64_t* __restrict__ offs, const uint64_t* __restrict__ adj,
-                              const uint32_t* __restrict__ bits, uint64_t* __restrict__ best) {
+constexpr int kNumCounters = 24;
+constexpr int kCntSwept = 16;
+__host__ __device__ constexpr int cnt_S(int set) { return 8 * set; }
+__host__ __device__ constexpr int cnt_F(int set, int b) { return 8 * set + 1 + b; }
+constexpr uint32_t kNoPtr = 0xffffffffu;
+
+__device__ __forceinline__ uint64_t make_pair(uint32_t lo, uint32_t hi) {
+  return (uint64_t)lo | ((uint64_t)hi << 32);
+}
+
+struct Bins {
+  uint64_t* list[kBins];
+};
+
+// A2 pointer phase on the frontier (rounds >= 2): G lanes per vertex (degree-binned).
+//   best[u] = max{ adj[j] : j in row(u), col != u, !matched(col) }   (Alg. 3 L5-8)
+// Keys are loaded U at a time per lane and the bitmap words of the candidates (keys above the
+// running max at batch start) are fetched together, so no L2 round trip sits on the loop-carried
+// max.  The new pointer is written to best[u] and into the frontier slot (for match/compaction).
+template <int G, int U>
+__device__ __forceinline__ uint64_t scan_row_available(const uint64_t* __restrict__ adj,
+                                                       const uint32_t* __restrict__ bits,
+                                                       int64_t s, int64_t e, uint32_t u, int gl) {
+  uint64_t b = 0;
+  for (int64_t j0 = s + gl; j0 < e; j0 += (int64_t)G * U) {
+    uint64_t k[U];
+#pragma unroll
+    for (int q = 0; q < U; ++q) {
+      const int64_t j = j0 + (int64_t)q * G;
+      k[q] = j < e ? __ldg(adj + j) : 0ull;
+    }
+    uint32_t wd[U];
+#pragma unroll
+    for (int q = 0; q < U; ++q) {
+      const uint32_t v = (uint32_t)k[q];
+      const bool cand = k[q] > b;  // zeroed self-loops never qualify
+      wd[q] = cand ? bits[v >> 5] : 0xffffffffu;
+    }
+#pragma unroll
+    for (int q = 0; q < U; ++q) {
+      const uint32_t v = (uint32_t)k[q];
+      if (!((wd[q] >> (v & 31)) & 1u) && k[q] > b) b = k[q];
+    }
+  }
+  return b;
+}
+
+template <int G, int U>
+__global__ void k_point_bin(uint64_t* __restrict__ list, const unsigned long long* cnt_ptr,
+                            const int64_t* __restrict__ offs, const uint64_t* __restrict__ adj,
+                            const uint32_t* __restrict__ bits, uint64_t* __restrict__ best) {
   const int64_t cnt = (int64_t)*cnt_ptr;
   const int lane = threadIdx.x & 31;
   const int gl = lane & (G - 1);
@@ -526,41 +811,35 @@ __global__ void k_point_group(const int32_t* __restrict__ list, const unsigned l
   const int64_t ng = ((int64_t)gridDim.x * blockDim.x) / G;
   for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / G; i < cnt; i += ng) {
     const uint32_t u = (uint32_t)list[i];
-    const int64_t s = offs[u], e = offs[u + 1];
-    uint64_t b = 0;
-    for (int64_t j = s + gl; j < e; j += G) {
-      const uint64_t key = adj[j];
-      const uint32_t v = (uint32_t)key;
-      if (v != u && key > b && !bit_test(bits, v)) b = key;
+    const uint64_t b = group_max_key(
+        scan_row_available<G, U>(adj, bits, offs[u], offs[u + 1], u, gl), gmask);
+    if (gl == 0) {
+      best[u] = b;
+      list[i] = make_pair(u, b ? (uint32_t)b : kNoPtr);
     }
-    b = group_max_key(b, gmask);
-    if (gl == 0) best[u] = b;
   }
 }
 
-template <int THREADS>
+template <int THREADS, int U>
 __global__ void __launch_bounds__(THREADS)
-    k_point_cta(const int32_t* __restrict__ list, const unsigned long long* cnt_ptr,
-                const int64_t* __restrict__ offs, const uint64_t* __restrict__ adj,
-                const uint32_t* __restrict__ bits, uint64_t* __restrict__ best) {
+    k_point_bin_cta(uint64_t* __restrict__ list, const unsigned long long* cnt_ptr,
+                    const int64_t* __restrict__ offs, const uint64_t* __restrict__ adj,
+                    const uint32_t* __restrict__ bits, uint64_t* __restrict__ best) {
   __shared__ uint64_t red[THREADS / 32];
   const int64_t cnt = (int64_t)*cnt_ptr;
   for (int64_t i = blockIdx.x; i < cnt; i += gridDim.x) {
     const uint32_t u = (uint32_t)list[i];
-    const int64_t s = offs[u], e = offs[u + 1];
-    uint64_t b = 0;
-    for (int64_t j = s + threadIdx.x; j < e; j += THREADS) {
-      const uint64_t key = adj[j];
-      const uint32_t v = (uint32_t)key;
-      if (v != u && key > b && !bit_test(bits, v)) b = key;
-    }
+    uint64_t b = scan_row_available<THREADS, U>(adj, bits, offs[u], offs[u + 1], u, threadIdx.x);
     b = group_max_key(b, 0xffffffffu);
     if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = b;
     __syncthreads();
     if (threadIdx.x < 32) {
       uint64_t x = threadIdx.x < THREADS / 32 ? red[threadIdx.x] : 0ull;
       x = group_max_key(x, 0xffffffffu);
-      if (threadIdx.x == 0) best[u] = x;
+      if (threadIdx.x == 0) {
+        best[u] = x;
+        list[i] = make_pair(u, x ? (uint32_t)x : kNoPtr);
+      }
     }
     __syncthreads();
   }
@@ -590,23 +869,19 @@ __global__ void k_match_all(const uint64_t* __restrict__ best, int64_t n, uint32
   }
 }
 
-// Rounds >= 2: the frontier (all bins).  A new mutual pair has at least one endpoint that
-// re-pointed this round (R3); that endpoint marks both.
-struct BinLists {
-  const int32_t* list[kBins];
-};
-__global__ void k_match_list(BinLists F, const unsigned long long* cnt,
+// Rounds >= 2: over the frontier's new pointers (pairs in the bins).  A new mutual pair has at
+// least one endpoint that re-pointed this round (R3); that endpoint marks both.
+__global__ void k_match_bins(Bins F, const unsigned long long* cntF,
                              const uint64_t* __restrict__ best, uint32_t* bits) {
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
 #pragma unroll
-  for (int b = 0; b < kBins; ++b) {
-    const int64_t c = (int64_t)cnt[b];
+  for (int bb = 0; bb < kBins; ++bb) {
+    const int64_t c = (int64_t)cntF[bb];
     for (int64_t i = tid; i < c; i += stride) {
-      const uint32_t u = (uint32_t)F.list[b][i];
-      const uint64_t k = best[u];
-      if (!k) continue;
-      const uint32_t v = (uint32_t)k;
+      const uint64_t p = F.list[bb][i];
+      const uint32_t u = (uint32_t)p, v = (uint32_t)(p >> 32);
+      if (v == kNoPtr) continue;
       const uint64_t kv = best[v];
       if (kv != 0 && (uint32_t)kv == u) {
         atomicOr(&bits[u >> 5], 1u << (u & 31));
@@ -617,77 +892,104 @@ __global__ void k_match_list(BinLists F, const unsigned long long* cnt,
 }
 
 // =============================================================================================
-// A6 frontier compaction (not in the paper, which rescans every unmatched vertex):
-//   L' = { u in L : !matched(u), best[u] != 0 }
-//   F' = { u in L' : matched(ptr u) }     binned by degree
-// counters layout: [0] |L'|, [1..kBins] |F'_b|, [kBins+1] sum of deg over F'
-// Each warp owns a chunk of 32*K items: pass 1 records the predicates in registers and counts,
-// ONE atomicAdd per list per warp reserves the output ranges, pass 2 writes -- so the global
-// counters see (items / 32K) atomics instead of one per 32 items.
+// A6 frontier compaction (not in the paper, which rescans every unmatched vertex).
+// The live set is kept as pairs (u, ptr u): S_r (pointers unchanged since an earlier round) and
+// the frontier bins of round r (fresh pointers).  For each live pair with u still unmatched:
+//   ptr u matched   -> u joins frontier bin deg(u) of round r+1 (pointer must be recomputed)
+//   ptr u unmatched -> (u, ptr u) joins S_{r+1}
+// Round 1 (ALL) derives the pairs from best[] over every vertex.  Inputs are streamed; the random
+// accesses are two bitmap bits (L2-resident) and, for frontier members only, deg(u).  Each warp
+// owns a chunk of 32*K items: ONE atomicAdd per output list per warp reserves its ranges.
 // =============================================================================================
 template <bool ALL, int K>
-__global__ void k_compact(const int32_t* __restrict__ L, const unsigned long long* Lcnt, int64_t n,
+__global__ void k_compact(const uint64_t* __restrict__ S, const unsigned long long* cntS,
+                          Bins Fin, const unsigned long long* cntFin, int64_t n,
                           const uint64_t* __restrict__ best, const uint32_t* __restrict__ bits,
-                          const int64_t* __restrict__ offs, int32_t* Lout, BinLists Fout,
-                          unsigned long long* counters) {
-  const int64_t cnt = ALL ? n : (int64_t)*Lcnt;
+                          const int64_t* __restrict__ offs, uint64_t* __restrict__ Sout,
+                          unsigned long long* cntSout, Bins Fout, unsigned long long* cntFout,
+                          unsigned long long* swept) {
+  int64_t c[1 + kBins];
+  c[0] = ALL ? n : (int64_t)*cntS;
+#pragma unroll
+  for (int b = 0; b < kBins; ++b) c[1 + b] = ALL ? 0 : (int64_t)cntFin[b];
+  int64_t cnt = 0;
+#pragma unroll
+  for (int b = 0; b <= kBins; ++b) cnt += c[b];
   const int lane = threadIdx.x & 31;
   const int64_t warp0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const unsigned lt = lanemask_lt();
   unsigned long long degsum = 0;
   for (int64_t c0 = warp0 * 32 * K; c0 < cnt; c0 += nwarps * 32 * K) {
-    uint32_t live = 0, binb[kBins] = {0, 0, 0, 0};
-    uint32_t uu[K];
+    uint32_t sbits = 0, fb[kBins] = {0, 0, 0, 0};
+    uint64_t pr[K];
 #pragma unroll
     for (int k = 0; k < K; ++k) {
-      const int64_t i = c0 + 32 * k + lane;
-      uu[k] = 0;
+      int64_t i = c0 + 32 * k + lane;
+      pr[k] = 0;
       if (i < cnt) {
-        const uint32_t u = ALL ? (uint32_t)i : (uint32_t)L[i];
-        uu[k] = u;
-        const uint64_t b = best[u];
-        if (b != 0 && !bit_test(bits, u)) {
-          live |= 1u << k;
-          if (bit_test(bits, (uint32_t)b)) {
+        uint32_t u, v;
+        if (ALL) {
+          u = (uint32_t)i;
+          const uint64_t bb = best[u];
+          v = bb ? (uint32_t)bb : kNoPtr;
+        } else {
+          uint64_t p;
+          if (i < c[0]) p = S[i];
+          else {
+            i -= c[0];
+            int b = 0;
+#pragma unroll
+            for (int q = 0; q < kBins - 1; ++q)
+              if (b == q && i >= c[1 + q]) { i -= c[1 + q]; b = q + 1; }
+            p = Fin.list[b][i];
+          }
+          u = (uint32_t)p;
+          v = (uint32_t)(p >> 32);
+        }
+        pr[k] = make_pair(u, v);
+        if (v != kNoPtr && !bit_test(bits, u)) {
+          if (bit_test(bits, v)) {
             const int64_t d = offs[u + 1] - offs[u];
-            binb[bin_of(d)] |= 1u << k;
+            fb[bin_of(d)] |= 1u << k;
             degsum += (unsigned long long)d;
+          } else {
+            sbits |= 1u << k;
           }
         }
       }
     }
-    // reserve output ranges: one atomic per list per warp
     unsigned long long base[1 + kBins];
     {
       unsigned tot[1 + kBins];
-      tot[0] = __reduce_add_sync(0xffffffffu, __popc(live));
+      tot[0] = __reduce_add_sync(0xffffffffu, __popc(sbits));
 #pragma unroll
-      for (int b = 0; b < kBins; ++b) tot[1 + b] = __reduce_add_sync(0xffffffffu, __popc(binb[b]));
+      for (int b = 0; b < kBins; ++b) tot[1 + b] = __reduce_add_sync(0xffffffffu, __popc(fb[b]));
+      unsigned long long x = 0;
+      if (lane == 0 && tot[0]) x = atomicAdd(cntSout, (unsigned long long)tot[0]);
 #pragma unroll
-      for (int q = 0; q < 1 + kBins; ++q) {
-        unsigned long long x = 0;
-        if (lane == q && tot[q]) x = atomicAdd(&counters[q], (unsigned long long)tot[q]);
-        base[q] = __shfl_sync(0xffffffffu, x, q);
-      }
+      for (int b = 0; b < kBins; ++b)
+        if (lane == 1 + b && tot[1 + b]) x = atomicAdd(&cntFout[b], (unsigned long long)tot[1 + b]);
+#pragma unroll
+      for (int q = 0; q <= kBins; ++q) base[q] = __shfl_sync(0xffffffffu, x, q);
     }
 #pragma unroll
     for (int k = 0; k < K; ++k) {
-      const bool pl = (live >> k) & 1u;
-      const unsigned bl = __ballot_sync(0xffffffffu, pl);
-      if (pl) Lout[base[0] + __popc(bl & lt)] = (int32_t)uu[k];
-      base[0] += __popc(bl);
+      const bool ps = (sbits >> k) & 1u;
+      const unsigned bls = __ballot_sync(0xffffffffu, ps);
+      if (ps) Sout[base[0] + __popc(bls & lt)] = pr[k];
+      base[0] += __popc(bls);
 #pragma unroll
       for (int b = 0; b < kBins; ++b) {
-        const bool pb = (binb[b] >> k) & 1u;
+        const bool pb = (fb[b] >> k) & 1u;
         const unsigned bb = __ballot_sync(0xffffffffu, pb);
-        if (pb) const_cast<int32_t*>(Fout.list[b])[base[1 + b] + __popc(bb & lt)] = (int32_t)uu[k];
+        if (pb) Fout.list[b][base[1 + b] + __popc(bb & lt)] = (uint64_t)(uint32_t)pr[k];
         base[1 + b] += __popc(bb);
       }
     }
   }
   for (int o = 16; o; o >>= 1) degsum += __shfl_xor_sync(0xffffffffu, degsum, o);
-  if (lane == 0 && degsum) atomicAdd(&counters[1 + kBins], degsum);
+  if (lane == 0 && degsum) atomicAdd(swept, degsum);
 }
 
 // =============================================================================================

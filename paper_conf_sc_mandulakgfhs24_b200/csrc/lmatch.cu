@@ -7,7 +7,9 @@
 //                    { A2 frontier pointer (per degree bin) -> A4 match -> A6 compact }* ->
 //                    A10 mate + A9 weight.  The loop ends when the next frontier is empty
 //                    (termination; R6).
+#include <cuda.h>
 #include <cuda_runtime.h>
+#include <cudaTypedefs.h>
 
 #include <algorithm>
 #include <climits>
@@ -16,6 +18,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <new>
+#include <vector>
 
 #include "../../include/lmatch.h"
 #include "kernels.cuh"
@@ -47,16 +50,38 @@ void set_err(const char* fmt, ...) {
   } while (0)
 
 // Round-1 sweep configuration (tuned on B200).
-constexpr int kSweepConsumers = 4;  // consumer warps (+1 TMA producer warp)
-constexpr int kSweepStages = 4;
-using Sweep = lm::SweepCfg<kSweepConsumers, kSweepStages>;
+#ifndef LM_SWEEP_TILE
+#define LM_SWEEP_TILE 512
+#endif
+#ifndef LM_SWEEP_RING
+#define LM_SWEEP_RING 2
+#endif
+#ifndef LM_SWEEP_WARPS
+#define LM_SWEEP_WARPS 8
+#endif
+#ifndef LM_SWEEP_WCAP
+#define LM_SWEEP_WCAP 72
+#endif
+constexpr int kSweepTile = LM_SWEEP_TILE;    // entries per warp tile
+constexpr int kSweepRing = LM_SWEEP_RING;    // TMA stages per warp
+constexpr int kSweepWarps = LM_SWEEP_WARPS;  // warps per CTA
+constexpr int kSweepWcap = LM_SWEEP_WCAP;    // staged row-window entries per stage
+#ifndef LM_SWEEP_IMPL
+#define LM_SWEEP_IMPL 1  // 2 = swizzled 2-D TMA + segmented scan; 1 = row-classified 1-D TMA
+#endif
+#if LM_SWEEP_IMPL == 2
+using Sweep = lm::Sweep2DCfg<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap>;
+#define SWEEP_KERNEL lm::k_sweep2d<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap>
+#else
+using Sweep = lm::SweepCfg<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap>;
+#define SWEEP_KERNEL lm::k_sweep<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap>
+#endif
 constexpr int kSweepThreads = Sweep::kThreads;
 constexpr int64_t kTile = Sweep::kTile;
 constexpr int kCompactK = 16;  // items per lane per compaction chunk
 
 constexpr int kFinBlocks = 592;  // 4 x 148 SMs: fixed => deterministic fp64 summation order
 constexpr int kFinThreads = 256;
-constexpr int kNumCounters = 2 * 8;
 
 int num_sms_cached = 0;
 
@@ -72,6 +97,7 @@ struct lmatch_graph {
   int64_t max_rounds = 0;
   int64_t upload_chunk = 1ll << 25;
   int sweep_grid = 0;
+  alignas(64) CUtensorMap tmap;  // adjacency as a [ceil(m/16)][16] u64 tensor, 128B swizzle
   int num_sms = 148;
   // graph
   int64_t* offs = nullptr;
@@ -85,9 +111,9 @@ struct lmatch_graph {
   // state
   uint64_t* best = nullptr;
   uint32_t* bits = nullptr;
-  int32_t* L[2] = {nullptr, nullptr};
-  int32_t* F[lm::kBins] = {};
-  unsigned long long* counters = nullptr;  // 2 sets of 8
+  uint64_t* S[2] = {nullptr, nullptr};      // stable live pairs (ping-pong)
+  lm::Bins F[2] = {};                       // frontier degree bins (ping-pong), pairs
+  unsigned long long* counters = nullptr;   // lm::kNumCounters
   unsigned long long* h_counters = nullptr;  // pinned mirror
   double* pw = nullptr;
   long long* pc = nullptr;
@@ -103,6 +129,7 @@ struct lmatch_graph {
   float* st_w[2] = {nullptr, nullptr};
   cudaEvent_t ev[8] = {};
   int64_t device_bytes = 0;
+  std::vector<int64_t> round_log;  // per round: |F_r|, |L_r|, E(F_r) (directed entries scanned)
 };
 
 namespace {
@@ -138,7 +165,9 @@ int check_args(const void* a, const void* b, const void* c, int64_t n, int64_t m
 int alloc_all(lmatch_graph* g) {
   const int64_t n = g->n, m = g->m;
   TRY(dmalloc(g, &g->offs, (size_t)n + 1));
-  TRY(dmalloc(g, &g->adj, (size_t)m + 2));
+  TRY(dmalloc(g, &g->adj, (size_t)m + 32));
+  // zero the padding past m: the sweep's 2-D tensor view reads whole 16-key rows
+  CK(cudaMemsetAsync(g->adj + m, 0, 32 * sizeof(uint64_t), g->stream));
   TRY(dmalloc(g, &g->noffs, (size_t)n + 5));
   TRY(dmalloc(g, &g->nzr, (size_t)n + 8));
   g->ntiles = (m + kTile - 1) / kTile;
@@ -147,16 +176,18 @@ int alloc_all(lmatch_graph* g) {
   TRY(dmalloc(g, &g->atomic_rows, (size_t)n + (size_t)g->ntiles + 1));
   TRY(dmalloc(g, &g->best, (size_t)n + 1));
   TRY(dmalloc(g, &g->bits, (size_t)((n + 31) / 32) + 1));
-  for (int i = 0; i < 2; ++i) TRY(dmalloc(g, &g->L[i], (size_t)n + 1));
-  for (int b = 0; b < lm::kBins; ++b) TRY(dmalloc(g, &g->F[b], (size_t)n + 1));
-  TRY(dmalloc(g, &g->counters, kNumCounters));
+  for (int i = 0; i < 2; ++i) {
+    TRY(dmalloc(g, &g->S[i], (size_t)n + 1));
+    for (int b = 0; b < lm::kBins; ++b) TRY(dmalloc(g, &g->F[i].list[b], (size_t)n + 1));
+  }
+  TRY(dmalloc(g, &g->counters, lm::kNumCounters));
   TRY(dmalloc(g, &g->pw, kFinBlocks));
   TRY(dmalloc(g, &g->pc, kFinBlocks));
   TRY(dmalloc(g, &g->res_w, 1));
   TRY(dmalloc(g, &g->res_c, 1));
   TRY(dmalloc(g, &g->perr, 1));
-  TRY(dmalloc(g, &g->werr, 1));
-  CK(cudaHostAlloc(reinterpret_cast<void**>(&g->h_counters), kNumCounters * 8, cudaHostAllocDefault));
+  TRY(dmalloc(g, &g->werr, 2));
+  CK(cudaHostAlloc(reinterpret_cast<void**>(&g->h_counters), lm::kNumCounters * 8, cudaHostAllocDefault));
   CK(cudaHostAlloc(reinterpret_cast<void**>(&g->h_res), 16, cudaHostAllocDefault));
   CK(cudaHostAlloc(reinterpret_cast<void**>(&g->h_resc), 16, cudaHostAllocDefault));
   // best[] = 0 for every vertex: empty rows are never written again (their pointer stays none)
@@ -194,8 +225,8 @@ int build_index(lmatch_graph* g, cudaStream_t st) {
     unsigned long long* cnt = nullptr;
     TRY(dmalloc(g, &cnt, 1));
     CK(cudaMemsetAsync(cnt, 0, 8, st));
-    lm::k_atomic_rows<<<grid_for(std::max(g->n_nz, g->ntiles), 256, 4096), 256, 0, st>>>(
-        g->noffs, g->nzr, g->n_nz, g->tile_nz, g->ntiles, kTile, Sweep::kPiece, g->atomic_rows, cnt);
+    lm::k_atomic_rows<<<grid_for(g->ntiles, 256, 4096), 256, 0, st>>>(
+        g->noffs, g->nzr, g->tile_nz, g->ntiles, kTile, g->atomic_rows, cnt);
     CKL();
     unsigned long long h_cnt = 0;
     CK(cudaMemcpyAsync(&h_cnt, cnt, 8, cudaMemcpyDeviceToHost, st));
@@ -306,16 +337,52 @@ int upload_device(lmatch_graph* g, const int64_t* d_offsets, const int32_t* d_co
   return LMATCH_OK;
 }
 
+int make_tensor_map(lmatch_graph* g) {
+  static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
+  if (!encode) {
+    cudaDriverEntryPointQueryResult q;
+    void* fn = nullptr;
+    CK(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q));
+    if (!fn || q != cudaDriverEntryPointSuccess) {
+      set_err("cuTensorMapEncodeTiled unavailable");
+      return LMATCH_ECUDA;
+    }
+    encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+  }
+  const cuuint64_t dims[2] = {16, (cuuint64_t)((g->m + 15) / 16)};
+  const cuuint64_t strides[1] = {128};
+  const cuuint32_t box[2] = {16, (cuuint32_t)(kTile / 16)};
+  const cuuint32_t es[2] = {1, 1};
+  const CUresult r = encode(&g->tmap, CU_TENSOR_MAP_DATA_TYPE_UINT64, 2, g->adj, dims, strides, box,
+                            es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) {
+    set_err("cuTensorMapEncodeTiled failed (%d)", (int)r);
+    return LMATCH_ECUDA;
+  }
+  return LMATCH_OK;
+}
+
 int finish_create(lmatch_graph* g, cudaStream_t st) {
+  if (g->m > 0) {
+    CK(cudaMemsetAsync(g->werr, 0, 8, st));
+    lm::k_zap_self_loops<<<grid_for(g->n * 8, 256, 16384), 256, 0, st>>>(
+        g->offs, g->adj, g->n, reinterpret_cast<unsigned long long*>(g->werr));
+    CKL();
+  }
   TRY(build_index(g, st));
+#if LM_SWEEP_IMPL == 2
+  if (g->ntiles > 0) TRY(make_tensor_map(g));
+#endif
   if (g->ntiles > 0) {
-    CK(cudaFuncSetAttribute(lm::k_sweep<kSweepConsumers, kSweepStages>,
+    CK(cudaFuncSetAttribute(SWEEP_KERNEL,
                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Sweep::kSmem));
     int occ = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-        &occ, lm::k_sweep<kSweepConsumers, kSweepStages>, kSweepThreads, Sweep::kSmem));
+        &occ, SWEEP_KERNEL, kSweepThreads, Sweep::kSmem));
     if (occ < 1) occ = 1;
-    g->sweep_grid = (int)std::min<int64_t>(g->ntiles, (int64_t)occ * g->num_sms);
+    g->sweep_grid = (int)std::min<int64_t>((g->ntiles + kSweepWarps - 1) / kSweepWarps,
+                                           (int64_t)occ * g->num_sms);
   }
   CK(cudaStreamSynchronize(st));
   return LMATCH_OK;
@@ -373,11 +440,13 @@ void lmatch_destroy(lmatch_graph* g) {
   if (!g) return;
   cudaSetDevice(g->device);
   if (g->stream) cudaStreamSynchronize(g->stream);
-  void* dev[] = {g->offs, g->adj, g->noffs, g->nzr, g->tile_nz, g->noffs_lo, g->atomic_rows, g->best, g->bits, g->L[0], g->L[1],
+  void* dev[] = {g->offs, g->adj, g->noffs, g->nzr, g->tile_nz, g->noffs_lo, g->atomic_rows, g->best,
+                 g->bits, g->S[0], g->S[1],
                  g->counters, g->pw, g->pc, g->res_w, g->res_c, g->mate_tmp, g->perr, g->werr,
                  g->st_col[0], g->st_col[1], g->st_w[0], g->st_w[1]};
   for (void* p : dev) if (p) cudaFree(p);
-  for (auto p : g->F) if (p) cudaFree(p);
+  for (auto& F : g->F)
+    for (auto p : F.list) if (p) cudaFree(p);
   if (g->h_counters) cudaFreeHost(g->h_counters);
   if (g->h_res) cudaFreeHost(g->h_res);
   if (g->h_resc) cudaFreeHost(g->h_resc);
@@ -443,6 +512,15 @@ int lmatch_reload(lmatch_graph* g, const int64_t* csr_offsets, const int32_t* co
   return LMATCH_OK;
 }
 
+int lmatch_round_log(const lmatch_graph* g, int64_t* out, int64_t cap, int64_t* nrounds) {
+  if (!g) { set_err("NULL handle"); return LMATCH_ESTATE; }
+  const int64_t r = (int64_t)g->round_log.size() / 3;
+  if (nrounds) *nrounds = r;
+  if (out)
+    for (int64_t i = 0; i < std::min<int64_t>(3 * r, 3 * cap); ++i) out[i] = g->round_log[(size_t)i];
+  return LMATCH_OK;
+}
+
 int lmatch_info(const lmatch_graph* g, int64_t* n, int64_t* m, int64_t* nonempty_rows,
                 int64_t* device_bytes) {
   if (!g) { set_err("NULL handle"); return LMATCH_ESTATE; }
@@ -461,64 +539,74 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
   cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
   const int64_t n = g->n;
   const bool tm = g->timing && stats;
-  int64_t launches = 0, rounds = 0, swept = 0, ftot_all = 0;
-  unsigned long long* cset[2] = {g->counters, g->counters + 8};
+  int64_t launches = 0, rounds = 0, ftot_all = 0;
+  unsigned long long* C = g->counters;
+  unsigned long long* hc = g->h_counters;
+  g->round_log.clear();
 
   if (tm) CK(cudaEventRecord(g->ev[0], st));
   // ---- reset (bitmap, counters, tile-crossing rows' best)
   const int64_t nwords = (n + 31) / 32;
   lm::k_reset<<<grid_for(std::max(nwords, g->n_atomic), 256, 4096), 256, 0, st>>>(
-      g->bits, nwords, g->best, g->atomic_rows, g->n_atomic, g->counters, kNumCounters);
+      g->bits, nwords, g->best, g->atomic_rows, g->n_atomic, C, lm::kNumCounters);
   CKL();
   ++launches;
   if (tm) CK(cudaEventRecord(g->ev[1], st));
   if (g->ntiles > 0 && n > 0) {
     // ---- round 1: A2 full sweep (no bitmap test), A4 match-all, A6 compact-all
+#if LM_SWEEP_IMPL == 2
+    lm::Sweep2DArgs A{g->noffs_lo, g->nzr, g->tile_nz, g->best, g->m, g->ntiles};
+    SWEEP_KERNEL<<<g->sweep_grid, kSweepThreads, Sweep::kSmem, st>>>(g->tmap, A);
+#else
     lm::SweepArgs A{g->adj, g->noffs_lo, g->nzr, g->tile_nz, g->best, g->m, g->ntiles};
-    lm::k_sweep<kSweepConsumers, kSweepStages>
-        <<<g->sweep_grid, kSweepThreads, Sweep::kSmem, st>>>(A);
+    SWEEP_KERNEL<<<g->sweep_grid, kSweepThreads, Sweep::kSmem, st>>>(A);
+#endif
     CKL();
-    ++launches;
     if (tm) CK(cudaEventRecord(g->ev[2], st));
     rounds = 1;
-    swept = g->m;
     lm::k_match_all<<<grid_for(nwords * 32, 256, 65536), 256, 0, st>>>(g->best, n, g->bits);
     CKL();
-    lm::BinLists Fl{};
-    for (int b = 0; b < lm::kBins; ++b) Fl.list[b] = g->F[b];
     lm::k_compact<true, kCompactK><<<grid_for((n + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
-        nullptr, nullptr, n, g->best, g->bits, g->offs, g->L[0], Fl, cset[0]);
+        nullptr, nullptr, lm::Bins{}, nullptr, n, g->best, g->bits, g->offs, g->S[0],
+        C + lm::cnt_S(0), g->F[0], C + lm::cnt_F(0, 0), C + lm::kCntSwept);
     CKL();
-    launches += 2;
-    CK(cudaMemcpyAsync(g->h_counters, cset[0], 64, cudaMemcpyDeviceToHost, st));
+    launches += 3;
+    CK(cudaMemcpyAsync(hc, C, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
     if (tm) CK(cudaEventRecord(g->ev[3], st));
+    g->round_log.insert(g->round_log.end(), {g->n_nz, n, g->m});
     int cur = 0;
+    unsigned long long swept_prev = 0;
     for (;;) {
-      const unsigned long long* hc = g->h_counters + 8 * cur;
-      int64_t fb[lm::kBins], ftot = 0;
-      for (int b = 0; b < lm::kBins; ++b) { fb[b] = (int64_t)hc[1 + b]; ftot += fb[b]; }
-      const int64_t lcnt = (int64_t)hc[0];
-      if (ftot == 0 || rounds >= g->max_rounds) break;
+      const int64_t nS = (int64_t)hc[lm::cnt_S(cur)];
+      int64_t nFb[lm::kBins], nF = 0;
+      for (int b = 0; b < lm::kBins; ++b) { nFb[b] = (int64_t)hc[lm::cnt_F(cur, b)]; nF += nFb[b]; }
+      if (nF == 0 || rounds >= g->max_rounds) break;
       ++rounds;
-      swept += (int64_t)hc[1 + lm::kBins];
-      ftot_all += ftot;
+      ftot_all += nF;
+      g->round_log.insert(g->round_log.end(),
+                          {nF, nS + nF, (int64_t)(hc[lm::kCntSwept] - swept_prev)});
+      swept_prev = hc[lm::kCntSwept];
+      const unsigned long long* cF = C + lm::cnt_F(cur, 0);
       // A2 frontier pointer phase, one launch per non-empty degree bin
-      if (fb[0]) { lm::k_point_group<4><<<grid_for(fb[0] * 4, 256, 65536), 256, 0, st>>>(g->F[0], cset[cur] + 1, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }
-      if (fb[1]) { lm::k_point_group<16><<<grid_for(fb[1] * 16, 256, 65536), 256, 0, st>>>(g->F[1], cset[cur] + 2, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }
-      if (fb[2]) { lm::k_point_group<32><<<grid_for(fb[2] * 32, 256, 65536), 256, 0, st>>>(g->F[2], cset[cur] + 3, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }
-      if (fb[3]) { lm::k_point_cta<256><<<(unsigned)std::min<int64_t>(fb[3], 65536), 256, 0, st>>>(g->F[3], cset[cur] + 4, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }
-      // A4 match
-      lm::k_match_list<<<grid_for(ftot, 256, 65536), 256, 0, st>>>(Fl, cset[cur] + 1, g->best, g->bits);
+      lm::Bins& Fb = g->F[cur];
+      if (nFb[0]) { lm::k_point_bin<4, 2><<<grid_for(nFb[0] * 4, 256, 65536), 256, 0, st>>>(Fb.list[0], cF + 0, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }
+      if (nFb[1]) { lm::k_point_bin<16, 4><<<grid_for(nFb[1] * 16, 256, 65536), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }
+      if (nFb[2]) { lm::k_point_bin<32, 4><<<grid_for(nFb[2] * 32, 256, 65536), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }
+      if (nFb[3]) { lm::k_point_bin_cta<256, 4><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }
+      // A4 match over the new pointers
+      lm::k_match_bins<<<grid_for(nF, 256, 65536), 256, 0, st>>>(Fb, cF, g->best, g->bits);
       CKL();
-      // A6 compaction of the live list
+      // A6 compaction of the live pairs
       const int nxt = cur ^ 1;
-      CK(cudaMemsetAsync(cset[nxt], 0, 64, st));
-      lm::k_compact<false, kCompactK><<<grid_for((lcnt + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
-          g->L[cur], cset[cur], n, g->best, g->bits, g->offs, g->L[nxt], Fl, cset[nxt]);
+      CK(cudaMemsetAsync(C + lm::cnt_S(nxt), 0, 8 * (1 + lm::kBins), st));
+      lm::k_compact<false, kCompactK>
+          <<<grid_for((nS + nF + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
+              g->S[cur], C + lm::cnt_S(cur), Fb, cF, n, g->best, g->bits, g->offs, g->S[nxt],
+              C + lm::cnt_S(nxt), g->F[nxt], C + lm::cnt_F(nxt, 0), C + lm::kCntSwept);
       CKL();
       launches += 2;
-      CK(cudaMemcpyAsync(g->h_counters + 8 * nxt, cset[nxt], 64, cudaMemcpyDeviceToHost, st));
+      CK(cudaMemcpyAsync(hc, C, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
       CK(cudaStreamSynchronize(st));
       cur = nxt;
     }
@@ -549,7 +637,8 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
     stats->matched_vertices = g->h_resc[0];
     stats->cardinality = g->h_resc[0] / 2;
     stats->weight = g->h_res[0];
-    stats->entries_swept = swept;
+    stats->entries_swept = 0;
+    for (size_t i = 2; i < g->round_log.size(); i += 3) stats->entries_swept += g->round_log[i];
     stats->frontier_total = ftot_all;
     stats->sweep_launches = (g->ntiles > 0 && n > 0) ? 1 : 0;
     stats->kernel_launches = launches;
