@@ -24,7 +24,7 @@
 namespace lm {
 
 constexpr int kBins = 4;               // frontier degree bins
-constexpr int kBinDeg0 = 8, kBinDeg1 = 128, kBinDeg2 = 4096;  // bins: G = 4, 16, 32 lanes, CTA
+constexpr int kBinDeg0 = 8, kBinDeg1 = 64, kBinDeg2 = 2048;  // bins: G = 1, 8, 32 lanes, CTA
 
 // --------------------------------------------------------------------------- small helpers
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -148,6 +148,21 @@ __global__ void k_zap_self_loops(const int64_t* __restrict__ offs, uint64_t* adj
       if ((uint32_t)adj[j] == (uint32_t)u) { adj[j] = 0ull; ++c; }
   for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
   if ((threadIdx.x & 31) == 0 && c) atomicAdd(count, c);
+}
+
+// number of vertices in each frontier degree bin (static capacity of the bin lists)
+__global__ void k_bin_sizes(const int64_t* __restrict__ offs, int64_t n, unsigned long long* cnt) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  unsigned long long c[kBins] = {0, 0, 0, 0};
+  for (int64_t u = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; u < n; u += stride) {
+    const int64_t d = offs[u + 1] - offs[u];
+    if (d > 0) ++c[bin_of(d)];
+  }
+#pragma unroll
+  for (int b = 0; b < kBins; ++b) {
+    for (int o = 16; o; o >>= 1) c[b] += __shfl_xor_sync(0xffffffffu, c[b], o);
+    if ((threadIdx.x & 31) == 0 && c[b]) atomicAdd(&cnt[b], c[b]);
+  }
 }
 
 __global__ void k_check_offsets(const int64_t* __restrict__ offs, int64_t n, int64_t m,
@@ -746,36 +761,45 @@ __global__ void k_low32(const int64_t* __restrict__ noffs, int64_t cnt, uint32_t
 }
 
 // =============================================================================================
-// Rounds >= 2.  Device counters (unsigned long long, RoundCounters layout, kNumCounters):
+// Rounds >= 2.  Device counters (unsigned long long, kNumCounters):
 //   [8 * set]               |S| of pair set `set` (stable live pairs)
 //   [8 * set + 1 + b]       |F_b| of frontier set `set`, degree bin b
 //   [16]                    adjacency entries of all frontiers produced so far (stats)
-// Lists: S = uint64 pairs (u | ptr u << 32); frontier bins = uint64 pairs (u | new ptr << 32):
-// the compaction writes (u, 0) and the pointer kernel overwrites the slot with its new pointer.
+// Lists: S = uint64 pairs (u | ptr u << 32).  Frontier bins = 16-byte entries
+//   .x = u | ptr << 32 (the pointer kernel overwrites ptr with the new pointer)
+//   .y = row start | degree << 40 (degree >= 2^24 stored as kBigDeg: read offs instead)
+// so the pointer kernel streams its row without a dependent offs[] lookup.
 // =============================================================================================
 constexpr int kNumCounters = 24;
 constexpr int kCntSwept = 16;
 __host__ __device__ constexpr int cnt_S(int set) { return 8 * set; }
 __host__ __device__ constexpr int cnt_F(int set, int b) { return 8 * set + 1 + b; }
 constexpr uint32_t kNoPtr = 0xffffffffu;
+constexpr uint64_t kBigDeg = (1ull << 24) - 1;
 
 __device__ __forceinline__ uint64_t make_pair(uint32_t lo, uint32_t hi) {
   return (uint64_t)lo | ((uint64_t)hi << 32);
 }
+__device__ __forceinline__ void row_range(const ulonglong2& e, const int64_t* __restrict__ offs,
+                                          int64_t* s, int64_t* en) {
+  const uint64_t d = e.y >> 40;
+  *s = (int64_t)(e.y & ((1ull << 40) - 1));
+  *en = d == kBigDeg ? offs[(uint32_t)e.x + 1] : *s + (int64_t)d;
+}
 
 struct Bins {
-  uint64_t* list[kBins];
+  ulonglong2* list[kBins];
 };
 
 // A2 pointer phase on the frontier (rounds >= 2): G lanes per vertex (degree-binned).
-//   best[u] = max{ adj[j] : j in row(u), col != u, !matched(col) }   (Alg. 3 L5-8)
+//   best[u] = max{ adj[j] : j in row(u), !matched(col) }   (Alg. 3 L5-8)
 // Keys are loaded U at a time per lane and the bitmap words of the candidates (keys above the
 // running max at batch start) are fetched together, so no L2 round trip sits on the loop-carried
-// max.  The new pointer is written to best[u] and into the frontier slot (for match/compaction).
+// max.  Zeroed self-loop keys never qualify.  The new pointer goes to best[u] and into the slot.
 template <int G, int U>
 __device__ __forceinline__ uint64_t scan_row_available(const uint64_t* __restrict__ adj,
                                                        const uint32_t* __restrict__ bits,
-                                                       int64_t s, int64_t e, uint32_t u, int gl) {
+                                                       int64_t s, int64_t e, int gl) {
   uint64_t b = 0;
   for (int64_t j0 = s + gl; j0 < e; j0 += (int64_t)G * U) {
     uint64_t k[U];
@@ -786,11 +810,7 @@ __device__ __forceinline__ uint64_t scan_row_available(const uint64_t* __restric
     }
     uint32_t wd[U];
 #pragma unroll
-    for (int q = 0; q < U; ++q) {
-      const uint32_t v = (uint32_t)k[q];
-      const bool cand = k[q] > b;  // zeroed self-loops never qualify
-      wd[q] = cand ? bits[v >> 5] : 0xffffffffu;
-    }
+    for (int q = 0; q < U; ++q) wd[q] = k[q] > b ? bits[(uint32_t)k[q] >> 5] : 0xffffffffu;
 #pragma unroll
     for (int q = 0; q < U; ++q) {
       const uint32_t v = (uint32_t)k[q];
@@ -801,7 +821,7 @@ __device__ __forceinline__ uint64_t scan_row_available(const uint64_t* __restric
 }
 
 template <int G, int U>
-__global__ void k_point_bin(uint64_t* __restrict__ list, const unsigned long long* cnt_ptr,
+__global__ void k_point_bin(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
                             const int64_t* __restrict__ offs, const uint64_t* __restrict__ adj,
                             const uint32_t* __restrict__ bits, uint64_t* __restrict__ best) {
   const int64_t cnt = (int64_t)*cnt_ptr;
@@ -810,26 +830,30 @@ __global__ void k_point_bin(uint64_t* __restrict__ list, const unsigned long lon
   const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
   const int64_t ng = ((int64_t)gridDim.x * blockDim.x) / G;
   for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / G; i < cnt; i += ng) {
-    const uint32_t u = (uint32_t)list[i];
-    const uint64_t b = group_max_key(
-        scan_row_available<G, U>(adj, bits, offs[u], offs[u + 1], u, gl), gmask);
+    const ulonglong2 e = list[i];
+    int64_t s, en;
+    row_range(e, offs, &s, &en);
+    const uint64_t b = group_max_key(scan_row_available<G, U>(adj, bits, s, en, gl), gmask);
     if (gl == 0) {
+      const uint32_t u = (uint32_t)e.x;
       best[u] = b;
-      list[i] = make_pair(u, b ? (uint32_t)b : kNoPtr);
+      list[i].x = make_pair(u, b ? (uint32_t)b : kNoPtr);
     }
   }
 }
 
 template <int THREADS, int U>
 __global__ void __launch_bounds__(THREADS)
-    k_point_bin_cta(uint64_t* __restrict__ list, const unsigned long long* cnt_ptr,
+    k_point_bin_cta(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
                     const int64_t* __restrict__ offs, const uint64_t* __restrict__ adj,
                     const uint32_t* __restrict__ bits, uint64_t* __restrict__ best) {
   __shared__ uint64_t red[THREADS / 32];
   const int64_t cnt = (int64_t)*cnt_ptr;
   for (int64_t i = blockIdx.x; i < cnt; i += gridDim.x) {
-    const uint32_t u = (uint32_t)list[i];
-    uint64_t b = scan_row_available<THREADS, U>(adj, bits, offs[u], offs[u + 1], u, threadIdx.x);
+    const ulonglong2 e = list[i];
+    int64_t s, en;
+    row_range(e, offs, &s, &en);
+    uint64_t b = scan_row_available<THREADS, U>(adj, bits, s, en, threadIdx.x);
     b = group_max_key(b, 0xffffffffu);
     if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = b;
     __syncthreads();
@@ -837,8 +861,9 @@ __global__ void __launch_bounds__(THREADS)
       uint64_t x = threadIdx.x < THREADS / 32 ? red[threadIdx.x] : 0ull;
       x = group_max_key(x, 0xffffffffu);
       if (threadIdx.x == 0) {
+        const uint32_t u = (uint32_t)e.x;
         best[u] = x;
-        list[i] = make_pair(u, x ? (uint32_t)x : kNoPtr);
+        list[i].x = make_pair(u, x ? (uint32_t)x : kNoPtr);
       }
     }
     __syncthreads();
@@ -879,7 +904,7 @@ __global__ void k_match_bins(Bins F, const unsigned long long* cntF,
   for (int bb = 0; bb < kBins; ++bb) {
     const int64_t c = (int64_t)cntF[bb];
     for (int64_t i = tid; i < c; i += stride) {
-      const uint64_t p = F.list[bb][i];
+      const uint64_t p = F.list[bb][i].x;
       const uint32_t u = (uint32_t)p, v = (uint32_t)(p >> 32);
       if (v == kNoPtr) continue;
       const uint64_t kv = best[v];
@@ -902,90 +927,128 @@ __global__ void k_match_bins(Bins F, const unsigned long long* cntF,
 // owns a chunk of 32*K items: ONE atomicAdd per output list per warp reserves its ranges.
 // =============================================================================================
 template <bool ALL, int K>
-__global__ void k_compact(const uint64_t* __restrict__ S, const unsigned long long* cntS,
-                          Bins Fin, const unsigned long long* cntFin, int64_t n,
-                          const uint64_t* __restrict__ best, const uint32_t* __restrict__ bits,
-                          const int64_t* __restrict__ offs, uint64_t* __restrict__ Sout,
-                          unsigned long long* cntSout, Bins Fout, unsigned long long* cntFout,
-                          unsigned long long* swept) {
-  int64_t c[1 + kBins];
-  c[0] = ALL ? n : (int64_t)*cntS;
-#pragma unroll
-  for (int b = 0; b < kBins; ++b) c[1 + b] = ALL ? 0 : (int64_t)cntFin[b];
-  int64_t cnt = 0;
-#pragma unroll
-  for (int b = 0; b <= kBins; ++b) cnt += c[b];
-  const int lane = threadIdx.x & 31;
-  const int64_t warp0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+__global__ void __launch_bounds__(256)
+    k_compact(const uint64_t* __restrict__ S, const unsigned long long* cntS, Bins Fin,
+              const unsigned long long* cntFin, int64_t n, const uint64_t* __restrict__ best,
+              const uint32_t* __restrict__ bits, const int64_t* __restrict__ offs,
+              uint64_t* __restrict__ Sout, unsigned long long* cntSout, Bins Fout,
+              unsigned long long* cntFout, unsigned long long* swept) {
+  constexpr int NW = 8, NL = 1 + kBins;  // warps per block (blockDim 256), output lists
+  __shared__ unsigned wtot[NW][NL];
+  __shared__ unsigned long long wbase[NW][NL];
+  // virtual concatenation S ++ F_0 ++ F_1 ++ F_2 ++ F_3 (prefix ends p0 < p1 < ... < p4)
+  const int64_t p0 = ALL ? n : (int64_t)*cntS;
+  const int64_t p1 = p0 + (ALL ? 0 : (int64_t)cntFin[0]);
+  const int64_t p2 = p1 + (ALL ? 0 : (int64_t)cntFin[1]);
+  const int64_t p3 = p2 + (ALL ? 0 : (int64_t)cntFin[2]);
+  const int64_t cnt = p3 + (ALL ? 0 : (int64_t)cntFin[3]);
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const unsigned lt = lanemask_lt();
+  constexpr int64_t BLK = (int64_t)NW * 32 * K;
   unsigned long long degsum = 0;
-  for (int64_t c0 = warp0 * 32 * K; c0 < cnt; c0 += nwarps * 32 * K) {
-    uint32_t sbits = 0, fb[kBins] = {0, 0, 0, 0};
-    uint64_t pr[K];
+  for (int64_t cb = (int64_t)blockIdx.x * BLK; cb < cnt; cb += (int64_t)gridDim.x * BLK) {
+    const int64_t c0 = cb + (int64_t)warp * 32 * K;
+    uint32_t sbits = 0, fb0 = 0, fb1 = 0, fb2 = 0, fb3 = 0;
+    uint64_t pr[K], rr[K];
+    // phase 1: every list element of the chunk (independent loads)
 #pragma unroll
     for (int k = 0; k < K; ++k) {
-      int64_t i = c0 + 32 * k + lane;
-      pr[k] = 0;
+      const int64_t i = c0 + 32 * k + lane;
+      uint64_t p = (uint64_t)kNoPtr << 32;
       if (i < cnt) {
-        uint32_t u, v;
         if (ALL) {
-          u = (uint32_t)i;
-          const uint64_t bb = best[u];
-          v = bb ? (uint32_t)bb : kNoPtr;
+          const uint64_t bb = best[i];
+          p = make_pair((uint32_t)i, bb ? (uint32_t)bb : kNoPtr);
         } else {
-          uint64_t p;
-          if (i < c[0]) p = S[i];
-          else {
-            i -= c[0];
-            int b = 0;
-#pragma unroll
-            for (int q = 0; q < kBins - 1; ++q)
-              if (b == q && i >= c[1 + q]) { i -= c[1 + q]; b = q + 1; }
-            p = Fin.list[b][i];
-          }
-          u = (uint32_t)p;
-          v = (uint32_t)(p >> 32);
-        }
-        pr[k] = make_pair(u, v);
-        if (v != kNoPtr && !bit_test(bits, u)) {
-          if (bit_test(bits, v)) {
-            const int64_t d = offs[u + 1] - offs[u];
-            fb[bin_of(d)] |= 1u << k;
-            degsum += (unsigned long long)d;
-          } else {
-            sbits |= 1u << k;
-          }
+          p = i < p0 ? S[i]
+              : i < p1 ? Fin.list[0][i - p0].x
+              : i < p2 ? Fin.list[1][i - p1].x
+              : i < p3 ? Fin.list[2][i - p2].x
+                       : Fin.list[3][i - p3].x;
         }
       }
+      pr[k] = p;
     }
-    unsigned long long base[1 + kBins];
-    {
-      unsigned tot[1 + kBins];
-      tot[0] = __reduce_add_sync(0xffffffffu, __popc(sbits));
+    // phase 2: matched bits of u and of its pointer (L2-resident bitmap; independent loads)
+    uint32_t wu[K], wv[K];
 #pragma unroll
-      for (int b = 0; b < kBins; ++b) tot[1 + b] = __reduce_add_sync(0xffffffffu, __popc(fb[b]));
-      unsigned long long x = 0;
-      if (lane == 0 && tot[0]) x = atomicAdd(cntSout, (unsigned long long)tot[0]);
+    for (int k = 0; k < K; ++k) {
+      const uint32_t u = (uint32_t)pr[k], v = (uint32_t)(pr[k] >> 32);
+      const bool ok = v != kNoPtr;
+      wu[k] = ok ? bits[u >> 5] : 0xffffffffu;
+      wv[k] = ok ? bits[v >> 5] : 0u;
+    }
+    // phase 3: classify; frontier members fetch their row range (independent loads)
+    int64_t os[K], oe[K];
 #pragma unroll
-      for (int b = 0; b < kBins; ++b)
-        if (lane == 1 + b && tot[1 + b]) x = atomicAdd(&cntFout[b], (unsigned long long)tot[1 + b]);
-#pragma unroll
-      for (int q = 0; q <= kBins; ++q) base[q] = __shfl_sync(0xffffffffu, x, q);
+    for (int k = 0; k < K; ++k) {
+      const uint32_t u = (uint32_t)pr[k], v = (uint32_t)(pr[k] >> 32);
+      const bool live = !((wu[k] >> (u & 31)) & 1u);
+      const bool tgt = (wv[k] >> (v & 31)) & 1u;
+      if (live && !tgt) sbits |= 1u << k;
+      const bool fr = live && tgt;
+      os[k] = fr ? offs[u] : 0;
+      oe[k] = fr ? offs[u + 1] : -1;
     }
 #pragma unroll
     for (int k = 0; k < K; ++k) {
-      const bool ps = (sbits >> k) & 1u;
-      const unsigned bls = __ballot_sync(0xffffffffu, ps);
-      if (ps) Sout[base[0] + __popc(bls & lt)] = pr[k];
-      base[0] += __popc(bls);
-#pragma unroll
-      for (int b = 0; b < kBins; ++b) {
-        const bool pb = (fb[b] >> k) & 1u;
-        const unsigned bb = __ballot_sync(0xffffffffu, pb);
-        if (pb) Fout.list[b][base[1 + b] + __popc(bb & lt)] = (uint64_t)(uint32_t)pr[k];
-        base[1 + b] += __popc(bb);
+      rr[k] = 0;
+      if (oe[k] >= 0) {
+        const int64_t d = oe[k] - os[k];
+        const int b = bin_of(d);
+        const uint32_t m = 1u << k;
+        fb0 |= b == 0 ? m : 0u;
+        fb1 |= b == 1 ? m : 0u;
+        fb2 |= b == 2 ? m : 0u;
+        fb3 |= b == 3 ? m : 0u;
+        rr[k] = (uint64_t)os[k] | ((uint64_t)(d < (int64_t)kBigDeg ? d : (int64_t)kBigDeg) << 40);
+        degsum += (unsigned long long)d;
       }
+    }
+    // reserve output ranges: warp totals -> block prefix -> ONE atomic per list per block
+    {
+      const unsigned ts = __reduce_add_sync(0xffffffffu, __popc(sbits));
+      const unsigned t0 = __reduce_add_sync(0xffffffffu, __popc(fb0));
+      const unsigned t1 = __reduce_add_sync(0xffffffffu, __popc(fb1));
+      const unsigned t2 = __reduce_add_sync(0xffffffffu, __popc(fb2));
+      const unsigned t3 = __reduce_add_sync(0xffffffffu, __popc(fb3));
+      if (lane == 0) {
+        wtot[warp][0] = ts; wtot[warp][1] = t0; wtot[warp][2] = t1;
+        wtot[warp][3] = t2; wtot[warp][4] = t3;
+      }
+    }
+    __syncthreads();
+    if (threadIdx.x < NL) {
+      const int q = threadIdx.x;
+      unsigned long long tot = 0;
+      for (int w = 0; w < NW; ++w) tot += wtot[w][q];
+      unsigned long long base = 0;
+      if (tot) base = atomicAdd(q == 0 ? cntSout : &cntFout[q - 1], tot);
+      for (int w = 0; w < NW; ++w) { wbase[w][q] = base; base += wtot[w][q]; }
+    }
+    __syncthreads();
+    unsigned long long bs = wbase[warp][0], bf0 = wbase[warp][1], bf1 = wbase[warp][2],
+                       bf2 = wbase[warp][3], bf3 = wbase[warp][4];
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+      const uint32_t m = 1u << k;
+      const bool ps = sbits & m;
+      const unsigned bls = __ballot_sync(0xffffffffu, ps);
+      if (ps) Sout[bs + __popc(bls & lt)] = pr[k];
+      bs += __popc(bls);
+      const ulonglong2 ent = make_ulonglong2(pr[k], rr[k]);
+      unsigned bb = __ballot_sync(0xffffffffu, (fb0 & m) != 0);
+      if (fb0 & m) Fout.list[0][bf0 + __popc(bb & lt)] = ent;
+      bf0 += __popc(bb);
+      bb = __ballot_sync(0xffffffffu, (fb1 & m) != 0);
+      if (fb1 & m) Fout.list[1][bf1 + __popc(bb & lt)] = ent;
+      bf1 += __popc(bb);
+      bb = __ballot_sync(0xffffffffu, (fb2 & m) != 0);
+      if (fb2 & m) Fout.list[2][bf2 + __popc(bb & lt)] = ent;
+      bf2 += __popc(bb);
+      bb = __ballot_sync(0xffffffffu, (fb3 & m) != 0);
+      if (fb3 & m) Fout.list[3][bf3 + __popc(bb & lt)] = ent;
+      bf3 += __popc(bb);
     }
   }
   for (int o = 16; o; o >>= 1) degsum += __shfl_xor_sync(0xffffffffu, degsum, o);

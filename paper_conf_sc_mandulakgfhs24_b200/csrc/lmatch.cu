@@ -78,7 +78,7 @@ using Sweep = lm::SweepCfg<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap>;
 #endif
 constexpr int kSweepThreads = Sweep::kThreads;
 constexpr int64_t kTile = Sweep::kTile;
-constexpr int kCompactK = 16;  // items per lane per compaction chunk
+constexpr int kCompactK = 8;  // items per lane per compaction chunk
 
 constexpr int kFinBlocks = 592;  // 4 x 148 SMs: fixed => deterministic fp64 summation order
 constexpr int kFinThreads = 256;
@@ -176,10 +176,7 @@ int alloc_all(lmatch_graph* g) {
   TRY(dmalloc(g, &g->atomic_rows, (size_t)n + (size_t)g->ntiles + 1));
   TRY(dmalloc(g, &g->best, (size_t)n + 1));
   TRY(dmalloc(g, &g->bits, (size_t)((n + 31) / 32) + 1));
-  for (int i = 0; i < 2; ++i) {
-    TRY(dmalloc(g, &g->S[i], (size_t)n + 1));
-    for (int b = 0; b < lm::kBins; ++b) TRY(dmalloc(g, &g->F[i].list[b], (size_t)n + 1));
-  }
+  for (int i = 0; i < 2; ++i) TRY(dmalloc(g, &g->S[i], (size_t)n + 1));
   TRY(dmalloc(g, &g->counters, lm::kNumCounters));
   TRY(dmalloc(g, &g->pw, kFinBlocks));
   TRY(dmalloc(g, &g->pc, kFinBlocks));
@@ -363,7 +360,27 @@ int make_tensor_map(lmatch_graph* g) {
   return LMATCH_OK;
 }
 
+// frontier bin lists: bin b can never hold more than the vertices of its degree class
+int alloc_bins(lmatch_graph* g, cudaStream_t st) {
+  if (g->F[0].list[0]) return LMATCH_OK;  // reload: same graph shape
+  unsigned long long* cnt = nullptr;
+  TRY(dmalloc(g, &cnt, lm::kBins));
+  CK(cudaMemsetAsync(cnt, 0, 8 * lm::kBins, st));
+  if (g->n > 0) {
+    lm::k_bin_sizes<<<grid_for(g->n, 256, 4096), 256, 0, st>>>(g->offs, g->n, cnt);
+    CKL();
+  }
+  unsigned long long h[lm::kBins];
+  CK(cudaMemcpyAsync(h, cnt, sizeof h, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  cudaFree(cnt);
+  for (int i = 0; i < 2; ++i)
+    for (int b = 0; b < lm::kBins; ++b) TRY(dmalloc(g, &g->F[i].list[b], (size_t)h[b] + 1));
+  return LMATCH_OK;
+}
+
 int finish_create(lmatch_graph* g, cudaStream_t st) {
+  TRY(alloc_bins(g, st));
   if (g->m > 0) {
     CK(cudaMemsetAsync(g->werr, 0, 8, st));
     lm::k_zap_self_loops<<<grid_for(g->n * 8, 256, 16384), 256, 0, st>>>(
@@ -590,9 +607,10 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
       const unsigned long long* cF = C + lm::cnt_F(cur, 0);
       // A2 frontier pointer phase, one launch per non-empty degree bin
       lm::Bins& Fb = g->F[cur];
-      if (nFb[0]) { lm::k_point_bin<4, 2><<<grid_for(nFb[0] * 4, 256, 65536), 256, 0, st>>>(Fb.list[0], cF + 0, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }
-      if (nFb[1]) { lm::k_point_bin<16, 4><<<grid_for(nFb[1] * 16, 256, 65536), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }
-      if (nFb[2]) { lm::k_point_bin<32, 4><<<grid_for(nFb[2] * 32, 256, 65536), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }
+      const int kMaxGrid = 65536;
+      if (nFb[0]) { lm::k_point_bin<1, 8><<<grid_for(nFb[0], 256, kMaxGrid), 256, 0, st>>>(Fb.list[0], cF + 0, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }    // deg <= 8: a thread each
+      if (nFb[1]) { lm::k_point_bin<8, 8><<<grid_for(nFb[1] * 8, 256, kMaxGrid), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }     // 9..64
+      if (nFb[2]) { lm::k_point_bin<32, 4><<<grid_for(nFb[2] * 32, 256, kMaxGrid), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }   // 65..2048
       if (nFb[3]) { lm::k_point_bin_cta<256, 4><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }
       // A4 match over the new pointers
       lm::k_match_bins<<<grid_for(nF, 256, 65536), 256, 0, st>>>(Fb, cF, g->best, g->bits);
