@@ -187,9 +187,12 @@ def cpu_baseline(a, sample_scale):
             "seconds": t}
 
 
-def cpu_sample_scale(a):
+def cpu_sample_scale(a, baseline: bool = True):
+    """cpu_baseline: ~10 s of single-core oracle work; reference-arm steps: ~2 s each."""
     if a.cpu_scale:
         return a.cpu_scale
+    if baseline:
+        return {"rmat": 22, "er": 22, "mesh": 22, "road": 22, "gradient": 18}[a.workload]
     return {"rmat": 20, "er": 20, "mesh": 20, "road": 20, "gradient": 18}[a.workload]
 
 
@@ -198,7 +201,7 @@ def run_reference(a, rank, world):
     if rank != 0:
         return 0
     import oracle
-    scale = cpu_sample_scale(a)
+    scale = cpu_sample_scale(a, baseline=False)
     g = make_graph_cpu(a, scale, a.seed)
     oracle.threads(1)
     for _ in range(a.warmup):
