@@ -42,7 +42,7 @@
 extern "C" {
 #endif
 
-#define LMATCH_ABI_VERSION 1
+#define LMATCH_ABI_VERSION 2
 
 #if defined(__GNUC__)
 #define LMATCH_API __attribute__((visibility("default")))
@@ -77,7 +77,14 @@ typedef struct lmatch_opts {
   int32_t timing;          /* 1 = record CUDA events per phase into lmatch_stats */
   int64_t max_rounds;      /* 0 = default: n/2 + 2 (the strict order bounds rounds by n/2+1) */
   int64_t upload_chunk;    /* entries per host->device upload chunk (0 = default 2^25) */
-  int32_t reserved[16];
+  int64_t hbm_budget_bytes;   /* 0 = adjacency fully resident.  Otherwise, if 8*m exceeds it, only a
+                                 prefix of the packed adjacency stays in HBM; the rest lives in
+                                 library-owned pinned host memory, is streamed through a device
+                                 ring in round 1 (LOADBATCH, Alg. 2 L10-12; double
+                                 buffering) and read zero-copy by later rounds */
+  int64_t stream_chunk;       /* entries per streamed chunk (0 = default 2^24; rounded to the
+                                 sweep tile) */
+  int32_t reserved[12];
 } lmatch_opts;
 
 /* Filled by lmatch_run / lmatch_run_device when non-NULL. */
@@ -95,7 +102,9 @@ typedef struct lmatch_stats {
   double ms_finish;          /* (timing=1) mate materialisation + weight reduction */
   int64_t sweep_launches;    /* kernel launches of the round-1 sweep (1) */
   int64_t kernel_launches;   /* all kernel launches issued by this run */
-  int64_t reserved[8];
+  int64_t bytes_streamed;    /* host->device adjacency bytes copied by this run (out-of-core) */
+  int64_t resident_entries;  /* adjacency entries resident in HBM (= m unless out-of-core) */
+  int64_t reserved[6];
 } lmatch_stats;
 
 /* Library / ABI identification.  Returns LMATCH_ABI_VERSION. */

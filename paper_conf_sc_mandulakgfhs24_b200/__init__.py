@@ -42,7 +42,8 @@ class Opts(ctypes.Structure):
         ("device", ctypes.c_int32), ("use_device", ctypes.c_int32),
         ("validate_level", ctypes.c_int32), ("timing", ctypes.c_int32),
         ("max_rounds", ctypes.c_int64), ("upload_chunk", ctypes.c_int64),
-        ("reserved", ctypes.c_int32 * 16),
+        ("hbm_budget_bytes", ctypes.c_int64), ("stream_chunk", ctypes.c_int64),
+        ("reserved", ctypes.c_int32 * 12),
     ]
 
 
@@ -55,7 +56,8 @@ class Stats(ctypes.Structure):
         ("ms_total", ctypes.c_double), ("ms_sweep", ctypes.c_double),
         ("ms_rounds", ctypes.c_double), ("ms_round1_rest", ctypes.c_double),
         ("ms_finish", ctypes.c_double), ("sweep_launches", ctypes.c_int64),
-        ("kernel_launches", ctypes.c_int64), ("reserved", ctypes.c_int64 * 8),
+        ("kernel_launches", ctypes.c_int64), ("bytes_streamed", ctypes.c_int64),
+        ("resident_entries", ctypes.c_int64), ("reserved", ctypes.c_int64 * 6),
     ]
 
     def as_dict(self) -> dict:
@@ -236,7 +238,7 @@ class Matcher:
 
     def __init__(self, offsets=None, col=None, w=None, *, handle: int | None = None,
                  validate_level: int = 1, timing: bool = False, upload_chunk: int = 0,
-                 max_rounds: int = 0):
+                 max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0):
         self.h = None
         if handle is not None:
             self.h = handle
@@ -245,7 +247,7 @@ class Matcher:
                 offsets, col, w = offsets.offsets, offsets.col, offsets.w
             self.h = lmatch_create_ex(offsets, col, w,
                                       opts=make_opts(validate_level, timing, upload_chunk,
-                                                     max_rounds))
+                                                     max_rounds, hbm_budget_bytes, stream_chunk))
         self.info = lmatch_info(self.h)
 
     @classmethod
@@ -287,8 +289,10 @@ class Matcher:
 
 
 def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int = 0,
-              max_rounds: int = 0) -> Opts:
+              max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0) -> Opts:
     o = Opts()
+    o.hbm_budget_bytes = int(hbm_budget_bytes)
+    o.stream_chunk = int(stream_chunk)
     o.validate_level = int(validate_level)
     o.timing = int(bool(timing))
     o.upload_chunk = int(upload_chunk)

@@ -26,6 +26,20 @@ namespace lm {
 constexpr int kBins = 4;               // frontier degree bins
 constexpr int kBinDeg0 = 8, kBinDeg1 = 64, kBinDeg2 = 2048;  // bins: G = 1, 8, 32 lanes, CTA
 
+// Adjacency view: entries [0, R) in HBM, [R, m) in pinned host memory mapped into the device
+// address space (out-of-core mode; R = m otherwise).  host_off is pre-offset by -R.
+struct AdjView {
+  const uint64_t* dev;
+  const uint64_t* host_off;
+  int64_t R;
+  __device__ __forceinline__ uint64_t at(int64_t j) const {
+    return j < R ? __ldg(dev + j) : host_off[j];
+  }
+  __device__ __forceinline__ uint64_t* ptr(int64_t j) const {
+    return const_cast<uint64_t*>(j < R ? dev + j : host_off + j);
+  }
+};
+
 // --------------------------------------------------------------------------- small helpers
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return (uint32_t)__cvta_generic_to_shared(p);
@@ -137,7 +151,7 @@ __global__ void k_pack(const int32_t* __restrict__ col, const float* __restrict_
 
 // Self-loops are ignored (simple graph): their keys become 0, which never wins a max, so
 // no kernel on the hot path needs a per-entry self test.  8 lanes per row.
-__global__ void k_zap_self_loops(const int64_t* __restrict__ offs, uint64_t* adj, int64_t n,
+__global__ void k_zap_self_loops(const int64_t* __restrict__ offs, AdjView adj, int64_t n,
                                  unsigned long long* count) {
   const int lane8 = threadIdx.x & 7;
   const int64_t g0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 3;
@@ -145,7 +159,7 @@ __global__ void k_zap_self_loops(const int64_t* __restrict__ offs, uint64_t* adj
   unsigned long long c = 0;
   for (int64_t u = g0; u < n; u += gs)
     for (int64_t j = offs[u] + lane8; j < offs[u + 1]; j += 8)
-      if ((uint32_t)adj[j] == (uint32_t)u) { adj[j] = 0ull; ++c; }
+      if ((uint32_t)adj.at(j) == (uint32_t)u && adj.at(j) != 0ull) { *adj.ptr(j) = 0ull; ++c; }
   for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
   if ((threadIdx.x & 31) == 0 && c) atomicAdd(count, c);
 }
@@ -184,15 +198,15 @@ __device__ __forceinline__ uint64_t mix64(uint64_t x) {
   x = (x ^ (x >> 27)) * 0x94D049BB133111EBull;
   return x ^ (x >> 31);
 }
-__global__ void k_symhash(const int64_t* __restrict__ offs, const uint64_t* __restrict__ adj,
-                          int64_t n, unsigned long long* acc) {
+__global__ void k_symhash(const int64_t* __restrict__ offs, AdjView adj, int64_t n,
+                          unsigned long long* acc) {
   const int lane8 = threadIdx.x & 7;
   const int64_t g0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 3;
   const int64_t gs = ((int64_t)gridDim.x * blockDim.x) >> 3;
   uint64_t s = 0;
   for (int64_t u = g0; u < n; u += gs) {
     for (int64_t j = offs[u] + lane8; j < offs[u + 1]; j += 8) {
-      const uint64_t k = adj[j];
+      const uint64_t k = adj.at(j);
       if (k == 0) continue;  // zeroed self-loop
       const uint64_t v = (uint32_t)k, wb = k >> 32;
       s += mix64(mix64((uint64_t)u * 0x100000001B3ull ^ v) ^ wb) -
@@ -345,12 +359,13 @@ __device__ __forceinline__ uint64_t umax_skip(uint64_t b, uint64_t key, uint32_t
 }
 
 struct SweepArgs {
-  const uint64_t* adj;
+  const uint64_t* adj;       // keys of entry tile_begin*TILE onward (HBM or a streamed chunk)
   const uint32_t* noffs_lo;  // low 32 bits of each non-empty row's start (+ m)
   const int32_t* nzr;
   const int32_t* tile_nz;
   uint64_t* best;
   int64_t m;
+  int64_t tile_begin;        // tiles [tile_begin, ntiles) of this launch
   int64_t ntiles;
 };
 
@@ -387,7 +402,7 @@ __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
   };
   (void)ids_of;
 
-  const int64_t gw = (int64_t)blockIdx.x * WARPS + warp;
+  const int64_t gw = A.tile_begin + (int64_t)blockIdx.x * WARPS + warp;
   const int64_t nwt = (int64_t)gridDim.x * WARPS;
   if (lane == 0) {
     for (int s = 0; s < RING; ++s) mbar_init(&bars[s], 1);
@@ -406,7 +421,7 @@ __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
     const uint32_t wbytes = (uint32_t)(((wcnt + 3) & ~3ll) * 4);
     fence_proxy_async_smem();
     mbar_arrive_expect_tx(&bars[s], kbytes + 2 * wbytes);
-    tma_bulk_g2s(keys_of(s), A.adj + e0, kbytes, &bars[s], pol);
+    tma_bulk_g2s(keys_of(s), A.adj + (t - A.tile_begin) * TILE, kbytes, &bars[s], pol);
     tma_bulk_g2s(win_of(s), A.noffs_lo + a4, wbytes, &bars[s], pol);
     tma_bulk_g2s(ids_of(s), A.nzr + a4, wbytes, &bars[s], pol);
   };
@@ -797,7 +812,7 @@ struct Bins {
 // running max at batch start) are fetched together, so no L2 round trip sits on the loop-carried
 // max.  Zeroed self-loop keys never qualify.  The new pointer goes to best[u] and into the slot.
 template <int G, int U>
-__device__ __forceinline__ uint64_t scan_row_available(const uint64_t* __restrict__ adj,
+__device__ __forceinline__ uint64_t scan_row_available(const AdjView adj,
                                                        const uint32_t* __restrict__ bits,
                                                        int64_t s, int64_t e, int gl) {
   uint64_t b = 0;
@@ -806,7 +821,7 @@ __device__ __forceinline__ uint64_t scan_row_available(const uint64_t* __restric
 #pragma unroll
     for (int q = 0; q < U; ++q) {
       const int64_t j = j0 + (int64_t)q * G;
-      k[q] = j < e ? __ldg(adj + j) : 0ull;
+      k[q] = j < e ? adj.at(j) : 0ull;
     }
     uint32_t wd[U];
 #pragma unroll
@@ -822,7 +837,7 @@ __device__ __forceinline__ uint64_t scan_row_available(const uint64_t* __restric
 
 template <int G, int U>
 __global__ void k_point_bin(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
-                            const int64_t* __restrict__ offs, const uint64_t* __restrict__ adj,
+                            const int64_t* __restrict__ offs, const AdjView adj,
                             const uint32_t* __restrict__ bits, uint64_t* __restrict__ best) {
   const int64_t cnt = (int64_t)*cnt_ptr;
   const int lane = threadIdx.x & 31;
@@ -845,7 +860,7 @@ __global__ void k_point_bin(ulonglong2* __restrict__ list, const unsigned long l
 template <int THREADS, int U>
 __global__ void __launch_bounds__(THREADS)
     k_point_bin_cta(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
-                    const int64_t* __restrict__ offs, const uint64_t* __restrict__ adj,
+                    const int64_t* __restrict__ offs, const AdjView adj,
                     const uint32_t* __restrict__ bits, uint64_t* __restrict__ best) {
   __shared__ uint64_t red[THREADS / 32];
   const int64_t cnt = (int64_t)*cnt_ptr;
@@ -1100,7 +1115,7 @@ __global__ void __launch_bounds__(THREADS)
 template <int THREADS>
 __global__ void __launch_bounds__(THREADS)
     k_weight_any(const int32_t* __restrict__ mate, int64_t n, const int64_t* __restrict__ offs,
-                 const uint64_t* __restrict__ adj, double* pw, long long* pc, unsigned* err) {
+                 const AdjView adj, double* pw, long long* pc, unsigned* err) {
   const int lane = threadIdx.x & 31, g8 = lane & 7;
   const unsigned gmask = 0xffu << (lane & ~7);
   double w = 0.0;
@@ -1120,8 +1135,8 @@ __global__ void __launch_bounds__(THREADS)
     if ((int64_t)v < u) continue;
     uint64_t found = 0;
     for (int64_t j = offs[u] + g8; j < offs[u + 1]; j += 8) {
-      const uint64_t k = adj[j];
-      if ((uint32_t)k == (uint32_t)v) found = k;
+      const uint64_t k = adj.at(j);
+      if (k != 0 && (uint32_t)k == (uint32_t)v) found = k;
     }
     found = group_max_key(found, gmask);
     if (g8 == 0) {

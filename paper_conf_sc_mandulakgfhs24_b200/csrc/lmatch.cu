@@ -96,6 +96,16 @@ struct lmatch_graph {
   int timing = 0;
   int64_t max_rounds = 0;
   int64_t upload_chunk = 1ll << 25;
+  // out-of-core: entries [0, R) resident; [R, m) in pinned mapped host memory, streamed in round 1
+  int64_t R = 0;
+  int64_t stream_chunk = 1ll << 24;
+  int64_t hbm_budget = 0;
+  bool streaming = false;
+  uint64_t* host_adj = nullptr;      // pinned, mapped: entries [R, m)
+  uint64_t* host_adj_dev = nullptr;  // its device alias
+  uint64_t* ring[2] = {nullptr, nullptr};
+  cudaStream_t cs = nullptr;         // copy stream for streaming
+  cudaEvent_t ev_full[2] = {}, ev_free[2] = {};
   int sweep_grid = 0;
   alignas(64) CUtensorMap tmap;  // adjacency as a [ceil(m/16)][16] u64 tensor, 128B swizzle
   int num_sms = 148;
@@ -130,6 +140,8 @@ struct lmatch_graph {
   cudaEvent_t ev[8] = {};
   int64_t device_bytes = 0;
   std::vector<int64_t> round_log;  // per round: |F_r|, |L_r|, E(F_r) (directed entries scanned)
+
+  lm::AdjView view() const { return lm::AdjView{adj, host_adj_dev - R, R}; }
 };
 
 namespace {
@@ -165,9 +177,31 @@ int check_args(const void* a, const void* b, const void* c, int64_t n, int64_t m
 int alloc_all(lmatch_graph* g) {
   const int64_t n = g->n, m = g->m;
   TRY(dmalloc(g, &g->offs, (size_t)n + 1));
-  TRY(dmalloc(g, &g->adj, (size_t)m + 32));
-  // zero the padding past m: the sweep's 2-D tensor view reads whole 16-key rows
-  CK(cudaMemsetAsync(g->adj + m, 0, 32 * sizeof(uint64_t), g->stream));
+  // out-of-core split: keep a prefix of R entries (multiple of the stream chunk) in HBM
+  g->R = m;
+  if (g->hbm_budget > 0 && 8 * m > g->hbm_budget) {
+    const int64_t C = std::max<int64_t>(kTile, (g->stream_chunk / kTile) * kTile);
+    g->stream_chunk = C;
+    g->R = std::max<int64_t>(0, (g->hbm_budget / 8 - 2 * C) / C * C);
+    g->R = std::min(g->R, (m / C) * C);
+    g->streaming = g->R < m;
+  }
+  TRY(dmalloc(g, &g->adj, (size_t)g->R + 32));
+  // zero the padding past the resident part (tile reads round up to 16 bytes)
+  CK(cudaMemsetAsync(g->adj + g->R, 0, 32 * sizeof(uint64_t), g->stream));
+  if (g->streaming) {
+    const size_t hb = ((size_t)(m - g->R) + 32) * 8;
+    CK(cudaHostAlloc(reinterpret_cast<void**>(&g->host_adj), hb, cudaHostAllocMapped));
+    std::memset(g->host_adj + (m - g->R), 0, 32 * 8);
+    CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&g->host_adj_dev), g->host_adj, 0));
+    for (int i = 0; i < 2; ++i) {
+      TRY(dmalloc(g, &g->ring[i], (size_t)g->stream_chunk + 32));
+      CK(cudaMemsetAsync(g->ring[i], 0, ((size_t)g->stream_chunk + 32) * 8, g->stream));
+      CK(cudaEventCreateWithFlags(&g->ev_full[i], cudaEventDisableTiming));
+      CK(cudaEventCreateWithFlags(&g->ev_free[i], cudaEventDisableTiming));
+    }
+    CK(cudaStreamCreateWithFlags(&g->cs, cudaStreamNonBlocking));
+  }
   TRY(dmalloc(g, &g->noffs, (size_t)n + 5));
   TRY(dmalloc(g, &g->nzr, (size_t)n + 8));
   g->ntiles = (m + kTile - 1) / kTile;
@@ -273,7 +307,7 @@ int check_pack(lmatch_graph* g, cudaStream_t st) {
     unsigned long long* acc = nullptr;
     TRY(dmalloc(g, &acc, 1));
     CK(cudaMemsetAsync(acc, 0, 8, st));
-    lm::k_symhash<<<grid_for(g->n * 8, 256, 8192), 256, 0, st>>>(g->offs, g->adj, g->n, acc);
+    lm::k_symhash<<<grid_for(g->n * 8, 256, 8192), 256, 0, st>>>(g->offs, g->view(), g->n, acc);
     CKL();
     unsigned long long hv = 0;
     CK(cudaMemcpyAsync(&hv, acc, 8, cudaMemcpyDeviceToHost, st));
@@ -310,9 +344,19 @@ int upload_host(lmatch_graph* g, const int64_t* offsets, const int32_t* col, con
     cudaStream_t s = g->up[i];
     CK(cudaMemcpyAsync(g->st_col[i], col + base, (size_t)cnt * 4, cudaMemcpyHostToDevice, s));
     CK(cudaMemcpyAsync(g->st_w[i], w + base, (size_t)cnt * 4, cudaMemcpyHostToDevice, s));
-    lm::k_pack<<<grid_for(cnt, 256, 16384), 256, 0, s>>>(g->st_col[i], g->st_w[i], cnt, n,
+    // entries below R go to HBM, the rest to the pinned host copy (written through its alias)
+    const int64_t nd = std::max<int64_t>(0, std::min(cnt, g->R - base));
+    if (nd > 0) {
+      lm::k_pack<<<grid_for(nd, 256, 16384), 256, 0, s>>>(g->st_col[i], g->st_w[i], nd, n,
                                                           g->adj + base, base, g->perr);
-    CKL();
+      CKL();
+    }
+    if (cnt > nd) {
+      lm::k_pack<<<grid_for(cnt - nd, 256, 16384), 256, 0, s>>>(
+          g->st_col[i] + nd, g->st_w[i] + nd, cnt - nd, n, g->host_adj_dev + (base + nd - g->R),
+          base + nd, g->perr);
+      CKL();
+    }
   }
   CK(cudaStreamSynchronize(g->up[0]));
   CK(cudaStreamSynchronize(g->up[1]));
@@ -327,8 +371,16 @@ int upload_device(lmatch_graph* g, const int64_t* d_offsets, const int32_t* d_co
   CK(cudaMemcpyAsync(g->offs, d_offsets, ((size_t)n + 1) * 8, cudaMemcpyDeviceToDevice, st));
   if (g->validate_level >= 0) TRY(check_offsets(g, st));
   if (m > 0) {
-    lm::k_pack<<<grid_for(m, 256, 65536), 256, 0, st>>>(d_col, d_w, m, n, g->adj, 0, g->perr);
-    CKL();
+    const int64_t nd = std::min(m, g->R);
+    if (nd > 0) {
+      lm::k_pack<<<grid_for(nd, 256, 65536), 256, 0, st>>>(d_col, d_w, nd, n, g->adj, 0, g->perr);
+      CKL();
+    }
+    if (m > nd) {
+      lm::k_pack<<<grid_for(m - nd, 256, 65536), 256, 0, st>>>(d_col + nd, d_w + nd, m - nd, n,
+                                                               g->host_adj_dev, nd, g->perr);
+      CKL();
+    }
   }
   TRY(check_pack(g, st));
   return LMATCH_OK;
@@ -384,11 +436,12 @@ int finish_create(lmatch_graph* g, cudaStream_t st) {
   if (g->m > 0) {
     CK(cudaMemsetAsync(g->werr, 0, 8, st));
     lm::k_zap_self_loops<<<grid_for(g->n * 8, 256, 16384), 256, 0, st>>>(
-        g->offs, g->adj, g->n, reinterpret_cast<unsigned long long*>(g->werr));
+        g->offs, g->view(), g->n, reinterpret_cast<unsigned long long*>(g->werr));
     CKL();
   }
   TRY(build_index(g, st));
 #if LM_SWEEP_IMPL == 2
+  if (g->streaming) { set_err("LM_SWEEP_IMPL=2 does not support out-of-core graphs"); return LMATCH_EINVAL; }
   if (g->ntiles > 0) TRY(make_tensor_map(g));
 #endif
   if (g->ntiles > 0) {
@@ -418,6 +471,8 @@ int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** 
     g->timing = opts->timing;
     g->max_rounds = opts->max_rounds;
     if (opts->upload_chunk > 0) g->upload_chunk = (opts->upload_chunk + 3) & ~3ll;
+    g->hbm_budget = opts->hbm_budget_bytes;
+    if (opts->stream_chunk > 0) g->stream_chunk = opts->stream_chunk;
   }
   CK(cudaGetDevice(&g->device));
   CK(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, g->device));
@@ -465,6 +520,13 @@ void lmatch_destroy(lmatch_graph* g) {
   for (auto& F : g->F)
     for (auto p : F.list) if (p) cudaFree(p);
   if (g->h_counters) cudaFreeHost(g->h_counters);
+  if (g->host_adj) cudaFreeHost(g->host_adj);
+  for (int i = 0; i < 2; ++i) {
+    if (g->ring[i]) cudaFree(g->ring[i]);
+    if (g->ev_full[i]) cudaEventDestroy(g->ev_full[i]);
+    if (g->ev_free[i]) cudaEventDestroy(g->ev_free[i]);
+  }
+  if (g->cs) cudaStreamDestroy(g->cs);
   if (g->h_res) cudaFreeHost(g->h_res);
   if (g->h_resc) cudaFreeHost(g->h_resc);
   for (auto e : g->ev) if (e) cudaEventDestroy(e);
@@ -556,7 +618,7 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
   cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
   const int64_t n = g->n;
   const bool tm = g->timing && stats;
-  int64_t launches = 0, rounds = 0, ftot_all = 0;
+  int64_t launches = 0, rounds = 0, ftot_all = 0, sweep_launches = 0, bytes_streamed = 0;
   unsigned long long* C = g->counters;
   unsigned long long* hc = g->h_counters;
   g->round_log.clear();
@@ -575,8 +637,34 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
     lm::Sweep2DArgs A{g->noffs_lo, g->nzr, g->tile_nz, g->best, g->m, g->ntiles};
     SWEEP_KERNEL<<<g->sweep_grid, kSweepThreads, Sweep::kSmem, st>>>(g->tmap, A);
 #else
-    lm::SweepArgs A{g->adj, g->noffs_lo, g->nzr, g->tile_nz, g->best, g->m, g->ntiles};
-    SWEEP_KERNEL<<<g->sweep_grid, kSweepThreads, Sweep::kSmem, st>>>(A);
+    // resident tiles [0, R/TILE), then the streamed chunks through a 2-slot device ring:
+    // the copy of chunk k+1 (copy stream) overlaps the sweep of chunk k (run stream).
+    const int64_t rt = g->streaming ? g->R / kTile : g->ntiles;
+    auto sweep_launch = [&](const uint64_t* base, int64_t t0, int64_t t1) -> int {
+      const int64_t grid = std::min<int64_t>((t1 - t0 + kSweepWarps - 1) / kSweepWarps, g->sweep_grid);
+      lm::SweepArgs A{base, g->noffs_lo, g->nzr, g->tile_nz, g->best, g->m, t0, t1};
+      SWEEP_KERNEL<<<(unsigned)std::max<int64_t>(grid, 1), kSweepThreads, Sweep::kSmem, st>>>(A);
+      CKL();
+      ++launches;
+      ++sweep_launches;
+      return LMATCH_OK;
+    };
+    if (rt > 0) TRY(sweep_launch(g->adj, 0, std::min(rt, g->ntiles)));
+    if (g->streaming) {
+      const int64_t C = g->stream_chunk;
+      for (int64_t e0 = g->R, k = 0; e0 < g->m; e0 += C, ++k) {
+        const int slot = (int)(k & 1);
+        const int64_t cnt = std::min(C, g->m - e0);
+        if (k >= 2) CK(cudaStreamWaitEvent(g->cs, g->ev_free[slot], 0));
+        CK(cudaMemcpyAsync(g->ring[slot], g->host_adj + (e0 - g->R), (size_t)cnt * 8,
+                           cudaMemcpyHostToDevice, g->cs));
+        CK(cudaEventRecord(g->ev_full[slot], g->cs));
+        bytes_streamed += cnt * 8;
+        CK(cudaStreamWaitEvent(st, g->ev_full[slot], 0));
+        TRY(sweep_launch(g->ring[slot], e0 / kTile, std::min(g->ntiles, (e0 + cnt + kTile - 1) / kTile)));
+        CK(cudaEventRecord(g->ev_free[slot], st));
+      }
+    }
 #endif
     CKL();
     if (tm) CK(cudaEventRecord(g->ev[2], st));
@@ -587,7 +675,7 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
         nullptr, nullptr, lm::Bins{}, nullptr, n, g->best, g->bits, g->offs, g->S[0],
         C + lm::cnt_S(0), g->F[0], C + lm::cnt_F(0, 0), C + lm::kCntSwept);
     CKL();
-    launches += 3;
+    launches += 2;
     CK(cudaMemcpyAsync(hc, C, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));
     if (tm) CK(cudaEventRecord(g->ev[3], st));
@@ -608,10 +696,10 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
       // A2 frontier pointer phase, one launch per non-empty degree bin
       lm::Bins& Fb = g->F[cur];
       const int kMaxGrid = 65536;
-      if (nFb[0]) { lm::k_point_bin<1, 8><<<grid_for(nFb[0], 256, kMaxGrid), 256, 0, st>>>(Fb.list[0], cF + 0, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }    // deg <= 8: a thread each
-      if (nFb[1]) { lm::k_point_bin<8, 8><<<grid_for(nFb[1] * 8, 256, kMaxGrid), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }     // 9..64
-      if (nFb[2]) { lm::k_point_bin<32, 4><<<grid_for(nFb[2] * 32, 256, kMaxGrid), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }   // 65..2048
-      if (nFb[3]) { lm::k_point_bin_cta<256, 4><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, g->adj, g->bits, g->best); CKL(); ++launches; }
+      if (nFb[0]) { lm::k_point_bin<1, 8><<<grid_for(nFb[0], 256, kMaxGrid), 256, 0, st>>>(Fb.list[0], cF + 0, g->offs, g->view(), g->bits, g->best); CKL(); ++launches; }    // deg <= 8: a thread each
+      if (nFb[1]) { lm::k_point_bin<8, 8><<<grid_for(nFb[1] * 8, 256, kMaxGrid), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, g->view(), g->bits, g->best); CKL(); ++launches; }     // 9..64
+      if (nFb[2]) { lm::k_point_bin<32, 4><<<grid_for(nFb[2] * 32, 256, kMaxGrid), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, g->view(), g->bits, g->best); CKL(); ++launches; }   // 65..2048
+      if (nFb[3]) { lm::k_point_bin_cta<256, 4><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, g->view(), g->bits, g->best); CKL(); ++launches; }
       // A4 match over the new pointers
       lm::k_match_bins<<<grid_for(nF, 256, 65536), 256, 0, st>>>(Fb, cF, g->best, g->bits);
       CKL();
@@ -658,7 +746,9 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
     stats->entries_swept = 0;
     for (size_t i = 2; i < g->round_log.size(); i += 3) stats->entries_swept += g->round_log[i];
     stats->frontier_total = ftot_all;
-    stats->sweep_launches = (g->ntiles > 0 && n > 0) ? 1 : 0;
+    stats->sweep_launches = sweep_launches;
+    stats->bytes_streamed = bytes_streamed;
+    stats->resident_entries = g->R;
     stats->kernel_launches = launches;
     if (tm) {
       float a = 0, b = 0, c = 0, d = 0, e = 0;
@@ -698,7 +788,7 @@ int lmatch_weight_device(lmatch_graph* g, const int32_t* d_mate, void* stream, d
   cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
   if (g->n == 0) { *out_weight = 0.0; return LMATCH_OK; }
   CK(cudaMemsetAsync(g->werr, 0, 4, st));
-  lm::k_weight_any<kFinThreads><<<kFinBlocks, kFinThreads, 0, st>>>(d_mate, g->n, g->offs, g->adj,
+  lm::k_weight_any<kFinThreads><<<kFinBlocks, kFinThreads, 0, st>>>(d_mate, g->n, g->offs, g->view(),
                                                                     g->pw, g->pc, g->werr);
   CKL();
   lm::k_final_sum<<<1, 32, 0, st>>>(g->pw, g->pc, kFinBlocks, g->res_w, g->res_c);
