@@ -51,6 +51,8 @@ def parse():
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--cpu-scale", type=int, default=None)
     p.add_argument("--gen", default="gpu", choices=["cpu", "gpu"])
+    p.add_argument("--partitioned", action="store_true",
+                   help="use the 1-D partitioned path even at N=1 (it is always used for N>1)")
     return p.parse_args()
 
 
@@ -226,6 +228,126 @@ def run_reference(a, rank, world):
     return 0
 
 
+# ------------------------------------------------------------------- partitioned arm (N >= 1)
+def run_partitioned(a, rank, world, local):
+    """One graph, 1-D vertex partition over the N ranks: each rank owns an
+    edge-balanced row range; pointer claims go to the owner of the target (all-to-all) and the
+    matched bitmap is allgathered each round, over NCCL (torch.distributed).  Strong scaling:
+    the graph is the same for every N."""
+    import torch
+    import torch.distributed as dist
+    import paper_conf_sc_mandulakgfhs24_b200 as lm  # noqa: F401  (loads liblmatch.so)
+    import paper_conf_sc_mandulakgfhs24_b200.dist as D
+
+    scale = a.scale or DEFAULT_SCALE[a.workload]
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream(dev)
+    t0 = time.time()
+    dg = make_graph_gpu(a, scale, a.seed, dev)  # same seed on every rank: one graph
+    n, m, m_u = dg.n, dg.m, dg.m_u
+    offs_h = dg.offsets.cpu().numpy()
+    bounds = D.edge_balanced_bounds(offs_h, world)
+    v0, v1 = int(bounds[rank]), int(bounds[rank + 1])
+    s0, s1 = int(offs_h[v0]), int(offs_h[v1])
+    lo = (dg.offsets[v0:v1 + 1] - s0).contiguous()
+    lc = dg.col[s0:s1].contiguous()
+    lw = dg.w[s0:s1].contiguous()
+    host = None
+    if not a.no_e2e:
+        host = (lo.cpu().numpy(), lc.cpu().numpy(), lw.cpu().numpy())
+    dg = None
+    torch.cuda.empty_cache()
+    gen_s = time.time() - t0
+    part = D.LibPart(lo, lc, lw, v0, n, bounds, rank, device=dev, stream=stream, timing=True)
+    del lo, lc, lw
+    torch.cuda.empty_cache()
+    tr = D.TorchTransport()
+
+    for _ in range(a.warmup):
+        D.run_parts([part], tr)
+    torch.cuda.synchronize(dev)
+    dist.barrier()
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    sweep_ms = []
+    with ClockSampler(local) as clk:
+        torch.cuda.synchronize(dev)
+        ev0.record(stream)
+        for _ in range(a.steps):
+            res = D.run_parts([part], tr)
+            sweep_ms.append(part.info()[1])
+        ev1.record(stream)
+        torch.cuda.synchronize(dev)
+    ms = ev0.elapsed_time(ev1)
+    t = torch.tensor([ms], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms = float(t.item())
+    ms_per_step = ms / a.steps
+    value = m_u * a.steps / (ms / 1e3) / 1e9
+
+    e2e = None
+    if host is not None and a.e2e_steps > 0:
+        cud = torch.cuda.cudart()
+        for arr in host:
+            if arr.nbytes:
+                cud.cudaHostRegister(arr.ctypes.data, arr.nbytes, 0)
+        mate_h = torch.empty(max(v1 - v0, 1), dtype=torch.int32, pin_memory=True)
+        dist.barrier()
+        t1 = time.perf_counter()
+        for _ in range(a.e2e_steps):
+            part.reload(*host)
+            r = D.run_parts([part], tr)
+            mate_h[: v1 - v0].copy_(r.mates[0])
+        el = time.perf_counter() - t1
+        te = torch.tensor([el], dtype=torch.float64, device=dev)
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+        el = float(te.item())
+        for arr in host:
+            if arr.nbytes:
+                cud.cudaHostUnregister(arr.ctypes.data)
+        hb = torch.tensor([sum(x.nbytes for x in host)], dtype=torch.float64, device=dev)
+        dist.all_reduce(hb)
+        e2e = {"value": m_u * a.e2e_steps / el / 1e9, "unit": UNIT,
+               "h2d_bytes_per_step": int(hb.item()), "d2h_bytes_per_step": int(4 * n),
+               "steps": a.e2e_steps, "ms_per_step": el / a.e2e_steps * 1e3,
+               "includes": "lmatch_reload of every rank's local CSR (H2D + pack + validate + index) "
+                           "+ partitioned run + owned mate[] slices D2H"}
+
+    # roofline of the dominant kernel: the slowest rank's round-1 sweep over its owned rows
+    m_loc = part.m_local
+    sweep_avg = float(np.mean(sweep_ms))
+    sw = torch.tensor([sweep_avg, float(m_loc)], dtype=torch.float64, device=dev)
+    allsw = [torch.empty_like(sw) for _ in range(world)]
+    dist.all_gather(allsw, sw)
+    worst = max(allsw, key=lambda x: float(x[0]))
+    peak, peak_src = load_peaks()
+    n_loc_nz = int(np.count_nonzero(np.diff(offs_h[v0:v1 + 1]))) if rank == 0 else 0
+    sweep_bytes = 8 * float(worst[1]) + 16 * n_loc_nz
+    achieved = sweep_bytes / (float(worst[0]) / 1e3) / 1e9 if float(worst[0]) > 0 else None
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": (achieved / peak) if achieved else None, "traffic": None,
+                "kernel": "k_sweep over the slowest rank's owned rows",
+                "launch_ms": float(worst[0]), "share_of_step": float(worst[0]) / ms_per_step,
+                "peak_source": peak_src}
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps,
+                "warmup": a.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+                "scaling": "strong", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+                "config": workload_config(a, scale, n, m) | {
+                    "parallelism": f"1-D vertex partition over {world} GPU(s): claims all-to-all + "
+                                   "bitmap allgather per round (NCCL)",
+                    "l2": f"inputs larger than L2 (adjacency {8 * m / 1e9:.1f} GB total); no flush",
+                    "gen_s": round(gen_s, 1), "part_bounds": [int(x) for x in bounds]},
+                "roofline": roofline, "cpu_baseline": None, "e2e": e2e,
+                "gpu_launches": None, "clocks": clk.summary(), "rounds": res.rounds,
+                "cardinality": res.matched // 2, "matched_weight": res.weight,
+                "claims_per_step_rank0": res.exchanged_claims}
+        print(json.dumps(line), flush=True)
+    part.close()
+    dist.destroy_process_group()
+    return 0
+
+
 # -------------------------------------------------------------------------------- our arm
 def main():
     a = parse()
@@ -240,8 +362,11 @@ def main():
     if not torch.cuda.is_available():
         raise SystemExit("bench.py needs a CUDA device (no CPU fallback)")
     torch.cuda.set_device(local)
-    if world > 1:
+    if world > 1 or a.partitioned:
+        if "MASTER_ADDR" not in os.environ:  # single-process partitioned run
+            os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT="29531", RANK="0", WORLD_SIZE="1")
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        return run_partitioned(a, rank, world, local)
     import paper_conf_sc_mandulakgfhs24_b200 as lm
 
     scale = a.scale or DEFAULT_SCALE[a.workload]

@@ -158,6 +158,71 @@ LMATCH_API int lmatch_info(const lmatch_graph* g, int64_t* n, int64_t* m, int64_
  * *nrounds receives the number of rounds.  (Fig. 8 "edges accessed per iteration".) */
 LMATCH_API int lmatch_round_log(const lmatch_graph* g, int64_t* out, int64_t cap, int64_t* nrounds);
 
+/* ---------------------------------------------------------------------------------------------
+ * Partitioned mode (multi-GPU, one process or thread per GPU).
+ *
+ * The vertex set is cut into nparts contiguous ranges part_bounds[0..nparts] (part_bounds[0] = 0,
+ * part_bounds[nparts] = n_global, every bound a multiple of 32), balanced by directed entries
+ * (P:96-98).  Each handle owns the rows of one range [v_begin, v_begin + n_local): a local
+ * CSR whose col_idx are GLOBAL vertex ids (cut edges appear in both owners' rows).
+ *
+ * The caller (e.g. paper_conf_sc_mandulakgfhs24_b200/dist.py over torch.distributed) drives the
+ * rounds and moves the data between handles:
+ *   lmatch_part_begin   -> round-1 pointers + claims         (per destination counts)
+ *   [exchange claims: segment p of every handle goes to the owner of part p]
+ *   lmatch_part_apply   -> record received claims, match       (mutual pointer check)
+ *   [allgather: every handle's owned bitmap words into every handle's bitmap]
+ *   lmatch_part_compact -> live set, next frontier             (local frontier size)
+ *   [stop when the SUM of frontier sizes over all parts is 0]
+ *   lmatch_part_point   -> frontier pointers + claims; then back to the exchange
+ *   lmatch_part_finish  -> owned mate[] slice, local w(M) share (edges with mate > u)
+ * A claim (v | u << 32) says "remote vertex u points to owned vertex v"; it replaces the paper's
+ * |V| x 64-bit nccl_AllReduce(pointers) (Alg. 2 L7), and the bitmap allgather (n/8 bytes)
+ * replaces nccl_AllReduce(mate) (Alg. 2 L9).  The result is bit-identical to the
+ * single-GPU run for every partition (Lemma III.1).  validate_level 2 and out-of-core
+ * are not available per partition (EINVAL).  Calls out of order return ESTATE.
+ * ------------------------------------------------------------------------------------------- */
+LMATCH_API int lmatch_create_part(const int64_t* csr_offsets, const int32_t* col_idx,
+                                  const float* weights, int64_t n_local, int64_t m_local,
+                                  int64_t v_begin, int64_t n_global, int32_t nparts,
+                                  const int64_t* part_bounds, const lmatch_opts* opts,
+                                  lmatch_graph** out);
+LMATCH_API int lmatch_create_part_device(const int64_t* d_offsets, const int32_t* d_col,
+                                         const float* d_weights, int64_t n_local, int64_t m_local,
+                                         int64_t v_begin, int64_t n_global, int32_t nparts,
+                                         const int64_t* part_bounds, const lmatch_opts* opts,
+                                         void* stream, lmatch_graph** out);
+/* Reset + round-1 pointer sweep over the owned rows + claims.  claim_counts: host int64[nparts]
+ * (claims destined to each part; the own part's entry is 0).  Synchronises `stream`. */
+LMATCH_API int lmatch_part_begin(lmatch_graph* g, void* stream, int64_t* claim_counts);
+/* seg_ptrs: host array of nparts DEVICE pointers; segment p holds claim_counts[p] uint64 claims. */
+LMATCH_API int lmatch_part_claims(const lmatch_graph* g, uint64_t** seg_ptrs);
+/* d_recv: DEVICE uint64[nrecv], all claims whose target this handle owns (any order). */
+LMATCH_API int lmatch_part_apply(lmatch_graph* g, const uint64_t* d_recv, int64_t nrecv,
+                                 void* stream);
+/* The replicated matched bitmap (DEVICE uint32[nwords_total]); this handle writes only words
+ * [word_begin, word_begin + nwords_own). */
+LMATCH_API int lmatch_part_bitmap(lmatch_graph* g, uint32_t** d_bits, int64_t* word_begin,
+                                  int64_t* nwords_own, int64_t* nwords_total);
+/* Copy helpers for callers that keep their exchange buffers elsewhere (e.g. torch tensors):
+ * claims of segment `part` (claim_counts[part] entries) -> d_dst; owned bitmap words -> d_dst;
+ * words [word_begin, word_begin + nwords) of the replicated bitmap <- d_src.  Stream-ordered. */
+LMATCH_API int lmatch_part_get_claims(const lmatch_graph* g, int32_t part, uint64_t* d_dst,
+                                      void* stream);
+LMATCH_API int lmatch_part_get_bits(const lmatch_graph* g, uint32_t* d_dst, void* stream);
+LMATCH_API int lmatch_part_set_bits(lmatch_graph* g, const uint32_t* d_src, int64_t word_begin,
+                                    int64_t nwords, void* stream);
+/* Rounds begun so far in this run; (timing=1) device ms of the last round-1 sweep. */
+LMATCH_API int lmatch_part_info(const lmatch_graph* g, int64_t* rounds, double* sweep_ms);
+/* Compaction; *nF_local = this part's next frontier size.  Synchronises `stream`. */
+LMATCH_API int lmatch_part_compact(lmatch_graph* g, void* stream, int64_t* nF_local);
+/* Pointer phase on the frontier + claims (counts as in lmatch_part_begin).  Synchronises. */
+LMATCH_API int lmatch_part_point(lmatch_graph* g, void* stream, int64_t* claim_counts);
+/* d_mate_local: DEVICE int32[n_local] (global ids, -1 unmatched); *w_local = sum of w over owned
+ * u with mate[u] > u (fp64); *matched_local = owned matched vertices.  Synchronises. */
+LMATCH_API int lmatch_part_finish(lmatch_graph* g, int32_t* d_mate_local, void* stream,
+                                  double* w_local, int64_t* matched_local);
+
 /* Release everything the handle owns.  NULL-safe. */
 LMATCH_API void lmatch_destroy(lmatch_graph* g);
 

@@ -152,14 +152,17 @@ __global__ void k_pack(const int32_t* __restrict__ col, const float* __restrict_
 // Self-loops are ignored (simple graph): their keys become 0, which never wins a max, so
 // no kernel on the hot path needs a per-entry self test.  8 lanes per row.
 __global__ void k_zap_self_loops(const int64_t* __restrict__ offs, AdjView adj, int64_t n,
-                                 unsigned long long* count) {
+                                 int64_t vbase, unsigned long long* count) {
   const int lane8 = threadIdx.x & 7;
   const int64_t g0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 3;
   const int64_t gs = ((int64_t)gridDim.x * blockDim.x) >> 3;
   unsigned long long c = 0;
   for (int64_t u = g0; u < n; u += gs)
     for (int64_t j = offs[u] + lane8; j < offs[u + 1]; j += 8)
-      if ((uint32_t)adj.at(j) == (uint32_t)u && adj.at(j) != 0ull) { *adj.ptr(j) = 0ull; ++c; }
+      if ((uint32_t)adj.at(j) == (uint32_t)(u + vbase) && adj.at(j) != 0ull) {
+        *adj.ptr(j) = 0ull;
+        ++c;
+      }
   for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
   if ((threadIdx.x & 31) == 0 && c) atomicAdd(count, c);
 }
@@ -796,10 +799,10 @@ __device__ __forceinline__ uint64_t make_pair(uint32_t lo, uint32_t hi) {
   return (uint64_t)lo | ((uint64_t)hi << 32);
 }
 __device__ __forceinline__ void row_range(const ulonglong2& e, const int64_t* __restrict__ offs,
-                                          int64_t* s, int64_t* en) {
+                                          int64_t vbase, int64_t* s, int64_t* en) {
   const uint64_t d = e.y >> 40;
   *s = (int64_t)(e.y & ((1ull << 40) - 1));
-  *en = d == kBigDeg ? offs[(uint32_t)e.x + 1] : *s + (int64_t)d;
+  *en = d == kBigDeg ? offs[(int64_t)(uint32_t)e.x - vbase + 1] : *s + (int64_t)d;
 }
 
 struct Bins {
@@ -838,7 +841,8 @@ __device__ __forceinline__ uint64_t scan_row_available(const AdjView adj,
 template <int G, int U>
 __global__ void k_point_bin(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
                             const int64_t* __restrict__ offs, const AdjView adj,
-                            const uint32_t* __restrict__ bits, uint64_t* __restrict__ best) {
+                            const uint32_t* __restrict__ bits, uint64_t* __restrict__ best,
+                            int64_t vbase) {
   const int64_t cnt = (int64_t)*cnt_ptr;
   const int lane = threadIdx.x & 31;
   const int gl = lane & (G - 1);
@@ -847,11 +851,11 @@ __global__ void k_point_bin(ulonglong2* __restrict__ list, const unsigned long l
   for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / G; i < cnt; i += ng) {
     const ulonglong2 e = list[i];
     int64_t s, en;
-    row_range(e, offs, &s, &en);
+    row_range(e, offs, vbase, &s, &en);
     const uint64_t b = group_max_key(scan_row_available<G, U>(adj, bits, s, en, gl), gmask);
     if (gl == 0) {
       const uint32_t u = (uint32_t)e.x;
-      best[u] = b;
+      best[u - vbase] = b;
       list[i].x = make_pair(u, b ? (uint32_t)b : kNoPtr);
     }
   }
@@ -861,13 +865,13 @@ template <int THREADS, int U>
 __global__ void __launch_bounds__(THREADS)
     k_point_bin_cta(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
                     const int64_t* __restrict__ offs, const AdjView adj,
-                    const uint32_t* __restrict__ bits, uint64_t* __restrict__ best) {
+                    const uint32_t* __restrict__ bits, uint64_t* __restrict__ best, int64_t vbase) {
   __shared__ uint64_t red[THREADS / 32];
   const int64_t cnt = (int64_t)*cnt_ptr;
   for (int64_t i = blockIdx.x; i < cnt; i += gridDim.x) {
     const ulonglong2 e = list[i];
     int64_t s, en;
-    row_range(e, offs, &s, &en);
+    row_range(e, offs, vbase, &s, &en);
     uint64_t b = scan_row_available<THREADS, U>(adj, bits, s, en, threadIdx.x);
     b = group_max_key(b, 0xffffffffu);
     if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = b;
@@ -877,7 +881,7 @@ __global__ void __launch_bounds__(THREADS)
       x = group_max_key(x, 0xffffffffu);
       if (threadIdx.x == 0) {
         const uint32_t u = (uint32_t)e.x;
-        best[u] = x;
+        best[u - vbase] = x;
         list[i].x = make_pair(u, x ? (uint32_t)x : kNoPtr);
       }
     }
@@ -947,7 +951,7 @@ __global__ void __launch_bounds__(256)
               const unsigned long long* cntFin, int64_t n, const uint64_t* __restrict__ best,
               const uint32_t* __restrict__ bits, const int64_t* __restrict__ offs,
               uint64_t* __restrict__ Sout, unsigned long long* cntSout, Bins Fout,
-              unsigned long long* cntFout, unsigned long long* swept) {
+              unsigned long long* cntFout, unsigned long long* swept, int64_t vbase) {
   constexpr int NW = 8, NL = 1 + kBins;  // warps per block (blockDim 256), output lists
   __shared__ unsigned wtot[NW][NL];
   __shared__ unsigned long long wbase[NW][NL];
@@ -973,7 +977,7 @@ __global__ void __launch_bounds__(256)
       if (i < cnt) {
         if (ALL) {
           const uint64_t bb = best[i];
-          p = make_pair((uint32_t)i, bb ? (uint32_t)bb : kNoPtr);
+          p = make_pair((uint32_t)(i + vbase), bb ? (uint32_t)bb : kNoPtr);
         } else {
           p = i < p0 ? S[i]
               : i < p1 ? Fin.list[0][i - p0].x
@@ -1002,8 +1006,8 @@ __global__ void __launch_bounds__(256)
       const bool tgt = (wv[k] >> (v & 31)) & 1u;
       if (live && !tgt) sbits |= 1u << k;
       const bool fr = live && tgt;
-      os[k] = fr ? offs[u] : 0;
-      oe[k] = fr ? offs[u + 1] : -1;
+      os[k] = fr ? offs[u - vbase] : 0;
+      oe[k] = fr ? offs[u - vbase + 1] : -1;
     }
 #pragma unroll
     for (int k = 0; k < K; ++k) {
@@ -1071,6 +1075,134 @@ __global__ void __launch_bounds__(256)
 }
 
 // =============================================================================================
+// Partitioned mode (A3/A5): this rank owns rows [vbase, vend) of a 1-D vertex
+// partition; the matched bitmap is replicated; ghost[x] holds, for a remote vertex x,
+// the owned vertex x last claimed to point to.  A pointer into u moves off u only after u is
+// matched, so a stale ghost is never consulted while u is live (extends Lemma III.1).
+// Claims (v | u << 32): "u points to v", sent to owner(v) instead of the paper's
+// |V| x 64-bit nccl_AllReduce(pointers) (Alg. 2 L7).
+// =============================================================================================
+__device__ __forceinline__ int owner_of(const int64_t* __restrict__ bounds, int P, uint32_t v) {
+  int lo = 0, hi = P - 1;  // last p with bounds[p] <= v
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (bounds[mid] <= (int64_t)v) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+__device__ __forceinline__ uint32_t ptr_of(const uint64_t* __restrict__ best,
+                                           const uint32_t* __restrict__ ghost, int64_t vbase,
+                                           int64_t vend, uint32_t v) {
+  if ((int64_t)v >= vbase && (int64_t)v < vend) {
+    const uint64_t k = best[v - vbase];
+    return k ? (uint32_t)k : kNoPtr;
+  }
+  return ghost[v];
+}
+struct Claims {
+  uint64_t* seg;               // P segments of `cap` claims each
+  int64_t cap;
+  unsigned long long* count;   // [P]
+  const int64_t* bounds;       // [P+1]
+  int P;
+};
+// warp-collective (all 32 lanes call it): lanes with the same destination share one atomic
+__device__ __forceinline__ void claim_append(const Claims& C, bool pred, uint32_t v, uint32_t u) {
+  const int d = pred ? owner_of(C.bounds, C.P, v) : -1;
+  const unsigned peers = __match_any_sync(0xffffffffu, d);
+  if (!pred) return;
+  const int lane = threadIdx.x & 31, leader = __ffs(peers) - 1;
+  unsigned long long base = 0;
+  if (lane == leader) base = atomicAdd(&C.count[d], (unsigned long long)__popc(peers));
+  base = __shfl_sync(peers, base, leader);
+  C.seg[(int64_t)d * C.cap + (int64_t)(base + __popc(peers & lanemask_lt()))] = make_pair(v, u);
+}
+// round 1: every owned vertex whose pointer targets a remote vertex
+__global__ void k_claims_all(const uint64_t* __restrict__ best, int64_t n_loc, int64_t vbase,
+                             int64_t vend, Claims C) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t n32 = (n_loc + 31) & ~31ll;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n32; i += stride) {
+    const uint64_t b = i < n_loc ? best[i] : 0ull;
+    const uint32_t v = (uint32_t)b;
+    claim_append(C, b != 0 && ((int64_t)v < vbase || (int64_t)v >= vend), v, (uint32_t)(i + vbase));
+  }
+}
+// rounds >= 2: the re-pointed frontier
+__global__ void k_claims_bins(Bins F, const unsigned long long* cntF, int64_t vbase, int64_t vend,
+                              Claims C) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+#pragma unroll
+  for (int bb = 0; bb < kBins; ++bb) {
+    const int64_t c = (int64_t)cntF[bb];
+    const int64_t c32 = (c + 31) & ~31ll;
+    for (int64_t i = tid; i < c32; i += stride) {
+      const uint64_t p = i < c ? F.list[bb][i].x : ((uint64_t)kNoPtr << 32);
+      const uint32_t u = (uint32_t)p, v = (uint32_t)(p >> 32);
+      claim_append(C, v != kNoPtr && ((int64_t)v < vbase || (int64_t)v >= vend), v, u);
+    }
+  }
+}
+// received claims (v owned, u remote): record the ghost pointer
+__global__ void k_apply_claims(const uint64_t* __restrict__ recv, int64_t nrecv, uint32_t* ghost) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nrecv; i += stride) {
+    const uint64_t c = recv[i];
+    ghost[(uint32_t)(c >> 32)] = (uint32_t)c;
+  }
+}
+// ... and match them: v (owned) with u (remote) iff ptr v == u
+__global__ void k_match_claims(const uint64_t* __restrict__ recv, int64_t nrecv,
+                               const uint64_t* __restrict__ best, int64_t vbase, uint32_t* bits) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nrecv; i += stride) {
+    const uint64_t c = recv[i];
+    const uint32_t v = (uint32_t)c, u = (uint32_t)(c >> 32);
+    const uint64_t kv = best[v - vbase];
+    if (kv != 0 && (uint32_t)kv == u) atomicOr(&bits[v >> 5], 1u << (v & 31));
+  }
+}
+// round 1 match over every owned vertex (owned range starts on a 32-vertex boundary)
+__global__ void k_match_part_all(const uint64_t* __restrict__ best, int64_t n_loc, int64_t vbase,
+                                 int64_t vend, const uint32_t* __restrict__ ghost, uint32_t* bits) {
+  const int64_t nwords = (n_loc + 31) >> 5;
+  const int lane = threadIdx.x & 31;
+  const int64_t w0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t ws = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t wi = w0; wi < nwords; wi += ws) {
+    const int64_t i = (wi << 5) + lane;
+    bool mutual = false;
+    if (i < n_loc) {
+      const uint64_t b = best[i];
+      if (b) mutual = ptr_of(best, ghost, vbase, vend, (uint32_t)b) == (uint32_t)(i + vbase);
+    }
+    const unsigned word = __ballot_sync(0xffffffffu, mutual);
+    if (lane == 0) bits[(vbase >> 5) + wi] = word;
+  }
+}
+// rounds >= 2 match over the re-pointed frontier
+__global__ void k_match_part_bins(Bins F, const unsigned long long* cntF,
+                                  const uint64_t* __restrict__ best, int64_t vbase, int64_t vend,
+                                  const uint32_t* __restrict__ ghost, uint32_t* bits) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+#pragma unroll
+  for (int bb = 0; bb < kBins; ++bb) {
+    const int64_t c = (int64_t)cntF[bb];
+    for (int64_t i = tid; i < c; i += stride) {
+      const uint64_t p = F.list[bb][i].x;
+      const uint32_t u = (uint32_t)p, v = (uint32_t)(p >> 32);
+      if (v == kNoPtr) continue;
+      if (ptr_of(best, ghost, vbase, vend, v) == u) {
+        atomicOr(&bits[u >> 5], 1u << (u & 31));
+        if ((int64_t)v >= vbase && (int64_t)v < vend) atomicOr(&bits[v >> 5], 1u << (v & 31));
+      }
+    }
+  }
+}
+
+// =============================================================================================
 // A10/A9: mate[] materialisation + deterministic fp64 weight / cardinality partial sums
 // =============================================================================================
 template <int THREADS>
@@ -1093,19 +1225,20 @@ __device__ __forceinline__ void block_sum2(double w, long long c, double* outw, 
 template <int THREADS>
 __global__ void __launch_bounds__(THREADS)
     k_materialize(const uint64_t* __restrict__ best, const uint32_t* __restrict__ bits, int64_t n,
-                  int32_t* __restrict__ mate, double* pw, long long* pc) {
+                  int64_t vbase, int32_t* __restrict__ mate, double* pw, long long* pc) {
   double w = 0.0;
   long long c = 0;
   const int64_t stride = (int64_t)gridDim.x * THREADS;
-  for (int64_t u = (int64_t)blockIdx.x * THREADS + threadIdx.x; u < n; u += stride) {
+  for (int64_t i = (int64_t)blockIdx.x * THREADS + threadIdx.x; i < n; i += stride) {
+    const int64_t u = i + vbase;
     int32_t v = -1;
     if (bit_test(bits, (uint32_t)u)) {
-      const uint64_t k = best[u];
+      const uint64_t k = best[i];
       v = (int32_t)(uint32_t)k;
       ++c;
       if ((int64_t)v > u) w += (double)__uint_as_float((uint32_t)(k >> 32));
     }
-    mate[u] = v;
+    mate[i] = v;
   }
   block_sum2<THREADS>(w, c, &pw[blockIdx.x], &pc[blockIdx.x]);
 }

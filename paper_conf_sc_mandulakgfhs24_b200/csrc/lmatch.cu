@@ -91,7 +91,18 @@ struct lmatch_graph {
   int device = 0;
   cudaStream_t stream = nullptr;   // handle stream
   cudaStream_t up[2] = {nullptr, nullptr};
-  int64_t n = 0, m = 0, n_nz = 0, ntiles = 0;
+  int64_t n = 0, m = 0, n_nz = 0, ntiles = 0;  // n, m: this handle's rows and entries
+  // partitioned mode (lmatch_create_part): rows [v0, v0 + n) of a graph with n_global vertices
+  int64_t v0 = 0, n_global = 0;
+  int P = 1;
+  int64_t* bounds = nullptr;         // device [P+1]
+  uint32_t* ghost = nullptr;         // device [n_global]
+  uint64_t* claims = nullptr;        // device [P * claim_cap]
+  int64_t claim_cap = 0;
+  unsigned long long* claim_cnt = nullptr;    // device [P]
+  unsigned long long* h_claim_cnt = nullptr;  // pinned [P]
+  int part_round = 0, part_cur = 0;
+  float part_sweep_ms = 0.f;  // (timing=1) last lmatch_part_begin's round-1 sweep
   int validate_level = 1;
   int timing = 0;
   int64_t max_rounds = 0;
@@ -209,7 +220,7 @@ int alloc_all(lmatch_graph* g) {
   TRY(dmalloc(g, &g->noffs_lo, (size_t)n + 9));
   TRY(dmalloc(g, &g->atomic_rows, (size_t)n + (size_t)g->ntiles + 1));
   TRY(dmalloc(g, &g->best, (size_t)n + 1));
-  TRY(dmalloc(g, &g->bits, (size_t)((n + 31) / 32) + 1));
+  TRY(dmalloc(g, &g->bits, (size_t)((g->n_global + 31) / 32) + 1));
   for (int i = 0; i < 2; ++i) TRY(dmalloc(g, &g->S[i], (size_t)n + 1));
   TRY(dmalloc(g, &g->counters, lm::kNumCounters));
   TRY(dmalloc(g, &g->pw, kFinBlocks));
@@ -347,13 +358,13 @@ int upload_host(lmatch_graph* g, const int64_t* offsets, const int32_t* col, con
     // entries below R go to HBM, the rest to the pinned host copy (written through its alias)
     const int64_t nd = std::max<int64_t>(0, std::min(cnt, g->R - base));
     if (nd > 0) {
-      lm::k_pack<<<grid_for(nd, 256, 16384), 256, 0, s>>>(g->st_col[i], g->st_w[i], nd, n,
+      lm::k_pack<<<grid_for(nd, 256, 16384), 256, 0, s>>>(g->st_col[i], g->st_w[i], nd, g->n_global,
                                                           g->adj + base, base, g->perr);
       CKL();
     }
     if (cnt > nd) {
       lm::k_pack<<<grid_for(cnt - nd, 256, 16384), 256, 0, s>>>(
-          g->st_col[i] + nd, g->st_w[i] + nd, cnt - nd, n, g->host_adj_dev + (base + nd - g->R),
+          g->st_col[i] + nd, g->st_w[i] + nd, cnt - nd, g->n_global, g->host_adj_dev + (base + nd - g->R),
           base + nd, g->perr);
       CKL();
     }
@@ -373,11 +384,11 @@ int upload_device(lmatch_graph* g, const int64_t* d_offsets, const int32_t* d_co
   if (m > 0) {
     const int64_t nd = std::min(m, g->R);
     if (nd > 0) {
-      lm::k_pack<<<grid_for(nd, 256, 65536), 256, 0, st>>>(d_col, d_w, nd, n, g->adj, 0, g->perr);
+      lm::k_pack<<<grid_for(nd, 256, 65536), 256, 0, st>>>(d_col, d_w, nd, g->n_global, g->adj, 0, g->perr);
       CKL();
     }
     if (m > nd) {
-      lm::k_pack<<<grid_for(m - nd, 256, 65536), 256, 0, st>>>(d_col + nd, d_w + nd, m - nd, n,
+      lm::k_pack<<<grid_for(m - nd, 256, 65536), 256, 0, st>>>(d_col + nd, d_w + nd, m - nd, g->n_global,
                                                                g->host_adj_dev, nd, g->perr);
       CKL();
     }
@@ -436,7 +447,7 @@ int finish_create(lmatch_graph* g, cudaStream_t st) {
   if (g->m > 0) {
     CK(cudaMemsetAsync(g->werr, 0, 8, st));
     lm::k_zap_self_loops<<<grid_for(g->n * 8, 256, 16384), 256, 0, st>>>(
-        g->offs, g->view(), g->n, reinterpret_cast<unsigned long long*>(g->werr));
+        g->offs, g->view(), g->n, g->v0, reinterpret_cast<unsigned long long*>(g->werr));
     CKL();
   }
   TRY(build_index(g, st));
@@ -458,13 +469,25 @@ int finish_create(lmatch_graph* g, cudaStream_t st) {
   return LMATCH_OK;
 }
 
+struct PartSpec {
+  int64_t v0 = 0, n_global = -1;
+  int P = 1;
+  const int64_t* bounds = nullptr;  // host [P+1]
+};
+
 int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** out,
-                  lmatch_graph** gp) {
+                  lmatch_graph** gp, const PartSpec* part = nullptr) {
   lmatch_graph* g = new (std::nothrow) lmatch_graph();
   if (!g) { set_err("host allocation failed"); return LMATCH_ENOMEM; }
   *gp = g;
   g->n = n;
   g->m = m;
+  g->n_global = n;
+  if (part) {
+    g->v0 = part->v0;
+    g->n_global = part->n_global;
+    g->P = part->P;
+  }
   if (opts) {
     if (opts->use_device) CK(cudaSetDevice(opts->device));
     if (opts->validate_level != 0) g->validate_level = opts->validate_level;
@@ -482,7 +505,64 @@ int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** 
   CK(cudaStreamCreateWithFlags(&g->up[1], cudaStreamNonBlocking));
   for (auto& e : g->ev) CK(cudaEventCreate(&e));
   TRY(alloc_all(g));
+  if (part) {
+    TRY(dmalloc(g, &g->bounds, (size_t)g->P + 1));
+    CK(cudaMemcpy(g->bounds, part->bounds, ((size_t)g->P + 1) * 8, cudaMemcpyHostToDevice));
+    TRY(dmalloc(g, &g->ghost, (size_t)g->n_global + 1));
+    g->claim_cap = std::max<int64_t>(n, 1);
+    TRY(dmalloc(g, &g->claims, (size_t)g->P * (size_t)g->claim_cap));
+    TRY(dmalloc(g, &g->claim_cnt, (size_t)g->P));
+    CK(cudaHostAlloc(reinterpret_cast<void**>(&g->h_claim_cnt), (size_t)g->P * 8, cudaHostAllocDefault));
+  }
   (void)out;
+  return LMATCH_OK;
+}
+
+// Round-1 pointer sweep (A2) over every local row: resident tiles, then (out-of-core) the
+// streamed chunks through a 2-slot device ring -- the copy of chunk k+1 on the copy stream
+// overlaps the sweep of chunk k on the run stream (LOADBATCH double buffering).
+int round1_sweep(lmatch_graph* g, cudaStream_t st, int64_t* launches_out, int64_t* sweep_out,
+                 int64_t* streamed_out) {
+  int64_t launches = 0, sweep_launches = 0, bytes_streamed = 0;
+#if LM_SWEEP_IMPL == 2
+  lm::Sweep2DArgs A{g->noffs_lo, g->nzr, g->tile_nz, g->best, g->m, g->ntiles};
+  SWEEP_KERNEL<<<g->sweep_grid, kSweepThreads, Sweep::kSmem, st>>>(g->tmap, A);
+  CKL();
+  ++launches;
+  ++sweep_launches;
+#else
+  // resident tiles [0, R/TILE), then the streamed chunks through a 2-slot device ring:
+  // the copy of chunk k+1 (copy stream) overlaps the sweep of chunk k (run stream).
+  const int64_t rt = g->streaming ? g->R / kTile : g->ntiles;
+  auto sweep_launch = [&](const uint64_t* base, int64_t t0, int64_t t1) -> int {
+    const int64_t grid = std::min<int64_t>((t1 - t0 + kSweepWarps - 1) / kSweepWarps, g->sweep_grid);
+    lm::SweepArgs A{base, g->noffs_lo, g->nzr, g->tile_nz, g->best, g->m, t0, t1};
+    SWEEP_KERNEL<<<(unsigned)std::max<int64_t>(grid, 1), kSweepThreads, Sweep::kSmem, st>>>(A);
+    CKL();
+    ++launches;
+    ++sweep_launches;
+    return LMATCH_OK;
+  };
+  if (rt > 0) TRY(sweep_launch(g->adj, 0, std::min(rt, g->ntiles)));
+  if (g->streaming) {
+    const int64_t C = g->stream_chunk;
+    for (int64_t e0 = g->R, k = 0; e0 < g->m; e0 += C, ++k) {
+      const int slot = (int)(k & 1);
+      const int64_t cnt = std::min(C, g->m - e0);
+      if (k >= 2) CK(cudaStreamWaitEvent(g->cs, g->ev_free[slot], 0));
+      CK(cudaMemcpyAsync(g->ring[slot], g->host_adj + (e0 - g->R), (size_t)cnt * 8,
+                         cudaMemcpyHostToDevice, g->cs));
+      CK(cudaEventRecord(g->ev_full[slot], g->cs));
+      bytes_streamed += cnt * 8;
+      CK(cudaStreamWaitEvent(st, g->ev_full[slot], 0));
+      TRY(sweep_launch(g->ring[slot], e0 / kTile, std::min(g->ntiles, (e0 + cnt + kTile - 1) / kTile)));
+      CK(cudaEventRecord(g->ev_free[slot], st));
+    }
+  }
+#endif
+  *launches_out += launches;
+  *sweep_out += sweep_launches;
+  *streamed_out += bytes_streamed;
   return LMATCH_OK;
 }
 
@@ -527,6 +607,9 @@ void lmatch_destroy(lmatch_graph* g) {
     if (g->ev_free[i]) cudaEventDestroy(g->ev_free[i]);
   }
   if (g->cs) cudaStreamDestroy(g->cs);
+  void* pdev[] = {g->bounds, g->ghost, g->claims, g->claim_cnt};
+  for (void* p : pdev) if (p) cudaFree(p);
+  if (g->h_claim_cnt) cudaFreeHost(g->h_claim_cnt);
   if (g->h_res) cudaFreeHost(g->h_res);
   if (g->h_resc) cudaFreeHost(g->h_resc);
   for (auto e : g->ev) if (e) cudaEventDestroy(e);
@@ -625,7 +708,7 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
 
   if (tm) CK(cudaEventRecord(g->ev[0], st));
   // ---- reset (bitmap, counters, tile-crossing rows' best)
-  const int64_t nwords = (n + 31) / 32;
+  const int64_t nwords = (g->n_global + 31) / 32;
   lm::k_reset<<<grid_for(std::max(nwords, g->n_atomic), 256, 4096), 256, 0, st>>>(
       g->bits, nwords, g->best, g->atomic_rows, g->n_atomic, C, lm::kNumCounters);
   CKL();
@@ -633,39 +716,7 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
   if (tm) CK(cudaEventRecord(g->ev[1], st));
   if (g->ntiles > 0 && n > 0) {
     // ---- round 1: A2 full sweep (no bitmap test), A4 match-all, A6 compact-all
-#if LM_SWEEP_IMPL == 2
-    lm::Sweep2DArgs A{g->noffs_lo, g->nzr, g->tile_nz, g->best, g->m, g->ntiles};
-    SWEEP_KERNEL<<<g->sweep_grid, kSweepThreads, Sweep::kSmem, st>>>(g->tmap, A);
-#else
-    // resident tiles [0, R/TILE), then the streamed chunks through a 2-slot device ring:
-    // the copy of chunk k+1 (copy stream) overlaps the sweep of chunk k (run stream).
-    const int64_t rt = g->streaming ? g->R / kTile : g->ntiles;
-    auto sweep_launch = [&](const uint64_t* base, int64_t t0, int64_t t1) -> int {
-      const int64_t grid = std::min<int64_t>((t1 - t0 + kSweepWarps - 1) / kSweepWarps, g->sweep_grid);
-      lm::SweepArgs A{base, g->noffs_lo, g->nzr, g->tile_nz, g->best, g->m, t0, t1};
-      SWEEP_KERNEL<<<(unsigned)std::max<int64_t>(grid, 1), kSweepThreads, Sweep::kSmem, st>>>(A);
-      CKL();
-      ++launches;
-      ++sweep_launches;
-      return LMATCH_OK;
-    };
-    if (rt > 0) TRY(sweep_launch(g->adj, 0, std::min(rt, g->ntiles)));
-    if (g->streaming) {
-      const int64_t C = g->stream_chunk;
-      for (int64_t e0 = g->R, k = 0; e0 < g->m; e0 += C, ++k) {
-        const int slot = (int)(k & 1);
-        const int64_t cnt = std::min(C, g->m - e0);
-        if (k >= 2) CK(cudaStreamWaitEvent(g->cs, g->ev_free[slot], 0));
-        CK(cudaMemcpyAsync(g->ring[slot], g->host_adj + (e0 - g->R), (size_t)cnt * 8,
-                           cudaMemcpyHostToDevice, g->cs));
-        CK(cudaEventRecord(g->ev_full[slot], g->cs));
-        bytes_streamed += cnt * 8;
-        CK(cudaStreamWaitEvent(st, g->ev_full[slot], 0));
-        TRY(sweep_launch(g->ring[slot], e0 / kTile, std::min(g->ntiles, (e0 + cnt + kTile - 1) / kTile)));
-        CK(cudaEventRecord(g->ev_free[slot], st));
-      }
-    }
-#endif
+    TRY(round1_sweep(g, st, &launches, &sweep_launches, &bytes_streamed));
     CKL();
     if (tm) CK(cudaEventRecord(g->ev[2], st));
     rounds = 1;
@@ -673,7 +724,7 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
     CKL();
     lm::k_compact<true, kCompactK><<<grid_for((n + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
         nullptr, nullptr, lm::Bins{}, nullptr, n, g->best, g->bits, g->offs, g->S[0],
-        C + lm::cnt_S(0), g->F[0], C + lm::cnt_F(0, 0), C + lm::kCntSwept);
+        C + lm::cnt_S(0), g->F[0], C + lm::cnt_F(0, 0), C + lm::kCntSwept, g->v0);
     CKL();
     launches += 2;
     CK(cudaMemcpyAsync(hc, C, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
@@ -696,10 +747,10 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
       // A2 frontier pointer phase, one launch per non-empty degree bin
       lm::Bins& Fb = g->F[cur];
       const int kMaxGrid = 65536;
-      if (nFb[0]) { lm::k_point_bin<1, 8><<<grid_for(nFb[0], 256, kMaxGrid), 256, 0, st>>>(Fb.list[0], cF + 0, g->offs, g->view(), g->bits, g->best); CKL(); ++launches; }    // deg <= 8: a thread each
-      if (nFb[1]) { lm::k_point_bin<8, 8><<<grid_for(nFb[1] * 8, 256, kMaxGrid), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, g->view(), g->bits, g->best); CKL(); ++launches; }     // 9..64
-      if (nFb[2]) { lm::k_point_bin<32, 4><<<grid_for(nFb[2] * 32, 256, kMaxGrid), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, g->view(), g->bits, g->best); CKL(); ++launches; }   // 65..2048
-      if (nFb[3]) { lm::k_point_bin_cta<256, 4><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, g->view(), g->bits, g->best); CKL(); ++launches; }
+      if (nFb[0]) { lm::k_point_bin<1, 8><<<grid_for(nFb[0], 256, kMaxGrid), 256, 0, st>>>(Fb.list[0], cF + 0, g->offs, g->view(), g->bits, g->best, g->v0); CKL(); ++launches; }    // deg <= 8: a thread each
+      if (nFb[1]) { lm::k_point_bin<8, 8><<<grid_for(nFb[1] * 8, 256, kMaxGrid), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, g->view(), g->bits, g->best, g->v0); CKL(); ++launches; }     // 9..64
+      if (nFb[2]) { lm::k_point_bin<32, 4><<<grid_for(nFb[2] * 32, 256, kMaxGrid), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, g->view(), g->bits, g->best, g->v0); CKL(); ++launches; }   // 65..2048
+      if (nFb[3]) { lm::k_point_bin_cta<256, 4><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, g->view(), g->bits, g->best, g->v0); CKL(); ++launches; }
       // A4 match over the new pointers
       lm::k_match_bins<<<grid_for(nF, 256, 65536), 256, 0, st>>>(Fb, cF, g->best, g->bits);
       CKL();
@@ -709,7 +760,7 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
       lm::k_compact<false, kCompactK>
           <<<grid_for((nS + nF + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
               g->S[cur], C + lm::cnt_S(cur), Fb, cF, n, g->best, g->bits, g->offs, g->S[nxt],
-              C + lm::cnt_S(nxt), g->F[nxt], C + lm::cnt_F(nxt, 0), C + lm::kCntSwept);
+              C + lm::cnt_S(nxt), g->F[nxt], C + lm::cnt_F(nxt, 0), C + lm::kCntSwept, g->v0);
       CKL();
       launches += 2;
       CK(cudaMemcpyAsync(hc, C, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
@@ -723,8 +774,8 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
   if (tm) CK(cudaEventRecord(g->ev[4], st));
   // ---- A10 mate[] + A9 w(M)
   if (n > 0) {
-    lm::k_materialize<kFinThreads><<<kFinBlocks, kFinThreads, 0, st>>>(g->best, g->bits, n, d_mate,
-                                                                       g->pw, g->pc);
+    lm::k_materialize<kFinThreads><<<kFinBlocks, kFinThreads, 0, st>>>(g->best, g->bits, n, g->v0,
+                                                                       d_mate, g->pw, g->pc);
     CKL();
     lm::k_final_sum<<<1, 32, 0, st>>>(g->pw, g->pc, kFinBlocks, g->res_w, g->res_c);
     CKL();
@@ -816,4 +867,283 @@ int lmatch_weight(lmatch_graph* g, const int32_t* mate, double* out_weight) {
   return lmatch_weight_device(g, g->mate_tmp, g->stream, out_weight);
 }
 
+// ------------------------------------------------------------------ partitioned mode (A3/A5)
+static int check_part(int64_t n_local, int64_t v_begin, int64_t n_global, int32_t nparts,
+                      const int64_t* bounds) {
+  if (nparts < 1 || !bounds) { set_err("nparts < 1 or NULL part_bounds"); return LMATCH_EINVAL; }
+  if (n_global < 0 || n_global >= ((int64_t)1 << 31)) { set_err("n_global out of range"); return LMATCH_ERANGE; }
+  if (bounds[0] != 0 || bounds[nparts] != n_global) { set_err("part_bounds must span [0, n_global]"); return LMATCH_EINVAL; }
+  bool found = false;
+  for (int p = 0; p < nparts; ++p) {
+    if (bounds[p + 1] < bounds[p]) { set_err("part_bounds decrease"); return LMATCH_EINVAL; }
+    if (bounds[p] % 32 != 0 && bounds[p] != n_global) { set_err("part_bounds must be multiples of 32"); return LMATCH_EINVAL; }
+    if (bounds[p] == v_begin && bounds[p + 1] == v_begin + n_local) found = true;
+  }
+  if (!found) { set_err("[v_begin, v_begin + n_local) is not a part of part_bounds"); return LMATCH_EINVAL; }
+  return LMATCH_OK;
+}
+
+int lmatch_create_part(const int64_t* csr_offsets, const int32_t* col_idx, const float* weights,
+                       int64_t n_local, int64_t m_local, int64_t v_begin, int64_t n_global,
+                       int32_t nparts, const int64_t* part_bounds, const lmatch_opts* opts,
+                       lmatch_graph** out) {
+  if (!out) { set_err("out == NULL"); return LMATCH_EINVAL; }
+  *out = nullptr;
+  g_err[0] = 0;
+  int s = check_args(csr_offsets, col_idx, weights, n_local, m_local);
+  if (!s) s = check_part(n_local, v_begin, n_global, nparts, part_bounds);
+  if (s) return s;
+  if (opts && opts->validate_level >= 2) { set_err("validate_level 2 is not available per partition"); return LMATCH_EINVAL; }
+  if (opts && opts->hbm_budget_bytes > 0) { set_err("out-of-core is not available per partition"); return LMATCH_EINVAL; }
+  PartSpec ps;
+  ps.v0 = v_begin; ps.n_global = n_global; ps.P = nparts; ps.bounds = part_bounds;
+  lmatch_graph* g = nullptr;
+  s = create_common(n_local, m_local, opts, out, &g, &ps);
+  if (!s) s = upload_host(g, csr_offsets, col_idx, weights);
+  if (!s) s = finish_create(g, g->stream);
+  if (s) { lmatch_destroy(g); return s; }
+  *out = g;
+  return LMATCH_OK;
+}
+
+int lmatch_create_part_device(const int64_t* d_offsets, const int32_t* d_col, const float* d_weights,
+                              int64_t n_local, int64_t m_local, int64_t v_begin, int64_t n_global,
+                              int32_t nparts, const int64_t* part_bounds, const lmatch_opts* opts,
+                              void* stream, lmatch_graph** out) {
+  if (!out) { set_err("out == NULL"); return LMATCH_EINVAL; }
+  *out = nullptr;
+  g_err[0] = 0;
+  int s = check_args(d_offsets, d_col, d_weights, n_local, m_local);
+  if (!s) s = check_part(n_local, v_begin, n_global, nparts, part_bounds);
+  if (s) return s;
+  if (opts && opts->validate_level >= 2) { set_err("validate_level 2 is not available per partition"); return LMATCH_EINVAL; }
+  if (opts && opts->hbm_budget_bytes > 0) { set_err("out-of-core is not available per partition"); return LMATCH_EINVAL; }
+  PartSpec ps;
+  ps.v0 = v_begin; ps.n_global = n_global; ps.P = nparts; ps.bounds = part_bounds;
+  lmatch_graph* g = nullptr;
+  s = create_common(n_local, m_local, opts, out, &g, &ps);
+  cudaStream_t st = stream ? (cudaStream_t)stream : (g ? g->stream : nullptr);
+  if (!s) {
+    cudaError_t e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) { set_err("stream sync: %s", cudaGetErrorString(e)); s = LMATCH_ECUDA; }
+  }
+  if (!s) s = upload_device(g, d_offsets, d_col, d_weights, st);
+  if (!s) s = finish_create(g, st);
+  if (s) { lmatch_destroy(g); return s; }
+  *out = g;
+  return LMATCH_OK;
+}
+
+static int part_claims_out(lmatch_graph* g, cudaStream_t st, int64_t* claim_counts) {
+  CK(cudaMemcpyAsync(g->h_claim_cnt, g->claim_cnt, (size_t)g->P * 8, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  if (claim_counts)
+    for (int p = 0; p < g->P; ++p) claim_counts[p] = (int64_t)g->h_claim_cnt[p];
+  return LMATCH_OK;
+}
+
+int lmatch_part_begin(lmatch_graph* g, void* stream, int64_t* claim_counts) {
+  if (!g || !g->ghost) { set_err("not a partition handle"); return LMATCH_ESTATE; }
+  g_err[0] = 0;
+  CK(cudaSetDevice(g->device));
+  cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
+  const int64_t nwords = (g->n_global + 31) / 32;
+  lm::k_reset<<<grid_for(std::max(nwords, g->n_atomic), 256, 4096), 256, 0, st>>>(
+      g->bits, nwords, g->best, g->atomic_rows, g->n_atomic, g->counters, lm::kNumCounters);
+  CKL();
+  CK(cudaMemsetAsync(g->ghost, 0xff, ((size_t)g->n_global + 1) * 4, st));
+  CK(cudaMemsetAsync(g->claim_cnt, 0, (size_t)g->P * 8, st));
+  int64_t l = 0, sl = 0, bs = 0;
+  if (g->timing) CK(cudaEventRecord(g->ev[1], st));
+  if (g->ntiles > 0 && g->n > 0) TRY(round1_sweep(g, st, &l, &sl, &bs));
+  if (g->timing) CK(cudaEventRecord(g->ev[2], st));
+  lm::Claims Cl{g->claims, g->claim_cap, g->claim_cnt, g->bounds, g->P};
+  if (g->n > 0) {
+    lm::k_claims_all<<<grid_for(g->n, 256, 65536), 256, 0, st>>>(g->best, g->n, g->v0,
+                                                                   g->v0 + g->n, Cl);
+    CKL();
+  }
+  g->part_round = 1;
+  g->round_log.clear();
+  const int rc = part_claims_out(g, st, claim_counts);
+  if (!rc && g->timing) CK(cudaEventElapsedTime(&g->part_sweep_ms, g->ev[1], g->ev[2]));
+  return rc;
+}
+
+int lmatch_part_claims(const lmatch_graph* g, uint64_t** seg_ptrs) {
+  if (!g || !g->ghost || !seg_ptrs) { set_err("not a partition handle / NULL"); return LMATCH_ESTATE; }
+  for (int p = 0; p < g->P; ++p) seg_ptrs[p] = g->claims + (int64_t)p * g->claim_cap;
+  return LMATCH_OK;
+}
+
+int lmatch_part_apply(lmatch_graph* g, const uint64_t* d_recv, int64_t nrecv, void* stream) {
+  if (!g || !g->ghost || g->part_round < 1) { set_err("lmatch_part_apply out of order"); return LMATCH_ESTATE; }
+  if (nrecv > 0 && !d_recv) { set_err("NULL claims"); return LMATCH_EINVAL; }
+  CK(cudaSetDevice(g->device));
+  cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
+  if (nrecv > 0) {
+    lm::k_apply_claims<<<grid_for(nrecv, 256, 65536), 256, 0, st>>>(d_recv, nrecv, g->ghost);
+    CKL();
+  }
+  if (g->part_round == 1) {
+    if (g->n > 0) {
+      lm::k_match_part_all<<<grid_for(((g->n + 31) / 32) * 32, 256, 65536), 256, 0, st>>>(
+          g->best, g->n, g->v0, g->v0 + g->n, g->ghost, g->bits);
+      CKL();
+    }
+  } else {
+    int64_t nF = 0;
+    for (int b = 0; b < lm::kBins; ++b) nF += (int64_t)g->h_counters[lm::cnt_F(g->part_cur, b)];
+    if (nF > 0) {
+      lm::k_match_part_bins<<<grid_for(nF, 256, 65536), 256, 0, st>>>(
+          g->F[g->part_cur], g->counters + lm::cnt_F(g->part_cur, 0), g->best, g->v0, g->v0 + g->n,
+          g->ghost, g->bits);
+      CKL();
+    }
+  }
+  if (nrecv > 0) {
+    lm::k_match_claims<<<grid_for(nrecv, 256, 65536), 256, 0, st>>>(d_recv, nrecv, g->best, g->v0,
+                                                                      g->bits);
+    CKL();
+  }
+  return LMATCH_OK;
+}
+
+int lmatch_part_info(const lmatch_graph* g, int64_t* rounds, double* sweep_ms) {
+  if (!g || !g->ghost) { set_err("not a partition handle"); return LMATCH_ESTATE; }
+  if (rounds) *rounds = g->part_round;
+  if (sweep_ms) *sweep_ms = g->part_sweep_ms;
+  return LMATCH_OK;
+}
+
+int lmatch_part_bitmap(lmatch_graph* g, uint32_t** d_bits, int64_t* word_begin, int64_t* nwords_own,
+                       int64_t* nwords_total) {
+  if (!g) { set_err("NULL handle"); return LMATCH_ESTATE; }
+  if (d_bits) *d_bits = g->bits;
+  if (word_begin) *word_begin = g->v0 / 32;
+  if (nwords_own) *nwords_own = (g->n + 31) / 32;
+  if (nwords_total) *nwords_total = (g->n_global + 31) / 32;
+  return LMATCH_OK;
+}
+
+int lmatch_part_compact(lmatch_graph* g, void* stream, int64_t* nF_local) {
+  if (!g || !g->ghost || g->part_round < 1) { set_err("lmatch_part_compact out of order"); return LMATCH_ESTATE; }
+  CK(cudaSetDevice(g->device));
+  cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
+  unsigned long long* C = g->counters;
+  const int64_t n = g->n;
+  if (g->part_round == 1) {
+    if (n > 0) {
+      lm::k_compact<true, kCompactK><<<grid_for((n + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
+          nullptr, nullptr, lm::Bins{}, nullptr, n, g->best, g->bits, g->offs, g->S[0],
+          C + lm::cnt_S(0), g->F[0], C + lm::cnt_F(0, 0), C + lm::kCntSwept, g->v0);
+      CKL();
+    }
+    g->part_cur = 0;
+    g->round_log.insert(g->round_log.end(), {g->n_nz, n, g->m});
+  } else {
+    const int cur = g->part_cur, nxt = cur ^ 1;
+    const int64_t nS = (int64_t)g->h_counters[lm::cnt_S(cur)];
+    int64_t nF = 0;
+    for (int b = 0; b < lm::kBins; ++b) nF += (int64_t)g->h_counters[lm::cnt_F(cur, b)];
+    CK(cudaMemsetAsync(C + lm::cnt_S(nxt), 0, 8 * (1 + lm::kBins), st));
+    if (nS + nF > 0) {
+      lm::k_compact<false, kCompactK>
+          <<<grid_for((nS + nF + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
+              g->S[cur], C + lm::cnt_S(cur), g->F[cur], C + lm::cnt_F(cur, 0), n, g->best, g->bits,
+              g->offs, g->S[nxt], C + lm::cnt_S(nxt), g->F[nxt], C + lm::cnt_F(nxt, 0),
+              C + lm::kCntSwept, g->v0);
+      CKL();
+    }
+    g->part_cur = nxt;
+  }
+  CK(cudaMemcpyAsync(g->h_counters, C, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  int64_t nF = 0;
+  for (int b = 0; b < lm::kBins; ++b) nF += (int64_t)g->h_counters[lm::cnt_F(g->part_cur, b)];
+  if (nF_local) *nF_local = nF;
+  return LMATCH_OK;
+}
+
+int lmatch_part_point(lmatch_graph* g, void* stream, int64_t* claim_counts) {
+  if (!g || !g->ghost || g->part_round < 1) { set_err("lmatch_part_point out of order"); return LMATCH_ESTATE; }
+  CK(cudaSetDevice(g->device));
+  cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
+  const int cur = g->part_cur;
+  int64_t nFb[lm::kBins], nF = 0;
+  for (int b = 0; b < lm::kBins; ++b) { nFb[b] = (int64_t)g->h_counters[lm::cnt_F(cur, b)]; nF += nFb[b]; }
+  const unsigned long long* cF = g->counters + lm::cnt_F(cur, 0);
+  lm::Bins& Fb = g->F[cur];
+  const lm::AdjView av = g->view();
+  if (nFb[0]) { lm::k_point_bin<1, 8><<<grid_for(nFb[0], 256, 65536), 256, 0, st>>>(Fb.list[0], cF + 0, g->offs, av, g->bits, g->best, g->v0); CKL(); }
+  if (nFb[1]) { lm::k_point_bin<8, 8><<<grid_for(nFb[1] * 8, 256, 65536), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, av, g->bits, g->best, g->v0); CKL(); }
+  if (nFb[2]) { lm::k_point_bin<32, 4><<<grid_for(nFb[2] * 32, 256, 65536), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, av, g->bits, g->best, g->v0); CKL(); }
+  if (nFb[3]) { lm::k_point_bin_cta<256, 4><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); }
+  CK(cudaMemsetAsync(g->claim_cnt, 0, (size_t)g->P * 8, st));
+  if (nF > 0) {
+    lm::Claims Cl{g->claims, g->claim_cap, g->claim_cnt, g->bounds, g->P};
+    lm::k_claims_bins<<<grid_for(nF, 256, 65536), 256, 0, st>>>(Fb, cF, g->v0, g->v0 + g->n, Cl);
+    CKL();
+  }
+  g->round_log.insert(g->round_log.end(), {nF, nF + (int64_t)g->h_counters[lm::cnt_S(cur)],
+                                           (int64_t)g->h_counters[lm::kCntSwept]});
+  ++g->part_round;
+  return part_claims_out(g, st, claim_counts);
+}
+
+int lmatch_part_finish(lmatch_graph* g, int32_t* d_mate_local, void* stream, double* w_local,
+                       int64_t* matched_local) {
+  if (!g || !g->ghost) { set_err("not a partition handle"); return LMATCH_ESTATE; }
+  CK(cudaSetDevice(g->device));
+  cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
+  if (g->n > 0) {
+    lm::k_materialize<kFinThreads><<<kFinBlocks, kFinThreads, 0, st>>>(g->best, g->bits, g->n, g->v0,
+                                                                       d_mate_local, g->pw, g->pc);
+    CKL();
+    lm::k_final_sum<<<1, 32, 0, st>>>(g->pw, g->pc, kFinBlocks, g->res_w, g->res_c);
+    CKL();
+    CK(cudaMemcpyAsync(g->h_res, g->res_w, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(g->h_resc, g->res_c, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+  } else {
+    g->h_res[0] = 0.0;
+    g->h_resc[0] = 0;
+  }
+  if (w_local) *w_local = g->h_res[0];
+  if (matched_local) *matched_local = g->h_resc[0];
+  return LMATCH_OK;
+}
+
+int lmatch_part_get_claims(const lmatch_graph* g, int32_t part, uint64_t* d_dst, void* stream) {
+  if (!g || !g->ghost || part < 0 || part >= g->P) { set_err("bad handle or part"); return LMATCH_ESTATE; }
+  CK(cudaSetDevice(g->device));
+  const int64_t c = (int64_t)g->h_claim_cnt[part];
+  if (c > 0)
+    CK(cudaMemcpyAsync(d_dst, g->claims + (int64_t)part * g->claim_cap, (size_t)c * 8,
+                       cudaMemcpyDeviceToDevice, stream ? (cudaStream_t)stream : g->stream));
+  return LMATCH_OK;
+}
+
+int lmatch_part_get_bits(const lmatch_graph* g, uint32_t* d_dst, void* stream) {
+  if (!g || !g->ghost) { set_err("not a partition handle"); return LMATCH_ESTATE; }
+  CK(cudaSetDevice(g->device));
+  const int64_t nw = (g->n + 31) / 32;
+  if (nw > 0)
+    CK(cudaMemcpyAsync(d_dst, g->bits + g->v0 / 32, (size_t)nw * 4, cudaMemcpyDeviceToDevice,
+                       stream ? (cudaStream_t)stream : g->stream));
+  return LMATCH_OK;
+}
+
+int lmatch_part_set_bits(lmatch_graph* g, const uint32_t* d_src, int64_t word_begin, int64_t nwords,
+                         void* stream) {
+  if (!g || !g->ghost) { set_err("not a partition handle"); return LMATCH_ESTATE; }
+  if (word_begin < 0 || word_begin + nwords > (g->n_global + 31) / 32) { set_err("word range"); return LMATCH_EINVAL; }
+  CK(cudaSetDevice(g->device));
+  if (nwords > 0)
+    CK(cudaMemcpyAsync(g->bits + word_begin, d_src, (size_t)nwords * 4, cudaMemcpyDeviceToDevice,
+                       stream ? (cudaStream_t)stream : g->stream));
+  return LMATCH_OK;
+}
+
 }  // extern "C"
+

@@ -1,0 +1,339 @@
+"""Partitioned (multi-GPU) matching: 1-D vertex partition, pointer claims and a bitmap allgather.
+
+SURVEY 8(e) / include/lmatch.h "Partitioned mode".  Every part owns a contiguous vertex range with
+all its rows, balanced by directed entries (binary search on the CSR prefix sums).
+One round (Alg. 2, with the exchange redesigned):
+
+    pointers (owned rows)           lmatch_part_begin / lmatch_part_point    [library kernels]
+    claims -> owner of the target   all-to-all      (replaces nccl_AllReduce(pointers))
+    match                           lmatch_part_apply                        [library kernels]
+    matched-bitmap slices           allgather       (replaces nccl_AllReduce(mate))
+    compaction, frontier size       lmatch_part_compact                      [library kernels]
+    termination                     allreduce of frontier sizes == 0
+
+The round loop (`run_parts`) is written over a list of local parts and a transport:
+  * `TorchTransport` -- one part per process, torch.distributed collectives (NCCL on GPUs; the
+    same calls run on gloo with CPU tensors, which is how the CPU tests cover this driver);
+  * `LocalTransport` -- several parts in one process (P logical partitions on one GPU), used to
+    prove partition invariance of the result on a single device.
+Data moves between parts only through the transport; the result is bit-identical to the
+single-GPU run for every partition (Lemma III.1).
+"""
+from __future__ import annotations
+
+import ctypes
+from dataclasses import dataclass
+
+import numpy as np
+
+from . import _check, _dev_ptr, _lib, _P, _I64, make_opts, LMatchError  # noqa: F401
+
+# ---------------------------------------------------------------------------- ctypes signatures
+_sig = {
+    "lmatch_create_part": ([_P, _P, _P, _I64, _I64, _I64, _I64, ctypes.c_int32, _P, _P,
+                            ctypes.POINTER(_P)], ctypes.c_int),
+    "lmatch_create_part_device": ([_P, _P, _P, _I64, _I64, _I64, _I64, ctypes.c_int32, _P, _P, _P,
+                                   ctypes.POINTER(_P)], ctypes.c_int),
+    "lmatch_part_begin": ([_P, _P, _P], ctypes.c_int),
+    "lmatch_part_claims": ([_P, _P], ctypes.c_int),
+    "lmatch_part_apply": ([_P, _P, _I64, _P], ctypes.c_int),
+    "lmatch_part_bitmap": ([_P, _P, _P, _P, _P], ctypes.c_int),
+    "lmatch_part_compact": ([_P, _P, ctypes.POINTER(_I64)], ctypes.c_int),
+    "lmatch_part_point": ([_P, _P, _P], ctypes.c_int),
+    "lmatch_part_finish": ([_P, _P, _P, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(_I64)],
+                           ctypes.c_int),
+    "lmatch_part_get_claims": ([_P, ctypes.c_int32, _P, _P], ctypes.c_int),
+    "lmatch_part_get_bits": ([_P, _P, _P], ctypes.c_int),
+    "lmatch_part_set_bits": ([_P, _P, _I64, _I64, _P], ctypes.c_int),
+    "lmatch_part_info": ([_P, ctypes.POINTER(_I64), ctypes.POINTER(ctypes.c_double)], ctypes.c_int),
+    "lmatch_reload": ([_P, _P, _P, _P], ctypes.c_int),
+}
+for _name, (_args, _res) in _sig.items():
+    _f = getattr(_lib, _name)
+    _f.argtypes = _args
+    _f.restype = _res
+
+
+# ------------------------------------------------------------------------------- partitioning
+def edge_balanced_bounds(offsets: np.ndarray, nparts: int, align: int = 32) -> np.ndarray:
+    """Contiguous vertex ranges with ~m/P directed entries each (binary search on the CSR prefix
+    sums); every bound is a multiple of `align` (bitmap words are owned by one part)."""
+    offsets = np.asarray(offsets, dtype=np.int64)
+    n = offsets.shape[0] - 1
+    m = int(offsets[-1])
+    b = np.zeros(nparts + 1, dtype=np.int64)
+    for p in range(1, nparts):
+        v = int(np.searchsorted(offsets, (m * p) // nparts, side="left"))
+        v = min(n, (v + align - 1) // align * align)
+        b[p] = max(b[p - 1], v)
+    b[nparts] = n
+    return b
+
+
+def part_words(bounds):
+    """(first bitmap word, word count) owned by each part."""
+    return [(int(bounds[p]) // 32, (int(bounds[p + 1]) - int(bounds[p]) + 31) // 32)
+            for p in range(len(bounds) - 1)]
+
+
+def local_csr(offsets, col, w, v0: int, v1: int):
+    """Rows [v0, v1) with their global column ids (cut edges live in both owners' rows)."""
+    offsets = np.asarray(offsets, dtype=np.int64)
+    s, e = int(offsets[v0]), int(offsets[v1])
+    return offsets[v0:v1 + 1] - s, np.asarray(col[s:e], dtype=np.int32), np.asarray(w[s:e], dtype=np.float32)
+
+
+# --------------------------------------------------------------------------------- transports
+class LocalTransport:
+    """All parts live in this process (P logical partitions, e.g. on one GPU)."""
+
+    def __init__(self, nparts: int):
+        self.nparts = nparts
+
+    def exchange(self, sends):
+        import torch
+        P = self.nparts
+        return [torch.cat([sends[s][d] for s in range(P)]) for d in range(P)]
+
+    def allgather(self, owns):
+        return [list(owns) for _ in owns]
+
+    def allreduce(self, xs):
+        t = sum(int(x) for x in xs)
+        return [t for _ in xs]
+
+
+class TorchTransport:
+    """One part per process; torch.distributed collectives (NCCL with CUDA tensors, gloo with
+    CPU tensors).  Every rank calls every method in the same order."""
+
+    def __init__(self, group=None):
+        import torch.distributed as dist
+        self.dist = dist
+        self.group = group
+        self.nparts = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        self._sizes = None  # owned bitmap word counts of every part (constant per run)
+
+    def exchange(self, sends):
+        import torch
+        (send,) = sends
+        dev = send[0].device
+        cnt_out = torch.tensor([t.numel() for t in send], dtype=torch.int64, device=dev)
+        cnt_in = torch.empty_like(cnt_out)
+        self.dist.all_to_all_single(cnt_in, cnt_out, group=self.group)
+        in_splits = [t.numel() for t in send]
+        out_splits = [int(c) for c in cnt_in.tolist()]
+        recv = torch.empty(sum(out_splits), dtype=send[0].dtype, device=dev)
+        self.dist.all_to_all_single(recv, torch.cat(list(send)), out_splits, in_splits,
+                                    group=self.group)
+        return [recv]
+
+    def allgather(self, owns):
+        import torch
+        (own,) = owns
+        if self._sizes is None:
+            n = torch.tensor([own.numel()], dtype=torch.int64, device=own.device)
+            sz = [torch.empty_like(n) for _ in range(self.nparts)]
+            self.dist.all_gather(sz, n, group=self.group)
+            self._sizes = [int(x.item()) for x in sz]
+        sizes = self._sizes
+        mx = max(sizes) if sizes else 0
+        pad = torch.zeros(mx, dtype=own.dtype, device=own.device)
+        pad[: own.numel()] = own
+        out = torch.empty(self.nparts * mx, dtype=own.dtype, device=own.device)
+        self.dist.all_gather_into_tensor(out, pad, group=self.group)
+        return [[out[p * mx: p * mx + sizes[p]] for p in range(self.nparts)]]
+
+    def allreduce(self, xs):
+        import torch
+        (x,) = xs
+        dev = "cuda" if self.dist.get_backend(self.group) == "nccl" else "cpu"
+        t = torch.tensor([int(x)], dtype=torch.int64, device=dev)
+        self.dist.all_reduce(t, group=self.group)
+        return [int(t.item())]
+
+
+# ------------------------------------------------------------------------- the GPU part backend
+class LibPart:
+    """One partition handle of liblmatch.so (rows [v0, v1) of a graph with n_global vertices)."""
+
+    def __init__(self, offsets_local, col_local, w_local, v0: int, n_global: int, bounds,
+                 part: int, device=None, stream=None, validate_level: int = 1, timing: bool = False):
+        import torch
+        self.torch = torch
+        self.dev = torch.device("cuda") if device is None else torch.device(device)
+        self.bounds = np.ascontiguousarray(bounds, dtype=np.int64)
+        self.P = self.bounds.shape[0] - 1
+        self.v0 = int(v0)
+        self.part = int(part)
+        self.n_local = int(len(offsets_local) - 1)
+        self.n_global = int(n_global)
+        self.stream = stream
+        h = _P()
+        opts = make_opts(validate_level=validate_level, timing=timing)
+        if hasattr(offsets_local, "is_cuda") and offsets_local.is_cuda:  # device CSR (torch)
+            self.m_local = int(col_local.numel())
+            with torch.cuda.device(self.dev):
+                _check(_lib.lmatch_create_part_device(
+                    offsets_local.data_ptr(), col_local.data_ptr(), w_local.data_ptr(), self.n_local,
+                    self.m_local, self.v0, self.n_global, self.P, self.bounds.ctypes.data,
+                    ctypes.byref(opts), self._s(), ctypes.byref(h)), "lmatch_create_part_device")
+        else:
+            off = np.ascontiguousarray(offsets_local, dtype=np.int64)
+            col = np.ascontiguousarray(col_local, dtype=np.int32)
+            w = np.ascontiguousarray(w_local, dtype=np.float32)
+            self.m_local = int(col.shape[0])
+            with torch.cuda.device(self.dev):
+                _check(_lib.lmatch_create_part(off.ctypes.data, col.ctypes.data, w.ctypes.data,
+                                               self.n_local, self.m_local, self.v0, self.n_global,
+                                               self.P, self.bounds.ctypes.data, ctypes.byref(opts),
+                                               ctypes.byref(h)), "lmatch_create_part")
+        self.h = h.value
+        self.counts = np.zeros(self.P, dtype=np.int64)
+        self.words = part_words(self.bounds)
+
+    def _s(self):
+        return None if self.stream is None else self.stream.cuda_stream
+
+    def begin(self):
+        _check(_lib.lmatch_part_begin(self.h, self._s(), self.counts.ctypes.data), "lmatch_part_begin")
+        return self.counts.copy()
+
+    def point(self):
+        _check(_lib.lmatch_part_point(self.h, self._s(), self.counts.ctypes.data), "lmatch_part_point")
+        return self.counts.copy()
+
+    def claims(self, counts):
+        torch = self.torch
+        out = []
+        for p in range(self.P):
+            t = torch.empty(int(counts[p]), dtype=torch.int64, device=self.dev)
+            if counts[p]:
+                _check(_lib.lmatch_part_get_claims(self.h, p, t.data_ptr(), self._s()),
+                       "lmatch_part_get_claims")
+            out.append(t)
+        return out
+
+    def apply(self, recv):
+        _check(_lib.lmatch_part_apply(self.h, recv.data_ptr() if recv.numel() else None,
+                                      recv.numel(), self._s()), "lmatch_part_apply")
+
+    def own_bits(self):
+        t = self.torch.empty(self.words[self._me()][1], dtype=self.torch.int32, device=self.dev)
+        if t.numel():
+            _check(_lib.lmatch_part_get_bits(self.h, t.data_ptr(), self._s()), "lmatch_part_get_bits")
+        return t
+
+    def set_bits(self, all_words):
+        for p, t in enumerate(all_words):
+            if p == self._me() or t.numel() == 0:
+                continue
+            src = t.to(self.dev).contiguous()
+            _check(_lib.lmatch_part_set_bits(self.h, src.data_ptr(), self.words[p][0], src.numel(),
+                                             self._s()), "lmatch_part_set_bits")
+
+    def reload(self, offsets_local, col_local, w_local):
+        """Re-upload the same-shaped local CSR from host arrays (end-to-end timing)."""
+        ptrs = [a.ctypes.data if isinstance(a, np.ndarray) else int(a)
+                for a in (offsets_local, col_local, w_local)]
+        _check(_lib.lmatch_reload(self.h, *ptrs), "lmatch_reload")
+
+    def info(self):
+        r, ms = _I64(), ctypes.c_double()
+        _check(_lib.lmatch_part_info(self.h, ctypes.byref(r), ctypes.byref(ms)), "lmatch_part_info")
+        return int(r.value), float(ms.value)
+
+    def compact(self):
+        nf = _I64()
+        _check(_lib.lmatch_part_compact(self.h, self._s(), ctypes.byref(nf)), "lmatch_part_compact")
+        return int(nf.value)
+
+    def finish(self):
+        torch = self.torch
+        mate = torch.empty(max(self.n_local, 1), dtype=torch.int32, device=self.dev)
+        w, c = ctypes.c_double(), _I64()
+        _check(_lib.lmatch_part_finish(self.h, mate.data_ptr(), self._s(), ctypes.byref(w),
+                                       ctypes.byref(c)), "lmatch_part_finish")
+        return mate[: self.n_local], float(w.value), int(c.value)
+
+    def _me(self):
+        return self.part
+
+    def close(self):
+        if self.h is not None:
+            _lib.lmatch_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+# ----------------------------------------------------------------------------- the round loop
+@dataclass
+class PartResult:
+    mates: list          # per local part: mate[] of its owned range (global ids)
+    weight: float        # w(M) over ALL parts (fp64)
+    matched: int         # matched vertices over all parts
+    rounds: int          # pointing phases executed
+    exchanged_claims: int  # claims sent by the local parts (all rounds)
+
+
+def run_parts(parts, transport) -> PartResult:
+    """Drive the rounds for the local `parts` (all parts with LocalTransport, one with
+    TorchTransport).  Part objects implement begin/point/claims/apply/own_bits/set_bits/compact/
+    finish (LibPart on GPUs; tests/dist_model.py on CPU)."""
+    counts = [p.begin() for p in parts]
+    rounds = 1
+    sent = 0
+    while True:
+        sends = [p.claims(c) for p, c in zip(parts, counts)]
+        sent += sum(int(np.sum(c)) for c in counts)
+        recvs = transport.exchange(sends)
+        for p, r in zip(parts, recvs):
+            p.apply(r)
+        alls = transport.allgather([p.own_bits() for p in parts])
+        for p, a in zip(parts, alls):
+            p.set_bits(a)
+        nF = transport.allreduce([p.compact() for p in parts])[0]
+        if nF == 0:
+            break
+        rounds += 1
+        counts = [p.point() for p in parts]
+    fin = [p.finish() for p in parts]
+    w = transport_sum_float(transport, [f[1] for f in fin])
+    c = transport.allreduce([f[2] for f in fin])[0]
+    return PartResult([f[0] for f in fin], w, c, rounds, sent)
+
+
+def transport_sum_float(transport, xs):
+    """fp64 sum over all parts (deterministic: gathered then summed in part order)."""
+    if isinstance(transport, LocalTransport):
+        return float(sum(xs))
+    import torch
+    (x,) = xs
+    dev = "cuda" if transport.dist.get_backend(transport.group) == "nccl" else "cpu"
+    t = torch.tensor([x], dtype=torch.float64, device=dev)
+    out = [torch.empty_like(t) for _ in range(transport.nparts)]
+    transport.dist.all_gather(out, t, group=transport.group)
+    return float(sum(float(o.item()) for o in out))
+
+
+def match_partitioned_local(offsets, col, w, nparts: int, device=None):
+    """P logical partitions of one graph on one device (LocalTransport).  Returns (mate, result)."""
+    offsets = np.asarray(offsets, dtype=np.int64)
+    n = offsets.shape[0] - 1
+    bounds = edge_balanced_bounds(offsets, nparts)
+    parts = []
+    for p in range(nparts):
+        v0, v1 = int(bounds[p]), int(bounds[p + 1])
+        lo, lc, lw = local_csr(offsets, col, w, v0, v1)
+        parts.append(LibPart(lo, lc, lw, v0, n, bounds, p, device=device))
+    res = run_parts(parts, LocalTransport(nparts))
+    mate = np.concatenate([m.cpu().numpy() for m in res.mates]) if n else np.zeros(0, np.int32)
+    for p in parts:
+        p.close()
+    return mate, res

@@ -1,0 +1,104 @@
+"""N>1 path on CPU: the product driver (paper_conf_sc_mandulakgfhs24_b200.dist.run_parts) with the
+numpy partition model, over (a) the in-process LocalTransport and (b) torch.distributed gloo with
+world_size 2 and 3 (TorchTransport, the same class the NCCL runs use).  The result must equal the
+oracle's unique matching for every partition (Lemma III.1)."""
+import math
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import graphgen
+import oracle
+from dist_model import NumpyPart
+
+dist_mod = pytest.importorskip("paper_conf_sc_mandulakgfhs24_b200.dist")
+
+
+def build_parts(g, P):
+    b = dist_mod.edge_balanced_bounds(g.offsets, P)
+    parts = []
+    for p in range(P):
+        lo, lc, lw = dist_mod.local_csr(g.offsets, g.col, g.w, int(b[p]), int(b[p + 1]))
+        parts.append(NumpyPart(lo, lc, lw, int(b[p]), g.n, b, p))
+    return b, parts
+
+
+def test_edge_balanced_bounds():
+    g = graphgen.rmat(12, 16, seed=3)
+    for P in (1, 2, 3, 4, 8):
+        b = dist_mod.edge_balanced_bounds(g.offsets, P)
+        assert b[0] == 0 and b[-1] == g.n and (np.diff(b) >= 0).all()
+        assert all(x % 32 == 0 for x in b[:-1])
+        per = np.diff(g.offsets[b])
+        assert per.max() <= g.m / P + 32 * g.degrees().max() + 1
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 5])
+def test_local_transport_numpy_model(P):
+
+    graphs = [graphgen.rmat(9, 8, seed=P), graphgen.er(600, 5.0, seed=P, weights="paper"),
+              graphgen.mesh(20, keep=0.7, seed=P, weights="ones")]
+    for g in graphs:
+        _, parts = build_parts(g, P)
+        res = dist_mod.run_parts(parts, dist_mod.LocalTransport(P))
+        mate = np.concatenate([m.numpy() for m in res.mates])
+        ref = oracle.greedy(g)
+        np.testing.assert_array_equal(mate, ref.mate)
+        _, ph, _ = oracle.ld_frontier(g)
+        assert res.rounds == ph
+        assert math.isclose(res.weight, ref.weight, rel_tol=1e-9)
+        assert res.matched == 2 * ref.cardinality
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, spec, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        kind, args = spec
+        g = getattr(graphgen, kind)(*args)
+        b = dist_mod.edge_balanced_bounds(g.offsets, world)
+        lo, lc, lw = dist_mod.local_csr(g.offsets, g.col, g.w, int(b[rank]), int(b[rank + 1]))
+        part = NumpyPart(lo, lc, lw, int(b[rank]), g.n, b, rank)
+        res = dist_mod.run_parts([part], dist_mod.TorchTransport())
+        q.put((rank, res.mates[0].numpy(), res.weight, res.matched, res.rounds))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,spec", [(2, ("rmat", (10, 8, 2))), (3, ("er", (700, 6.0, 3))),
+                                        (2, ("mesh", (24, 0.6, 4)))])
+def test_gloo_torchtransport(world, spec):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, spec, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    out = [q.get(timeout=120) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    out.sort(key=lambda x: x[0])
+    mate = np.concatenate([o[1] for o in out])
+    kind, args = spec
+    g = getattr(graphgen, kind)(*args)
+    ref = oracle.greedy(g)
+    np.testing.assert_array_equal(mate, ref.mate)
+    for o in out:
+        assert math.isclose(o[2], ref.weight, rel_tol=1e-9)
+        assert o[3] == 2 * ref.cardinality
+        assert o[4] == oracle.ld_frontier(g)[1]
