@@ -84,7 +84,13 @@ typedef struct lmatch_opts {
                                  buffering) and read zero-copy by later rounds */
   int64_t stream_chunk;       /* entries per streamed chunk (0 = default 2^24; rounded to the
                                  sweep tile) */
-  int32_t reserved[12];
+  int32_t round_loop;         /* 0 = default, hybrid: work-sized per-round launches while the
+                                 frontier is large, then ONE persistent cooperative kernel runs all
+                                 remaining rounds (grid barriers between phases, no host round
+                                 trips); 1 = host-driven per-round launches only; 2 = persistent
+                                 kernel for every round after round 1; 3 = CUDA graph {round 1,
+                                 persistent kernel}.  Out-of-core: 3 behaves as 2. */
+  int32_t reserved[11];
 } lmatch_opts;
 
 /* Filled by lmatch_run / lmatch_run_device when non-NULL. */

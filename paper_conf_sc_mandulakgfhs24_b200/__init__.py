@@ -43,7 +43,7 @@ class Opts(ctypes.Structure):
         ("validate_level", ctypes.c_int32), ("timing", ctypes.c_int32),
         ("max_rounds", ctypes.c_int64), ("upload_chunk", ctypes.c_int64),
         ("hbm_budget_bytes", ctypes.c_int64), ("stream_chunk", ctypes.c_int64),
-        ("reserved", ctypes.c_int32 * 12),
+        ("round_loop", ctypes.c_int32), ("reserved", ctypes.c_int32 * 11),
     ]
 
 
@@ -238,7 +238,8 @@ class Matcher:
 
     def __init__(self, offsets=None, col=None, w=None, *, handle: int | None = None,
                  validate_level: int = 1, timing: bool = False, upload_chunk: int = 0,
-                 max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0):
+                 max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
+                 round_loop: int = 0):
         self.h = None
         if handle is not None:
             self.h = handle
@@ -247,7 +248,8 @@ class Matcher:
                 offsets, col, w = offsets.offsets, offsets.col, offsets.w
             self.h = lmatch_create_ex(offsets, col, w,
                                       opts=make_opts(validate_level, timing, upload_chunk,
-                                                     max_rounds, hbm_budget_bytes, stream_chunk))
+                                                     max_rounds, hbm_budget_bytes, stream_chunk,
+                                                     round_loop))
         self.info = lmatch_info(self.h)
 
     @classmethod
@@ -289,8 +291,11 @@ class Matcher:
 
 
 def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int = 0,
-              max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0) -> Opts:
+              max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
+              round_loop: int = 0) -> Opts:
+    """round_loop: 0 = device-driven rounds in a CUDA graph (default), 1 = host-driven."""
     o = Opts()
+    o.round_loop = int(round_loop)
     o.hbm_budget_bytes = int(hbm_budget_bytes)
     o.stream_chunk = int(stream_chunk)
     o.validate_level = int(validate_level)

@@ -18,10 +18,13 @@
 //   F[b]   int32[]           frontier (vertices whose target was matched), binned by degree
 #pragma once
 #include <cstdint>
+#include <cooperative_groups.h>
 #include <cuda.h>
 #include <cuda_runtime.h>
 
 namespace lm {
+
+namespace cg = cooperative_groups;
 
 constexpr int kBins = 4;               // frontier degree bins
 constexpr int kBinDeg0 = 8, kBinDeg1 = 64, kBinDeg2 = 2048;  // bins: G = 1, 8, 32 lanes, CTA
@@ -809,6 +812,26 @@ struct Bins {
   ulonglong2* list[kBins];
 };
 
+// Device-resident round bookkeeping, so the round loop needs no host decision: the same launch
+// sequence runs host-driven or as a captured CUDA graph with a conditional WHILE node.
+struct RoundState {
+  int cur;               // index of the set holding the current live pairs S and frontier F
+  int cont;              // 1 = another round follows (host-driven mode reads it)
+  long long rounds;      // pointing phases executed (round 1 = the sweep)
+  long long max_rounds;
+  long long ftot;        // sum of frontier sizes over rounds >= 2
+  long long log_len;     // rows written to the per-round log
+  long long log_cap;
+  unsigned long long swept_prev;
+};
+struct RoundArgs {
+  uint64_t* S[2];
+  Bins F[2];
+  unsigned long long* cnt;  // kNumCounters; set s = cnt_S(s), cnt_F(s, b)
+  RoundState* st;
+  long long* log;           // [log_cap][3]: |F_r|, |S_r| + |F_r|, E(F_r)
+};
+
 // A2 pointer phase on the frontier (rounds >= 2): G lanes per vertex (degree-binned).
 //   best[u] = max{ adj[j] : j in row(u), !matched(col) }   (Alg. 3 L5-8)
 // Keys are loaded U at a time per lane and the bitmap words of the candidates (keys above the
@@ -839,16 +862,16 @@ __device__ __forceinline__ uint64_t scan_row_available(const AdjView adj,
 }
 
 template <int G, int U>
-__global__ void k_point_bin(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
-                            const int64_t* __restrict__ offs, const AdjView adj,
-                            const uint32_t* __restrict__ bits, uint64_t* __restrict__ best,
-                            int64_t vbase) {
-  const int64_t cnt = (int64_t)*cnt_ptr;
+__device__ __forceinline__ void point_bin_body(ulonglong2* __restrict__ list, int64_t cnt,
+                                               const int64_t* __restrict__ offs, const AdjView adj,
+                                               const uint32_t* __restrict__ bits,
+                                               uint64_t* __restrict__ best, int64_t vbase,
+                                               int64_t gtid, int64_t gthreads) {
   const int lane = threadIdx.x & 31;
   const int gl = lane & (G - 1);
   const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
-  const int64_t ng = ((int64_t)gridDim.x * blockDim.x) / G;
-  for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) / G; i < cnt; i += ng) {
+  const int64_t ng = gthreads / G;
+  for (int64_t i = gtid / G; i < cnt; i += ng) {
     const ulonglong2 e = list[i];
     int64_t s, en;
     row_range(e, offs, vbase, &s, &en);
@@ -860,15 +883,25 @@ __global__ void k_point_bin(ulonglong2* __restrict__ list, const unsigned long l
     }
   }
 }
+template <int G, int U>
+__global__ void k_point_bin(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
+                            const int64_t* __restrict__ offs, const AdjView adj,
+                            const uint32_t* __restrict__ bits, uint64_t* __restrict__ best,
+                            int64_t vbase) {
+  point_bin_body<G, U>(list, (int64_t)*cnt_ptr, offs, adj, bits, best, vbase,
+                       (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
+                       (int64_t)gridDim.x * blockDim.x);
+}
 
 template <int THREADS, int U>
-__global__ void __launch_bounds__(THREADS)
-    k_point_bin_cta(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
-                    const int64_t* __restrict__ offs, const AdjView adj,
-                    const uint32_t* __restrict__ bits, uint64_t* __restrict__ best, int64_t vbase) {
+__device__ __forceinline__ void point_bin_cta_body(ulonglong2* __restrict__ list, int64_t cnt,
+                                                   const int64_t* __restrict__ offs,
+                                                   const AdjView adj,
+                                                   const uint32_t* __restrict__ bits,
+                                                   uint64_t* __restrict__ best, int64_t vbase,
+                                                   int64_t bid, int64_t nblk) {
   __shared__ uint64_t red[THREADS / 32];
-  const int64_t cnt = (int64_t)*cnt_ptr;
-  for (int64_t i = blockIdx.x; i < cnt; i += gridDim.x) {
+  for (int64_t i = bid; i < cnt; i += nblk) {
     const ulonglong2 e = list[i];
     int64_t s, en;
     row_range(e, offs, vbase, &s, &en);
@@ -887,6 +920,14 @@ __global__ void __launch_bounds__(THREADS)
     }
     __syncthreads();
   }
+}
+template <int THREADS, int U>
+__global__ void __launch_bounds__(THREADS)
+    k_point_bin_cta(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
+                    const int64_t* __restrict__ offs, const AdjView adj,
+                    const uint32_t* __restrict__ bits, uint64_t* __restrict__ best, int64_t vbase) {
+  point_bin_cta_body<THREADS, U>(list, (int64_t)*cnt_ptr, offs, adj, bits, best, vbase, blockIdx.x,
+                                 gridDim.x);
 }
 
 // =============================================================================================
@@ -915,10 +956,9 @@ __global__ void k_match_all(const uint64_t* __restrict__ best, int64_t n, uint32
 
 // Rounds >= 2: over the frontier's new pointers (pairs in the bins).  A new mutual pair has at
 // least one endpoint that re-pointed this round (R3); that endpoint marks both.
-__global__ void k_match_bins(Bins F, const unsigned long long* cntF,
-                             const uint64_t* __restrict__ best, uint32_t* bits) {
-  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+__device__ __forceinline__ void match_bins_body(const Bins& F, const unsigned long long* cntF,
+                                                const uint64_t* __restrict__ best, uint32_t* bits,
+                                                int64_t tid, int64_t stride) {
 #pragma unroll
   for (int bb = 0; bb < kBins; ++bb) {
     const int64_t c = (int64_t)cntF[bb];
@@ -934,6 +974,11 @@ __global__ void k_match_bins(Bins F, const unsigned long long* cntF,
     }
   }
 }
+__global__ void k_match_bins(Bins F, const unsigned long long* cntF,
+                             const uint64_t* __restrict__ best, uint32_t* bits) {
+  match_bins_body(F, cntF, best, bits, (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
+                  (int64_t)gridDim.x * blockDim.x);
+}
 
 // =============================================================================================
 // A6 frontier compaction (not in the paper, which rescans every unmatched vertex).
@@ -945,14 +990,44 @@ __global__ void k_match_bins(Bins F, const unsigned long long* cntF,
 // accesses are two bitmap bits (L2-resident) and, for frontier members only, deg(u).  Each warp
 // owns a chunk of 32*K items: ONE atomicAdd per output list per warp reserves its ranges.
 // =============================================================================================
+// Set `in` (S and frontier bins) is read (ignored when ALL), set `out` is written.
+struct CompactIO {
+  const uint64_t* S;
+  Bins Fin;
+  uint64_t* Sout;
+  Bins Fout;
+  const unsigned long long* cin;  // counters of the input set (cnt_S .. cnt_F(.,3) contiguous)
+  unsigned long long* cout;       // counters of the output set
+  unsigned long long* swept;
+};
+__host__ __device__ inline CompactIO compact_io(const RoundArgs& a, int cur) {
+  CompactIO io;
+  io.S = a.S[cur];
+  io.Fin = a.F[cur];
+  io.Sout = a.S[cur ^ 1];
+  io.Fout = a.F[cur ^ 1];
+  io.cin = a.cnt + cnt_S(cur);
+  io.cout = a.cnt + cnt_S(cur ^ 1);
+  io.swept = a.cnt + kCntSwept;
+  return io;
+}
+
 template <bool ALL, int K>
-__global__ void __launch_bounds__(256)
-    k_compact(const uint64_t* __restrict__ S, const unsigned long long* cntS, Bins Fin,
-              const unsigned long long* cntFin, int64_t n, const uint64_t* __restrict__ best,
-              const uint32_t* __restrict__ bits, const int64_t* __restrict__ offs,
-              uint64_t* __restrict__ Sout, unsigned long long* cntSout, Bins Fout,
-              unsigned long long* cntFout, unsigned long long* swept, int64_t vbase) {
-  constexpr int NW = 8, NL = 1 + kBins;  // warps per block (blockDim 256), output lists
+__device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
+                                             const uint64_t* __restrict__ best,
+                                             const uint32_t* __restrict__ bits,
+                                             const int64_t* __restrict__ offs, int64_t vbase,
+                                             int64_t bid, int64_t nblk) {
+  constexpr int NW = 8, NL = 1 + kBins;  // blockDim must be 256
+  const uint64_t* __restrict__ S = io.S;
+  const unsigned long long* cntS = io.cin;
+  const Bins& Fin = io.Fin;
+  const unsigned long long* cntFin = io.cin + 1;
+  uint64_t* __restrict__ Sout = io.Sout;
+  unsigned long long* cntSout = io.cout;
+  const Bins& Fout = io.Fout;
+  unsigned long long* cntFout = io.cout + 1;
+  unsigned long long* swept = io.swept;  // warps per block (blockDim 256), output lists
   __shared__ unsigned wtot[NW][NL];
   __shared__ unsigned long long wbase[NW][NL];
   // virtual concatenation S ++ F_0 ++ F_1 ++ F_2 ++ F_3 (prefix ends p0 < p1 < ... < p4)
@@ -965,7 +1040,7 @@ __global__ void __launch_bounds__(256)
   const unsigned lt = lanemask_lt();
   constexpr int64_t BLK = (int64_t)NW * 32 * K;
   unsigned long long degsum = 0;
-  for (int64_t cb = (int64_t)blockIdx.x * BLK; cb < cnt; cb += (int64_t)gridDim.x * BLK) {
+  for (int64_t cb = bid * BLK; cb < cnt; cb += nblk * BLK) {
     const int64_t c0 = cb + (int64_t)warp * 32 * K;
     uint32_t sbits = 0, fb0 = 0, fb1 = 0, fb2 = 0, fb3 = 0;
     uint64_t pr[K], rr[K];
@@ -1072,6 +1147,102 @@ __global__ void __launch_bounds__(256)
   }
   for (int o = 16; o; o >>= 1) degsum += __shfl_xor_sync(0xffffffffu, degsum, o);
   if (lane == 0 && degsum) atomicAdd(swept, degsum);
+}
+template <bool ALL, int K>
+__global__ void __launch_bounds__(256)
+    k_compact(CompactIO io, int64_t n, const uint64_t* __restrict__ best,
+              const uint32_t* __restrict__ bits, const int64_t* __restrict__ offs, int64_t vbase) {
+  compact_body<ALL, K>(io, n, best, bits, offs, vbase, blockIdx.x, gridDim.x);
+}
+
+// =============================================================================================
+// Round bookkeeping on the device (termination; R6)
+// =============================================================================================
+__global__ void k_round_init(RoundState* st, long long max_rounds, long long log_cap,
+                             long long first_rounds) {
+  st->cur = 1;  // round 1's compaction (ALL) writes set 0 = cur ^ 1
+  st->cont = 0;
+  st->rounds = first_rounds;
+  st->max_rounds = max_rounds;
+  st->ftot = 0;
+  st->log_len = 0;
+  st->log_cap = log_cap;
+  st->swept_prev = 0;
+}
+// After a compaction: the output set becomes current; decide whether another round runs.
+// `graph_handle` != 0: running inside a CUDA graph -> set the WHILE node's condition.
+__device__ __forceinline__ int end_round_body(const RoundArgs* __restrict__ ra, long long first_log_rows) {
+  RoundState* st = ra->st;
+  const int cur = st->cur ^ 1;
+  st->cur = cur;
+  unsigned long long nF = 0;
+#pragma unroll
+  for (int b = 0; b < kBins; ++b) nF += ra->cnt[cnt_F(cur, b)];
+  const unsigned long long nS = ra->cnt[cnt_S(cur)];
+  const int cont = nF > 0 && st->rounds < st->max_rounds;
+  // zero the counters of the set the next compaction writes
+#pragma unroll
+  for (int q = 0; q < 1 + kBins; ++q) ra->cnt[cnt_S(cur ^ 1) + q] = 0ull;
+  if (cont) {
+    ++st->rounds;
+    st->ftot += (long long)nF;
+    const unsigned long long sw = ra->cnt[kCntSwept];
+    if (st->log_len < st->log_cap) {
+      long long* row = ra->log + 3 * (first_log_rows + st->log_len);
+      row[0] = (long long)nF;
+      row[1] = (long long)(nS + nF);
+      row[2] = (long long)(sw - st->swept_prev);
+      ++st->log_len;
+    }
+    st->swept_prev = sw;
+  }
+  st->cont = cont;
+  return cont;
+}
+__global__ void k_end_round(const RoundArgs* __restrict__ ra, cudaGraphConditionalHandle handle, int in_graph,
+                            long long first_log_rows) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  const int cont = end_round_body(ra, first_log_rows);
+  if (in_graph) cudaGraphSetConditional(handle, (unsigned)cont);
+}
+
+// All rounds >= 2 in ONE cooperative launch (grid = co-resident blocks): pointer phase (every
+// degree bin) | grid barrier | match | barrier | compaction | barrier | end of round | barrier.
+// No per-round launches or host decisions; the grid barrier's fence also invalidates L1, so
+// every phase reads the others' writes.
+template <int B0G, int B0U, int B1G, int B1U, int B2G, int B2U, int K>
+__global__ void __launch_bounds__(256)
+    k_rounds_persistent(const RoundArgs* __restrict__ ra, const int64_t* __restrict__ offs, const AdjView adj,
+                        uint32_t* bits, uint64_t* best, int64_t n, int64_t vbase) {
+  cg::grid_group grid = cg::this_grid();
+  const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t gthreads = (int64_t)gridDim.x * blockDim.x;
+  for (;;) {
+    if (!*reinterpret_cast<volatile int*>(&ra->st->cont)) break;  // uniform after the barrier
+    const int cur = *reinterpret_cast<volatile int*>(&ra->st->cur);
+    {
+      const Bins F = ra->F[cur];
+      const unsigned long long* c = ra->cnt + cnt_F(cur, 0);
+      point_bin_body<B0G, B0U>(F.list[0], (int64_t)c[0], offs, adj, bits, best, vbase, gtid, gthreads);
+      point_bin_body<B1G, B1U>(F.list[1], (int64_t)c[1], offs, adj, bits, best, vbase, gtid, gthreads);
+      point_bin_body<B2G, B2U>(F.list[2], (int64_t)c[2], offs, adj, bits, best, vbase, gtid, gthreads);
+      point_bin_cta_body<256, 4>(F.list[3], (int64_t)c[3], offs, adj, bits, best, vbase, blockIdx.x,
+                                 gridDim.x);
+    }
+    grid.sync();
+    match_bins_body(ra->F[cur], ra->cnt + cnt_F(cur, 0), best, bits, gtid, gthreads);
+    grid.sync();
+    {
+      const CompactIO io = compact_io(*ra, cur);
+      compact_body<false, K>(io, n, best, bits, offs, vbase, blockIdx.x, gridDim.x);
+    }
+    grid.sync();
+    if (gtid == 0) end_round_body(ra, 0);
+    grid.sync();
+  }
+}
+__global__ void k_set_cur(RoundState* st, int cur) {
+  if (threadIdx.x == 0 && blockIdx.x == 0) st->cur = cur;
 }
 
 // =============================================================================================

@@ -79,8 +79,27 @@ using Sweep = lm::SweepCfg<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap>;
 constexpr int kSweepThreads = Sweep::kThreads;
 constexpr int64_t kTile = Sweep::kTile;
 constexpr int kCompactK = 8;  // items per lane per compaction chunk
+constexpr long long kLogCap = 1 << 16;  // per-round log rows kept on the device
+// hybrid round loop: frontiers up to this size run in the persistent kernel
+#ifndef LM_PERSIST_BELOW
+#define LM_PERSIST_BELOW (1 << 16)
+#endif
+constexpr int64_t kPersistentBelow = LM_PERSIST_BELOW;
+// frontier pointer kernels: lanes per vertex (G) and keys per lane per batch (U), per degree bin
+#ifndef LM_B0_G
+#define LM_B0_G 1
+#define LM_B0_U 8
+#endif
+#ifndef LM_B1_G
+#define LM_B1_G 8
+#define LM_B1_U 8
+#endif
+#ifndef LM_B2_G
+#define LM_B2_G 32
+#define LM_B2_U 4
+#endif
 
-constexpr int kFinBlocks = 592;  // 4 x 148 SMs: fixed => deterministic fp64 summation order
+constexpr int kFinBlocks = 2368;  // 16 x 148 SMs: fixed => deterministic fp64 summation order
 constexpr int kFinThreads = 256;
 
 int num_sms_cached = 0;
@@ -151,8 +170,29 @@ struct lmatch_graph {
   cudaEvent_t ev[8] = {};
   int64_t device_bytes = 0;
   std::vector<int64_t> round_log;  // per round: |F_r|, |L_r|, E(F_r) (directed entries scanned)
+  // device-side round loop
+  lm::RoundState* rstate = nullptr;
+  lm::RoundArgs* d_rargs = nullptr;    // device copy of rargs() (kernels read it by pointer)
+  lm::RoundState* h_rstate = nullptr;  // pinned
+  long long* rlog = nullptr;           // device [kLogCap][3]
+  int round_loop = 0;                  // 0 = CUDA graph, 1 = host-driven
+  cudaGraphExec_t gexec = nullptr;
+  cudaGraph_t graph = nullptr;
+  cudaStream_t gstream = nullptr;      // stream the graph was captured on (capture needs its own)
 
   lm::AdjView view() const { return lm::AdjView{adj, host_adj_dev - R, R}; }
+  const lm::RoundArgs* ra() const { return d_rargs; }
+  lm::RoundArgs rargs() const {
+    lm::RoundArgs a;
+    a.S[0] = S[0];
+    a.S[1] = S[1];
+    a.F[0] = F[0];
+    a.F[1] = F[1];
+    a.cnt = counters;
+    a.st = rstate;
+    a.log = rlog;
+    return a;
+  }
 };
 
 namespace {
@@ -223,6 +263,10 @@ int alloc_all(lmatch_graph* g) {
   TRY(dmalloc(g, &g->bits, (size_t)((g->n_global + 31) / 32) + 1));
   for (int i = 0; i < 2; ++i) TRY(dmalloc(g, &g->S[i], (size_t)n + 1));
   TRY(dmalloc(g, &g->counters, lm::kNumCounters));
+  TRY(dmalloc(g, &g->rstate, 1));
+  TRY(dmalloc(g, &g->d_rargs, 1));
+  TRY(dmalloc(g, &g->rlog, 3 * (size_t)kLogCap + 3));
+  CK(cudaHostAlloc(reinterpret_cast<void**>(&g->h_rstate), sizeof(lm::RoundState), cudaHostAllocDefault));
   TRY(dmalloc(g, &g->pw, kFinBlocks));
   TRY(dmalloc(g, &g->pc, kFinBlocks));
   TRY(dmalloc(g, &g->res_w, 1));
@@ -439,6 +483,8 @@ int alloc_bins(lmatch_graph* g, cudaStream_t st) {
   cudaFree(cnt);
   for (int i = 0; i < 2; ++i)
     for (int b = 0; b < lm::kBins; ++b) TRY(dmalloc(g, &g->F[i].list[b], (size_t)h[b] + 1));
+  const lm::RoundArgs a = g->rargs();
+  CK(cudaMemcpy(g->d_rargs, &a, sizeof a, cudaMemcpyHostToDevice));
   return LMATCH_OK;
 }
 
@@ -496,6 +542,7 @@ int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** 
     if (opts->upload_chunk > 0) g->upload_chunk = (opts->upload_chunk + 3) & ~3ll;
     g->hbm_budget = opts->hbm_budget_bytes;
     if (opts->stream_chunk > 0) g->stream_chunk = opts->stream_chunk;
+    g->round_loop = opts->round_loop;
   }
   CK(cudaGetDevice(&g->device));
   CK(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, g->device));
@@ -607,7 +654,11 @@ void lmatch_destroy(lmatch_graph* g) {
     if (g->ev_free[i]) cudaEventDestroy(g->ev_free[i]);
   }
   if (g->cs) cudaStreamDestroy(g->cs);
-  void* pdev[] = {g->bounds, g->ghost, g->claims, g->claim_cnt};
+  if (g->gexec) cudaGraphExecDestroy(g->gexec);
+  if (g->graph) cudaGraphDestroy(g->graph);
+  if (g->gstream) cudaStreamDestroy(g->gstream);
+  if (g->h_rstate) cudaFreeHost(g->h_rstate);
+  void* pdev[] = {g->bounds, g->ghost, g->claims, g->claim_cnt, g->rstate, g->rlog, g->d_rargs};
   for (void* p : pdev) if (p) cudaFree(p);
   if (g->h_claim_cnt) cudaFreeHost(g->h_claim_cnt);
   if (g->h_res) cudaFreeHost(g->h_res);
@@ -693,83 +744,166 @@ int lmatch_info(const lmatch_graph* g, int64_t* n, int64_t* m, int64_t* nonempty
   return LMATCH_OK;
 }
 
+// ---- the launch sequence of one run (shared by the host-driven loop and the CUDA graph)
+static int seq_prefix(lmatch_graph* g, cudaStream_t st, cudaGraphConditionalHandle h, int in_graph,
+                      int64_t* launches, int64_t* sweep_launches, int64_t* bytes_streamed) {
+  const int64_t n = g->n;
+  const int64_t nwords = (g->n_global + 31) / 32;
+  const bool work = g->ntiles > 0 && n > 0;
+  lm::k_reset<<<grid_for(std::max(nwords, g->n_atomic), 256, 4096), 256, 0, st>>>(
+      g->bits, nwords, g->best, g->atomic_rows, g->n_atomic, g->counters, lm::kNumCounters);
+  CKL();
+  lm::k_round_init<<<1, 1, 0, st>>>(g->rstate, g->max_rounds, kLogCap, work ? 1 : 0);
+  CKL();
+  *launches += 2;
+  // phase events (inside a graph they become event-record nodes)
+  cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+  CK(cudaStreamIsCapturing(st, &cap));
+  auto mark = [&](int i) -> int {
+    if (g->timing) {
+      if (cap == cudaStreamCaptureStatusActive)
+        CK(cudaEventRecordWithFlags(g->ev[i], st, cudaEventRecordExternal));
+      else
+        CK(cudaEventRecord(g->ev[i], st));
+    }
+    return LMATCH_OK;
+  };
+  TRY(mark(1));
+  if (!work) {
+    if (in_graph) {
+      lm::k_end_round<<<1, 32, 0, st>>>(g->ra(), h, 1, 0);  // cont = 0
+      CKL();
+    }
+    TRY(mark(2));
+    TRY(mark(3));
+    return LMATCH_OK;
+  }
+  // round 1: A2 full sweep (no bitmap test), A4 match-all, A6 compact-all
+  TRY(round1_sweep(g, st, launches, sweep_launches, bytes_streamed));
+  TRY(mark(2));
+  lm::k_match_all<<<grid_for(nwords * 32, 256, 65536), 256, 0, st>>>(g->best, n, g->bits);
+  CKL();
+  // round-1 compaction: input set 1 (unused), output set 0; k_end_round makes set 0 current
+  lm::k_compact<true, kCompactK><<<grid_for((n + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
+      lm::compact_io(g->rargs(), 1), n, g->best, g->bits, g->offs, g->v0);
+  CKL();
+  lm::k_end_round<<<1, 32, 0, st>>>(g->ra(), h, in_graph, 0);
+  CKL();
+  *launches += 3;
+  TRY(mark(3));
+  return LMATCH_OK;
+}
+
+// rounds >= 2, host-driven: A2 frontier pointers, A4, A6, end of round, with the current set
+// `cur` and its sizes known on the host (grids fit the work; empty bins are skipped).
+static int seq_body(lmatch_graph* g, cudaStream_t st, int cur, const int64_t* nFb, int64_t nS,
+                    int64_t* launches) {
+  const lm::AdjView av = g->view();
+  const lm::Bins& Fb = g->F[cur];
+  const unsigned long long* cF = g->counters + lm::cnt_F(cur, 0);
+  int64_t nF = 0;
+  for (int b = 0; b < lm::kBins; ++b) nF += nFb[b];
+  if (nFb[0]) { lm::k_point_bin<LM_B0_G, LM_B0_U><<<grid_for(nFb[0] * LM_B0_G, 256, 65536), 256, 0, st>>>(Fb.list[0], cF + 0, g->offs, av, g->bits, g->best, g->v0); CKL(); ++*launches; }
+  if (nFb[1]) { lm::k_point_bin<LM_B1_G, LM_B1_U><<<grid_for(nFb[1] * LM_B1_G, 256, 65536), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, av, g->bits, g->best, g->v0); CKL(); ++*launches; }
+  if (nFb[2]) { lm::k_point_bin<LM_B2_G, LM_B2_U><<<grid_for(nFb[2] * LM_B2_G, 256, 65536), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, av, g->bits, g->best, g->v0); CKL(); ++*launches; }
+  if (nFb[3]) { lm::k_point_bin_cta<256, 4><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); ++*launches; }
+  lm::k_match_bins<<<grid_for(nF, 256, 65536), 256, 0, st>>>(Fb, cF, g->best, g->bits);
+  CKL();
+  lm::k_compact<false, kCompactK><<<grid_for((nS + nF + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
+      lm::compact_io(g->rargs(), cur), g->n, g->best, g->bits, g->offs, g->v0);
+  CKL();
+  lm::k_end_round<<<1, 32, 0, st>>>(g->ra(), 0, 0, 0);
+  CKL();
+  *launches += 3;
+  return LMATCH_OK;
+}
+
+#define PERSISTENT_KERNEL \
+  lm::k_rounds_persistent<LM_B0_G, LM_B0_U, LM_B1_G, LM_B1_U, LM_B2_G, LM_B2_U, kCompactK>
+
+// rounds >= 2 in one cooperative launch (grid = co-resident blocks)
+static int launch_persistent(lmatch_graph* g, cudaStream_t st, int64_t* launches) {
+  static int occ = 0;
+  if (!occ) {
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, PERSISTENT_KERNEL, 256, 0));
+    if (occ < 1) occ = 1;
+  }
+  const lm::RoundArgs* ra = g->ra();
+  const lm::AdjView av = g->view();
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(occ * g->num_sms));
+  cfg.blockDim = dim3(256);
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeCooperative;
+  attr[0].val.cooperative = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  CK(cudaLaunchKernelEx(&cfg, PERSISTENT_KERNEL, ra, (const int64_t*)g->offs, av, g->bits, g->best,
+                        g->n, g->v0));
+  ++*launches;
+  return LMATCH_OK;
+}
+
+// Capture reset .. round 1 + the persistent round kernel into one CUDA graph (built once).
+static int build_graph_persistent(lmatch_graph* g) {
+  if (!g->gstream) CK(cudaStreamCreateWithFlags(&g->gstream, cudaStreamNonBlocking));
+  cudaStream_t s = g->gstream;
+  int64_t l = 0, sl = 0, bs = 0;
+  CK(cudaStreamBeginCapture(s, cudaStreamCaptureModeRelaxed));
+  int rc = seq_prefix(g, s, 0, 0, &l, &sl, &bs);
+  if (!rc) rc = launch_persistent(g, s, &l);
+  cudaGraph_t graph = nullptr;
+  const cudaError_t e = cudaStreamEndCapture(s, &graph);
+  if (rc) { if (graph) cudaGraphDestroy(graph); return rc; }
+  if (e != cudaSuccess) { set_err("end capture: %s", cudaGetErrorString(e)); return LMATCH_ECUDA; }
+  g->graph = graph;
+  CK(cudaGraphInstantiate(&g->gexec, g->graph, 0));
+  return LMATCH_OK;
+}
+
 int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_stats* stats) {
   if (!g) { set_err("NULL handle"); return LMATCH_ESTATE; }
   if (!d_mate && g->n > 0) { set_err("d_mate == NULL"); return LMATCH_EINVAL; }
+  if (g->ghost) { set_err("partition handle: use the lmatch_part_* calls"); return LMATCH_ESTATE; }
   g_err[0] = 0;
   CK(cudaSetDevice(g->device));
   cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
   const int64_t n = g->n;
   const bool tm = g->timing && stats;
-  int64_t launches = 0, rounds = 0, ftot_all = 0, sweep_launches = 0, bytes_streamed = 0;
-  unsigned long long* C = g->counters;
-  unsigned long long* hc = g->h_counters;
-  g->round_log.clear();
+  // round_loop: 0 = hybrid: host-driven, work-sized launches while the frontier is large, then
+  //                 ONE persistent cooperative kernel for the remaining (small) rounds;
+  //              1 = host-driven launches for every round;
+  //              2 = persistent kernel for every round after round 1;
+  //              3 = CUDA graph {round 1, persistent kernel} (no host work per run).
+  const int mode = g->round_loop;
+  const bool use_graph = mode == 3 && !g->streaming;
+  int64_t launches = 0, sweep_launches = 0, bytes_streamed = 0;
 
   if (tm) CK(cudaEventRecord(g->ev[0], st));
-  // ---- reset (bitmap, counters, tile-crossing rows' best)
-  const int64_t nwords = (g->n_global + 31) / 32;
-  lm::k_reset<<<grid_for(std::max(nwords, g->n_atomic), 256, 4096), 256, 0, st>>>(
-      g->bits, nwords, g->best, g->atomic_rows, g->n_atomic, C, lm::kNumCounters);
-  CKL();
-  ++launches;
-  if (tm) CK(cudaEventRecord(g->ev[1], st));
-  if (g->ntiles > 0 && n > 0) {
-    // ---- round 1: A2 full sweep (no bitmap test), A4 match-all, A6 compact-all
-    TRY(round1_sweep(g, st, &launches, &sweep_launches, &bytes_streamed));
-    CKL();
-    if (tm) CK(cudaEventRecord(g->ev[2], st));
-    rounds = 1;
-    lm::k_match_all<<<grid_for(nwords * 32, 256, 65536), 256, 0, st>>>(g->best, n, g->bits);
-    CKL();
-    lm::k_compact<true, kCompactK><<<grid_for((n + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
-        nullptr, nullptr, lm::Bins{}, nullptr, n, g->best, g->bits, g->offs, g->S[0],
-        C + lm::cnt_S(0), g->F[0], C + lm::cnt_F(0, 0), C + lm::kCntSwept, g->v0);
-    CKL();
-    launches += 2;
-    CK(cudaMemcpyAsync(hc, C, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
-    if (tm) CK(cudaEventRecord(g->ev[3], st));
-    g->round_log.insert(g->round_log.end(), {g->n_nz, n, g->m});
-    int cur = 0;
-    unsigned long long swept_prev = 0;
+  if (use_graph) {
+    if (!g->gexec) TRY(build_graph_persistent(g));
+    CK(cudaGraphLaunch(g->gexec, st));
+  } else if (mode == 2) {
+    TRY(seq_prefix(g, st, 0, 0, &launches, &sweep_launches, &bytes_streamed));
+    if (g->ntiles > 0 && n > 0) TRY(launch_persistent(g, st, &launches));
+  } else {
+    TRY(seq_prefix(g, st, 0, 0, &launches, &sweep_launches, &bytes_streamed));
     for (;;) {
-      const int64_t nS = (int64_t)hc[lm::cnt_S(cur)];
-      int64_t nFb[lm::kBins], nF = 0;
-      for (int b = 0; b < lm::kBins; ++b) { nFb[b] = (int64_t)hc[lm::cnt_F(cur, b)]; nF += nFb[b]; }
-      if (nF == 0 || rounds >= g->max_rounds) break;
-      ++rounds;
-      ftot_all += nF;
-      g->round_log.insert(g->round_log.end(),
-                          {nF, nS + nF, (int64_t)(hc[lm::kCntSwept] - swept_prev)});
-      swept_prev = hc[lm::kCntSwept];
-      const unsigned long long* cF = C + lm::cnt_F(cur, 0);
-      // A2 frontier pointer phase, one launch per non-empty degree bin
-      lm::Bins& Fb = g->F[cur];
-      const int kMaxGrid = 65536;
-      if (nFb[0]) { lm::k_point_bin<1, 8><<<grid_for(nFb[0], 256, kMaxGrid), 256, 0, st>>>(Fb.list[0], cF + 0, g->offs, g->view(), g->bits, g->best, g->v0); CKL(); ++launches; }    // deg <= 8: a thread each
-      if (nFb[1]) { lm::k_point_bin<8, 8><<<grid_for(nFb[1] * 8, 256, kMaxGrid), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, g->view(), g->bits, g->best, g->v0); CKL(); ++launches; }     // 9..64
-      if (nFb[2]) { lm::k_point_bin<32, 4><<<grid_for(nFb[2] * 32, 256, kMaxGrid), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, g->view(), g->bits, g->best, g->v0); CKL(); ++launches; }   // 65..2048
-      if (nFb[3]) { lm::k_point_bin_cta<256, 4><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, g->view(), g->bits, g->best, g->v0); CKL(); ++launches; }
-      // A4 match over the new pointers
-      lm::k_match_bins<<<grid_for(nF, 256, 65536), 256, 0, st>>>(Fb, cF, g->best, g->bits);
-      CKL();
-      // A6 compaction of the live pairs
-      const int nxt = cur ^ 1;
-      CK(cudaMemsetAsync(C + lm::cnt_S(nxt), 0, 8 * (1 + lm::kBins), st));
-      lm::k_compact<false, kCompactK>
-          <<<grid_for((nS + nF + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
-              g->S[cur], C + lm::cnt_S(cur), Fb, cF, n, g->best, g->bits, g->offs, g->S[nxt],
-              C + lm::cnt_S(nxt), g->F[nxt], C + lm::cnt_F(nxt, 0), C + lm::kCntSwept, g->v0);
-      CKL();
-      launches += 2;
-      CK(cudaMemcpyAsync(hc, C, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
+      CK(cudaMemcpyAsync(g->h_rstate, g->rstate, sizeof(lm::RoundState), cudaMemcpyDeviceToHost, st));
+      CK(cudaMemcpyAsync(g->h_counters, g->counters, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
       CK(cudaStreamSynchronize(st));
-      cur = nxt;
+      if (!g->h_rstate->cont) break;
+      const int cur = g->h_rstate->cur;
+      int64_t nFb[lm::kBins], nF = 0;
+      for (int b = 0; b < lm::kBins; ++b) { nFb[b] = (int64_t)g->h_counters[lm::cnt_F(cur, b)]; nF += nFb[b]; }
+      const int64_t nS = (int64_t)g->h_counters[lm::cnt_S(cur)];
+      if (mode == 0 && nF <= kPersistentBelow) {  // the tail: every remaining round on the device
+        TRY(launch_persistent(g, st, &launches));
+        break;
+      }
+      TRY(seq_body(g, st, cur, nFb, nS, &launches));
     }
-  } else if (tm) {
-    CK(cudaEventRecord(g->ev[2], st));
-    CK(cudaEventRecord(g->ev[3], st));
   }
   if (tm) CK(cudaEventRecord(g->ev[4], st));
   // ---- A10 mate[] + A9 w(M)
@@ -786,8 +920,26 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
     g->h_res[0] = 0.0;
     g->h_resc[0] = 0;
   }
+  CK(cudaMemcpyAsync(g->h_rstate, g->rstate, sizeof(lm::RoundState), cudaMemcpyDeviceToHost, st));
   if (tm) CK(cudaEventRecord(g->ev[5], st));
   CK(cudaStreamSynchronize(st));
+  const lm::RoundState rs = *g->h_rstate;
+  const int64_t rounds = rs.rounds;
+  if (use_graph) {  // launches inside the graph
+    launches += (rounds > 0 ? 6 : 2) + (rounds > 0 ? 1 : 0);
+    sweep_launches = rounds > 0 ? 1 : 0;
+  }
+  // per-round log: round 1 from the host, later rounds from the device log
+  g->round_log.clear();
+  if (rounds > 0) {
+    g->round_log.insert(g->round_log.end(), {g->n_nz, n, g->m});
+    const int64_t rows = std::min<int64_t>(rs.log_len, kLogCap);
+    if (rows > 0) {
+      std::vector<long long> tmp(3 * (size_t)rows);
+      CK(cudaMemcpy(tmp.data(), g->rlog, tmp.size() * 8, cudaMemcpyDeviceToHost));
+      for (long long x : tmp) g->round_log.push_back(x);
+    }
+  }
   if (stats) {
     std::memset(stats, 0, sizeof *stats);
     stats->rounds = rounds;
@@ -796,18 +948,18 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
     stats->weight = g->h_res[0];
     stats->entries_swept = 0;
     for (size_t i = 2; i < g->round_log.size(); i += 3) stats->entries_swept += g->round_log[i];
-    stats->frontier_total = ftot_all;
+    stats->frontier_total = rs.ftot;
     stats->sweep_launches = sweep_launches;
+    stats->kernel_launches = launches;
     stats->bytes_streamed = bytes_streamed;
     stats->resident_entries = g->R;
-    stats->kernel_launches = launches;
     if (tm) {
       float a = 0, b = 0, c = 0, d = 0, e = 0;
       CK(cudaEventElapsedTime(&a, g->ev[0], g->ev[5]));
+      CK(cudaEventElapsedTime(&e, g->ev[4], g->ev[5]));
       CK(cudaEventElapsedTime(&b, g->ev[1], g->ev[2]));
       CK(cudaEventElapsedTime(&c, g->ev[2], g->ev[3]));
       CK(cudaEventElapsedTime(&d, g->ev[3], g->ev[4]));
-      CK(cudaEventElapsedTime(&e, g->ev[4], g->ev[5]));
       stats->ms_total = a;
       stats->ms_sweep = b;
       stats->ms_round1_rest = c;
@@ -951,6 +1103,8 @@ int lmatch_part_begin(lmatch_graph* g, void* stream, int64_t* claim_counts) {
   lm::k_reset<<<grid_for(std::max(nwords, g->n_atomic), 256, 4096), 256, 0, st>>>(
       g->bits, nwords, g->best, g->atomic_rows, g->n_atomic, g->counters, lm::kNumCounters);
   CKL();
+  lm::k_round_init<<<1, 1, 0, st>>>(g->rstate, g->max_rounds, kLogCap, 1);
+  CKL();
   CK(cudaMemsetAsync(g->ghost, 0xff, ((size_t)g->n_global + 1) * 4, st));
   CK(cudaMemsetAsync(g->claim_cnt, 0, (size_t)g->P * 8, st));
   int64_t l = 0, sl = 0, bs = 0;
@@ -1032,31 +1186,31 @@ int lmatch_part_compact(lmatch_graph* g, void* stream, int64_t* nF_local) {
   cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
   unsigned long long* C = g->counters;
   const int64_t n = g->n;
+  // the compaction reads set part_cur (round 1: none) and writes its other set; k_end_round
+  // makes that set current (and zeroes the counters the next compaction writes)
   if (g->part_round == 1) {
     if (n > 0) {
       lm::k_compact<true, kCompactK><<<grid_for((n + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
-          nullptr, nullptr, lm::Bins{}, nullptr, n, g->best, g->bits, g->offs, g->S[0],
-          C + lm::cnt_S(0), g->F[0], C + lm::cnt_F(0, 0), C + lm::kCntSwept, g->v0);
+          lm::compact_io(g->rargs(), 1), n, g->best, g->bits, g->offs, g->v0);
       CKL();
     }
     g->part_cur = 0;
     g->round_log.insert(g->round_log.end(), {g->n_nz, n, g->m});
   } else {
-    const int cur = g->part_cur, nxt = cur ^ 1;
+    const int cur = g->part_cur;
     const int64_t nS = (int64_t)g->h_counters[lm::cnt_S(cur)];
     int64_t nF = 0;
     for (int b = 0; b < lm::kBins; ++b) nF += (int64_t)g->h_counters[lm::cnt_F(cur, b)];
-    CK(cudaMemsetAsync(C + lm::cnt_S(nxt), 0, 8 * (1 + lm::kBins), st));
     if (nS + nF > 0) {
       lm::k_compact<false, kCompactK>
           <<<grid_for((nS + nF + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
-              g->S[cur], C + lm::cnt_S(cur), g->F[cur], C + lm::cnt_F(cur, 0), n, g->best, g->bits,
-              g->offs, g->S[nxt], C + lm::cnt_S(nxt), g->F[nxt], C + lm::cnt_F(nxt, 0),
-              C + lm::kCntSwept, g->v0);
+              lm::compact_io(g->rargs(), cur), n, g->best, g->bits, g->offs, g->v0);
       CKL();
     }
-    g->part_cur = nxt;
+    g->part_cur = cur ^ 1;
   }
+  lm::k_end_round<<<1, 32, 0, st>>>(g->ra(), 0, 0, 0);
+  CKL();
   CK(cudaMemcpyAsync(g->h_counters, C, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
   int64_t nF = 0;
@@ -1072,12 +1226,12 @@ int lmatch_part_point(lmatch_graph* g, void* stream, int64_t* claim_counts) {
   const int cur = g->part_cur;
   int64_t nFb[lm::kBins], nF = 0;
   for (int b = 0; b < lm::kBins; ++b) { nFb[b] = (int64_t)g->h_counters[lm::cnt_F(cur, b)]; nF += nFb[b]; }
-  const unsigned long long* cF = g->counters + lm::cnt_F(cur, 0);
-  lm::Bins& Fb = g->F[cur];
   const lm::AdjView av = g->view();
-  if (nFb[0]) { lm::k_point_bin<1, 8><<<grid_for(nFb[0], 256, 65536), 256, 0, st>>>(Fb.list[0], cF + 0, g->offs, av, g->bits, g->best, g->v0); CKL(); }
-  if (nFb[1]) { lm::k_point_bin<8, 8><<<grid_for(nFb[1] * 8, 256, 65536), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, av, g->bits, g->best, g->v0); CKL(); }
-  if (nFb[2]) { lm::k_point_bin<32, 4><<<grid_for(nFb[2] * 32, 256, 65536), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, av, g->bits, g->best, g->v0); CKL(); }
+  const lm::Bins& Fb = g->F[cur];
+  const unsigned long long* cF = g->counters + lm::cnt_F(cur, 0);
+  if (nFb[0]) { lm::k_point_bin<LM_B0_G, LM_B0_U><<<grid_for(nFb[0] * LM_B0_G, 256, 65536), 256, 0, st>>>(Fb.list[0], cF + 0, g->offs, av, g->bits, g->best, g->v0); CKL(); }
+  if (nFb[1]) { lm::k_point_bin<LM_B1_G, LM_B1_U><<<grid_for(nFb[1] * LM_B1_G, 256, 65536), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, av, g->bits, g->best, g->v0); CKL(); }
+  if (nFb[2]) { lm::k_point_bin<LM_B2_G, LM_B2_U><<<grid_for(nFb[2] * LM_B2_G, 256, 65536), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, av, g->bits, g->best, g->v0); CKL(); }
   if (nFb[3]) { lm::k_point_bin_cta<256, 4><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); }
   CK(cudaMemsetAsync(g->claim_cnt, 0, (size_t)g->P * 8, st));
   if (nF > 0) {

@@ -279,3 +279,39 @@ def test_partitioned_hub_rows(lm):
                             [(v, v + 1, 0.5) for v in range(100, 8000, 7)])
     mate, res = D.match_partitioned_local(g.offsets, g.col, g.w, 4)
     np.testing.assert_array_equal(mate, oracle.greedy(g).mate)
+
+
+# --------------------------------------------- round loop: CUDA graph (default) vs host-driven
+@pytest.mark.parametrize("maker", [
+    lambda: graphgen.rmat(14, 16, seed=21),
+    lambda: graphgen.rmat(17, 16, seed=24, weights="paper"),
+    lambda: graphgen.mesh(64, seed=22, weights="gradient"),     # ~130 rounds inside the graph
+    lambda: graphgen.from_edges(5, []),                         # no work: the WHILE never runs
+    lambda: graphgen.from_edges(301, [(i, i + 1, float(i + 1)) for i in range(300)]),
+])
+def test_round_loop_modes_identical(lm, maker):
+    g = maker()
+    ref = oracle.greedy(g).mate
+    ph = oracle.ld_frontier(g)[1]
+    out = [run_gpu(lm, g, round_loop=mode, timing=True) for mode in (0, 1, 2, 3)]
+    for mate, st in out:
+        np.testing.assert_array_equal(mate, ref)
+        assert st["rounds"] == ph
+        assert st["weight"] == out[0][1]["weight"]
+        assert st["frontier_total"] == out[0][1]["frontier_total"]
+        if g.m:
+            assert st["ms_sweep"] > 0
+
+
+def test_graph_replay_and_round_log(lm):
+    """The instantiated graph is replayed across runs; the per-round log matches the oracle's
+    frontier sizes (Fig. 8 analogue)."""
+    g = graphgen.rmat(15, 16, seed=23)
+    _, ph, fs = oracle.ld_frontier(g)
+    with lm.Matcher(g) as M:
+        for _ in range(3):
+            mate, st = M.run()
+            np.testing.assert_array_equal(mate, oracle.greedy(g).mate)
+            log = lm.lmatch_round_log(M.h)
+            assert log.shape[0] == st["rounds"] == ph
+            np.testing.assert_array_equal(log[:, 0], fs)
