@@ -366,6 +366,9 @@ __device__ __forceinline__ uint64_t umax_skip(uint64_t b, uint64_t key, uint32_t
 
 struct SweepArgs {
   const uint64_t* adj;       // keys of entry tile_begin*TILE onward (HBM or a streamed chunk)
+  uint64_t* zap;             // ZAP variant only: writable adjacency (self-loop keys -> 0)
+  unsigned long long* zapped;
+  uint32_t vbase;            // ZAP only: global id of local row 0 (partitioned handles)
   const uint32_t* noffs_lo;  // low 32 bits of each non-empty row's start (+ m)
   const int32_t* nzr;
   const int32_t* tile_nz;
@@ -391,8 +394,10 @@ struct SweepCfg {
   static_assert(kStageBytes % 16 == 0 && kWarpBytes % 16 == 0, "TMA needs 16-byte alignment");
 };
 
-template <int TILE, int RING, int WARPS, int WCAP>
+template <int TILE, int RING, int WARPS, int WCAP, bool ZAP = false>
 __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
+  // ZAP: the one-time ingest pass -- same tiles and rows, but instead of the max it zeroes the
+  // keys of self-loops (col == row; simple graph) in place.
   using C = SweepCfg<TILE, RING, WARPS, WCAP>;
   extern __shared__ __align__(128) unsigned char smem[];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -480,6 +485,30 @@ __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
       }
       const bool inside = rs >= 0 && re <= len;
       // short rows: a lane each
+      if (ZAP) {
+        // every entry of the window's rows inside this tile, lane-per-row then warp-per-row
+        if (L > 0 && L < 32) {
+          for (int j = max(rs, 0), je = min(re, len); j < je; ++j)
+            if ((uint32_t)K[j] == vid + A.vbase && K[j] != 0ull) {
+              A.zap[ts + j] = 0ull;
+              atomicAdd(A.zapped, 1ull);
+            }
+        }
+        unsigned zm = __ballot_sync(0xffffffffu, L >= 32);
+        while (zm) {
+          const int l = __ffs(zm) - 1;
+          zm &= zm - 1;
+          const int32_t ja = __shfl_sync(0xffffffffu, max(rs, 0), l);
+          const int32_t jb = __shfl_sync(0xffffffffu, min(re, len), l);
+          const uint32_t v = __shfl_sync(0xffffffffu, vid, l);
+          for (int j = ja + lane; j < jb; j += 32)
+            if ((uint32_t)K[j] == v + A.vbase && K[j] != 0ull) {
+              A.zap[ts + j] = 0ull;
+              atomicAdd(A.zapped, 1ull);
+            }
+        }
+        continue;
+      }
       if (L > 0 && L < 32) {
         uint64_t b0 = 0, b1 = 0, b2 = 0, b3 = 0;  // 4 independent max chains
         int j = max(rs, 0);

@@ -490,13 +490,29 @@ int alloc_bins(lmatch_graph* g, cudaStream_t st) {
 
 int finish_create(lmatch_graph* g, cudaStream_t st) {
   TRY(alloc_bins(g, st));
-  if (g->m > 0) {
-    CK(cudaMemsetAsync(g->werr, 0, 8, st));
-    lm::k_zap_self_loops<<<grid_for(g->n * 8, 256, 16384), 256, 0, st>>>(
-        g->offs, g->view(), g->n, g->v0, reinterpret_cast<unsigned long long*>(g->werr));
-    CKL();
-  }
   TRY(build_index(g, st));
+  if (g->m > 0) {
+    // self-loop keys -> 0: the sweep's tile pass over resident graphs, the row-based
+    // kernel over out-of-core ones (rows may live in host memory)
+    CK(cudaMemsetAsync(g->werr, 0, 8, st));
+    unsigned long long* zc = reinterpret_cast<unsigned long long*>(g->werr);
+    if (!g->streaming && g->ntiles > 0) {
+      CK(cudaFuncSetAttribute(lm::k_sweep<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap, true>,
+                              cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              (int)lm::SweepCfg<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap>::kSmem));
+      const int64_t grid = std::max<int64_t>(1, std::min<int64_t>((g->ntiles + kSweepWarps - 1) / kSweepWarps,
+                                                                  3 * (int64_t)g->num_sms));
+      lm::SweepArgs A{g->adj, g->adj, zc, (uint32_t)g->v0, g->noffs_lo, g->nzr, g->tile_nz, g->best, g->m, 0, g->ntiles};
+      lm::k_sweep<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap, true>
+          <<<(unsigned)grid, 32 * kSweepWarps,
+             lm::SweepCfg<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap>::kSmem, st>>>(A);
+      CKL();
+    } else {
+      lm::k_zap_self_loops<<<grid_for(g->n * 8, 256, 16384), 256, 0, st>>>(g->offs, g->view(), g->n,
+                                                                           g->v0, zc);
+      CKL();
+    }
+  }
 #if LM_SWEEP_IMPL == 2
   if (g->streaming) { set_err("LM_SWEEP_IMPL=2 does not support out-of-core graphs"); return LMATCH_EINVAL; }
   if (g->ntiles > 0) TRY(make_tensor_map(g));
@@ -583,7 +599,7 @@ int round1_sweep(lmatch_graph* g, cudaStream_t st, int64_t* launches_out, int64_
   const int64_t rt = g->streaming ? g->R / kTile : g->ntiles;
   auto sweep_launch = [&](const uint64_t* base, int64_t t0, int64_t t1) -> int {
     const int64_t grid = std::min<int64_t>((t1 - t0 + kSweepWarps - 1) / kSweepWarps, g->sweep_grid);
-    lm::SweepArgs A{base, g->noffs_lo, g->nzr, g->tile_nz, g->best, g->m, t0, t1};
+    lm::SweepArgs A{base, nullptr, nullptr, 0u, g->noffs_lo, g->nzr, g->tile_nz, g->best, g->m, t0, t1};
     SWEEP_KERNEL<<<(unsigned)std::max<int64_t>(grid, 1), kSweepThreads, Sweep::kSmem, st>>>(A);
     CKL();
     ++launches;

@@ -315,3 +315,42 @@ def test_graph_replay_and_round_log(lm):
             log = lm.lmatch_round_log(M.h)
             assert log.shape[0] == st["rounds"] == ph
             np.testing.assert_array_equal(log[:, 0], fs)
+
+
+# ------------------------------------------------------- self-loops (ignored) at ingest
+def _loopy_graph(seed):
+    """Random graph whose self-loops carry the LARGEST weights (they would win every row if not
+    ignored): short rows (< 32 entries), warp-width rows (32..512) and hub rows crossing many
+    512-entry sweep tiles all get a loop."""
+    rng = np.random.default_rng(seed)
+    n = 6000
+    edges = []
+    for u in range(n):
+        deg = int(rng.choice([1, 3, 40, 300])) if u % 97 else 0
+        for v in rng.integers(0, n, size=deg):
+            if int(v) != u:
+                edges.append((u, int(v), float(np.float32(0.5 * rng.random() + 0.01))))
+    for v in range(1, n):  # hub 0 spans many tiles
+        if v % 3:
+            edges.append((0, v, float(np.float32(0.5 * rng.random() + 0.01))))
+    for u in rng.choice(n, size=n // 2, replace=False):
+        edges.append((int(u), int(u), 2.0 + float(rng.random())))
+    edges.append((0, 0, 9.0))
+    return graphgen.from_edges(n, edges)
+
+
+@pytest.mark.parametrize("mode", ["resident", "streamed", "partitioned"])
+def test_self_loops_ignored(lm, mode):
+    g = _loopy_graph(21)
+    ref = oracle.greedy(g)
+    assert ref.cardinality > 0
+    if mode == "resident":
+        check_parity(lm, g)
+        check_parity(lm, g, upload_chunk=777)
+    elif mode == "streamed":
+        check_parity(lm, g, hbm_budget_bytes=8 * g.m // 3 + 2 * 8 * 1024, stream_chunk=1024)
+    else:
+        import paper_conf_sc_mandulakgfhs24_b200.dist as D
+        for P in (2, 3):
+            mate, res = D.match_partitioned_local(g.offsets, g.col, g.w, P)
+            np.testing.assert_array_equal(mate, ref.mate)
