@@ -51,6 +51,10 @@ def parse():
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--cpu-scale", type=int, default=None)
     p.add_argument("--gen", default="gpu", choices=["cpu", "gpu"])
+    p.add_argument("--hbm-budget-gb", type=float, default=0.0,
+                   help="out-of-core (A8): cap the HBM-resident adjacency; the rest is streamed "
+                        "from pinned host memory in round 1 and read zero-copy afterwards")
+    p.add_argument("--stream-chunk", type=int, default=0, help="entries per streamed chunk (0 = default)")
     p.add_argument("--partitioned", action="store_true",
                    help="use the 1-D partitioned path even at N=1 (it is always used for N>1)")
     return p.parse_args()
@@ -389,7 +393,8 @@ def main():
 
     # resident inputs: CSR on the device, handle built from device pointers (create is untimed,
     # P:179 excludes I/O, allocation, CSR construction and the initial transfer)
-    opts = lm.make_opts(validate_level=1, timing=1)
+    opts = lm.make_opts(validate_level=1, timing=1,
+                        hbm_budget_bytes=int(a.hbm_budget_gb * 1e9), stream_chunk=a.stream_chunk)
     h = lm.lmatch_create_device(d_off, d_col, d_w, n, m, opts, stream)
     if g is None and not a.no_e2e:  # host copies for the end-to-end leg
         import graphgen
@@ -480,6 +485,15 @@ def main():
                "ms_per_step": el / a.e2e_steps * 1e3,
                "includes": "lmatch_reload (H2D + pack + validate + index) + lmatch_run (+ mate D2H)"}
 
+    ooc = None
+    if a.hbm_budget_gb > 0:
+        ooc = {"hbm_budget_bytes": int(a.hbm_budget_gb * 1e9),
+               "resident_entries": int(last["resident_entries"]),
+               "resident_frac": last["resident_entries"] / max(m, 1),
+               "bytes_streamed_per_step": int(last["bytes_streamed"]),
+               "stream_gbs_in_sweep": last["bytes_streamed"] / max(sweep_avg_ms, 1e-9) / 1e6,
+               "note": "sweep = resident HBM tiles + host chunks over PCIe (2-slot ring); later "
+                       "rounds read host rows zero-copy"}
     round_log = lm.lmatch_round_log(h)
     lm.lmatch_destroy(h)
     del d_mate
@@ -499,6 +513,7 @@ def main():
                     "l2": f"inputs larger than L2 (adjacency {8 * m / 1e9:.1f} GB >> 126 MB); no flush",
                     "gen_s": round(gen_s, 1)},
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+                **({"out_of_core": ooc} if ooc else {}),
                 "gpu_launches": int(launches), "clocks": clk.summary(),
                 "rounds": int(rounds[-1]), "cardinality": int(last["cardinality"]),
                 "entries_swept": int(last["entries_swept"]), "frontier_total": int(last["frontier_total"]),

@@ -293,7 +293,9 @@ class Matcher:
 def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int = 0,
               max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
               round_loop: int = 0) -> Opts:
-    """round_loop: 0 = device-driven rounds in a CUDA graph (default), 1 = host-driven."""
+    """round_loop (include/lmatch.h): 0 = hybrid (work-sized launches, then one persistent kernel
+    for the tail; default), 1 = host-driven launches only, 2 = persistent kernel after round 1,
+    3 = CUDA graph {round 1, persistent kernel}."""
     o = Opts()
     o.round_loop = int(round_loop)
     o.hbm_budget_bytes = int(hbm_budget_bytes)
