@@ -78,11 +78,25 @@ def make_graph_cpu(a, scale, seed):
     return graphgen.mesh(side, seed=seed, weights="gradient")
 
 
-def make_graph_gpu(a, scale, seed, device):
+def host_assembly_needed(a, scale, device) -> bool:
+    """True when the generated device CSR (8 B/entry) plus the matcher's packed keys (8 B/entry)
+    and per-vertex state would not fit in HBM together (R-MAT s29 on one B200): the generator
+    then assembles the CSR in pinned host memory and the handle is created from host arrays."""
+    import torch
+    if a.workload != "rmat" or a.hbm_budget_gb > 0:
+        return False
+    n = 1 << scale
+    est = 2 * a.edgefactor * n
+    hbm = torch.cuda.get_device_properties(device).total_memory
+    return 16 * est + 48 * n > 0.85 * hbm
+
+
+def make_graph_gpu(a, scale, seed, device, host_out=False):
     import graphgen.gpu as gg
     wl = a.workload
     if wl == "rmat":
-        return gg.rmat(scale, a.edgefactor, seed=seed, weights=a.weights or "uniform", device=device)
+        return gg.rmat(scale, a.edgefactor, seed=seed, weights=a.weights or "uniform", device=device,
+                       host_out=host_out)
     if wl == "er":
         return gg.er(1 << scale, float(a.edgefactor), seed=seed, weights=a.weights or "uniform",
                      device=device)
@@ -385,17 +399,28 @@ def main():
         d_w = torch.from_numpy(g.w).to(dev)
         n, m, m_u = g.n, g.m, g.m_u
     else:
-        dg = make_graph_gpu(a, scale, seed, dev)
-        d_off, d_col, d_w = dg.offsets, dg.col, dg.w
+        host_out = host_assembly_needed(a, scale, dev)
+        dg = make_graph_gpu(a, scale, seed, dev, host_out=host_out)
         n, m, m_u = dg.n, dg.m, dg.m_u
-        g = None
+        if host_out:
+            import graphgen
+            g = graphgen.Graph(dg.offsets.numpy(), dg.col.numpy(), dg.w.numpy())
+            d_off = d_col = d_w = None
+        else:
+            d_off, d_col, d_w = dg.offsets, dg.col, dg.w
+            g = None
     gen_s = time.time() - t0
+    torch.cuda.empty_cache()
 
-    # resident inputs: CSR on the device, handle built from device pointers (create is untimed,
-    # P:179 excludes I/O, allocation, CSR construction and the initial transfer)
+    # handle built from the device CSR (or, when both do not fit in HBM, from the pinned host
+    # CSR); create is untimed: P:179 excludes I/O, allocation, CSR construction and the transfer
     opts = lm.make_opts(validate_level=1, timing=1,
                         hbm_budget_bytes=int(a.hbm_budget_gb * 1e9), stream_chunk=a.stream_chunk)
-    h = lm.lmatch_create_device(d_off, d_col, d_w, n, m, opts, stream)
+    pinned_host = d_off is None
+    if pinned_host:
+        h = lm.lmatch_create_ex(g.offsets, g.col, g.w, n, m, opts)
+    else:
+        h = lm.lmatch_create_device(d_off, d_col, d_w, n, m, opts, stream)
     if g is None and not a.no_e2e:  # host copies for the end-to-end leg
         import graphgen
         g = graphgen.Graph(d_off.cpu().numpy(), d_col.cpu().numpy(), d_w.cpu().numpy())
@@ -458,7 +483,7 @@ def main():
         cud = torch.cuda.cudart()
         regs = []
         for arr in (g.offsets, g.col, g.w):
-            if arr.nbytes:
+            if arr.nbytes and not pinned_host:
                 cud.cudaHostRegister(arr.ctypes.data, arr.nbytes, 0)
                 regs.append(arr)
         mate_h = torch.empty(n, dtype=torch.int32, pin_memory=True)
@@ -511,7 +536,9 @@ def main():
                 "config": workload_config(a, scale, n, m) | {
                     "parallelism": "1 GPU" if world == 1 else f"{world} independent instances (seed+rank), no collective",
                     "l2": f"inputs larger than L2 (adjacency {8 * m / 1e9:.1f} GB >> 126 MB); no flush",
-                    "gen_s": round(gen_s, 1)},
+                    "gen_s": round(gen_s, 1),
+                    "csr_for_create": "pinned host (device CSR + packed keys exceed HBM)" if pinned_host
+                                      else "device"},
                 "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
                 **({"out_of_core": ooc} if ooc else {}),
                 "gpu_launches": int(launches), "clocks": clk.summary(),

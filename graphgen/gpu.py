@@ -41,9 +41,11 @@ def _load():
         L.gg_cuda_temp_bytes.restype = i64
         L.gg_cuda_sort_unique.argtypes = [p, p, i64, i32, i32, p, i64, p, ctypes.POINTER(i32), p]
         L.gg_cuda_scatter.argtypes = [p, i64, i64, u64, i32, p, p, p, p]
+        L.gg_cuda_scatter_local.argtypes = [p, i64, i64, u64, i32, p, p, p, p]
         L.gg_cuda_mesh_deg.argtypes = [i64, i32, u64, p, p]
         L.gg_cuda_mesh_fill.argtypes = [i64, i32, u64, p, p, p, u64, i32, p]
         for f in ("gg_cuda_count", "gg_cuda_emit", "gg_cuda_sort_unique", "gg_cuda_scatter",
+                  "gg_cuda_scatter_local",
                   "gg_cuda_mesh_deg", "gg_cuda_mesh_fill"):
             getattr(L, f).restype = i32
         _lib = L
@@ -78,7 +80,10 @@ def _ck(rc, what):
         raise RuntimeError(f"{what} failed with CUDA error {rc}")
 
 
-def _edge_graph(kind, n, scale, M, seed, a, b, c, weights, wseed, device, bucket_entries, name):
+def _edge_graph(kind, n, scale, M, seed, a, b, c, weights, wseed, device, bucket_entries, name,
+                host_out=False):
+    """host_out: col/w (and offsets) are assembled bucket by bucket in PINNED HOST memory, so
+    graphs whose CSR cannot sit on the device next to the matcher's packed keys can be built."""
     import torch
     L = _load()
     dev = torch.device(device)
@@ -95,8 +100,14 @@ def _edge_graph(kind, n, scale, M, seed, a, b, c, weights, wseed, device, bucket
     keys = torch.empty(max(maxc, 1), dtype=torch.int64, device=dev)
     alt = torch.empty(max(maxc, 1), dtype=torch.int64, device=dev)
     temp = torch.empty(max(L.gg_cuda_temp_bytes(max(maxc, 1)), 1), dtype=torch.uint8, device=dev)
-    col = torch.empty(max(total, 1), dtype=torch.int32, device=dev)
-    w = torch.empty(max(total, 1), dtype=torch.float32, device=dev)
+    if host_out:
+        col = torch.empty(max(total, 1), dtype=torch.int32, pin_memory=True)
+        w = torch.empty(max(total, 1), dtype=torch.float32, pin_memory=True)
+        col_b = torch.empty(max(maxc, 1), dtype=torch.int32, device=dev)
+        w_b = torch.empty(max(maxc, 1), dtype=torch.float32, device=dev)
+    else:
+        col = torch.empty(max(total, 1), dtype=torch.int32, device=dev)
+        w = torch.empty(max(total, 1), dtype=torch.float32, device=dev)
     first = torch.full((n + 1,), INT64_MAX, dtype=torch.int64, device=dev)
     cur = torch.zeros(1, dtype=torch.int64, device=dev)
     nout = torch.zeros(1, dtype=torch.int64, device=dev)
@@ -116,23 +127,37 @@ def _edge_graph(kind, n, scale, M, seed, a, b, c, weights, wseed, device, bucket
                                   ctypes.byref(which), st), "sort_unique")
         cu = int(nout.item())
         src = keys if which.value == 0 else alt
-        _ck(L.gg_cuda_scatter(src.data_ptr(), cu, base, ws, mode, col.data_ptr(), w.data_ptr(),
-                              first.data_ptr(), st), "scatter")
+        if host_out:
+            _ck(L.gg_cuda_scatter_local(src.data_ptr(), cu, base, ws, mode, col_b.data_ptr(),
+                                        w_b.data_ptr(), first.data_ptr(), st), "scatter")
+            col[base:base + cu].copy_(col_b[:cu])
+            w[base:base + cu].copy_(w_b[:cu])
+        else:
+            _ck(L.gg_cuda_scatter(src.data_ptr(), cu, base, ws, mode, col.data_ptr(),
+                                  w.data_ptr(), first.data_ptr(), st), "scatter")
         base += cu
     del keys, alt, temp
+    if host_out:
+        del col_b, w_b
     m = base
     first[n] = m
     offsets = torch.flip(torch.cummin(torch.flip(first, [0]), 0).values, [0]).contiguous()
+    if host_out:
+        del first
+        offsets_h = torch.empty(n + 1, dtype=torch.int64, pin_memory=True)
+        offsets_h.copy_(offsets)
+        offsets = offsets_h
     torch.cuda.synchronize(dev)
     return DeviceGraph(offsets, col[:m], w[:m], n, m, name)
 
 
 def rmat(scale: int, edgefactor: int = 16, seed: int = 1, a: float = 0.57, b: float = 0.19,
          c: float = 0.19, weights: str = "uniform", wseed: int | None = None, device="cuda",
-         bucket_entries: int = 1 << 28) -> DeviceGraph:
+         bucket_entries: int = 1 << 28, host_out: bool = False) -> DeviceGraph:
+    """host_out=True: offsets/col/w come back as pinned CPU tensors (built on the GPU)."""
     n = 1 << scale
     return _edge_graph(1, n, scale, edgefactor * n, seed, a, b, c, weights, wseed, device,
-                       bucket_entries, f"rmat_s{scale}_ef{edgefactor}")
+                       bucket_entries, f"rmat_s{scale}_ef{edgefactor}", host_out)
 
 
 def er(n: int, avg_degree: float = 16.0, seed: int = 1, weights: str = "uniform",

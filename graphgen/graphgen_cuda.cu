@@ -79,14 +79,17 @@ __global__ void k_emit(GenSpec g, int64_t M, int64_t lo, int64_t hi, uint64_t* k
   }
 }
 
+// col/w are written at out_base + j (out_base = base: whole-graph device arrays; 0: a per-bucket
+// buffer that the caller copies out); first[] always gets the global entry index base + j
 __global__ void k_scatter(const uint64_t* __restrict__ keys, int64_t cnt, int64_t base,
-                          uint64_t ws, int mode, int32_t* col, float* w, int64_t* first) {
+                          int64_t out_base, uint64_t ws, int mode, int32_t* col, float* w,
+                          int64_t* first) {
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < cnt; j += stride) {
     const uint64_t k = keys[j];
     const int64_t u = (int64_t)(k >> 32), v = (int64_t)(uint32_t)k;
-    col[base + j] = (int32_t)v;
-    w[base + j] = gg_weight(ws, mode, u, v, 1);
+    col[out_base + j] = (int32_t)v;
+    w[out_base + j] = gg_weight(ws, mode, u, v, 1);
     if (j == 0 || (keys[j - 1] >> 32) != (k >> 32)) first[u] = base + j;
   }
 }
@@ -183,7 +186,16 @@ int gg_cuda_sort_unique(uint64_t* d_keys, uint64_t* d_alt, int64_t cnt, int begi
 int gg_cuda_scatter(const uint64_t* d_keys, int64_t cnt, int64_t base, uint64_t seed, int mode,
                     int32_t* d_col, float* d_w, int64_t* d_first, void* stream) {
   const uint64_t ws = gg_mix64(seed ^ 0x77u);
-  k_scatter<<<grid_of(cnt), 256, 0, (cudaStream_t)stream>>>(d_keys, cnt, base, ws, mode, d_col,
+  k_scatter<<<grid_of(cnt), 256, 0, (cudaStream_t)stream>>>(d_keys, cnt, base, base, ws, mode,
+                                                           d_col, d_w, d_first);
+  return (int)cudaGetLastError();
+}
+
+// same, but col/w of this bucket land at d_col[0..cnt) (for host-side assembly of big graphs)
+int gg_cuda_scatter_local(const uint64_t* d_keys, int64_t cnt, int64_t base, uint64_t seed, int mode,
+                          int32_t* d_col, float* d_w, int64_t* d_first, void* stream) {
+  const uint64_t ws = gg_mix64(seed ^ 0x77u);
+  k_scatter<<<grid_of(cnt), 256, 0, (cudaStream_t)stream>>>(d_keys, cnt, base, 0, ws, mode, d_col,
                                                            d_w, d_first);
   return (int)cudaGetLastError();
 }

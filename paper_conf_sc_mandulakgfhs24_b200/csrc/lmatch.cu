@@ -148,6 +148,10 @@ struct lmatch_graph {
   uint32_t* noffs_lo = nullptr;
   int32_t* atomic_rows = nullptr;
   int64_t n_atomic = 0;
+  // capacities of the buffers sized by the graph's shape (non-empty rows, bins); a reload with a
+  // different degree mix grows them and drops the captured CUDA graph
+  int64_t cap_noffs = -1, cap_nzr = -1, cap_nlo = -1, cap_S[2] = {-1, -1};
+  int64_t cap_bin[2][lm::kBins] = {{-1, -1, -1, -1}, {-1, -1, -1, -1}};
   // state
   uint64_t* best = nullptr;
   uint32_t* bits = nullptr;
@@ -210,6 +214,31 @@ int dmalloc(lmatch_graph* g, T** p, size_t count) {
   return LMATCH_OK;
 }
 
+void drop_graph(lmatch_graph* g);
+
+// (re)allocate *p to hold `need` elements unless it already does; contents are not preserved
+template <class T>
+int ensure(lmatch_graph* g, T** p, int64_t* cap, int64_t need) {
+  if (*p && *cap >= need) return LMATCH_OK;
+  if (*p) {
+    cudaFree(*p);
+    g->device_bytes -= (int64_t)std::max<size_t>((size_t)*cap * sizeof(T), 16);
+    *p = nullptr;
+    drop_graph(g);
+  }
+  *cap = -1;
+  TRY(dmalloc(g, p, (size_t)need));
+  *cap = need;
+  return LMATCH_OK;
+}
+
+void drop_graph(lmatch_graph* g) {
+  if (g->gexec) cudaGraphExecDestroy(g->gexec);
+  if (g->graph) cudaGraphDestroy(g->graph);
+  g->gexec = nullptr;
+  g->graph = nullptr;
+}
+
 int grid_for(int64_t work, int threads, int max_blocks) {
   int64_t b = (work + threads - 1) / threads;
   if (b < 1) b = 1;
@@ -253,15 +282,13 @@ int alloc_all(lmatch_graph* g) {
     }
     CK(cudaStreamCreateWithFlags(&g->cs, cudaStreamNonBlocking));
   }
-  TRY(dmalloc(g, &g->noffs, (size_t)n + 5));
-  TRY(dmalloc(g, &g->nzr, (size_t)n + 8));
+  // per non-empty row buffers (noffs, nzr, noffs_lo, S) are sized in build_index
   g->ntiles = (m + kTile - 1) / kTile;
   TRY(dmalloc(g, &g->tile_nz, (size_t)g->ntiles + 2));
-  TRY(dmalloc(g, &g->noffs_lo, (size_t)n + 9));
-  TRY(dmalloc(g, &g->atomic_rows, (size_t)n + (size_t)g->ntiles + 1));
+  // a tile-crossing row is listed once per tile boundary it crosses: <= ntiles entries
+  TRY(dmalloc(g, &g->atomic_rows, (size_t)g->ntiles + 1));
   TRY(dmalloc(g, &g->best, (size_t)n + 1));
   TRY(dmalloc(g, &g->bits, (size_t)((g->n_global + 31) / 32) + 1));
-  for (int i = 0; i < 2; ++i) TRY(dmalloc(g, &g->S[i], (size_t)n + 1));
   TRY(dmalloc(g, &g->counters, lm::kNumCounters));
   TRY(dmalloc(g, &g->rstate, 1));
   TRY(dmalloc(g, &g->d_rargs, 1));
@@ -284,7 +311,14 @@ int alloc_all(lmatch_graph* g) {
 // Sweep index: non-empty rows (noffs, nzr) + tile -> first row.  Also validates offsets.
 int build_index(lmatch_graph* g, cudaStream_t st) {
   const int64_t n = g->n, m = g->m;
-  if (n == 0) { g->n_nz = 0; return LMATCH_OK; }
+  if (n == 0) {
+    g->n_nz = 0;
+    TRY(ensure(g, &g->noffs, &g->cap_noffs, 5));
+    TRY(ensure(g, &g->nzr, &g->cap_nzr, 8));
+    TRY(ensure(g, &g->noffs_lo, &g->cap_nlo, 9));
+    for (int i = 0; i < 2; ++i) TRY(ensure(g, &g->S[i], &g->cap_S[i], 1));
+    return LMATCH_OK;
+  }
   const int64_t nb = (n + lm::kScanBlock - 1) / lm::kScanBlock;
   int64_t* bs = nullptr;
   int64_t* tot = nullptr;
@@ -294,12 +328,18 @@ int build_index(lmatch_graph* g, cudaStream_t st) {
   CKL();
   lm::k_scan_blocksums<<<1, 1024, 0, st>>>(bs, nb, tot);
   CKL();
-  lm::k_nz_scatter<<<(unsigned)nb, lm::kScanThreads, 0, st>>>(g->offs, n, bs, g->nzr, g->noffs);
-  CKL();
   int64_t h_tot = 0;
   CK(cudaMemcpyAsync(&h_tot, tot, 8, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
   g->n_nz = h_tot;
+  // sized by non-empty rows (R-MAT: ~45% of n); the +slack covers the sweep's TMA window reads,
+  // which round a tile's row window [a, bp+2) out to 4-entry groups
+  TRY(ensure(g, &g->noffs, &g->cap_noffs, h_tot + 5));
+  TRY(ensure(g, &g->nzr, &g->cap_nzr, h_tot + 8));
+  TRY(ensure(g, &g->noffs_lo, &g->cap_nlo, h_tot + 9));
+  for (int i = 0; i < 2; ++i) TRY(ensure(g, &g->S[i], &g->cap_S[i], h_tot + 1));
+  lm::k_nz_scatter<<<(unsigned)nb, lm::kScanThreads, 0, st>>>(g->offs, n, bs, g->nzr, g->noffs);
+  CKL();
   CK(cudaMemcpyAsync(g->noffs + h_tot, &m, 8, cudaMemcpyHostToDevice, st));
   CK(cudaStreamSynchronize(st));
   if (g->ntiles > 0) {
@@ -469,7 +509,6 @@ int make_tensor_map(lmatch_graph* g) {
 
 // frontier bin lists: bin b can never hold more than the vertices of its degree class
 int alloc_bins(lmatch_graph* g, cudaStream_t st) {
-  if (g->F[0].list[0]) return LMATCH_OK;  // reload: same graph shape
   unsigned long long* cnt = nullptr;
   TRY(dmalloc(g, &cnt, lm::kBins));
   CK(cudaMemsetAsync(cnt, 0, 8 * lm::kBins, st));
@@ -481,16 +520,18 @@ int alloc_bins(lmatch_graph* g, cudaStream_t st) {
   CK(cudaMemcpyAsync(h, cnt, sizeof h, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
   cudaFree(cnt);
+  g->device_bytes -= 16;
   for (int i = 0; i < 2; ++i)
-    for (int b = 0; b < lm::kBins; ++b) TRY(dmalloc(g, &g->F[i].list[b], (size_t)h[b] + 1));
+    for (int b = 0; b < lm::kBins; ++b)
+      TRY(ensure(g, &g->F[i].list[b], &g->cap_bin[i][b], (int64_t)h[b] + 1));
   const lm::RoundArgs a = g->rargs();
   CK(cudaMemcpy(g->d_rargs, &a, sizeof a, cudaMemcpyHostToDevice));
   return LMATCH_OK;
 }
 
 int finish_create(lmatch_graph* g, cudaStream_t st) {
-  TRY(alloc_bins(g, st));
   TRY(build_index(g, st));
+  TRY(alloc_bins(g, st));
   if (g->m > 0) {
     // self-loop keys -> 0: the sweep's tile pass over resident graphs, the row-based
     // kernel over out-of-core ones (rows may live in host memory)

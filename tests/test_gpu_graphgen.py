@@ -35,6 +35,13 @@ def test_rmat_many_buckets(ggpu):
     same(graphgen.rmat(13, 16, seed=4), ggpu.rmat(13, 16, seed=4, bucket_entries=1 << 12))
 
 
+def test_rmat_host_output(ggpu):
+    """host_out: bucket-by-bucket assembly in pinned host memory gives the same CSR."""
+    hg = ggpu.rmat(13, 16, seed=4, bucket_entries=1 << 12, host_out=True)
+    assert hg.offsets.device.type == "cpu" and hg.offsets.is_pinned()
+    same(graphgen.rmat(13, 16, seed=4), hg)
+
+
 @pytest.mark.parametrize("n,d", [(1000, 6.0), (1 << 15, 16.0), (12345, 3.5)])
 def test_er_identical(ggpu, n, d):
     same(graphgen.er(n, d, seed=7), ggpu.er(n, d, seed=7))

@@ -175,6 +175,31 @@ def test_reload(lm):
     np.testing.assert_array_equal(b, oracle.greedy(g2).mate)
 
 
+def _same_size_graphs(n=6000, k=2600, seed=5):
+    """Two graphs with equal n and m but opposite degree mixes: (a) one hub with k leaves plus a
+    sparse ring, (b) a ring plus k evenly spread chords (every row short)."""
+    rng = np.random.default_rng(seed)
+    wt = lambda: float(np.float32(1 - rng.random()))
+    ring = [(i, (i + 1) % n, wt()) for i in range(n)]
+    hub = [(0, v, wt()) for v in range(2, 2 + k)]
+    chords = [(i, (i + n // 2) % n, wt()) for i in range(1, 1 + k)]
+    a, b = graphgen.from_edges(n, ring + hub), graphgen.from_edges(n, ring + chords)
+    assert a.m == b.m and a.n == b.n
+    return a, b
+
+
+@pytest.mark.parametrize("round_loop", [0, 3])
+def test_reload_different_degree_mix(lm, round_loop):
+    """Reload with the same n, m but different rows: bin lists and per-row buffers are re-sized
+    (grown) and a captured CUDA graph is rebuilt; results match the oracle each time."""
+    a, b = _same_size_graphs()
+    with lm.Matcher(b, round_loop=round_loop) as M:
+        for g in (b, a, b, a):
+            M.reload(g.offsets, g.col, g.w)
+            mate, st = M.run()
+            np.testing.assert_array_equal(mate, oracle.greedy(g).mate)
+
+
 def test_validation_errors(lm):
     g, _, _, _ = load_golden("k4.txt")
     o, c, w = g.offsets, g.col, g.w
