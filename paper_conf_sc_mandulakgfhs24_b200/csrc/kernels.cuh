@@ -866,6 +866,9 @@ struct RoundArgs {
 // Keys are loaded U at a time per lane and the bitmap words of the candidates (keys above the
 // running max at batch start) are fetched together, so no L2 round trip sits on the loop-carried
 // max.  Zeroed self-loop keys never qualify.  The new pointer goes to best[u] and into the slot.
+#ifndef LM_PROBE
+#define LM_PROBE 0  // bitmap probes per batch: 0 = all candidates in parallel, 1 = descending, 2 = top first
+#endif
 template <int G, int U>
 __device__ __forceinline__ uint64_t scan_row_available(const AdjView adj,
                                                        const uint32_t* __restrict__ bits,
@@ -878,6 +881,36 @@ __device__ __forceinline__ uint64_t scan_row_available(const AdjView adj,
       const int64_t j = j0 + (int64_t)q * G;
       k[q] = j < e ? adj.at(j) : 0ull;
     }
+#if LM_PROBE == 1
+    // descending: probe the lane's largest candidate, drop it if matched, repeat
+    for (int it = 0; it < U; ++it) {
+      uint64_t mx = 0;
+#pragma unroll
+      for (int q = 0; q < U; ++q) mx = (k[q] > b && k[q] > mx) ? k[q] : mx;
+      if (!mx) break;
+      const uint32_t v = (uint32_t)mx;
+      if (!((bits[v >> 5] >> (v & 31)) & 1u)) { b = mx; break; }
+#pragma unroll
+      for (int q = 0; q < U; ++q) k[q] = k[q] == mx ? 0ull : k[q];
+    }
+#else
+#if LM_PROBE == 2
+    {
+      // the lane's largest candidate first: if available it is the lane's answer for the batch
+      uint64_t mx = 0;
+#pragma unroll
+      for (int q = 0; q < U; ++q) mx = (k[q] > b && k[q] > mx) ? k[q] : mx;
+      if (mx) {
+        const uint32_t v = (uint32_t)mx;
+        if (!((bits[v >> 5] >> (v & 31)) & 1u)) {
+          b = mx;
+          continue;
+        }
+#pragma unroll
+        for (int q = 0; q < U; ++q) k[q] = k[q] == mx ? 0ull : k[q];
+      }
+    }
+#endif
     uint32_t wd[U];
 #pragma unroll
     for (int q = 0; q < U; ++q) wd[q] = k[q] > b ? bits[(uint32_t)k[q] >> 5] : 0xffffffffu;
@@ -886,6 +919,7 @@ __device__ __forceinline__ uint64_t scan_row_available(const AdjView adj,
       const uint32_t v = (uint32_t)k[q];
       if (!((wd[q] >> (v & 31)) & 1u) && k[q] > b) b = k[q];
     }
+#endif
   }
   return b;
 }

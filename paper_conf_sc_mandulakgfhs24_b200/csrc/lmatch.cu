@@ -102,8 +102,6 @@ constexpr int64_t kPersistentBelow = LM_PERSIST_BELOW;
 constexpr int kFinBlocks = 2368;  // 16 x 148 SMs: fixed => deterministic fp64 summation order
 constexpr int kFinThreads = 256;
 
-int num_sms_cached = 0;
-
 }  // namespace
 
 struct lmatch_graph {
@@ -481,6 +479,7 @@ int upload_device(lmatch_graph* g, const int64_t* d_offsets, const int32_t* d_co
   return LMATCH_OK;
 }
 
+#if LM_SWEEP_IMPL == 2
 int make_tensor_map(lmatch_graph* g) {
   static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
   if (!encode) {
@@ -506,6 +505,7 @@ int make_tensor_map(lmatch_graph* g) {
   }
   return LMATCH_OK;
 }
+#endif
 
 // frontier bin lists: bin b can never hold more than the vertices of its degree class
 int alloc_bins(lmatch_graph* g, cudaStream_t st) {
