@@ -866,22 +866,79 @@ struct RoundArgs {
 // Keys are loaded U at a time per lane and the bitmap words of the candidates (keys above the
 // running max at batch start) are fetched together, so no L2 round trip sits on the loop-carried
 // max.  Zeroed self-loop keys never qualify.  The new pointer goes to best[u] and into the slot.
+#ifndef LM_PROBE3_MIN_G
+#define LM_PROBE3_MIN_G 32  // two-phase probing only for warp and CTA rows (measured: it slows
+                            // the 1- and 8-lane bins, speeds up the 32-lane and CTA bins ~10%)
+#endif
 #ifndef LM_PROBE
-#define LM_PROBE 0  // bitmap probes per batch: 0 = all candidates in parallel, 1 = descending, 2 = top first
+#define LM_PROBE 3  // bitmap probes per batch: 0 = all candidates in parallel, 1 = descending, 2 = top first,
+                    // 3 = two-phase (lane tops, then only keys above the group's best)
 #endif
 template <int G, int U>
 __device__ __forceinline__ uint64_t scan_row_available(const AdjView adj,
                                                        const uint32_t* __restrict__ bits,
-                                                       int64_t s, int64_t e, int gl) {
+                                                       int64_t s, int64_t e, int gl,
+                                                       unsigned rmask) {
   uint64_t b = 0;
-  for (int64_t j0 = s + gl; j0 < e; j0 += (int64_t)G * U) {
+  (void)rmask;
+  // batch loop with a group-uniform trip count (the group votes inside it)
+  for (int64_t jb = s; jb < e; jb += (int64_t)G * U) {
+    const int64_t j0 = jb + gl;
     uint64_t k[U];
 #pragma unroll
     for (int q = 0; q < U; ++q) {
       const int64_t j = j0 + (int64_t)q * G;
       k[q] = j < e ? adj.at(j) : 0ull;
     }
-#if LM_PROBE == 1
+#if LM_PROBE == 3
+    if (G >= LM_PROBE3_MIN_G) {
+    // Two-phase probe.  Phase 1: every lane probes only its largest candidate; C = the max of
+    // the available ones over the reduction group (rmask: the lanes sharing this row, or the
+    // warp for CTA rows).  Keys <= max(b, C) cannot be the answer, so phase 2 probes only the
+    // keys above it held by lanes whose top candidate was matched -- usually none.  b stays
+    // uniform over the reduction group.
+    {
+      uint64_t mx = 0;
+#pragma unroll
+      for (int q = 0; q < U; ++q) mx = (k[q] > b && k[q] > mx) ? k[q] : mx;
+      bool avail = false;
+      if (mx) avail = !((bits[(uint32_t)mx >> 5] >> ((uint32_t)mx & 31)) & 1u);
+      uint64_t c = avail ? mx : 0ull;
+      if (G > 1) c = group_max_key(c, rmask);
+      const uint64_t bb = c > b ? c : b;
+      bool need = false;
+      if (mx && !avail) {
+#pragma unroll
+        for (int q = 0; q < U; ++q) need |= (k[q] > bb && k[q] != mx);
+      }
+      const bool any = (G > 1) ? (__ballot_sync(rmask, need) & rmask) != 0u : need;
+      b = bb;
+      if (any) {
+        uint32_t wd[U];
+#pragma unroll
+        for (int q = 0; q < U; ++q)
+          wd[q] = (need && k[q] > bb && k[q] != mx) ? bits[(uint32_t)k[q] >> 5] : 0xffffffffu;
+        uint64_t c2 = 0;
+#pragma unroll
+        for (int q = 0; q < U; ++q) {
+          const uint32_t v = (uint32_t)k[q];
+          if (!((wd[q] >> (v & 31)) & 1u) && k[q] > c2) c2 = k[q];
+        }
+        if (G > 1) c2 = group_max_key(c2, rmask);
+        b = c2 > b ? c2 : b;
+      }
+    }
+    } else {
+      uint32_t wd[U];
+#pragma unroll
+      for (int q = 0; q < U; ++q) wd[q] = k[q] > b ? bits[(uint32_t)k[q] >> 5] : 0xffffffffu;
+#pragma unroll
+      for (int q = 0; q < U; ++q) {
+        const uint32_t v = (uint32_t)k[q];
+        if (!((wd[q] >> (v & 31)) & 1u) && k[q] > b) b = k[q];
+      }
+    }
+#elif LM_PROBE == 1
     // descending: probe the lane's largest candidate, drop it if matched, repeat
     for (int it = 0; it < U; ++it) {
       uint64_t mx = 0;
@@ -938,7 +995,7 @@ __device__ __forceinline__ void point_bin_body(ulonglong2* __restrict__ list, in
     const ulonglong2 e = list[i];
     int64_t s, en;
     row_range(e, offs, vbase, &s, &en);
-    const uint64_t b = group_max_key(scan_row_available<G, U>(adj, bits, s, en, gl), gmask);
+    const uint64_t b = group_max_key(scan_row_available<G, U>(adj, bits, s, en, gl, gmask), gmask);
     if (gl == 0) {
       const uint32_t u = (uint32_t)e.x;
       best[u - vbase] = b;
@@ -956,6 +1013,252 @@ __global__ void k_point_bin(ulonglong2* __restrict__ list, const unsigned long l
                        (int64_t)gridDim.x * blockDim.x);
 }
 
+// Software-pipelined variant for the big host-driven rounds (grid = one resident wave, so every
+// group walks many rows): the keys of the NEXT batch (the next batch of the same row, or the
+// first batch of the group's next row, whose list entry was prefetched one row earlier) are
+// loaded before the bitmap probes of the current batch, so a DRAM round trip and an L2 round
+// trip overlap instead of adding up per row.  Same result as point_bin_body (u64 max).
+template <int G, int U>
+__device__ __forceinline__ void load_batch(const AdjView adj, int64_t j0, int64_t e,
+                                           uint64_t (&k)[U]) {
+#pragma unroll
+  for (int q = 0; q < U; ++q) {
+    const int64_t j = j0 + (int64_t)q * G;
+    k[q] = j < e ? adj.at(j) : 0ull;
+  }
+}
+template <int U>
+__device__ __forceinline__ uint64_t probe_batch(const uint32_t* __restrict__ bits,
+                                                const uint64_t (&k)[U], uint64_t b) {
+  uint32_t wd[U];
+#pragma unroll
+  for (int q = 0; q < U; ++q) wd[q] = k[q] > b ? bits[(uint32_t)k[q] >> 5] : 0xffffffffu;
+#pragma unroll
+  for (int q = 0; q < U; ++q) {
+    const uint32_t v = (uint32_t)k[q];
+    if (!((wd[q] >> (v & 31)) & 1u) && k[q] > b) b = k[q];
+  }
+  return b;
+}
+// Two-phase probe of one batch (group-uniform b): lanes probe their top candidate; only keys
+// above the group's best available top are probed in a second step.
+#ifndef LM_PIPE_PROBE
+#define LM_PIPE_PROBE 0
+#endif
+template <int G, int U>
+__device__ __forceinline__ uint64_t probe_batch2(const uint32_t* __restrict__ bits,
+                                                 const uint64_t (&k)[U], uint64_t b,
+                                                 unsigned gmask) {
+  uint64_t mx = 0;
+#pragma unroll
+  for (int q = 0; q < U; ++q) mx = (k[q] > b && k[q] > mx) ? k[q] : mx;
+  bool avail = false;
+  if (mx) avail = !((bits[(uint32_t)mx >> 5] >> ((uint32_t)mx & 31)) & 1u);
+  uint64_t c = avail ? mx : 0ull;
+  if (G > 1) c = group_max_key(c, gmask);
+  const uint64_t bb = c > b ? c : b;
+  bool need = false;
+  if (mx && !avail) {
+#pragma unroll
+    for (int q = 0; q < U; ++q) need |= (k[q] > bb && k[q] != mx);
+  }
+  const bool any = G > 1 ? (__ballot_sync(gmask, need) & gmask) != 0u : need;
+  if (!any) return bb;
+  uint32_t wd[U];
+#pragma unroll
+  for (int q = 0; q < U; ++q)
+    wd[q] = (need && k[q] > bb && k[q] != mx) ? bits[(uint32_t)k[q] >> 5] : 0xffffffffu;
+  uint64_t c2 = 0;
+#pragma unroll
+  for (int q = 0; q < U; ++q) {
+    const uint32_t v = (uint32_t)k[q];
+    if (!((wd[q] >> (v & 31)) & 1u) && k[q] > c2) c2 = k[q];
+  }
+  if (G > 1) c2 = group_max_key(c2, gmask);
+  return c2 > bb ? c2 : bb;
+}
+
+template <int G, int U>
+__device__ __forceinline__ void point_pipe_body(ulonglong2* __restrict__ list, int64_t cnt,
+                                                const int64_t* __restrict__ offs, const AdjView adj,
+                                                const uint32_t* __restrict__ bits,
+                                                uint64_t* __restrict__ best, int64_t vbase,
+                                                int64_t gtid, int64_t gthreads) {
+  const int lane = threadIdx.x & 31;
+  const int gl = lane & (G - 1);
+  const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
+  const int64_t ng = gthreads / G;
+  constexpr int64_t B = (int64_t)G * U;
+  int64_t li = gtid / G;  // row of the load stream (group-uniform)
+  if (li >= cnt) return;
+  ulonglong2 le = list[li];
+  ulonglong2 pf = li + ng < cnt ? list[li + ng] : make_ulonglong2(0ull, 0ull);
+  int64_t ls, lend;
+  row_range(le, offs, vbase, &ls, &lend);
+  uint64_t kc[U];
+  load_batch<G, U>(adj, ls + gl, lend, kc);
+  int64_t ci = li;
+  uint32_t cu = (uint32_t)le.x;
+  bool clast = ls + B >= lend;
+  int64_t ljb = ls + B;  // next batch base of the load row
+  uint64_t b = 0;
+  for (;;) {
+    uint64_t kn[U];
+    int64_t ni = -1;
+    uint32_t nu = 0;
+    bool nlast = false;
+    if (ljb < lend) {  // next batch of the same row
+      load_batch<G, U>(adj, ljb + gl, lend, kn);
+      ni = li;
+      nu = (uint32_t)le.x;
+      nlast = ljb + B >= lend;
+      ljb += B;
+    } else if (li + ng < cnt) {  // first batch of the next row
+      li += ng;
+      le = pf;
+      pf = li + ng < cnt ? list[li + ng] : make_ulonglong2(0ull, 0ull);
+      row_range(le, offs, vbase, &ls, &lend);
+      load_batch<G, U>(adj, ls + gl, lend, kn);
+      ni = li;
+      nu = (uint32_t)le.x;
+      nlast = ls + B >= lend;
+      ljb = ls + B;
+    }
+#if LM_PIPE_PROBE == 3
+    b = probe_batch2<G, U>(bits, kc, b, gmask);  // group-uniform
+    if (clast) {
+      const uint64_t r = b;
+#else
+    b = probe_batch<U>(bits, kc, b);
+    if (clast) {
+      const uint64_t r = G > 1 ? group_max_key(b, gmask) : b;
+#endif
+      if (gl == 0) {
+        best[cu - vbase] = r;
+        list[ci].x = make_pair(cu, r ? (uint32_t)r : kNoPtr);
+      }
+      b = 0;
+    }
+    if (ni < 0) break;
+#pragma unroll
+    for (int q = 0; q < U; ++q) kc[q] = kn[q];
+    ci = ni;
+    cu = nu;
+    clast = nlast;
+  }
+}
+template <int G, int U>
+__global__ void __launch_bounds__(256)
+    k_point_pipe(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
+                 const int64_t* __restrict__ offs, const AdjView adj,
+                 const uint32_t* __restrict__ bits, uint64_t* __restrict__ best, int64_t vbase) {
+  point_pipe_body<G, U>(list, (int64_t)*cnt_ptr, offs, adj, bits, best, vbase,
+                        (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
+                        (int64_t)gridDim.x * blockDim.x);
+}
+
+// ---------------------------------------------------------------------------------------------
+// Asynchronous-copy variant for the big host-driven rounds.  Each lane keeps a private ring of
+// S stages x U keys in shared memory filled with cp.async (LDGSTS, zero-fill past the row end),
+// running S-1 (row, batch) items ahead of the bitmap probes, so the bytes in flight per SM no
+// longer depend on registers (the register-staged kernels top out near 36 KB in flight per SM,
+// ~3 TB/s).  A lane only reads keys it copied itself: cp.async.wait_group is the only sync.
+// Layout [stage][q][thread] keeps the 8-byte shared accesses of a warp conflict-free.
+__device__ __forceinline__ void cp_async8(void* sdst, const void* gsrc, uint32_t src_bytes) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 8, %2;" ::"r"(smem_u32(sdst)), "l"(gsrc),
+               "r"(src_bytes)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+template <int G, int U, int S>
+__global__ void __launch_bounds__(256)
+    k_point_async(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
+                  const int64_t* __restrict__ offs, const uint64_t* __restrict__ adj,
+                  const uint32_t* __restrict__ bits, uint64_t* __restrict__ best, int64_t vbase) {
+  extern __shared__ __align__(16) uint64_t sk[];  // [S][U][256]
+  const int tid = threadIdx.x;
+  const int lane = tid & 31;
+  const int gl = lane & (G - 1);
+  const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
+  const int64_t cnt = (int64_t)*cnt_ptr;
+  const int64_t ng = ((int64_t)gridDim.x * blockDim.x) / G;
+  constexpr int64_t B = (int64_t)G * U;
+  // load stream (group-uniform): current row li, next batch base ljb, row end lend
+  int64_t li = ((int64_t)blockIdx.x * blockDim.x + tid) / G;
+  bool lvalid = li < cnt;
+  int64_t ljb = 0, lend = 0;
+  uint32_t lu = 0;
+  ulonglong2 pf = make_ulonglong2(0ull, 0ull);
+  if (lvalid) {
+    const ulonglong2 e = list[li];
+    row_range(e, offs, vbase, &ljb, &lend);
+    lu = (uint32_t)e.x;
+    if (li + ng < cnt) pf = list[li + ng];
+  }
+  // per-stage tags (registers: every index below is a compile-time constant after unrolling)
+  int64_t tci[S];
+  uint32_t tu[S];
+  bool tlast[S], tval[S];
+  auto issue = [&](int st) {
+    if (lvalid && ljb >= lend) {  // row done: next row of this group
+      li += ng;
+      if (li < cnt) {
+        const ulonglong2 e = pf;
+        pf = li + ng < cnt ? list[li + ng] : make_ulonglong2(0ull, 0ull);
+        row_range(e, offs, vbase, &ljb, &lend);
+        lu = (uint32_t)e.x;
+      } else {
+        lvalid = false;
+      }
+    }
+    tval[st] = lvalid;
+    if (lvalid) {
+#pragma unroll
+      for (int q = 0; q < U; ++q) {
+        const int64_t j = ljb + gl + (int64_t)q * G;
+        const bool in = j < lend;
+        cp_async8(&sk[((size_t)st * U + q) * 256 + tid], in ? adj + j : adj, in ? 8u : 0u);
+      }
+      tci[st] = li;
+      tu[st] = lu;
+      tlast[st] = ljb + B >= lend;
+      ljb += B;
+    }
+    cp_async_commit();  // also when empty: keeps the group count uniform
+  };
+#pragma unroll
+  for (int st = 0; st < S - 1; ++st) issue(st);
+  uint64_t b = 0;
+  for (;;) {
+#pragma unroll
+    for (int st = 0; st < S; ++st) {
+      issue((st + S - 1) % S);  // the stage processed in the previous step
+      cp_async_wait<S - 1>();   // => stage st has landed
+      if (!tval[st]) goto done;
+      {
+        uint64_t k[U];
+#pragma unroll
+        for (int q = 0; q < U; ++q) k[q] = sk[((size_t)st * U + q) * 256 + tid];
+        b = probe_batch<U>(bits, k, b);
+      }
+      if (tlast[st]) {
+        const uint64_t r = G > 1 ? group_max_key(b, gmask) : b;
+        if (gl == 0) {
+          best[tu[st] - vbase] = r;
+          list[tci[st]].x = make_pair(tu[st], r ? (uint32_t)r : kNoPtr);
+        }
+        b = 0;
+      }
+    }
+  }
+done:
+  cp_async_wait<0>();
+}
+
 template <int THREADS, int U>
 __device__ __forceinline__ void point_bin_cta_body(ulonglong2* __restrict__ list, int64_t cnt,
                                                    const int64_t* __restrict__ offs,
@@ -968,7 +1271,7 @@ __device__ __forceinline__ void point_bin_cta_body(ulonglong2* __restrict__ list
     const ulonglong2 e = list[i];
     int64_t s, en;
     row_range(e, offs, vbase, &s, &en);
-    uint64_t b = scan_row_available<THREADS, U>(adj, bits, s, en, threadIdx.x);
+    uint64_t b = scan_row_available<THREADS, U>(adj, bits, s, en, threadIdx.x, 0xffffffffu);
     b = group_max_key(b, 0xffffffffu);
     if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = b;
     __syncthreads();

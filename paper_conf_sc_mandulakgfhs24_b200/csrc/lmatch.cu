@@ -23,6 +23,7 @@
 #include "../../include/lmatch.h"
 #include "kernels.cuh"
 
+
 namespace {
 
 thread_local char g_err[512] = "";
@@ -97,6 +98,47 @@ constexpr int64_t kPersistentBelow = LM_PERSIST_BELOW;
 #ifndef LM_B2_G
 #define LM_B2_G 32
 #define LM_B2_U 4
+#endif
+
+// host-driven rounds: software-pipelined pointer kernels (one resident wave) per bin: bit b of
+// LM_PIPE set = bin b uses k_point_pipe<LM_Pb_G, LM_Pb_U>
+#ifndef LM_PIPE
+#define LM_PIPE 1  // measured (R-MAT s26): pipelining helps the thread-per-row bin only (-10 to -20%)
+#endif
+#ifndef LM_P0_G
+#define LM_P0_G 1
+#define LM_P0_U 8
+#endif
+#ifndef LM_P1_G
+#define LM_P1_G 8
+#define LM_P1_U 4
+#endif
+#ifndef LM_P2_G
+#define LM_P2_G 32
+#define LM_P2_U 4
+#endif
+// bit b of LM_ASYNC set = bin b uses k_point_async<LM_Ab_G, LM_Ab_U, LM_ASYNC_S> (resident
+// adjacency only; takes precedence over LM_PIPE)
+#ifndef LM_ASYNC
+#define LM_ASYNC 0
+#endif
+#ifndef LM_ASYNC_S
+#define LM_ASYNC_S 4
+#endif
+#ifndef LM_A0_G
+#define LM_A0_G 1
+#define LM_A0_U 8
+#endif
+#ifndef LM_A1_G
+#define LM_A1_G 8
+#define LM_A1_U 4
+#endif
+#ifndef LM_A2_G
+#define LM_A2_G 32
+#define LM_A2_U 4
+#endif
+#ifndef LM_PIPE_WAVES
+#define LM_PIPE_WAVES 1
 #endif
 
 constexpr int kFinBlocks = 2368;  // 16 x 148 SMs: fixed => deterministic fp64 summation order
@@ -860,9 +902,40 @@ static int seq_body(lmatch_graph* g, cudaStream_t st, int cur, const int64_t* nF
   const unsigned long long* cF = g->counters + lm::cnt_F(cur, 0);
   int64_t nF = 0;
   for (int b = 0; b < lm::kBins; ++b) nF += nFb[b];
-  if (nFb[0]) { lm::k_point_bin<LM_B0_G, LM_B0_U><<<grid_for(nFb[0] * LM_B0_G, 256, 65536), 256, 0, st>>>(Fb.list[0], cF + 0, g->offs, av, g->bits, g->best, g->v0); CKL(); ++*launches; }
-  if (nFb[1]) { lm::k_point_bin<LM_B1_G, LM_B1_U><<<grid_for(nFb[1] * LM_B1_G, 256, 65536), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, av, g->bits, g->best, g->v0); CKL(); ++*launches; }
-  if (nFb[2]) { lm::k_point_bin<LM_B2_G, LM_B2_U><<<grid_for(nFb[2] * LM_B2_G, 256, 65536), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, av, g->bits, g->best, g->v0); CKL(); ++*launches; }
+#define PIPE_OR_BIN(b, PG, PU, BG, BU, AG, AU)                                                      \
+  if (nFb[b]) {                                                                                   \
+    if ((LM_ASYNC & (1 << b)) && !g->streaming) {                                                 \
+      constexpr size_t smem = (size_t)LM_ASYNC_S * AU * 256 * 8;                                  \
+      static int occ = 0;                                                                         \
+      if (!occ) {                                                                                 \
+        CK(cudaFuncSetAttribute(lm::k_point_async<AG, AU, LM_ASYNC_S>,                            \
+                                cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));         \
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, lm::k_point_async<AG, AU, LM_ASYNC_S>, 256, smem)); \
+        if (occ < 1) occ = 1;                                                                     \
+      }                                                                                           \
+      const int64_t wave = (int64_t)occ * g->num_sms;                                             \
+      lm::k_point_async<AG, AU, LM_ASYNC_S><<<(unsigned)std::min<int64_t>(wave, (nFb[b] * AG + 255) / 256), 256, smem, st>>>( \
+          Fb.list[b], cF + b, g->offs, g->adj, g->bits, g->best, g->v0);                          \
+    } else if (LM_PIPE & (1 << b)) {                                                              \
+      static int occ = 0;                                                                         \
+      if (!occ) {                                                                                 \
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, lm::k_point_pipe<PG, PU>, 256, 0)); \
+        if (occ < 1) occ = 1;                                                                     \
+      }                                                                                           \
+      const int64_t wave = (int64_t)occ * g->num_sms * LM_PIPE_WAVES;                              \
+      lm::k_point_pipe<PG, PU><<<(unsigned)std::min<int64_t>(wave, (nFb[b] * PG + 255) / 256), 256, 0, st>>>( \
+          Fb.list[b], cF + b, g->offs, av, g->bits, g->best, g->v0);                              \
+    } else {                                                                                      \
+      lm::k_point_bin<BG, BU><<<grid_for(nFb[b] * BG, 256, 65536), 256, 0, st>>>(                 \
+          Fb.list[b], cF + b, g->offs, av, g->bits, g->best, g->v0);                              \
+    }                                                                                             \
+    CKL();                                                                                        \
+    ++*launches;                                                                                  \
+  }
+  PIPE_OR_BIN(0, LM_P0_G, LM_P0_U, LM_B0_G, LM_B0_U, LM_A0_G, LM_A0_U)
+  PIPE_OR_BIN(1, LM_P1_G, LM_P1_U, LM_B1_G, LM_B1_U, LM_A1_G, LM_A1_U)
+  PIPE_OR_BIN(2, LM_P2_G, LM_P2_U, LM_B2_G, LM_B2_U, LM_A2_G, LM_A2_U)
+#undef PIPE_OR_BIN
   if (nFb[3]) { lm::k_point_bin_cta<256, 4><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); ++*launches; }
   lm::k_match_bins<<<grid_for(nF, 256, 65536), 256, 0, st>>>(Fb, cF, g->best, g->bits);
   CKL();

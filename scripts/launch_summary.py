@@ -12,7 +12,7 @@ for r in rows[hdr_i + 1:]:
     name = re.sub(r"\(.*", "", r[ik]).replace("void ", "")
     v = float(r[iv].replace(",", ""))
     unit = r[h.index("Metric Unit")]
-    us = v / 1000 if unit == "nsecond" else (v if unit == "usecond" else v * 1000)
+    us = {"nsecond": v / 1e3, "ns": v / 1e3, "usecond": v, "us": v, "msecond": v * 1e3, "ms": v * 1e3, "second": v * 1e6, "s": v * 1e6}.get(unit, v)
     seq.append((int(r[iid]), name, us))
     a = agg.setdefault(name, [0, 0.0])
     a[0] += 1
