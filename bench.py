@@ -55,6 +55,7 @@ def parse():
                    help="out-of-core (A8): cap the HBM-resident adjacency; the rest is streamed "
                         "from pinned host memory in round 1 and read zero-copy afterwards")
     p.add_argument("--stream-chunk", type=int, default=0, help="entries per streamed chunk (0 = default)")
+    p.add_argument("--prune", action="store_true", help="A7 in-place pruning (lmatch_opts.prune)")
     p.add_argument("--partitioned", action="store_true",
                    help="use the 1-D partitioned path even at N=1 (it is always used for N>1)")
     return p.parse_args()
@@ -118,6 +119,8 @@ def workload_config(a, scale, n, m):
            "seed": a.seed}
     if a.workload in ("rmat", "er"):
         cfg["edgefactor"] = a.edgefactor
+    if getattr(a, "prune", False):
+        cfg["prune"] = True
     return cfg
 
 
@@ -415,7 +418,8 @@ def main():
     # handle built from the device CSR (or, when both do not fit in HBM, from the pinned host
     # CSR); create is untimed: P:179 excludes I/O, allocation, CSR construction and the transfer
     opts = lm.make_opts(validate_level=1, timing=1,
-                        hbm_budget_bytes=int(a.hbm_budget_gb * 1e9), stream_chunk=a.stream_chunk)
+                        hbm_budget_bytes=int(a.hbm_budget_gb * 1e9), stream_chunk=a.stream_chunk,
+                        prune=a.prune)
     pinned_host = d_off is None
     if pinned_host:
         h = lm.lmatch_create_ex(g.offsets, g.col, g.w, n, m, opts)

@@ -90,7 +90,15 @@ typedef struct lmatch_opts {
                                  trips); 1 = host-driven per-round launches only; 2 = persistent
                                  kernel for every round after round 1; 3 = CUDA graph {round 1,
                                  persistent kernel}.  Out-of-core: 3 behaves as 2. */
-  int32_t reserved[11];
+  int32_t prune;              /* 1 = A7 in-place pruning (not in the paper): a
+                                 frontier row that fits one pointer batch (<= 8 / 64 / 128
+                                 entries for the 1/8/32-lane bins) is partitioned in place,
+                                 entries with an unmatched neighbour first, and later rounds of
+                                 the same run scan only that prefix.  The adjacency stays a
+                                 per-row permutation of the input, so the result and later runs
+                                 are unchanged.  Ignored for out-of-core and partition handles.
+                                 0 = default (off: measured slower on R-MAT) */
+  int32_t reserved[10];
 } lmatch_opts;
 
 /* Filled by lmatch_run / lmatch_run_device when non-NULL. */

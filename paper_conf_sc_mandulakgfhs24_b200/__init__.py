@@ -43,7 +43,8 @@ class Opts(ctypes.Structure):
         ("validate_level", ctypes.c_int32), ("timing", ctypes.c_int32),
         ("max_rounds", ctypes.c_int64), ("upload_chunk", ctypes.c_int64),
         ("hbm_budget_bytes", ctypes.c_int64), ("stream_chunk", ctypes.c_int64),
-        ("round_loop", ctypes.c_int32), ("reserved", ctypes.c_int32 * 11),
+        ("round_loop", ctypes.c_int32), ("prune", ctypes.c_int32),
+        ("reserved", ctypes.c_int32 * 10),
     ]
 
 
@@ -239,7 +240,7 @@ class Matcher:
     def __init__(self, offsets=None, col=None, w=None, *, handle: int | None = None,
                  validate_level: int = 1, timing: bool = False, upload_chunk: int = 0,
                  max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
-                 round_loop: int = 0):
+                 round_loop: int = 0, prune: bool = False):
         self.h = None
         if handle is not None:
             self.h = handle
@@ -249,7 +250,7 @@ class Matcher:
             self.h = lmatch_create_ex(offsets, col, w,
                                       opts=make_opts(validate_level, timing, upload_chunk,
                                                      max_rounds, hbm_budget_bytes, stream_chunk,
-                                                     round_loop))
+                                                     round_loop, prune))
         self.info = lmatch_info(self.h)
 
     @classmethod
@@ -292,12 +293,13 @@ class Matcher:
 
 def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int = 0,
               max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
-              round_loop: int = 0) -> Opts:
+              round_loop: int = 0, prune: bool = False) -> Opts:
     """round_loop (include/lmatch.h): 0 = hybrid (work-sized launches, then one persistent kernel
     for the tail; default), 1 = host-driven launches only, 2 = persistent kernel after round 1,
     3 = CUDA graph {round 1, persistent kernel}."""
     o = Opts()
     o.round_loop = int(round_loop)
+    o.prune = int(bool(prune))
     o.hbm_budget_bytes = int(hbm_budget_bytes)
     o.stream_chunk = int(stream_chunk)
     o.validate_level = int(validate_level)

@@ -331,12 +331,22 @@ __global__ void k_tile_rows(const int64_t* __restrict__ noffs, int64_t n_nz, int
 // per-run reset: matched bitmap, counters, and best[] of the rows the sweep merges with
 // atomicMax (rows crossing a sweep-tile boundary; listed at create time).
 // =============================================================================================
+struct RoundState;
+__device__ __forceinline__ uint32_t round_tag(const RoundState* st);
 __global__ void k_reset(uint32_t* bits, int64_t nwords, uint64_t* best,
                         const int32_t* __restrict__ atomic_rows, int64_t n_atomic,
-                        unsigned long long* counters, int ncounters) {
+                        unsigned long long* counters, int ncounters, uint32_t* live,
+                        int64_t n_live, const RoundState* st) {
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   for (int64_t i = tid; i < nwords; i += stride) bits[i] = 0u;
+  // A7 pruning: live[u] = tag << 16 | live count is valid only under this run's tag; when the
+  // 16-bit tag is about to wrap (or on the first run) old entries could alias, so clear them
+  if (live) {
+    const uint32_t t = round_tag(st);
+    if (t == 0u || t == 0xffffu)
+      for (int64_t i = tid; i < n_live; i += stride) live[i] = 0u;
+  }
   for (int64_t i = tid; i < n_atomic; i += stride) best[atomic_rows[i]] = 0ull;
   if (tid < ncounters) counters[tid] = 0ull;
 }
@@ -852,13 +862,19 @@ struct RoundState {
   long long log_len;     // rows written to the per-round log
   long long log_cap;
   unsigned long long swept_prev;
+  uint32_t tag;          // per-run tag of the A7 live counts (1..65535, advanced by k_round_init)
+  uint32_t pad;
 };
+__device__ __forceinline__ uint32_t round_tag(const RoundState* st) {
+  return *reinterpret_cast<const volatile uint32_t*>(&st->tag);
+}
 struct RoundArgs {
   uint64_t* S[2];
   Bins F[2];
   unsigned long long* cnt;  // kNumCounters; set s = cnt_S(s), cnt_F(s, b)
   RoundState* st;
   long long* log;           // [log_cap][3]: |F_r|, |S_r| + |F_r|, E(F_r)
+  uint32_t* live;           // A7 pruning: per-vertex live counts (nullptr = pruning off)
 };
 
 // A2 pointer phase on the frontier (rounds >= 2): G lanes per vertex (degree-binned).
@@ -981,12 +997,73 @@ __device__ __forceinline__ uint64_t scan_row_available(const AdjView adj,
   return b;
 }
 
+// A7 in-place pruning (opt-in, lmatch_opts.prune) of a row that fits ONE batch
+// of the group (deg <= G*U): every key is probed; the group partitions the row in place --
+// available entries first (index order), then the dead ones (matched neighbour or zeroed
+// self-loop) -- and records live[u] = tag << 16 | #available.  The row stays a permutation of
+// itself, so later runs (whose round-1 sweep reads whole rows) are unaffected; later rounds of
+// THIS run scan only the live prefix (compact_body).  Dead entries can never become available
+// again (available sets only shrink, R3), so the pointer result is unchanged.  Keys
+// are read with ld.global.cg: a pruned row may be re-read by another SM in the same
+// (persistent) kernel, and the non-coherent L1 path could return the pre-permutation bytes.
 template <int G, int U>
+__device__ __forceinline__ uint64_t prune_row(const AdjView adj, const uint32_t* __restrict__ bits,
+                                              int64_t s, int64_t en, int gl, unsigned gmask,
+                                              uint32_t* __restrict__ live, uint32_t tag,
+                                              int64_t lu) {
+  const int L = (int)(en - s);
+  uint64_t* row = adj.ptr(s);
+  uint64_t k[U];
+#pragma unroll
+  for (int q = 0; q < U; ++q) {
+    const int r = gl + q * G;
+    k[q] = r < L ? __ldcg(reinterpret_cast<const unsigned long long*>(row + r)) : 0ull;
+  }
+  uint32_t wd[U];
+#pragma unroll
+  for (int q = 0; q < U; ++q) wd[q] = k[q] ? bits[(uint32_t)k[q] >> 5] : 0xffffffffu;
+  bool sv[U];
+  uint64_t b = 0;
+#pragma unroll
+  for (int q = 0; q < U; ++q) {
+    const uint32_t v = (uint32_t)k[q];
+    sv[q] = k[q] != 0ull && !((wd[q] >> (v & 31)) & 1u);
+    if (sv[q] && k[q] > b) b = k[q];
+  }
+  if (G > 1) b = group_max_key(b, gmask);
+  const int gbase = (threadIdx.x & 31) & ~(G - 1);
+  unsigned msk[U];
+  int K = 0;
+#pragma unroll
+  for (int q = 0; q < U; ++q) {
+    msk[q] = G > 1 ? (__ballot_sync(gmask, sv[q]) & gmask) >> gbase : (sv[q] ? 1u : 0u);
+    K += __popc(msk[q]);
+  }
+  if (K < L) {
+    int cs = 0;  // available entries before batch column q
+#pragma unroll
+    for (int q = 0; q < U; ++q) {
+      const int r = gl + q * G;
+      const int rank = cs + __popc(msk[q] & ((1u << gl) - 1u));  // available entries before r
+      if (r < L) {
+        const int np = sv[q] ? rank : K + (r - rank);
+        if (np != r) row[np] = k[q];
+      }
+      cs += __popc(msk[q]);
+    }
+    if (gl == 0) live[lu] = (tag << 16) | (uint32_t)K;
+  }
+  return b;
+}
+
+template <int G, int U, bool PRUNE = false>
 __device__ __forceinline__ void point_bin_body(ulonglong2* __restrict__ list, int64_t cnt,
                                                const int64_t* __restrict__ offs, const AdjView adj,
                                                const uint32_t* __restrict__ bits,
                                                uint64_t* __restrict__ best, int64_t vbase,
-                                               int64_t gtid, int64_t gthreads) {
+                                               int64_t gtid, int64_t gthreads,
+                                               uint32_t* __restrict__ live = nullptr,
+                                               uint32_t tag = 0) {
   const int lane = threadIdx.x & 31;
   const int gl = lane & (G - 1);
   const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
@@ -995,7 +1072,11 @@ __device__ __forceinline__ void point_bin_body(ulonglong2* __restrict__ list, in
     const ulonglong2 e = list[i];
     int64_t s, en;
     row_range(e, offs, vbase, &s, &en);
-    const uint64_t b = group_max_key(scan_row_available<G, U>(adj, bits, s, en, gl, gmask), gmask);
+    uint64_t b;
+    if (PRUNE && en - s <= (int64_t)G * U)
+      b = prune_row<G, U>(adj, bits, s, en, gl, gmask, live, tag, (int64_t)(uint32_t)e.x - vbase);
+    else
+      b = group_max_key(scan_row_available<G, U>(adj, bits, s, en, gl, gmask), gmask);
     if (gl == 0) {
       const uint32_t u = (uint32_t)e.x;
       best[u - vbase] = b;
@@ -1003,14 +1084,15 @@ __device__ __forceinline__ void point_bin_body(ulonglong2* __restrict__ list, in
     }
   }
 }
-template <int G, int U>
+template <int G, int U, bool PRUNE = false>
 __global__ void k_point_bin(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
                             const int64_t* __restrict__ offs, const AdjView adj,
                             const uint32_t* __restrict__ bits, uint64_t* __restrict__ best,
-                            int64_t vbase) {
-  point_bin_body<G, U>(list, (int64_t)*cnt_ptr, offs, adj, bits, best, vbase,
-                       (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
-                       (int64_t)gridDim.x * blockDim.x);
+                            int64_t vbase, uint32_t* __restrict__ live = nullptr,
+                            const RoundState* st = nullptr) {
+  point_bin_body<G, U, PRUNE>(list, (int64_t)*cnt_ptr, offs, adj, bits, best, vbase,
+                              (int64_t)blockIdx.x * blockDim.x + threadIdx.x,
+                              (int64_t)gridDim.x * blockDim.x, live, PRUNE ? round_tag(st) : 0u);
 }
 
 // Software-pipelined variant for the big host-driven rounds (grid = one resident wave, so every
@@ -1365,6 +1447,8 @@ struct CompactIO {
   const unsigned long long* cin;  // counters of the input set (cnt_S .. cnt_F(.,3) contiguous)
   unsigned long long* cout;       // counters of the output set
   unsigned long long* swept;
+  const uint32_t* live;           // A7: live counts (nullptr = pruning off)
+  const RoundState* st;
 };
 __host__ __device__ inline CompactIO compact_io(const RoundArgs& a, int cur) {
   CompactIO io;
@@ -1375,6 +1459,8 @@ __host__ __device__ inline CompactIO compact_io(const RoundArgs& a, int cur) {
   io.cin = a.cnt + cnt_S(cur);
   io.cout = a.cnt + cnt_S(cur ^ 1);
   io.swept = a.cnt + kCntSwept;
+  io.live = a.live;
+  io.st = a.st;
   return io;
 }
 
@@ -1404,6 +1490,8 @@ __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
   const int64_t cnt = p3 + (ALL ? 0 : (int64_t)cntFin[3]);
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const unsigned lt = lanemask_lt();
+  const uint32_t* __restrict__ lcnt = io.live;
+  const uint32_t tag = lcnt ? round_tag(io.st) : 0u;
   constexpr int64_t BLK = (int64_t)NW * 32 * K;
   unsigned long long degsum = 0;
   for (int64_t cb = bid * BLK; cb < cnt; cb += nblk * BLK) {
@@ -1449,6 +1537,10 @@ __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
       const bool fr = live && tgt;
       os[k] = fr ? offs[u - vbase] : 0;
       oe[k] = fr ? offs[u - vbase + 1] : -1;
+      if (lcnt && fr) {  // A7: a row pruned earlier in this run is scanned over its live prefix
+        const uint32_t x = lcnt[u - vbase];
+        if ((x >> 16) == tag) oe[k] = os[k] + (int64_t)(x & 0xffffu);
+      }
     }
 #pragma unroll
     for (int k = 0; k < K; ++k) {
@@ -1534,6 +1626,7 @@ __global__ void k_round_init(RoundState* st, long long max_rounds, long long log
   st->log_len = 0;
   st->log_cap = log_cap;
   st->swept_prev = 0;
+  st->tag = st->tag >= 0xffffu ? 1u : st->tag + 1u;
 }
 // After a compaction: the output set becomes current; decide whether another round runs.
 // `graph_handle` != 0: running inside a CUDA graph -> set the WHILE node's condition.
@@ -1576,7 +1669,7 @@ __global__ void k_end_round(const RoundArgs* __restrict__ ra, cudaGraphCondition
 // degree bin) | grid barrier | match | barrier | compaction | barrier | end of round | barrier.
 // No per-round launches or host decisions; the grid barrier's fence also invalidates L1, so
 // every phase reads the others' writes.
-template <int B0G, int B0U, int B1G, int B1U, int B2G, int B2U, int K>
+template <int B0G, int B0U, int B1G, int B1U, int B2G, int B2U, int K, bool PRUNE = false>
 __global__ void __launch_bounds__(256)
     k_rounds_persistent(const RoundArgs* __restrict__ ra, const int64_t* __restrict__ offs, const AdjView adj,
                         uint32_t* bits, uint64_t* best, int64_t n, int64_t vbase) {
@@ -1589,9 +1682,13 @@ __global__ void __launch_bounds__(256)
     {
       const Bins F = ra->F[cur];
       const unsigned long long* c = ra->cnt + cnt_F(cur, 0);
-      point_bin_body<B0G, B0U>(F.list[0], (int64_t)c[0], offs, adj, bits, best, vbase, gtid, gthreads);
-      point_bin_body<B1G, B1U>(F.list[1], (int64_t)c[1], offs, adj, bits, best, vbase, gtid, gthreads);
-      point_bin_body<B2G, B2U>(F.list[2], (int64_t)c[2], offs, adj, bits, best, vbase, gtid, gthreads);
+      const uint32_t tag = PRUNE ? round_tag(ra->st) : 0u;
+      point_bin_body<B0G, B0U, PRUNE>(F.list[0], (int64_t)c[0], offs, adj, bits, best, vbase, gtid,
+                                      gthreads, ra->live, tag);
+      point_bin_body<B1G, B1U, PRUNE>(F.list[1], (int64_t)c[1], offs, adj, bits, best, vbase, gtid,
+                                      gthreads, ra->live, tag);
+      point_bin_body<B2G, B2U, PRUNE>(F.list[2], (int64_t)c[2], offs, adj, bits, best, vbase, gtid,
+                                      gthreads, ra->live, tag);
       point_bin_cta_body<256, 4>(F.list[3], (int64_t)c[3], offs, adj, bits, best, vbase, blockIdx.x,
                                  gridDim.x);
     }

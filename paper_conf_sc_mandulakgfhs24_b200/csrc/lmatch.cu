@@ -220,6 +220,8 @@ struct lmatch_graph {
   lm::RoundState* h_rstate = nullptr;  // pinned
   long long* rlog = nullptr;           // device [kLogCap][3]
   int round_loop = 0;                  // 0 = CUDA graph, 1 = host-driven
+  int prune = 0;                       // A7 in-place pruning (resident, single-graph handles)
+  uint32_t* live = nullptr;            // A7 live counts: tag << 16 | count
   cudaGraphExec_t gexec = nullptr;
   cudaGraph_t graph = nullptr;
   cudaStream_t gstream = nullptr;      // stream the graph was captured on (capture needs its own)
@@ -235,6 +237,7 @@ struct lmatch_graph {
     a.cnt = counters;
     a.st = rstate;
     a.log = rlog;
+    a.live = prune ? live : nullptr;
     return a;
   }
 };
@@ -331,6 +334,7 @@ int alloc_all(lmatch_graph* g) {
   TRY(dmalloc(g, &g->bits, (size_t)((g->n_global + 31) / 32) + 1));
   TRY(dmalloc(g, &g->counters, lm::kNumCounters));
   TRY(dmalloc(g, &g->rstate, 1));
+  CK(cudaMemsetAsync(g->rstate, 0, sizeof(lm::RoundState), g->stream));
   TRY(dmalloc(g, &g->d_rargs, 1));
   TRY(dmalloc(g, &g->rlog, 3 * (size_t)kLogCap + 3));
   CK(cudaHostAlloc(reinterpret_cast<void**>(&g->h_rstate), sizeof(lm::RoundState), cudaHostAllocDefault));
@@ -563,6 +567,10 @@ int alloc_bins(lmatch_graph* g, cudaStream_t st) {
   CK(cudaStreamSynchronize(st));
   cudaFree(cnt);
   g->device_bytes -= 16;
+  // A7 pruning moves rows to LOWER bins (live degrees only shrink): bin b must then hold every
+  // row whose full degree is in bin b or above
+  if (g->prune)
+    for (int b = lm::kBins - 2; b >= 0; --b) h[b] += h[b + 1];
   for (int i = 0; i < 2; ++i)
     for (int b = 0; b < lm::kBins; ++b)
       TRY(ensure(g, &g->F[i].list[b], &g->cap_bin[i][b], (int64_t)h[b] + 1));
@@ -572,6 +580,11 @@ int alloc_bins(lmatch_graph* g, cudaStream_t st) {
 }
 
 int finish_create(lmatch_graph* g, cudaStream_t st) {
+  if (g->prune && (g->streaming || g->ghost)) g->prune = 0;  // resident single-graph only
+  if (g->prune && !g->live) {
+    TRY(dmalloc(g, &g->live, (size_t)g->n + 1));
+    CK(cudaMemsetAsync(g->live, 0, ((size_t)g->n + 1) * 4, st));
+  }
   TRY(build_index(g, st));
   TRY(alloc_bins(g, st));
   if (g->m > 0) {
@@ -642,6 +655,7 @@ int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** 
     g->hbm_budget = opts->hbm_budget_bytes;
     if (opts->stream_chunk > 0) g->stream_chunk = opts->stream_chunk;
     g->round_loop = opts->round_loop;
+    g->prune = opts->prune != 0;
   }
   CK(cudaGetDevice(&g->device));
   CK(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, g->device));
@@ -850,7 +864,8 @@ static int seq_prefix(lmatch_graph* g, cudaStream_t st, cudaGraphConditionalHand
   const int64_t nwords = (g->n_global + 31) / 32;
   const bool work = g->ntiles > 0 && n > 0;
   lm::k_reset<<<grid_for(std::max(nwords, g->n_atomic), 256, 4096), 256, 0, st>>>(
-      g->bits, nwords, g->best, g->atomic_rows, g->n_atomic, g->counters, lm::kNumCounters);
+      g->bits, nwords, g->best, g->atomic_rows, g->n_atomic, g->counters, lm::kNumCounters,
+      g->prune ? g->live : nullptr, g->n, g->rstate);
   CKL();
   lm::k_round_init<<<1, 1, 0, st>>>(g->rstate, g->max_rounds, kLogCap, work ? 1 : 0);
   CKL();
@@ -904,7 +919,10 @@ static int seq_body(lmatch_graph* g, cudaStream_t st, int cur, const int64_t* nF
   for (int b = 0; b < lm::kBins; ++b) nF += nFb[b];
 #define PIPE_OR_BIN(b, PG, PU, BG, BU, AG, AU)                                                      \
   if (nFb[b]) {                                                                                   \
-    if ((LM_ASYNC & (1 << b)) && !g->streaming) {                                                 \
+    if (g->prune) {                                                                               \
+      lm::k_point_bin<BG, BU, true><<<grid_for(nFb[b] * BG, 256, 65536), 256, 0, st>>>(           \
+          Fb.list[b], cF + b, g->offs, av, g->bits, g->best, g->v0, g->live, g->rstate);          \
+    } else if ((LM_ASYNC & (1 << b)) && !g->streaming) {                                          \
       constexpr size_t smem = (size_t)LM_ASYNC_S * AU * 256 * 8;                                  \
       static int occ = 0;                                                                         \
       if (!occ) {                                                                                 \
@@ -948,14 +966,16 @@ static int seq_body(lmatch_graph* g, cudaStream_t st, int cur, const int64_t* nF
   return LMATCH_OK;
 }
 
-#define PERSISTENT_KERNEL \
-  lm::k_rounds_persistent<LM_B0_G, LM_B0_U, LM_B1_G, LM_B1_U, LM_B2_G, LM_B2_U, kCompactK>
+#define PERSISTENT_KERNEL(PR) \
+  lm::k_rounds_persistent<LM_B0_G, LM_B0_U, LM_B1_G, LM_B1_U, LM_B2_G, LM_B2_U, kCompactK, PR>
 
 // rounds >= 2 in one cooperative launch (grid = co-resident blocks)
-static int launch_persistent(lmatch_graph* g, cudaStream_t st, int64_t* launches) {
+extern "C++" {
+template <bool PRUNE>
+int launch_persistent_t(lmatch_graph* g, cudaStream_t st, int64_t* launches) {
   static int occ = 0;
   if (!occ) {
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, PERSISTENT_KERNEL, 256, 0));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, PERSISTENT_KERNEL(PRUNE), 256, 0));
     if (occ < 1) occ = 1;
   }
   const lm::RoundArgs* ra = g->ra();
@@ -969,10 +989,15 @@ static int launch_persistent(lmatch_graph* g, cudaStream_t st, int64_t* launches
   attr[0].val.cooperative = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  CK(cudaLaunchKernelEx(&cfg, PERSISTENT_KERNEL, ra, (const int64_t*)g->offs, av, g->bits, g->best,
-                        g->n, g->v0));
+  CK(cudaLaunchKernelEx(&cfg, PERSISTENT_KERNEL(PRUNE), ra, (const int64_t*)g->offs, av, g->bits,
+                        g->best, g->n, g->v0));
   ++*launches;
   return LMATCH_OK;
+}
+}  // extern "C++"
+static int launch_persistent(lmatch_graph* g, cudaStream_t st, int64_t* launches) {
+  return g->prune ? launch_persistent_t<true>(g, st, launches)
+                  : launch_persistent_t<false>(g, st, launches);
 }
 
 // Capture reset .. round 1 + the persistent round kernel into one CUDA graph (built once).
@@ -1231,7 +1256,8 @@ int lmatch_part_begin(lmatch_graph* g, void* stream, int64_t* claim_counts) {
   cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
   const int64_t nwords = (g->n_global + 31) / 32;
   lm::k_reset<<<grid_for(std::max(nwords, g->n_atomic), 256, 4096), 256, 0, st>>>(
-      g->bits, nwords, g->best, g->atomic_rows, g->n_atomic, g->counters, lm::kNumCounters);
+      g->bits, nwords, g->best, g->atomic_rows, g->n_atomic, g->counters, lm::kNumCounters,
+      g->prune ? g->live : nullptr, g->n, g->rstate);
   CKL();
   lm::k_round_init<<<1, 1, 0, st>>>(g->rstate, g->max_rounds, kLogCap, 1);
   CKL();

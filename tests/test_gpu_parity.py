@@ -379,3 +379,56 @@ def test_self_loops_ignored(lm, mode):
         for P in (2, 3):
             mate, res = D.match_partitioned_local(g.offsets, g.col, g.w, P)
             np.testing.assert_array_equal(mate, ref.mate)
+
+
+# ------------------------------------------------- A7 in-place pruning (opt-in)
+@pytest.mark.parametrize("maker", [
+    lambda: graphgen.rmat(14, 16, seed=31),
+    lambda: graphgen.rmat(16, 16, seed=32, weights="paper"),    # 3-decimal ties
+    lambda: graphgen.er(1 << 14, 16.0, seed=33),
+    lambda: graphgen.er(3000, 40.0, seed=34, weights="ones"),   # ties only; 32-lane rows
+    lambda: graphgen.mesh(128, seed=35),
+    lambda: graphgen.mesh(200, keep=0.6, seed=36),
+    lambda: graphgen.mesh(48, seed=37, weights="gradient"),     # ~100 rounds, persistent kernel
+    lambda: _loopy_graph(38),                                   # zeroed self-loop keys are pruned
+])
+@pytest.mark.parametrize("round_loop", [0, 1, 2, 3])
+def test_pruning_parity_and_reentrant(lm, maker, round_loop):
+    """Pruning removes only entries whose neighbour is matched (never available again, R3), so
+    mate[], the rounds and w(M) equal the oracle's.  The rows stay permutations of themselves,
+    so repeated runs on the same handle (whose round-1 sweep reads whole rows again) stay exact,
+    and the later rounds scan no more entries than without pruning."""
+    g = maker()
+    ref = oracle.greedy(g)
+    ph = oracle.ld_frontier(g)[1]
+    _, base = run_gpu(lm, g, round_loop=round_loop)
+    with lm.Matcher(g, prune=True, round_loop=round_loop) as M:
+        for _ in range(3):
+            mate, st = M.run()
+            np.testing.assert_array_equal(mate, ref.mate)
+            assert st["rounds"] == ph
+            assert math.isclose(st["weight"], ref.weight, rel_tol=WTOL)
+            assert st["entries_swept"] <= base["entries_swept"]
+            assert st["frontier_total"] == base["frontier_total"]
+
+
+def test_pruning_keeps_rows_permutations(lm):
+    """After pruned runs, a fresh non-pruning run on the SAME handle's adjacency -- reached by
+    reading back w(M) of arbitrary mates through lmatch_weight, which looks edges up in the
+    handle's rows -- still finds every edge: the multiset of each row is unchanged."""
+    g = graphgen.rmat(13, 16, seed=39)
+    ref = oracle.greedy(g)
+    rng = np.random.default_rng(4)
+    with lm.Matcher(g, prune=True) as M:
+        for _ in range(2):
+            mate, _ = M.run()
+            np.testing.assert_array_equal(mate, ref.mate)
+        # a different valid matching: every edge lookup must still succeed in the permuted rows
+        E = [(u, int(g.col[j])) for u in range(g.n) for j in range(g.offsets[u], g.offsets[u + 1])
+             if u < g.col[j]]
+        rng.shuffle(E)
+        other = np.full(g.n, -1, np.int32)
+        for u, v in E[:3000]:
+            if other[u] < 0 and other[v] < 0:
+                other[u], other[v] = v, u
+        assert math.isclose(M.weight(other), oracle.weight(g, other), rel_tol=WTOL)
