@@ -1382,23 +1382,30 @@ __global__ void __launch_bounds__(THREADS)
 // A4 match (SETMATES, Alg. 3 L10-13 P:152-155): mutual pointers are locally dominant edges.
 // =============================================================================================
 // Round 1: every vertex; the warp owning 32 consecutive vertices writes their bitmap word.
+// Each warp owns 4 bitmap words per step and issues the 4 random best[ptr u] reads together.
 __global__ void k_match_all(const uint64_t* __restrict__ best, int64_t n, uint32_t* bits) {
+  constexpr int V = 4;
   const int64_t nwords = (n + 31) >> 5;
   const int lane = threadIdx.x & 31;
   const int64_t w0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t ws = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  for (int64_t wi = w0; wi < nwords; wi += ws) {
-    const int64_t u = (wi << 5) + lane;
-    bool mutual = false;
-    if (u < n) {
-      const uint64_t b = best[u];
-      if (b) {
-        const uint64_t bv = best[(uint32_t)b];
-        mutual = bv != 0 && (uint32_t)bv == (uint32_t)u;
-      }
+  for (int64_t wb = w0; wb < nwords; wb += V * ws) {
+    uint64_t b[V], bv[V];
+#pragma unroll
+    for (int q = 0; q < V; ++q) {
+      const int64_t u = ((wb + q * ws) << 5) + lane;
+      b[q] = (wb + q * ws < nwords && u < n) ? best[u] : 0ull;
     }
-    const unsigned word = __ballot_sync(0xffffffffu, mutual);
-    if (lane == 0) bits[wi] = word;
+#pragma unroll
+    for (int q = 0; q < V; ++q) bv[q] = b[q] ? best[(uint32_t)b[q]] : 0ull;
+#pragma unroll
+    for (int q = 0; q < V; ++q) {
+      const int64_t wi = wb + q * ws;
+      const int64_t u = (wi << 5) + lane;
+      const bool mutual = bv[q] != 0 && (uint32_t)bv[q] == (uint32_t)u;
+      const unsigned word = __ballot_sync(0xffffffffu, mutual);
+      if (lane == 0 && wi < nwords) bits[wi] = word;
+    }
   }
 }
 
@@ -1860,19 +1867,38 @@ template <int THREADS>
 __global__ void __launch_bounds__(THREADS)
     k_materialize(const uint64_t* __restrict__ best, const uint32_t* __restrict__ bits, int64_t n,
                   int64_t vbase, int32_t* __restrict__ mate, double* pw, long long* pc) {
+  // 4 vertices per thread per step with their loads issued together (the per-vertex chain
+  // bitmap word -> best[] is latency-bound otherwise); fixed assignment => fixed fp64 order
+  constexpr int V = 4;
   double w = 0.0;
   long long c = 0;
   const int64_t stride = (int64_t)gridDim.x * THREADS;
-  for (int64_t i = (int64_t)blockIdx.x * THREADS + threadIdx.x; i < n; i += stride) {
-    const int64_t u = i + vbase;
-    int32_t v = -1;
-    if (bit_test(bits, (uint32_t)u)) {
-      const uint64_t k = best[i];
-      v = (int32_t)(uint32_t)k;
-      ++c;
-      if ((int64_t)v > u) w += (double)__uint_as_float((uint32_t)(k >> 32));
+  for (int64_t i0 = (int64_t)blockIdx.x * THREADS + threadIdx.x; i0 < n; i0 += V * stride) {
+    uint32_t wd[V];
+#pragma unroll
+    for (int q = 0; q < V; ++q) {
+      const int64_t i = i0 + q * stride;
+      wd[q] = i < n ? bits[(uint32_t)(i + vbase) >> 5] : 0u;
     }
-    mate[i] = v;
+    uint64_t k[V];
+#pragma unroll
+    for (int q = 0; q < V; ++q) {
+      const int64_t i = i0 + q * stride;
+      const bool mt = i < n && ((wd[q] >> ((uint32_t)(i + vbase) & 31)) & 1u);
+      k[q] = mt ? best[i] : ~0ull;
+    }
+#pragma unroll
+    for (int q = 0; q < V; ++q) {
+      const int64_t i = i0 + q * stride;
+      if (i >= n) break;
+      int32_t v = -1;
+      if (k[q] != ~0ull) {
+        v = (int32_t)(uint32_t)k[q];
+        ++c;
+        if ((int64_t)v > i + vbase) w += (double)__uint_as_float((uint32_t)(k[q] >> 32));
+      }
+      mate[i] = v;
+    }
   }
   block_sum2<THREADS>(w, c, &pw[blockIdx.x], &pc[blockIdx.x]);
 }
@@ -1914,12 +1940,20 @@ __global__ void __launch_bounds__(THREADS)
   block_sum2<THREADS>(w, c, &pw[blockIdx.x], &pc[blockIdx.x]);
 }
 
+// Fixed-order (deterministic) sum of the per-block partials: lane l adds partials l, l+32, ...
+// in index order, then a fixed butterfly.  Launch <<<1, 32>>>.
 __global__ void k_final_sum(const double* pw, const long long* pc, int nb, double* out_w,
                             long long* out_c) {
-  if (blockIdx.x == 0 && threadIdx.x == 0) {
-    double w = 0; long long c = 0;
-    for (int i = 0; i < nb; ++i) { w += pw[i]; c += pc[i]; }
-    *out_w = w; *out_c = c;
+  const int lane = threadIdx.x & 31;
+  double w = 0;
+  long long c = 0;
+  if (threadIdx.x < 32) {
+    for (int i = lane; i < nb; i += 32) { w += pw[i]; c += pc[i]; }
+    for (int o = 16; o; o >>= 1) {
+      w += __shfl_xor_sync(0xffffffffu, w, o);
+      c += __shfl_xor_sync(0xffffffffu, c, o);
+    }
+    if (lane == 0) { *out_w = w; *out_c = c; }
   }
 }
 
