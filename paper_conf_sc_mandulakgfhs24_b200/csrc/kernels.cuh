@@ -1456,6 +1456,7 @@ struct CompactIO {
   unsigned long long* swept;
   const uint32_t* live;           // A7: live counts (nullptr = pruning off)
   const RoundState* st;
+  const int32_t* nzr;             // ALL mode: iterate the non-empty rows only (nullptr = all n)
 };
 __host__ __device__ inline CompactIO compact_io(const RoundArgs& a, int cur) {
   CompactIO io;
@@ -1468,6 +1469,7 @@ __host__ __device__ inline CompactIO compact_io(const RoundArgs& a, int cur) {
   io.swept = a.cnt + kCntSwept;
   io.live = a.live;
   io.st = a.st;
+  io.nzr = nullptr;
   return io;
 }
 
@@ -1512,8 +1514,10 @@ __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
       uint64_t p = (uint64_t)kNoPtr << 32;
       if (i < cnt) {
         if (ALL) {
-          const uint64_t bb = best[i];
-          p = make_pair((uint32_t)(i + vbase), bb ? (uint32_t)bb : kNoPtr);
+          // an empty row never holds a pointer: with the non-empty row list only those are read
+          const int64_t r = io.nzr ? (int64_t)io.nzr[i] : i;
+          const uint64_t bb = best[r];
+          p = make_pair((uint32_t)(r + vbase), bb ? (uint32_t)bb : kNoPtr);
         } else {
           p = i < p0 ? S[i]
               : i < p1 ? Fin.list[0][i - p0].x
@@ -1614,7 +1618,10 @@ __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
   if (lane == 0 && degsum) atomicAdd(swept, degsum);
 }
 template <bool ALL, int K>
-__global__ void __launch_bounds__(256)
+#ifndef LM_COMPACT_MINB
+#define LM_COMPACT_MINB 3  // 85-register cap: 36% -> ~50% occupancy, no spills (round-1 compaction -30%)
+#endif
+__global__ void __launch_bounds__(256, LM_COMPACT_MINB)
     k_compact(CompactIO io, int64_t n, const uint64_t* __restrict__ best,
               const uint32_t* __restrict__ bits, const int64_t* __restrict__ offs, int64_t vbase) {
   compact_body<ALL, K>(io, n, best, bits, offs, vbase, blockIdx.x, gridDim.x);

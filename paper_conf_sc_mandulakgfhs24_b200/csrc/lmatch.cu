@@ -897,9 +897,14 @@ static int seq_prefix(lmatch_graph* g, cudaStream_t st, cudaGraphConditionalHand
   TRY(mark(2));
   lm::k_match_all<<<grid_for(nwords * 32, 256, 65536), 256, 0, st>>>(g->best, n, g->bits);
   CKL();
-  // round-1 compaction: input set 1 (unused), output set 0; k_end_round makes set 0 current
-  lm::k_compact<true, kCompactK><<<grid_for((n + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
-      lm::compact_io(g->rargs(), 1), n, g->best, g->bits, g->offs, g->v0);
+  // round-1 compaction: input set 1 (unused), output set 0; k_end_round makes set 0 current.
+  // Items are the non-empty rows (nzr): empty rows never hold a pointer.
+  {
+    lm::CompactIO io = lm::compact_io(g->rargs(), 1);
+    io.nzr = g->nzr;
+    lm::k_compact<true, kCompactK><<<grid_for((g->n_nz + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
+        io, g->n_nz, g->best, g->bits, g->offs, g->v0);
+  }
   CKL();
   lm::k_end_round<<<1, 32, 0, st>>>(g->ra(), h, in_graph, 0);
   CKL();
