@@ -1084,8 +1084,11 @@ __device__ __forceinline__ void point_bin_body(ulonglong2* __restrict__ list, in
     }
   }
 }
+#ifndef LM_BIN_MINB
+#define LM_BIN_MINB 6  // 40-register cap: more resident groups (32-lane bin -12%)
+#endif
 template <int G, int U, bool PRUNE = false>
-__global__ void k_point_bin(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
+__global__ void __launch_bounds__(256, LM_BIN_MINB) k_point_bin(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
                             const int64_t* __restrict__ offs, const AdjView adj,
                             const uint32_t* __restrict__ bits, uint64_t* __restrict__ best,
                             int64_t vbase, uint32_t* __restrict__ live = nullptr,
@@ -1229,8 +1232,11 @@ __device__ __forceinline__ void point_pipe_body(ulonglong2* __restrict__ list, i
     clast = nlast;
   }
 }
+#ifndef LM_PIPE_MINB
+#define LM_PIPE_MINB 1
+#endif
 template <int G, int U>
-__global__ void __launch_bounds__(256)
+__global__ void __launch_bounds__(256, LM_PIPE_MINB)
     k_point_pipe(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
                  const int64_t* __restrict__ offs, const AdjView adj,
                  const uint32_t* __restrict__ bits, uint64_t* __restrict__ best, int64_t vbase) {
