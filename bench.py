@@ -56,6 +56,8 @@ def parse():
                         "from pinned host memory in round 1 and read zero-copy afterwards")
     p.add_argument("--stream-chunk", type=int, default=0, help="entries per streamed chunk (0 = default)")
     p.add_argument("--prune", action="store_true", help="A7 in-place pruning (lmatch_opts.prune)")
+    p.add_argument("--no-host-cache", action="store_true",
+                   help="out-of-core: disable the top-8 host-row key cache (lmatch_opts.host_cache = -1)")
     p.add_argument("--partitioned", action="store_true",
                    help="use the 1-D partitioned path even at N=1 (it is always used for N>1)")
     return p.parse_args()
@@ -419,7 +421,7 @@ def main():
     # CSR); create is untimed: P:179 excludes I/O, allocation, CSR construction and the transfer
     opts = lm.make_opts(validate_level=1, timing=1,
                         hbm_budget_bytes=int(a.hbm_budget_gb * 1e9), stream_chunk=a.stream_chunk,
-                        prune=a.prune)
+                        prune=a.prune, host_cache=not a.no_host_cache)
     pinned_host = d_off is None
     if pinned_host:
         h = lm.lmatch_create_ex(g.offsets, g.col, g.w, n, m, opts)
@@ -521,8 +523,13 @@ def main():
                "resident_frac": last["resident_entries"] / max(m, 1),
                "bytes_streamed_per_step": int(last["bytes_streamed"]),
                "stream_gbs_in_sweep": last["bytes_streamed"] / max(sweep_avg_ms, 1e-9) / 1e6,
+               "host_cache": not a.no_host_cache,
+               "cache_bytes": int(last["cache_bytes"]),
+               "cache_rows_per_step": int(last["cache_rows"]),
+               "host_entries_read_per_step": int(last["host_entries_read"]),
                "note": "sweep = resident HBM tiles + host chunks over PCIe (2-slot ring); later "
-                       "rounds read host rows zero-copy"}
+                       "rounds read host rows zero-copy, except rows whose pointer the top-8 "
+                       "host-row key cache decides (filled in round 1; NEXT-1)"}
     round_log = lm.lmatch_round_log(h)
     lm.lmatch_destroy(h)
     del d_mate

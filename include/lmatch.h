@@ -98,7 +98,17 @@ typedef struct lmatch_opts {
                                  per-row permutation of the input, so the result and later runs
                                  are unchanged.  Ignored for out-of-core and partition handles.
                                  0 = default (off: measured slower on R-MAT) */
-  int32_t reserved[10];
+  int32_t host_cache;         /* out-of-core only: 0 = default (on), -1 = off.
+                                 Every row with entries beyond the resident prefix keeps its 8
+                                 largest keys in HBM (64 bytes per such row, allocated on top of
+                                 hbm_budget_bytes and reported in lmatch_stats.cache_bytes),
+                                 filled in round 1 from the streamed chunks.  Later rounds take
+                                 the pointer from the cache when one of the cached neighbours is
+                                 unmatched (the first such key is the row maximum over available
+                                 neighbours), so only rows whose 8 heaviest neighbours are all
+                                 matched are read from host memory.  Same result.  Rounds >= 2
+                                 of an out-of-core run with the cache are host-driven launches */
+  int32_t reserved[9];
 } lmatch_opts;
 
 /* Filled by lmatch_run / lmatch_run_device when non-NULL. */
@@ -118,7 +128,11 @@ typedef struct lmatch_stats {
   int64_t kernel_launches;   /* all kernel launches issued by this run */
   int64_t bytes_streamed;    /* host->device adjacency bytes copied by this run (out-of-core) */
   int64_t resident_entries;  /* adjacency entries resident in HBM (= m unless out-of-core) */
-  int64_t reserved[6];
+  int64_t cache_rows;        /* out-of-core host-row cache: frontier rows whose pointer the
+                                cache decided in rounds >= 2 (no host read) */
+  int64_t host_entries_read; /* out-of-core: host-resident entries read zero-copy in rounds >= 2 */
+  int64_t cache_bytes;       /* out-of-core: device bytes of the host-row cache (0 = none) */
+  int64_t reserved[3];
 } lmatch_stats;
 
 /* Library / ABI identification.  Returns LMATCH_ABI_VERSION. */

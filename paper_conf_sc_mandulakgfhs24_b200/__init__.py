@@ -44,7 +44,7 @@ class Opts(ctypes.Structure):
         ("max_rounds", ctypes.c_int64), ("upload_chunk", ctypes.c_int64),
         ("hbm_budget_bytes", ctypes.c_int64), ("stream_chunk", ctypes.c_int64),
         ("round_loop", ctypes.c_int32), ("prune", ctypes.c_int32),
-        ("reserved", ctypes.c_int32 * 10),
+        ("host_cache", ctypes.c_int32), ("reserved", ctypes.c_int32 * 9),
     ]
 
 
@@ -58,7 +58,9 @@ class Stats(ctypes.Structure):
         ("ms_rounds", ctypes.c_double), ("ms_round1_rest", ctypes.c_double),
         ("ms_finish", ctypes.c_double), ("sweep_launches", ctypes.c_int64),
         ("kernel_launches", ctypes.c_int64), ("bytes_streamed", ctypes.c_int64),
-        ("resident_entries", ctypes.c_int64), ("reserved", ctypes.c_int64 * 6),
+        ("resident_entries", ctypes.c_int64), ("cache_rows", ctypes.c_int64),
+        ("host_entries_read", ctypes.c_int64), ("cache_bytes", ctypes.c_int64),
+        ("reserved", ctypes.c_int64 * 3),
     ]
 
     def as_dict(self) -> dict:
@@ -240,7 +242,7 @@ class Matcher:
     def __init__(self, offsets=None, col=None, w=None, *, handle: int | None = None,
                  validate_level: int = 1, timing: bool = False, upload_chunk: int = 0,
                  max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
-                 round_loop: int = 0, prune: bool = False):
+                 round_loop: int = 0, prune: bool = False, host_cache: bool = True):
         self.h = None
         if handle is not None:
             self.h = handle
@@ -250,7 +252,7 @@ class Matcher:
             self.h = lmatch_create_ex(offsets, col, w,
                                       opts=make_opts(validate_level, timing, upload_chunk,
                                                      max_rounds, hbm_budget_bytes, stream_chunk,
-                                                     round_loop, prune))
+                                                     round_loop, prune, host_cache))
         self.info = lmatch_info(self.h)
 
     @classmethod
@@ -293,13 +295,14 @@ class Matcher:
 
 def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int = 0,
               max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
-              round_loop: int = 0, prune: bool = False) -> Opts:
+              round_loop: int = 0, prune: bool = False, host_cache: bool = True) -> Opts:
     """round_loop (include/lmatch.h): 0 = hybrid (work-sized launches, then one persistent kernel
     for the tail; default), 1 = host-driven launches only, 2 = persistent kernel after round 1,
     3 = CUDA graph {round 1, persistent kernel}."""
     o = Opts()
     o.round_loop = int(round_loop)
     o.prune = int(bool(prune))
+    o.host_cache = 0 if host_cache else -1
     o.hbm_budget_bytes = int(hbm_budget_bytes)
     o.stream_chunk = int(stream_chunk)
     o.validate_level = int(validate_level)

@@ -31,12 +31,16 @@ constexpr int kBinDeg0 = 8, kBinDeg1 = 64, kBinDeg2 = 2048;  // bins: G = 1, 8, 
 
 // Adjacency view: entries [0, R) in HBM, [R, m) in pinned host memory mapped into the device
 // address space (out-of-core mode; R = m otherwise).  host_off is pre-offset by -R.
+// Out-of-core with the host-row key cache (NEXT-1): indices >= M0 address the cache (HBM),
+// cache_off pre-offset by -M0, so a frontier entry can be redirected to cached keys.
 struct AdjView {
   const uint64_t* dev;
   const uint64_t* host_off;
   int64_t R;
+  const uint64_t* cache_off = nullptr;
+  int64_t M0 = INT64_MAX;
   __device__ __forceinline__ uint64_t at(int64_t j) const {
-    return j < R ? __ldg(dev + j) : host_off[j];
+    return j < R ? __ldg(dev + j) : (j < M0 ? host_off[j] : __ldg(cache_off + j));
   }
   __device__ __forceinline__ uint64_t* ptr(int64_t j) const {
     return const_cast<uint64_t*>(j < R ? dev + j : host_off + j);
@@ -832,6 +836,7 @@ __global__ void k_low32(const int64_t* __restrict__ noffs, int64_t cnt, uint32_t
 // =============================================================================================
 constexpr int kNumCounters = 24;
 constexpr int kCntSwept = 16;
+constexpr int kCntCache = 17;  // [17] rows served by the out-of-core cache, [18] host entries read
 __host__ __device__ constexpr int cnt_S(int set) { return 8 * set; }
 __host__ __device__ constexpr int cnt_F(int set, int b) { return 8 * set + 1 + b; }
 constexpr uint32_t kNoPtr = 0xffffffffu;
@@ -1967,6 +1972,172 @@ __global__ void k_final_sum(const double* pw, const long long* pc, int nb, doubl
       c += __shfl_xor_sync(0xffffffffu, c, o);
     }
     if (lane == 0) { *out_w = w; *out_c = c; }
+  }
+}
+
+// =============================================================================================
+// NEXT-1: out-of-core host-row key cache.  Every row with entries beyond the
+// resident prefix ("host row", u >= u_first) keeps its K largest keys in HBM, descending,
+// zero-padded.  They are filled in round 1 from the streamed chunks (the round is PCIe-bound,
+// so the extra pass over the chunk already in the device ring is free) and used by later rounds:
+// if a cached key's neighbour is unmatched, the FIRST such key is the row's maximum available
+// key (every larger key of the row is cached and unavailable; available sets only shrink,
+// R3), so the frontier entry is redirected to that one cached slot and the host row is not read.
+// A row with degree <= K is cached whole, so "no cached key available" means no pointer.  Only
+// rows with degree > K whose K cached neighbours are all matched are read zero-copy.
+// =============================================================================================
+constexpr int kCacheK = 8;
+
+// last row u with offs[u] <= j (the row holding entry j, for 0 <= j < offs[n])
+__device__ __forceinline__ int64_t row_of_entry(const int64_t* __restrict__ offs, int64_t n, int64_t j) {
+  int64_t lo = 0, hi = n;  // offs[lo] <= j < offs[hi]
+  while (hi - lo > 1) {
+    const int64_t mid = lo + ((hi - lo) >> 1);
+    if (offs[mid] <= j) lo = mid; else hi = mid;
+  }
+  return lo;
+}
+// out[k] = row holding entry min(first + k * step, last) for k in [0, cnt)
+__global__ void k_rows_of_entries(const int64_t* __restrict__ offs, int64_t n, int64_t first,
+                                  int64_t step, int64_t last, int64_t cnt, int64_t* out) {
+  const int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (k < cnt) out[k] = row_of_entry(offs, n, min(first + k * step, last));
+}
+
+// insert x into a descending register list (keeps the K largest)
+template <int K>
+__device__ __forceinline__ void topk_insert(uint64_t (&t)[K], uint64_t x) {
+#pragma unroll
+  for (int i = 0; i < K; ++i) {
+    const uint64_t a = t[i];
+    const bool gt = x > a;
+    t[i] = gt ? x : a;
+    x = gt ? a : x;
+  }
+}
+
+// K warp-wide pops of the per-lane descending lists: lane r < K receives the r-th largest key
+// (u64 max; equal keys of a repeated edge are popped one at a time).
+template <int K>
+__device__ __forceinline__ uint64_t warp_topk_pop(uint64_t (&t)[K]) {
+  const int lane = threadIdx.x & 31;
+  uint64_t mine = 0ull;
+#pragma unroll
+  for (int r = 0; r < K; ++r) {
+    const uint64_t mx = group_max_key(t[0], 0xffffffffu);
+    if (lane == r) mine = mx;
+    const unsigned own = __ballot_sync(0xffffffffu, mx != 0ull && t[0] == mx);
+    if (own && lane == __ffs(own) - 1) {
+#pragma unroll
+      for (int i = 0; i < K - 1; ++i) t[i] = t[i + 1];
+      t[K - 1] = 0ull;
+    }
+  }
+  return mine;
+}
+
+// Fill / merge the cache of rows [*plo, *phi] from entries [w0, w1) held at base[j - ebase].
+// A row starting inside the window overwrites its slots; a row that started before it (spans a
+// chunk boundary or the resident/streamed split) merges with the slots written earlier on the
+// same stream.  BIG = false: one warp per row of <= kCacheBigRow in-window entries; BIG = true:
+// one CTA per longer row (per-warp top-K, then warp 0 merges the 8 warps' lists in smem).
+constexpr int64_t kCacheBigRow = 4096;
+template <int K, bool BIG>
+__global__ void __launch_bounds__(256) k_cache_fill(const uint64_t* __restrict__ base, int64_t ebase,
+                                                    int64_t w0, int64_t w1,
+                                                    const int64_t* __restrict__ offs,
+                                                    const int64_t* __restrict__ plo,
+                                                    const int64_t* __restrict__ phi, int64_t u_first,
+                                                    uint64_t* __restrict__ cache) {
+  __shared__ uint64_t cand[8][K];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t ulo = *plo, uhi = *phi;
+  const int64_t first = BIG ? (int64_t)blockIdx.x : ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t step = BIG ? (int64_t)gridDim.x : ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const int64_t lstride = BIG ? (int64_t)blockDim.x : 32;
+  const int64_t lid = BIG ? (int64_t)threadIdx.x : lane;
+  for (int64_t u = ulo + first; u <= uhi; u += step) {
+    const int64_t s = offs[u], en = offs[u + 1];
+    const int64_t a = max(s, w0), b = min(en, w1);
+    if (a >= b || ((b - a > kCacheBigRow) != BIG)) continue;
+    uint64_t t[K];
+#pragma unroll
+    for (int i = 0; i < K; ++i) t[i] = 0ull;
+    for (int64_t j = a + lid; j < b; j += lstride) topk_insert<K>(t, base[j - ebase]);
+    uint64_t* c = cache + (u - u_first) * K;
+    if (s < w0 && lid < K) topk_insert<K>(t, c[lid]);
+    uint64_t mine = warp_topk_pop<K>(t);
+    if (BIG) {
+      if (lane < K) cand[warp][lane] = mine;
+      __syncthreads();
+      if (warp == 0) {
+#pragma unroll
+        for (int i = 0; i < K; ++i) t[i] = 0ull;
+        for (int q = lane; q < 8 * K; q += 32) topk_insert<K>(t, cand[q / K][q % K]);
+        mine = warp_topk_pop<K>(t);
+      }
+      __syncthreads();
+    }
+    if ((!BIG || warp == 0) && lane < K) c[lane] = mine;
+  }
+}
+
+// Rounds >= 2 (out-of-core): redirect frontier entries of host rows to the cache where it
+// decides the pointer.  .y becomes (1 << 40 | M0 + slot) for the first available cached key, or
+// an empty range when the whole row is cached and none is available; otherwise the entry keeps
+// its host range (read zero-copy).  cnt[0] += rows served by the cache, cnt[1] += host entries
+// left to the zero-copy path.
+template <int K>
+__global__ void k_cache_redirect(Bins F, const unsigned long long* __restrict__ cntF,
+                                 const int64_t* __restrict__ offs, const uint64_t* __restrict__ cache,
+                                 const uint32_t* __restrict__ bits, int64_t u_first, int64_t M0,
+                                 int64_t vbase, unsigned long long* cnt) {
+  const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  unsigned long long served = 0, left = 0;
+  for (int bb = 0; bb < kBins; ++bb) {
+    const int64_t c = (int64_t)cntF[bb];
+    for (int64_t i = tid; i < c; i += stride) {
+      ulonglong2 e = F.list[bb][i];
+      const int64_t u = (int64_t)(uint32_t)e.x - vbase;
+      if (u < u_first) continue;
+      int64_t s, en;
+      row_range(e, offs, vbase, &s, &en);
+      const int64_t slot = (u - u_first) * K;
+      const ulonglong2* cp = reinterpret_cast<const ulonglong2*>(cache + slot);
+      uint64_t k[K];
+#pragma unroll
+      for (int q = 0; q < K / 2; ++q) {
+        const ulonglong2 x = __ldg(cp + q);
+        k[2 * q] = x.x;
+        k[2 * q + 1] = x.y;
+      }
+      uint32_t wd[K];
+#pragma unroll
+      for (int q = 0; q < K; ++q) wd[q] = k[q] ? bits[(uint32_t)k[q] >> 5] : 0xffffffffu;
+      int hit = -1;
+#pragma unroll
+      for (int q = K - 1; q >= 0; --q)
+        if (!((wd[q] >> ((uint32_t)k[q] & 31)) & 1u)) hit = q;
+      if (hit >= 0) {
+        e.y = (1ull << 40) | (uint64_t)(M0 + slot + hit);
+      } else if (en - s <= K) {
+        e.y = (uint64_t)(M0 + slot);
+      } else {
+        left += (unsigned long long)(en - s);
+        continue;
+      }
+      F.list[bb][i].y = e.y;
+      ++served;
+    }
+  }
+  for (int o = 16; o; o >>= 1) {
+    served += __shfl_xor_sync(0xffffffffu, served, o);
+    left += __shfl_xor_sync(0xffffffffu, left, o);
+  }
+  if ((threadIdx.x & 31) == 0) {
+    if (served) atomicAdd(&cnt[0], served);
+    if (left) atomicAdd(&cnt[1], left);
   }
 }
 

@@ -175,6 +175,15 @@ struct lmatch_graph {
   uint64_t* host_adj_dev = nullptr;  // its device alias
   uint64_t* ring[2] = {nullptr, nullptr};
   cudaStream_t cs = nullptr;         // copy stream for streaming
+  // host-row key cache (NEXT-1): rows u >= u_first hold entries >= R; K keys per row in HBM,
+  // addressed through AdjView as indices >= M0
+  int host_cache = 1;
+  uint64_t* cache = nullptr;
+  int64_t cap_cache = -1;
+  int64_t u_first = 0, M0 = 0, nchunks = 0;
+  int64_t* chunk_rows = nullptr;     // device [nchunks + 1]: row holding each chunk's first entry
+  int64_t cap_chunk_rows = -1;
+  bool use_cache() const { return streaming && cache != nullptr; }
   cudaEvent_t ev_full[2] = {}, ev_free[2] = {};
   int sweep_grid = 0;
   alignas(64) CUtensorMap tmap;  // adjacency as a [ceil(m/16)][16] u64 tensor, 128B swizzle
@@ -226,7 +235,11 @@ struct lmatch_graph {
   cudaGraph_t graph = nullptr;
   cudaStream_t gstream = nullptr;      // stream the graph was captured on (capture needs its own)
 
-  lm::AdjView view() const { return lm::AdjView{adj, host_adj_dev - R, R}; }
+  lm::AdjView view() const {
+    lm::AdjView v{adj, host_adj_dev - R, R};
+    if (use_cache()) { v.cache_off = cache - M0; v.M0 = M0; }
+    return v;
+  }
   const lm::RoundArgs* ra() const { return d_rargs; }
   lm::RoundArgs rargs() const {
     lm::RoundArgs a;
@@ -579,6 +592,29 @@ int alloc_bins(lmatch_graph* g, cudaStream_t st) {
   return LMATCH_OK;
 }
 
+// Out-of-core host-row cache (NEXT-1): chunk k of the streamed part covers entries
+// [R + k C, min(R + (k+1) C, m)); chunk_rows[k] = row holding its first entry, chunk_rows[nchunks]
+// = row holding entry m - 1.  Host rows are u >= u_first = chunk_rows[0], kCacheK slots each.
+int build_cache_index(lmatch_graph* g, cudaStream_t st) {
+  if (!g->streaming || !g->host_cache || g->n == 0 || g->m == 0) {
+    g->M0 = 0;
+    return LMATCH_OK;
+  }
+  const int64_t C = g->stream_chunk;
+  g->nchunks = (g->m - g->R + C - 1) / C;
+  TRY(ensure(g, &g->chunk_rows, &g->cap_chunk_rows, g->nchunks + 1));
+  lm::k_rows_of_entries<<<grid_for(g->nchunks + 1, 256, 4096), 256, 0, st>>>(
+      g->offs, g->n, g->R, C, g->m - 1, g->nchunks + 1, g->chunk_rows);
+  CKL();
+  int64_t uf = 0;
+  CK(cudaMemcpyAsync(&uf, g->chunk_rows, 8, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  g->u_first = uf;
+  TRY(ensure(g, &g->cache, &g->cap_cache, (g->n - uf) * lm::kCacheK));
+  g->M0 = g->m + 64;  // past the host part and its padding
+  return LMATCH_OK;
+}
+
 int finish_create(lmatch_graph* g, cudaStream_t st) {
   if (g->prune && (g->streaming || g->ghost)) g->prune = 0;  // resident single-graph only
   if (g->prune && !g->live) {
@@ -587,6 +623,7 @@ int finish_create(lmatch_graph* g, cudaStream_t st) {
   }
   TRY(build_index(g, st));
   TRY(alloc_bins(g, st));
+  TRY(build_cache_index(g, st));
   if (g->m > 0) {
     // self-loop keys -> 0: the sweep's tile pass over resident graphs, the row-based
     // kernel over out-of-core ones (rows may live in host memory)
@@ -656,6 +693,7 @@ int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** 
     if (opts->stream_chunk > 0) g->stream_chunk = opts->stream_chunk;
     g->round_loop = opts->round_loop;
     g->prune = opts->prune != 0;
+    g->host_cache = opts->host_cache >= 0;
   }
   CK(cudaGetDevice(&g->device));
   CK(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, g->device));
@@ -704,6 +742,20 @@ int round1_sweep(lmatch_graph* g, cudaStream_t st, int64_t* launches_out, int64_
     return LMATCH_OK;
   };
   if (rt > 0) TRY(sweep_launch(g->adj, 0, std::min(rt, g->ntiles)));
+  // host-row cache fill over entries [w0, w1) held at base[j - ebase], rows [*plo, *phi]
+  auto cache_fill = [&](const uint64_t* base, int64_t ebase, int64_t w0, int64_t w1,
+                        const int64_t* plo, const int64_t* phi) -> int {
+    lm::k_cache_fill<lm::kCacheK, false><<<(unsigned)(8 * g->num_sms), 256, 0, st>>>(
+        base, ebase, w0, w1, g->offs, plo, phi, g->u_first, g->cache);
+    CKL();
+    lm::k_cache_fill<lm::kCacheK, true><<<(unsigned)g->num_sms, 256, 0, st>>>(
+        base, ebase, w0, w1, g->offs, plo, phi, g->u_first, g->cache);
+    CKL();
+    launches += 2;
+    return LMATCH_OK;
+  };
+  // the row holding entry R may start in the resident prefix: its resident part first
+  if (g->use_cache() && g->R > 0) TRY(cache_fill(g->adj, 0, 0, g->R, g->chunk_rows, g->chunk_rows));
   if (g->streaming) {
     const int64_t C = g->stream_chunk;
     for (int64_t e0 = g->R, k = 0; e0 < g->m; e0 += C, ++k) {
@@ -716,6 +768,8 @@ int round1_sweep(lmatch_graph* g, cudaStream_t st, int64_t* launches_out, int64_
       bytes_streamed += cnt * 8;
       CK(cudaStreamWaitEvent(st, g->ev_full[slot], 0));
       TRY(sweep_launch(g->ring[slot], e0 / kTile, std::min(g->ntiles, (e0 + cnt + kTile - 1) / kTile)));
+      if (g->use_cache())
+        TRY(cache_fill(g->ring[slot], e0, e0, e0 + cnt, g->chunk_rows + k, g->chunk_rows + k + 1));
       CK(cudaEventRecord(g->ev_free[slot], st));
     }
   }
@@ -771,7 +825,8 @@ void lmatch_destroy(lmatch_graph* g) {
   if (g->graph) cudaGraphDestroy(g->graph);
   if (g->gstream) cudaStreamDestroy(g->gstream);
   if (g->h_rstate) cudaFreeHost(g->h_rstate);
-  void* pdev[] = {g->bounds, g->ghost, g->claims, g->claim_cnt, g->rstate, g->rlog, g->d_rargs};
+  void* pdev[] = {g->bounds, g->ghost, g->claims, g->claim_cnt, g->rstate, g->rlog, g->d_rargs,
+                  g->cache, g->chunk_rows, g->live};
   for (void* p : pdev) if (p) cudaFree(p);
   if (g->h_claim_cnt) cudaFreeHost(g->h_claim_cnt);
   if (g->h_res) cudaFreeHost(g->h_res);
@@ -922,6 +977,12 @@ static int seq_body(lmatch_graph* g, cudaStream_t st, int cur, const int64_t* nF
   const unsigned long long* cF = g->counters + lm::cnt_F(cur, 0);
   int64_t nF = 0;
   for (int b = 0; b < lm::kBins; ++b) nF += nFb[b];
+  if (g->use_cache() && nF > 0) {
+    lm::k_cache_redirect<lm::kCacheK><<<grid_for(nF, 256, 65536), 256, 0, st>>>(
+        Fb, cF, g->offs, g->cache, g->bits, g->u_first, g->M0, g->v0, g->counters + lm::kCntCache);
+    CKL();
+    ++*launches;
+  }
 #define PIPE_OR_BIN(b, PG, PU, BG, BU, AG, AU)                                                      \
   if (nFb[b]) {                                                                                   \
     if (g->prune) {                                                                               \
@@ -1036,7 +1097,8 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
   //              1 = host-driven launches for every round;
   //              2 = persistent kernel for every round after round 1;
   //              3 = CUDA graph {round 1, persistent kernel} (no host work per run).
-  const int mode = g->round_loop;
+  // the cache redirect runs in the host-driven round body only
+  const int mode = g->use_cache() ? 1 : g->round_loop;
   const bool use_graph = mode == 3 && !g->streaming;
   int64_t launches = 0, sweep_launches = 0, bytes_streamed = 0;
 
@@ -1081,6 +1143,8 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
     g->h_resc[0] = 0;
   }
   CK(cudaMemcpyAsync(g->h_rstate, g->rstate, sizeof(lm::RoundState), cudaMemcpyDeviceToHost, st));
+  if (g->use_cache())
+    CK(cudaMemcpyAsync(g->h_counters, g->counters, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
   if (tm) CK(cudaEventRecord(g->ev[5], st));
   CK(cudaStreamSynchronize(st));
   const lm::RoundState rs = *g->h_rstate;
@@ -1113,6 +1177,11 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
     stats->kernel_launches = launches;
     stats->bytes_streamed = bytes_streamed;
     stats->resident_entries = g->R;
+    if (g->use_cache()) {
+      stats->cache_rows = (int64_t)g->h_counters[lm::kCntCache];
+      stats->host_entries_read = (int64_t)g->h_counters[lm::kCntCache + 1];
+      stats->cache_bytes = g->cap_cache * 8;
+    }
     if (tm) {
       float a = 0, b = 0, c = 0, d = 0, e = 0;
       CK(cudaEventElapsedTime(&a, g->ev[0], g->ev[5]));

@@ -265,6 +265,62 @@ def test_out_of_core_streaming(lm, maker, frac, chunk):
     assert st["sweep_launches"] >= 2
 
 
+def _hub_graph(seed=3):
+    """Hubs of 20k / 7k / 6k leaves (rows far longer than a stream chunk and than the cache
+    fill's 4096-entry CTA threshold), ties among hub edges, and random edges between leaves."""
+    rng = np.random.default_rng(seed)
+    edges = [(0, v, float(np.float32(rng.random() * 0.5 + 0.25))) for v in range(3, 20003)]
+    edges += [(1, v, float(np.float32(rng.random()))) for v in range(15000, 22001)]
+    edges += [(2, v, 0.5) for v in range(100, 6100)]
+    for _ in range(8000):
+        u, v = rng.integers(3, 22001, size=2)
+        if u != v:
+            edges.append((int(u), int(v), float(np.float32(1 - rng.random()))))
+    return graphgen.from_edges(22001, edges)
+
+
+@pytest.mark.parametrize("maker,frac,chunk", [
+    (lambda: graphgen.rmat(16, 16, seed=5), 0.3, 4096),
+    (lambda: graphgen.rmat(15, 16, seed=7, weights="paper"), 0.0, 1024),   # ties, nothing resident
+    (lambda: graphgen.er(1 << 15, 16.0, seed=2), 0.5, 8192),
+    (lambda: graphgen.mesh(200, keep=0.6, seed=3), 0.2, 2048),             # degree <= 4: all cached
+    (lambda: graphgen.mesh(48, seed=1, weights="gradient"), 0.4, 512),     # many rounds
+    (_hub_graph, 0.1, 1024),                                               # hubs span many chunks
+    (_hub_graph, 0.0, 4096),
+])
+def test_out_of_core_host_cache(lm, maker, frac, chunk):
+    """NEXT-1 host-row key cache (top-8 keys of every streamed row, filled in round 1): bit-exact
+    with the oracle and identical to the cache-off run; the cache must take rows off the
+    zero-copy path, and with the cache off every host frontier row is read from host memory."""
+    g = maker()
+    budget = int(8 * g.m * frac) + 2 * 8 * chunk
+    mate, st = check_parity(lm, g, hbm_budget_bytes=budget, stream_chunk=chunk)
+    assert st["resident_entries"] < g.m
+    assert st["cache_bytes"] > 0
+    mate0, st0 = run_gpu(lm, g, hbm_budget_bytes=budget, stream_chunk=chunk, host_cache=False)
+    np.testing.assert_array_equal(mate, mate0)
+    assert st0["cache_bytes"] == 0 and st0["cache_rows"] == 0
+    assert st["rounds"] == st0["rounds"] and st["weight"] == st0["weight"]
+    if st["rounds"] > 1:
+        assert st["cache_rows"] > 0
+
+
+def test_out_of_core_cache_repeat_and_reload(lm):
+    """The cache is refilled by every run (and after a reload with other weights)."""
+    g = graphgen.rmat(14, 16, seed=21)
+    g2 = graphgen.rmat(14, 16, seed=21, weights="paper")
+    assert g2.m == g.m and g2.n == g.n
+    budget = 8 * g.m // 4 + 2 * 8 * 1024
+    with lm.Matcher(g, hbm_budget_bytes=budget, stream_chunk=1024) as M:
+        a, _ = M.run()
+        b, _ = M.run()
+        np.testing.assert_array_equal(a, b)
+        np.testing.assert_array_equal(a, oracle.greedy(g).mate)
+        M.reload(g2.offsets, g2.col, g2.w)
+        c, _ = M.run()
+        np.testing.assert_array_equal(c, oracle.greedy(g2).mate)
+
+
 def test_out_of_core_weight_and_symmetry(lm):
     g = graphgen.rmat(13, 16, seed=9)
     with lm.Matcher(g, hbm_budget_bytes=8 * g.m // 3, stream_chunk=2048, validate_level=2) as M:
