@@ -56,6 +56,9 @@ def parse():
                         "from pinned host memory in round 1 and read zero-copy afterwards")
     p.add_argument("--stream-chunk", type=int, default=0, help="entries per streamed chunk (0 = default)")
     p.add_argument("--prune", action="store_true", help="A7 in-place pruning (lmatch_opts.prune)")
+    p.add_argument("--batches", type=int, default=0,
+                   help="paper-style batch count N_i (lmatch_opts.batches): B > 1 streams the whole "
+                        "adjacency from pinned host memory as B batches in round 1")
     p.add_argument("--no-host-cache", action="store_true",
                    help="out-of-core: disable the top-8 host-row key cache (lmatch_opts.host_cache = -1)")
     p.add_argument("--partitioned", action="store_true",
@@ -421,7 +424,8 @@ def main():
     # CSR); create is untimed: P:179 excludes I/O, allocation, CSR construction and the transfer
     opts = lm.make_opts(validate_level=1, timing=1,
                         hbm_budget_bytes=int(a.hbm_budget_gb * 1e9), stream_chunk=a.stream_chunk,
-                        prune=a.prune, host_cache=not a.no_host_cache)
+                        prune=a.prune, host_cache=not a.no_host_cache,
+                        batches=a.batches)
     pinned_host = d_off is None
     if pinned_host:
         h = lm.lmatch_create_ex(g.offsets, g.col, g.w, n, m, opts)
@@ -517,8 +521,8 @@ def main():
                "includes": "lmatch_reload (H2D + pack + validate + index) + lmatch_run (+ mate D2H)"}
 
     ooc = None
-    if a.hbm_budget_gb > 0:
-        ooc = {"hbm_budget_bytes": int(a.hbm_budget_gb * 1e9),
+    if a.hbm_budget_gb > 0 or a.batches > 1:
+        ooc = {"batches": a.batches,"hbm_budget_bytes": int(a.hbm_budget_gb * 1e9),
                "resident_entries": int(last["resident_entries"]),
                "resident_frac": last["resident_entries"] / max(m, 1),
                "bytes_streamed_per_step": int(last["bytes_streamed"]),

@@ -108,7 +108,14 @@ typedef struct lmatch_opts {
                                  neighbours), so only rows whose 8 heaviest neighbours are all
                                  matched are read from host memory.  Same result.  Rounds >= 2
                                  of an out-of-core run with the cache are host-driven launches */
-  int32_t reserved[9];
+  int32_t batches;            /* paper-style batch count N_i (Alg. 2 L3-5; SURVEY 8(f)
+                                 NEXT-2): 0 or 1 = default (resident, or hbm_budget_bytes decides);
+                                 B > 1 = nothing resident: the adjacency lives in pinned host
+                                 memory as B entry-balanced batches (tile-rounded; a row spanning
+                                 two batches is merged with the u64 max) streamed through the 2-slot device ring in round 1 (2 streams,
+                                 double buffering).  Overrides hbm_budget_bytes and
+                                 stream_chunk */
+  int32_t reserved[8];
 } lmatch_opts;
 
 /* Filled by lmatch_run / lmatch_run_device when non-NULL. */
@@ -250,6 +257,47 @@ LMATCH_API int lmatch_part_point(lmatch_graph* g, void* stream, int64_t* claim_c
  * u with mate[u] > u (fp64); *matched_local = owned matched vertices.  Synchronises. */
 LMATCH_API int lmatch_part_finish(lmatch_graph* g, int32_t* d_mate_local, void* stream,
                                   double* w_local, int64_t* matched_local);
+
+/* ---------------------------------------------------------------------------------------------
+ * Peer-memory exchange (the same partitioned round; the library's kernels move the data).
+ * Replaces the caller-side all-to-all / allgather / allreduce above with stores into the peers'
+ * memory (NVLink 5 / NVSwitch between GPUs; CUDA IPC across processes, plain pointers within one
+ * process), fused into the kernels that produce the data:
+ *   - the claims kernels store each claim (v | u << 32) straight into the owner's inbox segment
+ *     for this part and count it there with a system-scope atomic (replaces the pointer
+ *     exchange, Alg. 2 L7);
+ *   - the match step pushes every owned bitmap word that changed into every peer's replica
+ *     (replaces nccl_AllReduce(mate), Alg. 2 L9);
+ *   - the compaction pushes this part's frontier size into every peer's slot (termination,
+ *     P:159).
+ * Setup, on every part: lmatch_p2p_enable(g, part index) (allocates the exchange window: inbox
+ * nparts x max-part-size uint64, counts, slots), then for every other part either
+ * lmatch_p2p_attach_local(g, peer, peer_handle) (same process; peer access is enabled when the
+ * handles live on different devices) or lmatch_p2p_export on the peer + lmatch_p2p_attach(g, peer,
+ * handles) here (another process: 128 bytes = two cudaIpcMemHandle_t, passed by the caller).
+ * A round (the caller puts a barrier -- every part's stream drained, e.g. synchronise + a host
+ * barrier -- at each "|"):
+ *   | lmatch_p2p_begin / lmatch_p2p_point | lmatch_p2p_match | lmatch_p2p_compact |
+ *   lmatch_p2p_frontier_total -> stop when 0, else the next lmatch_p2p_point
+ * and lmatch_part_finish at the end.  Calls are stream-ordered and do not synchronise, except
+ * lmatch_p2p_compact and lmatch_p2p_frontier_total (they return host values).  Result: as above,
+ * bit-identical to the single-GPU run.  Calls on a handle without enable / with a peer missing
+ * return ESTATE; lmatch_part_begin/point/apply on an enabled handle return ESTATE.
+ * ------------------------------------------------------------------------------------------- */
+LMATCH_API int lmatch_p2p_enable(lmatch_graph* g, int32_t part_index);
+LMATCH_API int lmatch_p2p_attach_local(lmatch_graph* g, int32_t peer, lmatch_graph* peer_handle);
+/* handles: host buffer of 128 bytes (written by export, read by attach). */
+LMATCH_API int lmatch_p2p_export(const lmatch_graph* g, void* handles);
+LMATCH_API int lmatch_p2p_attach(lmatch_graph* g, int32_t peer, const void* handles);
+LMATCH_API int lmatch_p2p_begin(lmatch_graph* g, void* stream);
+LMATCH_API int lmatch_p2p_point(lmatch_graph* g, void* stream);
+LMATCH_API int lmatch_p2p_match(lmatch_graph* g, void* stream);
+/* *nF_local = this part's next frontier size (synchronises `stream`). */
+LMATCH_API int lmatch_p2p_compact(lmatch_graph* g, void* stream, int64_t* nF_local);
+/* *nF_total = the sum of every part's pushed frontier size (synchronises `stream`). */
+LMATCH_API int lmatch_p2p_frontier_total(lmatch_graph* g, void* stream, int64_t* nF_total);
+/* Synchronise `stream` (NULL = the handle's stream): the caller's half of a barrier. */
+LMATCH_API int lmatch_p2p_sync(lmatch_graph* g, void* stream);
 
 /* Release everything the handle owns.  NULL-safe. */
 LMATCH_API void lmatch_destroy(lmatch_graph* g);

@@ -44,7 +44,8 @@ class Opts(ctypes.Structure):
         ("max_rounds", ctypes.c_int64), ("upload_chunk", ctypes.c_int64),
         ("hbm_budget_bytes", ctypes.c_int64), ("stream_chunk", ctypes.c_int64),
         ("round_loop", ctypes.c_int32), ("prune", ctypes.c_int32),
-        ("host_cache", ctypes.c_int32), ("reserved", ctypes.c_int32 * 9),
+        ("host_cache", ctypes.c_int32), ("batches", ctypes.c_int32),
+        ("reserved", ctypes.c_int32 * 8),
     ]
 
 
@@ -242,7 +243,8 @@ class Matcher:
     def __init__(self, offsets=None, col=None, w=None, *, handle: int | None = None,
                  validate_level: int = 1, timing: bool = False, upload_chunk: int = 0,
                  max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
-                 round_loop: int = 0, prune: bool = False, host_cache: bool = True):
+                 round_loop: int = 0, prune: bool = False, host_cache: bool = True,
+                 batches: int = 0):
         self.h = None
         if handle is not None:
             self.h = handle
@@ -252,7 +254,7 @@ class Matcher:
             self.h = lmatch_create_ex(offsets, col, w,
                                       opts=make_opts(validate_level, timing, upload_chunk,
                                                      max_rounds, hbm_budget_bytes, stream_chunk,
-                                                     round_loop, prune, host_cache))
+                                                     round_loop, prune, host_cache, batches))
         self.info = lmatch_info(self.h)
 
     @classmethod
@@ -295,7 +297,8 @@ class Matcher:
 
 def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int = 0,
               max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
-              round_loop: int = 0, prune: bool = False, host_cache: bool = True) -> Opts:
+              round_loop: int = 0, prune: bool = False, host_cache: bool = True,
+              batches: int = 0) -> Opts:
     """round_loop (include/lmatch.h): 0 = hybrid (work-sized launches, then one persistent kernel
     for the tail; default), 1 = host-driven launches only, 2 = persistent kernel after round 1,
     3 = CUDA graph {round 1, persistent kernel}."""
@@ -303,6 +306,7 @@ def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int =
     o.round_loop = int(round_loop)
     o.prune = int(bool(prune))
     o.host_cache = 0 if host_cache else -1
+    o.batches = int(batches)
     o.hbm_budget_bytes = int(hbm_budget_bytes)
     o.stream_chunk = int(stream_chunk)
     o.validate_level = int(validate_level)

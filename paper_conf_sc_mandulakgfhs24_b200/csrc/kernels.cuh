@@ -1764,6 +1764,10 @@ struct Claims {
   unsigned long long* count;   // [P]
   const int64_t* bounds;       // [P+1]
   int P;
+  // peer-memory exchange (lmatch_p2p_*): claims for part d are stored straight into d's inbox
+  // segment for this part (dseg[d]) and counted there (dcnt[d]); NULL = local segments above
+  uint64_t* const* dseg = nullptr;
+  unsigned long long* const* dcnt = nullptr;
 };
 // warp-collective (all 32 lanes call it): lanes with the same destination share one atomic
 __device__ __forceinline__ void claim_append(const Claims& C, bool pred, uint32_t v, uint32_t u) {
@@ -1771,10 +1775,12 @@ __device__ __forceinline__ void claim_append(const Claims& C, bool pred, uint32_
   const unsigned peers = __match_any_sync(0xffffffffu, d);
   if (!pred) return;
   const int lane = threadIdx.x & 31, leader = __ffs(peers) - 1;
+  unsigned long long* cnt = C.dcnt ? C.dcnt[d] : &C.count[d];
+  uint64_t* seg = C.dseg ? C.dseg[d] : C.seg + (int64_t)d * C.cap;
   unsigned long long base = 0;
-  if (lane == leader) base = atomicAdd(&C.count[d], (unsigned long long)__popc(peers));
+  if (lane == leader) base = atomicAdd_system(cnt, (unsigned long long)__popc(peers));
   base = __shfl_sync(peers, base, leader);
-  C.seg[(int64_t)d * C.cap + (int64_t)(base + __popc(peers & lanemask_lt()))] = make_pair(v, u);
+  seg[(int64_t)(base + __popc(peers & lanemask_lt()))] = make_pair(v, u);
 }
 // round 1: every owned vertex whose pointer targets a remote vertex
 __global__ void k_claims_all(const uint64_t* __restrict__ best, int64_t n_loc, int64_t vbase,
@@ -1822,6 +1828,61 @@ __global__ void k_match_claims(const uint64_t* __restrict__ recv, int64_t nrecv,
     if (kv != 0 && (uint32_t)kv == u) atomicOr(&bits[v >> 5], 1u << (v & 31));
   }
 }
+// ---- peer-memory exchange (lmatch_p2p_*): the inbox holds P segments of `cap` claims, segment
+// s written by part s over NVLink / peer memory, with its count in cnt[s] (device-resident, so
+// no host round trip decides the grid: the kernels walk every segment).
+__global__ void k_apply_inbox(const uint64_t* __restrict__ inbox, int64_t cap,
+                              const unsigned long long* __restrict__ cnt, int P, uint32_t* ghost) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int s = 0; s < P; ++s) {
+    const int64_t c = (int64_t)cnt[s];
+    const uint64_t* seg = inbox + (int64_t)s * cap;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < c; i += stride) {
+      const uint64_t x = seg[i];
+      ghost[(uint32_t)(x >> 32)] = (uint32_t)x;
+    }
+  }
+}
+__global__ void k_match_inbox(const uint64_t* __restrict__ inbox, int64_t cap,
+                              unsigned long long* cnt, int P, const uint64_t* __restrict__ best,
+                              int64_t vbase, uint32_t* bits) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int s = 0; s < P; ++s) {
+    const int64_t c = (int64_t)cnt[s];
+    const uint64_t* seg = inbox + (int64_t)s * cap;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < c; i += stride) {
+      const uint64_t x = seg[i];
+      const uint32_t v = (uint32_t)x, u = (uint32_t)(x >> 32);
+      const uint64_t kv = best[v - vbase];
+      if (kv != 0 && (uint32_t)kv == u) atomicOr(&bits[v >> 5], 1u << (v & 31));
+    }
+  }
+}
+// Push the owned bitmap words that changed since the last push into every peer's replica
+// (plain 4-byte stores into peer memory; one owner per word, so no atomics).  Replaces the
+// bitmap allgather (nccl_AllReduce(mate), Alg. 2 L9) with n/8 bytes per round at most.
+__global__ void k_push_bits(const uint32_t* __restrict__ bits, uint32_t* __restrict__ shadow,
+                            int64_t w0, int64_t nw, uint32_t* const* __restrict__ peer_bits,
+                            int P, int me) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nw; i += stride) {
+    const uint32_t x = bits[w0 + i];
+    if (x == shadow[i]) continue;
+    shadow[i] = x;
+    for (int p = 0; p < P; ++p)
+      if (p != me) peer_bits[p][w0 + i] = x;
+  }
+}
+// frontier-size exchange for termination: this part's count into every peer's slot [me]
+__global__ void k_push_count(const unsigned long long* __restrict__ cnt, int ncnt,
+                             unsigned long long* const* __restrict__ peer_slot, int P) {
+  if (threadIdx.x == 0 && blockIdx.x == 0) {
+    unsigned long long t = 0;
+    for (int i = 0; i < ncnt; ++i) t += cnt[i];
+    for (int p = 0; p < P; ++p) peer_slot[p][0] = t;
+  }
+}
+
 // round 1 match over every owned vertex (owned range starts on a 32-vertex boundary)
 __global__ void k_match_part_all(const uint64_t* __restrict__ best, int64_t n_loc, int64_t vbase,
                                  int64_t vend, const uint32_t* __restrict__ ghost, uint32_t* bits) {
@@ -2039,46 +2100,106 @@ __device__ __forceinline__ uint64_t warp_topk_pop(uint64_t (&t)[K]) {
 // Fill / merge the cache of rows [*plo, *phi] from entries [w0, w1) held at base[j - ebase].
 // A row starting inside the window overwrites its slots; a row that started before it (spans a
 // chunk boundary or the resident/streamed split) merges with the slots written earlier on the
-// same stream.  BIG = false: one warp per row of <= kCacheBigRow in-window entries; BIG = true:
-// one CTA per longer row (per-warp top-K, then warp 0 merges the 8 warps' lists in smem).
+// same stream.  Each warp takes 32 consecutive rows: a row with <= 16 in-window entries is
+// reduced by its own lane (register top-K), a longer one by the whole warp (per-lane top-K, then
+// K warp-wide pops), and a row with more than kCacheBigRow entries is listed for
+// k_cache_fill_big (one CTA per row).
 constexpr int64_t kCacheBigRow = 4096;
-template <int K, bool BIG>
+template <int K>
+__device__ __forceinline__ void cache_row_warp(const uint64_t* __restrict__ base, int64_t ebase,
+                                               int64_t a, int64_t b, bool merge,
+                                               uint64_t* __restrict__ c) {
+  const int lane = threadIdx.x & 31;
+  uint64_t t[K];
+#pragma unroll
+  for (int i = 0; i < K; ++i) t[i] = 0ull;
+  for (int64_t j = a + lane; j < b; j += 32) topk_insert<K>(t, base[j - ebase]);
+  if (merge && lane < K) topk_insert<K>(t, c[lane]);
+  const uint64_t mine = warp_topk_pop<K>(t);
+  if (lane < K) c[lane] = mine;
+}
+template <int K>
 __global__ void __launch_bounds__(256) k_cache_fill(const uint64_t* __restrict__ base, int64_t ebase,
                                                     int64_t w0, int64_t w1,
                                                     const int64_t* __restrict__ offs,
                                                     const int64_t* __restrict__ plo,
                                                     const int64_t* __restrict__ phi, int64_t u_first,
-                                                    uint64_t* __restrict__ cache) {
+                                                    uint64_t* __restrict__ cache,
+                                                    int64_t* __restrict__ big,
+                                                    unsigned long long* __restrict__ nbig) {
+  const int lane = threadIdx.x & 31;
+  const int64_t ulo = *plo, uhi = *phi;
+  const int64_t nrows = uhi - ulo + 1;
+  const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t r0 = wid * 32; r0 < nrows; r0 += nw * 32) {
+    const int64_t u = ulo + r0 + lane;
+    int64_t s = 0, a = 0, b = 0;
+    if (u <= uhi) {
+      s = offs[u];
+      a = max(s, w0);
+      b = min(offs[u + 1], w1);
+    }
+    const int64_t len = b > a ? b - a : 0;
+    uint64_t* c = cache + (u - u_first) * K;
+    if (len > 0 && len <= 16) {
+      uint64_t t[K];
+#pragma unroll
+      for (int i = 0; i < K; ++i) t[i] = 0ull;
+      for (int64_t j = a; j < b; ++j) topk_insert<K>(t, base[j - ebase]);
+      if (s < w0) {
+#pragma unroll
+        for (int i = 0; i < K; ++i) topk_insert<K>(t, c[i]);
+      }
+      ulonglong2* c2 = reinterpret_cast<ulonglong2*>(c);
+#pragma unroll
+      for (int i = 0; i < K / 2; ++i) c2[i] = make_ulonglong2(t[2 * i], t[2 * i + 1]);
+    } else if (len > kCacheBigRow) {
+      big[atomicAdd(nbig, 1ull)] = u;
+    }
+    unsigned mid = __ballot_sync(0xffffffffu, len > 16 && len <= kCacheBigRow);
+    while (mid) {
+      const int l = __ffs(mid) - 1;
+      mid &= mid - 1;
+      const int64_t ul = __shfl_sync(0xffffffffu, u, l);
+      const int64_t al = __shfl_sync(0xffffffffu, a, l), bl = __shfl_sync(0xffffffffu, b, l);
+      const int64_t sl = __shfl_sync(0xffffffffu, s, l);
+      cache_row_warp<K>(base, ebase, al, bl, sl < w0, cache + (ul - u_first) * K);
+    }
+  }
+}
+// the listed long rows: one CTA per row (per-warp top-K, then warp 0 merges the 8 lists)
+template <int K>
+__global__ void __launch_bounds__(256) k_cache_fill_big(const uint64_t* __restrict__ base,
+                                                        int64_t ebase, int64_t w0, int64_t w1,
+                                                        const int64_t* __restrict__ offs,
+                                                        const int64_t* __restrict__ big,
+                                                        const unsigned long long* __restrict__ nbig,
+                                                        int64_t u_first, uint64_t* __restrict__ cache) {
   __shared__ uint64_t cand[8][K];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int64_t ulo = *plo, uhi = *phi;
-  const int64_t first = BIG ? (int64_t)blockIdx.x : ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int64_t step = BIG ? (int64_t)gridDim.x : ((int64_t)gridDim.x * blockDim.x) >> 5;
-  const int64_t lstride = BIG ? (int64_t)blockDim.x : 32;
-  const int64_t lid = BIG ? (int64_t)threadIdx.x : lane;
-  for (int64_t u = ulo + first; u <= uhi; u += step) {
-    const int64_t s = offs[u], en = offs[u + 1];
-    const int64_t a = max(s, w0), b = min(en, w1);
-    if (a >= b || ((b - a > kCacheBigRow) != BIG)) continue;
+  const int64_t nb = (int64_t)*nbig;
+  for (int64_t i = blockIdx.x; i < nb; i += gridDim.x) {
+    const int64_t u = big[i];
+    const int64_t s = offs[u];
+    const int64_t a = max(s, w0), b = min(offs[u + 1], w1);
     uint64_t t[K];
 #pragma unroll
-    for (int i = 0; i < K; ++i) t[i] = 0ull;
-    for (int64_t j = a + lid; j < b; j += lstride) topk_insert<K>(t, base[j - ebase]);
+    for (int q = 0; q < K; ++q) t[q] = 0ull;
+    for (int64_t j = a + threadIdx.x; j < b; j += blockDim.x) topk_insert<K>(t, base[j - ebase]);
     uint64_t* c = cache + (u - u_first) * K;
-    if (s < w0 && lid < K) topk_insert<K>(t, c[lid]);
+    if (s < w0 && threadIdx.x < K) topk_insert<K>(t, c[threadIdx.x]);
     uint64_t mine = warp_topk_pop<K>(t);
-    if (BIG) {
-      if (lane < K) cand[warp][lane] = mine;
-      __syncthreads();
-      if (warp == 0) {
+    if (lane < K) cand[warp][lane] = mine;
+    __syncthreads();
+    if (warp == 0) {
 #pragma unroll
-        for (int i = 0; i < K; ++i) t[i] = 0ull;
-        for (int q = lane; q < 8 * K; q += 32) topk_insert<K>(t, cand[q / K][q % K]);
-        mine = warp_topk_pop<K>(t);
-      }
-      __syncthreads();
+      for (int q = 0; q < K; ++q) t[q] = 0ull;
+      for (int q = lane; q < 8 * K; q += 32) topk_insert<K>(t, cand[q / K][q % K]);
+      mine = warp_topk_pop<K>(t);
+      if (lane < K) c[lane] = mine;
     }
-    if ((!BIG || warp == 0) && lane < K) c[lane] = mine;
+    __syncthreads();
   }
 }
 

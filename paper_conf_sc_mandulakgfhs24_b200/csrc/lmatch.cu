@@ -161,6 +161,22 @@ struct lmatch_graph {
   unsigned long long* claim_cnt = nullptr;    // device [P]
   unsigned long long* h_claim_cnt = nullptr;  // pinned [P]
   int part_round = 0, part_cur = 0;
+  std::vector<int64_t> hbounds;      // host copy of the part bounds [P+1]
+  // peer-memory exchange (lmatch_p2p_*): window = inbox [P][win_cap] u64 | inbox counts [P] |
+  // frontier-size slots [P]; peers store into it (and into `bits`) over NVLink / peer memory
+  int p2p = 0, me = 0;
+  int64_t win_cap = 0;
+  uint64_t* win = nullptr;
+  uint32_t* shadow = nullptr;        // owned bitmap words as last pushed to the peers
+  uint64_t** d_dseg = nullptr;       // device [P]: my inbox segment in each peer's window
+  unsigned long long** d_dcnt = nullptr;  // device [P]: its count
+  uint32_t** d_dbits = nullptr;      // device [P]: each peer's bitmap replica
+  unsigned long long** d_dnf = nullptr;   // device [P]: my frontier-size slot in each peer
+  std::vector<uint64_t*> h_dseg;
+  std::vector<unsigned long long*> h_dcnt, h_dnf;
+  std::vector<uint32_t*> h_dbits;
+  std::vector<void*> ipc_opened;     // peer allocations opened with cudaIpcOpenMemHandle
+  unsigned long long* h_nf = nullptr;  // pinned [P]
   float part_sweep_ms = 0.f;  // (timing=1) last lmatch_part_begin's round-1 sweep
   int validate_level = 1;
   int timing = 0;
@@ -170,6 +186,7 @@ struct lmatch_graph {
   int64_t R = 0;
   int64_t stream_chunk = 1ll << 24;
   int64_t hbm_budget = 0;
+  int batches = 0;                   // paper-style batch count (> 1: all streamed)
   bool streaming = false;
   uint64_t* host_adj = nullptr;      // pinned, mapped: entries [R, m)
   uint64_t* host_adj_dev = nullptr;  // its device alias
@@ -183,6 +200,8 @@ struct lmatch_graph {
   int64_t u_first = 0, M0 = 0, nchunks = 0;
   int64_t* chunk_rows = nullptr;     // device [nchunks + 1]: row holding each chunk's first entry
   int64_t cap_chunk_rows = -1;
+  int64_t* cache_big = nullptr;      // device [1 + cap]: count, then rows listed for the CTA fill
+  int64_t cap_cache_big = -1;
   bool use_cache() const { return streaming && cache != nullptr; }
   cudaEvent_t ev_full[2] = {}, ev_free[2] = {};
   int sweep_grid = 0;
@@ -315,7 +334,11 @@ int alloc_all(lmatch_graph* g) {
   TRY(dmalloc(g, &g->offs, (size_t)n + 1));
   // out-of-core split: keep a prefix of R entries (multiple of the stream chunk) in HBM
   g->R = m;
-  if (g->hbm_budget > 0 && 8 * m > g->hbm_budget) {
+  if (g->batches > 1 && m > 0) {  // paper-style batches: nothing resident, B streamed batches
+    g->stream_chunk = std::max<int64_t>(kTile, (m / g->batches + kTile - 1) / kTile * kTile);
+    g->R = 0;
+    g->streaming = true;
+  } else if (g->hbm_budget > 0 && 8 * m > g->hbm_budget) {
     const int64_t C = std::max<int64_t>(kTile, (g->stream_chunk / kTile) * kTile);
     g->stream_chunk = C;
     g->R = std::max<int64_t>(0, (g->hbm_budget / 8 - 2 * C) / C * C);
@@ -611,6 +634,8 @@ int build_cache_index(lmatch_graph* g, cudaStream_t st) {
   CK(cudaStreamSynchronize(st));
   g->u_first = uf;
   TRY(ensure(g, &g->cache, &g->cap_cache, (g->n - uf) * lm::kCacheK));
+  // a window holds at most (entries / kCacheBigRow) rows longer than kCacheBigRow
+  TRY(ensure(g, &g->cache_big, &g->cap_cache_big, std::max(C, g->R) / lm::kCacheBigRow + 8));
   g->M0 = g->m + 64;  // past the host part and its padding
   return LMATCH_OK;
 }
@@ -682,6 +707,7 @@ int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** 
     g->v0 = part->v0;
     g->n_global = part->n_global;
     g->P = part->P;
+    g->hbounds.assign(part->bounds, part->bounds + part->P + 1);
   }
   if (opts) {
     if (opts->use_device) CK(cudaSetDevice(opts->device));
@@ -694,6 +720,7 @@ int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** 
     g->round_loop = opts->round_loop;
     g->prune = opts->prune != 0;
     g->host_cache = opts->host_cache >= 0;
+    g->batches = opts->batches;
   }
   CK(cudaGetDevice(&g->device));
   CK(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, g->device));
@@ -745,11 +772,13 @@ int round1_sweep(lmatch_graph* g, cudaStream_t st, int64_t* launches_out, int64_
   // host-row cache fill over entries [w0, w1) held at base[j - ebase], rows [*plo, *phi]
   auto cache_fill = [&](const uint64_t* base, int64_t ebase, int64_t w0, int64_t w1,
                         const int64_t* plo, const int64_t* phi) -> int {
-    lm::k_cache_fill<lm::kCacheK, false><<<(unsigned)(8 * g->num_sms), 256, 0, st>>>(
-        base, ebase, w0, w1, g->offs, plo, phi, g->u_first, g->cache);
+    unsigned long long* nbig = reinterpret_cast<unsigned long long*>(g->cache_big);
+    CK(cudaMemsetAsync(nbig, 0, 8, st));
+    lm::k_cache_fill<lm::kCacheK><<<(unsigned)(8 * g->num_sms), 256, 0, st>>>(
+        base, ebase, w0, w1, g->offs, plo, phi, g->u_first, g->cache, g->cache_big + 1, nbig);
     CKL();
-    lm::k_cache_fill<lm::kCacheK, true><<<(unsigned)g->num_sms, 256, 0, st>>>(
-        base, ebase, w0, w1, g->offs, plo, phi, g->u_first, g->cache);
+    lm::k_cache_fill_big<lm::kCacheK><<<(unsigned)g->num_sms, 256, 0, st>>>(
+        base, ebase, w0, w1, g->offs, g->cache_big + 1, nbig, g->u_first, g->cache);
     CKL();
     launches += 2;
     return LMATCH_OK;
@@ -825,8 +854,11 @@ void lmatch_destroy(lmatch_graph* g) {
   if (g->graph) cudaGraphDestroy(g->graph);
   if (g->gstream) cudaStreamDestroy(g->gstream);
   if (g->h_rstate) cudaFreeHost(g->h_rstate);
+  for (void* p : g->ipc_opened) cudaIpcCloseMemHandle(p);
+  if (g->h_nf) cudaFreeHost(g->h_nf);
   void* pdev[] = {g->bounds, g->ghost, g->claims, g->claim_cnt, g->rstate, g->rlog, g->d_rargs,
-                  g->cache, g->chunk_rows, g->live};
+                  g->cache, g->chunk_rows, g->cache_big, g->live, g->win, g->shadow, g->d_dseg, g->d_dcnt,
+                  g->d_dbits, g->d_dnf};
   for (void* p : pdev) if (p) cudaFree(p);
   if (g->h_claim_cnt) cudaFreeHost(g->h_claim_cnt);
   if (g->h_res) cudaFreeHost(g->h_res);
@@ -1323,11 +1355,17 @@ static int part_claims_out(lmatch_graph* g, cudaStream_t st, int64_t* claim_coun
   return LMATCH_OK;
 }
 
-int lmatch_part_begin(lmatch_graph* g, void* stream, int64_t* claim_counts) {
-  if (!g || !g->ghost) { set_err("not a partition handle"); return LMATCH_ESTATE; }
-  g_err[0] = 0;
-  CK(cudaSetDevice(g->device));
-  cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
+static lm::Claims part_claims_desc(const lmatch_graph* g) {
+  lm::Claims Cl{g->claims, g->claim_cap, g->claim_cnt, g->bounds, g->P};
+  if (g->p2p) {
+    Cl.dseg = g->d_dseg;
+    Cl.dcnt = g->d_dcnt;
+  }
+  return Cl;
+}
+
+static int part_begin_impl(lmatch_graph* g, cudaStream_t st, int64_t* claim_counts) {
+  if (g->p2p) CK(cudaMemsetAsync(g->shadow, 0, (size_t)((g->n + 31) / 32 + 1) * 4, st));
   const int64_t nwords = (g->n_global + 31) / 32;
   lm::k_reset<<<grid_for(std::max(nwords, g->n_atomic), 256, 4096), 256, 0, st>>>(
       g->bits, nwords, g->best, g->atomic_rows, g->n_atomic, g->counters, lm::kNumCounters,
@@ -1341,7 +1379,7 @@ int lmatch_part_begin(lmatch_graph* g, void* stream, int64_t* claim_counts) {
   if (g->timing) CK(cudaEventRecord(g->ev[1], st));
   if (g->ntiles > 0 && g->n > 0) TRY(round1_sweep(g, st, &l, &sl, &bs));
   if (g->timing) CK(cudaEventRecord(g->ev[2], st));
-  lm::Claims Cl{g->claims, g->claim_cap, g->claim_cnt, g->bounds, g->P};
+  const lm::Claims Cl = part_claims_desc(g);
   if (g->n > 0) {
     lm::k_claims_all<<<grid_for(g->n, 256, 65536), 256, 0, st>>>(g->best, g->n, g->v0,
                                                                    g->v0 + g->n, Cl);
@@ -1349,9 +1387,20 @@ int lmatch_part_begin(lmatch_graph* g, void* stream, int64_t* claim_counts) {
   }
   g->part_round = 1;
   g->round_log.clear();
-  const int rc = part_claims_out(g, st, claim_counts);
-  if (!rc && g->timing) CK(cudaEventElapsedTime(&g->part_sweep_ms, g->ev[1], g->ev[2]));
+  const int rc = g->p2p ? LMATCH_OK : part_claims_out(g, st, claim_counts);
+  if (!rc && g->timing) {
+    CK(cudaStreamSynchronize(st));
+    CK(cudaEventElapsedTime(&g->part_sweep_ms, g->ev[1], g->ev[2]));
+  }
   return rc;
+}
+
+int lmatch_part_begin(lmatch_graph* g, void* stream, int64_t* claim_counts) {
+  if (!g || !g->ghost) { set_err("not a partition handle"); return LMATCH_ESTATE; }
+  if (g->p2p) { set_err("peer-memory handle: use lmatch_p2p_begin"); return LMATCH_ESTATE; }
+  g_err[0] = 0;
+  CK(cudaSetDevice(g->device));
+  return part_begin_impl(g, stream ? (cudaStream_t)stream : g->stream, claim_counts);
 }
 
 int lmatch_part_claims(const lmatch_graph* g, uint64_t** seg_ptrs) {
@@ -1362,6 +1411,7 @@ int lmatch_part_claims(const lmatch_graph* g, uint64_t** seg_ptrs) {
 
 int lmatch_part_apply(lmatch_graph* g, const uint64_t* d_recv, int64_t nrecv, void* stream) {
   if (!g || !g->ghost || g->part_round < 1) { set_err("lmatch_part_apply out of order"); return LMATCH_ESTATE; }
+  if (g->p2p) { set_err("peer-memory handle: use lmatch_p2p_match"); return LMATCH_ESTATE; }
   if (nrecv > 0 && !d_recv) { set_err("NULL claims"); return LMATCH_EINVAL; }
   CK(cudaSetDevice(g->device));
   cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
@@ -1449,10 +1499,7 @@ int lmatch_part_compact(lmatch_graph* g, void* stream, int64_t* nF_local) {
   return LMATCH_OK;
 }
 
-int lmatch_part_point(lmatch_graph* g, void* stream, int64_t* claim_counts) {
-  if (!g || !g->ghost || g->part_round < 1) { set_err("lmatch_part_point out of order"); return LMATCH_ESTATE; }
-  CK(cudaSetDevice(g->device));
-  cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
+static int part_point_impl(lmatch_graph* g, cudaStream_t st, int64_t* claim_counts) {
   const int cur = g->part_cur;
   int64_t nFb[lm::kBins], nF = 0;
   for (int b = 0; b < lm::kBins; ++b) { nFb[b] = (int64_t)g->h_counters[lm::cnt_F(cur, b)]; nF += nFb[b]; }
@@ -1463,16 +1510,23 @@ int lmatch_part_point(lmatch_graph* g, void* stream, int64_t* claim_counts) {
   if (nFb[1]) { lm::k_point_bin<LM_B1_G, LM_B1_U><<<grid_for(nFb[1] * LM_B1_G, 256, 65536), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, av, g->bits, g->best, g->v0); CKL(); }
   if (nFb[2]) { lm::k_point_bin<LM_B2_G, LM_B2_U><<<grid_for(nFb[2] * LM_B2_G, 256, 65536), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, av, g->bits, g->best, g->v0); CKL(); }
   if (nFb[3]) { lm::k_point_bin_cta<256, 4><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); }
-  CK(cudaMemsetAsync(g->claim_cnt, 0, (size_t)g->P * 8, st));
+  if (!g->p2p) CK(cudaMemsetAsync(g->claim_cnt, 0, (size_t)g->P * 8, st));
   if (nF > 0) {
-    lm::Claims Cl{g->claims, g->claim_cap, g->claim_cnt, g->bounds, g->P};
+    const lm::Claims Cl = part_claims_desc(g);
     lm::k_claims_bins<<<grid_for(nF, 256, 65536), 256, 0, st>>>(Fb, cF, g->v0, g->v0 + g->n, Cl);
     CKL();
   }
   g->round_log.insert(g->round_log.end(), {nF, nF + (int64_t)g->h_counters[lm::cnt_S(cur)],
                                            (int64_t)g->h_counters[lm::kCntSwept]});
   ++g->part_round;
-  return part_claims_out(g, st, claim_counts);
+  return g->p2p ? LMATCH_OK : part_claims_out(g, st, claim_counts);
+}
+
+int lmatch_part_point(lmatch_graph* g, void* stream, int64_t* claim_counts) {
+  if (!g || !g->ghost || g->part_round < 1) { set_err("lmatch_part_point out of order"); return LMATCH_ESTATE; }
+  if (g->p2p) { set_err("peer-memory handle: use lmatch_p2p_point"); return LMATCH_ESTATE; }
+  CK(cudaSetDevice(g->device));
+  return part_point_impl(g, stream ? (cudaStream_t)stream : g->stream, claim_counts);
 }
 
 int lmatch_part_finish(lmatch_graph* g, int32_t* d_mate_local, void* stream, double* w_local,
@@ -1529,5 +1583,194 @@ int lmatch_part_set_bits(lmatch_graph* g, const uint32_t* d_src, int64_t word_be
   return LMATCH_OK;
 }
 
-}  // extern "C"
+// ----------------------------------------------------------------- peer-memory exchange (A3/A5)
+// The partitioned round with the exchange done by the library's own kernels over peer memory
+// (CUDA IPC across processes / GPUs, plain pointers for parts in one process): the claims
+// kernels store straight into the owner's inbox, the match step pushes changed owned bitmap
+// words into every peer's replica, and the compaction pushes the frontier size into every
+// peer's slot.  The caller supplies the barriers between phases (include/lmatch.h).
+int lmatch_p2p_enable(lmatch_graph* g, int32_t me) {
+  if (!g || !g->ghost) { set_err("not a partition handle"); return LMATCH_ESTATE; }
+  if (me < 0 || me >= g->P || g->hbounds.size() != (size_t)g->P + 1 || g->hbounds[me] != g->v0 ||
+      g->hbounds[me + 1] != g->v0 + g->n) {
+    set_err("part index %d does not own rows [%lld, %lld)", me, (long long)g->v0, (long long)(g->v0 + g->n));
+    return LMATCH_EINVAL;
+  }
+  if (g->p2p) return LMATCH_OK;
+  CK(cudaSetDevice(g->device));
+  const int P = g->P;
+  int64_t cap = 1;
+  for (int p = 0; p < P; ++p) cap = std::max(cap, g->hbounds[p + 1] - g->hbounds[p]);
+  g->me = me;
+  g->win_cap = cap;
+  TRY(dmalloc(g, &g->win, (size_t)P * cap + 2 * (size_t)P));
+  CK(cudaMemset(g->win + (size_t)P * cap, 0, 2 * (size_t)P * 8));
+  TRY(dmalloc(g, &g->shadow, (size_t)(g->n + 31) / 32 + 1));
+  TRY(dmalloc(g, &g->d_dseg, (size_t)P));
+  TRY(dmalloc(g, &g->d_dcnt, (size_t)P));
+  TRY(dmalloc(g, &g->d_dbits, (size_t)P));
+  TRY(dmalloc(g, &g->d_dnf, (size_t)P));
+  CK(cudaHostAlloc(reinterpret_cast<void**>(&g->h_nf), (size_t)P * 8, cudaHostAllocDefault));
+  g->h_dseg.assign(P, nullptr);
+  g->h_dcnt.assign(P, nullptr);
+  g->h_dnf.assign(P, nullptr);
+  g->h_dbits.assign(P, nullptr);
+  g->p2p = 1;
+  // this part's own entries (its frontier-size slot is written like a peer's)
+  return lmatch_p2p_attach_local(g, me, g);
+}
 
+static int p2p_set_peer(lmatch_graph* g, int peer, uint64_t* pwin, uint32_t* pbits) {
+  const int P = g->P;
+  uint64_t* cnt = pwin + (size_t)P * g->win_cap;
+  g->h_dseg[peer] = pwin + (size_t)g->me * g->win_cap;
+  g->h_dcnt[peer] = reinterpret_cast<unsigned long long*>(cnt) + g->me;
+  g->h_dnf[peer] = reinterpret_cast<unsigned long long*>(cnt + P) + g->me;
+  g->h_dbits[peer] = pbits;
+  CK(cudaMemcpy(g->d_dseg, g->h_dseg.data(), (size_t)P * 8, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(g->d_dcnt, g->h_dcnt.data(), (size_t)P * 8, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(g->d_dnf, g->h_dnf.data(), (size_t)P * 8, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(g->d_dbits, g->h_dbits.data(), (size_t)P * 8, cudaMemcpyHostToDevice));
+  return LMATCH_OK;
+}
+
+int lmatch_p2p_attach_local(lmatch_graph* g, int32_t peer, lmatch_graph* pg) {
+  if (!g || !pg || !g->p2p || !pg->p2p) { set_err("lmatch_p2p_enable both handles first"); return LMATCH_ESTATE; }
+  if (peer < 0 || peer >= g->P || pg->me != peer || pg->P != g->P || pg->win_cap != g->win_cap ||
+      pg->n_global != g->n_global) {
+    set_err("peer handle does not match (part %d)", peer);
+    return LMATCH_EINVAL;
+  }
+  CK(cudaSetDevice(g->device));
+  if (pg->device != g->device) {
+    const cudaError_t e = cudaDeviceEnablePeerAccess(pg->device, 0);
+    if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) {
+      set_err("cudaDeviceEnablePeerAccess(%d): %s", pg->device, cudaGetErrorString(e));
+      return LMATCH_ECUDA;
+    }
+    cudaGetLastError();
+  }
+  return p2p_set_peer(g, peer, pg->win, pg->bits);
+}
+
+int lmatch_p2p_export(const lmatch_graph* g, void* handles) {
+  if (!g || !g->p2p || !handles) { set_err("lmatch_p2p_enable first / NULL"); return LMATCH_ESTATE; }
+  CK(cudaSetDevice(g->device));
+  cudaIpcMemHandle_t h[2];
+  CK(cudaIpcGetMemHandle(&h[0], g->win));
+  CK(cudaIpcGetMemHandle(&h[1], g->bits));
+  std::memcpy(handles, h, sizeof h);
+  return LMATCH_OK;
+}
+
+int lmatch_p2p_attach(lmatch_graph* g, int32_t peer, const void* handles) {
+  if (!g || !g->p2p || !handles) { set_err("lmatch_p2p_enable first / NULL"); return LMATCH_ESTATE; }
+  if (peer < 0 || peer >= g->P || peer == g->me) { set_err("bad peer %d", peer); return LMATCH_EINVAL; }
+  CK(cudaSetDevice(g->device));
+  cudaIpcMemHandle_t h[2];
+  std::memcpy(h, handles, sizeof h);
+  void* pw = nullptr;
+  void* pb = nullptr;
+  CK(cudaIpcOpenMemHandle(&pw, h[0], cudaIpcMemLazyEnablePeerAccess));
+  g->ipc_opened.push_back(pw);
+  CK(cudaIpcOpenMemHandle(&pb, h[1], cudaIpcMemLazyEnablePeerAccess));
+  g->ipc_opened.push_back(pb);
+  return p2p_set_peer(g, peer, static_cast<uint64_t*>(pw), static_cast<uint32_t*>(pb));
+}
+
+static int p2p_ready(const lmatch_graph* g) {
+  if (!g || !g->p2p) { set_err("not a peer-memory partition handle"); return LMATCH_ESTATE; }
+  for (int p = 0; p < g->P; ++p)
+    if (!g->h_dbits[p]) { set_err("peer %d not attached", p); return LMATCH_ESTATE; }
+  return LMATCH_OK;
+}
+
+int lmatch_p2p_begin(lmatch_graph* g, void* stream) {
+  TRY(p2p_ready(g));
+  g_err[0] = 0;
+  CK(cudaSetDevice(g->device));
+  return part_begin_impl(g, stream ? (cudaStream_t)stream : g->stream, nullptr);
+}
+
+int lmatch_p2p_point(lmatch_graph* g, void* stream) {
+  TRY(p2p_ready(g));
+  if (g->part_round < 1) { set_err("lmatch_p2p_point out of order"); return LMATCH_ESTATE; }
+  CK(cudaSetDevice(g->device));
+  return part_point_impl(g, stream ? (cudaStream_t)stream : g->stream, nullptr);
+}
+
+int lmatch_p2p_match(lmatch_graph* g, void* stream) {
+  TRY(p2p_ready(g));
+  if (g->part_round < 1) { set_err("lmatch_p2p_match out of order"); return LMATCH_ESTATE; }
+  CK(cudaSetDevice(g->device));
+  cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
+  const int P = g->P;
+  unsigned long long* icnt = reinterpret_cast<unsigned long long*>(g->win + (size_t)P * g->win_cap);
+  const int64_t grid = std::max<int64_t>(1, std::min<int64_t>((g->win_cap + 255) / 256, 4 * g->num_sms));
+  // received claims (v owned, u remote): ghost pointers, then the owned mutual checks
+  lm::k_apply_inbox<<<(unsigned)grid, 256, 0, st>>>(g->win, g->win_cap, icnt, P, g->ghost);
+  CKL();
+  if (g->part_round == 1) {
+    if (g->n > 0) {
+      lm::k_match_part_all<<<grid_for(((g->n + 31) / 32) * 32, 256, 65536), 256, 0, st>>>(
+          g->best, g->n, g->v0, g->v0 + g->n, g->ghost, g->bits);
+      CKL();
+    }
+  } else {
+    int64_t nF = 0;
+    for (int b = 0; b < lm::kBins; ++b) nF += (int64_t)g->h_counters[lm::cnt_F(g->part_cur, b)];
+    if (nF > 0) {
+      lm::k_match_part_bins<<<grid_for(nF, 256, 65536), 256, 0, st>>>(
+          g->F[g->part_cur], g->counters + lm::cnt_F(g->part_cur, 0), g->best, g->v0, g->v0 + g->n,
+          g->ghost, g->bits);
+      CKL();
+    }
+  }
+  lm::k_match_inbox<<<(unsigned)grid, 256, 0, st>>>(g->win, g->win_cap, icnt, P, g->best, g->v0,
+                                                     g->bits);
+  CKL();
+  // the inbox is consumed: its counts are zero again before any peer's next claims phase
+  CK(cudaMemsetAsync(icnt, 0, (size_t)P * 8, st));
+  const int64_t nw = (g->n + 31) / 32;
+  if (nw > 0) {
+    lm::k_push_bits<<<grid_for(nw, 256, 4 * g->num_sms), 256, 0, st>>>(g->bits, g->shadow, g->v0 / 32,
+                                                                      nw, g->d_dbits, P, g->me);
+    CKL();
+  }
+  return LMATCH_OK;
+}
+
+int lmatch_p2p_compact(lmatch_graph* g, void* stream, int64_t* nF_local) {
+  TRY(p2p_ready(g));
+  cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
+  int64_t nf = 0;
+  TRY(lmatch_part_compact(g, st, &nf));
+  lm::k_push_count<<<1, 32, 0, st>>>(g->counters + lm::cnt_F(g->part_cur, 0), lm::kBins, g->d_dnf, g->P);
+  CKL();
+  if (nF_local) *nF_local = nf;
+  return LMATCH_OK;
+}
+
+int lmatch_p2p_frontier_total(lmatch_graph* g, void* stream, int64_t* nF_total) {
+  TRY(p2p_ready(g));
+  if (!nF_total) { set_err("NULL nF_total"); return LMATCH_EINVAL; }
+  CK(cudaSetDevice(g->device));
+  cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
+  const int P = g->P;
+  CK(cudaMemcpyAsync(g->h_nf, g->win + (size_t)P * g->win_cap + P, (size_t)P * 8,
+                     cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  int64_t t = 0;
+  for (int p = 0; p < P; ++p) t += (int64_t)g->h_nf[p];
+  *nF_total = t;
+  return LMATCH_OK;
+}
+
+int lmatch_p2p_sync(lmatch_graph* g, void* stream) {
+  if (!g) { set_err("NULL handle"); return LMATCH_ESTATE; }
+  CK(cudaSetDevice(g->device));
+  CK(cudaStreamSynchronize(stream ? (cudaStream_t)stream : g->stream));
+  return LMATCH_OK;
+}
+
+}  // extern "C"

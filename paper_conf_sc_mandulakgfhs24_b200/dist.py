@@ -47,6 +47,16 @@ _sig = {
     "lmatch_part_set_bits": ([_P, _P, _I64, _I64, _P], ctypes.c_int),
     "lmatch_part_info": ([_P, ctypes.POINTER(_I64), ctypes.POINTER(ctypes.c_double)], ctypes.c_int),
     "lmatch_reload": ([_P, _P, _P, _P], ctypes.c_int),
+    "lmatch_p2p_enable": ([_P, ctypes.c_int32], ctypes.c_int),
+    "lmatch_p2p_attach_local": ([_P, ctypes.c_int32, _P], ctypes.c_int),
+    "lmatch_p2p_export": ([_P, _P], ctypes.c_int),
+    "lmatch_p2p_attach": ([_P, ctypes.c_int32, _P], ctypes.c_int),
+    "lmatch_p2p_begin": ([_P, _P], ctypes.c_int),
+    "lmatch_p2p_point": ([_P, _P], ctypes.c_int),
+    "lmatch_p2p_match": ([_P, _P], ctypes.c_int),
+    "lmatch_p2p_compact": ([_P, _P, ctypes.POINTER(_I64)], ctypes.c_int),
+    "lmatch_p2p_frontier_total": ([_P, _P, ctypes.POINTER(_I64)], ctypes.c_int),
+    "lmatch_p2p_sync": ([_P, _P], ctypes.c_int),
 }
 for _name, (_args, _res) in _sig.items():
     _f = getattr(_lib, _name)
@@ -260,6 +270,45 @@ class LibPart:
     def _me(self):
         return self.part
 
+    # ---- peer-memory exchange (include/lmatch.h "Peer-memory exchange")
+    def p2p_enable(self):
+        _check(_lib.lmatch_p2p_enable(self.h, self.part), "lmatch_p2p_enable")
+
+    def p2p_attach_local(self, peer: int, other: "LibPart"):
+        _check(_lib.lmatch_p2p_attach_local(self.h, int(peer), other.h), "lmatch_p2p_attach_local")
+
+    def p2p_export(self) -> bytes:
+        buf = ctypes.create_string_buffer(128)
+        _check(_lib.lmatch_p2p_export(self.h, buf), "lmatch_p2p_export")
+        return buf.raw
+
+    def p2p_attach(self, peer: int, handles: bytes):
+        buf = ctypes.create_string_buffer(bytes(handles), 128)
+        _check(_lib.lmatch_p2p_attach(self.h, int(peer), buf), "lmatch_p2p_attach")
+
+    def p2p_begin(self):
+        _check(_lib.lmatch_p2p_begin(self.h, self._s()), "lmatch_p2p_begin")
+
+    def p2p_point(self):
+        _check(_lib.lmatch_p2p_point(self.h, self._s()), "lmatch_p2p_point")
+
+    def p2p_match(self):
+        _check(_lib.lmatch_p2p_match(self.h, self._s()), "lmatch_p2p_match")
+
+    def p2p_compact(self) -> int:
+        nf = _I64()
+        _check(_lib.lmatch_p2p_compact(self.h, self._s(), ctypes.byref(nf)), "lmatch_p2p_compact")
+        return int(nf.value)
+
+    def p2p_frontier_total(self) -> int:
+        t = _I64()
+        _check(_lib.lmatch_p2p_frontier_total(self.h, self._s(), ctypes.byref(t)),
+               "lmatch_p2p_frontier_total")
+        return int(t.value)
+
+    def p2p_sync(self):
+        _check(_lib.lmatch_p2p_sync(self.h, self._s()), "lmatch_p2p_sync")
+
     def close(self):
         if self.h is not None:
             _lib.lmatch_destroy(self.h)
@@ -309,6 +358,79 @@ def run_parts(parts, transport) -> PartResult:
     return PartResult([f[0] for f in fin], w, c, rounds, sent)
 
 
+def connect_p2p_local(parts):
+    """Peer-memory exchange between parts living in this process (plain device pointers)."""
+    for p in parts:
+        p.p2p_enable()
+    for p in parts:
+        for q in parts:
+            if q is not p:
+                p.p2p_attach_local(q.part, q)
+
+
+def connect_p2p_torch(part, group=None):
+    """Peer-memory exchange between processes: every rank exports its window handles (CUDA IPC),
+    the handles are all-gathered over torch.distributed, and every rank opens its peers'."""
+    import torch.distributed as dist
+    part.p2p_enable()
+    mine = part.p2p_export()
+    allh = [None] * dist.get_world_size(group)
+    dist.all_gather_object(allh, (part.part, mine), group=group)
+    for peer, h in allh:
+        if peer != part.part:
+            part.p2p_attach(peer, h)
+
+
+def barrier_local(parts):
+    """Barrier for parts in one process: drain every part's stream."""
+    def b():
+        for p in parts:
+            p.p2p_sync()
+    return b
+
+
+def barrier_torch(parts, group=None):
+    """Barrier across processes: drain the local streams, then a torch.distributed barrier."""
+    import torch.distributed as dist
+
+    def b():
+        for p in parts:
+            p.p2p_sync()
+        dist.barrier(group=group)
+    return b
+
+
+def run_parts_p2p(parts, barrier, transport) -> PartResult:
+    """The partitioned round with the exchange inside the library's kernels (peer-memory stores:
+    claims into the owners' inboxes, changed bitmap words into every replica, frontier sizes into
+    every part's slot).  `barrier()` separates the phases; `transport` is used only for the final
+    w(M) / |M| sums.  Same result as run_parts."""
+    barrier()                      # every part is done with its previous run
+    for p in parts:
+        p.p2p_begin()
+    rounds = 1
+    while True:
+        barrier()                  # claims are in the owners' inboxes
+        for p in parts:
+            p.p2p_match()
+        barrier()                  # bitmap replicas are complete
+        for p in parts:
+            p.p2p_compact()
+        barrier()                  # frontier sizes are in every slot
+        totals = [p.p2p_frontier_total() for p in parts]
+        if any(t != totals[0] for t in totals):
+            raise LMatchError(f"frontier totals differ between parts: {totals}")
+        if totals[0] == 0:
+            break
+        rounds += 1
+        for p in parts:
+            p.p2p_point()
+    fin = [p.finish() for p in parts]
+    w = transport_sum_float(transport, [f[1] for f in fin])
+    c = transport.allreduce([f[2] for f in fin])[0]
+    return PartResult([f[0] for f in fin], w, c, rounds, 0)
+
+
 def transport_sum_float(transport, xs):
     """fp64 sum over all parts (deterministic: gathered then summed in part order)."""
     if isinstance(transport, LocalTransport):
@@ -322,8 +444,10 @@ def transport_sum_float(transport, xs):
     return float(sum(float(o.item()) for o in out))
 
 
-def match_partitioned_local(offsets, col, w, nparts: int, device=None):
-    """P logical partitions of one graph on one device (LocalTransport).  Returns (mate, result)."""
+def match_partitioned_local(offsets, col, w, nparts: int, device=None, exchange: str = "transport"):
+    """P logical partitions of one graph on one device.  exchange = "transport": LocalTransport
+    moves the claims / bitmap words; "p2p": the library's kernels store them into the other parts'
+    memory (peer-memory exchange).  Returns (mate, result)."""
     offsets = np.asarray(offsets, dtype=np.int64)
     n = offsets.shape[0] - 1
     bounds = edge_balanced_bounds(offsets, nparts)
@@ -332,7 +456,11 @@ def match_partitioned_local(offsets, col, w, nparts: int, device=None):
         v0, v1 = int(bounds[p]), int(bounds[p + 1])
         lo, lc, lw = local_csr(offsets, col, w, v0, v1)
         parts.append(LibPart(lo, lc, lw, v0, n, bounds, p, device=device))
-    res = run_parts(parts, LocalTransport(nparts))
+    if exchange == "p2p":
+        connect_p2p_local(parts)
+        res = run_parts_p2p(parts, barrier_local(parts), LocalTransport(nparts))
+    else:
+        res = run_parts(parts, LocalTransport(nparts))
     mate = np.concatenate([m.cpu().numpy() for m in res.mates]) if n else np.zeros(0, np.int32)
     for p in parts:
         p.close()

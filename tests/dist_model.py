@@ -139,3 +139,102 @@ class NumpyPart:
                 if v > u:
                     w += float(np.uint32(k >> 32).view(np.float32))
         return torch.from_numpy(mate), w, c
+
+
+class NumpyP2PPart(NumpyPart):
+    """The peer-memory exchange protocol of lmatch_p2p_* (include/lmatch.h) on CPU: the exchange
+    window (inbox [P][cap], counts [P], frontier-size slots [P]) and the replicated bitmap live in
+    POSIX shared memory, and peers store into them directly -- the CPU stand-in for the library's
+    stores over NVLink / CUDA IPC.  Same driver (dist.run_parts_p2p), same barriers."""
+
+    def p2p_enable(self):
+        from multiprocessing import shared_memory
+        P = self.P
+        self.cap = int(max(1, np.diff(self.bounds).max()))
+        nwin = P * self.cap + 2 * P
+        self._shm = [shared_memory.SharedMemory(create=True, size=8 * nwin),
+                     shared_memory.SharedMemory(create=True, size=self.N + 1)]
+        self.win = np.ndarray((nwin,), dtype=np.uint64, buffer=self._shm[0].buf)
+        self.win[:] = 0
+        self.bits = np.ndarray((self.N + 1,), dtype=bool, buffer=self._shm[1].buf)
+        self.bits[:] = False
+        self.peer_win = [None] * P
+        self.peer_bits = [None] * P
+        self._opened = []
+        self.peer_win[self.part] = self.win
+        self.peer_bits[self.part] = self.bits
+
+    def p2p_export(self):
+        return (self._shm[0].name, self._shm[1].name)
+
+    def p2p_attach(self, peer, names):
+        from multiprocessing import shared_memory
+        a = shared_memory.SharedMemory(name=names[0])
+        b = shared_memory.SharedMemory(name=names[1])
+        self._opened += [a, b]
+        self.peer_win[peer] = np.ndarray((self.P * self.cap + 2 * self.P,), dtype=np.uint64, buffer=a.buf)
+        self.peer_bits[peer] = np.ndarray((self.N + 1,), dtype=bool, buffer=b.buf)
+
+    def p2p_attach_local(self, peer, other):
+        self.peer_win[peer] = other.win
+        self.peer_bits[peer] = other.bits
+
+    def _push_claims(self):
+        P, cap = self.P, self.cap
+        for d in range(P):
+            out = self.out[d]
+            if not out:
+                continue
+            w = self.peer_win[d]
+            base = int(w[P * cap + self.part])
+            w[self.part * cap + base: self.part * cap + base + len(out)] = np.array(out, dtype=np.uint64)
+            w[P * cap + self.part] = np.uint64(base + len(out))
+
+    def p2p_begin(self):
+        self.best = np.zeros(self.n, dtype=np.uint64)
+        self.ghost = np.full(self.N + 1, NOPTR, dtype=np.int64)
+        self.bits[:] = False
+        self.round = 1
+        for i in range(self.n):
+            self._point(i)
+        self.F = list(range(self.v0, self.v0 + self.n))
+        self._claims_for(self.F)
+        self._push_claims()
+
+    def p2p_point(self):
+        self.point()
+        self._push_claims()
+
+    def p2p_match(self):
+        P, cap = self.P, self.cap
+        segs = [self.win[s * cap: s * cap + int(self.win[P * cap + s])] for s in range(P)]
+        recv = torch.from_numpy(np.concatenate(segs).view(np.int64).copy()) if segs else \
+            torch.zeros(0, dtype=torch.int64)
+        self.apply(recv)
+        self.win[P * cap: P * cap + P] = 0
+        lo, hi = self.bounds[self.part], self.bounds[self.part + 1]
+        for p in range(P):
+            if p != self.part:
+                self.peer_bits[p][lo:hi] = self.bits[lo:hi]
+
+    def p2p_compact(self):
+        nf = self.compact()
+        P, cap = self.P, self.cap
+        for p in range(P):
+            self.peer_win[p][P * cap + P + self.part] = np.uint64(nf)
+        return nf
+
+    def p2p_frontier_total(self):
+        P, cap = self.P, self.cap
+        return int(self.win[P * cap + P: P * cap + 2 * P].sum())
+
+    def p2p_sync(self):
+        pass
+
+    def close(self):
+        for s in getattr(self, "_opened", []):
+            s.close()
+        for s in getattr(self, "_shm", []):
+            s.close()
+            s.unlink()
+        self._opened, self._shm = [], []

@@ -14,7 +14,7 @@ import torch.multiprocessing as mp
 
 import graphgen
 import oracle
-from dist_model import NumpyPart
+from dist_model import NumpyP2PPart, NumpyPart
 
 dist_mod = pytest.importorskip("paper_conf_sc_mandulakgfhs24_b200.dist")
 
@@ -98,6 +98,88 @@ def test_gloo_torchtransport(world, spec):
     g = getattr(graphgen, kind)(*args)
     ref = oracle.greedy(g)
     np.testing.assert_array_equal(mate, ref.mate)
+    for o in out:
+        assert math.isclose(o[2], ref.weight, rel_tol=1e-9)
+        assert o[3] == 2 * ref.cardinality
+        assert o[4] == oracle.ld_frontier(g)[1]
+
+
+# ------------------------------------------------------------ peer-memory exchange (lmatch_p2p_*)
+@pytest.mark.parametrize("P", [1, 2, 3, 5])
+def test_p2p_local_numpy_model(P):
+    """run_parts_p2p (the peer-memory protocol: claims stored into the owners' inboxes, changed
+    bitmap words pushed into every replica, frontier sizes into every slot) with parts in one
+    process: the oracle's unique matching and its round count for every P."""
+    for g in (graphgen.rmat(9, 8, seed=P), graphgen.mesh(20, keep=0.7, seed=P, weights="ones"),
+              graphgen.mesh(12, seed=P, weights="gradient")):
+        b = dist_mod.edge_balanced_bounds(g.offsets, P)
+        parts = []
+        for p in range(P):
+            lo, lc, lw = dist_mod.local_csr(g.offsets, g.col, g.w, int(b[p]), int(b[p + 1]))
+            parts.append(NumpyP2PPart(lo, lc, lw, int(b[p]), g.n, b, p))
+        try:
+            for p in parts:
+                p.p2p_enable()
+            for p in parts:
+                for q in parts:
+                    if q is not p:
+                        p.p2p_attach_local(q.part, q)
+            res = dist_mod.run_parts_p2p(parts, dist_mod.barrier_local(parts),
+                                         dist_mod.LocalTransport(P))
+        finally:
+            for p in parts:
+                p.close()
+        ref = oracle.greedy(g)
+        np.testing.assert_array_equal(np.concatenate([m.numpy() for m in res.mates]), ref.mate)
+        assert res.rounds == oracle.ld_frontier(g)[1]
+        assert math.isclose(res.weight, ref.weight, rel_tol=1e-9)
+
+
+def _p2p_worker(rank, world, port, spec, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    part = None
+    try:
+        kind, args = spec
+        g = getattr(graphgen, kind)(*args)
+        b = dist_mod.edge_balanced_bounds(g.offsets, world)
+        lo, lc, lw = dist_mod.local_csr(g.offsets, g.col, g.w, int(b[rank]), int(b[rank + 1]))
+        part = NumpyP2PPart(lo, lc, lw, int(b[rank]), g.n, b, rank)
+        part.p2p_enable()
+        allh = [None] * world
+        dist.all_gather_object(allh, (rank, part.p2p_export()))
+        for peer, h in allh:
+            if peer != rank:
+                part.p2p_attach(peer, h)
+        res = dist_mod.run_parts_p2p([part], dist_mod.barrier_torch([part]),
+                                     dist_mod.TorchTransport())
+        q.put((rank, res.mates[0].numpy(), res.weight, res.matched, res.rounds))
+        dist.barrier()   # nobody unlinks its window while a peer may still read it
+    finally:
+        if part is not None:
+            part.close()
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,spec", [(2, ("rmat", (10, 8, 2))), (3, ("er", (700, 6.0, 3)))])
+def test_gloo_p2p(world, spec):
+    """The peer-memory driver across processes (shared-memory windows, gloo barriers)."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_p2p_worker, args=(r, world, port, spec, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    out = [q.get(timeout=180) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    out.sort(key=lambda x: x[0])
+    kind, args = spec
+    g = getattr(graphgen, kind)(*args)
+    ref = oracle.greedy(g)
+    np.testing.assert_array_equal(np.concatenate([o[1] for o in out]), ref.mate)
     for o in out:
         assert math.isclose(o[2], ref.weight, rel_tol=1e-9)
         assert o[3] == 2 * ref.cardinality

@@ -305,6 +305,21 @@ def test_out_of_core_host_cache(lm, maker, frac, chunk):
         assert st["cache_rows"] > 0
 
 
+@pytest.mark.parametrize("B", [2, 3, 7])
+@pytest.mark.parametrize("cache", [True, False])
+def test_paper_style_batches(lm, B, cache):
+    """NEXT-2 batch knob (Alg. 2 L3-5): the whole adjacency streamed as B batches
+    through the 2-slot ring (nothing resident); bit-exact for every B, with and without the
+    host-row cache."""
+    for g in (graphgen.rmat(15, 16, seed=8), _hub_graph(5)):
+        mate, st = check_parity(lm, g, batches=B, host_cache=cache)
+        assert st["resident_entries"] == 0
+        assert st["bytes_streamed"] == 8 * g.m
+        C = max(512, (g.m // B + 511) // 512 * 512)  # batch size, rounded to the sweep tile
+        nb = -(-g.m // C)
+        assert st["sweep_launches"] == nb, (st["sweep_launches"], nb)
+
+
 def test_out_of_core_cache_repeat_and_reload(lm):
     """The cache is refilled by every run (and after a reload with other weights)."""
     g = graphgen.rmat(14, 16, seed=21)
