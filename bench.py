@@ -61,6 +61,10 @@ def parse():
                         "adjacency from pinned host memory as B batches in round 1")
     p.add_argument("--no-host-cache", action="store_true",
                    help="out-of-core: disable the top-8 host-row key cache (lmatch_opts.host_cache = -1)")
+    p.add_argument("--exchange", default="p2p", choices=["p2p", "nccl"],
+                   help="partitioned path: p2p = the library's kernels store claims / bitmap words / "
+                        "frontier sizes into the peers' memory (CUDA IPC over NVLink; lmatch_p2p_*), "
+                        "nccl = torch.distributed all-to-all + allgather + allreduce (TorchTransport)")
     p.add_argument("--partitioned", action="store_true",
                    help="use the 1-D partitioned path even at N=1 (it is always used for N>1)")
     return p.parse_args()
@@ -284,13 +288,20 @@ def run_partitioned(a, rank, world, local):
     dg = None
     torch.cuda.empty_cache()
     gen_s = time.time() - t0
-    part = D.LibPart(lo, lc, lw, v0, n, bounds, rank, device=dev, stream=stream, timing=True)
+    part = D.LibPart(lo, lc, lw, v0, n, bounds, rank, device=dev, timing=True)
+    stream = part.stream  # the stream every library kernel of this part is launched on
     del lo, lc, lw
     torch.cuda.empty_cache()
     tr = D.TorchTransport()
+    if a.exchange == "p2p":
+        D.connect_p2p_torch(part)
+        barrier = D.barrier_torch([part])
+        run = lambda: D.run_parts_p2p([part], barrier, tr)  # noqa: E731
+    else:
+        run = lambda: D.run_parts([part], tr)  # noqa: E731
 
     for _ in range(a.warmup):
-        D.run_parts([part], tr)
+        run()
     torch.cuda.synchronize(dev)
     dist.barrier()
     ev0 = torch.cuda.Event(enable_timing=True)
@@ -298,12 +309,14 @@ def run_partitioned(a, rank, world, local):
     sweep_ms = []
     with ClockSampler(local) as clk:
         torch.cuda.synchronize(dev)
+        l0 = D.kernel_launch_count()
         ev0.record(stream)
         for _ in range(a.steps):
-            res = D.run_parts([part], tr)
+            res = run()
             sweep_ms.append(part.info()[1])
         ev1.record(stream)
         torch.cuda.synchronize(dev)
+        launches = D.kernel_launch_count() - l0
     ms = ev0.elapsed_time(ev1)
     t = torch.tensor([ms], dtype=torch.float64, device=dev)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -322,7 +335,7 @@ def run_partitioned(a, rank, world, local):
         t1 = time.perf_counter()
         for _ in range(a.e2e_steps):
             part.reload(*host)
-            r = D.run_parts([part], tr)
+            r = run()
             mate_h[: v1 - v0].copy_(r.mates[0])
         el = time.perf_counter() - t1
         te = torch.tensor([el], dtype=torch.float64, device=dev)
@@ -360,12 +373,16 @@ def run_partitioned(a, rank, world, local):
                 "warmup": a.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
                 "scaling": "strong", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
                 "config": workload_config(a, scale, n, m) | {
-                    "parallelism": f"1-D vertex partition over {world} GPU(s): claims all-to-all + "
-                                   "bitmap allgather per round (NCCL)",
+                    "parallelism": f"1-D vertex partition over {world} GPU(s): " + (
+                        "claims / changed bitmap words / frontier sizes stored into the peers' memory "
+                        "by the library's kernels (CUDA IPC, lmatch_p2p_*), host barriers"
+                        if a.exchange == "p2p" else
+                        "claims all-to-all + bitmap allgather + frontier allreduce per round (NCCL)"),
+                    "exchange": a.exchange,
                     "l2": f"inputs larger than L2 (adjacency {8 * m / 1e9:.1f} GB total); no flush",
                     "gen_s": round(gen_s, 1), "part_bounds": [int(x) for x in bounds]},
                 "roofline": roofline, "cpu_baseline": None, "e2e": e2e,
-                "gpu_launches": None, "clocks": clk.summary(), "rounds": res.rounds,
+                "gpu_launches": int(launches), "clocks": clk.summary(), "rounds": res.rounds,
                 "cardinality": res.matched // 2, "matched_weight": res.weight,
                 "claims_per_step_rank0": res.exchanged_claims}
         print(json.dumps(line), flush=True)

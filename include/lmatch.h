@@ -42,7 +42,7 @@
 extern "C" {
 #endif
 
-#define LMATCH_ABI_VERSION 2
+#define LMATCH_ABI_VERSION 3
 
 #if defined(__GNUC__)
 #define LMATCH_API __attribute__((visibility("default")))
@@ -112,7 +112,8 @@ typedef struct lmatch_opts {
                                  NEXT-2): 0 or 1 = default (resident, or hbm_budget_bytes decides);
                                  B > 1 = nothing resident: the adjacency lives in pinned host
                                  memory as B entry-balanced batches (tile-rounded; a row spanning
-                                 two batches is merged with the u64 max) streamed through the 2-slot device ring in round 1 (2 streams,
+                                 two batches is merged with the u64 max) streamed through
+                                 the 2-slot device ring in round 1 (2 streams,
                                  double buffering).  Overrides hbm_budget_bytes and
                                  stream_chunk */
   int32_t reserved[8];
@@ -144,6 +145,9 @@ typedef struct lmatch_stats {
 
 /* Library / ABI identification.  Returns LMATCH_ABI_VERSION. */
 LMATCH_API int lmatch_abi_version(void);
+/* Kernels this library has launched in this process so far (all handles; a captured CUDA graph
+ * counts its launches once, at capture).  Callers take differences around a region. */
+LMATCH_API int64_t lmatch_kernel_launch_count(void);
 
 /* Build a handle from HOST CSR arrays (copied to the device in chunks, packed into 64-bit
  * (weight-bits << 32 | neighbour) keys, validated, and indexed for the round-1 sweep).

@@ -12,6 +12,7 @@
 #include <cudaTypedefs.h>
 
 #include <algorithm>
+#include <atomic>
 #include <climits>
 #include <cstdarg>
 #include <cstdio>
@@ -43,7 +44,14 @@ void set_err(const char* fmt, ...) {
       return (e_ == cudaErrorMemoryAllocation) ? LMATCH_ENOMEM : LMATCH_ECUDA;          \
     }                                                                                   \
   } while (0)
-#define CKL() CK(cudaGetLastError())
+// every kernel launch of the library is followed by CKL(): it also counts the launch (process-wide,
+// lmatch_kernel_launch_count)
+static std::atomic<long long> g_launch_count{0};
+#define CKL()                                            \
+  do {                                                   \
+    g_launch_count.fetch_add(1, std::memory_order_relaxed); \
+    CK(cudaGetLastError());                              \
+  } while (0)
 #define TRY(x)                 \
   do {                         \
     int s_ = (x);              \
@@ -816,6 +824,8 @@ extern "C" {
 
 int lmatch_abi_version(void) { return LMATCH_ABI_VERSION; }
 
+int64_t lmatch_kernel_launch_count(void) { return (int64_t)g_launch_count.load(); }
+
 const char* lmatch_strerror(int status) {
   switch (status) {
     case LMATCH_OK: return "ok";
@@ -1089,6 +1099,7 @@ int launch_persistent_t(lmatch_graph* g, cudaStream_t st, int64_t* launches) {
   cfg.numAttrs = 1;
   CK(cudaLaunchKernelEx(&cfg, PERSISTENT_KERNEL(PRUNE), ra, (const int64_t*)g->offs, av, g->bits,
                         g->best, g->n, g->v0));
+  g_launch_count.fetch_add(1, std::memory_order_relaxed);
   ++*launches;
   return LMATCH_OK;
 }

@@ -57,6 +57,7 @@ _sig = {
     "lmatch_p2p_compact": ([_P, _P, ctypes.POINTER(_I64)], ctypes.c_int),
     "lmatch_p2p_frontier_total": ([_P, _P, ctypes.POINTER(_I64)], ctypes.c_int),
     "lmatch_p2p_sync": ([_P, _P], ctypes.c_int),
+    "lmatch_kernel_launch_count": ([], _I64),
 }
 for _name, (_args, _res) in _sig.items():
     _f = getattr(_lib, _name)
@@ -179,10 +180,17 @@ class LibPart:
         self.part = int(part)
         self.n_local = int(len(offsets_local) - 1)
         self.n_global = int(n_global)
+        # every call of this part (library kernels, torch copies of claims / bitmap words) is
+        # ordered on ONE non-default stream (a NULL stream would make the library use its own
+        # handle stream, unordered with torch's legacy default stream); tensors crossing to the
+        # caller's stream are synchronised (producers) or waited for (consumers)
+        if stream is None or stream.cuda_stream == 0:
+            stream = torch.cuda.Stream(self.dev)
         self.stream = stream
         h = _P()
         opts = make_opts(validate_level=validate_level, timing=timing)
         if hasattr(offsets_local, "is_cuda") and offsets_local.is_cuda:  # device CSR (torch)
+            torch.cuda.current_stream(self.dev).synchronize()  # the arrays' producer
             self.m_local = int(col_local.numel())
             with torch.cuda.device(self.dev):
                 _check(_lib.lmatch_create_part_device(
@@ -204,7 +212,14 @@ class LibPart:
         self.words = part_words(self.bounds)
 
     def _s(self):
-        return None if self.stream is None else self.stream.cuda_stream
+        return self.stream.cuda_stream
+
+    def _consume(self, t):
+        """Order this part's stream after the caller's current stream, which produced `t`, and
+        keep t's memory from being reused before this stream is done with it."""
+        torch = self.torch
+        self.stream.wait_stream(torch.cuda.current_stream(self.dev))
+        t.record_stream(self.stream)
 
     def begin(self):
         _check(_lib.lmatch_part_begin(self.h, self._s(), self.counts.ctypes.data), "lmatch_part_begin")
@@ -217,22 +232,29 @@ class LibPart:
     def claims(self, counts):
         torch = self.torch
         out = []
-        for p in range(self.P):
-            t = torch.empty(int(counts[p]), dtype=torch.int64, device=self.dev)
-            if counts[p]:
-                _check(_lib.lmatch_part_get_claims(self.h, p, t.data_ptr(), self._s()),
-                       "lmatch_part_get_claims")
-            out.append(t)
+        with torch.cuda.stream(self.stream):
+            for p in range(self.P):
+                t = torch.empty(int(counts[p]), dtype=torch.int64, device=self.dev)
+                if counts[p]:
+                    _check(_lib.lmatch_part_get_claims(self.h, p, t.data_ptr(), self._s()),
+                           "lmatch_part_get_claims")
+                out.append(t)
+        self.stream.synchronize()
         return out
 
     def apply(self, recv):
+        if recv.numel():
+            self._consume(recv)
         _check(_lib.lmatch_part_apply(self.h, recv.data_ptr() if recv.numel() else None,
                                       recv.numel(), self._s()), "lmatch_part_apply")
 
     def own_bits(self):
-        t = self.torch.empty(self.words[self._me()][1], dtype=self.torch.int32, device=self.dev)
-        if t.numel():
-            _check(_lib.lmatch_part_get_bits(self.h, t.data_ptr(), self._s()), "lmatch_part_get_bits")
+        with self.torch.cuda.stream(self.stream):
+            t = self.torch.empty(self.words[self._me()][1], dtype=self.torch.int32, device=self.dev)
+            if t.numel():
+                _check(_lib.lmatch_part_get_bits(self.h, t.data_ptr(), self._s()),
+                       "lmatch_part_get_bits")
+        self.stream.synchronize()
         return t
 
     def set_bits(self, all_words):
@@ -240,6 +262,7 @@ class LibPart:
             if p == self._me() or t.numel() == 0:
                 continue
             src = t.to(self.dev).contiguous()
+            self._consume(src)
             _check(_lib.lmatch_part_set_bits(self.h, src.data_ptr(), self.words[p][0], src.numel(),
                                              self._s()), "lmatch_part_set_bits")
 
@@ -261,7 +284,8 @@ class LibPart:
 
     def finish(self):
         torch = self.torch
-        mate = torch.empty(max(self.n_local, 1), dtype=torch.int32, device=self.dev)
+        with torch.cuda.stream(self.stream):
+            mate = torch.empty(max(self.n_local, 1), dtype=torch.int32, device=self.dev)
         w, c = ctypes.c_double(), _I64()
         _check(_lib.lmatch_part_finish(self.h, mate.data_ptr(), self._s(), ctypes.byref(w),
                                        ctypes.byref(c)), "lmatch_part_finish")
@@ -356,6 +380,11 @@ def run_parts(parts, transport) -> PartResult:
     w = transport_sum_float(transport, [f[1] for f in fin])
     c = transport.allreduce([f[2] for f in fin])[0]
     return PartResult([f[0] for f in fin], w, c, rounds, sent)
+
+
+def kernel_launch_count() -> int:
+    """Kernels liblmatch.so has launched in this process so far (lmatch_kernel_launch_count)."""
+    return int(_lib.lmatch_kernel_launch_count())
 
 
 def connect_p2p_local(parts):

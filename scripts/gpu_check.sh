@@ -1,8 +1,4 @@
-# one gpurun call: GPU tests + quick benches (outputs under gpurun_out/)
 mkdir -p gpurun_out
-timeout 600 python -m pytest tests/test_gpu_p2p.py -x -q 2>&1 | tail -15 > gpurun_out/t_p2p.log
-timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -15 > gpurun_out/t_gpu3.log
-for c in "--batches 2" "--batches 10" "--hbm-budget-gb 6"; do
-  python bench.py --no-cpu --no-e2e --steps 3 $c >> gpurun_out/b_fill.jsonl 2>> gpurun_out/b_fill.err
-done
-tail -3 gpurun_out/t_p2p.log gpurun_out/t_gpu3.log
+timeout 900 python -m pytest tests/test_gpu_p2p.py tests/test_gpu_parity.py -k "partition or p2p" -x -q 2>&1 | tail -5 > gpurun_out/t_p2p2.log
+timeout 900 python scripts/bench_parts_local.py --scale 24 --parts 1 4 8 > gpurun_out/parts_local_s24b.jsonl 2> gpurun_out/parts_local.err
+cat gpurun_out/t_p2p2.log

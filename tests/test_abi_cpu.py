@@ -93,7 +93,7 @@ def test_host_side_argument_errors(pkg):
     assert lib.lmatch_info(None, None, None, None, None) == pkg.LMATCH_ESTATE
     lib.lmatch_destroy(None)  # NULL-safe
     assert pkg.lmatch_strerror(pkg.LMATCH_EINVAL).startswith("invalid")
-    assert pkg.lmatch_abi_version() == 2
+    assert pkg.lmatch_abi_version() == 3
     assert "n" in pkg.lmatch_last_error() or pkg.lmatch_last_error() == ""
 
 

@@ -55,6 +55,49 @@ def test_p2p_local_invariance(D, P, maker):
     _check(g, mate, res)
 
 
+@pytest.mark.parametrize("exchange", ["transport", "p2p"])
+def test_partitioned_larger_graph(D, exchange):
+    """R-MAT scale 20 over 4 and 7 parts (rounds with millions of claims): both exchanges stay
+    bit-exact (the in-process transport once raced against the parts' own streams here)."""
+    g = graphgen.rmat(20, 16, seed=3)
+    for P in (4, 7):
+        mate, res = D.match_partitioned_local(g.offsets, g.col, g.w, P, exchange=exchange)
+        _check(g, mate, res)
+
+
+@pytest.mark.parametrize("exchange", ["transport", "p2p"])
+def test_partitioned_scale24_repeat_vs_single(D, exchange):
+    """R-MAT scale 24 (configs[1]) over 2 parts, three runs on the same parts: every run equals
+    the single-GPU result (itself certified exact at this size by test_full_size_rmat24_certificate).
+    At this size an unordered stream once made the in-process transport nondeterministic."""
+    import torch
+    import graphgen.gpu as gg
+    import paper_conf_sc_mandulakgfhs24_b200 as lm
+    g = gg.rmat(24, 16, seed=1, device=torch.device("cuda"))
+    off, col, w = g.offsets.cpu().numpy(), g.col.cpu().numpy(), g.w.cpu().numpy()
+    del g
+    with lm.Matcher(off, col, w) as M:
+        ref, st = M.run()
+    b = D.edge_balanced_bounds(off, 2)
+    parts = []
+    for p in range(2):
+        lo, lc, lw = D.local_csr(off, col, w, int(b[p]), int(b[p + 1]))
+        parts.append(D.LibPart(lo, lc, lw, int(b[p]), len(off) - 1, b, p))
+    if exchange == "p2p":
+        D.connect_p2p_local(parts)
+        run = lambda: D.run_parts_p2p(parts, D.barrier_local(parts), D.LocalTransport(2))  # noqa: E731
+    else:
+        run = lambda: D.run_parts(parts, D.LocalTransport(2))  # noqa: E731
+    for _ in range(3):
+        res = run()
+        mate = np.concatenate([m.cpu().numpy() for m in res.mates])
+        np.testing.assert_array_equal(mate, ref)
+        assert res.rounds == st["rounds"]
+        assert math.isclose(res.weight, st["weight"], rel_tol=WTOL)
+    for p in parts:
+        p.close()
+
+
 def test_p2p_hub_rows_and_repeat(D):
     """Hub rows cut across parts; two runs on the same connected handles give the same result
     (inbox counts are left at zero by every round, the bitmap shadow is reset per run)."""
