@@ -61,6 +61,10 @@ def parse():
                         "adjacency from pinned host memory as B batches in round 1")
     p.add_argument("--no-host-cache", action="store_true",
                    help="out-of-core: disable the top-8 host-row key cache (lmatch_opts.host_cache = -1)")
+    p.add_argument("--algorithm", default="ld", choices=["ld", "suitor", "hybrid"],
+                   help="ld = the pointer-based locally dominant iteration (the paper's method); "
+                        "suitor = Suitor proposals with atomicMax (NEXT-4, same unique result); "
+                        "hybrid = ld, with a Suitor tail after 32 pointing phases")
     p.add_argument("--exchange", default="p2p", choices=["p2p", "nccl"],
                    help="partitioned path: p2p = the library's kernels store claims / bitmap words / "
                         "frontier sizes into the peers' memory (CUDA IPC over NVLink; lmatch_p2p_*), "
@@ -130,6 +134,8 @@ def workload_config(a, scale, n, m):
         cfg["edgefactor"] = a.edgefactor
     if getattr(a, "prune", False):
         cfg["prune"] = True
+    if getattr(a, "algorithm", "ld") != "ld":
+        cfg["algorithm"] = a.algorithm
     return cfg
 
 
@@ -368,6 +374,11 @@ def run_partitioned(a, rank, world, local):
                 "kernel": "k_sweep over the slowest rank's owned rows",
                 "launch_ms": float(worst[0]), "share_of_step": float(worst[0]) / ms_per_step,
                 "peak_source": peak_src}
+    ms_all = [float(x[0]) for x in allsw]
+    ent_all = [float(x[1]) for x in allsw]
+    imbalance = {"entries_max_over_mean": max(ent_all) / max(np.mean(ent_all), 1.0),
+                 "sweep_ms_max_over_mean": max(ms_all) / max(np.mean(ms_all), 1e-9),
+                 "entries_per_rank": [int(x) for x in ent_all]}
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps,
                 "warmup": a.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
@@ -384,7 +395,7 @@ def run_partitioned(a, rank, world, local):
                 "roofline": roofline, "cpu_baseline": None, "e2e": e2e,
                 "gpu_launches": int(launches), "clocks": clk.summary(), "rounds": res.rounds,
                 "cardinality": res.matched // 2, "matched_weight": res.weight,
-                "claims_per_step_rank0": res.exchanged_claims}
+                "claims_per_step_rank0": res.exchanged_claims, "imbalance": imbalance}
         print(json.dumps(line), flush=True)
     part.close()
     dist.destroy_process_group()
@@ -442,7 +453,7 @@ def main():
     opts = lm.make_opts(validate_level=1, timing=1,
                         hbm_budget_bytes=int(a.hbm_budget_gb * 1e9), stream_chunk=a.stream_chunk,
                         prune=a.prune, host_cache=not a.no_host_cache,
-                        batches=a.batches)
+                        batches=a.batches, algorithm=a.algorithm)
     pinned_host = d_off is None
     if pinned_host:
         h = lm.lmatch_create_ex(g.offsets, g.col, g.w, n, m, opts)
@@ -539,12 +550,29 @@ def main():
                "includes": "lmatch_reload (H2D + pack + validate + index) + lmatch_run (+ mate D2H)"}
 
     ooc = None
+    pcie_peak = None
+    if a.hbm_budget_gb > 0 or a.batches > 1:
+        # the bound of the streamed round: pinned H2D copy rate of this box (1 GiB, best of 3)
+        src = torch.empty(1 << 30, dtype=torch.uint8, pin_memory=True)
+        dst = torch.empty(1 << 30, dtype=torch.uint8, device=dev)
+        best = 0.0
+        for _ in range(3):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            dst.copy_(src, non_blocking=True)
+            e1.record(stream)
+            e1.synchronize()
+            best = max(best, (1 << 30) / (e0.elapsed_time(e1) / 1e3) / 1e9)
+        del src, dst
+        pcie_peak = best
     if a.hbm_budget_gb > 0 or a.batches > 1:
         ooc = {"batches": a.batches,"hbm_budget_bytes": int(a.hbm_budget_gb * 1e9),
                "resident_entries": int(last["resident_entries"]),
                "resident_frac": last["resident_entries"] / max(m, 1),
                "bytes_streamed_per_step": int(last["bytes_streamed"]),
                "stream_gbs_in_sweep": last["bytes_streamed"] / max(sweep_avg_ms, 1e-9) / 1e6,
+               "pcie_h2d_peak_gbs": pcie_peak,
+               "pcie_frac_in_sweep": (last["bytes_streamed"] / max(sweep_avg_ms, 1e-9) / 1e6) / pcie_peak,
                "host_cache": not a.no_host_cache,
                "cache_bytes": int(last["cache_bytes"]),
                "cache_rows_per_step": int(last["cache_rows"]),

@@ -116,7 +116,19 @@ typedef struct lmatch_opts {
                                  the 2-slot device ring in round 1 (2 streams,
                                  double buffering).  Overrides hbm_budget_bytes and
                                  stream_chunk */
-  int32_t reserved[8];
+  int32_t algorithm;          /* 0 = default: the pointer-based LD iteration (Alg. 1-3).  1 = Suitor
+                                 (the paper's SR comparison algorithm,
+                                 P:84-86): proposals accepted by a u64 atomicMax on the receiver's
+                                 best offer, displaced proposers try again; no synchronous
+                                 rounds of mutual checks.  Same unique result under R1 (the
+                                 certificate and the oracle decide).  2 = hybrid: the LD
+                                 iteration, and if a frontier is left after 32 pointing phases
+                                 (many-round graphs, e.g. weight gradients along paths), Suitor on
+                                 the graph without the vertices matched so far completes the same
+                                 matching (lmatch_stats.tail_passes).  1 and 2: resident
+                                 single-graph handles only (1: EINVAL with out-of-core /
+                                 partition handles; 2 behaves as 0 there) */
+  int32_t reserved[7];
 } lmatch_opts;
 
 /* Filled by lmatch_run / lmatch_run_device when non-NULL. */
@@ -140,7 +152,9 @@ typedef struct lmatch_stats {
                                 cache decided in rounds >= 2 (no host read) */
   int64_t host_entries_read; /* out-of-core: host-resident entries read zero-copy in rounds >= 2 */
   int64_t cache_bytes;       /* out-of-core: device bytes of the host-row cache (0 = none) */
-  int64_t reserved[3];
+  int64_t tail_passes;       /* algorithm 2: Suitor passes that completed the run after the LD
+                                iteration stopped at 32 pointing phases (0 = not needed) */
+  int64_t reserved[2];
 } lmatch_stats;
 
 /* Library / ABI identification.  Returns LMATCH_ABI_VERSION. */

@@ -45,7 +45,7 @@ class Opts(ctypes.Structure):
         ("hbm_budget_bytes", ctypes.c_int64), ("stream_chunk", ctypes.c_int64),
         ("round_loop", ctypes.c_int32), ("prune", ctypes.c_int32),
         ("host_cache", ctypes.c_int32), ("batches", ctypes.c_int32),
-        ("reserved", ctypes.c_int32 * 8),
+        ("algorithm", ctypes.c_int32), ("reserved", ctypes.c_int32 * 7),
     ]
 
 
@@ -61,7 +61,7 @@ class Stats(ctypes.Structure):
         ("kernel_launches", ctypes.c_int64), ("bytes_streamed", ctypes.c_int64),
         ("resident_entries", ctypes.c_int64), ("cache_rows", ctypes.c_int64),
         ("host_entries_read", ctypes.c_int64), ("cache_bytes", ctypes.c_int64),
-        ("reserved", ctypes.c_int64 * 3),
+        ("tail_passes", ctypes.c_int64), ("reserved", ctypes.c_int64 * 2),
     ]
 
     def as_dict(self) -> dict:
@@ -244,7 +244,7 @@ class Matcher:
                  validate_level: int = 1, timing: bool = False, upload_chunk: int = 0,
                  max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
                  round_loop: int = 0, prune: bool = False, host_cache: bool = True,
-                 batches: int = 0):
+                 batches: int = 0, algorithm: str = "ld"):
         self.h = None
         if handle is not None:
             self.h = handle
@@ -254,14 +254,16 @@ class Matcher:
             self.h = lmatch_create_ex(offsets, col, w,
                                       opts=make_opts(validate_level, timing, upload_chunk,
                                                      max_rounds, hbm_budget_bytes, stream_chunk,
-                                                     round_loop, prune, host_cache, batches))
+                                                     round_loop, prune, host_cache, batches,
+                                                     algorithm))
         self.info = lmatch_info(self.h)
 
     @classmethod
     def from_device(cls, d_offsets, d_col, d_w, n, m, stream=None, **kw):
         h = lmatch_create_device(d_offsets, d_col, d_w, n, m,
                                  make_opts(kw.get("validate_level", 1), kw.get("timing", False),
-                                           0, kw.get("max_rounds", 0)), stream)
+                                           0, kw.get("max_rounds", 0),
+                                           algorithm=kw.get("algorithm", "ld")), stream)
         return cls(handle=h)
 
     def run(self, mate_out=None):
@@ -298,7 +300,7 @@ class Matcher:
 def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int = 0,
               max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
               round_loop: int = 0, prune: bool = False, host_cache: bool = True,
-              batches: int = 0) -> Opts:
+              batches: int = 0, algorithm: str = "ld") -> Opts:
     """round_loop (include/lmatch.h): 0 = hybrid (work-sized launches, then one persistent kernel
     for the tail; default), 1 = host-driven launches only, 2 = persistent kernel after round 1,
     3 = CUDA graph {round 1, persistent kernel}."""
@@ -307,6 +309,7 @@ def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int =
     o.prune = int(bool(prune))
     o.host_cache = 0 if host_cache else -1
     o.batches = int(batches)
+    o.algorithm = {"ld": 0, "suitor": 1, "hybrid": 2}[algorithm]
     o.hbm_budget_bytes = int(hbm_budget_bytes)
     o.stream_chunk = int(stream_chunk)
     o.validate_level = int(validate_level)

@@ -372,6 +372,9 @@ __global__ void k_reset(uint32_t* bits, int64_t nwords, uint64_t* best,
 //     => identical to one sequential scan; such rows are zeroed by k_reset).
 // Self-loop keys were zeroed at ingest (k_zap_self_loops).  No bitmap test in round 1.
 // =============================================================================================
+#ifndef LM_SWEEP_MID
+#define LM_SWEEP_MID 0  // 1 = rows of 8..31 in-tile entries by 8-lane groups (build knob)
+#endif
 __device__ __forceinline__ uint64_t umax64(uint64_t a, uint64_t b) { return a > b ? a : b; }
 // max(b, key) unless key is the self-loop entry of vertex `self`
 __device__ __forceinline__ uint64_t umax_skip(uint64_t b, uint64_t key, uint32_t self) {
@@ -523,7 +526,40 @@ __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
         }
         continue;
       }
+#if LM_SWEEP_MID
+      // medium rows (8 <= L < 32): 8-lane groups, four rows per step, so the lane-per-row loop
+      // below only runs as long as the longest row under 8 entries (no long divergent tail)
+      unsigned mm = __ballot_sync(0xffffffffu, L >= 8 && L < 32);
+      while (mm) {
+        const int q = lane >> 3, gl = lane & 7;
+        unsigned m2 = mm;
+        for (int i = 0; i < q && m2; ++i) m2 &= m2 - 1;
+        const int l = m2 ? __ffs(m2) - 1 : 0;
+        const bool has = m2 != 0u;
+        for (int i = 0; i < 4 && mm; ++i) mm &= mm - 1;
+        const int32_t ja = __shfl_sync(0xffffffffu, max(rs, 0), l);
+        const int32_t jl = __shfl_sync(0xffffffffu, min(re, len), l);
+        const int32_t jb = has ? jl : ja;
+        const uint32_t v = __shfl_sync(0xffffffffu, vid, l);
+        const bool ins = __shfl_sync(0xffffffffu, (int)inside, l) != 0;
+        uint64_t b0 = 0, b1 = 0;
+        int j = ja + gl;
+        for (; j + 8 < jb; j += 16) {
+          b0 = umax64(b0, K[j]);
+          b1 = umax64(b1, K[j + 8]);
+        }
+        if (j < jb) b0 = umax64(b0, K[j]);
+        const unsigned gmask = 0xffu << (q * 8);
+        const uint64_t b = group_max_key(umax64(b0, b1), gmask);
+        if (has && gl == 0) {
+          if (ins) A.best[v] = b;
+          else if (b) atomicMax(reinterpret_cast<unsigned long long*>(&A.best[v]), (unsigned long long)b);
+        }
+      }
+      if (L > 0 && L < 8) {
+#else
       if (L > 0 && L < 32) {
+#endif
         uint64_t b0 = 0, b1 = 0, b2 = 0, b3 = 0;  // 4 independent max chains
         int j = max(rs, 0);
         const int je = min(re, len);
@@ -2260,6 +2296,220 @@ __global__ void k_cache_redirect(Bins F, const unsigned long long* __restrict__ 
     if (served) atomicAdd(&cnt[0], served);
     if (left) atomicAdd(&cnt[1], left);
   }
+}
+
+// =============================================================================================
+// NEXT-4: the Suitor algorithm (Manne & Halappanavar; the paper's SR-OMP / SR-GPU
+// comparison algorithm) under the same strict order, which reaches the same unique
+// locally dominant matching without synchronous rounds of mutual checks.
+//   suitor[v] = the best proposal v has received: (bits(w(u,v)) << 32) | u  -- v's order over its
+//               proposers (R1), so "better proposal" is a u64 compare and acceptance an atomicMax.
+//   A vertex u without a standing proposal scans its row for the heaviest neighbour v (its own
+//   order, key = bits(w) << 32 | v) whose current suitor is worse than u's offer, and proposes
+//   with atomicMax.  A displaced suitor, or a proposer that lost the race, proposes again in the
+//   next pass.  When no vertex is left, suitor[] is symmetric: mate[u] = proposer in suitor[u].
+// Pass 1 needs no scan: with every suitor[] empty, u's choice is its row maximum, which the
+// round-1 sweep already computed into best[u].
+// =============================================================================================
+constexpr uint64_t kHi32 = 0xffffffff00000000ull;
+
+// u proposes `key` (its chosen neighbour); returns the vertex that must propose again next pass
+// (the displaced previous suitor, or u itself when a better proposal got there first), or kNoPtr
+__device__ __forceinline__ uint32_t suitor_propose(uint64_t* suitor, uint32_t u, uint64_t key) {
+  const uint32_t v = (uint32_t)key;
+  const uint64_t p = (key & kHi32) | u;
+  const uint64_t old = atomicMax(reinterpret_cast<unsigned long long*>(&suitor[v]),
+                                 (unsigned long long)p);
+  if (old < p) return old ? (uint32_t)old : kNoPtr;
+  return u;
+}
+// warp-aggregated append of the lanes' `again` vertices (all 32 lanes call it)
+__device__ __forceinline__ void suitor_push(uint32_t again, uint32_t* next, unsigned long long* ncnt) {
+  const unsigned b = __ballot_sync(0xffffffffu, again != kNoPtr);
+  if (!b) return;
+  const int lane = threadIdx.x & 31, leader = __ffs(b) - 1;
+  unsigned long long base = 0;
+  if (lane == leader) base = atomicAdd(ncnt, (unsigned long long)__popc(b));
+  base = __shfl_sync(0xffffffffu, base, leader);
+  if (again != kNoPtr) next[base + __popc(b & lanemask_lt())] = again;
+}
+
+// pass 1: every vertex proposes to its row maximum (best[] from the sweep)
+__global__ void k_suitor_first(const uint64_t* __restrict__ best, int64_t n, uint64_t* suitor,
+                               uint32_t* next, unsigned long long* ncnt) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t n32 = (n + 31) & ~31ll;
+  for (int64_t u = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; u < n32; u += stride) {
+    const uint64_t k = u < n ? best[u] : 0ull;
+    suitor_push(k ? suitor_propose(suitor, (uint32_t)u, k) : kNoPtr, next, ncnt);
+  }
+}
+
+// the best neighbour of u over entries [a, b) whose suitor would accept u
+__device__ __forceinline__ uint64_t suitor_best(const uint64_t* __restrict__ adj, int64_t a,
+                                                int64_t b, int64_t step, uint32_t u,
+                                                const uint64_t* suitor) {
+  uint64_t best = 0;
+  for (int64_t j = a; j < b; j += step) {
+    const uint64_t k = __ldg(adj + j);
+    if (k <= best) continue;
+    const uint64_t p = (k & kHi32) | u;
+    if (p > __ldcg(suitor + (uint32_t)k)) best = k;
+  }
+  return best;
+}
+
+// passes >= 2 over the worklist: a row of <= 32 entries is scanned by its lane, up to
+// kSuitorBig entries by the warp, longer rows are listed for k_suitor_scan_big
+constexpr int64_t kSuitorBig = 4096;
+__global__ void __launch_bounds__(256) k_suitor_scan(const uint32_t* __restrict__ wl,
+                                                     const unsigned long long* __restrict__ wcnt,
+                                                     const int64_t* __restrict__ offs,
+                                                     const uint64_t* __restrict__ adj,
+                                                     uint64_t* suitor, uint32_t* next,
+                                                     unsigned long long* ncnt, uint32_t* big,
+                                                     unsigned long long* nbig,
+                                                     unsigned long long* scanned) {
+  const int lane = threadIdx.x & 31;
+  const int64_t c = (int64_t)*wcnt;
+  const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  unsigned long long sc = 0;
+  for (int64_t i0 = wid * 32; i0 < c; i0 += nw * 32) {
+    const int64_t i = i0 + lane;
+    uint32_t u = 0;
+    int64_t s = 0, e = 0;
+    if (i < c) {
+      u = wl[i];
+      s = offs[u];
+      e = offs[u + 1];
+    }
+    const int64_t d = e - s;
+    uint32_t again = kNoPtr;
+    if (d > 0 && d <= 32) {
+      sc += (unsigned long long)d;
+      const uint64_t b = suitor_best(adj, s, e, 1, u, suitor);
+      if (b) again = suitor_propose(suitor, u, b);
+    } else if (d > kSuitorBig) {
+      big[atomicAdd(nbig, 1ull)] = u;
+    }
+    suitor_push(again, next, ncnt);
+    unsigned mid = __ballot_sync(0xffffffffu, d > 32 && d <= kSuitorBig);
+    while (mid) {
+      const int l = __ffs(mid) - 1;
+      mid &= mid - 1;
+      const uint32_t ul = __shfl_sync(0xffffffffu, u, l);
+      const int64_t sl = __shfl_sync(0xffffffffu, s, l), el = __shfl_sync(0xffffffffu, e, l);
+      if (lane == 0) sc += (unsigned long long)(el - sl);
+      const uint64_t b = group_max_key(suitor_best(adj, sl + lane, el, 32, ul, suitor), 0xffffffffu);
+      uint32_t ag = kNoPtr;
+      if (lane == 0 && b) ag = suitor_propose(suitor, ul, b);
+      if (ag != kNoPtr) next[atomicAdd(ncnt, 1ull)] = ag;
+    }
+  }
+  for (int o = 16; o; o >>= 1) sc += __shfl_xor_sync(0xffffffffu, sc, o);
+  if (lane == 0 && sc) atomicAdd(scanned, sc);
+}
+
+// the listed long rows: one CTA per row
+__global__ void __launch_bounds__(256) k_suitor_scan_big(const uint32_t* __restrict__ big,
+                                                         const unsigned long long* __restrict__ nbig,
+                                                         const int64_t* __restrict__ offs,
+                                                         const uint64_t* __restrict__ adj,
+                                                         uint64_t* suitor, uint32_t* next,
+                                                         unsigned long long* ncnt,
+                                                         unsigned long long* scanned) {
+  __shared__ uint64_t red[8];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t nb = (int64_t)*nbig;
+  for (int64_t i = blockIdx.x; i < nb; i += gridDim.x) {
+    const uint32_t u = big[i];
+    const int64_t s = offs[u], e = offs[u + 1];
+    uint64_t b = group_max_key(suitor_best(adj, s + threadIdx.x, e, blockDim.x, u, suitor),
+                               0xffffffffu);
+    if (lane == 0) red[warp] = b;
+    __syncthreads();
+    if (warp == 0) {
+      b = group_max_key(lane < 8 ? red[lane] : 0ull, 0xffffffffu);
+      if (lane == 0) {
+        const uint32_t ag = b ? suitor_propose(suitor, u, b) : kNoPtr;
+        if (ag != kNoPtr) next[atomicAdd(ncnt, 1ull)] = ag;
+        atomicAdd(scanned, (unsigned long long)(e - s));
+      }
+    }
+    __syncthreads();
+  }
+}
+
+// mate[] + w(M) from suitor[] (fixed assignment, fixed fp64 order, like k_materialize)
+template <int THREADS>
+__global__ void __launch_bounds__(THREADS)
+    k_suitor_finish(const uint64_t* __restrict__ suitor, int64_t n, int32_t* __restrict__ mate,
+                    double* pw, long long* pc) {
+  double w = 0.0;
+  long long c = 0;
+  const int64_t stride = (int64_t)gridDim.x * THREADS;
+  for (int64_t i = (int64_t)blockIdx.x * THREADS + threadIdx.x; i < n; i += stride) {
+    const uint64_t k = suitor[i];
+    int32_t v = -1;
+    if (k) {
+      v = (int32_t)(uint32_t)k;
+      ++c;
+      if ((int64_t)v > i) w += (double)__uint_as_float((uint32_t)(k >> 32));
+    }
+    mate[i] = v;
+  }
+  block_sum2<THREADS>(w, c, &pw[blockIdx.x], &pc[blockIdx.x]);
+}
+
+// ---- hybrid (algorithm 2): the LD iteration hands a long tail over to Suitor.  The vertices it
+// matched are final (each mutual pair is in the unique matching M*) and the rest of M* is the
+// unique LD matching of the graph without them (an M* edge at an unmatched vertex has an
+// unmatched other end), so Suitor on that residual graph completes the same result.  Matched
+// vertices get the sentinel suitor ~0, which no proposal exceeds.
+__global__ void k_suitor_tail_init(const uint32_t* __restrict__ bits, int64_t n, uint64_t* suitor) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t u = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; u < n; u += stride)
+    suitor[u] = bit_test(bits, (uint32_t)u) ? ~0ull : 0ull;
+}
+// worklist = the live vertices: stable pairs S and the frontier bins of the current set
+__global__ void k_suitor_tail_list(const uint64_t* __restrict__ S, const unsigned long long* cntS,
+                                   Bins F, const unsigned long long* cntF, uint32_t* wl,
+                                   unsigned long long* wcnt) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t ns = (int64_t)*cntS;
+  for (int64_t i = tid; i < ns; i += stride) wl[atomicAdd(wcnt, 1ull)] = (uint32_t)S[i];
+  for (int bb = 0; bb < kBins; ++bb) {
+    const int64_t c = (int64_t)cntF[bb];
+    for (int64_t i = tid; i < c; i += stride) wl[atomicAdd(wcnt, 1ull)] = (uint32_t)F.list[bb][i].x;
+  }
+}
+// mate[] + w(M): LD-matched vertices from best[] (their pointer), the rest from suitor[]
+template <int THREADS>
+__global__ void __launch_bounds__(THREADS)
+    k_hybrid_finish(const uint64_t* __restrict__ best, const uint32_t* __restrict__ bits,
+                    const uint64_t* __restrict__ suitor, int64_t n, int32_t* __restrict__ mate,
+                    double* pw, long long* pc) {
+  double w = 0.0;
+  long long c = 0;
+  const int64_t stride = (int64_t)gridDim.x * THREADS;
+  for (int64_t i = (int64_t)blockIdx.x * THREADS + threadIdx.x; i < n; i += stride) {
+    uint64_t k = 0;
+    if (bit_test(bits, (uint32_t)i)) k = best[i];
+    else {
+      const uint64_t sk = suitor[i];
+      if (sk != ~0ull) k = sk;
+    }
+    int32_t v = -1;
+    if (k) {
+      v = (int32_t)(uint32_t)k;
+      ++c;
+      if ((int64_t)v > i) w += (double)__uint_as_float((uint32_t)(k >> 32));
+    }
+    mate[i] = v;
+  }
+  block_sum2<THREADS>(w, c, &pw[blockIdx.x], &pc[blockIdx.x]);
 }
 
 }  // namespace lm

@@ -94,6 +94,7 @@ constexpr long long kLogCap = 1 << 16;  // per-round log rows kept on the device
 #define LM_PERSIST_BELOW (1 << 16)
 #endif
 constexpr int64_t kPersistentBelow = LM_PERSIST_BELOW;
+constexpr int64_t kHandoffRounds = 32;  // hybrid (algorithm 2): LD pointing phases before the Suitor tail
 // frontier pointer kernels: lanes per vertex (G) and keys per lane per batch (U), per degree bin
 #ifndef LM_B0_G
 #define LM_B0_G 1
@@ -195,6 +196,11 @@ struct lmatch_graph {
   int64_t stream_chunk = 1ll << 24;
   int64_t hbm_budget = 0;
   int batches = 0;                   // paper-style batch count (> 1: all streamed)
+  int algorithm = 0;                 // 0 = LD pointer iteration, 1 = Suitor (NEXT-4)
+  uint64_t* suitor = nullptr;        // Suitor: best proposal received, (w << 32) | proposer
+  uint32_t* wl[2] = {nullptr, nullptr};   // Suitor worklists
+  uint32_t* wl_big = nullptr;             // Suitor: rows listed for the CTA scan
+  unsigned long long* wl_cnt = nullptr;   // [0..1] worklist sizes, [2] big rows, [3] entries scanned
   bool streaming = false;
   uint64_t* host_adj = nullptr;      // pinned, mapped: entries [R, m)
   uint64_t* host_adj_dev = nullptr;  // its device alias
@@ -729,6 +735,7 @@ int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** 
     g->prune = opts->prune != 0;
     g->host_cache = opts->host_cache >= 0;
     g->batches = opts->batches;
+    g->algorithm = opts->algorithm;
   }
   CK(cudaGetDevice(&g->device));
   CK(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, g->device));
@@ -867,7 +874,8 @@ void lmatch_destroy(lmatch_graph* g) {
   for (void* p : g->ipc_opened) cudaIpcCloseMemHandle(p);
   if (g->h_nf) cudaFreeHost(g->h_nf);
   void* pdev[] = {g->bounds, g->ghost, g->claims, g->claim_cnt, g->rstate, g->rlog, g->d_rargs,
-                  g->cache, g->chunk_rows, g->cache_big, g->live, g->win, g->shadow, g->d_dseg, g->d_dcnt,
+                  g->cache, g->chunk_rows, g->cache_big, g->live, g->win, g->suitor, g->wl[0],
+                  g->wl[1], g->wl_big, g->wl_cnt, g->shadow, g->d_dseg, g->d_dcnt,
                   g->d_dbits, g->d_dnf};
   for (void* p : pdev) if (p) cudaFree(p);
   if (g->h_claim_cnt) cudaFreeHost(g->h_claim_cnt);
@@ -964,7 +972,11 @@ static int seq_prefix(lmatch_graph* g, cudaStream_t st, cudaGraphConditionalHand
       g->bits, nwords, g->best, g->atomic_rows, g->n_atomic, g->counters, lm::kNumCounters,
       g->prune ? g->live : nullptr, g->n, g->rstate);
   CKL();
-  lm::k_round_init<<<1, 1, 0, st>>>(g->rstate, g->max_rounds, kLogCap, work ? 1 : 0);
+  // hybrid (algorithm 2): the LD iteration stops after kHandoffRounds pointing phases and
+  // lmatch_run_device hands the rest to Suitor
+  const int64_t rcap = g->algorithm == 2 && !g->streaming ? std::min<int64_t>(g->max_rounds, kHandoffRounds)
+                                                          : g->max_rounds;
+  lm::k_round_init<<<1, 1, 0, st>>>(g->rstate, rcap, kLogCap, work ? 1 : 0);
   CKL();
   *launches += 2;
   // phase events (inside a graph they become event-record nodes)
@@ -1126,8 +1138,129 @@ static int build_graph_persistent(lmatch_graph* g) {
   return LMATCH_OK;
 }
 
+static int ensure_suitor(lmatch_graph* g) {
+  if (g->suitor) return LMATCH_OK;
+  const int64_t n = g->n;
+  TRY(dmalloc(g, &g->suitor, (size_t)n + 1));
+  TRY(dmalloc(g, &g->wl[0], (size_t)n + 1));
+  TRY(dmalloc(g, &g->wl[1], (size_t)n + 1));
+  TRY(dmalloc(g, &g->wl_big, (size_t)(g->m / lm::kSuitorBig) + 2));  // rows longer than kSuitorBig
+  TRY(dmalloc(g, &g->wl_cnt, 4));
+  return LMATCH_OK;
+}
+
+// Suitor passes over the worklist wl[0] (size wl_cnt[0]) until no proposer is left; each pass
+// scans the proposers' rows (lane / warp / listed CTA per row) and proposes with atomicMax.
+static int suitor_loop(lmatch_graph* g, cudaStream_t st, int64_t* launches, int64_t* passes) {
+  int cur = 0;
+  unsigned long long* hc = g->h_counters;
+  for (;;) {
+    CK(cudaMemcpyAsync(hc, g->wl_cnt, 4 * 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    const int64_t c = (int64_t)hc[cur];
+    if (c == 0) break;
+    if (*passes >= g->max_rounds) { set_err("Suitor did not converge in %lld passes", (long long)*passes); return LMATCH_ECUDA; }
+    unsigned long long* nc = g->wl_cnt + (cur ^ 1);
+    CK(cudaMemsetAsync(nc, 0, 8, st));
+    CK(cudaMemsetAsync(g->wl_cnt + 2, 0, 8, st));
+    lm::k_suitor_scan<<<grid_for(c, 256, 65536), 256, 0, st>>>(
+        g->wl[cur], g->wl_cnt + cur, g->offs, g->adj, g->suitor, g->wl[cur ^ 1], nc, g->wl_big,
+        g->wl_cnt + 2, g->wl_cnt + 3);
+    CKL();
+    lm::k_suitor_scan_big<<<(unsigned)(2 * g->num_sms), 256, 0, st>>>(
+        g->wl_big, g->wl_cnt + 2, g->offs, g->adj, g->suitor, g->wl[cur ^ 1], nc, g->wl_cnt + 3);
+    CKL();
+    *launches += 2;
+    ++*passes;
+    cur ^= 1;
+  }
+  // leave the final (empty) list in slot 0 for the next call
+  if (cur) CK(cudaMemsetAsync(g->wl_cnt, 0, 2 * 8, st));
+  return LMATCH_OK;
+}
+
+// Suitor (NEXT-4): reset, the round-1 sweep (pass 1 proposes to every row maximum), then
+// host-driven passes over the worklist of proposers without a standing proposal.
+static int run_suitor(lmatch_graph* g, int32_t* d_mate, cudaStream_t st, lmatch_stats* stats) {
+  const int64_t n = g->n;
+  const bool tm = g->timing && stats;
+  TRY(ensure_suitor(g));
+  int64_t launches = 0, sweep_launches = 0, bytes_streamed = 0, passes = 0;
+  if (tm) CK(cudaEventRecord(g->ev[0], st));
+  CK(cudaMemsetAsync(g->suitor, 0, ((size_t)n + 1) * 8, st));
+  CK(cudaMemsetAsync(g->wl_cnt, 0, 4 * 8, st));
+  lm::k_reset<<<grid_for(std::max<int64_t>(g->n_atomic, 1), 256, 4096), 256, 0, st>>>(
+      g->bits, 0, g->best, g->atomic_rows, g->n_atomic, g->counters, lm::kNumCounters, nullptr, 0,
+      g->rstate);
+  CKL();
+  ++launches;
+  if (tm) CK(cudaEventRecord(g->ev[1], st));
+  const bool work = g->ntiles > 0 && n > 0;
+  if (work) TRY(round1_sweep(g, st, &launches, &sweep_launches, &bytes_streamed));
+  if (tm) CK(cudaEventRecord(g->ev[2], st));
+  if (work) {
+    lm::k_suitor_first<<<grid_for(n, 256, 65536), 256, 0, st>>>(g->best, n, g->suitor, g->wl[0],
+                                                                  g->wl_cnt + 0);
+    CKL();
+    ++launches;
+    passes = 1;
+  }
+  if (tm) CK(cudaEventRecord(g->ev[3], st));
+  unsigned long long* hc = g->h_counters;
+  if (work) TRY(suitor_loop(g, st, &launches, &passes));
+  if (tm) CK(cudaEventRecord(g->ev[4], st));
+  if (n > 0) {
+    lm::k_suitor_finish<kFinThreads><<<kFinBlocks, kFinThreads, 0, st>>>(g->suitor, n, d_mate, g->pw, g->pc);
+    CKL();
+    lm::k_final_sum<<<1, 32, 0, st>>>(g->pw, g->pc, kFinBlocks, g->res_w, g->res_c);
+    CKL();
+    launches += 2;
+    CK(cudaMemcpyAsync(g->h_res, g->res_w, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(g->h_resc, g->res_c, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(hc, g->wl_cnt, 4 * 8, cudaMemcpyDeviceToHost, st));
+  } else {
+    g->h_res[0] = 0.0;
+    g->h_resc[0] = 0;
+  }
+  if (tm) CK(cudaEventRecord(g->ev[5], st));
+  CK(cudaStreamSynchronize(st));
+  g->round_log.clear();
+  if (stats) {
+    std::memset(stats, 0, sizeof *stats);
+    stats->rounds = passes;
+    stats->matched_vertices = g->h_resc[0];
+    stats->cardinality = g->h_resc[0] / 2;
+    stats->weight = g->h_res[0];
+    stats->entries_swept = (work ? g->m : 0) + (n > 0 ? (int64_t)hc[3] : 0);
+    stats->sweep_launches = sweep_launches;
+    stats->kernel_launches = launches;
+    stats->resident_entries = g->R;
+    if (tm) {
+      float a = 0, b = 0, c = 0, d = 0, e = 0;
+      CK(cudaEventElapsedTime(&a, g->ev[0], g->ev[5]));
+      CK(cudaEventElapsedTime(&b, g->ev[1], g->ev[2]));
+      CK(cudaEventElapsedTime(&c, g->ev[2], g->ev[3]));
+      CK(cudaEventElapsedTime(&d, g->ev[3], g->ev[4]));
+      CK(cudaEventElapsedTime(&e, g->ev[4], g->ev[5]));
+      stats->ms_total = a;
+      stats->ms_sweep = b;
+      stats->ms_round1_rest = c;
+      stats->ms_rounds = d;
+      stats->ms_finish = e;
+    }
+  }
+  return LMATCH_OK;
+}
+
 int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_stats* stats) {
   if (!g) { set_err("NULL handle"); return LMATCH_ESTATE; }
+  if (g->algorithm == 1) {
+    if (!d_mate && g->n > 0) { set_err("d_mate == NULL"); return LMATCH_EINVAL; }
+    if (g->ghost || g->streaming) { set_err("Suitor: resident single-graph handles only"); return LMATCH_EINVAL; }
+    g_err[0] = 0;
+    CK(cudaSetDevice(g->device));
+    return run_suitor(g, d_mate, stream ? (cudaStream_t)stream : g->stream, stats);
+  }
   if (!d_mate && g->n > 0) { set_err("d_mate == NULL"); return LMATCH_EINVAL; }
   if (g->ghost) { set_err("partition handle: use the lmatch_part_* calls"); return LMATCH_ESTATE; }
   g_err[0] = 0;
@@ -1170,9 +1303,41 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
       TRY(seq_body(g, st, cur, nFb, nS, &launches));
     }
   }
+  // ---- hybrid: a frontier left after kHandoffRounds phases goes to Suitor on the residual graph
+  int64_t tail_passes = 0;
+  if (g->algorithm == 2 && !g->streaming && g->ntiles > 0 && n > 0) {
+    CK(cudaMemcpyAsync(g->h_rstate, g->rstate, sizeof(lm::RoundState), cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(g->h_counters, g->counters, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    const int cur = g->h_rstate->cur;
+    int64_t nF = 0;
+    for (int b = 0; b < lm::kBins; ++b) nF += (int64_t)g->h_counters[lm::cnt_F(cur, b)];
+    if (nF > 0) {
+      TRY(ensure_suitor(g));
+      CK(cudaMemsetAsync(g->wl_cnt, 0, 4 * 8, st));
+      lm::k_suitor_tail_init<<<grid_for(n, 256, 65536), 256, 0, st>>>(g->bits, n, g->suitor);
+      CKL();
+      const int64_t nS = (int64_t)g->h_counters[lm::cnt_S(cur)];
+      lm::k_suitor_tail_list<<<grid_for(nS + nF, 256, 65536), 256, 0, st>>>(
+          g->S[cur], g->counters + lm::cnt_S(cur), g->F[cur], g->counters + lm::cnt_F(cur, 0),
+          g->wl[0], g->wl_cnt);
+      CKL();
+      launches += 2;
+      TRY(suitor_loop(g, st, &launches, &tail_passes));
+    }
+  }
   if (tm) CK(cudaEventRecord(g->ev[4], st));
   // ---- A10 mate[] + A9 w(M)
-  if (n > 0) {
+  if (n > 0 && tail_passes > 0) {
+    lm::k_hybrid_finish<kFinThreads><<<kFinBlocks, kFinThreads, 0, st>>>(g->best, g->bits, g->suitor, n,
+                                                                         d_mate, g->pw, g->pc);
+    CKL();
+    lm::k_final_sum<<<1, 32, 0, st>>>(g->pw, g->pc, kFinBlocks, g->res_w, g->res_c);
+    CKL();
+    launches += 2;
+    CK(cudaMemcpyAsync(g->h_res, g->res_w, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(g->h_resc, g->res_c, 8, cudaMemcpyDeviceToHost, st));
+  } else if (n > 0) {
     lm::k_materialize<kFinThreads><<<kFinBlocks, kFinThreads, 0, st>>>(g->best, g->bits, n, g->v0,
                                                                        d_mate, g->pw, g->pc);
     CKL();
@@ -1220,6 +1385,7 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
     stats->kernel_launches = launches;
     stats->bytes_streamed = bytes_streamed;
     stats->resident_entries = g->R;
+    stats->tail_passes = tail_passes;
     if (g->use_cache()) {
       stats->cache_rows = (int64_t)g->h_counters[lm::kCntCache];
       stats->host_entries_read = (int64_t)g->h_counters[lm::kCntCache + 1];

@@ -55,11 +55,12 @@ def test_struct_layout_matches_header(pkg):
 #include <stddef.h>
 #include "lmatch.h"
 int main(void){
-  printf("%zu %zu %zu %zu %zu %zu %zu %zu %zu\n", sizeof(lmatch_opts), sizeof(lmatch_stats),
+  printf("%zu %zu %zu %zu %zu %zu %zu %zu %zu %zu %zu\n", sizeof(lmatch_opts), sizeof(lmatch_stats),
          offsetof(lmatch_stats, weight), offsetof(lmatch_stats, ms_sweep),
          offsetof(lmatch_opts, upload_chunk), offsetof(lmatch_opts, host_cache),
          offsetof(lmatch_opts, batches), offsetof(lmatch_stats, cache_rows),
-         offsetof(lmatch_stats, cache_bytes));
+         offsetof(lmatch_stats, cache_bytes), offsetof(lmatch_opts, algorithm),
+         offsetof(lmatch_stats, tail_passes));
   return 0; }'''
     tmp = os.path.join(ROOT, "build")
     os.makedirs(tmp, exist_ok=True)
@@ -71,7 +72,8 @@ int main(void){
     S, O = pkg.Stats, pkg.Opts
     assert got == [ctypes.sizeof(O), ctypes.sizeof(S), S.weight.offset, S.ms_sweep.offset,
                    O.upload_chunk.offset, O.host_cache.offset, O.batches.offset,
-                   S.cache_rows.offset, S.cache_bytes.offset]
+                   S.cache_rows.offset, S.cache_bytes.offset, O.algorithm.offset,
+                   S.tail_passes.offset]
 
 
 def test_host_side_argument_errors(pkg):

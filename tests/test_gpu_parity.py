@@ -503,3 +503,81 @@ def test_pruning_keeps_rows_permutations(lm):
             if other[u] < 0 and other[v] < 0:
                 other[u], other[v] = v, u
         assert math.isclose(M.weight(other), oracle.weight(g, other), rel_tol=WTOL)
+
+
+# ---------------------------------------------------------- NEXT-4: the Suitor algorithm
+def check_suitor(lm, g):
+    """Suitor under the strict order R1 reaches the same unique matching (mate[] bit-exact,
+    w(M) within 1e-9); its pass count is its own, so rounds are not compared."""
+    return check_parity(lm, g, rounds=False, algorithm="suitor")
+
+
+@pytest.mark.parametrize("name", golden_names())
+def test_suitor_golden(lm, name):
+    g, mate, _, weight = load_golden(name)
+    got, st = run_gpu(lm, g, algorithm="suitor")
+    np.testing.assert_array_equal(got, mate)
+    assert math.isclose(st["weight"], weight, rel_tol=1e-12)
+
+
+def test_suitor_random_tiny_and_paths(lm):
+    rng = np.random.default_rng(23)
+    for _ in range(60):
+        n = int(rng.integers(2, 40))
+        g = graphgen.random_small(n, float(rng.choice([.1, .3, .7])), rng,
+                                  levels=int(rng.choice([0, 2, 5])) or None)
+        check_suitor(lm, g)
+    for n in (2, 3, 17, 301):
+        check_suitor(lm, graphgen.from_edges(n, [(i, i + 1, float(i + 1)) for i in range(n - 1)]))
+    check_suitor(lm, graphgen.from_edges(7, []))
+
+
+@pytest.mark.parametrize("maker", [
+    lambda: graphgen.er(1 << 16, 16.0, seed=1),
+    lambda: graphgen.er(5000, 30.0, seed=3, weights="ones"),
+    lambda: graphgen.rmat(16, 16, seed=1),
+    lambda: graphgen.rmat(15, 16, seed=4, weights="paper"),
+    lambda: graphgen.mesh(256, seed=1),
+    lambda: graphgen.mesh(300, keep=0.6, seed=1),
+    lambda: graphgen.mesh(128, seed=1, weights="gradient"),
+    lambda: _hub_graph(4),
+])
+def test_suitor_synthetic(lm, maker):
+    check_suitor(lm, maker())
+
+
+def test_suitor_repeat_reload_and_rmat24(lm):
+    """Repeated runs and a reload on one Suitor handle; configs[1] at full size against the O(m)
+    certificate and the LD path's result."""
+    g = graphgen.rmat(14, 16, seed=21)
+    g2 = graphgen.rmat(14, 16, seed=21, weights="paper")
+    with lm.Matcher(g, algorithm="suitor") as M:
+        a, _ = M.run()
+        b, _ = M.run()
+        np.testing.assert_array_equal(a, b)
+        np.testing.assert_array_equal(a, oracle.greedy(g).mate)
+        M.reload(g2.offsets, g2.col, g2.w)
+        c, _ = M.run()
+        np.testing.assert_array_equal(c, oracle.greedy(g2).mate)
+    g = graphgen.rmat(24, 16, seed=1)
+    mate, st = run_gpu(lm, g, algorithm="suitor")
+    code, bad = oracle.certificate(g, mate)
+    assert code == 0, (code, bad)
+    ref, _ = run_gpu(lm, g)
+    np.testing.assert_array_equal(mate, ref)
+
+
+@pytest.mark.parametrize("round_loop", [0, 1, 2, 3])
+def test_hybrid_tail(lm, round_loop):
+    """algorithm 2: the LD iteration stops after 32 pointing phases and Suitor finishes on the
+    graph without the vertices matched so far.  Many-round graphs take the tail and stay
+    bit-exact; graphs that finish within 32 phases are untouched (same phase count as Alg. 1)."""
+    for g in (graphgen.mesh(64, seed=1, weights="gradient"),       # ~2*side phases
+              graphgen.from_edges(301, [(i, i + 1, float(i + 1)) for i in range(300)]),
+              graphgen.mesh(90, keep=0.6, seed=2, weights="gradient")):
+        mate, st = check_parity(lm, g, rounds=False, algorithm="hybrid", round_loop=round_loop)
+        assert st["tail_passes"] > 0
+        assert st["rounds"] == 32
+    for g in (graphgen.rmat(16, 16, seed=1), graphgen.mesh(200, seed=3)):
+        mate, st = check_parity(lm, g, algorithm="hybrid", round_loop=round_loop)
+        assert st["tail_passes"] == 0
