@@ -2479,10 +2479,16 @@ __global__ void k_suitor_tail_list(const uint64_t* __restrict__ S, const unsigne
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const int64_t ns = (int64_t)*cntS;
-  for (int64_t i = tid; i < ns; i += stride) wl[atomicAdd(wcnt, 1ull)] = (uint32_t)S[i];
+  for (int64_t i0 = tid - (threadIdx.x & 31); i0 < ns; i0 += stride) {  // warp-uniform trips
+    const int64_t i = i0 + (threadIdx.x & 31);
+    suitor_push(i < ns ? (uint32_t)S[i] : kNoPtr, wl, wcnt);
+  }
   for (int bb = 0; bb < kBins; ++bb) {
     const int64_t c = (int64_t)cntF[bb];
-    for (int64_t i = tid; i < c; i += stride) wl[atomicAdd(wcnt, 1ull)] = (uint32_t)F.list[bb][i].x;
+    for (int64_t i0 = tid - (threadIdx.x & 31); i0 < c; i0 += stride) {
+      const int64_t i = i0 + (threadIdx.x & 31);
+      suitor_push(i < c ? (uint32_t)F.list[bb][i].x : kNoPtr, wl, wcnt);
+    }
   }
 }
 // mate[] + w(M): LD-matched vertices from best[] (their pointer), the rest from suitor[]
