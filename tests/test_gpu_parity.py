@@ -246,6 +246,41 @@ def test_full_size_rmat24_certificate(lm):
     assert st["cardinality"] == int((mate >= 0).sum()) // 2
 
 
+def _full_size_from_device(maker):
+    """A full-size workload generated on the GPU (the generator is bit-identical to the CPU one,
+    tests/test_gpu_graphgen.py), run from the device CSR like bench.py, then brought to the host
+    for the oracle's O(m) certificate."""
+    import torch
+    dg = maker(torch.device("cuda"))
+    h = dg.offsets.cpu().numpy(), dg.col.cpu().numpy(), dg.w.cpu().numpy()
+    return dg, graphgen.Graph(*h)
+
+
+@pytest.mark.parametrize("name", ["rmat_s26", "mesh_8192", "road_8192"])
+def test_full_size_bench_workloads_certificate(lm, name):
+    """The workloads bench.py times, at full size and in its launch configuration (device CSR,
+    default round loop): R-MAT scale 26 (the headline, 2.1e9 directed entries) and configs[2],
+    the 8192 x 8192 mesh and its road-like thinning.  mate[] is checked exactly by the O(m)
+    certificate (C(M) holds iff M is the unique LD matching, R1 iii), w(M) against the
+    oracle's fp64 weight of the same mate[]."""
+    import torch
+    import graphgen.gpu as gg
+    makers = {"rmat_s26": lambda d: gg.rmat(26, 16, seed=1, device=d),
+              "mesh_8192": lambda d: gg.mesh(8192, seed=1, device=d),
+              "road_8192": lambda d: gg.mesh(8192, keep=0.6, seed=1, device=d)}
+    dg, g = _full_size_from_device(makers[name])
+    M = lm.Matcher.from_device(dg.offsets, dg.col, dg.w, dg.n, dg.m,
+                               stream=torch.cuda.current_stream())
+    del dg
+    torch.cuda.empty_cache()
+    mate, st = M.run()
+    M.close()
+    code, bad = oracle.certificate(g, mate)
+    assert code == 0, (code, bad)
+    assert math.isclose(st["weight"], oracle.weight(g, mate), rel_tol=WTOL)
+    assert st["cardinality"] == int((mate >= 0).sum()) // 2
+
+
 # ------------------------------------------------------------------ A8 out-of-core streaming
 @pytest.mark.parametrize("maker,frac,chunk", [
     (lambda: graphgen.rmat(16, 16, seed=5), 0.3, 4096),
