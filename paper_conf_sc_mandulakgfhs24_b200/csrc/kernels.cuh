@@ -33,6 +33,18 @@ constexpr int kBinDeg0 = 8, kBinDeg1 = 64, kBinDeg2 = 2048;  // bins: G = 1, 8, 
 // address space (out-of-core mode; R = m otherwise).  host_off is pre-offset by -R.
 // Out-of-core with the host-row key cache (NEXT-1): indices >= M0 address the cache (HBM),
 // cache_off pre-offset by -M0, so a frontier entry can be redirected to cached keys.
+#ifndef LM_ADJ_NOALLOC
+#define LM_ADJ_NOALLOC 0  // 1 = frontier row reads bypass L1 (keep L1 for the bitmap probes)
+#endif
+__device__ __forceinline__ uint64_t ld_stream_u64(const uint64_t* p) {
+#if LM_ADJ_NOALLOC
+  uint64_t v;
+  asm("ld.global.nc.L1::no_allocate.u64 %0, [%1];" : "=l"(v) : "l"(p));
+  return v;
+#else
+  return __ldg(p);
+#endif
+}
 struct AdjView {
   const uint64_t* dev;
   const uint64_t* host_off;
@@ -40,7 +52,7 @@ struct AdjView {
   const uint64_t* cache_off = nullptr;
   int64_t M0 = INT64_MAX;
   __device__ __forceinline__ uint64_t at(int64_t j) const {
-    return j < R ? __ldg(dev + j) : (j < M0 ? host_off[j] : __ldg(cache_off + j));
+    return j < R ? ld_stream_u64(dev + j) : (j < M0 ? host_off[j] : __ldg(cache_off + j));
   }
   __device__ __forceinline__ uint64_t* ptr(int64_t j) const {
     return const_cast<uint64_t*>(j < R ? dev + j : host_off + j);

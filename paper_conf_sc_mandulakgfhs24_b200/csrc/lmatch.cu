@@ -654,7 +654,25 @@ int build_cache_index(lmatch_graph* g, cudaStream_t st) {
   return LMATCH_OK;
 }
 
+#ifndef LM_MAXL1
+#define LM_MAXL1 0  // 1 = prefer the maximum L1 carveout for the frontier pointer kernels
+#endif
+static int prefer_l1() {
+#if LM_MAXL1
+  static bool done = false;
+  if (done) return LMATCH_OK;
+  done = true;
+  const int c = cudaSharedmemCarveoutMaxL1;
+  CK(cudaFuncSetAttribute(lm::k_point_bin<LM_B1_G, LM_B1_U>, cudaFuncAttributePreferredSharedMemoryCarveout, c));
+  CK(cudaFuncSetAttribute(lm::k_point_bin<LM_B2_G, LM_B2_U>, cudaFuncAttributePreferredSharedMemoryCarveout, c));
+  CK(cudaFuncSetAttribute(lm::k_point_pipe<LM_P0_G, LM_P0_U>, cudaFuncAttributePreferredSharedMemoryCarveout, c));
+  CK(cudaFuncSetAttribute(lm::k_point_bin_cta<256, 4>, cudaFuncAttributePreferredSharedMemoryCarveout, c));
+#endif
+  return LMATCH_OK;
+}
+
 int finish_create(lmatch_graph* g, cudaStream_t st) {
+  TRY(prefer_l1());
   if (g->prune && (g->streaming || g->ghost)) g->prune = 0;  // resident single-graph only
   if (g->prune && !g->live) {
     TRY(dmalloc(g, &g->live, (size_t)g->n + 1));
