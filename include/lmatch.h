@@ -295,8 +295,10 @@ LMATCH_API int lmatch_part_finish(lmatch_graph* g, int32_t* d_mate_local, void* 
  * handles) here (another process: 128 bytes = two cudaIpcMemHandle_t, passed by the caller).
  * A round (the caller puts a barrier -- every part's stream drained, e.g. synchronise + a host
  * barrier -- at each "|"):
- *   | lmatch_p2p_begin / lmatch_p2p_point | lmatch_p2p_match | lmatch_p2p_compact |
- *   lmatch_p2p_frontier_total -> stop when 0, else the next lmatch_p2p_point
+ *   lmatch_p2p_begin / lmatch_p2p_point | [lmatch_p2p_frontier_total of the previous compaction
+ *   -> stop when 0] lmatch_p2p_match | lmatch_p2p_compact, then the next lmatch_p2p_point
+ * (the frontier sizes are pushed by the compaction, so they are visible after the next barrier;
+ * a pointer phase on an empty frontier launches nothing and sends no claims).
  * and lmatch_part_finish at the end.  Calls are stream-ordered and do not synchronise, except
  * lmatch_p2p_compact and lmatch_p2p_frontier_total (they return host values).  Result: as above,
  * bit-identical to the single-GPU run.  Calls on a handle without enable / with a peer missing

@@ -438,20 +438,26 @@ def run_parts_p2p(parts, barrier, transport) -> PartResult:
     for p in parts:
         p.p2p_begin()
     rounds = 1
+    compacted = False
     while True:
-        barrier()                  # claims are in the owners' inboxes
+        # claims are in the owners' inboxes, and the frontier sizes pushed by the last compaction
+        # are in every slot (they were stored before each part's pointer phase)
+        barrier()
+        if compacted:
+            totals = [p.p2p_frontier_total() for p in parts]
+            if any(t != totals[0] for t in totals):
+                raise LMatchError(f"frontier totals differ between parts: {totals}")
+            if totals[0] == 0:
+                break
+            rounds += 1
         for p in parts:
             p.p2p_match()
         barrier()                  # bitmap replicas are complete
         for p in parts:
             p.p2p_compact()
-        barrier()                  # frontier sizes are in every slot
-        totals = [p.p2p_frontier_total() for p in parts]
-        if any(t != totals[0] for t in totals):
-            raise LMatchError(f"frontier totals differ between parts: {totals}")
-        if totals[0] == 0:
-            break
-        rounds += 1
+        compacted = True
+        # the next pointer phase runs before the termination test (two barriers per round, not
+        # three): when the global frontier is empty every part's frontier is, and it does nothing
         for p in parts:
             p.p2p_point()
     fin = [p.finish() for p in parts]
