@@ -1701,7 +1701,23 @@ static int part_point_impl(lmatch_graph* g, cudaStream_t st, int64_t* claim_coun
   const lm::AdjView av = g->view();
   const lm::Bins& Fb = g->F[cur];
   const unsigned long long* cF = g->counters + lm::cnt_F(cur, 0);
-  if (nFb[0]) { lm::k_point_bin<LM_B0_G, LM_B0_U><<<grid_for(nFb[0] * LM_B0_G, 256, 65536), 256, 0, st>>>(Fb.list[0], cF + 0, g->offs, av, g->bits, g->best, g->v0); CKL(); }
+  if (nFb[0]) {
+#if LM_PIPE & 1
+    // the software-pipelined thread-per-row kernel, one resident wave (as in the single-graph
+    // round loop, seq_body)
+    static int occ = 0;
+    if (!occ) {
+      CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, lm::k_point_pipe<LM_P0_G, LM_P0_U>, 256, 0));
+      if (occ < 1) occ = 1;
+    }
+    const int64_t wave = (int64_t)occ * g->num_sms * LM_PIPE_WAVES;
+    lm::k_point_pipe<LM_P0_G, LM_P0_U><<<(unsigned)std::min<int64_t>(wave, (nFb[0] * LM_P0_G + 255) / 256), 256, 0, st>>>(
+        Fb.list[0], cF + 0, g->offs, av, g->bits, g->best, g->v0);
+#else
+    lm::k_point_bin<LM_B0_G, LM_B0_U><<<grid_for(nFb[0] * LM_B0_G, 256, 65536), 256, 0, st>>>(Fb.list[0], cF + 0, g->offs, av, g->bits, g->best, g->v0);
+#endif
+    CKL();
+  }
   if (nFb[1]) { lm::k_point_bin<LM_B1_G, LM_B1_U><<<grid_for(nFb[1] * LM_B1_G, 256, 65536), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, av, g->bits, g->best, g->v0); CKL(); }
   if (nFb[2]) { lm::k_point_bin<LM_B2_G, LM_B2_U><<<grid_for(nFb[2] * LM_B2_G, 256, 65536), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, av, g->bits, g->best, g->v0); CKL(); }
   if (nFb[3]) { lm::k_point_bin_cta<256, 4><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); }
