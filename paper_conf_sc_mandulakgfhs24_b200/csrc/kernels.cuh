@@ -943,21 +943,46 @@ struct RoundArgs {
 #define LM_PROBE 3  // bitmap probes per batch: 0 = all candidates in parallel, 1 = descending, 2 = top first,
                     // 3 = two-phase (lane tops, then only keys above the group's best)
 #endif
-template <int G, int U>
-__device__ __forceinline__ uint64_t scan_row_available(const AdjView adj,
-                                                       const uint32_t* __restrict__ bits,
-                                                       int64_t s, int64_t e, int gl,
-                                                       unsigned rmask) {
+#ifndef LM_IDX32
+#define LM_IDX32 0  // 1 = resident rows indexed with 32-bit offsets from the row start
+#endif
+#ifndef LM_RES_FAST
+#define LM_RES_FAST 1  // rows wholly in the HBM-resident prefix load keys straight from adj.dev
+#endif
+// RES: the row lies in the HBM-resident prefix (e <= R), so keys are plain loads from adj.dev
+// instead of AdjView's per-key region test (decided once per row; group-uniform)
+template <int G, int U, bool RES>
+__device__ __forceinline__ uint64_t scan_row_available_t(const AdjView adj,
+                                                         const uint32_t* __restrict__ bits,
+                                                         int64_t s, int64_t e, int gl,
+                                                         unsigned rmask) {
   uint64_t b = 0;
   (void)rmask;
+#if LM_IDX32
+  // resident rows: 32-bit offsets from the row start (a row has < 2^31 entries)
+  const uint64_t* rp = adj.dev + s;
+  const int32_t len32 = RES ? (int32_t)(e - s) : 0;
+#endif
   // batch loop with a group-uniform trip count (the group votes inside it)
   for (int64_t jb = s; jb < e; jb += (int64_t)G * U) {
     const int64_t j0 = jb + gl;
     uint64_t k[U];
+#if LM_IDX32
+    if (RES) {
+      const int32_t o0 = (int32_t)(jb - s) + gl;
+#pragma unroll
+      for (int q = 0; q < U; ++q) {
+        const int32_t o = o0 + q * G;
+        k[q] = o < len32 ? ld_stream_u64(rp + o) : 0ull;
+      }
+    } else
+#endif
+    {
 #pragma unroll
     for (int q = 0; q < U; ++q) {
       const int64_t j = j0 + (int64_t)q * G;
-      k[q] = j < e ? adj.at(j) : 0ull;
+      k[q] = j < e ? (RES ? ld_stream_u64(adj.dev + j) : adj.at(j)) : 0ull;
+    }
     }
 #if LM_PROBE == 3
     if (G >= LM_PROBE3_MIN_G) {
@@ -1048,6 +1073,16 @@ __device__ __forceinline__ uint64_t scan_row_available(const AdjView adj,
 #endif
   }
   return b;
+}
+template <int G, int U>
+__device__ __forceinline__ uint64_t scan_row_available(const AdjView adj,
+                                                       const uint32_t* __restrict__ bits,
+                                                       int64_t s, int64_t e, int gl,
+                                                       unsigned rmask) {
+#if LM_RES_FAST
+  if (e <= adj.R) return scan_row_available_t<G, U, true>(adj, bits, s, e, gl, rmask);
+#endif
+  return scan_row_available_t<G, U, false>(adj, bits, s, e, gl, rmask);
 }
 
 // A7 in-place pruning (opt-in, lmatch_opts.prune) of a row that fits ONE batch
@@ -1159,6 +1194,16 @@ __global__ void __launch_bounds__(256, LM_BIN_MINB) k_point_bin(ulonglong2* __re
 template <int G, int U>
 __device__ __forceinline__ void load_batch(const AdjView adj, int64_t j0, int64_t e,
                                            uint64_t (&k)[U]) {
+#if LM_RES_FAST
+  if (e <= adj.R) {
+#pragma unroll
+    for (int q = 0; q < U; ++q) {
+      const int64_t j = j0 + (int64_t)q * G;
+      k[q] = j < e ? ld_stream_u64(adj.dev + j) : 0ull;
+    }
+    return;
+  }
+#endif
 #pragma unroll
   for (int q = 0; q < U; ++q) {
     const int64_t j = j0 + (int64_t)q * G;
