@@ -943,6 +943,9 @@ struct RoundArgs {
 #define LM_PROBE 3  // bitmap probes per batch: 0 = all candidates in parallel, 1 = descending, 2 = top first,
                     // 3 = two-phase (lane tops, then only keys above the group's best)
 #endif
+#ifndef LM_MAX1
+#define LM_MAX1 1  // two-phase probe: lane max first, then one compare with the running best (0 = per-key test)
+#endif
 #ifndef LM_IDX32
 #define LM_IDX32 0  // 1 = resident rows indexed with 32-bit offsets from the row start
 #endif
@@ -994,7 +997,12 @@ __device__ __forceinline__ uint64_t scan_row_available_t(const AdjView adj,
     {
       uint64_t mx = 0;
 #pragma unroll
+#if LM_MAX1
+      for (int q = 0; q < U; ++q) mx = umax64(mx, k[q]);
+      if (mx <= b) mx = 0;
+#else
       for (int q = 0; q < U; ++q) mx = (k[q] > b && k[q] > mx) ? k[q] : mx;
+#endif
       bool avail = false;
       if (mx) avail = !((bits[(uint32_t)mx >> 5] >> ((uint32_t)mx & 31)) & 1u);
       uint64_t c = avail ? mx : 0ull;
