@@ -100,13 +100,15 @@ constexpr int64_t kHandoffRounds = 32;  // hybrid (algorithm 2): LD pointing pha
 #define LM_B0_G 1
 #define LM_B0_U 8
 #endif
+// measured at the end of round 1 (R-MAT s26, variants in one call): 32-lane bin U 4 -> 8 and
+// 9..64-entry bin 8x8 -> 16x4 lanes x keys: rounds 8.35 -> 8.10 ms (U = 16: 9.08 ms; 4x16: 9.6 ms)
 #ifndef LM_B1_G
-#define LM_B1_G 8
-#define LM_B1_U 8
+#define LM_B1_G 16
+#define LM_B1_U 4
 #endif
 #ifndef LM_B2_G
 #define LM_B2_G 32
-#define LM_B2_U 4
+#define LM_B2_U 8
 #endif
 
 // host-driven rounds: software-pipelined pointer kernels (one resident wave) per bin: bit b of
