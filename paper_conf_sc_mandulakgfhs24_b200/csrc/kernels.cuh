@@ -27,7 +27,18 @@ namespace lm {
 namespace cg = cooperative_groups;
 
 constexpr int kBins = 4;               // frontier degree bins
-constexpr int kBinDeg0 = 8, kBinDeg1 = 64, kBinDeg2 = 2048;  // bins: G = 1, 8, 32 lanes, CTA
+#ifndef LM_BIN0
+#define LM_BIN0 8
+#endif
+#ifndef LM_BIN1
+#define LM_BIN1 64
+#endif
+#ifndef LM_BIN2
+#define LM_BIN2 2048
+#endif
+// frontier degree bins: <= kBinDeg0 one lane, <= kBinDeg1 a sub-warp group, <= kBinDeg2 a warp,
+// else a CTA (group sizes: LM_B*_G in lmatch.cu)
+constexpr int kBinDeg0 = LM_BIN0, kBinDeg1 = LM_BIN1, kBinDeg2 = LM_BIN2;
 
 // Adjacency view: entries [0, R) in HBM, [R, m) in pinned host memory mapped into the device
 // address space (out-of-core mode; R = m otherwise).  host_off is pre-offset by -R.
@@ -1181,7 +1192,7 @@ __device__ __forceinline__ void point_bin_body(ulonglong2* __restrict__ list, in
   }
 }
 #ifndef LM_BIN_MINB
-#define LM_BIN_MINB 6  // 40-register cap: more resident groups (32-lane bin -12%)
+#define LM_BIN_MINB 8  // 32-register cap, full occupancy (6 -> 8 with the 16x4 / 32x8 bins: rounds 8.09 -> 7.74 ms)
 #endif
 template <int G, int U, bool PRUNE = false>
 __global__ void __launch_bounds__(256, LM_BIN_MINB) k_point_bin(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
