@@ -954,6 +954,9 @@ struct RoundArgs {
 #define LM_PROBE 3  // bitmap probes per batch: 0 = all candidates in parallel, 1 = descending, 2 = top first,
                     // 3 = two-phase (lane tops, then only keys above the group's best)
 #endif
+#ifndef LM_MATCH_V
+#define LM_MATCH_V 4  // frontier entries per thread step in the match, loads batched (1 -> 4: -0.4%)
+#endif
 #ifndef LM_MAX1
 #define LM_MAX1 1  // two-phase probe: lane max first, then one compare with the running best (0 = per-key test)
 #endif
@@ -1537,6 +1540,36 @@ __global__ void k_match_all(const uint64_t* __restrict__ best, int64_t n, uint32
 __device__ __forceinline__ void match_bins_body(const Bins& F, const unsigned long long* cntF,
                                                 const uint64_t* __restrict__ best, uint32_t* bits,
                                                 int64_t tid, int64_t stride) {
+#if LM_MATCH_V > 1
+  // LM_MATCH_V entries per thread step with their dependent loads batched (the chain
+  // entry -> best[ptr] is latency-bound otherwise)
+  constexpr int V = LM_MATCH_V;
+#pragma unroll
+  for (int bb = 0; bb < kBins; ++bb) {
+    const int64_t c = (int64_t)cntF[bb];
+    for (int64_t i0 = tid; i0 < c; i0 += V * stride) {
+      uint64_t p[V], kv[V];
+#pragma unroll
+      for (int q = 0; q < V; ++q) {
+        const int64_t i = i0 + q * stride;
+        p[q] = i < c ? F.list[bb][i].x : ((uint64_t)kNoPtr << 32);
+      }
+#pragma unroll
+      for (int q = 0; q < V; ++q) {
+        const uint32_t v = (uint32_t)(p[q] >> 32);
+        kv[q] = v != kNoPtr ? best[v] : 0ull;
+      }
+#pragma unroll
+      for (int q = 0; q < V; ++q) {
+        const uint32_t u = (uint32_t)p[q], v = (uint32_t)(p[q] >> 32);
+        if (kv[q] != 0 && (uint32_t)kv[q] == u) {
+          atomicOr(&bits[u >> 5], 1u << (u & 31));
+          atomicOr(&bits[v >> 5], 1u << (v & 31));
+        }
+      }
+    }
+  }
+#else
 #pragma unroll
   for (int bb = 0; bb < kBins; ++bb) {
     const int64_t c = (int64_t)cntF[bb];
@@ -1551,6 +1584,7 @@ __device__ __forceinline__ void match_bins_body(const Bins& F, const unsigned lo
       }
     }
   }
+#endif
 }
 __global__ void k_match_bins(Bins F, const unsigned long long* cntF,
                              const uint64_t* __restrict__ best, uint32_t* bits) {

@@ -1095,7 +1095,7 @@ static int seq_body(lmatch_graph* g, cudaStream_t st, int cur, const int64_t* nF
   PIPE_OR_BIN(2, LM_P2_G, LM_P2_U, LM_B2_G, LM_B2_U, LM_A2_G, LM_A2_U)
 #undef PIPE_OR_BIN
   if (nFb[3]) { lm::k_point_bin_cta<256, 4><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); ++*launches; }
-  lm::k_match_bins<<<grid_for(nF, 256, 65536), 256, 0, st>>>(Fb, cF, g->best, g->bits);
+  lm::k_match_bins<<<grid_for((nF + LM_MATCH_V - 1) / LM_MATCH_V, 256, 65536), 256, 0, st>>>(Fb, cF, g->best, g->bits);
   CKL();
   lm::k_compact<false, kCompactK><<<grid_for((nS + nF + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
       lm::compact_io(g->rargs(), cur), g->n, g->best, g->bits, g->offs, g->v0);
