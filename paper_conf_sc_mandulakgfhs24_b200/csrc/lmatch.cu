@@ -106,6 +106,9 @@ constexpr int64_t kHandoffRounds = 32;  // hybrid (algorithm 2): LD pointing pha
 #define LM_B1_G 16
 #define LM_B1_U 4
 #endif
+#ifndef LM_CTA_U
+#define LM_CTA_U 16  // keys per thread per batch in the CTA-per-row bin (4 -> 8 -> 16: rounds 7.73 -> 7.64 -> 7.60 ms)
+#endif
 #ifndef LM_B2_G
 #define LM_B2_G 32
 #define LM_B2_U 8
@@ -668,7 +671,7 @@ static int prefer_l1() {
   CK(cudaFuncSetAttribute(lm::k_point_bin<LM_B1_G, LM_B1_U>, cudaFuncAttributePreferredSharedMemoryCarveout, c));
   CK(cudaFuncSetAttribute(lm::k_point_bin<LM_B2_G, LM_B2_U>, cudaFuncAttributePreferredSharedMemoryCarveout, c));
   CK(cudaFuncSetAttribute(lm::k_point_pipe<LM_P0_G, LM_P0_U>, cudaFuncAttributePreferredSharedMemoryCarveout, c));
-  CK(cudaFuncSetAttribute(lm::k_point_bin_cta<256, 4>, cudaFuncAttributePreferredSharedMemoryCarveout, c));
+  CK(cudaFuncSetAttribute(lm::k_point_bin_cta<256, LM_CTA_U>, cudaFuncAttributePreferredSharedMemoryCarveout, c));
 #endif
   return LMATCH_OK;
 }
@@ -1094,7 +1097,7 @@ static int seq_body(lmatch_graph* g, cudaStream_t st, int cur, const int64_t* nF
   PIPE_OR_BIN(1, LM_P1_G, LM_P1_U, LM_B1_G, LM_B1_U, LM_A1_G, LM_A1_U)
   PIPE_OR_BIN(2, LM_P2_G, LM_P2_U, LM_B2_G, LM_B2_U, LM_A2_G, LM_A2_U)
 #undef PIPE_OR_BIN
-  if (nFb[3]) { lm::k_point_bin_cta<256, 4><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); ++*launches; }
+  if (nFb[3]) { lm::k_point_bin_cta<256, LM_CTA_U><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); ++*launches; }
   lm::k_match_bins<<<grid_for((nF + LM_MATCH_V - 1) / LM_MATCH_V, 256, 65536), 256, 0, st>>>(Fb, cF, g->best, g->bits);
   CKL();
   lm::k_compact<false, kCompactK><<<grid_for((nS + nF + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
@@ -1722,7 +1725,7 @@ static int part_point_impl(lmatch_graph* g, cudaStream_t st, int64_t* claim_coun
   }
   if (nFb[1]) { lm::k_point_bin<LM_B1_G, LM_B1_U><<<grid_for(nFb[1] * LM_B1_G, 256, 65536), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, av, g->bits, g->best, g->v0); CKL(); }
   if (nFb[2]) { lm::k_point_bin<LM_B2_G, LM_B2_U><<<grid_for(nFb[2] * LM_B2_G, 256, 65536), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, av, g->bits, g->best, g->v0); CKL(); }
-  if (nFb[3]) { lm::k_point_bin_cta<256, 4><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); }
+  if (nFb[3]) { lm::k_point_bin_cta<256, LM_CTA_U><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); }
   if (!g->p2p) CK(cudaMemsetAsync(g->claim_cnt, 0, (size_t)g->P * 8, st));
   if (nF > 0) {
     const lm::Claims Cl = part_claims_desc(g);
