@@ -106,6 +106,9 @@ constexpr int64_t kHandoffRounds = 32;  // hybrid (algorithm 2): LD pointing pha
 #define LM_B1_G 16
 #define LM_B1_U 4
 #endif
+#ifndef LM_BIN_STREAMS
+#define LM_BIN_STREAMS 1  // frontier bins of a round on concurrent side streams (R-MAT s26 rounds 7.64 -> 7.50 ms)
+#endif
 #ifndef LM_CTA_U
 #define LM_CTA_U 16  // keys per thread per batch in the CTA-per-row bin (4 -> 8 -> 16: rounds 7.73 -> 7.64 -> 7.60 ms)
 #endif
@@ -164,6 +167,8 @@ struct lmatch_graph {
   int device = 0;
   cudaStream_t stream = nullptr;   // handle stream
   cudaStream_t up[2] = {nullptr, nullptr};
+  cudaStream_t bs[3] = {nullptr, nullptr, nullptr};  // side streams for the frontier bins
+  cudaEvent_t ev_fork = nullptr, ev_join[3] = {nullptr, nullptr, nullptr};
   int64_t n = 0, m = 0, n_nz = 0, ntiles = 0;  // n, m: this handle's rows and entries
   // partitioned mode (lmatch_create_part): rows [v0, v0 + n) of a graph with n_global vertices
   int64_t v0 = 0, n_global = 0;
@@ -766,6 +771,13 @@ int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** 
   CK(cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking));
   CK(cudaStreamCreateWithFlags(&g->up[0], cudaStreamNonBlocking));
   CK(cudaStreamCreateWithFlags(&g->up[1], cudaStreamNonBlocking));
+  if (LM_BIN_STREAMS) {
+    for (int i = 0; i < 3; ++i) {
+      CK(cudaStreamCreateWithFlags(&g->bs[i], cudaStreamNonBlocking));
+      CK(cudaEventCreateWithFlags(&g->ev_join[i], cudaEventDisableTiming));
+    }
+    CK(cudaEventCreateWithFlags(&g->ev_fork, cudaEventDisableTiming));
+  }
   for (auto& e : g->ev) CK(cudaEventCreate(&e));
   TRY(alloc_all(g));
   if (part) {
@@ -907,6 +919,9 @@ void lmatch_destroy(lmatch_graph* g) {
   for (auto e : g->ev) if (e) cudaEventDestroy(e);
   if (g->stream) cudaStreamDestroy(g->stream);
   for (auto s : g->up) if (s) cudaStreamDestroy(s);
+  for (auto s : g->bs) if (s) cudaStreamDestroy(s);
+  for (auto e : g->ev_join) if (e) cudaEventDestroy(e);
+  if (g->ev_fork) cudaEventDestroy(g->ev_fork);
   delete g;
 }
 
@@ -1093,11 +1108,38 @@ static int seq_body(lmatch_graph* g, cudaStream_t st, int cur, const int64_t* nF
     CKL();                                                                                        \
     ++*launches;                                                                                  \
   }
+  // the bins of a round are independent (disjoint rows, read-only bitmap): with LM_BIN_STREAMS
+  // the 16-lane, 32-lane and CTA bins run on side streams next to the thread bin, so the tail
+  // of one kernel overlaps the others; the match waits for all of them
+  const int nbusy = (nFb[0] > 0) + (nFb[1] > 0) + (nFb[2] > 0) + (nFb[3] > 0);
+  const bool fork = LM_BIN_STREAMS && g->bs[0] && nbusy > 1;
+  if (fork) {
+    CK(cudaEventRecord(g->ev_fork, st));
+    for (int i = 0; i < 3; ++i) CK(cudaStreamWaitEvent(g->bs[i], g->ev_fork, 0));
+  }
+  {
+    cudaStream_t st_main = st;
+    {
+      cudaStream_t st = fork ? g->bs[0] : st_main;
+      PIPE_OR_BIN(1, LM_P1_G, LM_P1_U, LM_B1_G, LM_B1_U, LM_A1_G, LM_A1_U)
+    }
+    {
+      cudaStream_t st = fork ? g->bs[1] : st_main;
+      PIPE_OR_BIN(2, LM_P2_G, LM_P2_U, LM_B2_G, LM_B2_U, LM_A2_G, LM_A2_U)
+    }
+    {
+      cudaStream_t st = fork ? g->bs[2] : st_main;
+      if (nFb[3]) { lm::k_point_bin_cta<256, LM_CTA_U><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); ++*launches; }
+    }
+  }
   PIPE_OR_BIN(0, LM_P0_G, LM_P0_U, LM_B0_G, LM_B0_U, LM_A0_G, LM_A0_U)
-  PIPE_OR_BIN(1, LM_P1_G, LM_P1_U, LM_B1_G, LM_B1_U, LM_A1_G, LM_A1_U)
-  PIPE_OR_BIN(2, LM_P2_G, LM_P2_U, LM_B2_G, LM_B2_U, LM_A2_G, LM_A2_U)
 #undef PIPE_OR_BIN
-  if (nFb[3]) { lm::k_point_bin_cta<256, LM_CTA_U><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); ++*launches; }
+  if (fork) {
+    for (int i = 0; i < 3; ++i) {
+      CK(cudaEventRecord(g->ev_join[i], g->bs[i]));
+      CK(cudaStreamWaitEvent(st, g->ev_join[i], 0));
+    }
+  }
   lm::k_match_bins<<<grid_for((nF + LM_MATCH_V - 1) / LM_MATCH_V, 256, 65536), 256, 0, st>>>(Fb, cF, g->best, g->bits);
   CKL();
   lm::k_compact<false, kCompactK><<<grid_for((nS + nF + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
