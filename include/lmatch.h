@@ -133,11 +133,15 @@ typedef struct lmatch_opts {
 
 /* Filled by lmatch_run / lmatch_run_device when non-NULL. */
 typedef struct lmatch_stats {
-  int64_t rounds;            /* pointing phases executed (round 1 = full sweep) */
+  int64_t rounds;            /* pointing phases executed (round 1 = full sweep); algorithm 1:
+                                Suitor passes (pass 1 = the sweep's row maxima); algorithm 2:
+                                LD phases before the handoff (see tail_passes) */
   int64_t matched_vertices;  /* 2 x |M| */
   int64_t cardinality;       /* |M| */
   double weight;             /* w(M) = sum of matched edge weights, fp64 */
-  int64_t entries_swept;     /* adjacency entries scanned over all rounds */
+  int64_t entries_swept;     /* adjacency entries of the rows scanned over all rounds (rows the
+                                out-of-core cache decided are counted with their full degree;
+                                host_entries_read has the host part actually read) */
   int64_t frontier_total;    /* sum over rounds >= 2 of |F_r| (vertices re-pointed) */
   double ms_total;           /* (timing=1) lmatch_run_device body, device time */
   double ms_sweep;           /* (timing=1) round-1 pointer sweep kernel alone */
