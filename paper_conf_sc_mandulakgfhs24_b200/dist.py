@@ -418,6 +418,27 @@ def barrier_local(parts):
     return b
 
 
+def barrier_events(parts):
+    """Barrier for parts in one process without draining any stream: every part records an
+    event on its stream and every part's stream waits for all the others' events (works across
+    devices too), so the phases stay ordered on the GPUs while the host runs ahead."""
+    import torch
+
+    def b():
+        # gather on part 0's stream, then release everyone from it: 2(P-1) waits instead of P^2
+        hub = parts[0].stream
+        for p in parts[1:]:
+            e = torch.cuda.Event()
+            e.record(p.stream)
+            hub.wait_event(e)
+        if len(parts) > 1:
+            e = torch.cuda.Event()
+            e.record(hub)
+            for p in parts[1:]:
+                p.stream.wait_event(e)
+    return b
+
+
 def barrier_torch(parts, group=None):
     """Barrier across processes: drain the local streams, then a torch.distributed barrier."""
     import torch.distributed as dist
@@ -482,7 +503,8 @@ def transport_sum_float(transport, xs):
 def match_partitioned_local(offsets, col, w, nparts: int, device=None, exchange: str = "transport"):
     """P logical partitions of one graph on one device.  exchange = "transport": LocalTransport
     moves the claims / bitmap words; "p2p": the library's kernels store them into the other parts'
-    memory (peer-memory exchange).  Returns (mate, result)."""
+    memory (peer-memory exchange), phases ordered by cross-stream events; "p2p_sync": the same with
+    host-synchronising barriers.  Returns (mate, result)."""
     offsets = np.asarray(offsets, dtype=np.int64)
     n = offsets.shape[0] - 1
     bounds = edge_balanced_bounds(offsets, nparts)
@@ -491,9 +513,10 @@ def match_partitioned_local(offsets, col, w, nparts: int, device=None, exchange:
         v0, v1 = int(bounds[p]), int(bounds[p + 1])
         lo, lc, lw = local_csr(offsets, col, w, v0, v1)
         parts.append(LibPart(lo, lc, lw, v0, n, bounds, p, device=device))
-    if exchange == "p2p":
+    if exchange in ("p2p", "p2p_sync"):
         connect_p2p_local(parts)
-        res = run_parts_p2p(parts, barrier_local(parts), LocalTransport(nparts))
+        barrier = barrier_events(parts) if exchange == "p2p" else barrier_local(parts)
+        res = run_parts_p2p(parts, barrier, LocalTransport(nparts))
     else:
         res = run_parts(parts, LocalTransport(nparts))
     mate = np.concatenate([m.cpu().numpy() for m in res.mates]) if n else np.zeros(0, np.int32)

@@ -36,14 +36,15 @@ def main():
     ref = None
     for P in a.parts:
         b = D.edge_balanced_bounds(off, P)
-        for ex in ("transport", "p2p"):
+        for ex in ("transport", "p2p", "p2p_events"):
             parts = []
             for p in range(P):
                 lo, lc, lw = D.local_csr(off, col, w, int(b[p]), int(b[p + 1]))
                 parts.append(D.LibPart(lo, lc, lw, int(b[p]), g.n, b, p, device=dev))
-            if ex == "p2p":
+            if ex.startswith("p2p"):
                 D.connect_p2p_local(parts)
-                run = lambda: D.run_parts_p2p(parts, D.barrier_local(parts), D.LocalTransport(P))  # noqa: E731
+                bar = D.barrier_events(parts) if ex == "p2p_events" else D.barrier_local(parts)
+                run = lambda: D.run_parts_p2p(parts, bar, D.LocalTransport(P))  # noqa: E731
             else:
                 run = lambda: D.run_parts(parts, D.LocalTransport(P))  # noqa: E731
             for _ in range(a.warmup):

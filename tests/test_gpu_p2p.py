@@ -50,9 +50,11 @@ def _check(g, mate, res):
     lambda: graphgen.mesh(40, seed=14, weights="gradient"),
 ])
 def test_p2p_local_invariance(D, P, maker):
+    """Cross-stream event barriers (default) and host-synchronising barriers."""
     g = maker()
-    mate, res = D.match_partitioned_local(g.offsets, g.col, g.w, P, exchange="p2p")
-    _check(g, mate, res)
+    for ex in ("p2p", "p2p_sync"):
+        mate, res = D.match_partitioned_local(g.offsets, g.col, g.w, P, exchange=ex)
+        _check(g, mate, res)
 
 
 @pytest.mark.parametrize("exchange", ["transport", "p2p"])
