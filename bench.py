@@ -301,7 +301,10 @@ def run_partitioned(a, rank, world, local):
     tr = D.TorchTransport()
     if a.exchange == "p2p":
         D.connect_p2p_torch(part)
-        barrier = D.barrier_torch([part])
+        # phases ordered by interprocess CUDA events (a gloo host barrier only orders the
+        # records before the waits; no stream is drained), see dist.barrier_torch_events
+        D.connect_events_torch(part)
+        barrier = D.barrier_torch_events([part], dist.new_group(backend="gloo"))
         run = lambda: D.run_parts_p2p([part], barrier, tr)  # noqa: E731
     else:
         run = lambda: D.run_parts([part], tr)  # noqa: E731
@@ -386,7 +389,7 @@ def run_partitioned(a, rank, world, local):
                 "config": workload_config(a, scale, n, m) | {
                     "parallelism": f"1-D vertex partition over {world} GPU(s): " + (
                         "claims / changed bitmap words / frontier sizes stored into the peers' memory "
-                        "by the library's kernels (CUDA IPC, lmatch_p2p_*), host barriers"
+                        "by the library's kernels (CUDA IPC, lmatch_p2p_*), interprocess-event barriers"
                         if a.exchange == "p2p" else
                         "claims all-to-all + bitmap allgather + frontier allreduce per round (NCCL)"),
                     "exchange": a.exchange,

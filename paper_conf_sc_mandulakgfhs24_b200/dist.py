@@ -439,6 +439,37 @@ def barrier_events(parts):
     return b
 
 
+def connect_events_torch(part, group=None):
+    """Cross-process event barrier setup: an interprocess CUDA event per rank, its IPC handle
+    all-gathered, the peers' events opened here (part.peer_events)."""
+    import torch
+    import torch.distributed as dist
+    part.ev = torch.cuda.Event(interprocess=True)
+    part.ev.record(part.stream)  # an event must be recorded once before its handle is exported
+    allh = [None] * dist.get_world_size(group)
+    dist.all_gather_object(allh, (part.part, part.ev.ipc_handle()), group=group)
+    part.peer_events = [torch.cuda.Event.from_ipc_handle(part.dev, h) for peer, h in allh
+                        if peer != part.part]
+
+
+def barrier_torch_events(parts, cpu_group=None):
+    """Barrier across processes that drains no stream: each rank records its interprocess event,
+    a host barrier (cpu_group, e.g. gloo) guarantees every record is issued, then each rank's
+    stream waits for the peers' events.  A rank may run one barrier ahead; a wait then refers to
+    a later record of the peer's event, which over-orders but cannot deadlock (a record never
+    waits on anything behind it)."""
+    import torch.distributed as dist
+
+    def b():
+        for p in parts:
+            p.ev.record(p.stream)
+        dist.barrier(group=cpu_group)
+        for p in parts:
+            for e in p.peer_events:
+                p.stream.wait_event(e)
+    return b
+
+
 def barrier_torch(parts, group=None):
     """Barrier across processes: drain the local streams, then a torch.distributed barrier."""
     import torch.distributed as dist

@@ -147,7 +147,7 @@ def _free_port():
     return port
 
 
-def _ipc_worker(rank, world, port, spec, q):
+def _ipc_worker(rank, world, port, spec, q, events=False):
     import torch
     import torch.distributed as dist
     import paper_conf_sc_mandulakgfhs24_b200.dist as D
@@ -163,9 +163,14 @@ def _ipc_worker(rank, world, port, spec, q):
         lo, lc, lw = D.local_csr(g.offsets, g.col, g.w, int(b[rank]), int(b[rank + 1]))
         part = D.LibPart(lo, lc, lw, int(b[rank]), g.n, b, rank)
         D.connect_p2p_torch(part)
+        if events:
+            D.connect_events_torch(part)
+            barrier = D.barrier_torch_events([part])
+        else:
+            barrier = D.barrier_torch([part])
         out = []
         for _ in range(2):
-            res = D.run_parts_p2p([part], D.barrier_torch([part]), D.TorchTransport())
+            res = D.run_parts_p2p([part], barrier, D.TorchTransport())
             out.append((res.mates[0].cpu().numpy(), res.weight, res.matched, res.rounds))
         q.put((rank, out))
         dist.barrier()   # no rank releases its window while a peer may still store into it
@@ -178,15 +183,19 @@ def _ipc_worker(rank, world, port, spec, q):
         dist.destroy_process_group()
 
 
+@pytest.mark.parametrize("events", [False, True])
 @pytest.mark.parametrize("world,spec", [(2, ("rmat", (14, 16, 5))), (3, ("mesh", (60, 0.6, 2)))])
-def test_p2p_ipc_processes(D, world, spec):
+def test_p2p_ipc_processes(D, world, spec, events):
     """`world` processes on the one GPU, windows and bitmaps opened through CUDA IPC handles
-    exchanged with all_gather_object, barriers over gloo; run twice on the same connection."""
+    exchanged with all_gather_object; barriers either drain the stream + gloo barrier, or
+    interprocess CUDA events (record, gloo barrier, stream waits: no stream drained); run twice
+    on the same connection."""
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_ipc_worker, args=(r, world, port, spec, q)) for r in range(world)]
+    procs = [ctx.Process(target=_ipc_worker, args=(r, world, port, spec, q, events))
+             for r in range(world)]
     for p in procs:
         p.start()
     got = [q.get(timeout=300) for _ in range(world)]
