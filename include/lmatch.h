@@ -304,7 +304,8 @@ LMATCH_API int lmatch_part_finish(lmatch_graph* g, int32_t* d_mate_local, void* 
  * (the frontier sizes are pushed by the compaction, so they are visible after the next barrier;
  * a pointer phase on an empty frontier launches nothing and sends no claims).
  * and lmatch_part_finish at the end.  Calls are stream-ordered and do not synchronise, except
- * lmatch_p2p_compact and lmatch_p2p_frontier_total (they return host values).  Result: as above,
+ * lmatch_p2p_frontier_total (and lmatch_p2p_compact when asked for the local size): one host
+ * read per round.  Result: as above,
  * bit-identical to the single-GPU run.  Calls on a handle without enable / with a peer missing
  * return ESTATE; lmatch_part_begin/point/apply on an enabled handle return ESTATE.
  * ------------------------------------------------------------------------------------------- */
@@ -316,7 +317,10 @@ LMATCH_API int lmatch_p2p_attach(lmatch_graph* g, int32_t peer, const void* hand
 LMATCH_API int lmatch_p2p_begin(lmatch_graph* g, void* stream);
 LMATCH_API int lmatch_p2p_point(lmatch_graph* g, void* stream);
 LMATCH_API int lmatch_p2p_match(lmatch_graph* g, void* stream);
-/* *nF_local = this part's next frontier size (synchronises `stream`). */
+/* Compaction, then this part's frontier size pushed into every peer's slot.  nF_local NULL:
+ * stream-ordered, no synchronisation (peer-memory rounds size their launches from the
+ * device-resident counts, so nothing is read back); non-NULL: synchronises `stream` and returns
+ * this part's next frontier size. */
 LMATCH_API int lmatch_p2p_compact(lmatch_graph* g, void* stream, int64_t* nF_local);
 /* *nF_total = the sum of every part's pushed frontier size (synchronises `stream`). */
 LMATCH_API int lmatch_p2p_frontier_total(lmatch_graph* g, void* stream, int64_t* nF_total);

@@ -1702,11 +1702,9 @@ int lmatch_part_bitmap(lmatch_graph* g, uint32_t** d_bits, int64_t* word_begin, 
   return LMATCH_OK;
 }
 
-int lmatch_part_compact(lmatch_graph* g, void* stream, int64_t* nF_local) {
-  if (!g || !g->ghost || g->part_round < 1) { set_err("lmatch_part_compact out of order"); return LMATCH_ESTATE; }
-  CK(cudaSetDevice(g->device));
-  cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
-  unsigned long long* C = g->counters;
+// the compaction launches of a partition round; the set sizes come from h_counters, or (peer-
+// memory rounds, which do not read them back every round) a full resident wave per kernel
+static int part_compact_launch(lmatch_graph* g, cudaStream_t st) {
   const int64_t n = g->n;
   // the compaction reads set part_cur (round 1: none) and writes its other set; k_end_round
   // makes that set current (and zeroes the counters the next compaction writes)
@@ -1723,16 +1721,26 @@ int lmatch_part_compact(lmatch_graph* g, void* stream, int64_t* nF_local) {
     const int64_t nS = (int64_t)g->h_counters[lm::cnt_S(cur)];
     int64_t nF = 0;
     for (int b = 0; b < lm::kBins; ++b) nF += (int64_t)g->h_counters[lm::cnt_F(cur, b)];
-    if (nS + nF > 0) {
-      lm::k_compact<false, kCompactK>
-          <<<grid_for((nS + nF + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
-              lm::compact_io(g->rargs(), cur), n, g->best, g->bits, g->offs, g->v0);
+    if (g->p2p || nS + nF > 0) {
+      const unsigned grid = g->p2p ? (unsigned)(4 * g->num_sms)
+                                   : grid_for((nS + nF + 31) / 32, 8 * kCompactK, 65536);
+      lm::k_compact<false, kCompactK><<<grid, 256, 0, st>>>(
+          lm::compact_io(g->rargs(), cur), n, g->best, g->bits, g->offs, g->v0);
       CKL();
     }
     g->part_cur = cur ^ 1;
   }
   lm::k_end_round<<<1, 32, 0, st>>>(g->ra(), 0, 0, 0);
   CKL();
+  return LMATCH_OK;
+}
+
+int lmatch_part_compact(lmatch_graph* g, void* stream, int64_t* nF_local) {
+  if (!g || !g->ghost || g->part_round < 1) { set_err("lmatch_part_compact out of order"); return LMATCH_ESTATE; }
+  CK(cudaSetDevice(g->device));
+  cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
+  unsigned long long* C = g->counters;
+  TRY(part_compact_launch(g, st));
   CK(cudaMemcpyAsync(g->h_counters, C, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
   int64_t nF = 0;
@@ -1745,6 +1753,13 @@ static int part_point_impl(lmatch_graph* g, cudaStream_t st, int64_t* claim_coun
   const int cur = g->part_cur;
   int64_t nFb[lm::kBins], nF = 0;
   for (int b = 0; b < lm::kBins; ++b) { nFb[b] = (int64_t)g->h_counters[lm::cnt_F(cur, b)]; nF += nFb[b]; }
+  if (g->p2p) {
+    // peer-memory rounds do not read the bin sizes back: every kernel below loops over the
+    // device-resident count, so launch each bin with a full resident wave (an empty bin exits)
+    const int64_t wave = 8ll * g->num_sms;
+    for (int b = 0; b < lm::kBins; ++b) nFb[b] = wave * 256;
+    nF = wave * 256;
+  }
   const lm::AdjView av = g->view();
   const lm::Bins& Fb = g->F[cur];
   const unsigned long long* cF = g->counters + lm::cnt_F(cur, 0);
@@ -1767,15 +1782,16 @@ static int part_point_impl(lmatch_graph* g, cudaStream_t st, int64_t* claim_coun
   }
   if (nFb[1]) { lm::k_point_bin<LM_B1_G, LM_B1_U><<<grid_for(nFb[1] * LM_B1_G, 256, 65536), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, av, g->bits, g->best, g->v0); CKL(); }
   if (nFb[2]) { lm::k_point_bin<LM_B2_G, LM_B2_U><<<grid_for(nFb[2] * LM_B2_G, 256, 65536), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, av, g->bits, g->best, g->v0); CKL(); }
-  if (nFb[3]) { lm::k_point_bin_cta<256, LM_CTA_U><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); }
+  if (nFb[3]) { lm::k_point_bin_cta<256, LM_CTA_U><<<(unsigned)std::min<int64_t>(nFb[3], g->p2p ? 8ll * g->num_sms : 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); }
   if (!g->p2p) CK(cudaMemsetAsync(g->claim_cnt, 0, (size_t)g->P * 8, st));
   if (nF > 0) {
     const lm::Claims Cl = part_claims_desc(g);
     lm::k_claims_bins<<<grid_for(nF, 256, 65536), 256, 0, st>>>(Fb, cF, g->v0, g->v0 + g->n, Cl);
     CKL();
   }
-  g->round_log.insert(g->round_log.end(), {nF, nF + (int64_t)g->h_counters[lm::cnt_S(cur)],
-                                           (int64_t)g->h_counters[lm::kCntSwept]});
+  if (!g->p2p)
+    g->round_log.insert(g->round_log.end(), {nF, nF + (int64_t)g->h_counters[lm::cnt_S(cur)],
+                                             (int64_t)g->h_counters[lm::kCntSwept]});
   ++g->part_round;
   return g->p2p ? LMATCH_OK : part_claims_out(g, st, claim_counts);
 }
@@ -1975,14 +1991,11 @@ int lmatch_p2p_match(lmatch_graph* g, void* stream) {
       CKL();
     }
   } else {
-    int64_t nF = 0;
-    for (int b = 0; b < lm::kBins; ++b) nF += (int64_t)g->h_counters[lm::cnt_F(g->part_cur, b)];
-    if (nF > 0) {
-      lm::k_match_part_bins<<<grid_for(nF, 256, 65536), 256, 0, st>>>(
-          g->F[g->part_cur], g->counters + lm::cnt_F(g->part_cur, 0), g->best, g->v0, g->v0 + g->n,
-          g->ghost, g->bits);
-      CKL();
-    }
+    // the frontier size is device-resident (not read back in peer-memory rounds): one wave
+    lm::k_match_part_bins<<<(unsigned)(8 * g->num_sms), 256, 0, st>>>(
+        g->F[g->part_cur], g->counters + lm::cnt_F(g->part_cur, 0), g->best, g->v0, g->v0 + g->n,
+        g->ghost, g->bits);
+    CKL();
   }
   lm::k_match_inbox<<<(unsigned)grid, 256, 0, st>>>(g->win, g->win_cap, icnt, P, g->best, g->v0,
                                                      g->bits);
@@ -2001,11 +2014,14 @@ int lmatch_p2p_match(lmatch_graph* g, void* stream) {
 int lmatch_p2p_compact(lmatch_graph* g, void* stream, int64_t* nF_local) {
   TRY(p2p_ready(g));
   cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
-  int64_t nf = 0;
-  TRY(lmatch_part_compact(g, st, &nf));
+  if (nF_local) {
+    TRY(lmatch_part_compact(g, st, nF_local));  // synchronising variant (host needs the size)
+  } else {
+    CK(cudaSetDevice(g->device));
+    TRY(part_compact_launch(g, st));
+  }
   lm::k_push_count<<<1, 32, 0, st>>>(g->counters + lm::cnt_F(g->part_cur, 0), lm::kBins, g->d_dnf, g->P);
   CKL();
-  if (nF_local) *nF_local = nf;
   return LMATCH_OK;
 }
 

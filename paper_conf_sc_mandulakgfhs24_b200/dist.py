@@ -319,7 +319,12 @@ class LibPart:
     def p2p_match(self):
         _check(_lib.lmatch_p2p_match(self.h, self._s()), "lmatch_p2p_match")
 
-    def p2p_compact(self) -> int:
+    def p2p_compact(self, local_size: bool = False):
+        """Compaction + frontier-size push; stream-ordered (no sync) unless local_size=True,
+        which synchronises and returns this part's next frontier size."""
+        if not local_size:
+            _check(_lib.lmatch_p2p_compact(self.h, self._s(), None), "lmatch_p2p_compact")
+            return None
         nf = _I64()
         _check(_lib.lmatch_p2p_compact(self.h, self._s(), ctypes.byref(nf)), "lmatch_p2p_compact")
         return int(nf.value)
