@@ -395,6 +395,9 @@ __global__ void k_reset(uint32_t* bits, int64_t nwords, uint64_t* best,
 //     => identical to one sequential scan; such rows are zeroed by k_reset).
 // Self-loop keys were zeroed at ingest (k_zap_self_loops).  No bitmap test in round 1.
 // =============================================================================================
+#ifndef LM_SWEEP_LONG
+#define LM_SWEEP_LONG 32  // in-tile rows with at least this many entries are reduced by the warp
+#endif
 #ifndef LM_SWEEP_MID
 #define LM_SWEEP_MID 0  // 1 = rows of 8..31 in-tile entries by 8-lane groups (build knob)
 #endif
@@ -581,7 +584,7 @@ __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
       }
       if (L > 0 && L < 8) {
 #else
-      if (L > 0 && L < 32) {
+      if (L > 0 && L < LM_SWEEP_LONG) {
 #endif
         uint64_t b0 = 0, b1 = 0, b2 = 0, b3 = 0;  // 4 independent max chains
         int j = max(rs, 0);
@@ -600,7 +603,7 @@ __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
         else if (b) atomicMax(reinterpret_cast<unsigned long long*>(&A.best[vid]), (unsigned long long)b);
       }
       // long rows: the whole warp, one row at a time
-      unsigned lm = __ballot_sync(0xffffffffu, L >= 32);
+      unsigned lm = __ballot_sync(0xffffffffu, L >= LM_SWEEP_LONG);
       while (lm) {
         const int l = __ffs(lm) - 1;
         lm &= lm - 1;
