@@ -2361,7 +2361,9 @@ template <int K>
 __global__ void k_cache_redirect(Bins F, const unsigned long long* __restrict__ cntF,
                                  const int64_t* __restrict__ offs, const uint64_t* __restrict__ cache,
                                  const uint32_t* __restrict__ bits, int64_t u_first, int64_t M0,
-                                 int64_t vbase, unsigned long long* cnt) {
+                                 int64_t vbase, unsigned long long* cnt,
+                                 uint64_t* __restrict__ rescan = nullptr,
+                                 unsigned long long* nrescan = nullptr) {
   const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   unsigned long long served = 0, left = 0;
@@ -2395,6 +2397,9 @@ __global__ void k_cache_redirect(Bins F, const unsigned long long* __restrict__ 
         e.y = (uint64_t)(M0 + slot);
       } else {
         left += (unsigned long long)(en - s);
+        // refill path: k_host_rescan reads the row once, refills the cache with its K largest
+        // available keys and redirects this entry to the first of them
+        if (rescan) rescan[atomicAdd(nrescan, 1ull)] = ((uint64_t)bb << 40) | (uint64_t)i;
         continue;
       }
       F.list[bb][i].y = e.y;
@@ -2408,6 +2413,47 @@ __global__ void k_cache_redirect(Bins F, const unsigned long long* __restrict__ 
   if ((threadIdx.x & 31) == 0) {
     if (served) atomicAdd(&cnt[0], served);
     if (left) atomicAdd(&cnt[1], left);
+  }
+}
+
+// Refill (rounds >= 2, out of core): one warp per listed frontier entry whose cached keys are all
+// matched.  The warp reads the host row zero-copy once, keeps the K largest AVAILABLE keys
+// (per-lane top-K, then K warp pops) and writes them back as the row's cache: every key of the
+// row above the K-th is unavailable now and stays so (R3), so the first available cached key is
+// again the row maximum over available neighbours in later rounds.  The entry is redirected to
+// the first refilled slot (or to an empty range when nothing is available).
+template <int K>
+__global__ void __launch_bounds__(256) k_host_rescan(Bins F, const uint64_t* __restrict__ rescan,
+                                                     const unsigned long long* __restrict__ nrescan,
+                                                     const int64_t* __restrict__ offs, AdjView adj,
+                                                     const uint32_t* __restrict__ bits,
+                                                     uint64_t* __restrict__ cache, int64_t u_first,
+                                                     int64_t M0, int64_t vbase) {
+  const int lane = threadIdx.x & 31;
+  const int64_t c = (int64_t)*nrescan;
+  const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t w = wid; w < c; w += nw) {
+    const uint64_t r = rescan[w];
+    const int bb = (int)(r >> 40);
+    const int64_t i = (int64_t)(r & ((1ull << 40) - 1));
+    const ulonglong2 e = F.list[bb][i];
+    const int64_t u = (int64_t)(uint32_t)e.x - vbase;
+    int64_t s, en;
+    row_range(e, offs, vbase, &s, &en);
+    uint64_t t[K];
+#pragma unroll
+    for (int q = 0; q < K; ++q) t[q] = 0ull;
+    for (int64_t j = s + lane; j < en; j += 32) {
+      const uint64_t k = adj.at(j);
+      if (k && !bit_test(bits, (uint32_t)k)) topk_insert<K>(t, k);
+    }
+    const uint64_t mine = warp_topk_pop<K>(t);
+    const int64_t slot = (u - u_first) * K;
+    if (lane < K) cache[slot + lane] = mine;
+    const uint64_t top = __shfl_sync(0xffffffffu, mine, 0);
+    if (lane == 0)
+      F.list[bb][i].y = top ? ((1ull << 40) | (uint64_t)(M0 + slot)) : (uint64_t)(M0 + slot);
   }
 }
 

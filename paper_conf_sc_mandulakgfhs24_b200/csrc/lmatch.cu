@@ -106,6 +106,9 @@ constexpr int64_t kHandoffRounds = 32;  // hybrid (algorithm 2): LD pointing pha
 #define LM_B1_G 16
 #define LM_B1_U 4
 #endif
+#ifndef LM_CACHE_REFILL
+#define LM_CACHE_REFILL 1  // out of core: refill a host row's cache when its cached keys run dry
+#endif
 #ifndef LM_BIN_STREAMS
 #define LM_BIN_STREAMS 1  // frontier bins of a round on concurrent side streams (R-MAT s26 rounds 7.64 -> 7.50 ms)
 #endif
@@ -224,6 +227,9 @@ struct lmatch_graph {
   int64_t u_first = 0, M0 = 0, nchunks = 0;
   int64_t* chunk_rows = nullptr;     // device [nchunks + 1]: row holding each chunk's first entry
   int64_t cap_chunk_rows = -1;
+  uint64_t* rescan = nullptr;        // device [n_hrows]: frontier entries whose cache ran dry
+  unsigned long long* rescan_cnt = nullptr;
+  int64_t cap_rescan = -1;
   int64_t* cache_big = nullptr;      // device [1 + cap]: count, then rows listed for the CTA fill
   int64_t cap_cache_big = -1;
   bool use_cache() const { return streaming && cache != nullptr; }
@@ -658,6 +664,8 @@ int build_cache_index(lmatch_graph* g, cudaStream_t st) {
   CK(cudaStreamSynchronize(st));
   g->u_first = uf;
   TRY(ensure(g, &g->cache, &g->cap_cache, (g->n - uf) * lm::kCacheK));
+  TRY(ensure(g, &g->rescan, &g->cap_rescan, g->n - uf + 1));
+  if (!g->rescan_cnt) TRY(dmalloc(g, &g->rescan_cnt, 1));
   // a window holds at most (entries / kCacheBigRow) rows longer than kCacheBigRow
   TRY(ensure(g, &g->cache_big, &g->cap_cache_big, std::max(C, g->R) / lm::kCacheBigRow + 8));
   g->M0 = g->m + 64;  // past the host part and its padding
@@ -909,7 +917,7 @@ void lmatch_destroy(lmatch_graph* g) {
   for (void* p : g->ipc_opened) cudaIpcCloseMemHandle(p);
   if (g->h_nf) cudaFreeHost(g->h_nf);
   void* pdev[] = {g->bounds, g->ghost, g->claims, g->claim_cnt, g->rstate, g->rlog, g->d_rargs,
-                  g->cache, g->chunk_rows, g->cache_big, g->live, g->win, g->suitor, g->wl[0],
+                  g->cache, g->chunk_rows, g->cache_big, g->rescan, g->rescan_cnt, g->live, g->win, g->suitor, g->wl[0],
                   g->wl[1], g->wl_big, g->wl_cnt, g->shadow, g->d_dseg, g->d_dcnt,
                   g->d_dbits, g->d_dnf};
   for (void* p : pdev) if (p) cudaFree(p);
@@ -1070,10 +1078,20 @@ static int seq_body(lmatch_graph* g, cudaStream_t st, int cur, const int64_t* nF
   int64_t nF = 0;
   for (int b = 0; b < lm::kBins; ++b) nF += nFb[b];
   if (g->use_cache() && nF > 0) {
+    const bool refill = LM_CACHE_REFILL != 0;
+    if (refill) CK(cudaMemsetAsync(g->rescan_cnt, 0, 8, st));
     lm::k_cache_redirect<lm::kCacheK><<<grid_for(nF, 256, 65536), 256, 0, st>>>(
-        Fb, cF, g->offs, g->cache, g->bits, g->u_first, g->M0, g->v0, g->counters + lm::kCntCache);
+        Fb, cF, g->offs, g->cache, g->bits, g->u_first, g->M0, g->v0, g->counters + lm::kCntCache,
+        refill ? g->rescan : nullptr, refill ? g->rescan_cnt : nullptr);
     CKL();
     ++*launches;
+    if (refill) {
+      lm::k_host_rescan<lm::kCacheK><<<(unsigned)(8 * g->num_sms), 256, 0, st>>>(
+          Fb, g->rescan, g->rescan_cnt, g->offs, g->view(), g->bits, g->cache, g->u_first, g->M0,
+          g->v0);
+      CKL();
+      ++*launches;
+    }
   }
 #define PIPE_OR_BIN(b, PG, PU, BG, BU, AG, AU)                                                      \
   if (nFb[b]) {                                                                                   \

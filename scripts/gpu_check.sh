@@ -1,7 +1,7 @@
 mkdir -p gpurun_out
-bash scripts/profile_round.sh r01g > gpurun_out/profile_r01g.log 2>&1
-rm -f gpurun_out/other_g.jsonl
-for wl in "--scale 24" "--workload er" "--workload mesh" "--workload road" "--workload gradient --scale 20" "--workload gradient --scale 20 --algorithm hybrid" "--scale 28"; do
-  timeout 600 python bench.py --no-cpu --no-e2e --steps 5 $wl 2>/dev/null | grep '^{' >> gpurun_out/other_g.jsonl
+timeout 900 python -m pytest tests/test_gpu_parity.py -x -q -k "out_of_core or batches" 2>&1 | tail -2
+for v in base norefill; do
+  for c in "--hbm-budget-gb 6" "--batches 3"; do
+    LMATCH_LIB=$PWD/build/variants/lm_$v.so python bench.py --no-cpu --no-e2e --steps 3 $c 2>/dev/null | grep '^{' | python -c "import json,sys; d=json.loads(sys.stdin.read()); o=d['out_of_core']; print('$v', '$c', round(d['value'],3), round(d['ms_per_step'],1), {k: round(x,1) for k,x in d['phase_ms'].items()}, o['host_entries_read_per_step'])"
+  done
 done
-ls gpurun_out | head -50
