@@ -127,7 +127,15 @@ typedef struct lmatch_opts {
                                  the graph without the vertices matched so far completes the same
                                  matching (lmatch_stats.tail_passes).  1 and 2: resident
                                  single-graph handles only (1: EINVAL with out-of-core /
-                                 partition handles; 2 behaves as 0 there) */
+                                 partition handles; 2 behaves as 0 there).
+                                 3 = sorted adjacency + cursor: the first run
+                                 after create/reload sorts every row by key, descending, in place
+                                 (the row's entries are permuted, never changed; this time is
+                                 lmatch_stats.ms_sort), then each vertex's pointer is the first
+                                 entry at or after its cursor whose neighbour is unmatched (Alg. 1
+                                 L4).  Same unique result under R1.  Resident single-graph
+                                 handles only (EINVAL otherwise).  The sort needs min(m, 2^30) x 8 B
+                                 of scratch device memory, freed before the run */
   int32_t reserved[7];
 } lmatch_opts;
 
@@ -158,7 +166,9 @@ typedef struct lmatch_stats {
   int64_t cache_bytes;       /* out-of-core: device bytes of the host-row cache (0 = none) */
   int64_t tail_passes;       /* algorithm 2: Suitor passes that completed the run after the LD
                                 iteration stopped at 32 pointing phases (0 = not needed) */
-  int64_t reserved[2];
+  double ms_sort;            /* algorithm 3: device time of the row sort this run performed (the
+                                first run after create/reload); 0 when the rows were already sorted */
+  int64_t reserved[1];
 } lmatch_stats;
 
 /* Library / ABI identification.  Returns LMATCH_ABI_VERSION. */

@@ -61,7 +61,7 @@ class Stats(ctypes.Structure):
         ("kernel_launches", ctypes.c_int64), ("bytes_streamed", ctypes.c_int64),
         ("resident_entries", ctypes.c_int64), ("cache_rows", ctypes.c_int64),
         ("host_entries_read", ctypes.c_int64), ("cache_bytes", ctypes.c_int64),
-        ("tail_passes", ctypes.c_int64), ("reserved", ctypes.c_int64 * 2),
+        ("tail_passes", ctypes.c_int64), ("ms_sort", ctypes.c_double), ("reserved", ctypes.c_int64 * 1),
     ]
 
     def as_dict(self) -> dict:
@@ -309,7 +309,7 @@ def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int =
     o.prune = int(bool(prune))
     o.host_cache = 0 if host_cache else -1
     o.batches = int(batches)
-    o.algorithm = {"ld": 0, "suitor": 1, "hybrid": 2}[algorithm]
+    o.algorithm = {"ld": 0, "suitor": 1, "hybrid": 2, "sorted": 3}[algorithm]
     o.hbm_budget_bytes = int(hbm_budget_bytes)
     o.stream_chunk = int(stream_chunk)
     o.validate_level = int(validate_level)

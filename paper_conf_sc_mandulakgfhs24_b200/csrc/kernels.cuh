@@ -2677,4 +2677,85 @@ __global__ void __launch_bounds__(THREADS)
   block_sum2<THREADS>(w, c, &pw[blockIdx.x], &pc[blockIdx.x]);
 }
 
+
+// =============================================================================================
+// Sorted adjacency + cursor (algorithm 3).  Every row is sorted once by key,
+// descending (the R1 order: weight bits, then neighbour id), so self-loop keys (0) sit at the row
+// end.  u's pointer (Alg. 1 L4: the heaviest available neighbour) is then the first entry at
+// or after cur[u] whose neighbour is unmatched; matched is permanent, so cur[u] only moves forward
+// and the whole run reads each entry at most once (plus one re-check per live vertex per round).
+// =============================================================================================
+// row-relative int32 segment offsets of rows [r0, r1] for the segmented sort of one chunk
+__global__ void k_sc_seg_offsets(const int64_t* __restrict__ offs, int64_t r0, int64_t r1,
+                                 int32_t* __restrict__ seg) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t base = offs[r0];
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i <= r1 - r0; i += stride)
+    seg[i] = (int32_t)(offs[r0 + i] - base);
+}
+
+// SETPOINTERS with cursors: for u in the live list L (or every vertex when L == nullptr, round 1)
+// whose pointer target is matched (only those change: Alg. 3's frontier) advance cur[u]
+// past matched neighbours; ptr[u] = the key there, or 0 when the row ran dry.
+// One thread per vertex; `reads` counts adjacency entries loaded.
+__global__ void k_sc_point(const uint32_t* __restrict__ L, const unsigned long long* __restrict__ nL,
+                           int64_t n_all, const int64_t* __restrict__ offs,
+                           const uint64_t* __restrict__ adj, int64_t* __restrict__ cur,
+                           const uint32_t* __restrict__ bits, uint64_t* __restrict__ ptr,
+                           unsigned long long* reads) {
+  const int64_t cnt = L ? (int64_t)*nL : n_all;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  unsigned long long r = 0;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += stride) {
+    const uint32_t u = L ? L[i] : (uint32_t)i;
+    int64_t j;
+    if (L) {  // a live u points at an unmatched v: keep it unless v was matched last round
+      if (!bit_test(bits, (uint32_t)ptr[u])) continue;
+      j = cur[u] + 1;
+    } else {
+      j = offs[u];
+    }
+    const int64_t e = offs[u + 1];
+    uint64_t k = 0;
+    for (; j < e; ++j) {
+      k = __ldg(adj + j);
+      ++r;
+      if (k == 0ull || !bit_test(bits, (uint32_t)k)) break;
+    }
+    if (j >= e) k = 0ull;
+    cur[u] = j;
+    ptr[u] = k;
+  }
+  for (int o = 16; o; o >>= 1) r += __shfl_xor_sync(0xffffffffu, r, o);
+  if ((threadIdx.x & 31) == 0 && r) atomicAdd(reads, r);
+}
+
+// SETMATES (Alg. 1 L6-9): u with ptr[ptr[u]] == u is matched (mate key stored, bit set); a live
+// u that is not matched stays in the next list; u with no available neighbour leaves for good.
+__global__ void k_sc_match(const uint32_t* __restrict__ L, const unsigned long long* __restrict__ nL,
+                           int64_t n_all, const uint64_t* __restrict__ ptr, uint32_t* bits,
+                           uint64_t* __restrict__ matek, uint32_t* __restrict__ next,
+                           unsigned long long* ncnt) {
+  const int64_t cnt = L ? (int64_t)*nL : n_all;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t c32 = (cnt + 31) & ~31ll;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < c32; i += stride) {
+    uint32_t keep = kNoPtr;
+    if (i < cnt) {
+      const uint32_t u = L ? L[i] : (uint32_t)i;
+      const uint64_t k = ptr[u];
+      if (k) {
+        const uint32_t v = (uint32_t)k;
+        if ((uint32_t)__ldg(ptr + v) == u && __ldg(ptr + v) != 0ull) {
+          matek[u] = k;
+          atomicOr(bits + (u >> 5), 1u << (u & 31));
+        } else {
+          keep = u;
+        }
+      }
+    }
+    suitor_push(keep, next, ncnt);
+  }
+}
+
 }  // namespace lm

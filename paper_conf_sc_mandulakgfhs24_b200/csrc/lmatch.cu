@@ -24,6 +24,8 @@
 #include "../../include/lmatch.h"
 #include "kernels.cuh"
 
+#include <cub/device/device_segmented_sort.cuh>
+
 
 namespace {
 
@@ -209,7 +211,11 @@ struct lmatch_graph {
   int64_t stream_chunk = 1ll << 24;
   int64_t hbm_budget = 0;
   int batches = 0;                   // paper-style batch count (> 1: all streamed)
-  int algorithm = 0;                 // 0 = LD pointer iteration, 1 = Suitor (NEXT-4)
+  int algorithm = 0;                 // 0 = LD pointer iteration, 1 = Suitor (NEXT-4), 3 = sorted+cursor
+  bool sorted = false;               // algorithm 3: rows sorted by key, descending (NEXT-3)
+  float ms_sort = 0.f;               // algorithm 3: device time of the last row sort
+  int64_t* sc_cur = nullptr;         // algorithm 3: per-vertex cursor (absolute entry index)
+  uint64_t* sc_ptr = nullptr;        // algorithm 3: per-vertex pointer key (0 = none)
   uint64_t* suitor = nullptr;        // Suitor: best proposal received, (w << 32) | proposer
   uint32_t* wl[2] = {nullptr, nullptr};   // Suitor worklists
   uint32_t* wl_big = nullptr;             // Suitor: rows listed for the CTA scan
@@ -696,6 +702,7 @@ int finish_create(lmatch_graph* g, cudaStream_t st) {
     TRY(dmalloc(g, &g->live, (size_t)g->n + 1));
     CK(cudaMemsetAsync(g->live, 0, ((size_t)g->n + 1) * 4, st));
   }
+  g->sorted = false;  // (re)loaded adjacency: algorithm 3 sorts it again on the next run
   TRY(build_index(g, st));
   TRY(alloc_bins(g, st));
   TRY(build_cache_index(g, st));
@@ -918,7 +925,7 @@ void lmatch_destroy(lmatch_graph* g) {
   if (g->h_nf) cudaFreeHost(g->h_nf);
   void* pdev[] = {g->bounds, g->ghost, g->claims, g->claim_cnt, g->rstate, g->rlog, g->d_rargs,
                   g->cache, g->chunk_rows, g->cache_big, g->rescan, g->rescan_cnt, g->live, g->win, g->suitor, g->wl[0],
-                  g->wl[1], g->wl_big, g->wl_cnt, g->shadow, g->d_dseg, g->d_dcnt,
+                  g->wl[1], g->wl_big, g->wl_cnt, g->sc_cur, g->sc_ptr, g->shadow, g->d_dseg, g->d_dcnt,
                   g->d_dbits, g->d_dnf};
   for (void* p : pdev) if (p) cudaFree(p);
   if (g->h_claim_cnt) cudaFreeHost(g->h_claim_cnt);
@@ -1335,6 +1342,189 @@ static int run_suitor(lmatch_graph* g, int32_t* d_mate, cudaStream_t st, lmatch_
   return LMATCH_OK;
 }
 
+
+// ---- algorithm 3 (NEXT-3): sort every row by key, descending, in place.  Rows are grouped into
+// chunks of at most kSortChunk entries (cub's segmented sort takes int sizes), each sorted into a
+// scratch buffer and copied back.  Done once per loaded graph; the time goes to lmatch_stats.ms_sort.
+constexpr int64_t kSortChunk = 1ll << 30;
+
+static int64_t host_off(lmatch_graph* g, int64_t r, cudaStream_t st, int* err) {
+  int64_t v = 0;
+  if (cudaMemcpyAsync(&v, g->offs + r, 8, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+      cudaStreamSynchronize(st) != cudaSuccess) *err = 1;
+  return v;
+}
+
+static int sort_rows(lmatch_graph* g, cudaStream_t st) {
+  const int64_t n = g->n, m = g->m;
+  CK(cudaEventRecord(g->ev[6], st));
+  if (m > 0 && n > 0) {
+    int err = 0;
+    const int64_t cap = std::min<int64_t>(m, kSortChunk);
+    uint64_t* alt = nullptr;
+    int32_t* seg = nullptr;
+    void* tmp = nullptr;
+    size_t tmp_bytes = 0, need = 0;
+    CK(cudaMalloc(&alt, (size_t)cap * 8));
+    int rc = LMATCH_OK;
+    int64_t r0 = 0;
+    std::vector<int64_t> cuts;
+    while (r0 < n && rc == LMATCH_OK) {  // rows [r0, r1): the longest run of rows within cap entries
+      const int64_t b0 = host_off(g, r0, st, &err);
+      int64_t lo = r0 + 1, hi = n;  // largest r1 with offs[r1] - b0 <= cap (at least one row)
+      if (host_off(g, n, st, &err) - b0 <= cap) lo = n;
+      else {
+        while (lo < hi) {
+          const int64_t mid = lo + (hi - lo + 1) / 2;
+          if (host_off(g, mid, st, &err) - b0 <= cap) lo = mid; else hi = mid - 1;
+        }
+      }
+      if (err) { set_err("offset read failed"); rc = LMATCH_ECUDA; break; }
+      const int64_t r1 = lo, cnt = host_off(g, r1, st, &err) - b0;
+      if (cnt > INT_MAX) { set_err("row %lld has more than 2^31-1 entries", (long long)r0); rc = LMATCH_EINVAL; break; }
+      cuts.push_back(r0);
+      r0 = r1;
+    }
+    cuts.push_back(n);
+    int64_t maxrows = 0;
+    for (size_t c = 0; c + 1 < cuts.size(); ++c) maxrows = std::max(maxrows, cuts[c + 1] - cuts[c]);
+    if (rc == LMATCH_OK && cudaMalloc(&seg, (size_t)(maxrows + 1) * 4) != cudaSuccess) {
+      set_err("cudaMalloc(segment offsets) failed"); rc = LMATCH_ENOMEM;
+    }
+    for (size_t c = 0; rc == LMATCH_OK && c + 1 < cuts.size(); ++c) {
+      const int64_t a = cuts[c], b = cuts[c + 1];
+      const int64_t base = host_off(g, a, st, &err), cnt = host_off(g, b, st, &err) - base;
+      if (cnt == 0) continue;
+      lm::k_sc_seg_offsets<<<grid_for(b - a + 1, 256, 65536), 256, 0, st>>>(g->offs, a, b, seg);
+      if (cudaGetLastError() != cudaSuccess) { rc = LMATCH_ECUDA; break; }
+      if (cub::DeviceSegmentedSort::SortKeysDescending(nullptr, need, g->adj + base, alt, (int)cnt,
+                                                       (int)(b - a), seg, seg + 1, st) != cudaSuccess) {
+        set_err("segmented sort sizing failed"); rc = LMATCH_ECUDA; break;
+      }
+      if (need > tmp_bytes) {
+        if (tmp) cudaFree(tmp);
+        tmp = nullptr;
+        if (cudaMalloc(&tmp, need) != cudaSuccess) { set_err("cudaMalloc(sort temp) failed"); rc = LMATCH_ENOMEM; break; }
+        tmp_bytes = need;
+      }
+      if (cub::DeviceSegmentedSort::SortKeysDescending(tmp, need, g->adj + base, alt, (int)cnt,
+                                                       (int)(b - a), seg, seg + 1, st) != cudaSuccess ||
+          cudaMemcpyAsync(g->adj + base, alt, (size_t)cnt * 8, cudaMemcpyDeviceToDevice, st) != cudaSuccess) {
+        set_err("segmented sort failed"); rc = LMATCH_ECUDA; break;
+      }
+    }
+    cudaStreamSynchronize(st);
+    if (tmp) cudaFree(tmp);
+    if (seg) cudaFree(seg);
+    cudaFree(alt);
+    if (rc != LMATCH_OK) return rc;
+  }
+  CK(cudaEventRecord(g->ev[7], st));
+  CK(cudaEventSynchronize(g->ev[7]));
+  CK(cudaEventElapsedTime(&g->ms_sort, g->ev[6], g->ev[7]));
+  g->sorted = true;
+  return LMATCH_OK;
+}
+
+// algorithm 3: round 1 points every vertex at its first available entry, then host-driven rounds
+// over the live list (point, match) until it is empty; mate[] and w(M) as for Suitor.
+static int run_sorted(lmatch_graph* g, int32_t* d_mate, cudaStream_t st, lmatch_stats* stats) {
+  const int64_t n = g->n;
+  const bool tm = g->timing && stats;
+  bool sorted_now = false;
+  if (!g->sorted) { TRY(sort_rows(g, st)); sorted_now = true; }
+  TRY(ensure_suitor(g));
+  if (!g->sc_cur) {
+    TRY(dmalloc(g, &g->sc_cur, (size_t)n + 1));
+    TRY(dmalloc(g, &g->sc_ptr, (size_t)n + 1));
+  }
+  int64_t launches = 0, rounds = 0;
+  unsigned long long* hc = g->h_counters;
+  if (tm) CK(cudaEventRecord(g->ev[0], st));
+  CK(cudaMemsetAsync(g->suitor, 0, ((size_t)n + 1) * 8, st));
+  CK(cudaMemsetAsync(g->bits, 0, (size_t)((n + 31) / 32) * 4, st));
+  CK(cudaMemsetAsync(g->wl_cnt, 0, 4 * 8, st));
+  if (tm) CK(cudaEventRecord(g->ev[1], st));
+  int cur = 0;
+  const bool work = g->ntiles > 0 && n > 0;
+  if (work) {
+    lm::k_sc_point<<<grid_for(n, 256, 65536), 256, 0, st>>>(nullptr, nullptr, n, g->offs, g->adj,
+                                                             g->sc_cur, g->bits, g->sc_ptr, g->wl_cnt + 2);
+    CKL();
+    if (tm) CK(cudaEventRecord(g->ev[2], st));
+    lm::k_sc_match<<<grid_for(n, 256, 65536), 256, 0, st>>>(nullptr, nullptr, n, g->sc_ptr, g->bits,
+                                                             g->suitor, g->wl[0], g->wl_cnt + 0);
+    CKL();
+    launches += 2;
+    rounds = 1;
+  } else if (tm) {
+    CK(cudaEventRecord(g->ev[2], st));
+  }
+  if (tm) CK(cudaEventRecord(g->ev[3], st));
+  for (;;) {
+    if (!work) break;
+    CK(cudaMemcpyAsync(hc, g->wl_cnt, 4 * 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    const int64_t c = (int64_t)hc[cur];
+    if (c == 0) break;
+    if (rounds >= g->max_rounds) { set_err("sorted LD did not converge in %lld rounds", (long long)rounds); return LMATCH_ECUDA; }
+    CK(cudaMemsetAsync(g->wl_cnt + (cur ^ 1), 0, 8, st));
+    lm::k_sc_point<<<grid_for(c, 256, 65536), 256, 0, st>>>(g->wl[cur], g->wl_cnt + cur, 0, g->offs,
+                                                             g->adj, g->sc_cur, g->bits, g->sc_ptr,
+                                                             g->wl_cnt + 2);
+    CKL();
+    lm::k_sc_match<<<grid_for(c, 256, 65536), 256, 0, st>>>(g->wl[cur], g->wl_cnt + cur, 0, g->sc_ptr,
+                                                             g->bits, g->suitor, g->wl[cur ^ 1],
+                                                             g->wl_cnt + (cur ^ 1));
+    CKL();
+    launches += 2;
+    ++rounds;
+    cur ^= 1;
+  }
+  if (tm) CK(cudaEventRecord(g->ev[4], st));
+  if (n > 0) {
+    lm::k_suitor_finish<kFinThreads><<<kFinBlocks, kFinThreads, 0, st>>>(g->suitor, n, d_mate, g->pw, g->pc);
+    CKL();
+    lm::k_final_sum<<<1, 32, 0, st>>>(g->pw, g->pc, kFinBlocks, g->res_w, g->res_c);
+    CKL();
+    launches += 2;
+    CK(cudaMemcpyAsync(g->h_res, g->res_w, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(g->h_resc, g->res_c, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(hc, g->wl_cnt, 4 * 8, cudaMemcpyDeviceToHost, st));
+  } else {
+    g->h_res[0] = 0.0;
+    g->h_resc[0] = 0;
+  }
+  if (tm) CK(cudaEventRecord(g->ev[5], st));
+  CK(cudaStreamSynchronize(st));
+  g->round_log.clear();
+  if (stats) {
+    std::memset(stats, 0, sizeof *stats);
+    stats->rounds = rounds;
+    stats->matched_vertices = g->h_resc[0];
+    stats->cardinality = g->h_resc[0] / 2;
+    stats->weight = g->h_res[0];
+    stats->entries_swept = work ? (int64_t)hc[2] : 0;
+    stats->kernel_launches = launches;
+    stats->resident_entries = g->R;
+    stats->ms_sort = sorted_now ? g->ms_sort : 0.0;
+    if (tm) {
+      float a = 0, b = 0, c = 0, d = 0, e = 0;
+      CK(cudaEventElapsedTime(&a, g->ev[0], g->ev[5]));
+      CK(cudaEventElapsedTime(&b, g->ev[1], g->ev[2]));
+      CK(cudaEventElapsedTime(&c, g->ev[2], g->ev[3]));
+      CK(cudaEventElapsedTime(&d, g->ev[3], g->ev[4]));
+      CK(cudaEventElapsedTime(&e, g->ev[4], g->ev[5]));
+      stats->ms_total = a;
+      stats->ms_sweep = b;
+      stats->ms_round1_rest = c;
+      stats->ms_rounds = d;
+      stats->ms_finish = e;
+    }
+  }
+  return LMATCH_OK;
+}
+
 int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_stats* stats) {
   if (!g) { set_err("NULL handle"); return LMATCH_ESTATE; }
   if (g->algorithm == 1) {
@@ -1343,6 +1533,13 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
     g_err[0] = 0;
     CK(cudaSetDevice(g->device));
     return run_suitor(g, d_mate, stream ? (cudaStream_t)stream : g->stream, stats);
+  }
+  if (g->algorithm == 3) {
+    if (!d_mate && g->n > 0) { set_err("d_mate == NULL"); return LMATCH_EINVAL; }
+    if (g->ghost || g->streaming) { set_err("sorted LD: resident single-graph handles only"); return LMATCH_EINVAL; }
+    g_err[0] = 0;
+    CK(cudaSetDevice(g->device));
+    return run_sorted(g, d_mate, stream ? (cudaStream_t)stream : g->stream, stats);
   }
   if (!d_mate && g->n > 0) { set_err("d_mate == NULL"); return LMATCH_EINVAL; }
   if (g->ghost) { set_err("partition handle: use the lmatch_part_* calls"); return LMATCH_ESTATE; }

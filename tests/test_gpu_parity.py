@@ -616,3 +616,74 @@ def test_hybrid_tail(lm, round_loop):
     for g in (graphgen.rmat(16, 16, seed=1), graphgen.mesh(200, seed=3)):
         mate, st = check_parity(lm, g, algorithm="hybrid", round_loop=round_loop)
         assert st["tail_passes"] == 0
+
+
+# ---------------------------------------------------------- NEXT-3: sorted adjacency + cursor
+def check_sorted(lm, g, rounds=True):
+    """algorithm 3 computes Alg. 1's pointers (heaviest unmatched neighbour, R1 order) from rows
+    sorted once by key, so mate[] is bit-exact and the pointing-phase count is Alg. 1's."""
+    return check_parity(lm, g, rounds=rounds, algorithm="sorted")
+
+
+@pytest.mark.parametrize("name", golden_names())
+def test_sorted_golden(lm, name):
+    g, mate, _, weight = load_golden(name)
+    got, st = run_gpu(lm, g, algorithm="sorted")
+    np.testing.assert_array_equal(got, mate)
+    assert math.isclose(st["weight"], weight, rel_tol=1e-12)
+
+
+def test_sorted_random_tiny_and_paths(lm):
+    rng = np.random.default_rng(29)
+    for _ in range(60):
+        n = int(rng.integers(2, 40))
+        g = graphgen.random_small(n, float(rng.choice([.1, .3, .7])), rng,
+                                  levels=int(rng.choice([0, 2, 5])) or None)
+        check_sorted(lm, g)
+    for n in (2, 3, 17, 301):
+        check_sorted(lm, graphgen.from_edges(n, [(i, i + 1, float(i + 1)) for i in range(n - 1)]))
+    check_sorted(lm, graphgen.from_edges(7, []))
+    # self-loops (zero keys after ingest) sort to the row end and are never pointed at
+    check_sorted(lm, graphgen.from_edges(4, [(0, 0, 9.0), (0, 1, 1.0), (1, 1, 5.0), (2, 3, 2.0)]))
+
+
+@pytest.mark.parametrize("maker", [
+    lambda: graphgen.er(1 << 16, 16.0, seed=1),
+    lambda: graphgen.er(5000, 30.0, seed=3, weights="ones"),
+    lambda: graphgen.rmat(16, 16, seed=1),
+    lambda: graphgen.rmat(15, 16, seed=4, weights="paper"),
+    lambda: graphgen.mesh(256, seed=1),
+    lambda: graphgen.mesh(300, keep=0.6, seed=1),
+    lambda: graphgen.mesh(128, seed=1, weights="gradient"),
+    lambda: _hub_graph(4),
+    lambda: _loopy_graph(38),
+])
+def test_sorted_synthetic(lm, maker):
+    check_sorted(lm, maker())
+
+
+def test_sorted_repeat_reload_weight_and_rmat24(lm):
+    """The sort runs once per loaded graph (ms_sort > 0 on the first run only, again after a
+    reload); lmatch_weight still reads the permuted rows correctly; configs[1] at full size
+    against the O(m) certificate and the LD path's result."""
+    g = graphgen.rmat(14, 16, seed=21)
+    g2 = graphgen.rmat(14, 16, seed=21, weights="paper")
+    with lm.Matcher(g, algorithm="sorted", timing=1) as M:
+        a, sa = M.run()
+        b, sb = M.run()
+        np.testing.assert_array_equal(a, b)
+        np.testing.assert_array_equal(a, oracle.greedy(g).mate)
+        assert sa["ms_sort"] > 0 and sb["ms_sort"] == 0
+        assert math.isclose(M.weight(a), oracle.weight(g, a), rel_tol=WTOL)
+        M.reload(g2.offsets, g2.col, g2.w)
+        c, sc = M.run()
+        assert sc["ms_sort"] > 0
+        np.testing.assert_array_equal(c, oracle.greedy(g2).mate)
+    g = graphgen.rmat(24, 16, seed=1)
+    mate, st = run_gpu(lm, g, algorithm="sorted")
+    code, bad = oracle.certificate(g, mate)
+    assert code == 0, (code, bad)
+    ref, sref = run_gpu(lm, g)
+    np.testing.assert_array_equal(mate, ref)
+    assert st["rounds"] == sref["rounds"]
+    assert st["entries_swept"] < sref["entries_swept"]
