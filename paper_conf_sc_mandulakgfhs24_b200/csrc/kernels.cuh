@@ -2694,67 +2694,168 @@ __global__ void k_sc_seg_offsets(const int64_t* __restrict__ offs, int64_t r0, i
     seg[i] = (int32_t)(offs[r0 + i] - base);
 }
 
-// SETPOINTERS with cursors: for u in the live list L (or every vertex when L == nullptr, round 1)
-// whose pointer target is matched (only those change: Alg. 3's frontier) advance cur[u]
-// past matched neighbours; ptr[u] = the key there, or 0 when the row ran dry.
-// One thread per vertex; `reads` counts adjacency entries loaded.
-__global__ void k_sc_point(const uint32_t* __restrict__ L, const unsigned long long* __restrict__ nL,
+// SETPOINTERS with cursors.  Round 1 (L == nullptr): every vertex points at its row's first key
+// (nothing is matched yet; a 0 key = self-loops only or an empty row).  Rounds >= 2: the live list
+// holds (u, current pointer key) pairs; only u whose target was matched last round change (Alg. 3's
+// frontier): cur[u] (row-relative, 0 after round 1) moves past matched neighbours and the
+// pair and ptr[u] get the new key (0 when the row ran dry).  A thread walks at most kScSerial
+// entries; rows that need more go to the `big` list (list index) for k_sc_point_warp.
+// `reads` counts adjacency entries read.
+constexpr int kScSerial = 8;
+__global__ void k_sc_point(ulonglong2* __restrict__ L, const unsigned long long* __restrict__ nL,
                            int64_t n_all, const int64_t* __restrict__ offs,
-                           const uint64_t* __restrict__ adj, int64_t* __restrict__ cur,
+                           const uint64_t* __restrict__ adj, uint32_t* __restrict__ cur,
                            const uint32_t* __restrict__ bits, uint64_t* __restrict__ ptr,
+                           uint32_t* __restrict__ big, unsigned long long* nbig,
                            unsigned long long* reads) {
   const int64_t cnt = L ? (int64_t)*nL : n_all;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   unsigned long long r = 0;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += stride) {
-    const uint32_t u = L ? L[i] : (uint32_t)i;
-    int64_t j;
-    if (L) {  // a live u points at an unmatched v: keep it unless v was matched last round
-      if (!bit_test(bits, (uint32_t)ptr[u])) continue;
-      j = cur[u] + 1;
-    } else {
-      j = offs[u];
+    if (!L) {
+      const int64_t a = offs[i];
+      uint64_t k = 0;
+      if (a < offs[i + 1]) { k = __ldg(adj + a); ++r; }
+      ptr[i] = k;
+      continue;
     }
-    const int64_t e = offs[u + 1];
+    ulonglong2 p = L[i];
+    if (!bit_test(bits, (uint32_t)p.y)) continue;  // target still unmatched: pointer unchanged
+    const uint32_t u = (uint32_t)p.x;
+    const int64_t a = offs[u], e = offs[u + 1];
+    int64_t j = a + cur[u] + 1;
+    const int64_t stop = j + kScSerial < e ? j + kScSerial : e;
     uint64_t k = 0;
-    for (; j < e; ++j) {
+    bool found = false;
+    for (; j < stop; ++j) {
       k = __ldg(adj + j);
       ++r;
-      if (k == 0ull || !bit_test(bits, (uint32_t)k)) break;
+      if (k == 0ull) { j = e; break; }
+      if (!bit_test(bits, (uint32_t)k)) { found = true; break; }
     }
-    if (j >= e) k = 0ull;
-    cur[u] = j;
+    cur[u] = (uint32_t)(j - a);
+    if (!found && j < e) {  // long skip: hand the row to a warp
+      big[atomicAdd(nbig, 1ull)] = (uint32_t)i;
+      continue;
+    }
+    if (!found) k = 0ull;
     ptr[u] = k;
+    p.y = k;
+    L[i] = p;
   }
   for (int o = 16; o; o >>= 1) r += __shfl_xor_sync(0xffffffffu, r, o);
   if ((threadIdx.x & 31) == 0 && r) atomicAdd(reads, r);
 }
 
+// the long skips: one warp per listed row scans 32 entries per step from cur[u] and takes the
+// first (lowest-index, i.e. heaviest) available key
+__global__ void k_sc_point_warp(ulonglong2* __restrict__ L, const uint32_t* __restrict__ big,
+                                const unsigned long long* __restrict__ nbig,
+                                const int64_t* __restrict__ offs, const uint64_t* __restrict__ adj,
+                                uint32_t* __restrict__ cur, const uint32_t* __restrict__ bits,
+                                uint64_t* __restrict__ ptr, unsigned long long* reads) {
+  const int lane = threadIdx.x & 31;
+  const int64_t w0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t ws = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const int64_t cnt = (int64_t)*nbig;
+  unsigned long long r = 0;
+  for (int64_t w = w0; w < cnt; w += ws) {
+    const uint32_t i = big[w];
+    ulonglong2 p = L[i];
+    const uint32_t u = (uint32_t)p.x;
+    const int64_t a = offs[u], e = offs[u + 1];
+    uint64_t k = 0;
+    int64_t j = a + cur[u];
+    for (; j < e; j += 32) {
+      const int64_t jj = j + lane;
+      const uint64_t kk = jj < e ? __ldg(adj + jj) : 0ull;
+      r += jj < e;
+      const bool ok = kk != 0ull && !bit_test(bits, (uint32_t)kk);
+      const unsigned zb = __ballot_sync(0xffffffffu, jj < e && kk == 0ull);
+      const unsigned ob = __ballot_sync(0xffffffffu, ok);
+      // keys are descending: a 0 key ends the row's available part
+      const unsigned first_zero = zb ? (unsigned)(__ffs(zb) - 1) : 32u;
+      if (ob && (unsigned)(__ffs(ob) - 1) < first_zero) {
+        const int src = __ffs(ob) - 1;
+        k = __shfl_sync(0xffffffffu, kk, src);
+        j += src;
+        break;
+      }
+      if (zb) { j = e; break; }
+    }
+    if (j >= e) { k = 0ull; j = e; }
+    if (lane == 0) {
+      cur[u] = (uint32_t)(j - a);
+      ptr[u] = k;
+      p.y = k;
+      L[i] = p;
+    }
+  }
+  for (int o = 16; o; o >>= 1) r += __shfl_xor_sync(0xffffffffu, r, o);
+  if (lane == 0 && r) atomicAdd(reads, r);
+}
+
 // SETMATES (Alg. 1 L6-9): u with ptr[ptr[u]] == u is matched (mate key stored, bit set); a live
-// u that is not matched stays in the next list; u with no available neighbour leaves for good.
-__global__ void k_sc_match(const uint32_t* __restrict__ L, const unsigned long long* __restrict__ nL,
-                           int64_t n_all, const uint64_t* __restrict__ ptr, uint32_t* bits,
-                           uint64_t* __restrict__ matek, uint32_t* __restrict__ next,
-                           unsigned long long* ncnt) {
+// u that is not matched goes to the next list with its pointer; u with no available neighbour
+// (key 0) leaves for good.  Round 1 (L == nullptr) reads the pairs (u, ptr[u]) for every u.
+// Each thread takes kScItems pairs per block step and the block reserves its output with one
+// atomicAdd (per-warp reservations on one counter serialised the kernel).
+constexpr int kScThreads = 256, kScItems = 4;
+__global__ void __launch_bounds__(kScThreads)
+    k_sc_match(const ulonglong2* __restrict__ L, const unsigned long long* __restrict__ nL,
+               int64_t n_all, const uint64_t* __restrict__ ptr, uint32_t* bits,
+               uint64_t* __restrict__ matek, ulonglong2* __restrict__ next,
+               unsigned long long* ncnt) {
+  __shared__ int s_warp[kScThreads / 32];
+  __shared__ unsigned long long s_base;
   const int64_t cnt = L ? (int64_t)*nL : n_all;
-  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  const int64_t c32 = (cnt + 31) & ~31ll;
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < c32; i += stride) {
-    uint32_t keep = kNoPtr;
-    if (i < cnt) {
-      const uint32_t u = L ? L[i] : (uint32_t)i;
-      const uint64_t k = ptr[u];
-      if (k) {
-        const uint32_t v = (uint32_t)k;
-        if ((uint32_t)__ldg(ptr + v) == u && __ldg(ptr + v) != 0ull) {
-          matek[u] = k;
-          atomicOr(bits + (u >> 5), 1u << (u & 31));
-        } else {
-          keep = u;
-        }
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  constexpr int64_t kStep = (int64_t)kScThreads * kScItems;
+  for (int64_t b0 = (int64_t)blockIdx.x * kStep; b0 < cnt; b0 += (int64_t)gridDim.x * kStep) {
+    ulonglong2 p[kScItems];
+    bool keep[kScItems];
+    int mine = 0;
+#pragma unroll
+    for (int t = 0; t < kScItems; ++t) {
+      const int64_t i = b0 + t * kScThreads + threadIdx.x;
+      keep[t] = false;
+      p[t] = make_ulonglong2(0ull, 0ull);
+      if (i < cnt) p[t] = L ? L[i] : make_ulonglong2((unsigned long long)i, ptr[i]);
+    }
+    uint64_t kv[kScItems];
+#pragma unroll
+    for (int t = 0; t < kScItems; ++t) kv[t] = p[t].y ? __ldg(ptr + (uint32_t)p[t].y) : 0ull;
+#pragma unroll
+    for (int t = 0; t < kScItems; ++t) {
+      if (!p[t].y) continue;
+      const uint32_t u = (uint32_t)p[t].x;
+      if ((uint32_t)kv[t] == u && kv[t] != 0ull) {
+        matek[u] = p[t].y;
+        atomicOr(bits + (u >> 5), 1u << (u & 31));
+      } else {
+        keep[t] = true;
+        ++mine;
       }
     }
-    suitor_push(keep, next, ncnt);
+    // block-wide exclusive scan of `mine`
+    int incl = mine;
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xffffffffu, incl, o);
+      if (lane >= o) incl += y;
+    }
+    if (lane == 31) s_warp[wid] = incl;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      int tot = 0;
+      for (int w = 0; w < kScThreads / 32; ++w) { const int c = s_warp[w]; s_warp[w] = tot; tot += c; }
+      s_base = tot ? atomicAdd(ncnt, (unsigned long long)tot) : 0ull;
+    }
+    __syncthreads();
+    unsigned long long o = s_base + s_warp[wid] + (incl - mine);
+#pragma unroll
+    for (int t = 0; t < kScItems; ++t)
+      if (keep[t]) next[o++] = p[t];
+    __syncthreads();
   }
 }
 

@@ -214,7 +214,8 @@ struct lmatch_graph {
   int algorithm = 0;                 // 0 = LD pointer iteration, 1 = Suitor (NEXT-4), 3 = sorted+cursor
   bool sorted = false;               // algorithm 3: rows sorted by key, descending (NEXT-3)
   float ms_sort = 0.f;               // algorithm 3: device time of the last row sort
-  int64_t* sc_cur = nullptr;         // algorithm 3: per-vertex cursor (absolute entry index)
+  uint32_t* sc_cur = nullptr;        // algorithm 3: per-vertex cursor (row-relative entry index)
+  ulonglong2* sc_L[2] = {nullptr, nullptr};  // algorithm 3: live (u, pointer key) pairs
   uint64_t* sc_ptr = nullptr;        // algorithm 3: per-vertex pointer key (0 = none)
   uint64_t* suitor = nullptr;        // Suitor: best proposal received, (w << 32) | proposer
   uint32_t* wl[2] = {nullptr, nullptr};   // Suitor worklists
@@ -925,7 +926,7 @@ void lmatch_destroy(lmatch_graph* g) {
   if (g->h_nf) cudaFreeHost(g->h_nf);
   void* pdev[] = {g->bounds, g->ghost, g->claims, g->claim_cnt, g->rstate, g->rlog, g->d_rargs,
                   g->cache, g->chunk_rows, g->cache_big, g->rescan, g->rescan_cnt, g->live, g->win, g->suitor, g->wl[0],
-                  g->wl[1], g->wl_big, g->wl_cnt, g->sc_cur, g->sc_ptr, g->shadow, g->d_dseg, g->d_dcnt,
+                  g->wl[1], g->wl_big, g->wl_cnt, g->sc_cur, g->sc_ptr, g->sc_L[0], g->sc_L[1], g->shadow, g->d_dseg, g->d_dcnt,
                   g->d_dbits, g->d_dnf};
   for (void* p : pdev) if (p) cudaFree(p);
   if (g->h_claim_cnt) cudaFreeHost(g->h_claim_cnt);
@@ -1426,6 +1427,11 @@ static int sort_rows(lmatch_graph* g, cudaStream_t st) {
   return LMATCH_OK;
 }
 
+static unsigned sc_grid(const lmatch_graph* g, int64_t work) {
+  const int64_t per = (int64_t)lm::kScThreads * lm::kScItems;
+  return (unsigned)std::max<int64_t>(1, std::min<int64_t>((work + per - 1) / per, 16ll * g->num_sms));
+}
+
 // algorithm 3: round 1 points every vertex at its first available entry, then host-driven rounds
 // over the live list (point, match) until it is empty; mate[] and w(M) as for Suitor.
 static int run_sorted(lmatch_graph* g, int32_t* d_mate, cudaStream_t st, lmatch_stats* stats) {
@@ -1437,6 +1443,8 @@ static int run_sorted(lmatch_graph* g, int32_t* d_mate, cudaStream_t st, lmatch_
   if (!g->sc_cur) {
     TRY(dmalloc(g, &g->sc_cur, (size_t)n + 1));
     TRY(dmalloc(g, &g->sc_ptr, (size_t)n + 1));
+    TRY(dmalloc(g, &g->sc_L[0], (size_t)n + 1));
+    TRY(dmalloc(g, &g->sc_L[1], (size_t)n + 1));
   }
   int64_t launches = 0, rounds = 0;
   unsigned long long* hc = g->h_counters;
@@ -1444,16 +1452,18 @@ static int run_sorted(lmatch_graph* g, int32_t* d_mate, cudaStream_t st, lmatch_
   CK(cudaMemsetAsync(g->suitor, 0, ((size_t)n + 1) * 8, st));
   CK(cudaMemsetAsync(g->bits, 0, (size_t)((n + 31) / 32) * 4, st));
   CK(cudaMemsetAsync(g->wl_cnt, 0, 4 * 8, st));
+  CK(cudaMemsetAsync(g->sc_cur, 0, ((size_t)n + 1) * 4, st));
   if (tm) CK(cudaEventRecord(g->ev[1], st));
   int cur = 0;
   const bool work = g->ntiles > 0 && n > 0;
   if (work) {
     lm::k_sc_point<<<grid_for(n, 256, 65536), 256, 0, st>>>(nullptr, nullptr, n, g->offs, g->adj,
-                                                             g->sc_cur, g->bits, g->sc_ptr, g->wl_cnt + 2);
+                                                             g->sc_cur, g->bits, g->sc_ptr, nullptr,
+                                                             nullptr, g->wl_cnt + 2);
     CKL();
     if (tm) CK(cudaEventRecord(g->ev[2], st));
-    lm::k_sc_match<<<grid_for(n, 256, 65536), 256, 0, st>>>(nullptr, nullptr, n, g->sc_ptr, g->bits,
-                                                             g->suitor, g->wl[0], g->wl_cnt + 0);
+    lm::k_sc_match<<<sc_grid(g, n), lm::kScThreads, 0, st>>>(nullptr, nullptr, n, g->sc_ptr, g->bits,
+                                                             g->suitor, g->sc_L[0], g->wl_cnt + 0);
     CKL();
     launches += 2;
     rounds = 1;
@@ -1469,15 +1479,20 @@ static int run_sorted(lmatch_graph* g, int32_t* d_mate, cudaStream_t st, lmatch_
     if (c == 0) break;
     if (rounds >= g->max_rounds) { set_err("sorted LD did not converge in %lld rounds", (long long)rounds); return LMATCH_ECUDA; }
     CK(cudaMemsetAsync(g->wl_cnt + (cur ^ 1), 0, 8, st));
-    lm::k_sc_point<<<grid_for(c, 256, 65536), 256, 0, st>>>(g->wl[cur], g->wl_cnt + cur, 0, g->offs,
+    CK(cudaMemsetAsync(g->wl_cnt + 3, 0, 8, st));
+    lm::k_sc_point<<<grid_for(c, 256, 65536), 256, 0, st>>>(g->sc_L[cur], g->wl_cnt + cur, 0, g->offs,
                                                              g->adj, g->sc_cur, g->bits, g->sc_ptr,
-                                                             g->wl_cnt + 2);
+                                                             g->wl[0], g->wl_cnt + 3, g->wl_cnt + 2);
     CKL();
-    lm::k_sc_match<<<grid_for(c, 256, 65536), 256, 0, st>>>(g->wl[cur], g->wl_cnt + cur, 0, g->sc_ptr,
-                                                             g->bits, g->suitor, g->wl[cur ^ 1],
+    lm::k_sc_point_warp<<<(unsigned)(4 * g->num_sms), 512, 0, st>>>(g->sc_L[cur], g->wl[0], g->wl_cnt + 3,
+                                                                    g->offs, g->adj, g->sc_cur, g->bits,
+                                                                    g->sc_ptr, g->wl_cnt + 2);
+    CKL();
+    lm::k_sc_match<<<sc_grid(g, c), lm::kScThreads, 0, st>>>(g->sc_L[cur], g->wl_cnt + cur, 0, g->sc_ptr,
+                                                             g->bits, g->suitor, g->sc_L[cur ^ 1],
                                                              g->wl_cnt + (cur ^ 1));
     CKL();
-    launches += 2;
+    launches += 3;
     ++rounds;
     cur ^= 1;
   }
