@@ -2698,11 +2698,18 @@ __global__ void k_sc_seg_offsets(const int64_t* __restrict__ offs, int64_t r0, i
 // (nothing is matched yet; a 0 key = self-loops only or an empty row).  Rounds >= 2: the live list
 // holds (u, current pointer key) pairs; only u whose target was matched last round change (Alg. 3's
 // frontier): cur[u] (row-relative, 0 after round 1) moves past matched neighbours and the
-// pair and ptr[u] get the new key (0 when the row ran dry).  A thread walks at most kScSerial
+// pair and ptr[u] get the new key (0 when the row ran dry).  A thread walks at most kScSerial (64;
+// 2/4/8/16/32/128/512 measured slower or equal)
 // entries; rows that need more go to the `big` list (list index) for k_sc_point_warp.
 // `reads` counts adjacency entries read.
-constexpr int kScSerial = 8;
-__global__ void k_sc_point(ulonglong2* __restrict__ L, const unsigned long long* __restrict__ nL,
+#ifndef LM_SC_SERIAL
+#define LM_SC_SERIAL 64
+#endif
+#ifndef LM_SC_MINB
+#define LM_SC_MINB 8
+#endif
+constexpr int kScSerial = LM_SC_SERIAL;
+__global__ void __launch_bounds__(256, LM_SC_MINB) k_sc_point(ulonglong2* __restrict__ L, const unsigned long long* __restrict__ nL,
                            int64_t n_all, const int64_t* __restrict__ offs,
                            const uint64_t* __restrict__ adj, uint32_t* __restrict__ cur,
                            const uint32_t* __restrict__ bits, uint64_t* __restrict__ ptr,
