@@ -687,3 +687,12 @@ def test_sorted_repeat_reload_weight_and_rmat24(lm):
     np.testing.assert_array_equal(mate, ref)
     assert st["rounds"] == sref["rounds"]
     assert st["entries_swept"] < sref["entries_swept"]
+
+
+def test_sorted_rejects_out_of_core(lm):
+    """algorithm 3 needs the whole adjacency resident (it sorts it in place): an out-of-core
+    handle's run fails loudly with EINVAL instead of falling back."""
+    g = graphgen.rmat(12, 16, seed=2)
+    with lm.Matcher(g, algorithm="sorted", hbm_budget_bytes=8 * g.m // 2, stream_chunk=1024) as M:
+        with pytest.raises(lm.LMatchError):
+            M.run()
