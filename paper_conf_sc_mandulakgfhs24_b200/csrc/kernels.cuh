@@ -2807,7 +2807,10 @@ __global__ void k_sc_point_warp(ulonglong2* __restrict__ L, const uint32_t* __re
 // (key 0) leaves for good.  Round 1 (L == nullptr) reads the pairs (u, ptr[u]) for every u.
 // Each thread takes kScItems pairs per block step and the block reserves its output with one
 // atomicAdd (per-warp reservations on one counter serialised the kernel).
-constexpr int kScThreads = 256, kScItems = 4;
+#ifndef LM_SC_ITEMS
+#define LM_SC_ITEMS 4
+#endif
+constexpr int kScThreads = 256, kScItems = LM_SC_ITEMS;
 __global__ void __launch_bounds__(kScThreads)
     k_sc_match(const ulonglong2* __restrict__ L, const unsigned long long* __restrict__ nL,
                int64_t n_all, const uint64_t* __restrict__ ptr, uint32_t* bits,

@@ -1427,6 +1427,9 @@ static int sort_rows(lmatch_graph* g, cudaStream_t st) {
   return LMATCH_OK;
 }
 
+#ifndef LM_SC_POINT_BPS
+#define LM_SC_POINT_BPS 32  // rounds >= 2 point kernel: blocks per SM (4 and 442 measured slower)
+#endif
 static unsigned sc_grid(const lmatch_graph* g, int64_t work) {
   const int64_t per = (int64_t)lm::kScThreads * lm::kScItems;
   return (unsigned)std::max<int64_t>(1, std::min<int64_t>((work + per - 1) / per, 16ll * g->num_sms));
@@ -1480,7 +1483,7 @@ static int run_sorted(lmatch_graph* g, int32_t* d_mate, cudaStream_t st, lmatch_
     if (rounds >= g->max_rounds) { set_err("sorted LD did not converge in %lld rounds", (long long)rounds); return LMATCH_ECUDA; }
     CK(cudaMemsetAsync(g->wl_cnt + (cur ^ 1), 0, 8, st));
     CK(cudaMemsetAsync(g->wl_cnt + 3, 0, 8, st));
-    lm::k_sc_point<<<grid_for(c, 256, 65536), 256, 0, st>>>(g->sc_L[cur], g->wl_cnt + cur, 0, g->offs,
+    lm::k_sc_point<<<grid_for(c, 256, LM_SC_POINT_BPS * g->num_sms), 256, 0, st>>>(g->sc_L[cur], g->wl_cnt + cur, 0, g->offs,
                                                              g->adj, g->sc_cur, g->bits, g->sc_ptr,
                                                              g->wl[0], g->wl_cnt + 3, g->wl_cnt + 2);
     CKL();
