@@ -32,3 +32,7 @@ clean:
 
 graphgen/libgraphgen_cuda.so: graphgen/graphgen_cuda.cu graphgen/gg_common.h
 	$(NVCC) -O3 -std=c++17 -fmad=false $(ARCH) -Xcompiler -fPIC -shared $< -o $@
+
+# builder tooling (not product): TMA read-stream microbenchmark, built on demand
+scripts/microbench_stream: scripts/microbench_stream.cu $(PKG)/csrc/kernels.cuh
+	$(NVCC) -O3 -std=c++17 $(ARCH) -lineinfo $< -o $@

@@ -42,7 +42,7 @@
 extern "C" {
 #endif
 
-#define LMATCH_ABI_VERSION 3
+#define LMATCH_ABI_VERSION 4
 
 #if defined(__GNUC__)
 #define LMATCH_API __attribute__((visibility("default")))
@@ -59,7 +59,11 @@ typedef enum lmatch_status {
   LMATCH_ENOMEM = -3, /* device or pinned-host allocation failed */
   LMATCH_ECUDA = -4,  /* CUDA runtime / kernel failure (detail in lmatch_last_error) */
   LMATCH_ENCCL = -5,  /* reserved for the multi-GPU exchange */
-  LMATCH_ESTATE = -6  /* misuse: NULL handle, size mismatch on reload, ... */
+  LMATCH_ESTATE = -6, /* misuse: NULL handle, size mismatch on reload, ... */
+  LMATCH_EROUNDS = -7 /* the round cap (lmatch_opts.max_rounds) stopped the iteration with vertices
+                         still to re-point: the contents of the mate output are unspecified.
+                         Never returned with the default cap (n/2 + 2 bounds the pointing phases,
+                         DESIGN.md R6) */
 } lmatch_status;
 
 /* Opaque handle: one graph resident on one GPU (packed adjacency + per-vertex state). */
@@ -72,10 +76,18 @@ typedef struct lmatch_opts {
                               Set use_device = 1 to honour `device`. */
   int32_t use_device;
   int32_t validate_level;  /* 0 = default (1); 1 = ranges + weights + offsets;
-                              2 = also symmetry (64-bit multiset hash of (u,v,w) vs (v,u,w));
+                              2 = also symmetry and repeated edges ("simple undirected
+                              graph"; SURVEY 8(b) EINVAL rule): the multiset of (u,v,w) must equal
+                              that of (v,u,w) (a 64-bit multiset hash: a false accept needs a
+                              hash collision), and a pair (u,v) listed more than once in row u
+                              must repeat the same weight (exact: every row is sorted by
+                              (v, weight bits) in scratch memory, in chunks of <= 2^27 entries,
+                              and neighbouring entries are compared);
                               -1 = skip validation (caller guarantees a valid CSR) */
   int32_t timing;          /* 1 = record CUDA events per phase into lmatch_stats */
-  int64_t max_rounds;      /* 0 = default: n/2 + 2 (the strict order bounds rounds by n/2+1) */
+  int64_t max_rounds;      /* 0 = default: n/2 + 2 (the strict order bounds rounds by n/2+1).
+                              A smaller cap that stops the iteration with a non-empty frontier
+                              makes lmatch_run* return LMATCH_EROUNDS (all algorithms) */
   int64_t upload_chunk;    /* entries per host->device upload chunk (0 = default 2^25) */
   int64_t hbm_budget_bytes;   /* 0 = adjacency fully resident.  Otherwise, if 8*m exceeds it, only a
                                  prefix of the packed adjacency stays in HBM; the rest lives in
@@ -134,9 +146,16 @@ typedef struct lmatch_opts {
                                  lmatch_stats.ms_sort), then each vertex's pointer is the first
                                  entry at or after its cursor whose neighbour is unmatched (Alg. 1
                                  L4).  Same unique result under R1.  Resident single-graph
-                                 handles only (EINVAL otherwise).  The sort needs min(m, 2^30) x 8 B
-                                 of scratch device memory, freed before the run */
-  int32_t reserved[7];
+                                 handles only (EINVAL otherwise).  The sort needs
+                                 max(min(m, sort_chunk), longest row) x 8 B of scratch device memory
+                                 for the keys, plus cub's temporary storage and 4 B per row of a
+                                 chunk for its segment offsets, all freed before the run (ENOMEM,
+                                 with the size, when they cannot be allocated) */
+  int32_t sort_chunk_log2;    /* algorithm 3: rows are sorted in chunks of at most 2^sort_chunk_log2
+                                 entries (a longer row is one chunk of its own); 0 = default (30).
+                                 Valid 4..30 (EINVAL otherwise); small values exercise the chunking.
+                                 Also caps the chunks of the validate_level-2 duplicate check */
+  int32_t reserved[6];
 } lmatch_opts;
 
 /* Filled by lmatch_run / lmatch_run_device when non-NULL. */

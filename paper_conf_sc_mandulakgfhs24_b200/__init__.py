@@ -33,7 +33,7 @@ if not os.path.exists(lib_path):
 _lib = ctypes.CDLL(lib_path)
 
 LMATCH_OK, LMATCH_EINVAL, LMATCH_ERANGE, LMATCH_ENOMEM = 0, -1, -2, -3
-LMATCH_ECUDA, LMATCH_ENCCL, LMATCH_ESTATE = -4, -5, -6
+LMATCH_ECUDA, LMATCH_ENCCL, LMATCH_ESTATE, LMATCH_EROUNDS = -4, -5, -6, -7
 
 
 class Opts(ctypes.Structure):
@@ -45,7 +45,8 @@ class Opts(ctypes.Structure):
         ("hbm_budget_bytes", ctypes.c_int64), ("stream_chunk", ctypes.c_int64),
         ("round_loop", ctypes.c_int32), ("prune", ctypes.c_int32),
         ("host_cache", ctypes.c_int32), ("batches", ctypes.c_int32),
-        ("algorithm", ctypes.c_int32), ("reserved", ctypes.c_int32 * 7),
+        ("algorithm", ctypes.c_int32), ("sort_chunk_log2", ctypes.c_int32),
+        ("reserved", ctypes.c_int32 * 6),
     ]
 
 
@@ -244,7 +245,7 @@ class Matcher:
                  validate_level: int = 1, timing: bool = False, upload_chunk: int = 0,
                  max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
                  round_loop: int = 0, prune: bool = False, host_cache: bool = True,
-                 batches: int = 0, algorithm: str = "ld"):
+                 batches: int = 0, algorithm: str = "ld", sort_chunk_log2: int = 0):
         self.h = None
         if handle is not None:
             self.h = handle
@@ -255,7 +256,7 @@ class Matcher:
                                       opts=make_opts(validate_level, timing, upload_chunk,
                                                      max_rounds, hbm_budget_bytes, stream_chunk,
                                                      round_loop, prune, host_cache, batches,
-                                                     algorithm))
+                                                     algorithm, sort_chunk_log2))
         self.info = lmatch_info(self.h)
 
     @classmethod
@@ -300,7 +301,7 @@ class Matcher:
 def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int = 0,
               max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
               round_loop: int = 0, prune: bool = False, host_cache: bool = True,
-              batches: int = 0, algorithm: str = "ld") -> Opts:
+              batches: int = 0, algorithm: str = "ld", sort_chunk_log2: int = 0) -> Opts:
     """round_loop (include/lmatch.h): 0 = hybrid (work-sized launches, then one persistent kernel
     for the tail; default), 1 = host-driven launches only, 2 = persistent kernel after round 1,
     3 = CUDA graph {round 1, persistent kernel}."""
@@ -310,6 +311,7 @@ def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int =
     o.host_cache = 0 if host_cache else -1
     o.batches = int(batches)
     o.algorithm = {"ld": 0, "suitor": 1, "hybrid": 2, "sorted": 3}[algorithm]
+    o.sort_chunk_log2 = int(sort_chunk_log2)
     o.hbm_budget_bytes = int(hbm_budget_bytes)
     o.stream_chunk = int(stream_chunk)
     o.validate_level = int(validate_level)

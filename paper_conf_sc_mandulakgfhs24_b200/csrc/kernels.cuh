@@ -47,13 +47,48 @@ constexpr int kBinDeg0 = LM_BIN0, kBinDeg1 = LM_BIN1, kBinDeg2 = LM_BIN2;
 #ifndef LM_ADJ_NOALLOC
 #define LM_ADJ_NOALLOC 0  // 1 = frontier row reads bypass L1 (keep L1 for the bitmap probes)
 #endif
+// L2 policy of the frontier rounds: the row keys a pointer kernel reads are
+// used once per round, while the matched bitmap (n/8 bytes, 8 MB at 2^26) is probed for almost
+// every key; LM_KEY_HINT = 1 loads the keys L1::no_allocate with an L2 evict_first policy and
+// LM_BIT_HINT = 1 probes the bitmap with an L2 evict_last policy, so the key stream does not push
+// the bitmap out of L2.
+#ifndef LM_KEY_HINT
+#define LM_KEY_HINT 0
+#endif
+#ifndef LM_BIT_HINT
+#define LM_BIT_HINT 0
+#endif
+__device__ __forceinline__ uint64_t l2_policy_first() {
+  uint64_t p;
+  asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t l2_policy_last() {
+  uint64_t p;
+  asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
 __device__ __forceinline__ uint64_t ld_stream_u64(const uint64_t* p) {
-#if LM_ADJ_NOALLOC
+#if LM_KEY_HINT
+  uint64_t v;
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(l2_policy_first()));
+  return v;
+#elif LM_ADJ_NOALLOC
   uint64_t v;
   asm("ld.global.nc.L1::no_allocate.u64 %0, [%1];" : "=l"(v) : "l"(p));
   return v;
 #else
   return __ldg(p);
+#endif
+}
+// the bitmap word holding vertex v's matched bit, as probed by the pointer phase
+__device__ __forceinline__ uint32_t probe_word(const uint32_t* __restrict__ bits, uint32_t v) {
+#if LM_BIT_HINT
+  uint32_t x;
+  asm("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(x) : "l"(bits + (v >> 5)), "l"(l2_policy_last()));
+  return x;
+#else
+  return bits[v >> 5];
 #endif
 }
 struct AdjView {
@@ -248,6 +283,29 @@ __global__ void k_symhash(const int64_t* __restrict__ offs, AdjView adj, int64_t
   }
   for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
   if ((threadIdx.x & 31) == 0) atomicAdd(acc, (unsigned long long)s);
+}
+
+// validate_level 2, repeated edges: entries [base, base + cnt) as (neighbour << 32 | weight bits)
+// keys, so a segmented ascending sort groups each row's copies of one neighbour together
+__global__ void k_dup_keys(AdjView adj, int64_t base, int64_t cnt, uint64_t* __restrict__ out) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += stride) {
+    const uint64_t k = adj.at(base + i);
+    out[i] = (k << 32) | (k >> 32);
+  }
+}
+// ... and neighbouring sorted keys of one row with the same neighbour must be equal; *bad = the
+// smallest offending row (global id row0 + r).  8 lanes per row.
+__global__ void k_dup_check(const uint64_t* __restrict__ keys, const int32_t* __restrict__ seg,
+                            int64_t nrows, int64_t row0, unsigned long long* bad) {
+  const int lane8 = threadIdx.x & 7;
+  const int64_t g0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 3;
+  const int64_t gs = ((int64_t)gridDim.x * blockDim.x) >> 3;
+  for (int64_t r = g0; r < nrows; r += gs)
+    for (int64_t j = (int64_t)seg[r] + 1 + lane8; j < (int64_t)seg[r + 1]; j += 8) {
+      const uint64_t a = keys[j - 1], b = keys[j];
+      if ((a >> 32) == (b >> 32) && a != b) atomicMin(bad, (unsigned long long)(row0 + r));
+    }
 }
 
 // =============================================================================================
@@ -1021,7 +1079,7 @@ __device__ __forceinline__ uint64_t scan_row_available_t(const AdjView adj,
       for (int q = 0; q < U; ++q) mx = (k[q] > b && k[q] > mx) ? k[q] : mx;
 #endif
       bool avail = false;
-      if (mx) avail = !((bits[(uint32_t)mx >> 5] >> ((uint32_t)mx & 31)) & 1u);
+      if (mx) avail = !((probe_word(bits, (uint32_t)mx) >> ((uint32_t)mx & 31)) & 1u);
       uint64_t c = avail ? mx : 0ull;
       if (G > 1) c = group_max_key(c, rmask);
       const uint64_t bb = c > b ? c : b;
@@ -1036,7 +1094,7 @@ __device__ __forceinline__ uint64_t scan_row_available_t(const AdjView adj,
         uint32_t wd[U];
 #pragma unroll
         for (int q = 0; q < U; ++q)
-          wd[q] = (need && k[q] > bb && k[q] != mx) ? bits[(uint32_t)k[q] >> 5] : 0xffffffffu;
+          wd[q] = (need && k[q] > bb && k[q] != mx) ? probe_word(bits, (uint32_t)k[q]) : 0xffffffffu;
         uint64_t c2 = 0;
 #pragma unroll
         for (int q = 0; q < U; ++q) {
@@ -1050,7 +1108,7 @@ __device__ __forceinline__ uint64_t scan_row_available_t(const AdjView adj,
     } else {
       uint32_t wd[U];
 #pragma unroll
-      for (int q = 0; q < U; ++q) wd[q] = k[q] > b ? bits[(uint32_t)k[q] >> 5] : 0xffffffffu;
+      for (int q = 0; q < U; ++q) wd[q] = k[q] > b ? probe_word(bits, (uint32_t)k[q]) : 0xffffffffu;
 #pragma unroll
       for (int q = 0; q < U; ++q) {
         const uint32_t v = (uint32_t)k[q];
@@ -1065,7 +1123,7 @@ __device__ __forceinline__ uint64_t scan_row_available_t(const AdjView adj,
       for (int q = 0; q < U; ++q) mx = (k[q] > b && k[q] > mx) ? k[q] : mx;
       if (!mx) break;
       const uint32_t v = (uint32_t)mx;
-      if (!((bits[v >> 5] >> (v & 31)) & 1u)) { b = mx; break; }
+      if (!((probe_word(bits, v) >> (v & 31)) & 1u)) { b = mx; break; }
 #pragma unroll
       for (int q = 0; q < U; ++q) k[q] = k[q] == mx ? 0ull : k[q];
     }
@@ -1078,7 +1136,7 @@ __device__ __forceinline__ uint64_t scan_row_available_t(const AdjView adj,
       for (int q = 0; q < U; ++q) mx = (k[q] > b && k[q] > mx) ? k[q] : mx;
       if (mx) {
         const uint32_t v = (uint32_t)mx;
-        if (!((bits[v >> 5] >> (v & 31)) & 1u)) {
+        if (!((probe_word(bits, v) >> (v & 31)) & 1u)) {
           b = mx;
           continue;
         }
@@ -1089,7 +1147,7 @@ __device__ __forceinline__ uint64_t scan_row_available_t(const AdjView adj,
 #endif
     uint32_t wd[U];
 #pragma unroll
-    for (int q = 0; q < U; ++q) wd[q] = k[q] > b ? bits[(uint32_t)k[q] >> 5] : 0xffffffffu;
+    for (int q = 0; q < U; ++q) wd[q] = k[q] > b ? probe_word(bits, (uint32_t)k[q]) : 0xffffffffu;
 #pragma unroll
     for (int q = 0; q < U; ++q) {
       const uint32_t v = (uint32_t)k[q];
@@ -1134,7 +1192,7 @@ __device__ __forceinline__ uint64_t prune_row(const AdjView adj, const uint32_t*
   }
   uint32_t wd[U];
 #pragma unroll
-  for (int q = 0; q < U; ++q) wd[q] = k[q] ? bits[(uint32_t)k[q] >> 5] : 0xffffffffu;
+  for (int q = 0; q < U; ++q) wd[q] = k[q] ? probe_word(bits, (uint32_t)k[q]) : 0xffffffffu;
   bool sv[U];
   uint64_t b = 0;
 #pragma unroll
@@ -1240,7 +1298,7 @@ __device__ __forceinline__ uint64_t probe_batch(const uint32_t* __restrict__ bit
                                                 const uint64_t (&k)[U], uint64_t b) {
   uint32_t wd[U];
 #pragma unroll
-  for (int q = 0; q < U; ++q) wd[q] = k[q] > b ? bits[(uint32_t)k[q] >> 5] : 0xffffffffu;
+  for (int q = 0; q < U; ++q) wd[q] = k[q] > b ? probe_word(bits, (uint32_t)k[q]) : 0xffffffffu;
 #pragma unroll
   for (int q = 0; q < U; ++q) {
     const uint32_t v = (uint32_t)k[q];
@@ -1261,7 +1319,7 @@ __device__ __forceinline__ uint64_t probe_batch2(const uint32_t* __restrict__ bi
 #pragma unroll
   for (int q = 0; q < U; ++q) mx = (k[q] > b && k[q] > mx) ? k[q] : mx;
   bool avail = false;
-  if (mx) avail = !((bits[(uint32_t)mx >> 5] >> ((uint32_t)mx & 31)) & 1u);
+  if (mx) avail = !((probe_word(bits, (uint32_t)mx) >> ((uint32_t)mx & 31)) & 1u);
   uint64_t c = avail ? mx : 0ull;
   if (G > 1) c = group_max_key(c, gmask);
   const uint64_t bb = c > b ? c : b;
@@ -1275,7 +1333,7 @@ __device__ __forceinline__ uint64_t probe_batch2(const uint32_t* __restrict__ bi
   uint32_t wd[U];
 #pragma unroll
   for (int q = 0; q < U; ++q)
-    wd[q] = (need && k[q] > bb && k[q] != mx) ? bits[(uint32_t)k[q] >> 5] : 0xffffffffu;
+    wd[q] = (need && k[q] > bb && k[q] != mx) ? probe_word(bits, (uint32_t)k[q]) : 0xffffffffu;
   uint64_t c2 = 0;
 #pragma unroll
   for (int q = 0; q < U; ++q) {

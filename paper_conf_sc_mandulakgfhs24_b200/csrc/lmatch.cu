@@ -162,6 +162,12 @@ constexpr int64_t kHandoffRounds = 32;  // hybrid (algorithm 2): LD pointing pha
 #ifndef LM_PIPE_WAVES
 #define LM_PIPE_WAVES 1
 #endif
+// 1 = the frontier pointer kernels are launched with a persisting L2 access-policy window over
+// the matched bitmap (cudaLaunchAttributeAccessPolicyWindow; the device's persisting L2 set-aside
+// is sized to the bitmap at create time), so the streamed row keys do not evict it
+#ifndef LM_L2_WINDOW
+#define LM_L2_WINDOW 0
+#endif
 
 constexpr int kFinBlocks = 2368;  // 16 x 148 SMs: fixed => deterministic fp64 summation order
 constexpr int kFinThreads = 256;
@@ -212,6 +218,7 @@ struct lmatch_graph {
   int64_t hbm_budget = 0;
   int batches = 0;                   // paper-style batch count (> 1: all streamed)
   int algorithm = 0;                 // 0 = LD pointer iteration, 1 = Suitor (NEXT-4), 3 = sorted+cursor
+  int64_t sort_chunk = 1ll << 30;    // algorithm 3: entries per segmented-sort chunk
   bool sorted = false;               // algorithm 3: rows sorted by key, descending (NEXT-3)
   float ms_sort = 0.f;               // algorithm 3: device time of the last row sort
   uint32_t* sc_cur = nullptr;        // algorithm 3: per-vertex cursor (row-relative entry index)
@@ -244,6 +251,7 @@ struct lmatch_graph {
   int sweep_grid = 0;
   alignas(64) CUtensorMap tmap;  // adjacency as a [ceil(m/16)][16] u64 tensor, 128B swizzle
   int num_sms = 148;
+  cudaAccessPolicyWindow bits_window = {};  // LM_L2_WINDOW: the matched bitmap, persisting
   // graph
   int64_t* offs = nullptr;
   uint64_t* adj = nullptr;
@@ -356,6 +364,28 @@ int grid_for(int64_t work, int threads, int max_blocks) {
   if (b < 1) b = 1;
   if (b > max_blocks) b = max_blocks;
   return (int)b;
+}
+
+// launch with the bitmap's persisting L2 window (LM_L2_WINDOW), else a plain launch
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pw(const lmatch_graph* g, void (*k)(KArgs...), unsigned grid, unsigned block,
+                      cudaStream_t st, Args... args) {
+#if LM_L2_WINDOW
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(block);
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeAccessPolicyWindow;
+  at[0].val.accessPolicyWindow = g->bits_window;
+  cfg.attrs = at;
+  cfg.numAttrs = g->bits_window.num_bytes > 0 ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, k, args...);
+#else
+  (void)g;
+  k<<<grid, block, 0, st>>>(args...);
+  return cudaGetLastError();
+#endif
 }
 
 int check_args(const void* a, const void* b, const void* c, int64_t n, int64_t m) {
@@ -507,6 +537,117 @@ int reset_err(lmatch_graph* g, cudaStream_t st) {
   return LMATCH_OK;
 }
 
+int64_t host_off(lmatch_graph* g, int64_t r, cudaStream_t st, int* err) {
+  int64_t v = 0;
+  if (cudaMemcpyAsync(&v, g->offs + r, 8, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+      cudaStreamSynchronize(st) != cudaSuccess) *err = 1;
+  return v;
+}
+
+// Cut rows [0, n) into chunks of at most `cap` entries (a longer row is a chunk of its own):
+// cuts[c] .. cuts[c+1]; *maxcnt / *maxrows = the largest chunk's entries / rows.
+int row_chunks(lmatch_graph* g, cudaStream_t st, int64_t cap, std::vector<int64_t>* cuts,
+               int64_t* maxcnt, int64_t* maxrows) {
+  const int64_t n = g->n;
+  int err = 0;
+  *maxcnt = 0;
+  *maxrows = 0;
+  cuts->clear();
+  const int64_t mtot = host_off(g, n, st, &err);
+  for (int64_t r0 = 0; r0 < n;) {
+    const int64_t b0 = host_off(g, r0, st, &err);
+    int64_t lo = r0 + 1, hi = n;  // largest r1 with offs[r1] - b0 <= cap (at least one row)
+    if (mtot - b0 <= cap) lo = n;
+    else {
+      while (lo < hi) {
+        const int64_t mid = lo + (hi - lo + 1) / 2;
+        if (host_off(g, mid, st, &err) - b0 <= cap) lo = mid; else hi = mid - 1;
+      }
+    }
+    if (err) { set_err("offset read failed"); return LMATCH_ECUDA; }
+    const int64_t cnt = host_off(g, lo, st, &err) - b0;
+    if (cnt > INT_MAX) { set_err("row %lld has more than 2^31-1 entries", (long long)r0); return LMATCH_EINVAL; }
+    cuts->push_back(r0);
+    *maxcnt = std::max(*maxcnt, cnt);
+    *maxrows = std::max(*maxrows, lo - r0);
+    r0 = lo;
+  }
+  cuts->push_back(n);
+  return err ? LMATCH_ECUDA : LMATCH_OK;
+}
+
+// validate_level 2, repeated edges ("duplicate edges with unequal weights" -> EINVAL):
+// every row's (neighbour << 32 | weight bits) keys are sorted ascending in scratch memory, chunk by
+// chunk, and neighbouring keys of one row with the same neighbour must be equal.  Exact.
+constexpr int64_t kDupChunk = 1ll << 27;
+int check_duplicates(lmatch_graph* g, cudaStream_t st) {
+  if (g->n == 0 || g->m == 0) return LMATCH_OK;
+  std::vector<int64_t> cuts;
+  int64_t maxcnt = 0, maxrows = 0;
+  TRY(row_chunks(g, st, std::min(g->m, std::min(kDupChunk, g->sort_chunk)), &cuts, &maxcnt, &maxrows));
+  uint64_t *kin = nullptr, *kout = nullptr;
+  int32_t* seg = nullptr;
+  unsigned long long* bad = nullptr;
+  void* tmp = nullptr;
+  size_t tmp_bytes = 0, need = 0;
+  int rc = LMATCH_OK;
+  auto fail_alloc = [&](const char* what, size_t bytes) {
+    cudaGetLastError();
+    set_err("validate_level 2: cannot allocate %zu bytes (%s)", bytes, what);
+    rc = LMATCH_ENOMEM;
+  };
+  const size_t kb = (size_t)std::max<int64_t>(maxcnt, 1) * 8;
+  if (cudaMalloc(&kin, kb) != cudaSuccess) fail_alloc("row keys", kb);
+  if (!rc && cudaMalloc(&kout, kb) != cudaSuccess) fail_alloc("sorted row keys", kb);
+  if (!rc && cudaMalloc(&seg, (size_t)(maxrows + 1) * 4) != cudaSuccess) fail_alloc("segments", (size_t)(maxrows + 1) * 4);
+  if (!rc && cudaMalloc(&bad, 8) != cudaSuccess) fail_alloc("flag", 8);
+  if (!rc && cudaMemsetAsync(bad, 0xff, 8, st) != cudaSuccess) rc = LMATCH_ECUDA;
+  int err = 0;
+  for (size_t c = 0; rc == LMATCH_OK && c + 1 < cuts.size(); ++c) {
+    const int64_t a = cuts[c], b = cuts[c + 1];
+    const int64_t base = host_off(g, a, st, &err), cnt = host_off(g, b, st, &err) - base;
+    if (err) { set_err("offset read failed"); rc = LMATCH_ECUDA; break; }
+    if (cnt == 0) continue;
+    lm::k_sc_seg_offsets<<<grid_for(b - a + 1, 256, 65536), 256, 0, st>>>(g->offs, a, b, seg);
+    lm::k_dup_keys<<<grid_for(cnt, 256, 65536), 256, 0, st>>>(g->view(), base, cnt, kin);
+    if (cudaGetLastError() != cudaSuccess) { set_err("duplicate check launch failed"); rc = LMATCH_ECUDA; break; }
+    g_launch_count.fetch_add(2, std::memory_order_relaxed);
+    if (cub::DeviceSegmentedSort::SortKeys(nullptr, need, kin, kout, (int)cnt, (int)(b - a), seg, seg + 1,
+                                           st) != cudaSuccess) {
+      set_err("duplicate check: sort sizing failed"); rc = LMATCH_ECUDA; break;
+    }
+    if (need > tmp_bytes) {
+      if (tmp) cudaFree(tmp);
+      tmp = nullptr;
+      tmp_bytes = 0;
+      if (cudaMalloc(&tmp, need) != cudaSuccess) { fail_alloc("sort temporary storage", need); break; }
+      tmp_bytes = need;
+    }
+    if (cub::DeviceSegmentedSort::SortKeys(tmp, need, kin, kout, (int)cnt, (int)(b - a), seg, seg + 1,
+                                           st) != cudaSuccess) {
+      set_err("duplicate check: sort failed"); rc = LMATCH_ECUDA; break;
+    }
+    lm::k_dup_check<<<grid_for((b - a) * 8, 256, 16384), 256, 0, st>>>(kout, seg, b - a, a, bad);
+    if (cudaGetLastError() != cudaSuccess) { set_err("duplicate check launch failed"); rc = LMATCH_ECUDA; break; }
+    g_launch_count.fetch_add(1, std::memory_order_relaxed);
+  }
+  unsigned long long hbad = ULLONG_MAX;
+  if (rc == LMATCH_OK && cudaMemcpyAsync(&hbad, bad, 8, cudaMemcpyDeviceToHost, st) != cudaSuccess) rc = LMATCH_ECUDA;
+  const cudaError_t se = cudaStreamSynchronize(st);
+  if (tmp) cudaFree(tmp);
+  if (seg) cudaFree(seg);
+  if (kin) cudaFree(kin);
+  if (kout) cudaFree(kout);
+  if (bad) cudaFree(bad);
+  if (rc != LMATCH_OK) return rc;
+  if (se != cudaSuccess) { set_err("duplicate check: %s", cudaGetErrorString(se)); return LMATCH_ECUDA; }
+  if (hbad != ULLONG_MAX) {
+    set_err("row %llu lists a neighbour twice with unequal weights", hbad);
+    return LMATCH_EINVAL;
+  }
+  return LMATCH_OK;
+}
+
 int check_pack(lmatch_graph* g, cudaStream_t st) {
   lm::PackErr h{};
   CK(cudaMemcpyAsync(&h, g->perr, sizeof h, cudaMemcpyDeviceToHost, st));
@@ -530,6 +671,7 @@ int check_pack(lmatch_graph* g, cudaStream_t st) {
       set_err("graph is not symmetric: multiset of (u,v,w) differs from (v,u,w)");
       return LMATCH_EINVAL;
     }
+    TRY(check_duplicates(g, st));
   }
   return LMATCH_OK;
 }
@@ -698,12 +840,36 @@ static int prefer_l1() {
 
 int finish_create(lmatch_graph* g, cudaStream_t st) {
   TRY(prefer_l1());
+#if LM_L2_WINDOW
+  {
+    int maxp = 0, maxw = 0;
+    CK(cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, g->device));
+    CK(cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, g->device));
+    const size_t bytes = (size_t)((g->n_global + 31) / 32) * 4;
+    if (maxp > 0 && maxw > 0 && bytes > 0) {
+      size_t limit = 0;
+      CK(cudaDeviceGetLimit(&limit, cudaLimitPersistingL2CacheSize));
+      if (limit < std::min(bytes, (size_t)maxp))
+        CK(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, std::min(bytes, (size_t)maxp)));
+      CK(cudaDeviceGetLimit(&limit, cudaLimitPersistingL2CacheSize));
+      g->bits_window.base_ptr = g->bits;
+      g->bits_window.num_bytes = std::min(bytes, (size_t)maxw);
+      g->bits_window.hitRatio = std::min(1.0f, (float)limit / (float)g->bits_window.num_bytes);
+      g->bits_window.hitProp = cudaAccessPropertyPersisting;
+      g->bits_window.missProp = cudaAccessPropertyStreaming;
+    }
+  }
+#endif
   if (g->prune && (g->streaming || g->ghost)) g->prune = 0;  // resident single-graph only
   if (g->prune && !g->live) {
     TRY(dmalloc(g, &g->live, (size_t)g->n + 1));
     CK(cudaMemsetAsync(g->live, 0, ((size_t)g->n + 1) * 4, st));
   }
   g->sorted = false;  // (re)loaded adjacency: algorithm 3 sorts it again on the next run
+  // best[] = 0 for every vertex: the sweep writes non-empty rows only, so a row that is empty in
+  // a reloaded graph must not keep the pointer of the previous graph (Suitor's first pass and the
+  // partitioned claims read best[] of every vertex)
+  CK(cudaMemsetAsync(g->best, 0, ((size_t)g->n + 1) * 8, st));
   TRY(build_index(g, st));
   TRY(alloc_bins(g, st));
   TRY(build_cache_index(g, st));
@@ -780,6 +946,13 @@ int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** 
     g->host_cache = opts->host_cache >= 0;
     g->batches = opts->batches;
     g->algorithm = opts->algorithm;
+    if (opts->sort_chunk_log2 != 0) {
+      if (opts->sort_chunk_log2 < 4 || opts->sort_chunk_log2 > 30) {
+        set_err("sort_chunk_log2 = %d outside 4..30", opts->sort_chunk_log2);
+        return LMATCH_EINVAL;
+      }
+      g->sort_chunk = 1ll << opts->sort_chunk_log2;
+    }
   }
   CK(cudaGetDevice(&g->device));
   CK(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, g->device));
@@ -893,6 +1066,7 @@ const char* lmatch_strerror(int status) {
     case LMATCH_ECUDA: return "CUDA error";
     case LMATCH_ENCCL: return "NCCL error";
     case LMATCH_ESTATE: return "invalid state";
+    case LMATCH_EROUNDS: return "round cap reached before the matching was maximal";
     default: return "unknown status";
   }
 }
@@ -1125,11 +1299,13 @@ static int seq_body(lmatch_graph* g, cudaStream_t st, int cur, const int64_t* nF
         if (occ < 1) occ = 1;                                                                     \
       }                                                                                           \
       const int64_t wave = (int64_t)occ * g->num_sms * LM_PIPE_WAVES;                              \
-      lm::k_point_pipe<PG, PU><<<(unsigned)std::min<int64_t>(wave, (nFb[b] * PG + 255) / 256), 256, 0, st>>>( \
-          Fb.list[b], cF + b, g->offs, av, g->bits, g->best, g->v0);                              \
+      CK(launch_pw(g, lm::k_point_pipe<PG, PU>, (unsigned)std::min<int64_t>(wave, (nFb[b] * PG + 255) / 256), \
+                   256, st, Fb.list[b], cF + b, (const int64_t*)g->offs, av, (const uint32_t*)g->bits, \
+                   g->best, g->v0));                                                              \
     } else {                                                                                      \
-      lm::k_point_bin<BG, BU><<<grid_for(nFb[b] * BG, 256, 65536), 256, 0, st>>>(                 \
-          Fb.list[b], cF + b, g->offs, av, g->bits, g->best, g->v0);                              \
+      CK(launch_pw(g, lm::k_point_bin<BG, BU, false>, (unsigned)grid_for(nFb[b] * BG, 256, 65536), 256, st, \
+                   Fb.list[b], cF + b, (const int64_t*)g->offs, av, (const uint32_t*)g->bits, g->best, \
+                   g->v0, (uint32_t*)nullptr, (const lm::RoundState*)nullptr));                 \
     }                                                                                             \
     CKL();                                                                                        \
     ++*launches;                                                                                  \
@@ -1155,7 +1331,12 @@ static int seq_body(lmatch_graph* g, cudaStream_t st, int cur, const int64_t* nF
     }
     {
       cudaStream_t st = fork ? g->bs[2] : st_main;
-      if (nFb[3]) { lm::k_point_bin_cta<256, LM_CTA_U><<<(unsigned)std::min<int64_t>(nFb[3], 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); ++*launches; }
+      if (nFb[3]) {
+        CK(launch_pw(g, lm::k_point_bin_cta<256, LM_CTA_U>, (unsigned)std::min<int64_t>(nFb[3], 65536), 256, st,
+                     Fb.list[3], cF + 3, (const int64_t*)g->offs, av, (const uint32_t*)g->bits, g->best, g->v0));
+        CKL();
+        ++*launches;
+      }
     }
   }
   PIPE_OR_BIN(0, LM_P0_G, LM_P0_U, LM_B0_G, LM_B0_U, LM_A0_G, LM_A0_U)
@@ -1195,11 +1376,13 @@ int launch_persistent_t(lmatch_graph* g, cudaStream_t st, int64_t* launches) {
   cfg.gridDim = dim3((unsigned)(occ * g->num_sms));
   cfg.blockDim = dim3(256);
   cfg.stream = st;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributeCooperative;
   attr[0].val.cooperative = 1;
+  attr[1].id = cudaLaunchAttributeAccessPolicyWindow;
+  attr[1].val.accessPolicyWindow = g->bits_window;
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = (LM_L2_WINDOW && g->bits_window.num_bytes > 0) ? 2 : 1;
   CK(cudaLaunchKernelEx(&cfg, PERSISTENT_KERNEL(PRUNE), ra, (const int64_t*)g->offs, av, g->bits,
                         g->best, g->n, g->v0));
   g_launch_count.fetch_add(1, std::memory_order_relaxed);
@@ -1250,7 +1433,10 @@ static int suitor_loop(lmatch_graph* g, cudaStream_t st, int64_t* launches, int6
     CK(cudaStreamSynchronize(st));
     const int64_t c = (int64_t)hc[cur];
     if (c == 0) break;
-    if (*passes >= g->max_rounds) { set_err("Suitor did not converge in %lld passes", (long long)*passes); return LMATCH_ECUDA; }
+    if (*passes >= g->max_rounds) {
+      set_err("Suitor: %lld proposers left after the pass cap (%lld)", (long long)c, (long long)g->max_rounds);
+      return LMATCH_EROUNDS;
+    }
     unsigned long long* nc = g->wl_cnt + (cur ^ 1);
     CK(cudaMemsetAsync(nc, 0, 8, st));
     CK(cudaMemsetAsync(g->wl_cnt + 2, 0, 8, st));
@@ -1345,59 +1531,44 @@ static int run_suitor(lmatch_graph* g, int32_t* d_mate, cudaStream_t st, lmatch_
 
 
 // ---- algorithm 3 (NEXT-3): sort every row by key, descending, in place.  Rows are grouped into
-// chunks of at most kSortChunk entries (cub's segmented sort takes int sizes), each sorted into a
-// scratch buffer and copied back.  Done once per loaded graph; the time goes to lmatch_stats.ms_sort.
-constexpr int64_t kSortChunk = 1ll << 30;
-
-static int64_t host_off(lmatch_graph* g, int64_t r, cudaStream_t st, int* err) {
-  int64_t v = 0;
-  if (cudaMemcpyAsync(&v, g->offs + r, 8, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
-      cudaStreamSynchronize(st) != cudaSuccess) *err = 1;
-  return v;
-}
-
+// chunks of at most g->sort_chunk entries (cub's segmented sort takes int sizes; a longer row is a
+// chunk of its own), each sorted into a scratch buffer sized for the largest chunk and copied back.
+// Done once per loaded graph; the time goes to lmatch_stats.ms_sort.
 static int sort_rows(lmatch_graph* g, cudaStream_t st) {
   const int64_t n = g->n, m = g->m;
   CK(cudaEventRecord(g->ev[6], st));
   if (m > 0 && n > 0) {
     int err = 0;
-    const int64_t cap = std::min<int64_t>(m, kSortChunk);
+    const int64_t cap = std::min<int64_t>(m, g->sort_chunk);
+    // cut pass: rows [cuts[c], cuts[c+1]) = the longest run of rows within cap entries (at least
+    // one row); the scratch buffer is sized for the largest chunk
+    std::vector<int64_t> cuts;
+    int64_t maxcnt = 0, maxrows = 0;
+    TRY(row_chunks(g, st, cap, &cuts, &maxcnt, &maxrows));
     uint64_t* alt = nullptr;
     int32_t* seg = nullptr;
     void* tmp = nullptr;
     size_t tmp_bytes = 0, need = 0;
-    CK(cudaMalloc(&alt, (size_t)cap * 8));
     int rc = LMATCH_OK;
-    int64_t r0 = 0;
-    std::vector<int64_t> cuts;
-    while (r0 < n && rc == LMATCH_OK) {  // rows [r0, r1): the longest run of rows within cap entries
-      const int64_t b0 = host_off(g, r0, st, &err);
-      int64_t lo = r0 + 1, hi = n;  // largest r1 with offs[r1] - b0 <= cap (at least one row)
-      if (host_off(g, n, st, &err) - b0 <= cap) lo = n;
-      else {
-        while (lo < hi) {
-          const int64_t mid = lo + (hi - lo + 1) / 2;
-          if (host_off(g, mid, st, &err) - b0 <= cap) lo = mid; else hi = mid - 1;
-        }
-      }
-      if (err) { set_err("offset read failed"); rc = LMATCH_ECUDA; break; }
-      const int64_t r1 = lo, cnt = host_off(g, r1, st, &err) - b0;
-      if (cnt > INT_MAX) { set_err("row %lld has more than 2^31-1 entries", (long long)r0); rc = LMATCH_EINVAL; break; }
-      cuts.push_back(r0);
-      r0 = r1;
+    if (cudaMalloc(&alt, (size_t)std::max<int64_t>(maxcnt, 1) * 8) != cudaSuccess) {
+      cudaGetLastError();
+      set_err("sorted LD: cannot allocate %lld bytes of sort scratch (largest chunk %lld entries)",
+              (long long)(std::max<int64_t>(maxcnt, 1) * 8), (long long)maxcnt);
+      return LMATCH_ENOMEM;
     }
-    cuts.push_back(n);
-    int64_t maxrows = 0;
-    for (size_t c = 0; c + 1 < cuts.size(); ++c) maxrows = std::max(maxrows, cuts[c + 1] - cuts[c]);
-    if (rc == LMATCH_OK && cudaMalloc(&seg, (size_t)(maxrows + 1) * 4) != cudaSuccess) {
-      set_err("cudaMalloc(segment offsets) failed"); rc = LMATCH_ENOMEM;
+    if (cudaMalloc(&seg, (size_t)(maxrows + 1) * 4) != cudaSuccess) {
+      cudaGetLastError();
+      set_err("sorted LD: cannot allocate %lld bytes of segment offsets", (long long)((maxrows + 1) * 4));
+      rc = LMATCH_ENOMEM;
     }
     for (size_t c = 0; rc == LMATCH_OK && c + 1 < cuts.size(); ++c) {
       const int64_t a = cuts[c], b = cuts[c + 1];
       const int64_t base = host_off(g, a, st, &err), cnt = host_off(g, b, st, &err) - base;
+      if (err) { set_err("offset read failed"); rc = LMATCH_ECUDA; break; }
       if (cnt == 0) continue;
       lm::k_sc_seg_offsets<<<grid_for(b - a + 1, 256, 65536), 256, 0, st>>>(g->offs, a, b, seg);
-      if (cudaGetLastError() != cudaSuccess) { rc = LMATCH_ECUDA; break; }
+      if (cudaGetLastError() != cudaSuccess) { set_err("segment offsets launch failed"); rc = LMATCH_ECUDA; break; }
+      g_launch_count.fetch_add(1, std::memory_order_relaxed);
       if (cub::DeviceSegmentedSort::SortKeysDescending(nullptr, need, g->adj + base, alt, (int)cnt,
                                                        (int)(b - a), seg, seg + 1, st) != cudaSuccess) {
         set_err("segmented sort sizing failed"); rc = LMATCH_ECUDA; break;
@@ -1405,7 +1576,13 @@ static int sort_rows(lmatch_graph* g, cudaStream_t st) {
       if (need > tmp_bytes) {
         if (tmp) cudaFree(tmp);
         tmp = nullptr;
-        if (cudaMalloc(&tmp, need) != cudaSuccess) { set_err("cudaMalloc(sort temp) failed"); rc = LMATCH_ENOMEM; break; }
+        tmp_bytes = 0;
+        if (cudaMalloc(&tmp, need) != cudaSuccess) {
+          cudaGetLastError();
+          set_err("sorted LD: cannot allocate %zu bytes of sort temporary storage", need);
+          rc = LMATCH_ENOMEM;
+          break;
+        }
         tmp_bytes = need;
       }
       if (cub::DeviceSegmentedSort::SortKeysDescending(tmp, need, g->adj + base, alt, (int)cnt,
@@ -1414,11 +1591,12 @@ static int sort_rows(lmatch_graph* g, cudaStream_t st) {
         set_err("segmented sort failed"); rc = LMATCH_ECUDA; break;
       }
     }
-    cudaStreamSynchronize(st);
+    const cudaError_t se = cudaStreamSynchronize(st);
     if (tmp) cudaFree(tmp);
     if (seg) cudaFree(seg);
     cudaFree(alt);
     if (rc != LMATCH_OK) return rc;
+    if (se != cudaSuccess) { set_err("row sort: %s", cudaGetErrorString(se)); return LMATCH_ECUDA; }
   }
   CK(cudaEventRecord(g->ev[7], st));
   CK(cudaEventSynchronize(g->ev[7]));
@@ -1480,7 +1658,11 @@ static int run_sorted(lmatch_graph* g, int32_t* d_mate, cudaStream_t st, lmatch_
     CK(cudaStreamSynchronize(st));
     const int64_t c = (int64_t)hc[cur];
     if (c == 0) break;
-    if (rounds >= g->max_rounds) { set_err("sorted LD did not converge in %lld rounds", (long long)rounds); return LMATCH_ECUDA; }
+    if (rounds >= g->max_rounds) {
+      set_err("sorted LD: %lld vertices still to re-point after the round cap (%lld)", (long long)c,
+              (long long)g->max_rounds);
+      return LMATCH_EROUNDS;
+    }
     CK(cudaMemsetAsync(g->wl_cnt + (cur ^ 1), 0, 8, st));
     CK(cudaMemsetAsync(g->wl_cnt + 3, 0, 8, st));
     lm::k_sc_point<<<grid_for(c, 256, LM_SC_POINT_BPS * g->num_sms), 256, 0, st>>>(g->sc_L[cur], g->wl_cnt + cur, 0, g->offs,
@@ -1649,12 +1831,16 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
     g->h_resc[0] = 0;
   }
   CK(cudaMemcpyAsync(g->h_rstate, g->rstate, sizeof(lm::RoundState), cudaMemcpyDeviceToHost, st));
-  if (g->use_cache())
-    CK(cudaMemcpyAsync(g->h_counters, g->counters, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
+  CK(cudaMemcpyAsync(g->h_counters, g->counters, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
   if (tm) CK(cudaEventRecord(g->ev[5], st));
   CK(cudaStreamSynchronize(st));
   const lm::RoundState rs = *g->h_rstate;
   const int64_t rounds = rs.rounds;
+  // a frontier left in the current set means the round cap stopped the iteration (the hybrid's
+  // own 32-phase cap hands that frontier to the Suitor tail instead)
+  int64_t nF_left = 0;
+  if (g->ntiles > 0 && n > 0 && !(g->algorithm == 2 && !g->streaming))
+    for (int b = 0; b < lm::kBins; ++b) nF_left += (int64_t)g->h_counters[lm::cnt_F(rs.cur, b)];
   if (use_graph) {  // launches inside the graph
     launches += (rounds > 0 ? 6 : 2) + (rounds > 0 ? 1 : 0);
     sweep_launches = rounds > 0 ? 1 : 0;
@@ -1702,6 +1888,11 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
       stats->ms_rounds = d;
       stats->ms_finish = e;
     }
+  }
+  if (nF_left > 0) {
+    set_err("%lld vertices still to re-point after the round cap (%lld pointing phases)",
+            (long long)nF_left, (long long)rounds);
+    return LMATCH_EROUNDS;
   }
   return LMATCH_OK;
 }

@@ -55,12 +55,12 @@ def test_struct_layout_matches_header(pkg):
 #include <stddef.h>
 #include "lmatch.h"
 int main(void){
-  printf("%zu %zu %zu %zu %zu %zu %zu %zu %zu %zu %zu\n", sizeof(lmatch_opts), sizeof(lmatch_stats),
+  printf("%zu %zu %zu %zu %zu %zu %zu %zu %zu %zu %zu %zu\n", sizeof(lmatch_opts), sizeof(lmatch_stats),
          offsetof(lmatch_stats, weight), offsetof(lmatch_stats, ms_sweep),
          offsetof(lmatch_opts, upload_chunk), offsetof(lmatch_opts, host_cache),
          offsetof(lmatch_opts, batches), offsetof(lmatch_stats, cache_rows),
          offsetof(lmatch_stats, cache_bytes), offsetof(lmatch_opts, algorithm),
-         offsetof(lmatch_stats, tail_passes));
+         offsetof(lmatch_stats, tail_passes), offsetof(lmatch_opts, sort_chunk_log2));
   return 0; }'''
     tmp = os.path.join(ROOT, "build")
     os.makedirs(tmp, exist_ok=True)
@@ -73,7 +73,7 @@ int main(void){
     assert got == [ctypes.sizeof(O), ctypes.sizeof(S), S.weight.offset, S.ms_sweep.offset,
                    O.upload_chunk.offset, O.host_cache.offset, O.batches.offset,
                    S.cache_rows.offset, S.cache_bytes.offset, O.algorithm.offset,
-                   S.tail_passes.offset]
+                   S.tail_passes.offset, O.sort_chunk_log2.offset]
 
 
 def test_host_side_argument_errors(pkg):
@@ -95,7 +95,8 @@ def test_host_side_argument_errors(pkg):
     assert lib.lmatch_info(None, None, None, None, None) == pkg.LMATCH_ESTATE
     lib.lmatch_destroy(None)  # NULL-safe
     assert pkg.lmatch_strerror(pkg.LMATCH_EINVAL).startswith("invalid")
-    assert pkg.lmatch_abi_version() == 3
+    assert pkg.lmatch_abi_version() == 4
+    assert pkg.lmatch_strerror(pkg.LMATCH_EROUNDS).startswith("round cap")
     assert "n" in pkg.lmatch_last_error() or pkg.lmatch_last_error() == ""
 
 
