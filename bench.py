@@ -59,6 +59,8 @@ def parse():
     p.add_argument("--batches", type=int, default=0,
                    help="paper-style batch count N_i (lmatch_opts.batches): B > 1 streams the whole "
                         "adjacency from pinned host memory as B batches in round 1")
+    p.add_argument("--no-key-cache", action="store_true",
+                   help="resident: disable the round-1 top-4 key cache (lmatch_opts.key_cache = -1)")
     p.add_argument("--no-host-cache", action="store_true",
                    help="out-of-core: disable the top-8 host-row key cache (lmatch_opts.host_cache = -1)")
     p.add_argument("--algorithm", default="ld", choices=["ld", "suitor", "hybrid", "sorted"],
@@ -458,7 +460,7 @@ def main():
     opts = lm.make_opts(validate_level=1, timing=1,
                         hbm_budget_bytes=int(a.hbm_budget_gb * 1e9), stream_chunk=a.stream_chunk,
                         prune=a.prune, host_cache=not a.no_host_cache,
-                        batches=a.batches, algorithm=a.algorithm)
+                        batches=a.batches, algorithm=a.algorithm, key_cache=not a.no_key_cache)
     pinned_host = d_off is None
     if pinned_host:
         h = lm.lmatch_create_ex(g.offsets, g.col, g.w, n, m, opts)

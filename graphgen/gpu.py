@@ -151,6 +151,114 @@ def _edge_graph(kind, n, scale, M, seed, a, b, c, weights, wseed, device, bucket
     return DeviceGraph(offsets, col[:m], w[:m], n, m, name)
 
 
+def _edge_graph_rows(kind, n, scale, M, seed, a, b, c, weights, wseed, device, bucket_entries, name,
+                     rows=None, offsets=None):
+    """Row-range generation for one rank of a partitioned run (each rank holds only its rows):
+    rows=None -> pass 1: the graph's full CSR offsets (torch int64[n+1] on `device`; col/w of each
+    bucket go to scratch and are dropped); rows=(v0, v1) with the pass-1 offsets -> pass 2: the
+    local CSR of rows [v0, v1) (offsets rebased to 0, GLOBAL column ids), generating only the
+    buckets that hold those rows.  Same edges and weights as _edge_graph (same kernels)."""
+    import torch
+    L = _load()
+    dev = torch.device(device)
+    st = torch.cuda.current_stream(dev).cuda_stream
+    bits = max(1, (n - 1).bit_length())
+    nb = 1
+    while nb < 4096 and nb * bucket_entries < 2 * M and (nb << 1) <= (1 << bits):
+        nb <<= 1
+    shift = bits - (nb.bit_length() - 1)
+    counts = torch.zeros(nb, dtype=torch.int64, device=dev)
+    _ck(L.gg_cuda_count(kind, n, scale, seed, a, b, c, M, shift, nb, counts.data_ptr(), st), "count")
+    counts_h = counts.cpu().tolist()
+    maxc = max(counts_h) if counts_h else 0
+    keys = torch.empty(max(maxc, 1), dtype=torch.int64, device=dev)
+    alt = torch.empty(max(maxc, 1), dtype=torch.int64, device=dev)
+    temp = torch.empty(max(L.gg_cuda_temp_bytes(max(maxc, 1)), 1), dtype=torch.uint8, device=dev)
+    col_b = torch.empty(max(maxc, 1), dtype=torch.int32, device=dev)
+    w_b = torch.empty(max(maxc, 1), dtype=torch.float32, device=dev)
+    first = torch.full((n + 1,), INT64_MAX, dtype=torch.int64, device=dev)
+    cur = torch.zeros(1, dtype=torch.int64, device=dev)
+    nout = torch.zeros(1, dtype=torch.int64, device=dev)
+    mode = WEIGHT_MODES[weights]
+    ws = seed if wseed is None else wseed
+    which = ctypes.c_int(0)
+    if rows is not None:
+        v0, v1 = int(rows[0]), int(rows[1])
+        offs_h = offsets.cpu() if offsets.is_cuda else offsets
+        S, E = int(offs_h[v0]), int(offs_h[v1])
+        col = torch.empty(max(E - S, 1), dtype=torch.int32, device=dev)
+        w = torch.empty(max(E - S, 1), dtype=torch.float32, device=dev)
+    base = 0
+    for bkt in range(nb):
+        if counts_h[bkt] == 0:
+            continue
+        lo, hi = bkt << shift, min(n, (bkt + 1) << shift)
+        if rows is not None:
+            if hi <= v0 or lo >= v1:
+                continue
+            base = int(offs_h[lo])
+        cur.zero_()
+        _ck(L.gg_cuda_emit(kind, n, scale, seed, a, b, c, M, lo, hi, keys.data_ptr(),
+                           cur.data_ptr(), st), "emit")
+        _ck(L.gg_cuda_sort_unique(keys.data_ptr(), alt.data_ptr(), counts_h[bkt], 0, 32 + bits,
+                                  temp.data_ptr(), temp.numel(), nout.data_ptr(),
+                                  ctypes.byref(which), st), "sort_unique")
+        cu = int(nout.item())
+        src = keys if which.value == 0 else alt
+        _ck(L.gg_cuda_scatter_local(src.data_ptr(), cu, base, ws, mode, col_b.data_ptr(),
+                                    w_b.data_ptr(), first.data_ptr(), st), "scatter")
+        if rows is None:
+            base += cu
+        else:
+            g0, g1 = max(base, S), min(base + cu, E)
+            if g1 > g0:
+                col[g0 - S:g1 - S].copy_(col_b[g0 - base:g1 - base])
+                w[g0 - S:g1 - S].copy_(w_b[g0 - base:g1 - base])
+    del keys, alt, temp, col_b, w_b
+    if rows is None:
+        first[n] = base
+        offsets = torch.flip(torch.cummin(torch.flip(first, [0]), 0).values, [0]).contiguous()
+        torch.cuda.synchronize(dev)
+        return offsets
+    del first
+    loff = (offsets[v0:v1 + 1].to(dev) - S).contiguous()
+    torch.cuda.synchronize(dev)
+    return DeviceGraph(loff, col[:E - S], w[:E - S], v1 - v0, E - S, name + f"_rows{v0}-{v1}")
+
+
+def rmat_offsets(scale: int, edgefactor: int = 16, seed: int = 1, a: float = 0.57, b: float = 0.19,
+                 c: float = 0.19, device="cuda", bucket_entries: int = 1 << 28):
+    """CSR offsets (torch int64[n+1] on `device`) of rmat(scale, edgefactor, seed, ...)."""
+    n = 1 << scale
+    return _edge_graph_rows(1, n, scale, edgefactor * n, seed, a, b, c, "uniform", None, device,
+                            bucket_entries, f"rmat_s{scale}_ef{edgefactor}")
+
+
+def rmat_rows(scale: int, v0: int, v1: int, offsets, edgefactor: int = 16, seed: int = 1,
+              a: float = 0.57, b: float = 0.19, c: float = 0.19, weights: str = "uniform",
+              wseed: int | None = None, device="cuda", bucket_entries: int = 1 << 28) -> DeviceGraph:
+    """Rows [v0, v1) of rmat(scale, ...) as a local CSR (global column ids); `offsets` from
+    rmat_offsets.  n / m of the result are the LOCAL row and entry counts."""
+    n = 1 << scale
+    return _edge_graph_rows(1, n, scale, edgefactor * n, seed, a, b, c, weights, wseed, device,
+                            bucket_entries, f"rmat_s{scale}_ef{edgefactor}", (v0, v1), offsets)
+
+
+def er_offsets(n: int, avg_degree: float = 16.0, seed: int = 1, device="cuda",
+               bucket_entries: int = 1 << 28):
+    M = int(round(n * avg_degree / 2.0))
+    return _edge_graph_rows(0, n, 0, M, seed, 0.0, 0.0, 0.0, "uniform", None, device, bucket_entries,
+                            f"er_n{n}_d{avg_degree:g}")
+
+
+def er_rows(n: int, v0: int, v1: int, offsets, avg_degree: float = 16.0, seed: int = 1,
+            weights: str = "uniform", wseed: int | None = None, device="cuda",
+            bucket_entries: int = 1 << 28) -> DeviceGraph:
+    M = int(round(n * avg_degree / 2.0))
+    return _edge_graph_rows(0, n, 0, M, seed, 0.0, 0.0, 0.0, weights, wseed, device, bucket_entries,
+                            f"er_n{n}_d{avg_degree:g}", (v0, v1), offsets)
+
+
 def rmat(scale: int, edgefactor: int = 16, seed: int = 1, a: float = 0.57, b: float = 0.19,
          c: float = 0.19, weights: str = "uniform", wseed: int | None = None, device="cuda",
          bucket_entries: int = 1 << 28, host_out: bool = False) -> DeviceGraph:

@@ -58,7 +58,9 @@ typedef enum lmatch_status {
   LMATCH_ERANGE = -2, /* n >= 2^31 or n < 0 or m < 0 */
   LMATCH_ENOMEM = -3, /* device or pinned-host allocation failed */
   LMATCH_ECUDA = -4,  /* CUDA runtime / kernel failure (detail in lmatch_last_error) */
-  LMATCH_ENCCL = -5,  /* reserved for the multi-GPU exchange */
+  LMATCH_ENCCL = -5,  /* multi-GPU exchange failure: a rank did not join a lmatch_create_dist
+                         rendezvous or reach a device barrier in time, or the rendezvous
+                         could not be created */
   LMATCH_ESTATE = -6, /* misuse: NULL handle, size mismatch on reload, ... */
   LMATCH_EROUNDS = -7 /* the round cap (lmatch_opts.max_rounds) stopped the iteration with vertices
                          still to re-point: the contents of the mate output are unspecified.
@@ -155,7 +157,17 @@ typedef struct lmatch_opts {
                                  entries (a longer row is one chunk of its own); 0 = default (30).
                                  Valid 4..30 (EINVAL otherwise); small values exercise the chunking.
                                  Also caps the chunks of the validate_level-2 duplicate check */
-  int32_t reserved[6];
+  int32_t key_cache;          /* resident handles, algorithms 0 and 2:
+                                 0 = default (on when the cache fits in device memory), -1 = off.
+                                 The round-1 sweep keeps the 4 largest keys of every row (32 bytes
+                                 per vertex, plus 64 bytes per sweep tile of scratch); a vertex
+                                 whose target was matched then takes the first available cached
+                                 key as its new pointer -- Alg. 1's pointer, since every larger key
+                                 of the row is cached and matched -- and only rows whose cached
+                                 keys are all matched are scanned again.  Same result, same
+                                 pointing phases; lmatch_stats.entries_swept counts the rows
+                                 actually scanned, cache_rows the pointers the cache decided */
+  int32_t reserved[5];
 } lmatch_opts;
 
 /* Filled by lmatch_run / lmatch_run_device when non-NULL. */
@@ -179,8 +191,9 @@ typedef struct lmatch_stats {
   int64_t kernel_launches;   /* all kernel launches issued by this run */
   int64_t bytes_streamed;    /* host->device adjacency bytes copied by this run (out-of-core) */
   int64_t resident_entries;  /* adjacency entries resident in HBM (= m unless out-of-core) */
-  int64_t cache_rows;        /* out-of-core host-row cache: frontier rows whose pointer the
-                                cache decided in rounds >= 2 (no host read) */
+  int64_t cache_rows;        /* rounds >= 2: frontier rows whose pointer a key cache decided
+                                without scanning the row (out of core: the host-row cache;
+                                resident: the key cache, opts.key_cache) */
   int64_t host_entries_read; /* out-of-core: host-resident entries read zero-copy in rounds >= 2 */
   int64_t cache_bytes;       /* out-of-core: device bytes of the host-row cache (0 = none) */
   int64_t tail_passes;       /* algorithm 2: Suitor passes that completed the run after the LD
@@ -355,6 +368,69 @@ LMATCH_API int lmatch_p2p_compact(lmatch_graph* g, void* stream, int64_t* nF_loc
 LMATCH_API int lmatch_p2p_frontier_total(lmatch_graph* g, void* stream, int64_t* nF_total);
 /* Synchronise `stream` (NULL = the handle's stream): the caller's half of a barrier. */
 LMATCH_API int lmatch_p2p_sync(lmatch_graph* g, void* stream);
+
+/* ---------------------------------------------------------------------------------------------
+ * Library-owned multi-GPU driver (SURVEY 8(b) lmatch_create_dist, 8(e)).  One process (or one
+ * thread) per GPU calls these; the library partitions, sets up the peer-memory exchange above by
+ * itself and runs the whole round loop -- Alg. 2's per-device loop with the exchange
+ * redesigned (claims into the owners' inboxes instead of nccl_AllReduce(pointers); changed
+ * bitmap words instead of nccl_AllReduce(mate); frontier sizes for termination).
+ * The phases of a round are separated by DEVICE-side barriers over the exchange windows
+ * (system-scope release/acquire flags stored into the peers' memory), so no host barrier is
+ * involved; each rank reads one value set per round (the P frontier sizes).
+ * ------------------------------------------------------------------------------------------- */
+
+/* Edge-balanced 1-D partition of a CSR ("binary search on the prefix sums"): bounds[0] = 0,
+ * bounds[nparts] = n, and for 0 < p < nparts bounds[p] = the first row whose start offset reaches
+ * floor(m p / nparts), rounded up to a multiple of `align` (0 = 32: each matched-bitmap word then
+ * has one owner) and kept non-decreasing.  csr_offsets: HOST int64[n+1]; bounds: HOST
+ * int64[nparts+1], caller-allocated.  Host-only (no CUDA call).  EINVAL on NULL / offsets[0] != 0
+ * / nparts < 1; ERANGE on n out of [0, 2^31). */
+LMATCH_API int lmatch_partition(const int64_t* csr_offsets, int64_t n, int32_t nparts, int32_t align,
+                                int64_t* bounds);
+
+/* Rendezvous name shared by the ranks of one lmatch_create_dist group (like an ncclUniqueId):
+ * one rank creates it with lmatch_dist_id_new and sends the 64 bytes to the others (e.g. a
+ * torch.distributed broadcast).  The ranks meet in a POSIX shared-memory segment named after it
+ * (one node), which the last rank to attach removes.  Host-only. */
+typedef struct lmatch_dist_id {
+  char bytes[64];
+} lmatch_dist_id;
+LMATCH_API int lmatch_dist_id_new(lmatch_dist_id* id);
+
+/* Rank `rank` of `world` creates its part: rows [v_begin, v_begin + n_local) of a graph with
+ * n_global vertices, given as a HOST local CSR whose col_idx are GLOBAL ids (cut edges appear in
+ * both owners' rows); part_bounds: HOST int64[world+1] as lmatch_partition returns (every
+ * rank passes the same bounds; v_begin must be part_bounds[rank]).  Blocks until all `world`
+ * ranks of `id` have joined (ENCCL after 60 s), then opens every peer's exchange window: plain
+ * device pointers for ranks in the same process (peer access enabled across devices), CUDA IPC
+ * for other processes.  opts: as for lmatch_create_ex, except validate_level 2, hbm_budget_bytes
+ * and algorithm != 0 (EINVAL).  The returned handle is used with lmatch_run_dist* and
+ * lmatch_destroy (and lmatch_info / lmatch_reload); it is a partition handle, so the
+ * lmatch_part_* / lmatch_p2p_* calls return ESTATE or act on the same state -- do not mix. */
+LMATCH_API int lmatch_create_dist(const int64_t* csr_offsets, const int32_t* col_idx,
+                                  const float* weights, int64_t n_local, int64_t m_local,
+                                  int64_t v_begin, int64_t n_global, int32_t rank, int32_t world,
+                                  const int64_t* part_bounds, const lmatch_dist_id* id,
+                                  const lmatch_opts* opts, lmatch_graph** out);
+/* Same with the three local arrays on the DEVICE (ordered on `stream`). */
+LMATCH_API int lmatch_create_dist_device(const int64_t* d_offsets, const int32_t* d_col,
+                                         const float* d_weights, int64_t n_local, int64_t m_local,
+                                         int64_t v_begin, int64_t n_global, int32_t rank,
+                                         int32_t world, const int64_t* part_bounds,
+                                         const lmatch_dist_id* id, const lmatch_opts* opts,
+                                         void* stream, lmatch_graph** out);
+/* Every rank calls it (collective): the whole matching.  d_mate_local: DEVICE int32[n_local], the
+ * owned slice of mate[] (global ids, -1 = unmatched).  stats (optional): rounds = pointing phases,
+ * cardinality / matched_vertices / weight = the WHOLE graph's (every rank's share summed in rank
+ * order, so every rank gets the same fp64 w(M)), entries_swept / kernel_launches / ms_* = this
+ * rank's.  The result is bit-identical to the single-GPU run for every partition (Lemma III.1,
+ * P:167-175).  Synchronises `stream` (NULL = the handle's stream).  ENCCL if a peer does not reach
+ * a device barrier within 60 s; EROUNDS as for lmatch_run. */
+LMATCH_API int lmatch_run_dist_device(lmatch_graph* g, int32_t* d_mate_local, void* stream,
+                                      lmatch_stats* stats);
+/* Same with a HOST int32[n_local] output. */
+LMATCH_API int lmatch_run_dist(lmatch_graph* g, int32_t* mate_local, lmatch_stats* stats);
 
 /* Release everything the handle owns.  NULL-safe. */
 LMATCH_API void lmatch_destroy(lmatch_graph* g);

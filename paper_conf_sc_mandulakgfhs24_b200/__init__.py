@@ -46,7 +46,7 @@ class Opts(ctypes.Structure):
         ("round_loop", ctypes.c_int32), ("prune", ctypes.c_int32),
         ("host_cache", ctypes.c_int32), ("batches", ctypes.c_int32),
         ("algorithm", ctypes.c_int32), ("sort_chunk_log2", ctypes.c_int32),
-        ("reserved", ctypes.c_int32 * 6),
+        ("key_cache", ctypes.c_int32), ("reserved", ctypes.c_int32 * 5),
     ]
 
 
@@ -245,7 +245,8 @@ class Matcher:
                  validate_level: int = 1, timing: bool = False, upload_chunk: int = 0,
                  max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
                  round_loop: int = 0, prune: bool = False, host_cache: bool = True,
-                 batches: int = 0, algorithm: str = "ld", sort_chunk_log2: int = 0):
+                 batches: int = 0, algorithm: str = "ld", sort_chunk_log2: int = 0,
+                 key_cache: bool = True):
         self.h = None
         if handle is not None:
             self.h = handle
@@ -256,7 +257,7 @@ class Matcher:
                                       opts=make_opts(validate_level, timing, upload_chunk,
                                                      max_rounds, hbm_budget_bytes, stream_chunk,
                                                      round_loop, prune, host_cache, batches,
-                                                     algorithm, sort_chunk_log2))
+                                                     algorithm, sort_chunk_log2, key_cache))
         self.info = lmatch_info(self.h)
 
     @classmethod
@@ -301,7 +302,8 @@ class Matcher:
 def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int = 0,
               max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
               round_loop: int = 0, prune: bool = False, host_cache: bool = True,
-              batches: int = 0, algorithm: str = "ld", sort_chunk_log2: int = 0) -> Opts:
+              batches: int = 0, algorithm: str = "ld", sort_chunk_log2: int = 0,
+              key_cache: bool = True) -> Opts:
     """round_loop (include/lmatch.h): 0 = hybrid (work-sized launches, then one persistent kernel
     for the tail; default), 1 = host-driven launches only, 2 = persistent kernel after round 1,
     3 = CUDA graph {round 1, persistent kernel}."""
@@ -312,6 +314,7 @@ def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int =
     o.batches = int(batches)
     o.algorithm = {"ld": 0, "suitor": 1, "hybrid": 2, "sorted": 3}[algorithm]
     o.sort_chunk_log2 = int(sort_chunk_log2)
+    o.key_cache = 0 if key_cache else -1
     o.hbm_budget_bytes = int(hbm_budget_bytes)
     o.stream_chunk = int(stream_chunk)
     o.validate_level = int(validate_level)

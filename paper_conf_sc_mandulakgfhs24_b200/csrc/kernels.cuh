@@ -26,7 +26,9 @@ namespace lm {
 
 namespace cg = cooperative_groups;
 
-constexpr int kBins = 4;               // frontier degree bins
+constexpr int kDegBins = 4;            // frontier degree bins (rows scanned by the pointer kernels)
+constexpr int kDecided = 4;            // frontier list of rows whose pointer the key cache decided
+constexpr int kBins = 5;               // frontier lists: the degree bins + the decided list
 #ifndef LM_BIN0
 #define LM_BIN0 8
 #endif
@@ -121,6 +123,38 @@ __device__ __forceinline__ uint64_t group_max_key(uint64_t key, unsigned mask) {
   const uint32_t mlo = __reduce_max_sync(mask, lo);
   return ((uint64_t)mhi << 32) | mlo;
 }
+// insert x into a descending register list (keeps the K largest)
+template <int K>
+__device__ __forceinline__ void topk_insert(uint64_t (&t)[K], uint64_t x) {
+#pragma unroll
+  for (int i = 0; i < K; ++i) {
+    const uint64_t a = t[i];
+    const bool gt = x > a;
+    t[i] = gt ? x : a;
+    x = gt ? a : x;
+  }
+}
+
+// K warp-wide pops of the per-lane descending lists: lane r < K receives the r-th largest key
+// (u64 max; equal keys of a repeated edge are popped one at a time).
+template <int K>
+__device__ __forceinline__ uint64_t warp_topk_pop(uint64_t (&t)[K]) {
+  const int lane = threadIdx.x & 31;
+  uint64_t mine = 0ull;
+#pragma unroll
+  for (int r = 0; r < K; ++r) {
+    const uint64_t mx = group_max_key(t[0], 0xffffffffu);
+    if (lane == r) mine = mx;
+    const unsigned own = __ballot_sync(0xffffffffu, mx != 0ull && t[0] == mx);
+    if (own && lane == __ffs(own) - 1) {
+#pragma unroll
+      for (int i = 0; i < K - 1; ++i) t[i] = t[i + 1];
+      t[K - 1] = 0ull;
+    }
+  }
+  return mine;
+}
+
 __device__ __forceinline__ int bin_of(int64_t deg) {
   return deg <= kBinDeg0 ? 0 : deg <= kBinDeg1 ? 1 : deg <= kBinDeg2 ? 2 : 3;
 }
@@ -235,13 +269,13 @@ __global__ void k_zap_self_loops(const int64_t* __restrict__ offs, AdjView adj, 
 // number of vertices in each frontier degree bin (static capacity of the bin lists)
 __global__ void k_bin_sizes(const int64_t* __restrict__ offs, int64_t n, unsigned long long* cnt) {
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  unsigned long long c[kBins] = {0, 0, 0, 0};
+  unsigned long long c[kDegBins] = {0, 0, 0, 0};
   for (int64_t u = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; u < n; u += stride) {
     const int64_t d = offs[u + 1] - offs[u];
     if (d > 0) ++c[bin_of(d)];
   }
 #pragma unroll
-  for (int b = 0; b < kBins; ++b) {
+  for (int b = 0; b < kDegBins; ++b) {
     for (int o = 16; o; o >>= 1) c[b] += __shfl_xor_sync(0xffffffffu, c[b], o);
     if ((threadIdx.x & 31) == 0 && c[b]) atomicAdd(&cnt[b], c[b]);
   }
@@ -465,6 +499,27 @@ __device__ __forceinline__ uint64_t umax_skip(uint64_t b, uint64_t key, uint32_t
   return ((uint32_t)key != self && key > b) ? key : b;
 }
 
+// Resident key cache ("key cache"): the round-1 sweep also keeps the kKC
+// largest keys of every row, descending (0-padded), in kc[u][0..kKC).  From round 2 on, a vertex
+// whose target was matched takes its new pointer from the cache when one of them is available:
+// every key of the row above the first available cached key is cached and matched, and matched
+// is permanent (R3), so that key is the row maximum over available neighbours -- exactly Alg. 1's
+// pointer (L4).  Only rows whose cached keys are all matched (and that hold more than the
+// cached keys) are scanned again.  A row crossing a sweep tile writes its per-tile top-kKC into
+// xpart[tile][slot] (slot 0: the row began before the tile; 1: it continues after it), merged by
+// k_kc_merge.
+constexpr int kKC = 4;
+// insert key k into the descending list t0 >= t1 >= t2 >= t3 (keeps the kKC largest)
+__device__ __forceinline__ void top4_insert(uint64_t& t0, uint64_t& t1, uint64_t& t2, uint64_t& t3,
+                                            uint64_t k) {
+  if (k > t3) {
+    t3 = k;
+    if (t3 > t2) { const uint64_t x = t2; t2 = t3; t3 = x; }
+    if (t2 > t1) { const uint64_t x = t1; t1 = t2; t2 = x; }
+    if (t1 > t0) { const uint64_t x = t0; t0 = t1; t1 = x; }
+  }
+}
+
 struct SweepArgs {
   const uint64_t* adj;       // keys of entry tile_begin*TILE onward (HBM or a streamed chunk)
   uint64_t* zap;             // ZAP variant only: writable adjacency (self-loop keys -> 0)
@@ -477,6 +532,8 @@ struct SweepArgs {
   int64_t m;
   int64_t tile_begin;        // tiles [tile_begin, ntiles) of this launch
   int64_t ntiles;
+  uint64_t* kc = nullptr;    // KC variant: key cache [n][kKC]
+  uint64_t* xpart = nullptr; // KC variant: per-tile partial lists of crossing rows [ntiles][2][kKC]
 };
 
 template <int TILE, int RING, int WARPS, int WCAP>
@@ -495,7 +552,7 @@ struct SweepCfg {
   static_assert(kStageBytes % 16 == 0 && kWarpBytes % 16 == 0, "TMA needs 16-byte alignment");
 };
 
-template <int TILE, int RING, int WARPS, int WCAP, bool ZAP = false>
+template <int TILE, int RING, int WARPS, int WCAP, bool ZAP = false, bool KC = false>
 __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
   // ZAP: the one-time ingest pass -- same tiles and rows, but instead of the max it zeroes the
   // keys of self-loops (col == row; simple graph) in place.
@@ -642,7 +699,22 @@ __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
       }
       if (L > 0 && L < 8) {
 #else
-      if (L > 0 && L < LM_SWEEP_LONG) {
+      if (KC && L > 0 && L < LM_SWEEP_LONG) {
+        // the row's 4 largest keys (descending); rows wholly in the tile store them in the cache
+        uint64_t t0 = 0, t1 = 0, t2 = 0, t3 = 0;
+        for (int j = max(rs, 0), je = min(re, len); j < je; ++j) top4_insert(t0, t1, t2, t3, K[j]);
+        if (inside) {
+          A.best[vid] = t0;
+          ulonglong2* c = reinterpret_cast<ulonglong2*>(A.kc + (size_t)vid * kKC);
+          c[0] = make_ulonglong2(t0, t1);
+          c[1] = make_ulonglong2(t2, t3);
+        } else {
+          ulonglong2* c = reinterpret_cast<ulonglong2*>(A.xpart + ((size_t)t * 2 + (rs < 0 ? 0 : 1)) * kKC);
+          c[0] = make_ulonglong2(t0, t1);
+          c[1] = make_ulonglong2(t2, t3);
+        }
+      }
+      if (!KC && L > 0 && L < LM_SWEEP_LONG) {
 #endif
         uint64_t b0 = 0, b1 = 0, b2 = 0, b3 = 0;  // 4 independent max chains
         int j = max(rs, 0);
@@ -669,6 +741,18 @@ __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
         const int32_t jb = __shfl_sync(0xffffffffu, min(re, len), l);
         const uint32_t v = __shfl_sync(0xffffffffu, vid, l);
         const bool ins = __shfl_sync(0xffffffffu, (int)inside, l) != 0;
+        if (KC) {
+          // per-lane top 4 over the lane's keys, then 4 warp-wide pops: lane q < 4 holds the
+          // row segment's q-th largest key
+          uint64_t tt[kKC] = {0, 0, 0, 0};
+          for (int j = ja + lane; j < jb; j += 32) top4_insert(tt[0], tt[1], tt[2], tt[3], K[j]);
+          const uint64_t mine = warp_topk_pop<kKC>(tt);
+          const bool rs_neg = __shfl_sync(0xffffffffu, (int)(rs < 0), l) != 0;
+          uint64_t* dst = ins ? A.kc + (size_t)v * kKC : A.xpart + ((size_t)t * 2 + (rs_neg ? 0 : 1)) * kKC;
+          if (lane < kKC) dst[lane] = mine;
+          if (ins && lane == 0) A.best[v] = mine;
+          continue;
+        }
         uint64_t b0 = 0, b1 = 0, b2 = 0, b3 = 0;  // 4 independent max chains
         int j = ja + lane;
         for (; j + 96 < jb; j += 128) {
@@ -938,6 +1022,46 @@ __global__ void k_atomic_rows(const int64_t* __restrict__ noffs, const int32_t* 
   }
 }
 
+// key cache: the non-empty rows (nz index) that cross a sweep-tile boundary, each listed once
+__global__ void k_kc_xrows(const int64_t* __restrict__ noffs, int64_t n_nz, int64_t tile,
+                           int32_t* out, unsigned long long* count) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t lim = (n_nz + 31) & ~31ll;
+  for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < lim; r += stride) {
+    const bool cross = r < n_nz && noffs[r] / tile != (noffs[r + 1] - 1) / tile;
+    warp_append(cross, (int32_t)r, out, count);
+  }
+}
+// key cache: merge the per-tile partial top-kKC lists of every crossing row (tiles tf..tl; the
+// row continues after tile tf -> slot 1 there, began before every later tile -> slot 0) into its
+// cache line and its pointer best[u] (the row maximum).  One warp per row.
+__global__ void k_kc_merge(const int32_t* __restrict__ xrows, const unsigned long long* __restrict__ nx,
+                           const int64_t* __restrict__ noffs, const int32_t* __restrict__ nzr,
+                           const uint64_t* __restrict__ xpart, int64_t tile, uint64_t* __restrict__ kc,
+                           uint64_t* __restrict__ best) {
+  const int lane = threadIdx.x & 31;
+  const int64_t cnt = (int64_t)*nx;
+  const int64_t w0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t ws = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t i = w0; i < cnt; i += ws) {
+    const int64_t r = xrows[i];
+    const int64_t tf = noffs[r] / tile, tl = (noffs[r + 1] - 1) / tile;
+    uint64_t t[kKC] = {0, 0, 0, 0};
+    for (int64_t tt = tf + lane; tt <= tl; tt += 32) {
+      const ulonglong2* p = reinterpret_cast<const ulonglong2*>(xpart + ((size_t)tt * 2 + (tt == tf ? 1 : 0)) * kKC);
+      const ulonglong2 a = p[0], b = p[1];
+      topk_insert<kKC>(t, a.x);
+      topk_insert<kKC>(t, a.y);
+      topk_insert<kKC>(t, b.x);
+      topk_insert<kKC>(t, b.y);
+    }
+    const uint64_t mine = warp_topk_pop<kKC>(t);
+    const uint32_t u = (uint32_t)nzr[r];
+    if (lane < kKC) kc[(size_t)u * kKC + lane] = mine;
+    if (lane == 0) best[u] = mine;
+  }
+}
+
 __global__ void k_low32(const int64_t* __restrict__ noffs, int64_t cnt, uint32_t* lo) {
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < cnt; i += stride)
@@ -1000,6 +1124,8 @@ struct RoundArgs {
   RoundState* st;
   long long* log;           // [log_cap][3]: |F_r|, |S_r| + |F_r|, E(F_r)
   uint32_t* live;           // A7 pruning: per-vertex live counts (nullptr = pruning off)
+  const uint64_t* kc;       // resident key cache [n][kKC] (nullptr = off)
+  uint64_t* best;           // per-vertex pointers (the compaction writes the cache-decided ones)
 };
 
 // A2 pointer phase on the frontier (rounds >= 2): G lanes per vertex (degree-binned).
@@ -1669,12 +1795,14 @@ struct CompactIO {
   Bins Fin;
   uint64_t* Sout;
   Bins Fout;
-  const unsigned long long* cin;  // counters of the input set (cnt_S .. cnt_F(.,3) contiguous)
+  const unsigned long long* cin;  // counters of the input set (cnt_S .. cnt_F(.,kBins-1) contiguous)
   unsigned long long* cout;       // counters of the output set
   unsigned long long* swept;
   const uint32_t* live;           // A7: live counts (nullptr = pruning off)
   const RoundState* st;
   const int32_t* nzr;             // ALL mode: iterate the non-empty rows only (nullptr = all n)
+  const uint64_t* kc;             // key cache [n][kKC] (nullptr = off)
+  uint64_t* best_w;               // key cache: pointers decided by the compaction (= best)
 };
 __host__ __device__ inline CompactIO compact_io(const RoundArgs& a, int cur) {
   CompactIO io;
@@ -1688,7 +1816,28 @@ __host__ __device__ inline CompactIO compact_io(const RoundArgs& a, int cur) {
   io.live = a.live;
   io.st = a.st;
   io.nzr = nullptr;
+  io.kc = a.kc;
+  io.best_w = a.best;
   return io;
+}
+
+// key cache: the new pointer of frontier vertex u from its cached keys, as Alg. 1 L4 would
+// compute it now (the bitmap holds every match up to this round): the first available cached key
+// (descending), or "none" when the row has fewer than kKC keys and all are matched (the cache
+// holds the whole row).  Returns false when the row must be scanned.
+__device__ __forceinline__ bool kc_decide(const uint64_t* __restrict__ kc, const uint32_t* __restrict__ bits,
+                                          int64_t lu, uint64_t* key) {
+  const ulonglong2* c = reinterpret_cast<const ulonglong2*>(kc + (size_t)lu * kKC);
+  const ulonglong2 c01 = c[0], c23 = c[1];
+  const uint64_t k[kKC] = {c01.x, c01.y, c23.x, c23.y};
+  uint32_t wd[kKC];
+#pragma unroll
+  for (int q = 0; q < kKC; ++q) wd[q] = k[q] ? bits[(uint32_t)k[q] >> 5] : 0xffffffffu;
+#pragma unroll
+  for (int q = 0; q < kKC; ++q)
+    if (k[q] && !((wd[q] >> ((uint32_t)k[q] & 31)) & 1u)) { *key = k[q]; return true; }
+  *key = 0;
+  return k[kKC - 1] == 0;
 }
 
 template <bool ALL, int K>
@@ -1709,25 +1858,26 @@ __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
   unsigned long long* swept = io.swept;  // warps per block (blockDim 256), output lists
   __shared__ unsigned wtot[NW][NL];
   __shared__ unsigned long long wbase[NW][NL];
-  // virtual concatenation S ++ F_0 ++ F_1 ++ F_2 ++ F_3 (prefix ends p0 < p1 < ... < p4)
-  const int64_t p0 = ALL ? n : (int64_t)*cntS;
-  const int64_t p1 = p0 + (ALL ? 0 : (int64_t)cntFin[0]);
-  const int64_t p2 = p1 + (ALL ? 0 : (int64_t)cntFin[1]);
-  const int64_t p3 = p2 + (ALL ? 0 : (int64_t)cntFin[2]);
-  const int64_t cnt = p3 + (ALL ? 0 : (int64_t)cntFin[3]);
+  // virtual concatenation S ++ F_0 ++ ... ++ F_{kBins-1} (prefix ends p[0] < p[1] < ...)
+  int64_t pe[kBins + 1];
+  pe[0] = ALL ? n : (int64_t)*cntS;
+#pragma unroll
+  for (int q = 0; q < kBins; ++q) pe[q + 1] = pe[q] + (ALL ? 0 : (int64_t)cntFin[q]);
+  const int64_t cnt = pe[kBins];
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const unsigned lt = lanemask_lt();
   const uint32_t* __restrict__ lcnt = io.live;
   const uint32_t tag = lcnt ? round_tag(io.st) : 0u;
   constexpr int64_t BLK = (int64_t)NW * 32 * K;
-  unsigned long long degsum = 0;
+  unsigned long long degsum = 0, decided = 0;
   for (int64_t cb = bid * BLK; cb < cnt; cb += nblk * BLK) {
     const int64_t c0 = cb + (int64_t)warp * 32 * K;
-    uint32_t sbits = 0, fb0 = 0, fb1 = 0, fb2 = 0, fb3 = 0;
+    uint32_t sbits = 0, fb[kBins] = {0, 0, 0, 0, 0};
     uint64_t pr[K], rr[K];
     // phase 1: every list element of the chunk (independent loads)
 #pragma unroll
     for (int k = 0; k < K; ++k) {
+      rr[k] = 0;
       const int64_t i = c0 + 32 * k + lane;
       uint64_t p = (uint64_t)kNoPtr << 32;
       if (i < cnt) {
@@ -1737,11 +1887,12 @@ __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
           const uint64_t bb = best[r];
           p = make_pair((uint32_t)(r + vbase), bb ? (uint32_t)bb : kNoPtr);
         } else {
-          p = i < p0 ? S[i]
-              : i < p1 ? Fin.list[0][i - p0].x
-              : i < p2 ? Fin.list[1][i - p1].x
-              : i < p3 ? Fin.list[2][i - p2].x
-                       : Fin.list[3][i - p3].x;
+          p = i < pe[0] ? S[i]
+              : i < pe[1] ? Fin.list[0][i - pe[0]].x
+              : i < pe[2] ? Fin.list[1][i - pe[1]].x
+              : i < pe[3] ? Fin.list[2][i - pe[2]].x
+              : i < pe[4] ? Fin.list[3][i - pe[3]].x
+                          : Fin.list[4][i - pe[4]].x;
         }
       }
       pr[k] = p;
@@ -1755,15 +1906,36 @@ __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
       wu[k] = ok ? bits[u >> 5] : 0xffffffffu;
       wv[k] = ok ? bits[v >> 5] : 0u;
     }
-    // phase 3: classify; frontier members fetch their row range (independent loads)
-    int64_t os[K], oe[K];
+    // phase 3: classify; frontier members take their pointer from the key cache when it decides
+    // it (-> the decided list), else fetch their row range (-> a degree bin)
+    uint32_t frm = 0;
 #pragma unroll
     for (int k = 0; k < K; ++k) {
       const uint32_t u = (uint32_t)pr[k], v = (uint32_t)(pr[k] >> 32);
       const bool live = !((wu[k] >> (u & 31)) & 1u);
       const bool tgt = (wv[k] >> (v & 31)) & 1u;
       if (live && !tgt) sbits |= 1u << k;
-      const bool fr = live && tgt;
+      if (live && tgt) frm |= 1u << k;
+    }
+    if (io.kc) {
+#pragma unroll
+      for (int k = 0; k < K; ++k) {
+        if (!(frm & (1u << k))) continue;
+        const uint32_t u = (uint32_t)pr[k];
+        uint64_t key;
+        if (kc_decide(io.kc, bits, (int64_t)u - vbase, &key)) {
+          frm &= ~(1u << k);
+          fb[kDecided] |= 1u << k;
+          pr[k] = make_pair(u, key ? (uint32_t)key : kNoPtr);
+          io.best_w[(int64_t)u - vbase] = key;
+        }
+      }
+    }
+    int64_t os[K], oe[K];
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+      const uint32_t u = (uint32_t)pr[k];
+      const bool fr = (frm >> k) & 1u;
       os[k] = fr ? offs[u - vbase] : 0;
       oe[k] = fr ? offs[u - vbase + 1] : -1;
       if (lcnt && fr) {  // A7: a row pruned earlier in this run is scanned over its live prefix
@@ -1773,29 +1945,25 @@ __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
     }
 #pragma unroll
     for (int k = 0; k < K; ++k) {
-      rr[k] = 0;
       if (oe[k] >= 0) {
         const int64_t d = oe[k] - os[k];
         const int b = bin_of(d);
         const uint32_t m = 1u << k;
-        fb0 |= b == 0 ? m : 0u;
-        fb1 |= b == 1 ? m : 0u;
-        fb2 |= b == 2 ? m : 0u;
-        fb3 |= b == 3 ? m : 0u;
+#pragma unroll
+        for (int q = 0; q < kDegBins; ++q) fb[q] |= b == q ? m : 0u;
         rr[k] = (uint64_t)os[k] | ((uint64_t)(d < (int64_t)kBigDeg ? d : (int64_t)kBigDeg) << 40);
         degsum += (unsigned long long)d;
       }
     }
+    decided += (unsigned long long)__popc(fb[kDecided]);
     // reserve output ranges: warp totals -> block prefix -> ONE atomic per list per block
     {
       const unsigned ts = __reduce_add_sync(0xffffffffu, __popc(sbits));
-      const unsigned t0 = __reduce_add_sync(0xffffffffu, __popc(fb0));
-      const unsigned t1 = __reduce_add_sync(0xffffffffu, __popc(fb1));
-      const unsigned t2 = __reduce_add_sync(0xffffffffu, __popc(fb2));
-      const unsigned t3 = __reduce_add_sync(0xffffffffu, __popc(fb3));
-      if (lane == 0) {
-        wtot[warp][0] = ts; wtot[warp][1] = t0; wtot[warp][2] = t1;
-        wtot[warp][3] = t2; wtot[warp][4] = t3;
+      if (lane == 0) wtot[warp][0] = ts;
+#pragma unroll
+      for (int q = 0; q < kBins; ++q) {
+        const unsigned tq = __reduce_add_sync(0xffffffffu, __popc(fb[q]));
+        if (lane == 0) wtot[warp][1 + q] = tq;
       }
     }
     __syncthreads();
@@ -1808,8 +1976,9 @@ __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
       for (int w = 0; w < NW; ++w) { wbase[w][q] = base; base += wtot[w][q]; }
     }
     __syncthreads();
-    unsigned long long bs = wbase[warp][0], bf0 = wbase[warp][1], bf1 = wbase[warp][2],
-                       bf2 = wbase[warp][3], bf3 = wbase[warp][4];
+    unsigned long long bs = wbase[warp][0], bf[kBins];
+#pragma unroll
+    for (int q = 0; q < kBins; ++q) bf[q] = wbase[warp][1 + q];
 #pragma unroll
     for (int k = 0; k < K; ++k) {
       const uint32_t m = 1u << k;
@@ -1818,22 +1987,20 @@ __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
       if (ps) Sout[bs + __popc(bls & lt)] = pr[k];
       bs += __popc(bls);
       const ulonglong2 ent = make_ulonglong2(pr[k], rr[k]);
-      unsigned bb = __ballot_sync(0xffffffffu, (fb0 & m) != 0);
-      if (fb0 & m) Fout.list[0][bf0 + __popc(bb & lt)] = ent;
-      bf0 += __popc(bb);
-      bb = __ballot_sync(0xffffffffu, (fb1 & m) != 0);
-      if (fb1 & m) Fout.list[1][bf1 + __popc(bb & lt)] = ent;
-      bf1 += __popc(bb);
-      bb = __ballot_sync(0xffffffffu, (fb2 & m) != 0);
-      if (fb2 & m) Fout.list[2][bf2 + __popc(bb & lt)] = ent;
-      bf2 += __popc(bb);
-      bb = __ballot_sync(0xffffffffu, (fb3 & m) != 0);
-      if (fb3 & m) Fout.list[3][bf3 + __popc(bb & lt)] = ent;
-      bf3 += __popc(bb);
+#pragma unroll
+      for (int q = 0; q < kBins; ++q) {
+        const unsigned bb = __ballot_sync(0xffffffffu, (fb[q] & m) != 0);
+        if (fb[q] & m) Fout.list[q][bf[q] + __popc(bb & lt)] = ent;
+        bf[q] += __popc(bb);
+      }
     }
   }
-  for (int o = 16; o; o >>= 1) degsum += __shfl_xor_sync(0xffffffffu, degsum, o);
+  for (int o = 16; o; o >>= 1) {
+    degsum += __shfl_xor_sync(0xffffffffu, degsum, o);
+    decided += __shfl_xor_sync(0xffffffffu, decided, o);
+  }
   if (lane == 0 && degsum) atomicAdd(swept, degsum);
+  if (lane == 0 && decided) atomicAdd(swept + (kCntCache - kCntSwept), decided);
 }
 template <bool ALL, int K>
 #ifndef LM_COMPACT_MINB
@@ -2090,6 +2257,61 @@ __global__ void k_push_count(const unsigned long long* __restrict__ cnt, int ncn
   }
 }
 
+// ---- library-owned multi-GPU driver (lmatch_create_dist / lmatch_run_dist): a device-side
+// barrier over the exchange windows, so no host barrier separates the phases of a round.
+// Part `me` stores the barrier's epoch into slot [me] of every peer's flag array with a
+// system-scope release (after a system-scope fence: the claims and bitmap words this GPU stored
+// into peer memory before the barrier are visible to the peer when it sees the flag), then
+// waits until every peer's epoch has arrived in its own array (system-scope acquire).  One
+// thread; a peer missing for `timeout_ns` sets *err and returns (the host reports ENCCL) instead
+// of hanging the GPU.
+__device__ __forceinline__ void st_release_sys(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned long long global_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__global__ void k_dist_barrier(const unsigned long long* my_flags,
+                               unsigned long long* const* __restrict__ peer_flag, int P, int me,
+                               unsigned long long epoch, unsigned long long timeout_ns,
+                               unsigned* err) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  __threadfence_system();
+  for (int p = 0; p < P; ++p)
+    if (p != me) st_release_sys(peer_flag[p], epoch);
+  const unsigned long long t0 = global_ns();
+  for (int q = 0; q < P; ++q) {
+    if (q == me) continue;
+    while (ld_acquire_sys(my_flags + q) < epoch) {
+      if (global_ns() - t0 > timeout_ns) {
+        atomicOr(err, 1u);
+        return;
+      }
+      __nanosleep(256);
+    }
+  }
+}
+// this part's w(M) share and matched count into every part's result slots [me] (fp64 bits), so
+// each part sums the P shares in part order after a barrier (same total on every part)
+__global__ void k_push_result(const double* __restrict__ w, const long long* __restrict__ c,
+                              unsigned long long* const* __restrict__ peer_w,
+                              unsigned long long* const* __restrict__ peer_c, int P) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  const unsigned long long wb = (unsigned long long)__double_as_longlong(*w);
+  const unsigned long long cb = (unsigned long long)*c;
+  for (int p = 0; p < P; ++p) {
+    peer_w[p][0] = wb;
+    peer_c[p][0] = cb;
+  }
+}
+
 // round 1 match over every owned vertex (owned range starts on a 32-vertex boundary)
 __global__ void k_match_part_all(const uint64_t* __restrict__ best, int64_t n_loc, int64_t vbase,
                                  int64_t vend, const uint32_t* __restrict__ ghost, uint32_t* bits) {
@@ -2272,38 +2494,6 @@ __global__ void k_rows_of_entries(const int64_t* __restrict__ offs, int64_t n, i
   if (k < cnt) out[k] = row_of_entry(offs, n, min(first + k * step, last));
 }
 
-// insert x into a descending register list (keeps the K largest)
-template <int K>
-__device__ __forceinline__ void topk_insert(uint64_t (&t)[K], uint64_t x) {
-#pragma unroll
-  for (int i = 0; i < K; ++i) {
-    const uint64_t a = t[i];
-    const bool gt = x > a;
-    t[i] = gt ? x : a;
-    x = gt ? a : x;
-  }
-}
-
-// K warp-wide pops of the per-lane descending lists: lane r < K receives the r-th largest key
-// (u64 max; equal keys of a repeated edge are popped one at a time).
-template <int K>
-__device__ __forceinline__ uint64_t warp_topk_pop(uint64_t (&t)[K]) {
-  const int lane = threadIdx.x & 31;
-  uint64_t mine = 0ull;
-#pragma unroll
-  for (int r = 0; r < K; ++r) {
-    const uint64_t mx = group_max_key(t[0], 0xffffffffu);
-    if (lane == r) mine = mx;
-    const unsigned own = __ballot_sync(0xffffffffu, mx != 0ull && t[0] == mx);
-    if (own && lane == __ffs(own) - 1) {
-#pragma unroll
-      for (int i = 0; i < K - 1; ++i) t[i] = t[i + 1];
-      t[K - 1] = 0ull;
-    }
-  }
-  return mine;
-}
-
 // Fill / merge the cache of rows [*plo, *phi] from entries [w0, w1) held at base[j - ebase].
 // A row starting inside the window overwrites its slots; a row that started before it (spans a
 // chunk boundary or the resident/streamed split) merges with the slots written earlier on the
@@ -2425,7 +2615,7 @@ __global__ void k_cache_redirect(Bins F, const unsigned long long* __restrict__ 
   const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   unsigned long long served = 0, left = 0;
-  for (int bb = 0; bb < kBins; ++bb) {
+  for (int bb = 0; bb < kDegBins; ++bb) {
     const int64_t c = (int64_t)cntF[bb];
     for (int64_t i = tid; i < c; i += stride) {
       ulonglong2 e = F.list[bb][i];

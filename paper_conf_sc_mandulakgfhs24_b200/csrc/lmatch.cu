@@ -21,6 +21,12 @@
 #include <new>
 #include <vector>
 
+#include <fcntl.h>
+#include <sys/mman.h>
+#include <sys/stat.h>
+#include <time.h>
+#include <unistd.h>
+
 #include "../../include/lmatch.h"
 #include "kernels.cuh"
 
@@ -49,9 +55,14 @@ void set_err(const char* fmt, ...) {
 // every kernel launch of the library is followed by CKL(): it also counts the launch (process-wide,
 // lmatch_kernel_launch_count)
 static std::atomic<long long> g_launch_count{0};
+static thread_local long long t_launch_count = 0;  // this thread's launches (lmatch_run_dist stats)
+static inline void count_launches(long long k) {
+  g_launch_count.fetch_add(k, std::memory_order_relaxed);
+  t_launch_count += k;
+}
 #define CKL()                                            \
   do {                                                   \
-    g_launch_count.fetch_add(1, std::memory_order_relaxed); \
+    count_launches(1);                                   \
     CK(cudaGetLastError());                              \
   } while (0)
 #define TRY(x)                 \
@@ -87,6 +98,8 @@ using Sweep = lm::Sweep2DCfg<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap>;
 using Sweep = lm::SweepCfg<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap>;
 #define SWEEP_KERNEL lm::k_sweep<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap>
 #endif
+// the round-1 sweep that also fills the resident key cache (opts.key_cache)
+#define SWEEP_KERNEL_KC lm::k_sweep<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap, false, true>
 constexpr int kSweepThreads = Sweep::kThreads;
 constexpr int64_t kTile = Sweep::kTile;
 constexpr int kCompactK = 8;  // items per lane per compaction chunk
@@ -193,7 +206,8 @@ struct lmatch_graph {
   int part_round = 0, part_cur = 0;
   std::vector<int64_t> hbounds;      // host copy of the part bounds [P+1]
   // peer-memory exchange (lmatch_p2p_*): window = inbox [P][win_cap] u64 | inbox counts [P] |
-  // frontier-size slots [P]; peers store into it (and into `bits`) over NVLink / peer memory
+  // frontier-size slots [P] | barrier flags [P] | w(M) shares [P] | matched counts [P]; peers
+  // store into it (and into `bits`) over NVLink / peer memory
   int p2p = 0, me = 0;
   int64_t win_cap = 0;
   uint64_t* win = nullptr;
@@ -202,8 +216,16 @@ struct lmatch_graph {
   unsigned long long** d_dcnt = nullptr;  // device [P]: its count
   uint32_t** d_dbits = nullptr;      // device [P]: each peer's bitmap replica
   unsigned long long** d_dnf = nullptr;   // device [P]: my frontier-size slot in each peer
+  unsigned long long** d_dflag = nullptr;  // device [P]: my barrier flag in each peer (lmatch_run_dist)
+  unsigned long long** d_dresw = nullptr;  // device [P]: my w(M) share slot in each peer
+  unsigned long long** d_dresc = nullptr;  // device [P]: my matched-count slot in each peer
   std::vector<uint64_t*> h_dseg;
-  std::vector<unsigned long long*> h_dcnt, h_dnf;
+  std::vector<unsigned long long*> h_dcnt, h_dnf, h_dflag, h_dresw, h_dresc;
+  // library-owned multi-GPU driver (lmatch_create_dist): device barrier epoch and error flag
+  int dist = 0;
+  unsigned long long epoch = 0;
+  unsigned* d_berr = nullptr;
+  unsigned long long* h_res6 = nullptr;  // pinned [3P]: frontier sizes, w shares, counts
   std::vector<uint32_t*> h_dbits;
   std::vector<void*> ipc_opened;     // peer allocations opened with cudaIpcOpenMemHandle
   unsigned long long* h_nf = nullptr;  // pinned [P]
@@ -219,6 +241,15 @@ struct lmatch_graph {
   int batches = 0;                   // paper-style batch count (> 1: all streamed)
   int algorithm = 0;                 // 0 = LD pointer iteration, 1 = Suitor (NEXT-4), 3 = sorted+cursor
   int64_t sort_chunk = 1ll << 30;    // algorithm 3: entries per segmented-sort chunk
+  // resident key cache (opts.key_cache): the 4 largest keys of every row, filled by the sweep
+  int key_cache = 1;
+  int kc_attr = 0;
+  uint64_t* kcache = nullptr;        // the active cache: kc_buf, or nullptr = off for this graph
+  uint64_t* kc_buf = nullptr;        // [n + 1][kKC]
+  uint64_t* xpart = nullptr;         // [ntiles][2][kKC] partial lists of tile-crossing rows
+  int32_t* xrows = nullptr;          // nz index of every tile-crossing row
+  unsigned long long* nx = nullptr;  // |xrows|
+  int64_t cap_kc_buf = -1, cap_xpart = -1, cap_xrows = -1;
   bool sorted = false;               // algorithm 3: rows sorted by key, descending (NEXT-3)
   float ms_sort = 0.f;               // algorithm 3: device time of the last row sort
   uint32_t* sc_cur = nullptr;        // algorithm 3: per-vertex cursor (row-relative entry index)
@@ -264,7 +295,7 @@ struct lmatch_graph {
   // capacities of the buffers sized by the graph's shape (non-empty rows, bins); a reload with a
   // different degree mix grows them and drops the captured CUDA graph
   int64_t cap_noffs = -1, cap_nzr = -1, cap_nlo = -1, cap_S[2] = {-1, -1};
-  int64_t cap_bin[2][lm::kBins] = {{-1, -1, -1, -1}, {-1, -1, -1, -1}};
+  int64_t cap_bin[2][lm::kBins] = {{-1, -1, -1, -1, -1}, {-1, -1, -1, -1, -1}};
   // state
   uint64_t* best = nullptr;
   uint32_t* bits = nullptr;
@@ -315,6 +346,8 @@ struct lmatch_graph {
     a.st = rstate;
     a.log = rlog;
     a.live = prune ? live : nullptr;
+    a.kc = kcache;
+    a.best = best;
     return a;
   }
 };
@@ -611,7 +644,7 @@ int check_duplicates(lmatch_graph* g, cudaStream_t st) {
     lm::k_sc_seg_offsets<<<grid_for(b - a + 1, 256, 65536), 256, 0, st>>>(g->offs, a, b, seg);
     lm::k_dup_keys<<<grid_for(cnt, 256, 65536), 256, 0, st>>>(g->view(), base, cnt, kin);
     if (cudaGetLastError() != cudaSuccess) { set_err("duplicate check launch failed"); rc = LMATCH_ECUDA; break; }
-    g_launch_count.fetch_add(2, std::memory_order_relaxed);
+    count_launches(2);
     if (cub::DeviceSegmentedSort::SortKeys(nullptr, need, kin, kout, (int)cnt, (int)(b - a), seg, seg + 1,
                                            st) != cudaSuccess) {
       set_err("duplicate check: sort sizing failed"); rc = LMATCH_ECUDA; break;
@@ -629,7 +662,7 @@ int check_duplicates(lmatch_graph* g, cudaStream_t st) {
     }
     lm::k_dup_check<<<grid_for((b - a) * 8, 256, 16384), 256, 0, st>>>(kout, seg, b - a, a, bad);
     if (cudaGetLastError() != cudaSuccess) { set_err("duplicate check launch failed"); rc = LMATCH_ECUDA; break; }
-    g_launch_count.fetch_add(1, std::memory_order_relaxed);
+    count_launches(1);
   }
   unsigned long long hbad = ULLONG_MAX;
   if (rc == LMATCH_OK && cudaMemcpyAsync(&hbad, bad, 8, cudaMemcpyDeviceToHost, st) != cudaSuccess) rc = LMATCH_ECUDA;
@@ -784,8 +817,11 @@ int alloc_bins(lmatch_graph* g, cudaStream_t st) {
   g->device_bytes -= 16;
   // A7 pruning moves rows to LOWER bins (live degrees only shrink): bin b must then hold every
   // row whose full degree is in bin b or above
+  // the decided list (key cache) can hold any non-empty row
+  h[lm::kDecided] = 0;
+  for (int b = 0; b < lm::kDegBins; ++b) h[lm::kDecided] += h[b];
   if (g->prune)
-    for (int b = lm::kBins - 2; b >= 0; --b) h[b] += h[b + 1];
+    for (int b = lm::kDegBins - 2; b >= 0; --b) h[b] += h[b + 1];
   for (int i = 0; i < 2; ++i)
     for (int b = 0; b < lm::kBins; ++b)
       TRY(ensure(g, &g->F[i].list[b], &g->cap_bin[i][b], (int64_t)h[b] + 1));
@@ -838,6 +874,38 @@ static int prefer_l1() {
   return LMATCH_OK;
 }
 
+// Resident key cache (opts.key_cache): allocated for resident handles running the LD iteration
+// when it fits in free device memory (with 1 GiB to spare); the list of tile-crossing rows it
+// merges after the sweep is built here.  Off otherwise (kcache = nullptr).
+int setup_key_cache(lmatch_graph* g, cudaStream_t st) {
+  const bool want = g->key_cache && !g->streaming && (g->algorithm == 0 || g->algorithm == 2) &&
+                    g->n > 0 && g->ntiles > 0 && LM_SWEEP_IMPL == 1;
+  g->kcache = nullptr;  // buffers of an earlier graph stay allocated for a later reload
+  if (!want) return LMATCH_OK;
+  const int64_t need_kc = (g->n + 1) * lm::kKC, need_xp = g->ntiles * 2 * lm::kKC + 8;
+  int64_t extra = 0;
+  if (!(g->kc_buf && g->cap_kc_buf >= need_kc)) extra += need_kc * 8;
+  if (!(g->xpart && g->cap_xpart >= need_xp)) extra += need_xp * 8;
+  if (!(g->xrows && g->cap_xrows >= g->ntiles + 1)) extra += (g->ntiles + 1) * 4;
+  size_t fr = 0, tot = 0;
+  CK(cudaMemGetInfo(&fr, &tot));
+  if ((size_t)extra + (1ull << 30) > fr) return LMATCH_OK;
+  TRY(ensure(g, &g->kc_buf, &g->cap_kc_buf, need_kc));
+  g->kcache = g->kc_buf;
+  TRY(ensure(g, &g->xpart, &g->cap_xpart, need_xp));
+  TRY(ensure(g, &g->xrows, &g->cap_xrows, g->ntiles + 1));
+  if (!g->nx) TRY(dmalloc(g, &g->nx, 1));
+  CK(cudaMemsetAsync(g->nx, 0, 8, st));
+  lm::k_kc_xrows<<<grid_for((g->n_nz + 31) & ~31ll, 256, 8192), 256, 0, st>>>(g->noffs, g->n_nz, kTile,
+                                                                              g->xrows, g->nx);
+  CKL();
+  if (!g->kc_attr) {
+    CK(cudaFuncSetAttribute(SWEEP_KERNEL_KC, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Sweep::kSmem));
+    g->kc_attr = 1;
+  }
+  return LMATCH_OK;
+}
+
 int finish_create(lmatch_graph* g, cudaStream_t st) {
   TRY(prefer_l1());
 #if LM_L2_WINDOW
@@ -871,6 +939,7 @@ int finish_create(lmatch_graph* g, cudaStream_t st) {
   // partitioned claims read best[] of every vertex)
   CK(cudaMemsetAsync(g->best, 0, ((size_t)g->n + 1) * 8, st));
   TRY(build_index(g, st));
+  TRY(setup_key_cache(g, st));
   TRY(alloc_bins(g, st));
   TRY(build_cache_index(g, st));
   if (g->m > 0) {
@@ -946,6 +1015,7 @@ int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** 
     g->host_cache = opts->host_cache >= 0;
     g->batches = opts->batches;
     g->algorithm = opts->algorithm;
+    g->key_cache = opts->key_cache >= 0;
     if (opts->sort_chunk_log2 != 0) {
       if (opts->sort_chunk_log2 < 4 || opts->sort_chunk_log2 > 30) {
         set_err("sort_chunk_log2 = %d outside 4..30", opts->sort_chunk_log2);
@@ -1001,13 +1071,26 @@ int round1_sweep(lmatch_graph* g, cudaStream_t st, int64_t* launches_out, int64_
   auto sweep_launch = [&](const uint64_t* base, int64_t t0, int64_t t1) -> int {
     const int64_t grid = std::min<int64_t>((t1 - t0 + kSweepWarps - 1) / kSweepWarps, g->sweep_grid);
     lm::SweepArgs A{base, nullptr, nullptr, 0u, g->noffs_lo, g->nzr, g->tile_nz, g->best, g->m, t0, t1};
-    SWEEP_KERNEL<<<(unsigned)std::max<int64_t>(grid, 1), kSweepThreads, Sweep::kSmem, st>>>(A);
+    if (g->kcache) {
+      A.kc = g->kcache;
+      A.xpart = g->xpart;
+      SWEEP_KERNEL_KC<<<(unsigned)std::max<int64_t>(grid, 1), kSweepThreads, Sweep::kSmem, st>>>(A);
+    } else {
+      SWEEP_KERNEL<<<(unsigned)std::max<int64_t>(grid, 1), kSweepThreads, Sweep::kSmem, st>>>(A);
+    }
     CKL();
     ++launches;
     ++sweep_launches;
     return LMATCH_OK;
   };
   if (rt > 0) TRY(sweep_launch(g->adj, 0, std::min(rt, g->ntiles)));
+  if (g->kcache && rt > 0) {
+    // the rows crossing a tile boundary: merge their per-tile top-4 lists (also their pointer)
+    lm::k_kc_merge<<<(unsigned)(8 * g->num_sms), 256, 0, st>>>(g->xrows, g->nx, g->noffs, g->nzr, g->xpart,
+                                                               kTile, g->kcache, g->best);
+    CKL();
+    ++launches;
+  }
   // host-row cache fill over entries [w0, w1) held at base[j - ebase], rows [*plo, *phi]
   auto cache_fill = [&](const uint64_t* base, int64_t ebase, int64_t w0, int64_t w1,
                         const int64_t* plo, const int64_t* phi) -> int {
@@ -1098,10 +1181,12 @@ void lmatch_destroy(lmatch_graph* g) {
   if (g->h_rstate) cudaFreeHost(g->h_rstate);
   for (void* p : g->ipc_opened) cudaIpcCloseMemHandle(p);
   if (g->h_nf) cudaFreeHost(g->h_nf);
+  if (g->h_res6) cudaFreeHost(g->h_res6);
   void* pdev[] = {g->bounds, g->ghost, g->claims, g->claim_cnt, g->rstate, g->rlog, g->d_rargs,
                   g->cache, g->chunk_rows, g->cache_big, g->rescan, g->rescan_cnt, g->live, g->win, g->suitor, g->wl[0],
                   g->wl[1], g->wl_big, g->wl_cnt, g->sc_cur, g->sc_ptr, g->sc_L[0], g->sc_L[1], g->shadow, g->d_dseg, g->d_dcnt,
-                  g->d_dbits, g->d_dnf};
+                  g->d_dbits, g->d_dnf, g->d_dflag, g->d_dresw, g->d_dresc, g->d_berr,
+                  g->kc_buf, g->xpart, g->xrows, g->nx};
   for (void* p : pdev) if (p) cudaFree(p);
   if (g->h_claim_cnt) cudaFreeHost(g->h_claim_cnt);
   if (g->h_res) cudaFreeHost(g->h_res);
@@ -1385,7 +1470,7 @@ int launch_persistent_t(lmatch_graph* g, cudaStream_t st, int64_t* launches) {
   cfg.numAttrs = (LM_L2_WINDOW && g->bits_window.num_bytes > 0) ? 2 : 1;
   CK(cudaLaunchKernelEx(&cfg, PERSISTENT_KERNEL(PRUNE), ra, (const int64_t*)g->offs, av, g->bits,
                         g->best, g->n, g->v0));
-  g_launch_count.fetch_add(1, std::memory_order_relaxed);
+  count_launches(1);
   ++*launches;
   return LMATCH_OK;
 }
@@ -1568,7 +1653,7 @@ static int sort_rows(lmatch_graph* g, cudaStream_t st) {
       if (cnt == 0) continue;
       lm::k_sc_seg_offsets<<<grid_for(b - a + 1, 256, 65536), 256, 0, st>>>(g->offs, a, b, seg);
       if (cudaGetLastError() != cudaSuccess) { set_err("segment offsets launch failed"); rc = LMATCH_ECUDA; break; }
-      g_launch_count.fetch_add(1, std::memory_order_relaxed);
+      count_launches(1);
       if (cub::DeviceSegmentedSort::SortKeysDescending(nullptr, need, g->adj + base, alt, (int)cnt,
                                                        (int)(b - a), seg, seg + 1, st) != cudaSuccess) {
         set_err("segmented sort sizing failed"); rc = LMATCH_ECUDA; break;
@@ -1870,6 +1955,7 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
     stats->bytes_streamed = bytes_streamed;
     stats->resident_entries = g->R;
     stats->tail_passes = tail_passes;
+    if (g->kcache) stats->cache_rows = (int64_t)g->h_counters[lm::kCntCache];
     if (g->use_cache()) {
       stats->cache_rows = (int64_t)g->h_counters[lm::kCntCache];
       stats->host_entries_read = (int64_t)g->h_counters[lm::kCntCache + 1];
@@ -2301,17 +2387,23 @@ int lmatch_p2p_enable(lmatch_graph* g, int32_t me) {
   for (int p = 0; p < P; ++p) cap = std::max(cap, g->hbounds[p + 1] - g->hbounds[p]);
   g->me = me;
   g->win_cap = cap;
-  TRY(dmalloc(g, &g->win, (size_t)P * cap + 2 * (size_t)P));
-  CK(cudaMemset(g->win + (size_t)P * cap, 0, 2 * (size_t)P * 8));
+  TRY(dmalloc(g, &g->win, (size_t)P * cap + 6 * (size_t)P));
+  CK(cudaMemset(g->win + (size_t)P * cap, 0, 6 * (size_t)P * 8));
   TRY(dmalloc(g, &g->shadow, (size_t)(g->n + 31) / 32 + 1));
   TRY(dmalloc(g, &g->d_dseg, (size_t)P));
   TRY(dmalloc(g, &g->d_dcnt, (size_t)P));
   TRY(dmalloc(g, &g->d_dbits, (size_t)P));
   TRY(dmalloc(g, &g->d_dnf, (size_t)P));
+  TRY(dmalloc(g, &g->d_dflag, (size_t)P));
+  TRY(dmalloc(g, &g->d_dresw, (size_t)P));
+  TRY(dmalloc(g, &g->d_dresc, (size_t)P));
   CK(cudaHostAlloc(reinterpret_cast<void**>(&g->h_nf), (size_t)P * 8, cudaHostAllocDefault));
   g->h_dseg.assign(P, nullptr);
   g->h_dcnt.assign(P, nullptr);
   g->h_dnf.assign(P, nullptr);
+  g->h_dflag.assign(P, nullptr);
+  g->h_dresw.assign(P, nullptr);
+  g->h_dresc.assign(P, nullptr);
   g->h_dbits.assign(P, nullptr);
   g->p2p = 1;
   // this part's own entries (its frontier-size slot is written like a peer's)
@@ -2324,11 +2416,17 @@ static int p2p_set_peer(lmatch_graph* g, int peer, uint64_t* pwin, uint32_t* pbi
   g->h_dseg[peer] = pwin + (size_t)g->me * g->win_cap;
   g->h_dcnt[peer] = reinterpret_cast<unsigned long long*>(cnt) + g->me;
   g->h_dnf[peer] = reinterpret_cast<unsigned long long*>(cnt + P) + g->me;
+  g->h_dflag[peer] = reinterpret_cast<unsigned long long*>(cnt + 2 * P) + g->me;
+  g->h_dresw[peer] = reinterpret_cast<unsigned long long*>(cnt + 3 * P) + g->me;
+  g->h_dresc[peer] = reinterpret_cast<unsigned long long*>(cnt + 4 * P) + g->me;
   g->h_dbits[peer] = pbits;
   CK(cudaMemcpy(g->d_dseg, g->h_dseg.data(), (size_t)P * 8, cudaMemcpyHostToDevice));
   CK(cudaMemcpy(g->d_dcnt, g->h_dcnt.data(), (size_t)P * 8, cudaMemcpyHostToDevice));
   CK(cudaMemcpy(g->d_dnf, g->h_dnf.data(), (size_t)P * 8, cudaMemcpyHostToDevice));
   CK(cudaMemcpy(g->d_dbits, g->h_dbits.data(), (size_t)P * 8, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(g->d_dflag, g->h_dflag.data(), (size_t)P * 8, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(g->d_dresw, g->h_dresw.data(), (size_t)P * 8, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(g->d_dresc, g->h_dresc.data(), (size_t)P * 8, cudaMemcpyHostToDevice));
   return LMATCH_OK;
 }
 
@@ -2469,6 +2567,371 @@ int lmatch_p2p_sync(lmatch_graph* g, void* stream) {
   CK(cudaSetDevice(g->device));
   CK(cudaStreamSynchronize(stream ? (cudaStream_t)stream : g->stream));
   return LMATCH_OK;
+}
+
+
+// ------------------------------------------------------------- library-owned multi-GPU driver
+// lmatch_partition / lmatch_create_dist / lmatch_run_dist: the 1-D
+// edge-balanced partition (binary search on the CSR prefix sums), the peer-memory
+// exchange set up by the library itself (the ranks find each other through a POSIX shared-memory
+// rendezvous named by an lmatch_dist_id, like an ncclUniqueId), and the whole round loop --
+// Alg. 2's per-device loop with the exchange redesigned -- driven by the library,
+// with device-side barriers between the phases (no host barrier, one host read per round).
+int lmatch_partition(const int64_t* offsets, int64_t n, int32_t nparts, int32_t align,
+                     int64_t* bounds) {
+  g_err[0] = 0;
+  if (!offsets || !bounds) { set_err("NULL offsets or bounds"); return LMATCH_EINVAL; }
+  if (n < 0 || n >= ((int64_t)1 << 31)) { set_err("n = %lld out of range", (long long)n); return LMATCH_ERANGE; }
+  if (nparts < 1) { set_err("nparts = %d < 1", nparts); return LMATCH_EINVAL; }
+  if (align <= 0) align = 32;
+  if (offsets[0] != 0) { set_err("offsets[0] != 0"); return LMATCH_EINVAL; }
+  const int64_t m = offsets[n];
+  if (m < 0) { set_err("offsets[n] < 0"); return LMATCH_EINVAL; }
+  bounds[0] = 0;
+  for (int p = 1; p < nparts; ++p) {
+    // first row whose start reaches p/P of the entries (floor(m p / P) without overflow)
+    const int64_t target = (m / nparts) * p + ((m % nparts) * p) / nparts;
+    const int64_t v = std::lower_bound(offsets, offsets + n + 1, target) - offsets;
+    const int64_t va = std::min<int64_t>(n, (v + align - 1) / align * align);
+    bounds[p] = std::max(bounds[p - 1], va);
+  }
+  bounds[nparts] = n;
+  return LMATCH_OK;
+}
+
+int lmatch_dist_id_new(lmatch_dist_id* id) {
+  if (!id) { set_err("NULL id"); return LMATCH_EINVAL; }
+  unsigned long long r = 0;
+  const int fd = open("/dev/urandom", O_RDONLY);
+  if (fd >= 0) {
+    if (read(fd, &r, sizeof r) != (ssize_t)sizeof r) r = 0;
+    close(fd);
+  }
+  struct timespec ts;
+  clock_gettime(CLOCK_REALTIME, &ts);
+  std::memset(id->bytes, 0, sizeof id->bytes);
+  snprintf(id->bytes, sizeof id->bytes, "lmatch-%x-%llx-%llx", (unsigned)getpid(),
+           (unsigned long long)ts.tv_sec * 1000000000ull + (unsigned long long)ts.tv_nsec, r);
+  return LMATCH_OK;
+}
+
+namespace {
+constexpr uint32_t kShmMagic = 0x4c4d4431u;  // "LMD1"
+constexpr unsigned long long kDistTimeoutNs = 60ull * 1000000000ull;
+struct DistSlot {
+  uint32_t valid;
+  int32_t pid;
+  int32_t device;
+  int32_t nparts;
+  int64_t v0, n, n_global, win_cap;
+  uint64_t raw_win, raw_bits;   // device pointers, meaningful to a peer in the same process
+  unsigned char ipc[128];       // lmatch_p2p_export handles, for peers in other processes
+};
+struct DistShm {
+  uint32_t magic;
+  int32_t world;
+  int32_t attached;
+  int32_t pad;
+  DistSlot slot[1];
+};
+
+int shm_name(const lmatch_dist_id* id, char* out, size_t cap) {
+  size_t k = 0;
+  out[k++] = '/';
+  for (size_t i = 0; i < sizeof id->bytes && id->bytes[i] && k + 1 < cap; ++i) {
+    const char c = id->bytes[i];
+    if ((c >= 'a' && c <= 'z') || (c >= 'A' && c <= 'Z') || (c >= '0' && c <= '9') || c == '-' || c == '_')
+      out[k++] = c;
+  }
+  out[k] = 0;
+  if (k < 8) { set_err("lmatch_dist_id is empty or malformed (use lmatch_dist_id_new)"); return LMATCH_EINVAL; }
+  return LMATCH_OK;
+}
+
+// every rank publishes its window / bitmap (IPC handles and raw pointers) in the rendezvous,
+// waits for all ranks, then attaches each peer: plain pointers within one process (peer access
+// enabled across devices), CUDA IPC across processes.  The last rank to attach unlinks it.
+int dist_bootstrap(lmatch_graph* g, const lmatch_dist_id* id, int rank, int world) {
+  char name[96];
+  TRY(shm_name(id, name, sizeof name));
+  const size_t bytes = sizeof(DistShm) + (size_t)world * sizeof(DistSlot);
+  const int fd = shm_open(name, O_CREAT | O_RDWR, 0600);
+  if (fd < 0) { set_err("shm_open(%s) failed", name); return LMATCH_ENCCL; }
+  struct stat sb;
+  if (fstat(fd, &sb) != 0 || ((size_t)sb.st_size < bytes && ftruncate(fd, (off_t)bytes) != 0)) {
+    close(fd);
+    set_err("rendezvous %s: cannot size it", name);
+    return LMATCH_ENCCL;
+  }
+  void* mp = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+  close(fd);
+  if (mp == MAP_FAILED) { set_err("rendezvous %s: mmap failed", name); return LMATCH_ENCCL; }
+  DistShm* h = static_cast<DistShm*>(mp);
+  int rc = LMATCH_OK;
+  uint32_t zero = 0;
+  __atomic_compare_exchange_n(&h->magic, &zero, kShmMagic, false, __ATOMIC_ACQ_REL, __ATOMIC_ACQUIRE);
+  int32_t w0 = 0;
+  __atomic_compare_exchange_n(&h->world, &w0, world, false, __ATOMIC_ACQ_REL, __ATOMIC_ACQUIRE);
+  if (__atomic_load_n(&h->magic, __ATOMIC_ACQUIRE) != kShmMagic || __atomic_load_n(&h->world, __ATOMIC_ACQUIRE) != world) {
+    set_err("rendezvous %s: world size mismatch (%d here)", name, world);
+    rc = LMATCH_EINVAL;
+  }
+  DistSlot* me = &h->slot[rank];
+  if (!rc) {
+    if (__atomic_load_n(&me->valid, __ATOMIC_ACQUIRE)) {
+      set_err("rendezvous %s: rank %d joined twice", name, rank);
+      rc = LMATCH_EINVAL;
+    }
+  }
+  if (!rc) {
+    me->pid = (int32_t)getpid();
+    me->device = g->device;
+    me->nparts = g->P;
+    me->v0 = g->v0;
+    me->n = g->n;
+    me->n_global = g->n_global;
+    me->win_cap = g->win_cap;
+    me->raw_win = (uint64_t)(uintptr_t)g->win;
+    me->raw_bits = (uint64_t)(uintptr_t)g->bits;
+    rc = lmatch_p2p_export(g, me->ipc);
+    if (!rc) __atomic_store_n(&me->valid, 1u, __ATOMIC_RELEASE);
+  }
+  // wait for every rank
+  struct timespec t0, t1;
+  clock_gettime(CLOCK_MONOTONIC, &t0);
+  for (int q = 0; !rc && q < world; ++q) {
+    while (!__atomic_load_n(&h->slot[q].valid, __ATOMIC_ACQUIRE)) {
+      clock_gettime(CLOCK_MONOTONIC, &t1);
+      if ((t1.tv_sec - t0.tv_sec) * 1000000000ll + (t1.tv_nsec - t0.tv_nsec) > (long long)kDistTimeoutNs) {
+        set_err("rendezvous %s: rank %d did not join within %llu s", name, q, kDistTimeoutNs / 1000000000ull);
+        rc = LMATCH_ENCCL;
+        break;
+      }
+      usleep(200);
+    }
+  }
+  for (int q = 0; !rc && q < world; ++q) {
+    if (q == rank) continue;
+    const DistSlot& s = h->slot[q];
+    if (s.nparts != g->P || s.n_global != g->n_global || s.win_cap != g->win_cap ||
+        s.v0 != g->hbounds[q] || s.v0 + s.n != g->hbounds[q + 1]) {
+      set_err("rank %d: partition does not match rank %d's part_bounds / n_global", q, rank);
+      rc = LMATCH_EINVAL;
+      break;
+    }
+    if (s.pid == (int32_t)getpid()) {
+      if (s.device != g->device) {
+        const cudaError_t e = cudaDeviceEnablePeerAccess(s.device, 0);
+        if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) {
+          set_err("cudaDeviceEnablePeerAccess(%d): %s", s.device, cudaGetErrorString(e));
+          rc = LMATCH_ECUDA;
+          break;
+        }
+        cudaGetLastError();
+      }
+      rc = p2p_set_peer(g, q, reinterpret_cast<uint64_t*>((uintptr_t)s.raw_win),
+                        reinterpret_cast<uint32_t*>((uintptr_t)s.raw_bits));
+    } else {
+      rc = lmatch_p2p_attach(g, q, s.ipc);
+    }
+  }
+  if (__atomic_add_fetch(&h->attached, 1, __ATOMIC_ACQ_REL) == world) shm_unlink(name);
+  munmap(mp, bytes);
+  return rc;
+}
+
+int dist_check(int64_t n_local, int64_t v_begin, int64_t n_global, int32_t rank, int32_t world,
+               const int64_t* bounds, const lmatch_dist_id* id, const lmatch_opts* opts) {
+  if (world < 1 || rank < 0 || rank >= world) { set_err("rank %d / world %d out of range", rank, world); return LMATCH_EINVAL; }
+  if (!id) { set_err("NULL lmatch_dist_id"); return LMATCH_EINVAL; }
+  TRY(check_part(n_local, v_begin, n_global, world, bounds));
+  if (bounds[rank] != v_begin) { set_err("v_begin is not part_bounds[rank]"); return LMATCH_EINVAL; }
+  if (opts && opts->validate_level >= 2) { set_err("validate_level 2 is not available per partition"); return LMATCH_EINVAL; }
+  if (opts && opts->hbm_budget_bytes > 0) { set_err("out-of-core is not available per partition"); return LMATCH_EINVAL; }
+  if (opts && opts->algorithm != 0) { set_err("lmatch_run_dist runs the LD iteration (algorithm 0) only"); return LMATCH_EINVAL; }
+  return LMATCH_OK;
+}
+
+int dist_finish_create(lmatch_graph* g, int rank, int world, const lmatch_dist_id* id) {
+  TRY(lmatch_p2p_enable(g, rank));
+  TRY(dmalloc(g, &g->d_berr, 1));
+  CK(cudaMemset(g->d_berr, 0, 4));
+  CK(cudaHostAlloc(reinterpret_cast<void**>(&g->h_res6), (size_t)6 * g->P * 8 + 8, cudaHostAllocDefault));
+  if (world > 1) TRY(dist_bootstrap(g, id, rank, world));
+  g->dist = 1;
+  return LMATCH_OK;
+}
+}  // namespace
+
+int lmatch_create_dist(const int64_t* csr_offsets, const int32_t* col_idx, const float* weights,
+                       int64_t n_local, int64_t m_local, int64_t v_begin, int64_t n_global,
+                       int32_t rank, int32_t world, const int64_t* part_bounds,
+                       const lmatch_dist_id* id, const lmatch_opts* opts, lmatch_graph** out) {
+  if (!out) { set_err("out == NULL"); return LMATCH_EINVAL; }
+  *out = nullptr;
+  g_err[0] = 0;
+  int s = check_args(csr_offsets, col_idx, weights, n_local, m_local);
+  if (!s) s = dist_check(n_local, v_begin, n_global, rank, world, part_bounds, id, opts);
+  if (s) return s;
+  PartSpec ps;
+  ps.v0 = v_begin; ps.n_global = n_global; ps.P = world; ps.bounds = part_bounds;
+  lmatch_graph* g = nullptr;
+  s = create_common(n_local, m_local, opts, out, &g, &ps);
+  if (!s) s = upload_host(g, csr_offsets, col_idx, weights);
+  if (!s) s = finish_create(g, g->stream);
+  if (!s) s = dist_finish_create(g, rank, world, id);
+  if (s) { lmatch_destroy(g); return s; }
+  *out = g;
+  return LMATCH_OK;
+}
+
+int lmatch_create_dist_device(const int64_t* d_offsets, const int32_t* d_col, const float* d_weights,
+                              int64_t n_local, int64_t m_local, int64_t v_begin, int64_t n_global,
+                              int32_t rank, int32_t world, const int64_t* part_bounds,
+                              const lmatch_dist_id* id, const lmatch_opts* opts, void* stream,
+                              lmatch_graph** out) {
+  if (!out) { set_err("out == NULL"); return LMATCH_EINVAL; }
+  *out = nullptr;
+  g_err[0] = 0;
+  int s = check_args(d_offsets, d_col, d_weights, n_local, m_local);
+  if (!s) s = dist_check(n_local, v_begin, n_global, rank, world, part_bounds, id, opts);
+  if (s) return s;
+  PartSpec ps;
+  ps.v0 = v_begin; ps.n_global = n_global; ps.P = world; ps.bounds = part_bounds;
+  lmatch_graph* g = nullptr;
+  s = create_common(n_local, m_local, opts, out, &g, &ps);
+  cudaStream_t st = stream ? (cudaStream_t)stream : (g ? g->stream : nullptr);
+  if (!s) {
+    cudaError_t e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) { set_err("stream sync: %s", cudaGetErrorString(e)); s = LMATCH_ECUDA; }
+  }
+  if (!s) s = upload_device(g, d_offsets, d_col, d_weights, st);
+  if (!s) s = finish_create(g, st);
+  if (!s) s = dist_finish_create(g, rank, world, id);
+  if (s) { lmatch_destroy(g); return s; }
+  *out = g;
+  return LMATCH_OK;
+}
+
+int lmatch_run_dist_device(lmatch_graph* g, int32_t* d_mate_local, void* stream, lmatch_stats* stats) {
+  if (!g || !g->dist) { set_err("not a lmatch_create_dist handle"); return LMATCH_ESTATE; }
+  if (!d_mate_local && g->n > 0) { set_err("d_mate_local == NULL"); return LMATCH_EINVAL; }
+  g_err[0] = 0;
+  CK(cudaSetDevice(g->device));
+  cudaStream_t st = stream ? (cudaStream_t)stream : g->stream;
+  const int P = g->P;
+  const long long l0 = t_launch_count;
+  unsigned long long* wslots = reinterpret_cast<unsigned long long*>(g->win + (size_t)P * g->win_cap);
+  // wslots: [0,P) inbox counts, [P,2P) frontier sizes, [2P,3P) barrier flags, [3P,4P) w shares,
+  // [4P,5P) matched counts
+  auto barrier = [&]() -> int {
+    if (P == 1) return LMATCH_OK;
+    ++g->epoch;
+    lm::k_dist_barrier<<<1, 32, 0, st>>>(wslots + 2 * P, g->d_dflag, P, g->me, g->epoch,
+                                         kDistTimeoutNs, g->d_berr);
+    CKL();
+    return LMATCH_OK;
+  };
+  // one host read: the P frontier sizes (and the barrier error flag)
+  auto read_slots = [&](int64_t* total) -> int {
+    CK(cudaMemcpyAsync(g->h_res6, wslots + P, (size_t)P * 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(g->h_res6 + 5 * P, g->d_berr, 4, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (*reinterpret_cast<unsigned*>(g->h_res6 + 5 * P)) {
+      set_err("a peer did not reach a device barrier within %llu s", kDistTimeoutNs / 1000000000ull);
+      return LMATCH_ENCCL;
+    }
+    int64_t t = 0;
+    for (int p = 0; p < P; ++p) t += (int64_t)g->h_res6[p];
+    *total = t;
+    return LMATCH_OK;
+  };
+  if (g->timing && stats) CK(cudaEventRecord(g->ev[0], st));
+  CK(cudaMemsetAsync(g->d_berr, 0, 4, st));
+  TRY(barrier());  // every part is done with its previous run (inboxes, replicas, slots)
+  TRY(part_begin_impl(g, st, nullptr));
+  int64_t rounds = 1;
+  bool compacted = false, capped = false;
+  for (;;) {
+    TRY(barrier());  // claims are in the owners' inboxes; frontier sizes in every slot
+    if (compacted) {
+      int64_t total = 0;
+      TRY(read_slots(&total));
+      if (total == 0) break;
+      if (rounds >= g->max_rounds) { capped = true; break; }  // same decision on every part
+      ++rounds;
+    }
+    TRY(lmatch_p2p_match(g, st));
+    TRY(barrier());  // bitmap replicas complete
+    TRY(lmatch_p2p_compact(g, st, nullptr));
+    compacted = true;
+    TRY(part_point_impl(g, st, nullptr));  // an empty global frontier launches only empty work
+  }
+  // A10 owned mate[] slice + A9: this part's w(M) share, then every part's shares summed in part
+  // order (the same fp64 total on every part)
+  if (g->n > 0) {
+    lm::k_materialize<kFinThreads><<<kFinBlocks, kFinThreads, 0, st>>>(g->best, g->bits, g->n, g->v0,
+                                                                       d_mate_local, g->pw, g->pc);
+    CKL();
+    lm::k_final_sum<<<1, 32, 0, st>>>(g->pw, g->pc, kFinBlocks, g->res_w, g->res_c);
+    CKL();
+  } else {
+    CK(cudaMemsetAsync(g->res_w, 0, 8, st));
+    CK(cudaMemsetAsync(g->res_c, 0, 8, st));
+  }
+  lm::k_push_result<<<1, 32, 0, st>>>(g->res_w, g->res_c, g->d_dresw, g->d_dresc, P);
+  CKL();
+  TRY(barrier());
+  CK(cudaMemcpyAsync(g->h_res6 + P, wslots + 3 * P, (size_t)2 * P * 8, cudaMemcpyDeviceToHost, st));
+  CK(cudaMemcpyAsync(g->h_counters, g->counters, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
+  int64_t dummy = 0;
+  TRY(read_slots(&dummy));  // also synchronises and checks the barrier flag
+  if (g->timing && stats) CK(cudaEventRecord(g->ev[5], st));
+  double wsum = 0.0;
+  int64_t csum = 0;
+  for (int p = 0; p < P; ++p) {
+    double w;
+    std::memcpy(&w, &g->h_res6[P + p], 8);
+    wsum += w;
+    csum += (int64_t)g->h_res6[2 * P + p];
+  }
+  if (stats) {
+    std::memset(stats, 0, sizeof *stats);
+    stats->rounds = rounds;
+    stats->matched_vertices = csum;
+    stats->cardinality = csum / 2;
+    stats->weight = wsum;
+    stats->entries_swept = g->m + (int64_t)g->h_counters[lm::kCntSwept];
+    stats->kernel_launches = t_launch_count - l0;
+    stats->sweep_launches = 1;
+    stats->resident_entries = g->R;
+    if (g->timing) {
+      float a = 0;
+      CK(cudaEventSynchronize(g->ev[5]));
+      CK(cudaEventElapsedTime(&a, g->ev[0], g->ev[5]));
+      stats->ms_total = a;
+      stats->ms_sweep = g->part_sweep_ms;
+    }
+  }
+  if (capped) {
+    set_err("frontier left after the round cap (%lld pointing phases)", (long long)rounds);
+    return LMATCH_EROUNDS;
+  }
+  return LMATCH_OK;
+}
+
+int lmatch_run_dist(lmatch_graph* g, int32_t* mate_local, lmatch_stats* stats) {
+  if (!g || !g->dist) { set_err("not a lmatch_create_dist handle"); return LMATCH_ESTATE; }
+  if (!mate_local && g->n > 0) { set_err("mate_local == NULL"); return LMATCH_EINVAL; }
+  CK(cudaSetDevice(g->device));
+  if (!g->mate_tmp) TRY(dmalloc(g, &g->mate_tmp, (size_t)g->n + 1));
+  const int rc = lmatch_run_dist_device(g, g->mate_tmp, g->stream, stats);
+  if (rc != LMATCH_OK && rc != LMATCH_EROUNDS) return rc;
+  if (g->n > 0) {
+    CK(cudaMemcpyAsync(mate_local, g->mate_tmp, (size_t)g->n * 4, cudaMemcpyDeviceToHost, g->stream));
+    CK(cudaStreamSynchronize(g->stream));
+  }
+  return rc;
 }
 
 }  // extern "C"

@@ -58,6 +58,14 @@ _sig = {
     "lmatch_p2p_frontier_total": ([_P, _P, ctypes.POINTER(_I64)], ctypes.c_int),
     "lmatch_p2p_sync": ([_P, _P], ctypes.c_int),
     "lmatch_kernel_launch_count": ([], _I64),
+    "lmatch_partition": ([_P, _I64, ctypes.c_int32, ctypes.c_int32, _P], ctypes.c_int),
+    "lmatch_dist_id_new": ([_P], ctypes.c_int),
+    "lmatch_create_dist": ([_P, _P, _P, _I64, _I64, _I64, _I64, ctypes.c_int32, ctypes.c_int32, _P, _P,
+                            _P, ctypes.POINTER(_P)], ctypes.c_int),
+    "lmatch_create_dist_device": ([_P, _P, _P, _I64, _I64, _I64, _I64, ctypes.c_int32, ctypes.c_int32,
+                                   _P, _P, _P, _P, ctypes.POINTER(_P)], ctypes.c_int),
+    "lmatch_run_dist": ([_P, _P, _P], ctypes.c_int),
+    "lmatch_run_dist_device": ([_P, _P, _P, _P], ctypes.c_int),
 }
 for _name, (_args, _res) in _sig.items():
     _f = getattr(_lib, _name)
@@ -68,17 +76,21 @@ for _name, (_args, _res) in _sig.items():
 # ------------------------------------------------------------------------------- partitioning
 def edge_balanced_bounds(offsets: np.ndarray, nparts: int, align: int = 32) -> np.ndarray:
     """Contiguous vertex ranges with ~m/P directed entries each (binary search on the CSR prefix
-    sums); every bound is a multiple of `align` (bitmap words are owned by one part)."""
-    offsets = np.asarray(offsets, dtype=np.int64)
+    sums); every bound is a multiple of `align` (bitmap words are owned by one part).
+    Computed by the library (lmatch_partition, host-only)."""
+    offsets = np.ascontiguousarray(offsets, dtype=np.int64)
     n = offsets.shape[0] - 1
-    m = int(offsets[-1])
     b = np.zeros(nparts + 1, dtype=np.int64)
-    for p in range(1, nparts):
-        v = int(np.searchsorted(offsets, (m * p) // nparts, side="left"))
-        v = min(n, (v + align - 1) // align * align)
-        b[p] = max(b[p - 1], v)
-    b[nparts] = n
+    _check(_lib.lmatch_partition(offsets.ctypes.data, n, int(nparts), int(align), b.ctypes.data),
+           "lmatch_partition")
     return b
+
+
+def dist_id_new() -> bytes:
+    """64-byte rendezvous id for one lmatch_create_dist group (lmatch_dist_id_new)."""
+    buf = ctypes.create_string_buffer(64)
+    _check(_lib.lmatch_dist_id_new(buf), "lmatch_dist_id_new")
+    return buf.raw
 
 
 def part_words(bounds):
@@ -348,6 +360,122 @@ class LibPart:
             self.close()
         except Exception:
             pass
+
+
+# ------------------------------------------------------------- the library-owned driver (C ABI)
+class DistMatcher:
+    """One rank of a lmatch_create_dist group: the library partitions nothing itself here (the
+    caller passes the rank's rows and the common bounds, e.g. from edge_balanced_bounds), opens
+    the peers' exchange windows through the rendezvous `dist_id`, and runs the whole round loop
+    with device-side barriers (include/lmatch.h "Library-owned multi-GPU driver")."""
+
+    def __init__(self, offsets_local, col_local, w_local, v0: int, n_global: int, rank: int,
+                 world: int, bounds, dist_id: bytes, device=None, stream=None, timing: bool = False,
+                 max_rounds: int = 0, validate_level: int = 1):
+        import torch
+        self.torch = torch
+        self.dev = torch.device("cuda") if device is None else torch.device(device)
+        self.bounds = np.ascontiguousarray(bounds, dtype=np.int64)
+        self.rank, self.world = int(rank), int(world)
+        self.v0, self.n_global = int(v0), int(n_global)
+        self.n_local = int(len(offsets_local) - 1)
+        if stream is None or stream.cuda_stream == 0:
+            stream = torch.cuda.Stream(self.dev)
+        self.stream = stream
+        self._id = ctypes.create_string_buffer(bytes(dist_id)[:64], 64)
+        opts = make_opts(validate_level=validate_level, timing=timing, max_rounds=max_rounds)
+        h = _P()
+        with torch.cuda.device(self.dev):
+            if hasattr(offsets_local, "is_cuda") and offsets_local.is_cuda:
+                torch.cuda.current_stream(self.dev).synchronize()
+                self.m_local = int(col_local.numel())
+                _check(_lib.lmatch_create_dist_device(
+                    offsets_local.data_ptr(), col_local.data_ptr(), w_local.data_ptr(), self.n_local,
+                    self.m_local, self.v0, self.n_global, self.rank, self.world, self.bounds.ctypes.data,
+                    self._id, ctypes.byref(opts), self.stream.cuda_stream, ctypes.byref(h)),
+                    "lmatch_create_dist_device")
+            else:
+                off = np.ascontiguousarray(offsets_local, dtype=np.int64)
+                col = np.ascontiguousarray(col_local, dtype=np.int32)
+                w = np.ascontiguousarray(w_local, dtype=np.float32)
+                self.m_local = int(col.shape[0])
+                _check(_lib.lmatch_create_dist(
+                    off.ctypes.data, col.ctypes.data, w.ctypes.data, self.n_local, self.m_local,
+                    self.v0, self.n_global, self.rank, self.world, self.bounds.ctypes.data, self._id,
+                    ctypes.byref(opts), ctypes.byref(h)), "lmatch_create_dist")
+        self.h = h.value
+
+    def run_device(self, d_mate=None):
+        """Collective: every rank calls it.  Returns (owned mate slice as a CUDA tensor, Stats)."""
+        from . import Stats
+        torch = self.torch
+        if d_mate is None:
+            with torch.cuda.stream(self.stream):
+                d_mate = torch.empty(max(self.n_local, 1), dtype=torch.int32, device=self.dev)
+        st = Stats()
+        _check(_lib.lmatch_run_dist_device(self.h, d_mate.data_ptr(), self.stream.cuda_stream,
+                                           ctypes.byref(st)), "lmatch_run_dist_device")
+        return d_mate[: self.n_local], st
+
+    def run(self):
+        """Collective; host output.  Returns (owned mate slice as numpy int32, Stats)."""
+        from . import Stats
+        mate = np.empty(max(self.n_local, 1), dtype=np.int32)
+        st = Stats()
+        _check(_lib.lmatch_run_dist(self.h, mate.ctypes.data, ctypes.byref(st)), "lmatch_run_dist")
+        return mate[: self.n_local], st
+
+    def reload(self, offsets_local, col_local, w_local):
+        ptrs = [a.ctypes.data if isinstance(a, np.ndarray) else int(a)
+                for a in (offsets_local, col_local, w_local)]
+        _check(_lib.lmatch_reload(self.h, *ptrs), "lmatch_reload")
+
+    def close(self):
+        if self.h is not None:
+            _lib.lmatch_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def match_dist_threads(offsets, col, w, nparts: int, devices=None, max_rounds: int = 0):
+    """P ranks of one lmatch_create_dist group as P threads of this process (one GPU each, or all
+    on the current GPU): the rendezvous gives them plain device pointers.  Returns (mate, stats
+    of rank 0, [stats of every rank])."""
+    import threading
+    offsets = np.asarray(offsets, dtype=np.int64)
+    n = offsets.shape[0] - 1
+    bounds = edge_balanced_bounds(offsets, nparts)
+    did = dist_id_new()
+    out, errs = [None] * nparts, [None] * nparts
+
+    def rank_main(r):
+        try:
+            dev = None if devices is None else devices[r % len(devices)]
+            v0, v1 = int(bounds[r]), int(bounds[r + 1])
+            lo, lc, lw = local_csr(offsets, col, w, v0, v1)
+            M = DistMatcher(lo, lc, lw, v0, n, r, nparts, bounds, did, device=dev, max_rounds=max_rounds)
+            try:
+                out[r] = M.run()
+            finally:
+                M.close()
+        except Exception as e:  # reported by the caller
+            errs[r] = e
+
+    ts = [threading.Thread(target=rank_main, args=(r,)) for r in range(nparts)]
+    for t in ts:
+        t.start()
+    for t in ts:
+        t.join()
+    for e in errs:
+        if e is not None:
+            raise e
+    mate = np.concatenate([o[0] for o in out]) if n else np.zeros(0, np.int32)
+    return mate, out[0][1], [o[1] for o in out]
 
 
 # ----------------------------------------------------------------------------- the round loop

@@ -38,6 +38,48 @@ def test_edge_balanced_bounds():
         assert per.max() <= g.m / P + 32 * g.degrees().max() + 1
 
 
+def _bounds_by_definition(offsets, P, align):
+    """The partition rule of include/lmatch.h written out: bound p = the first row whose start
+    offset reaches floor(m p / P) (np.searchsorted, side='left'), rounded up to `align`, capped at
+    n and kept non-decreasing."""
+    n = len(offsets) - 1
+    m = int(offsets[-1])
+    b = [0]
+    for p in range(1, P):
+        v = int(np.searchsorted(offsets, (m * p) // P, side="left"))
+        b.append(max(b[-1], min(n, -(-v // align) * align)))
+    return np.array(b + [n], dtype=np.int64)
+
+
+def test_partition_in_c_matches_definition():
+    """lmatch_partition (the C partitioner, host-only) against the rule written out, on R-MAT,
+    a single-hub star (one row holds half the entries), empty graphs and P > n."""
+    rng = np.random.default_rng(5)
+    hub = graphgen.from_edges(500, [(0, v, 1.0) for v in range(1, 500)])
+    cases = [graphgen.rmat(12, 16, seed=3).offsets, graphgen.er(3000, 5.0, seed=2).offsets,
+             hub.offsets, np.zeros(1, np.int64), np.zeros(40, np.int64),
+             np.concatenate([[0], np.cumsum(rng.integers(0, 50, 777))]).astype(np.int64)]
+    for off in cases:
+        for P in (1, 2, 3, 7, 64):
+            for align in (1, 32, 64):
+                got = np.zeros(P + 1, np.int64)
+                rc = dist_mod._lib.lmatch_partition(off.ctypes.data, len(off) - 1, P, align,
+                                                    got.ctypes.data)
+                assert rc == 0
+                np.testing.assert_array_equal(got, _bounds_by_definition(off, P, align))
+    bad = np.array([1, 2], np.int64)
+    got = np.zeros(3, np.int64)
+    assert dist_mod._lib.lmatch_partition(bad.ctypes.data, 1, 2, 32, got.ctypes.data) == -1
+    assert dist_mod._lib.lmatch_partition(bad.ctypes.data, 1, 0, 32, got.ctypes.data) == -1
+
+
+def test_dist_id_new_unique():
+    ids = {dist_mod.dist_id_new() for _ in range(20)}
+    assert len(ids) == 20
+    for x in ids:
+        assert x.startswith(b"lmatch-") and len(x) == 64
+
+
 @pytest.mark.parametrize("P", [1, 2, 3, 5])
 def test_local_transport_numpy_model(P):
 

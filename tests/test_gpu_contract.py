@@ -239,3 +239,34 @@ def test_sort_chunk_option_range(lm):
         with pytest.raises(lm.LMatchError) as ei:
             lm.Matcher(g, algorithm="sorted", sort_chunk_log2=bad)
         assert ei.value.status == lm.LMATCH_EINVAL
+
+
+@pytest.mark.parametrize("round_loop", [0, 1, 2, 3])
+@pytest.mark.parametrize("maker", [
+    lambda: graphgen.rmat(16, 16, seed=11),
+    lambda: graphgen.er(30000, 12.0, seed=4, weights="paper"),
+    lambda: graphgen.mesh(200, keep=0.6, seed=5),
+    lambda: graphgen.from_edges(5000, [(0, v, float(np.float32(1.0 / (1 + v % 61)))) for v in range(1, 5000)]
+                                + [(v, v + 1, float(np.float32(0.3 + (v % 7) / 10))) for v in range(1, 4999)]),
+])
+def test_key_cache_identity(lm, maker, round_loop):
+    """The resident key cache (opts.key_cache; rows' 4 largest keys from the round-1 sweep, tile-
+    crossing rows merged) decides most pointers of rounds >= 2 without scanning the row: same
+    mate[], same pointing phases as Alg. 1 and as the cache-off path, fewer entries scanned."""
+    g = maker()
+    ref = oracle.greedy(g)
+    _, ph, _ = oracle.ld_frontier(g)
+    out = {}
+    for kc in (True, False):
+        with lm.Matcher(g, key_cache=kc, round_loop=round_loop) as M:
+            mate, st = M.run()
+            mate2, st2 = M.run()
+        np.testing.assert_array_equal(mate, ref.mate)
+        np.testing.assert_array_equal(mate2, ref.mate)
+        assert st["rounds"] == ph and st2["rounds"] == ph
+        assert math.isclose(st["weight"], ref.weight, rel_tol=WTOL)
+        out[kc] = st
+    if ph > 1:
+        assert out[True]["cache_rows"] > 0
+        assert out[True]["entries_swept"] <= out[False]["entries_swept"]
+    assert out[False]["cache_rows"] == 0
