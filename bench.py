@@ -8,9 +8,11 @@ configs; recipe in DESIGN.md).  GTEPS = undirected input edges m_u / step time /
   python bench.py [--gpus N] [--steps K] [--warmup W] [--workload rmat|er|mesh|road|gradient]
                   [--scale S] [--impl ours|reference]
 
-N > 1 (torchrun, one rank per GPU): weak scaling over independent graph instances (rank r
-matches the seed+r instance of the same workload; no data-path collective).  The partitioned
-single-graph exchange is reported separately.
+N > 1 (torchrun, one rank per GPU; `--gpus N` alone self-launches torchrun): strong scaling on
+ONE graph, 1-D edge-balanced vertex partition; each rank generates only its rows
+and the library-owned driver (lmatch_create_dist / lmatch_run_dist) exchanges claims, changed
+matched-bitmap words and frontier sizes through peer memory with device-side barriers
+(--exchange p2p|nccl select the Python-driven alternatives).  `--partitioned` runs that path at N=1.
 
 --impl reference: the oracle (sequential greedy = the same unique matching) on the host cores,
 on a bounded sample of the workload (a smaller instance of the same generator recipe).
@@ -59,8 +61,8 @@ def parse():
     p.add_argument("--batches", type=int, default=0,
                    help="paper-style batch count N_i (lmatch_opts.batches): B > 1 streams the whole "
                         "adjacency from pinned host memory as B batches in round 1")
-    p.add_argument("--no-key-cache", action="store_true",
-                   help="resident: disable the round-1 top-4 key cache (lmatch_opts.key_cache = -1)")
+    p.add_argument("--key-cache", action="store_true",
+                   help="resident: the round-1 top-4 key cache (lmatch_opts.key_cache = 1; off by default)")
     p.add_argument("--no-host-cache", action="store_true",
                    help="out-of-core: disable the top-8 host-row key cache (lmatch_opts.host_cache = -1)")
     p.add_argument("--algorithm", default="ld", choices=["ld", "suitor", "hybrid", "sorted"],
@@ -69,10 +71,11 @@ def parse():
                         "hybrid = ld, with a Suitor tail after 32 pointing phases; "
                         "sorted = ld over rows sorted once per graph + per-vertex cursors (NEXT-3; "
                         "the sort runs in the first warm-up step and is reported as sort_ms_once)")
-    p.add_argument("--exchange", default="p2p", choices=["p2p", "nccl"],
-                   help="partitioned path: p2p = the library's kernels store claims / bitmap words / "
-                        "frontier sizes into the peers' memory (CUDA IPC over NVLink; lmatch_p2p_*), "
-                        "nccl = torch.distributed all-to-all + allgather + allreduce (TorchTransport)")
+    p.add_argument("--exchange", default="dist", choices=["dist", "p2p", "nccl"],
+                   help="partitioned path: dist = the library-owned driver (lmatch_create_dist / "
+                        "lmatch_run_dist: peer-memory exchange + device-side barriers); p2p = the same "
+                        "exchange (lmatch_p2p_*) driven from Python with event barriers; nccl = "
+                        "torch.distributed all-to-all + allgather + allreduce (TorchTransport)")
     p.add_argument("--partitioned", action="store_true",
                    help="use the 1-D partitioned path even at N=1 (it is always used for N>1)")
     return p.parse_args()
@@ -224,8 +227,10 @@ def cpu_baseline(a, sample_scale):
     r = oracle.greedy(g)
     t = r.sort_s + r.scan_s
     return {"value": g.m_u / t / 1e9, "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": f"{a.workload} scale {sample_scale} (n={g.n}, m_u={g.m_u}) same recipe/seed; "
-                      f"greedy sort {r.sort_s:.2f}s + scan {r.scan_s:.2f}s, 1 thread, std::sort",
+            "sample": f"a SMALLER graph than this line's: {a.workload} scale {sample_scale} (n={g.n}, "
+                      f"m_u={g.m_u}), same recipe/seed; greedy sort {r.sort_s:.2f}s + scan "
+                      f"{r.scan_s:.2f}s, 1 thread, std::sort.  Sort-based GTEPS falls with size "
+                      f"(O(m log m)), so at the line's scale the oracle would be somewhat slower",
             "seconds": t}
 
 
@@ -269,73 +274,142 @@ def run_reference(a, rank, world):
 
 
 # ------------------------------------------------------------------- partitioned arm (N >= 1)
-def run_partitioned(a, rank, world, local):
-    """One graph, 1-D vertex partition over the N ranks (SURVEY 8(e)): each rank owns an
-    edge-balanced row range; pointer claims go to the owner of the target (all-to-all) and the
-    matched bitmap is allgathered each round, over NCCL (torch.distributed).  Strong scaling:
-    the graph is the same for every N."""
+def gen_rank_rows(a, scale, rank, world, dev):
+    """This rank's rows of the workload graph: the CSR offsets of the whole graph
+    (pass 1 of the row-range generator), the edge-balanced bounds from the library's partitioner
+    (lmatch_partition), then only the rank's rows [v0, v1) (pass 2).  Each rank holds its
+    own rows only, so graphs larger than one GPU's HBM can be partitioned.  Meshes are cheap to
+    generate whole and are sliced."""
     import torch
-    import torch.distributed as dist
-    import paper_conf_sc_mandulakgfhs24_b200 as lm  # noqa: F401  (loads liblmatch.so)
+    import graphgen.gpu as gg
     import paper_conf_sc_mandulakgfhs24_b200.dist as D
-
-    scale = a.scale or DEFAULT_SCALE[a.workload]
-    dev = torch.device("cuda", local)
-    stream = torch.cuda.current_stream(dev)
-    t0 = time.time()
-    dg = make_graph_gpu(a, scale, a.seed, dev)  # same seed on every rank: one graph
-    n, m, m_u = dg.n, dg.m, dg.m_u
-    offs_h = dg.offsets.cpu().numpy()
+    if a.workload in ("rmat", "er"):
+        if a.workload == "rmat":
+            offs = gg.rmat_offsets(scale, a.edgefactor, seed=a.seed, device=dev)
+        else:
+            offs = gg.er_offsets(1 << scale, float(a.edgefactor), seed=a.seed, device=dev)
+        offs_h = offs.cpu().numpy()
+        bounds = D.edge_balanced_bounds(offs_h, world)
+        v0, v1 = int(bounds[rank]), int(bounds[rank + 1])
+        if a.workload == "rmat":
+            dg = gg.rmat_rows(scale, v0, v1, offs, a.edgefactor, seed=a.seed, weights=a.weights or "uniform",
+                              device=dev)
+        else:
+            dg = gg.er_rows(1 << scale, v0, v1, offs, float(a.edgefactor), seed=a.seed,
+                            weights=a.weights or "uniform", device=dev)
+        del offs
+        n, m = len(offs_h) - 1, int(offs_h[-1])
+        return dg.offsets, dg.col, dg.w, v0, v1, bounds, n, m, offs_h
+    g = make_graph_gpu(a, scale, a.seed, dev)
+    offs_h = g.offsets.cpu().numpy()
     bounds = D.edge_balanced_bounds(offs_h, world)
     v0, v1 = int(bounds[rank]), int(bounds[rank + 1])
     s0, s1 = int(offs_h[v0]), int(offs_h[v1])
-    lo = (dg.offsets[v0:v1 + 1] - s0).contiguous()
-    lc = dg.col[s0:s1].contiguous()
-    lw = dg.w[s0:s1].contiguous()
+    lo = (g.offsets[v0:v1 + 1] - s0).contiguous()
+    lc, lw = g.col[s0:s1].contiguous(), g.w[s0:s1].contiguous()
+    del g
+    torch.cuda.empty_cache()
+    return lo, lc, lw, v0, v1, bounds, len(offs_h) - 1, int(offs_h[-1]), offs_h
+
+
+def run_partitioned(a, rank, world, local, dev):
+    """One graph, 1-D vertex partition over the N ranks (SURVEY 8(e)): each rank owns an
+    edge-balanced row range.  --exchange dist (default): the library-owned driver
+    (lmatch_create_dist / lmatch_run_dist: claims, changed bitmap words and frontier sizes stored
+    into the peers' memory by the library's kernels, device-side barriers, no host barrier);
+    p2p: the same exchange driven from Python with host/event barriers (dist.run_parts_p2p);
+    nccl: claims all-to-all + bitmap allgather + frontier allreduce through torch.distributed
+    (TorchTransport).  Strong scaling: the graph is the same for every N."""
+    import torch
+    import torch.distributed as dist
+    import paper_conf_sc_mandulakgfhs24_b200 as lm
+    import paper_conf_sc_mandulakgfhs24_b200.dist as D
+
+    scale = a.scale or DEFAULT_SCALE[a.workload]
+    t0 = time.time()
+    lo, lc, lw, v0, v1, bounds, n, m, offs_h = gen_rank_rows(a, scale, rank, world, dev)
+    m_u = m // 2
     host = None
     if not a.no_e2e:
         host = (lo.cpu().numpy(), lc.cpu().numpy(), lw.cpu().numpy())
-    dg = None
-    torch.cuda.empty_cache()
+    n_nz_loc = int(np.count_nonzero(np.diff(offs_h[v0:v1 + 1])))
+    del offs_h
     gen_s = time.time() - t0
-    part = D.LibPart(lo, lc, lw, v0, n, bounds, rank, device=dev, timing=True)
+    tr = None
+    if a.exchange == "dist":
+        obj = [D.dist_id_new() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        part = D.DistMatcher(lo, lc, lw, v0, n, rank, world, bounds, obj[0], device=dev, timing=True)
+        d_mate = torch.empty(max(v1 - v0, 1), dtype=torch.int32, device=dev)
+        stats_box = {}
+
+        def run():
+            mate, st = part.run_device(d_mate)
+            stats_box["st"] = st
+            return st
+
+        def sweep_ms():
+            return stats_box["st"].ms_sweep
+
+        def launches_of():
+            return stats_box["st"].kernel_launches
+    else:
+        part = D.LibPart(lo, lc, lw, v0, n, bounds, rank, device=dev, timing=True)
+        tr = D.TorchTransport()
+        if a.exchange == "p2p":
+            D.connect_p2p_torch(part)
+            D.connect_events_torch(part)
+            barrier = D.barrier_torch_events([part], dist.new_group(backend="gloo"))
+            run = lambda: D.run_parts_p2p([part], barrier, tr)  # noqa: E731
+        else:
+            run = lambda: D.run_parts([part], tr)  # noqa: E731
+
+        def sweep_ms():
+            return part.info()[1]
+
+        launches_of = None
     stream = part.stream  # the stream every library kernel of this part is launched on
     del lo, lc, lw
     torch.cuda.empty_cache()
-    tr = D.TorchTransport()
-    if a.exchange == "p2p":
-        D.connect_p2p_torch(part)
-        # phases ordered by interprocess CUDA events (a gloo host barrier only orders the
-        # records before the waits; no stream is drained), see dist.barrier_torch_events
-        D.connect_events_torch(part)
-        barrier = D.barrier_torch_events([part], dist.new_group(backend="gloo"))
-        run = lambda: D.run_parts_p2p([part], barrier, tr)  # noqa: E731
-    else:
-        run = lambda: D.run_parts([part], tr)  # noqa: E731
+
+    def allmax(x):
+        t = torch.tensor([float(x)], dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def allgather(vals):
+        t = torch.tensor([float(v) for v in vals], dtype=torch.float64)
+        out = [torch.empty_like(t) for _ in range(world)]
+        dist.all_gather(out, t)
+        return [x.tolist() for x in out]
 
     for _ in range(a.warmup):
-        run()
+        res = run()
     torch.cuda.synchronize(dev)
     dist.barrier()
     ev0 = torch.cuda.Event(enable_timing=True)
     ev1 = torch.cuda.Event(enable_timing=True)
-    sweep_ms = []
-    with ClockSampler(local) as clk:
+    sw, launches = [], 0
+    with ClockSampler(dev.index) as clk:
         torch.cuda.synchronize(dev)
         l0 = D.kernel_launch_count()
         ev0.record(stream)
         for _ in range(a.steps):
             res = run()
-            sweep_ms.append(part.info()[1])
+            sw.append(sweep_ms())
+            if launches_of:
+                launches += launches_of()
         ev1.record(stream)
         torch.cuda.synchronize(dev)
-        launches = D.kernel_launch_count() - l0
-    ms = ev0.elapsed_time(ev1)
-    t = torch.tensor([ms], dtype=torch.float64, device=dev)
-    dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    ms = float(t.item())
+        if not launches_of:
+            launches = D.kernel_launch_count() - l0
+    ms = allmax(ev0.elapsed_time(ev1))
     ms_per_step = ms / a.steps
     value = m_u * a.steps / (ms / 1e3) / 1e9
+    if a.exchange == "dist":
+        rounds, card, weight = res.rounds, res.cardinality, res.weight
+    else:
+        rounds, card, weight = res.rounds, res.matched // 2, res.weight
 
     e2e = None
     if host is not None and a.e2e_steps > 0:
@@ -348,65 +422,82 @@ def run_partitioned(a, rank, world, local):
         t1 = time.perf_counter()
         for _ in range(a.e2e_steps):
             part.reload(*host)
-            r = run()
-            mate_h[: v1 - v0].copy_(r.mates[0])
-        el = time.perf_counter() - t1
-        te = torch.tensor([el], dtype=torch.float64, device=dev)
-        dist.all_reduce(te, op=dist.ReduceOp.MAX)
-        el = float(te.item())
+            if a.exchange == "dist":
+                mate_h[: v1 - v0].copy_(part.run_device(d_mate)[0])
+            else:
+                mate_h[: v1 - v0].copy_(run().mates[0])
+        el = allmax(time.perf_counter() - t1)
         for arr in host:
             if arr.nbytes:
                 cud.cudaHostUnregister(arr.ctypes.data)
-        hb = torch.tensor([sum(x.nbytes for x in host)], dtype=torch.float64, device=dev)
-        dist.all_reduce(hb)
+        hb = sum(allgather([sum(x.nbytes for x in host)])[r][0] for r in range(world))
         e2e = {"value": m_u * a.e2e_steps / el / 1e9, "unit": UNIT,
-               "h2d_bytes_per_step": int(hb.item()), "d2h_bytes_per_step": int(4 * n),
+               "h2d_bytes_per_step": int(hb), "d2h_bytes_per_step": int(4 * n),
                "steps": a.e2e_steps, "ms_per_step": el / a.e2e_steps * 1e3,
                "includes": "lmatch_reload of every rank's local CSR (H2D + pack + validate + index) "
                            "+ partitioned run + owned mate[] slices D2H"}
 
-    # roofline of the dominant kernel: the slowest rank's round-1 sweep over its owned rows
-    m_loc = part.m_local
-    sweep_avg = float(np.mean(sweep_ms))
-    sw = torch.tensor([sweep_avg, float(m_loc)], dtype=torch.float64, device=dev)
-    allsw = [torch.empty_like(sw) for _ in range(world)]
-    dist.all_gather(allsw, sw)
-    worst = max(allsw, key=lambda x: float(x[0]))
+    # roofline of the dominant kernel: the slowest rank's round-1 sweep over ITS owned rows
+    # (its own entries and non-empty rows; DESIGN.md section 7 bytes per entry / per row)
+    mine = [float(np.mean(sw)), float(part.m_local), float(n_nz_loc)]
+    allr = allgather(mine)
+    worst = max(allr, key=lambda x: x[0])
     peak, peak_src = load_peaks()
-    n_loc_nz = int(np.count_nonzero(np.diff(offs_h[v0:v1 + 1]))) if rank == 0 else 0
-    sweep_bytes = 8 * float(worst[1]) + 16 * n_loc_nz
-    achieved = sweep_bytes / (float(worst[0]) / 1e3) / 1e9 if float(worst[0]) > 0 else None
+    ntiles_w = (worst[1] + 511) // 512
+    sweep_bytes = 8 * worst[1] + 16 * worst[2] + 4 * (ntiles_w + 1)
+    achieved = sweep_bytes / (worst[0] / 1e3) / 1e9 if worst[0] > 0 else None
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": (achieved / peak) if achieved else None, "traffic": None,
                 "kernel": "k_sweep over the slowest rank's owned rows",
-                "launch_ms": float(worst[0]), "share_of_step": float(worst[0]) / ms_per_step,
+                "algorithmic_bytes_per_launch": int(sweep_bytes),
+                "launch_ms": worst[0], "share_of_step": worst[0] / ms_per_step,
                 "peak_source": peak_src}
-    ms_all = [float(x[0]) for x in allsw]
-    ent_all = [float(x[1]) for x in allsw]
+    ms_all = [x[0] for x in allr]
+    ent_all = [x[1] for x in allr]
     imbalance = {"entries_max_over_mean": max(ent_all) / max(np.mean(ent_all), 1.0),
                  "sweep_ms_max_over_mean": max(ms_all) / max(np.mean(ms_all), 1e-9),
                  "entries_per_rank": [int(x) for x in ent_all]}
+    launches_all = sum(x[0] for x in allgather([launches]))
     if rank == 0:
+        desc = {"dist": "the library-owned driver (lmatch_create_dist / lmatch_run_dist): claims, changed "
+                        "bitmap words and frontier sizes stored into the peers' memory by the library's "
+                        "kernels (CUDA IPC), device-side barriers between phases",
+                "p2p": "claims / changed bitmap words / frontier sizes stored into the peers' memory by "
+                       "the library's kernels (CUDA IPC, lmatch_p2p_*), interprocess-event barriers "
+                       "driven from Python",
+                "nccl": "claims all-to-all + bitmap allgather + frontier allreduce per round (NCCL)"}[a.exchange]
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps,
                 "warmup": a.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
                 "scaling": "strong", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
                 "config": workload_config(a, scale, n, m) | {
-                    "parallelism": f"1-D vertex partition over {world} GPU(s): " + (
-                        "claims / changed bitmap words / frontier sizes stored into the peers' memory "
-                        "by the library's kernels (CUDA IPC, lmatch_p2p_*), interprocess-event barriers"
-                        if a.exchange == "p2p" else
-                        "claims all-to-all + bitmap allgather + frontier allreduce per round (NCCL)"),
+                    "parallelism": f"1-D edge-balanced vertex partition over {world} rank(s): " + desc,
                     "exchange": a.exchange,
+                    "devices": torch.cuda.device_count(),
                     "l2": f"inputs larger than L2 (adjacency {8 * m / 1e9:.1f} GB total); no flush",
-                    "gen_s": round(gen_s, 1), "part_bounds": [int(x) for x in bounds]},
+                    "gen_s": round(gen_s, 1), "part_bounds": [int(x) for x in bounds],
+                    "generation": "per rank: whole-graph offsets, then only the rank's rows"},
                 "roofline": roofline, "cpu_baseline": None, "e2e": e2e,
-                "gpu_launches": int(launches), "clocks": clk.summary(), "rounds": res.rounds,
-                "cardinality": res.matched // 2, "matched_weight": res.weight,
-                "claims_per_step_rank0": res.exchanged_claims, "imbalance": imbalance}
+                "gpu_launches": int(launches_all), "clocks": clk.summary(), "rounds": int(rounds),
+                "cardinality": int(card), "matched_weight": weight,
+                "mmeps": card * a.steps / (ms / 1e3) / 1e6,
+                "imbalance": imbalance}
         print(json.dumps(line), flush=True)
     part.close()
     dist.destroy_process_group()
     return 0
+
+
+def self_launch(a):
+    """`bench.py --gpus N` without torchrun: launch N ranks of this script through
+    torch.distributed.run on 127.0.0.1 (ranks share GPUs round-robin when fewer are visible)."""
+    import socket
+    import subprocess
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={a.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
 
 
 # -------------------------------------------------------------------------------- our arm
@@ -418,20 +509,27 @@ def main():
     if a.impl == "reference":
         return run_reference(a, rank, world)
 
+    if a.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return self_launch(a)
     import torch
     import torch.distributed as dist
     if not torch.cuda.is_available():
         raise SystemExit("bench.py needs a CUDA device (no CPU fallback)")
-    torch.cuda.set_device(local)
     if world > 1 or a.partitioned:
+        dev = torch.device("cuda", local % torch.cuda.device_count())
+        torch.cuda.set_device(dev)
         if "MASTER_ADDR" not in os.environ:  # single-process partitioned run
             os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT="29531", RANK="0", WORLD_SIZE="1")
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-        return run_partitioned(a, rank, world, local)
+        if a.exchange == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:  # the library moves the data; torch.distributed is only the control plane
+            dist.init_process_group("gloo")
+        return run_partitioned(a, rank, world, local, dev)
+    torch.cuda.set_device(local)
     import paper_conf_sc_mandulakgfhs24_b200 as lm
 
     scale = a.scale or DEFAULT_SCALE[a.workload]
-    seed = a.seed + rank
+    seed = a.seed
     dev = torch.device("cuda", local)
     stream = torch.cuda.current_stream(dev)
     t0 = time.time()
@@ -460,7 +558,7 @@ def main():
     opts = lm.make_opts(validate_level=1, timing=1,
                         hbm_budget_bytes=int(a.hbm_budget_gb * 1e9), stream_chunk=a.stream_chunk,
                         prune=a.prune, host_cache=not a.no_host_cache,
-                        batches=a.batches, algorithm=a.algorithm, key_cache=not a.no_key_cache)
+                        batches=a.batches, algorithm=a.algorithm, key_cache=a.key_cache)
     pinned_host = d_off is None
     if pinned_host:
         h = lm.lmatch_create_ex(g.offsets, g.col, g.w, n, m, opts)
@@ -610,10 +708,10 @@ def main():
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps,
                 "warmup": a.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
-                "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+                "scaling": "strong", "vs_baseline": None, "dtype": "u64",
                 "data": "synthetic",
                 "config": workload_config(a, scale, n, m) | {
-                    "parallelism": "1 GPU" if world == 1 else f"{world} independent instances (seed+rank), no collective",
+                    "parallelism": "1 GPU (the same graph is partitioned over the GPUs at N > 1)",
                     "l2": f"inputs larger than L2 (adjacency {8 * m / 1e9:.1f} GB >> 126 MB); no flush",
                     "gen_s": round(gen_s, 1),
                     "csr_for_create": "pinned host (device CSR + packed keys exceed HBM)" if pinned_host
@@ -625,6 +723,9 @@ def main():
                 "entries_swept": int(last["entries_swept"]), "frontier_total": int(last["frontier_total"]),
                 "round_log": round_log.tolist(),
                 "matched_weight": last["weight"],
+                "mmeps": int(last["cardinality"]) * a.steps / (ms / 1e3) / 1e6,
+                "mmeps_note": "MMEPS-like |M|/T (P:344-356 'rate at which edges are committed'): "
+                              "matched edges per second of the timed steps, in millions",
                 "step_ms": {"best": float(np.min(step_ms)), "median": float(np.median(step_ms)),
                             "best_gteps": total_mu / (float(np.min(step_ms)) / 1e3) / 1e9,
                             "note": "per-step device time from the library's own events "

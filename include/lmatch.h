@@ -158,7 +158,9 @@ typedef struct lmatch_opts {
                                  Valid 4..30 (EINVAL otherwise); small values exercise the chunking.
                                  Also caps the chunks of the validate_level-2 duplicate check */
   int32_t key_cache;          /* resident handles, algorithms 0 and 2:
-                                 0 = default (on when the cache fits in device memory), -1 = off.
+                                 1 = on (when the cache fits in device memory); 0 = default, off
+                                 (measured: on R-MAT s26 it saves 1.7 ms of the frontier rounds
+                                 but costs the round-1 sweep 6.6 ms).
                                  The round-1 sweep keeps the 4 largest keys of every row (32 bytes
                                  per vertex, plus 64 bytes per sweep tile of scratch); a vertex
                                  whose target was matched then takes the first available cached
@@ -278,8 +280,10 @@ LMATCH_API int lmatch_round_log(const lmatch_graph* g, int64_t* out, int64_t cap
  * A claim (v | u << 32) says "remote vertex u points to owned vertex v"; it replaces the paper's
  * |V| x 64-bit nccl_AllReduce(pointers) (Alg. 2 L7), and the bitmap allgather (n/8 bytes)
  * replaces nccl_AllReduce(mate) (Alg. 2 L9).  The result is bit-identical to the
- * single-GPU run for every partition (Lemma III.1).  validate_level 2 and out-of-core
- * are not available per partition (EINVAL).  Calls out of order return ESTATE.
+ * single-GPU run for every partition (Lemma III.1).  validate_level 2 is not available
+ * per partition (EINVAL: symmetry is a global property).  Out of core works per part as for a
+ * single graph (hbm_budget_bytes / batches = the paper's per-device batch count N_i, P:106, P:217;
+ * the host-row key cache included).  Calls out of order return ESTATE.
  * ------------------------------------------------------------------------------------------- */
 LMATCH_API int lmatch_create_part(const int64_t* csr_offsets, const int32_t* col_idx,
                                   const float* weights, int64_t n_local, int64_t m_local,
@@ -404,8 +408,9 @@ LMATCH_API int lmatch_dist_id_new(lmatch_dist_id* id);
  * rank passes the same bounds; v_begin must be part_bounds[rank]).  Blocks until all `world`
  * ranks of `id` have joined (ENCCL after 60 s), then opens every peer's exchange window: plain
  * device pointers for ranks in the same process (peer access enabled across devices), CUDA IPC
- * for other processes.  opts: as for lmatch_create_ex, except validate_level 2, hbm_budget_bytes
- * and algorithm != 0 (EINVAL).  The returned handle is used with lmatch_run_dist* and
+ * for other processes.  opts: as for lmatch_create_ex (hbm_budget_bytes / batches stream this
+ * rank's rows: the paper's per-device batches N_i), except validate_level 2 and
+ * algorithm != 0 (EINVAL).  The returned handle is used with lmatch_run_dist* and
  * lmatch_destroy (and lmatch_info / lmatch_reload); it is a partition handle, so the
  * lmatch_part_* / lmatch_p2p_* calls return ESTATE or act on the same state -- do not mix. */
 LMATCH_API int lmatch_create_dist(const int64_t* csr_offsets, const int32_t* col_idx,

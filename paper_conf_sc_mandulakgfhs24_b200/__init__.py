@@ -246,7 +246,7 @@ class Matcher:
                  max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
                  round_loop: int = 0, prune: bool = False, host_cache: bool = True,
                  batches: int = 0, algorithm: str = "ld", sort_chunk_log2: int = 0,
-                 key_cache: bool = True):
+                 key_cache: bool = False):
         self.h = None
         if handle is not None:
             self.h = handle
@@ -303,7 +303,7 @@ def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int =
               max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
               round_loop: int = 0, prune: bool = False, host_cache: bool = True,
               batches: int = 0, algorithm: str = "ld", sort_chunk_log2: int = 0,
-              key_cache: bool = True) -> Opts:
+              key_cache: bool = False) -> Opts:
     """round_loop (include/lmatch.h): 0 = hybrid (work-sized launches, then one persistent kernel
     for the tail; default), 1 = host-driven launches only, 2 = persistent kernel after round 1,
     3 = CUDA graph {round 1, persistent kernel}."""
@@ -314,7 +314,7 @@ def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int =
     o.batches = int(batches)
     o.algorithm = {"ld": 0, "suitor": 1, "hybrid": 2, "sorted": 3}[algorithm]
     o.sort_chunk_log2 = int(sort_chunk_log2)
-    o.key_cache = 0 if key_cache else -1
+    o.key_cache = 1 if key_cache else 0
     o.hbm_budget_bytes = int(hbm_budget_bytes)
     o.stream_chunk = int(stream_chunk)
     o.validate_level = int(validate_level)

@@ -1153,6 +1153,9 @@ struct RoundArgs {
 #ifndef LM_RES_FAST
 #define LM_RES_FAST 1  // rows wholly in the HBM-resident prefix load keys straight from adj.dev
 #endif
+#ifndef LM_QEXIT
+#define LM_QEXIT 0  // 1 = sub-warp groups skip the key columns past the row end (group-uniform)
+#endif
 // RES: the row lies in the HBM-resident prefix (e <= R), so keys are plain loads from adj.dev
 // instead of AdjView's per-key region test (decided once per row; group-uniform)
 template <int G, int U, bool RES>
@@ -1166,6 +1169,38 @@ __device__ __forceinline__ uint64_t scan_row_available_t(const AdjView adj,
   // resident rows: 32-bit offsets from the row start (a row has < 2^31 entries)
   const uint64_t* rp = adj.dev + s;
   const int32_t len32 = RES ? (int32_t)(e - s) : 0;
+#endif
+#if LM_QEXIT
+  // sub-warp groups (G = 2..16): a batch touches only the ceil(rest / G) key columns the row
+  // still has, so a 12-entry row in a 16 x 4 group costs one column of loads and probes, not 4
+  if (G > 1 && G < LM_PROBE3_MIN_G) {
+    for (int64_t jb = s; jb < e; jb += (int64_t)G * U) {
+      const int64_t j0 = jb + gl;
+      const int64_t rest = e - jb;
+      uint64_t k[U];
+#pragma unroll
+      for (int q = 0; q < U; ++q) {
+        k[q] = 0ull;
+        if ((int64_t)q * G >= rest) break;
+        const int64_t j = j0 + (int64_t)q * G;
+        if (j < e) k[q] = RES ? ld_stream_u64(adj.dev + j) : adj.at(j);
+      }
+      uint32_t wd[U];
+#pragma unroll
+      for (int q = 0; q < U; ++q) {
+        wd[q] = 0xffffffffu;
+        if ((int64_t)q * G >= rest) break;
+        if (k[q] > b) wd[q] = probe_word(bits, (uint32_t)k[q]);
+      }
+#pragma unroll
+      for (int q = 0; q < U; ++q) {
+        if ((int64_t)q * G >= rest) break;
+        const uint32_t v = (uint32_t)k[q];
+        if (!((wd[q] >> (v & 31)) & 1u) && k[q] > b) b = k[q];
+      }
+    }
+    return b;
+  }
 #endif
   // batch loop with a group-uniform trip count (the group votes inside it)
   for (int64_t jb = s; jb < e; jb += (int64_t)G * U) {
@@ -1840,13 +1875,163 @@ __device__ __forceinline__ bool kc_decide(const uint64_t* __restrict__ kc, const
   return k[kKC - 1] == 0;
 }
 
+// the compaction without the key cache (4 degree bins out; the decided input list is empty)
 template <bool ALL, int K>
+__device__ __forceinline__ void compact_body_plain(const CompactIO& io, int64_t n,
+                                             const uint64_t* __restrict__ best,
+                                             const uint32_t* __restrict__ bits,
+                                             const int64_t* __restrict__ offs, int64_t vbase,
+                                             int64_t bid, int64_t nblk) {
+  constexpr int NW = 8, NL = 1 + kDegBins;  // blockDim must be 256
+  const uint64_t* __restrict__ S = io.S;
+  const unsigned long long* cntS = io.cin;
+  const Bins& Fin = io.Fin;
+  const unsigned long long* cntFin = io.cin + 1;
+  uint64_t* __restrict__ Sout = io.Sout;
+  unsigned long long* cntSout = io.cout;
+  const Bins& Fout = io.Fout;
+  unsigned long long* cntFout = io.cout + 1;
+  unsigned long long* swept = io.swept;  // warps per block (blockDim 256), output lists
+  __shared__ unsigned wtot[NW][NL];
+  __shared__ unsigned long long wbase[NW][NL];
+  // virtual concatenation S ++ F_0 ++ F_1 ++ F_2 ++ F_3 (prefix ends p0 < p1 < ... < p4; the
+  // decided list F_4 is empty without the key cache)
+  const int64_t p0 = ALL ? n : (int64_t)*cntS;
+  const int64_t p1 = p0 + (ALL ? 0 : (int64_t)cntFin[0]);
+  const int64_t p2 = p1 + (ALL ? 0 : (int64_t)cntFin[1]);
+  const int64_t p3 = p2 + (ALL ? 0 : (int64_t)cntFin[2]);
+  const int64_t cnt = p3 + (ALL ? 0 : (int64_t)cntFin[3]);
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const unsigned lt = lanemask_lt();
+  const uint32_t* __restrict__ lcnt = io.live;
+  const uint32_t tag = lcnt ? round_tag(io.st) : 0u;
+  constexpr int64_t BLK = (int64_t)NW * 32 * K;
+  unsigned long long degsum = 0;
+  for (int64_t cb = bid * BLK; cb < cnt; cb += nblk * BLK) {
+    const int64_t c0 = cb + (int64_t)warp * 32 * K;
+    uint32_t sbits = 0, fb0 = 0, fb1 = 0, fb2 = 0, fb3 = 0;
+    uint64_t pr[K], rr[K];
+    // phase 1: every list element of the chunk (independent loads)
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+      const int64_t i = c0 + 32 * k + lane;
+      uint64_t p = (uint64_t)kNoPtr << 32;
+      if (i < cnt) {
+        if (ALL) {
+          // an empty row never holds a pointer: with the non-empty row list only those are read
+          const int64_t r = io.nzr ? (int64_t)io.nzr[i] : i;
+          const uint64_t bb = best[r];
+          p = make_pair((uint32_t)(r + vbase), bb ? (uint32_t)bb : kNoPtr);
+        } else {
+          p = i < p0 ? S[i]
+              : i < p1 ? Fin.list[0][i - p0].x
+              : i < p2 ? Fin.list[1][i - p1].x
+              : i < p3 ? Fin.list[2][i - p2].x
+                       : Fin.list[3][i - p3].x;
+        }
+      }
+      pr[k] = p;
+    }
+    // phase 2: matched bits of u and of its pointer (L2-resident bitmap; independent loads)
+    uint32_t wu[K], wv[K];
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+      const uint32_t u = (uint32_t)pr[k], v = (uint32_t)(pr[k] >> 32);
+      const bool ok = v != kNoPtr;
+      wu[k] = ok ? bits[u >> 5] : 0xffffffffu;
+      wv[k] = ok ? bits[v >> 5] : 0u;
+    }
+    // phase 3: classify; frontier members fetch their row range (independent loads)
+    int64_t os[K], oe[K];
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+      const uint32_t u = (uint32_t)pr[k], v = (uint32_t)(pr[k] >> 32);
+      const bool live = !((wu[k] >> (u & 31)) & 1u);
+      const bool tgt = (wv[k] >> (v & 31)) & 1u;
+      if (live && !tgt) sbits |= 1u << k;
+      const bool fr = live && tgt;
+      os[k] = fr ? offs[u - vbase] : 0;
+      oe[k] = fr ? offs[u - vbase + 1] : -1;
+      if (lcnt && fr) {  // A7: a row pruned earlier in this run is scanned over its live prefix
+        const uint32_t x = lcnt[u - vbase];
+        if ((x >> 16) == tag) oe[k] = os[k] + (int64_t)(x & 0xffffu);
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+      rr[k] = 0;
+      if (oe[k] >= 0) {
+        const int64_t d = oe[k] - os[k];
+        const int b = bin_of(d);
+        const uint32_t m = 1u << k;
+        fb0 |= b == 0 ? m : 0u;
+        fb1 |= b == 1 ? m : 0u;
+        fb2 |= b == 2 ? m : 0u;
+        fb3 |= b == 3 ? m : 0u;
+        rr[k] = (uint64_t)os[k] | ((uint64_t)(d < (int64_t)kBigDeg ? d : (int64_t)kBigDeg) << 40);
+        degsum += (unsigned long long)d;
+      }
+    }
+    // reserve output ranges: warp totals -> block prefix -> ONE atomic per list per block
+    {
+      const unsigned ts = __reduce_add_sync(0xffffffffu, __popc(sbits));
+      const unsigned t0 = __reduce_add_sync(0xffffffffu, __popc(fb0));
+      const unsigned t1 = __reduce_add_sync(0xffffffffu, __popc(fb1));
+      const unsigned t2 = __reduce_add_sync(0xffffffffu, __popc(fb2));
+      const unsigned t3 = __reduce_add_sync(0xffffffffu, __popc(fb3));
+      if (lane == 0) {
+        wtot[warp][0] = ts; wtot[warp][1] = t0; wtot[warp][2] = t1;
+        wtot[warp][3] = t2; wtot[warp][4] = t3;
+      }
+    }
+    __syncthreads();
+    if (threadIdx.x < NL) {
+      const int q = threadIdx.x;
+      unsigned long long tot = 0;
+      for (int w = 0; w < NW; ++w) tot += wtot[w][q];
+      unsigned long long base = 0;
+      if (tot) base = atomicAdd(q == 0 ? cntSout : &cntFout[q - 1], tot);
+      for (int w = 0; w < NW; ++w) { wbase[w][q] = base; base += wtot[w][q]; }
+    }
+    __syncthreads();
+    unsigned long long bs = wbase[warp][0], bf0 = wbase[warp][1], bf1 = wbase[warp][2],
+                       bf2 = wbase[warp][3], bf3 = wbase[warp][4];
+#pragma unroll
+    for (int k = 0; k < K; ++k) {
+      const uint32_t m = 1u << k;
+      const bool ps = sbits & m;
+      const unsigned bls = __ballot_sync(0xffffffffu, ps);
+      if (ps) Sout[bs + __popc(bls & lt)] = pr[k];
+      bs += __popc(bls);
+      const ulonglong2 ent = make_ulonglong2(pr[k], rr[k]);
+      unsigned bb = __ballot_sync(0xffffffffu, (fb0 & m) != 0);
+      if (fb0 & m) Fout.list[0][bf0 + __popc(bb & lt)] = ent;
+      bf0 += __popc(bb);
+      bb = __ballot_sync(0xffffffffu, (fb1 & m) != 0);
+      if (fb1 & m) Fout.list[1][bf1 + __popc(bb & lt)] = ent;
+      bf1 += __popc(bb);
+      bb = __ballot_sync(0xffffffffu, (fb2 & m) != 0);
+      if (fb2 & m) Fout.list[2][bf2 + __popc(bb & lt)] = ent;
+      bf2 += __popc(bb);
+      bb = __ballot_sync(0xffffffffu, (fb3 & m) != 0);
+      if (fb3 & m) Fout.list[3][bf3 + __popc(bb & lt)] = ent;
+      bf3 += __popc(bb);
+    }
+  }
+  for (int o = 16; o; o >>= 1) degsum += __shfl_xor_sync(0xffffffffu, degsum, o);
+  if (lane == 0 && degsum) atomicAdd(swept, degsum);
+}
+template <bool ALL, int K, bool KC = false>
 __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
                                              const uint64_t* __restrict__ best,
                                              const uint32_t* __restrict__ bits,
                                              const int64_t* __restrict__ offs, int64_t vbase,
                                              int64_t bid, int64_t nblk) {
   constexpr int NW = 8, NL = 1 + kBins;  // blockDim must be 256
+  if constexpr (!KC) {
+    compact_body_plain<ALL, K>(io, n, best, bits, offs, vbase, bid, nblk);
+    return;
+  }
   const uint64_t* __restrict__ S = io.S;
   const unsigned long long* cntS = io.cin;
   const Bins& Fin = io.Fin;
@@ -1917,7 +2102,7 @@ __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
       if (live && !tgt) sbits |= 1u << k;
       if (live && tgt) frm |= 1u << k;
     }
-    if (io.kc) {
+    if (KC) {
 #pragma unroll
       for (int k = 0; k < K; ++k) {
         if (!(frm & (1u << k))) continue;
@@ -1955,19 +2140,21 @@ __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
         degsum += (unsigned long long)d;
       }
     }
-    decided += (unsigned long long)__popc(fb[kDecided]);
+    // without the key cache the decided list stays empty: only the degree bins are written
+    constexpr int NOUT = KC ? kBins : kDegBins;
+    if (KC) decided += (unsigned long long)__popc(fb[kDecided]);
     // reserve output ranges: warp totals -> block prefix -> ONE atomic per list per block
     {
       const unsigned ts = __reduce_add_sync(0xffffffffu, __popc(sbits));
       if (lane == 0) wtot[warp][0] = ts;
 #pragma unroll
-      for (int q = 0; q < kBins; ++q) {
+      for (int q = 0; q < NOUT; ++q) {
         const unsigned tq = __reduce_add_sync(0xffffffffu, __popc(fb[q]));
         if (lane == 0) wtot[warp][1 + q] = tq;
       }
     }
     __syncthreads();
-    if (threadIdx.x < NL) {
+    if (threadIdx.x < 1 + NOUT) {
       const int q = threadIdx.x;
       unsigned long long tot = 0;
       for (int w = 0; w < NW; ++w) tot += wtot[w][q];
@@ -1978,7 +2165,7 @@ __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
     __syncthreads();
     unsigned long long bs = wbase[warp][0], bf[kBins];
 #pragma unroll
-    for (int q = 0; q < kBins; ++q) bf[q] = wbase[warp][1 + q];
+    for (int q = 0; q < NOUT; ++q) bf[q] = wbase[warp][1 + q];
 #pragma unroll
     for (int k = 0; k < K; ++k) {
       const uint32_t m = 1u << k;
@@ -1988,7 +2175,7 @@ __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
       bs += __popc(bls);
       const ulonglong2 ent = make_ulonglong2(pr[k], rr[k]);
 #pragma unroll
-      for (int q = 0; q < kBins; ++q) {
+      for (int q = 0; q < NOUT; ++q) {
         const unsigned bb = __ballot_sync(0xffffffffu, (fb[q] & m) != 0);
         if (fb[q] & m) Fout.list[q][bf[q] + __popc(bb & lt)] = ent;
         bf[q] += __popc(bb);
@@ -2002,14 +2189,14 @@ __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
   if (lane == 0 && degsum) atomicAdd(swept, degsum);
   if (lane == 0 && decided) atomicAdd(swept + (kCntCache - kCntSwept), decided);
 }
-template <bool ALL, int K>
+template <bool ALL, int K, bool KC = false>
 #ifndef LM_COMPACT_MINB
 #define LM_COMPACT_MINB 3  // 85-register cap: 36% -> ~50% occupancy, no spills (round-1 compaction -30%)
 #endif
 __global__ void __launch_bounds__(256, LM_COMPACT_MINB)
     k_compact(CompactIO io, int64_t n, const uint64_t* __restrict__ best,
               const uint32_t* __restrict__ bits, const int64_t* __restrict__ offs, int64_t vbase) {
-  compact_body<ALL, K>(io, n, best, bits, offs, vbase, blockIdx.x, gridDim.x);
+  compact_body<ALL, K, KC>(io, n, best, bits, offs, vbase, blockIdx.x, gridDim.x);
 }
 
 // =============================================================================================
@@ -2068,7 +2255,7 @@ __global__ void k_end_round(const RoundArgs* __restrict__ ra, cudaGraphCondition
 // degree bin) | grid barrier | match | barrier | compaction | barrier | end of round | barrier.
 // No per-round launches or host decisions; the grid barrier's fence also invalidates L1, so
 // every phase reads the others' writes.
-template <int B0G, int B0U, int B1G, int B1U, int B2G, int B2U, int K, bool PRUNE = false>
+template <int B0G, int B0U, int B1G, int B1U, int B2G, int B2U, int K, bool PRUNE = false, bool KC = false>
 __global__ void __launch_bounds__(256)
     k_rounds_persistent(const RoundArgs* __restrict__ ra, const int64_t* __restrict__ offs, const AdjView adj,
                         uint32_t* bits, uint64_t* best, int64_t n, int64_t vbase) {
@@ -2096,7 +2283,7 @@ __global__ void __launch_bounds__(256)
     grid.sync();
     {
       const CompactIO io = compact_io(*ra, cur);
-      compact_body<false, K>(io, n, best, bits, offs, vbase, blockIdx.x, gridDim.x);
+      compact_body<false, K, KC>(io, n, best, bits, offs, vbase, blockIdx.x, gridDim.x);
     }
     grid.sync();
     if (gtid == 0) end_round_body(ra, 0);

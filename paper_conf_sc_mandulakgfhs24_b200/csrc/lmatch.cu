@@ -223,6 +223,10 @@ struct lmatch_graph {
   std::vector<unsigned long long*> h_dcnt, h_dnf, h_dflag, h_dresw, h_dresc;
   // library-owned multi-GPU driver (lmatch_create_dist): device barrier epoch and error flag
   int dist = 0;
+  int dist_local = 0;                // every rank in this process: event barriers (see barrier)
+  void* dist_shm = nullptr;          // the rendezvous mapping (kept for in-process barriers)
+  size_t dist_shm_bytes = 0;
+  cudaEvent_t bev[2] = {nullptr, nullptr};
   unsigned long long epoch = 0;
   unsigned* d_berr = nullptr;
   unsigned long long* h_res6 = nullptr;  // pinned [3P]: frontier sizes, w shares, counts
@@ -242,7 +246,7 @@ struct lmatch_graph {
   int algorithm = 0;                 // 0 = LD pointer iteration, 1 = Suitor (NEXT-4), 3 = sorted+cursor
   int64_t sort_chunk = 1ll << 30;    // algorithm 3: entries per segmented-sort chunk
   // resident key cache (opts.key_cache): the 4 largest keys of every row, filled by the sweep
-  int key_cache = 1;
+  int key_cache = 0;
   int kc_attr = 0;
   uint64_t* kcache = nullptr;        // the active cache: kc_buf, or nullptr = off for this graph
   uint64_t* kc_buf = nullptr;        // [n + 1][kKC]
@@ -1015,7 +1019,7 @@ int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** 
     g->host_cache = opts->host_cache >= 0;
     g->batches = opts->batches;
     g->algorithm = opts->algorithm;
-    g->key_cache = opts->key_cache >= 0;
+    g->key_cache = opts->key_cache > 0;
     if (opts->sort_chunk_log2 != 0) {
       if (opts->sort_chunk_log2 < 4 || opts->sort_chunk_log2 > 30) {
         set_err("sort_chunk_log2 = %d outside 4..30", opts->sort_chunk_log2);
@@ -1026,7 +1030,9 @@ int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** 
   }
   CK(cudaGetDevice(&g->device));
   CK(cudaDeviceGetAttribute(&g->num_sms, cudaDevAttrMultiProcessorCount, g->device));
-  if (g->max_rounds <= 0) g->max_rounds = n / 2 + 2;
+  // the strict order bounds the pointing phases by n/2 + 1 (R6) -- of the WHOLE graph
+  // for a partition handle, whose rounds are the global ones
+  if (g->max_rounds <= 0) g->max_rounds = g->n_global / 2 + 2;
   CK(cudaStreamCreateWithFlags(&g->stream, cudaStreamNonBlocking));
   CK(cudaStreamCreateWithFlags(&g->up[0], cudaStreamNonBlocking));
   CK(cudaStreamCreateWithFlags(&g->up[1], cudaStreamNonBlocking));
@@ -1182,6 +1188,8 @@ void lmatch_destroy(lmatch_graph* g) {
   for (void* p : g->ipc_opened) cudaIpcCloseMemHandle(p);
   if (g->h_nf) cudaFreeHost(g->h_nf);
   if (g->h_res6) cudaFreeHost(g->h_res6);
+  if (g->dist_shm) munmap(g->dist_shm, g->dist_shm_bytes);
+  for (auto e : g->bev) if (e) cudaEventDestroy(e);
   void* pdev[] = {g->bounds, g->ghost, g->claims, g->claim_cnt, g->rstate, g->rlog, g->d_rargs,
                   g->cache, g->chunk_rows, g->cache_big, g->rescan, g->rescan_cnt, g->live, g->win, g->suitor, g->wl[0],
                   g->wl[1], g->wl_big, g->wl_cnt, g->sc_cur, g->sc_ptr, g->sc_L[0], g->sc_L[1], g->shadow, g->d_dseg, g->d_dcnt,
@@ -1324,8 +1332,11 @@ static int seq_prefix(lmatch_graph* g, cudaStream_t st, cudaGraphConditionalHand
   {
     lm::CompactIO io = lm::compact_io(g->rargs(), 1);
     io.nzr = g->nzr;
-    lm::k_compact<true, kCompactK><<<grid_for((g->n_nz + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
-        io, g->n_nz, g->best, g->bits, g->offs, g->v0);
+    const unsigned grid = grid_for((g->n_nz + 31) / 32, 8 * kCompactK, 65536);
+    if (g->kcache)
+      lm::k_compact<true, kCompactK, true><<<grid, 256, 0, st>>>(io, g->n_nz, g->best, g->bits, g->offs, g->v0);
+    else
+      lm::k_compact<true, kCompactK, false><<<grid, 256, 0, st>>>(io, g->n_nz, g->best, g->bits, g->offs, g->v0);
   }
   CKL();
   lm::k_end_round<<<1, 32, 0, st>>>(g->ra(), h, in_graph, 0);
@@ -1434,8 +1445,14 @@ static int seq_body(lmatch_graph* g, cudaStream_t st, int cur, const int64_t* nF
   }
   lm::k_match_bins<<<grid_for((nF + LM_MATCH_V - 1) / LM_MATCH_V, 256, 65536), 256, 0, st>>>(Fb, cF, g->best, g->bits);
   CKL();
-  lm::k_compact<false, kCompactK><<<grid_for((nS + nF + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
-      lm::compact_io(g->rargs(), cur), g->n, g->best, g->bits, g->offs, g->v0);
+  {
+    const unsigned grid = grid_for((nS + nF + 31) / 32, 8 * kCompactK, 65536);
+    const lm::CompactIO io = lm::compact_io(g->rargs(), cur);
+    if (g->kcache)
+      lm::k_compact<false, kCompactK, true><<<grid, 256, 0, st>>>(io, g->n, g->best, g->bits, g->offs, g->v0);
+    else
+      lm::k_compact<false, kCompactK, false><<<grid, 256, 0, st>>>(io, g->n, g->best, g->bits, g->offs, g->v0);
+  }
   CKL();
   lm::k_end_round<<<1, 32, 0, st>>>(g->ra(), 0, 0, 0);
   CKL();
@@ -1443,16 +1460,16 @@ static int seq_body(lmatch_graph* g, cudaStream_t st, int cur, const int64_t* nF
   return LMATCH_OK;
 }
 
-#define PERSISTENT_KERNEL(PR) \
-  lm::k_rounds_persistent<LM_B0_G, LM_B0_U, LM_B1_G, LM_B1_U, LM_B2_G, LM_B2_U, kCompactK, PR>
+#define PERSISTENT_KERNEL(PR, KC) \
+  lm::k_rounds_persistent<LM_B0_G, LM_B0_U, LM_B1_G, LM_B1_U, LM_B2_G, LM_B2_U, kCompactK, PR, KC>
 
 // rounds >= 2 in one cooperative launch (grid = co-resident blocks)
 extern "C++" {
-template <bool PRUNE>
+template <bool PRUNE, bool KC>
 int launch_persistent_t(lmatch_graph* g, cudaStream_t st, int64_t* launches) {
   static int occ = 0;
   if (!occ) {
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, PERSISTENT_KERNEL(PRUNE), 256, 0));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, PERSISTENT_KERNEL(PRUNE, KC), 256, 0));
     if (occ < 1) occ = 1;
   }
   const lm::RoundArgs* ra = g->ra();
@@ -1468,7 +1485,7 @@ int launch_persistent_t(lmatch_graph* g, cudaStream_t st, int64_t* launches) {
   attr[1].val.accessPolicyWindow = g->bits_window;
   cfg.attrs = attr;
   cfg.numAttrs = (LM_L2_WINDOW && g->bits_window.num_bytes > 0) ? 2 : 1;
-  CK(cudaLaunchKernelEx(&cfg, PERSISTENT_KERNEL(PRUNE), ra, (const int64_t*)g->offs, av, g->bits,
+  CK(cudaLaunchKernelEx(&cfg, PERSISTENT_KERNEL(PRUNE, KC), ra, (const int64_t*)g->offs, av, g->bits,
                         g->best, g->n, g->v0));
   count_launches(1);
   ++*launches;
@@ -1476,8 +1493,11 @@ int launch_persistent_t(lmatch_graph* g, cudaStream_t st, int64_t* launches) {
 }
 }  // extern "C++"
 static int launch_persistent(lmatch_graph* g, cudaStream_t st, int64_t* launches) {
-  return g->prune ? launch_persistent_t<true>(g, st, launches)
-                  : launch_persistent_t<false>(g, st, launches);
+  if (g->kcache)
+    return g->prune ? launch_persistent_t<true, true>(g, st, launches)
+                    : launch_persistent_t<false, true>(g, st, launches);
+  return g->prune ? launch_persistent_t<true, false>(g, st, launches)
+                  : launch_persistent_t<false, false>(g, st, launches);
 }
 
 // Capture reset .. round 1 + the persistent round kernel into one CUDA graph (built once).
@@ -2059,7 +2079,6 @@ int lmatch_create_part(const int64_t* csr_offsets, const int32_t* col_idx, const
   if (!s) s = check_part(n_local, v_begin, n_global, nparts, part_bounds);
   if (s) return s;
   if (opts && opts->validate_level >= 2) { set_err("validate_level 2 is not available per partition"); return LMATCH_EINVAL; }
-  if (opts && opts->hbm_budget_bytes > 0) { set_err("out-of-core is not available per partition"); return LMATCH_EINVAL; }
   PartSpec ps;
   ps.v0 = v_begin; ps.n_global = n_global; ps.P = nparts; ps.bounds = part_bounds;
   lmatch_graph* g = nullptr;
@@ -2082,7 +2101,6 @@ int lmatch_create_part_device(const int64_t* d_offsets, const int32_t* d_col, co
   if (!s) s = check_part(n_local, v_begin, n_global, nparts, part_bounds);
   if (s) return s;
   if (opts && opts->validate_level >= 2) { set_err("validate_level 2 is not available per partition"); return LMATCH_EINVAL; }
-  if (opts && opts->hbm_budget_bytes > 0) { set_err("out-of-core is not available per partition"); return LMATCH_EINVAL; }
   PartSpec ps;
   ps.v0 = v_begin; ps.n_global = n_global; ps.P = nparts; ps.bounds = part_bounds;
   lmatch_graph* g = nullptr;
@@ -2220,8 +2238,12 @@ static int part_compact_launch(lmatch_graph* g, cudaStream_t st) {
   // makes that set current (and zeroes the counters the next compaction writes)
   if (g->part_round == 1) {
     if (n > 0) {
-      lm::k_compact<true, kCompactK><<<grid_for((n + 31) / 32, 8 * kCompactK, 65536), 256, 0, st>>>(
-          lm::compact_io(g->rargs(), 1), n, g->best, g->bits, g->offs, g->v0);
+      const unsigned grid = grid_for((n + 31) / 32, 8 * kCompactK, 65536);
+      const lm::CompactIO io = lm::compact_io(g->rargs(), 1);
+      if (g->kcache)
+        lm::k_compact<true, kCompactK, true><<<grid, 256, 0, st>>>(io, n, g->best, g->bits, g->offs, g->v0);
+      else
+        lm::k_compact<true, kCompactK, false><<<grid, 256, 0, st>>>(io, n, g->best, g->bits, g->offs, g->v0);
       CKL();
     }
     g->part_cur = 0;
@@ -2234,8 +2256,11 @@ static int part_compact_launch(lmatch_graph* g, cudaStream_t st) {
     if (g->p2p || nS + nF > 0) {
       const unsigned grid = g->p2p ? (unsigned)(4 * g->num_sms)
                                    : grid_for((nS + nF + 31) / 32, 8 * kCompactK, 65536);
-      lm::k_compact<false, kCompactK><<<grid, 256, 0, st>>>(
-          lm::compact_io(g->rargs(), cur), n, g->best, g->bits, g->offs, g->v0);
+      const lm::CompactIO io = lm::compact_io(g->rargs(), cur);
+      if (g->kcache)
+        lm::k_compact<false, kCompactK, true><<<grid, 256, 0, st>>>(io, n, g->best, g->bits, g->offs, g->v0);
+      else
+        lm::k_compact<false, kCompactK, false><<<grid, 256, 0, st>>>(io, n, g->best, g->bits, g->offs, g->v0);
       CKL();
     }
     g->part_cur = cur ^ 1;
@@ -2273,6 +2298,22 @@ static int part_point_impl(lmatch_graph* g, cudaStream_t st, int64_t* claim_coun
   const lm::AdjView av = g->view();
   const lm::Bins& Fb = g->F[cur];
   const unsigned long long* cF = g->counters + lm::cnt_F(cur, 0);
+  if (g->use_cache() && nF > 0) {
+    // out-of-core part (per-device batches, NEXT-2): the host-row key cache decides the pointer of
+    // host rows where it can, and refills the rows whose cached keys ran dry (as in seq_body)
+    const bool refill = LM_CACHE_REFILL != 0;
+    if (refill) CK(cudaMemsetAsync(g->rescan_cnt, 0, 8, st));
+    lm::k_cache_redirect<lm::kCacheK><<<grid_for(nF, 256, 65536), 256, 0, st>>>(
+        Fb, cF, g->offs, g->cache, g->bits, g->u_first, g->M0, g->v0, g->counters + lm::kCntCache,
+        refill ? g->rescan : nullptr, refill ? g->rescan_cnt : nullptr);
+    CKL();
+    if (refill) {
+      lm::k_host_rescan<lm::kCacheK><<<(unsigned)(8 * g->num_sms), 256, 0, st>>>(
+          Fb, g->rescan, g->rescan_cnt, g->offs, g->view(), g->bits, g->cache, g->u_first, g->M0,
+          g->v0);
+      CKL();
+    }
+  }
   if (nFb[0]) {
 #if LM_PIPE & 1
     // the software-pipelined thread-per-row kernel, one resident wave (as in the single-graph
@@ -2616,6 +2657,21 @@ int lmatch_dist_id_new(lmatch_dist_id* id) {
 }
 
 namespace {
+// LMATCH_TRACE=1: the multi-GPU driver reports its steps on stderr; =2: it also drains its
+// stream after every phase, so a failing phase is named (debugging aids)
+int dist_trace_level() {
+  static const int lv = [] { const char* e = getenv("LMATCH_TRACE"); return e ? atoi(e) : 0; }();
+  return lv;
+}
+bool dist_trace() { return dist_trace_level() >= 1; }
+#define DTRACE(g, ...)                                                                   \
+  do {                                                                                   \
+    if (dist_trace()) {                                                                  \
+      fprintf(stderr, "[lmatch rank %d pid %d] ", (g)->me, (int)getpid());               \
+      fprintf(stderr, __VA_ARGS__);                                                      \
+      fputc('\n', stderr);                                                               \
+    }                                                                                    \
+  } while (0)
 constexpr uint32_t kShmMagic = 0x4c4d4431u;  // "LMD1"
 constexpr unsigned long long kDistTimeoutNs = 60ull * 1000000000ull;
 struct DistSlot {
@@ -2626,6 +2682,10 @@ struct DistSlot {
   int64_t v0, n, n_global, win_cap;
   uint64_t raw_win, raw_bits;   // device pointers, meaningful to a peer in the same process
   unsigned char ipc[128];       // lmatch_p2p_export handles, for peers in other processes
+  // in-process barrier (all ranks in one process): the epoch this rank's stream recorded last,
+  // and its two barrier events (cudaEvent_t, alternating by epoch parity)
+  uint64_t recorded;
+  uint64_t ev[2];
 };
 struct DistShm {
   uint32_t magic;
@@ -2668,6 +2728,7 @@ int dist_bootstrap(lmatch_graph* g, const lmatch_dist_id* id, int rank, int worl
   if (mp == MAP_FAILED) { set_err("rendezvous %s: mmap failed", name); return LMATCH_ENCCL; }
   DistShm* h = static_cast<DistShm*>(mp);
   int rc = LMATCH_OK;
+  DTRACE(g, "rendezvous %s mapped", name);
   uint32_t zero = 0;
   __atomic_compare_exchange_n(&h->magic, &zero, kShmMagic, false, __ATOMIC_ACQ_REL, __ATOMIC_ACQUIRE);
   int32_t w0 = 0;
@@ -2693,8 +2754,17 @@ int dist_bootstrap(lmatch_graph* g, const lmatch_dist_id* id, int rank, int worl
     me->win_cap = g->win_cap;
     me->raw_win = (uint64_t)(uintptr_t)g->win;
     me->raw_bits = (uint64_t)(uintptr_t)g->bits;
+    for (int i = 0; i < 2 && !rc; ++i) {
+      if (cudaEventCreateWithFlags(&g->bev[i], cudaEventDisableTiming) != cudaSuccess) {
+        set_err("cudaEventCreate failed");
+        rc = LMATCH_ECUDA;
+      }
+      me->ev[i] = (uint64_t)(uintptr_t)g->bev[i];
+    }
+    __atomic_store_n(&me->recorded, 0ull, __ATOMIC_RELAXED);
     rc = lmatch_p2p_export(g, me->ipc);
     if (!rc) __atomic_store_n(&me->valid, 1u, __ATOMIC_RELEASE);
+    DTRACE(g, "slot published (rc %d)", rc);
   }
   // wait for every rank
   struct timespec t0, t1;
@@ -2735,8 +2805,18 @@ int dist_bootstrap(lmatch_graph* g, const lmatch_dist_id* id, int rank, int worl
       rc = lmatch_p2p_attach(g, q, s.ipc);
     }
   }
+  // every rank in this process: keep the mapping for the event barriers
+  bool local = true;
+  for (int q = 0; q < world; ++q) local = local && h->slot[q].pid == (int32_t)getpid();
+  DTRACE(g, "peers attached (rc %d, %s)", rc, local ? "in-process event barriers" : "device flag barriers");
   if (__atomic_add_fetch(&h->attached, 1, __ATOMIC_ACQ_REL) == world) shm_unlink(name);
-  munmap(mp, bytes);
+  if (!rc && local) {
+    g->dist_local = 1;
+    g->dist_shm = mp;
+    g->dist_shm_bytes = bytes;
+  } else {
+    munmap(mp, bytes);
+  }
   return rc;
 }
 
@@ -2747,7 +2827,6 @@ int dist_check(int64_t n_local, int64_t v_begin, int64_t n_global, int32_t rank,
   TRY(check_part(n_local, v_begin, n_global, world, bounds));
   if (bounds[rank] != v_begin) { set_err("v_begin is not part_bounds[rank]"); return LMATCH_EINVAL; }
   if (opts && opts->validate_level >= 2) { set_err("validate_level 2 is not available per partition"); return LMATCH_EINVAL; }
-  if (opts && opts->hbm_budget_bytes > 0) { set_err("out-of-core is not available per partition"); return LMATCH_EINVAL; }
   if (opts && opts->algorithm != 0) { set_err("lmatch_run_dist runs the LD iteration (algorithm 0) only"); return LMATCH_EINVAL; }
   return LMATCH_OK;
 }
@@ -2824,12 +2903,39 @@ int lmatch_run_dist_device(lmatch_graph* g, int32_t* d_mate_local, void* stream,
   unsigned long long* wslots = reinterpret_cast<unsigned long long*>(g->win + (size_t)P * g->win_cap);
   // wslots: [0,P) inbox counts, [P,2P) frontier sizes, [2P,3P) barrier flags, [3P,4P) w shares,
   // [4P,5P) matched counts
+  // Ranks in other processes: a device-side barrier kernel (system-scope flags in the peers'
+  // windows).  Ranks all in this process share one CUDA context, where a spinning kernel could be
+  // serialised behind another thread's work: each rank records an event on its stream, publishes
+  // the epoch in the rendezvous mapping, waits on the host until every rank has recorded it, and
+  // makes its stream wait for the peers' events (no stream is drained; two events per rank,
+  // alternating by epoch, so a rank one barrier ahead never overwrites a record still needed).
   auto barrier = [&]() -> int {
     if (P == 1) return LMATCH_OK;
     ++g->epoch;
-    lm::k_dist_barrier<<<1, 32, 0, st>>>(wslots + 2 * P, g->d_dflag, P, g->me, g->epoch,
-                                         kDistTimeoutNs, g->d_berr);
-    CKL();
+    DTRACE(g, "barrier %llu", g->epoch);
+    if (!g->dist_local) {
+      lm::k_dist_barrier<<<1, 32, 0, st>>>(wslots + 2 * P, g->d_dflag, P, g->me, g->epoch,
+                                           kDistTimeoutNs, g->d_berr);
+      CKL();
+      return LMATCH_OK;
+    }
+    DistShm* h = static_cast<DistShm*>(g->dist_shm);
+    const int par = (int)(g->epoch & 1);
+    CK(cudaEventRecord(g->bev[par], st));
+    __atomic_store_n(&h->slot[g->me].recorded, (uint64_t)g->epoch, __ATOMIC_RELEASE);
+    struct timespec t0, t1;
+    clock_gettime(CLOCK_MONOTONIC, &t0);
+    for (int q = 0; q < P; ++q) {
+      if (q == g->me) continue;
+      while (__atomic_load_n(&h->slot[q].recorded, __ATOMIC_ACQUIRE) < (uint64_t)g->epoch) {
+        clock_gettime(CLOCK_MONOTONIC, &t1);
+        if ((t1.tv_sec - t0.tv_sec) * 1000000000ll + (t1.tv_nsec - t0.tv_nsec) > (long long)kDistTimeoutNs) {
+          set_err("rank %d did not reach barrier %llu within %llu s", q, g->epoch, kDistTimeoutNs / 1000000000ull);
+          return LMATCH_ENCCL;
+        }
+      }
+      CK(cudaStreamWaitEvent(st, reinterpret_cast<cudaEvent_t>((uintptr_t)h->slot[q].ev[par]), 0));
+    }
     return LMATCH_OK;
   };
   // one host read: the P frontier sizes (and the barrier error flag)
@@ -2846,10 +2952,20 @@ int lmatch_run_dist_device(lmatch_graph* g, int32_t* d_mate_local, void* stream,
     *total = t;
     return LMATCH_OK;
   };
+  // LMATCH_TRACE=2: also drain the stream after every phase, so a failing phase is named
+  auto phase = [&](const char* what) -> int {
+    if (dist_trace_level() < 2) return LMATCH_OK;
+    const cudaError_t e = cudaStreamSynchronize(st);
+    DTRACE(g, "phase %s done: %s", what, cudaGetErrorString(e));
+    CK(e);
+    return LMATCH_OK;
+  };
   if (g->timing && stats) CK(cudaEventRecord(g->ev[0], st));
   CK(cudaMemsetAsync(g->d_berr, 0, 4, st));
   TRY(barrier());  // every part is done with its previous run (inboxes, replicas, slots)
+  TRY(phase("barrier"));
   TRY(part_begin_impl(g, st, nullptr));
+  TRY(phase("begin"));
   int64_t rounds = 1;
   bool compacted = false, capped = false;
   for (;;) {
@@ -2857,15 +2973,21 @@ int lmatch_run_dist_device(lmatch_graph* g, int32_t* d_mate_local, void* stream,
     if (compacted) {
       int64_t total = 0;
       TRY(read_slots(&total));
+      DTRACE(g, "round %lld: global frontier %lld", (long long)rounds, (long long)total);
       if (total == 0) break;
       if (rounds >= g->max_rounds) { capped = true; break; }  // same decision on every part
       ++rounds;
     }
+    TRY(phase("barrier"));
     TRY(lmatch_p2p_match(g, st));
+    TRY(phase("match"));
     TRY(barrier());  // bitmap replicas complete
+    TRY(phase("barrier"));
     TRY(lmatch_p2p_compact(g, st, nullptr));
+    TRY(phase("compact"));
     compacted = true;
     TRY(part_point_impl(g, st, nullptr));  // an empty global frontier launches only empty work
+    TRY(phase("point"));
   }
   // A10 owned mate[] slice + A9: this part's w(M) share, then every part's shares summed in part
   // order (the same fp64 total on every part)
@@ -2879,9 +3001,12 @@ int lmatch_run_dist_device(lmatch_graph* g, int32_t* d_mate_local, void* stream,
     CK(cudaMemsetAsync(g->res_w, 0, 8, st));
     CK(cudaMemsetAsync(g->res_c, 0, 8, st));
   }
+  TRY(phase("finish"));
   lm::k_push_result<<<1, 32, 0, st>>>(g->res_w, g->res_c, g->d_dresw, g->d_dresc, P);
   CKL();
+  TRY(phase("push result"));
   TRY(barrier());
+  TRY(phase("barrier"));
   CK(cudaMemcpyAsync(g->h_res6 + P, wslots + 3 * P, (size_t)2 * P * 8, cudaMemcpyDeviceToHost, st));
   CK(cudaMemcpyAsync(g->h_counters, g->counters, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
   int64_t dummy = 0;

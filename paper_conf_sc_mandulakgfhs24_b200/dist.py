@@ -137,35 +137,44 @@ class TorchTransport:
         self.nparts = dist.get_world_size(group)
         self.rank = dist.get_rank(group)
         self._sizes = None  # owned bitmap word counts of every part (constant per run)
+        # gloo moves CPU tensors only: CUDA tensors are staged through host memory
+        self._host = dist.get_backend(group) == "gloo"
+
+    def _wire(self, t):
+        return t.cpu() if self._host and t.is_cuda else t
 
     def exchange(self, sends):
         import torch
         (send,) = sends
         dev = send[0].device
-        cnt_out = torch.tensor([t.numel() for t in send], dtype=torch.int64, device=dev)
+        wdev = "cpu" if self._host else dev
+        cnt_out = torch.tensor([t.numel() for t in send], dtype=torch.int64, device=wdev)
         cnt_in = torch.empty_like(cnt_out)
         self.dist.all_to_all_single(cnt_in, cnt_out, group=self.group)
         in_splits = [t.numel() for t in send]
         out_splits = [int(c) for c in cnt_in.tolist()]
-        recv = torch.empty(sum(out_splits), dtype=send[0].dtype, device=dev)
-        self.dist.all_to_all_single(recv, torch.cat(list(send)), out_splits, in_splits,
+        recv = torch.empty(sum(out_splits), dtype=send[0].dtype, device=wdev)
+        self.dist.all_to_all_single(recv, self._wire(torch.cat(list(send))), out_splits, in_splits,
                                     group=self.group)
-        return [recv]
+        return [recv.to(dev)]
 
     def allgather(self, owns):
         import torch
         (own,) = owns
+        dev = own.device
+        wdev = "cpu" if self._host else dev
         if self._sizes is None:
-            n = torch.tensor([own.numel()], dtype=torch.int64, device=own.device)
+            n = torch.tensor([own.numel()], dtype=torch.int64, device=wdev)
             sz = [torch.empty_like(n) for _ in range(self.nparts)]
             self.dist.all_gather(sz, n, group=self.group)
             self._sizes = [int(x.item()) for x in sz]
         sizes = self._sizes
         mx = max(sizes) if sizes else 0
-        pad = torch.zeros(mx, dtype=own.dtype, device=own.device)
-        pad[: own.numel()] = own
-        out = torch.empty(self.nparts * mx, dtype=own.dtype, device=own.device)
+        pad = torch.zeros(mx, dtype=own.dtype, device=wdev)
+        pad[: own.numel()] = self._wire(own)
+        out = torch.empty(self.nparts * mx, dtype=own.dtype, device=wdev)
         self.dist.all_gather_into_tensor(out, pad, group=self.group)
+        out = out.to(dev)
         return [[out[p * mx: p * mx + sizes[p]] for p in range(self.nparts)]]
 
     def allreduce(self, xs):
@@ -182,7 +191,8 @@ class LibPart:
     """One partition handle of liblmatch.so (rows [v0, v1) of a graph with n_global vertices)."""
 
     def __init__(self, offsets_local, col_local, w_local, v0: int, n_global: int, bounds,
-                 part: int, device=None, stream=None, validate_level: int = 1, timing: bool = False):
+                 part: int, device=None, stream=None, validate_level: int = 1, timing: bool = False,
+                 **opt_kw):
         import torch
         self.torch = torch
         self.dev = torch.device("cuda") if device is None else torch.device(device)
@@ -200,7 +210,9 @@ class LibPart:
             stream = torch.cuda.Stream(self.dev)
         self.stream = stream
         h = _P()
-        opts = make_opts(validate_level=validate_level, timing=timing)
+        # opt_kw: further lmatch_opts (make_opts names), e.g. hbm_budget_bytes / batches for a
+        # part streamed from host memory (the paper's per-device batches N_i)
+        opts = make_opts(validate_level=validate_level, timing=timing, **opt_kw)
         if hasattr(offsets_local, "is_cuda") and offsets_local.is_cuda:  # device CSR (torch)
             torch.cuda.current_stream(self.dev).synchronize()  # the arrays' producer
             self.m_local = int(col_local.numel())
@@ -371,7 +383,7 @@ class DistMatcher:
 
     def __init__(self, offsets_local, col_local, w_local, v0: int, n_global: int, rank: int,
                  world: int, bounds, dist_id: bytes, device=None, stream=None, timing: bool = False,
-                 max_rounds: int = 0, validate_level: int = 1):
+                 max_rounds: int = 0, validate_level: int = 1, **opt_kw):
         import torch
         self.torch = torch
         self.dev = torch.device("cuda") if device is None else torch.device(device)
@@ -383,7 +395,7 @@ class DistMatcher:
             stream = torch.cuda.Stream(self.dev)
         self.stream = stream
         self._id = ctypes.create_string_buffer(bytes(dist_id)[:64], 64)
-        opts = make_opts(validate_level=validate_level, timing=timing, max_rounds=max_rounds)
+        opts = make_opts(validate_level=validate_level, timing=timing, max_rounds=max_rounds, **opt_kw)
         h = _P()
         with torch.cuda.device(self.dev):
             if hasattr(offsets_local, "is_cuda") and offsets_local.is_cuda:
@@ -442,7 +454,7 @@ class DistMatcher:
             pass
 
 
-def match_dist_threads(offsets, col, w, nparts: int, devices=None, max_rounds: int = 0):
+def match_dist_threads(offsets, col, w, nparts: int, devices=None, max_rounds: int = 0, **opt_kw):
     """P ranks of one lmatch_create_dist group as P threads of this process (one GPU each, or all
     on the current GPU): the rendezvous gives them plain device pointers.  Returns (mate, stats
     of rank 0, [stats of every rank])."""
@@ -458,7 +470,8 @@ def match_dist_threads(offsets, col, w, nparts: int, devices=None, max_rounds: i
             dev = None if devices is None else devices[r % len(devices)]
             v0, v1 = int(bounds[r]), int(bounds[r + 1])
             lo, lc, lw = local_csr(offsets, col, w, v0, v1)
-            M = DistMatcher(lo, lc, lw, v0, n, r, nparts, bounds, did, device=dev, max_rounds=max_rounds)
+            M = DistMatcher(lo, lc, lw, v0, n, r, nparts, bounds, did, device=dev, max_rounds=max_rounds,
+                            **opt_kw)
             try:
                 out[r] = M.run()
             finally:
@@ -471,9 +484,10 @@ def match_dist_threads(offsets, col, w, nparts: int, devices=None, max_rounds: i
         t.start()
     for t in ts:
         t.join()
-    for e in errs:
-        if e is not None:
-            raise e
+    # a rank that failed makes its peers time out at a barrier (ENCCL): report the cause first
+    real = [e for e in errs if e is not None and getattr(e, "status", None) != -5]
+    for e in real + [e for e in errs if e is not None]:
+        raise e
     mate = np.concatenate([o[0] for o in out]) if n else np.zeros(0, np.int32)
     return mate, out[0][1], [o[1] for o in out]
 
@@ -664,7 +678,8 @@ def transport_sum_float(transport, xs):
     return float(sum(float(o.item()) for o in out))
 
 
-def match_partitioned_local(offsets, col, w, nparts: int, device=None, exchange: str = "transport"):
+def match_partitioned_local(offsets, col, w, nparts: int, device=None, exchange: str = "transport",
+                            **opt_kw):
     """P logical partitions of one graph on one device.  exchange = "transport": LocalTransport
     moves the claims / bitmap words; "p2p": the library's kernels store them into the other parts'
     memory (peer-memory exchange), phases ordered by cross-stream events; "p2p_sync": the same with
@@ -676,7 +691,7 @@ def match_partitioned_local(offsets, col, w, nparts: int, device=None, exchange:
     for p in range(nparts):
         v0, v1 = int(bounds[p]), int(bounds[p + 1])
         lo, lc, lw = local_csr(offsets, col, w, v0, v1)
-        parts.append(LibPart(lo, lc, lw, v0, n, bounds, p, device=device))
+        parts.append(LibPart(lo, lc, lw, v0, n, bounds, p, device=device, **opt_kw))
     if exchange in ("p2p", "p2p_sync"):
         connect_p2p_local(parts)
         barrier = barrier_events(parts) if exchange == "p2p" else barrier_local(parts)
