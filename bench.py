@@ -63,6 +63,8 @@ def parse():
                         "adjacency from pinned host memory as B batches in round 1")
     p.add_argument("--key-cache", action="store_true",
                    help="resident: the round-1 top-4 key cache (lmatch_opts.key_cache = 1; off by default)")
+    p.add_argument("--residual-mb", type=int, default=0,
+                   help="out of core: MiB of HBM for copies of rescanned host rows (lmatch_opts.residual_mb)")
     p.add_argument("--no-host-cache", action="store_true",
                    help="out-of-core: disable the top-8 host-row key cache (lmatch_opts.host_cache = -1)")
     p.add_argument("--algorithm", default="ld", choices=["ld", "suitor", "hybrid", "sorted"],
@@ -215,6 +217,30 @@ def load_traffic(config_key: str):
         return None if e is None else float(e["dram_bytes_per_launch"])
     except Exception:
         return None
+
+
+def per_round_roofline(round_log, round_ms, tail_from, peak):
+    """HBM roofline of every host-driven round >= 2 of the last timed step (and of the persistent
+    tail as one entry): algorithmic bytes = 8 B per adjacency entry scanned (E_r) + 64 B per
+    frontier vertex (F_r: bin entry 16, pointer write 8, list write 8, match: entry 8 + partner
+    pointer 8 + bitmap 16) + 16 B per live vertex the compaction reads and writes (L_r) -- DESIGN.md
+    section 7 -- over the round's device time (CUDA events on the launch stream)."""
+    out = []
+    rows = [list(map(int, r)) for r in round_log[1:]]  # rounds 2, 3, ...
+    for i, ms in enumerate(round_ms):
+        sel = rows[i:] if i == tail_from else rows[i:i + 1]
+        if not sel or ms <= 0:
+            continue
+        F = sum(r[0] for r in sel)
+        L = sum(r[1] for r in sel)
+        E = sum(r[2] for r in sel)
+        alg = 8 * E + 64 * F + 16 * L
+        gbs = alg / (ms / 1e3) / 1e9
+        out.append({"round": i + 2, "rounds": len(sel), "ms": round(float(ms), 4), "frontier": F,
+                    "live": L, "entries": E, "algorithmic_bytes": alg, "achieved_gbs": round(gbs, 1),
+                    "frac": round(gbs / peak, 3),
+                    **({"persistent_tail": True} if i == tail_from else {})})
+    return out
 
 
 # ------------------------------------------------------------------------------ cpu baseline
@@ -558,7 +584,7 @@ def main():
     opts = lm.make_opts(validate_level=1, timing=1,
                         hbm_budget_bytes=int(a.hbm_budget_gb * 1e9), stream_chunk=a.stream_chunk,
                         prune=a.prune, host_cache=not a.no_host_cache,
-                        batches=a.batches, algorithm=a.algorithm, key_cache=a.key_cache)
+                        batches=a.batches, algorithm=a.algorithm, key_cache=a.key_cache, residual_mb=a.residual_mb)
     pinned_host = d_off is None
     if pinned_host:
         h = lm.lmatch_create_ex(g.offsets, g.col, g.w, n, m, opts)
@@ -693,10 +719,12 @@ def main():
                "cache_bytes": int(last["cache_bytes"]),
                "cache_rows_per_step": int(last["cache_rows"]),
                "host_entries_read_per_step": int(last["host_entries_read"]),
+               "residual_mb": a.residual_mb, "residual_rows_per_step": int(last["residual_rows"]),
                "note": "sweep = resident HBM tiles + host chunks over PCIe (2-slot ring); later "
                        "rounds read host rows zero-copy, except rows whose pointer the top-8 "
                        "host-row key cache decides (filled in round 1; NEXT-1)"}
     round_log = lm.lmatch_round_log(h)
+    rounds_roofline = per_round_roofline(round_log, *lm.lmatch_round_ms(h), load_peaks()[0])
     lm.lmatch_destroy(h)
     del d_mate
     torch.cuda.empty_cache()
@@ -722,6 +750,7 @@ def main():
                 "rounds": int(rounds[-1]), "cardinality": int(last["cardinality"]),
                 "entries_swept": int(last["entries_swept"]), "frontier_total": int(last["frontier_total"]),
                 "round_log": round_log.tolist(),
+                "rounds_roofline": rounds_roofline,
                 "matched_weight": last["weight"],
                 "mmeps": int(last["cardinality"]) * a.steps / (ms / 1e3) / 1e6,
                 "mmeps_note": "MMEPS-like |M|/T (P:344-356 'rate at which edges are committed'): "

@@ -169,7 +169,15 @@ typedef struct lmatch_opts {
                                  keys are all matched are scanned again.  Same result, same
                                  pointing phases; lmatch_stats.entries_swept counts the rows
                                  actually scanned, cache_rows the pointers the cache decided */
-  int32_t reserved[5];
+  int32_t residual_mb;        /* out of core with the host-row cache (residual
+                                 rows): 0 = default (off); R > 0 = up to R MiB of HBM (on top of
+                                 hbm_budget_bytes, capped by free memory) for copies of host rows.
+                                 A host row that is rescanned (its 8 cached keys all matched) is
+                                 read over PCIe anyway; it is then also copied into this buffer
+                                 while space lasts, and later rounds -- and later runs on the same
+                                 graph -- scan the HBM copy instead (no extra PCIe traffic).
+                                 lmatch_stats.residual_rows counts the rows scanned from it */
+  int32_t reserved[4];
 } lmatch_opts;
 
 /* Filled by lmatch_run / lmatch_run_device when non-NULL. */
@@ -202,7 +210,8 @@ typedef struct lmatch_stats {
                                 iteration stopped at 32 pointing phases (0 = not needed) */
   double ms_sort;            /* algorithm 3: device time of the row sort this run performed (the
                                 first run after create/reload); 0 when the rows were already sorted */
-  int64_t reserved[1];
+  int64_t residual_rows;     /* out of core, opts.residual_mb: frontier rows of rounds >= 2
+                                scanned from their HBM residual copy instead of host memory */
 } lmatch_stats;
 
 /* Library / ABI identification.  Returns LMATCH_ABI_VERSION. */
@@ -258,6 +267,13 @@ LMATCH_API int lmatch_info(const lmatch_graph* g, int64_t* n, int64_t* m, int64_
  * by the compaction), out[3r+2] = E(F_r) (adjacency entries scanned).  Writes at most `cap` rounds;
  * *nrounds receives the number of rounds.  (Fig. 8 "edges accessed per iteration".) */
 LMATCH_API int lmatch_round_log(const lmatch_graph* g, int64_t* out, int64_t cap, int64_t* nrounds);
+
+/* (timing = 1) Device time of the host-driven rounds >= 2 of the last lmatch_run* on a
+ * single-graph handle: ms[i] = round i + 2 (writes at most `cap`), *nrounds = how many were timed.
+ * When the default round loop handed the small tail to the persistent kernel, the LAST timed entry
+ * is that whole tail and *tail_from = its index (else -1).  0 rounds without timing. */
+LMATCH_API int lmatch_round_ms(const lmatch_graph* g, double* ms, int64_t cap, int64_t* nrounds,
+                               int64_t* tail_from);
 
 /* ---------------------------------------------------------------------------------------------
  * Partitioned mode (multi-GPU, one process or thread per GPU).

@@ -20,7 +20,8 @@ __all__ = [
     "LMatchError", "Opts", "Stats", "Matcher", "lib_path",
     "lmatch_abi_version", "lmatch_create", "lmatch_create_ex", "lmatch_create_device",
     "lmatch_reload", "lmatch_run", "lmatch_run_device", "lmatch_weight", "lmatch_weight_device",
-    "lmatch_info", "lmatch_round_log", "lmatch_destroy", "lmatch_strerror", "lmatch_last_error",
+    "lmatch_info", "lmatch_round_log", "lmatch_round_ms", "lmatch_destroy", "lmatch_strerror",
+    "lmatch_last_error",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -46,7 +47,8 @@ class Opts(ctypes.Structure):
         ("round_loop", ctypes.c_int32), ("prune", ctypes.c_int32),
         ("host_cache", ctypes.c_int32), ("batches", ctypes.c_int32),
         ("algorithm", ctypes.c_int32), ("sort_chunk_log2", ctypes.c_int32),
-        ("key_cache", ctypes.c_int32), ("reserved", ctypes.c_int32 * 5),
+        ("key_cache", ctypes.c_int32), ("residual_mb", ctypes.c_int32),
+        ("reserved", ctypes.c_int32 * 4),
     ]
 
 
@@ -62,11 +64,11 @@ class Stats(ctypes.Structure):
         ("kernel_launches", ctypes.c_int64), ("bytes_streamed", ctypes.c_int64),
         ("resident_entries", ctypes.c_int64), ("cache_rows", ctypes.c_int64),
         ("host_entries_read", ctypes.c_int64), ("cache_bytes", ctypes.c_int64),
-        ("tail_passes", ctypes.c_int64), ("ms_sort", ctypes.c_double), ("reserved", ctypes.c_int64 * 1),
+        ("tail_passes", ctypes.c_int64), ("ms_sort", ctypes.c_double), ("residual_rows", ctypes.c_int64),
     ]
 
     def as_dict(self) -> dict:
-        return {k: getattr(self, k) for k, _ in self._fields_ if k != "reserved"}
+        return {k: getattr(self, k) for k, _ in self._fields_}
 
 
 _P = ctypes.c_void_p
@@ -85,6 +87,7 @@ _sig = {
     "lmatch_info": ([_P, ctypes.POINTER(_I64), ctypes.POINTER(_I64), ctypes.POINTER(_I64),
                      ctypes.POINTER(_I64)], ctypes.c_int),
     "lmatch_round_log": ([_P, _P, _I64, ctypes.POINTER(_I64)], ctypes.c_int),
+    "lmatch_round_ms": ([_P, _P, _I64, ctypes.POINTER(_I64), ctypes.POINTER(_I64)], ctypes.c_int),
     "lmatch_destroy": ([_P], None),
     "lmatch_strerror": ([ctypes.c_int], ctypes.c_char_p),
     "lmatch_last_error": ([], ctypes.c_char_p),
@@ -232,6 +235,17 @@ def lmatch_round_log(h: int) -> np.ndarray:
     return out[: nr.value]
 
 
+def lmatch_round_ms(h: int):
+    """(timing=1) per-round device ms of the host-driven rounds >= 2 of the last run, and the index
+    of the entry that covers the persistent-kernel tail (-1 if none)."""
+    nr, tf = _I64(), _I64()
+    _check(_lib.lmatch_round_ms(h, None, 0, ctypes.byref(nr), ctypes.byref(tf)), "lmatch_round_ms")
+    out = np.zeros(max(nr.value, 1), dtype=np.float64)
+    _check(_lib.lmatch_round_ms(h, out.ctypes.data, nr.value, ctypes.byref(nr), ctypes.byref(tf)),
+           "lmatch_round_ms")
+    return out[: nr.value], int(tf.value)
+
+
 def lmatch_destroy(h: int | None) -> None:
     _lib.lmatch_destroy(h)
 
@@ -246,7 +260,7 @@ class Matcher:
                  max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
                  round_loop: int = 0, prune: bool = False, host_cache: bool = True,
                  batches: int = 0, algorithm: str = "ld", sort_chunk_log2: int = 0,
-                 key_cache: bool = False):
+                 key_cache: bool = False, residual_mb: int = 0):
         self.h = None
         if handle is not None:
             self.h = handle
@@ -257,7 +271,8 @@ class Matcher:
                                       opts=make_opts(validate_level, timing, upload_chunk,
                                                      max_rounds, hbm_budget_bytes, stream_chunk,
                                                      round_loop, prune, host_cache, batches,
-                                                     algorithm, sort_chunk_log2, key_cache))
+                                                     algorithm, sort_chunk_log2, key_cache,
+                                                     residual_mb))
         self.info = lmatch_info(self.h)
 
     @classmethod
@@ -303,7 +318,7 @@ def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int =
               max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
               round_loop: int = 0, prune: bool = False, host_cache: bool = True,
               batches: int = 0, algorithm: str = "ld", sort_chunk_log2: int = 0,
-              key_cache: bool = False) -> Opts:
+              key_cache: bool = False, residual_mb: int = 0) -> Opts:
     """round_loop (include/lmatch.h): 0 = hybrid (work-sized launches, then one persistent kernel
     for the tail; default), 1 = host-driven launches only, 2 = persistent kernel after round 1,
     3 = CUDA graph {round 1, persistent kernel}."""
@@ -315,6 +330,7 @@ def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int =
     o.algorithm = {"ld": 0, "suitor": 1, "hybrid": 2, "sorted": 3}[algorithm]
     o.sort_chunk_log2 = int(sort_chunk_log2)
     o.key_cache = 1 if key_cache else 0
+    o.residual_mb = int(residual_mb)
     o.hbm_budget_bytes = int(hbm_budget_bytes)
     o.stream_chunk = int(stream_chunk)
     o.validate_level = int(validate_level)

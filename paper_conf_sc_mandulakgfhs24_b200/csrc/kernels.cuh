@@ -99,8 +99,13 @@ struct AdjView {
   int64_t R;
   const uint64_t* cache_off = nullptr;
   int64_t M0 = INT64_MAX;
+  // out of core, residual rows (NEXT-1): host rows copied into HBM when first rescanned, at
+  // indices >= M2 (res_off pre-offset by -M2)
+  const uint64_t* res_off = nullptr;
+  int64_t M2 = INT64_MAX;
   __device__ __forceinline__ uint64_t at(int64_t j) const {
-    return j < R ? ld_stream_u64(dev + j) : (j < M0 ? host_off[j] : __ldg(cache_off + j));
+    return j < R ? ld_stream_u64(dev + j)
+                 : (j < M0 ? host_off[j] : (j < M2 ? __ldg(cache_off + j) : __ldg(res_off + j)));
   }
   __device__ __forceinline__ uint64_t* ptr(int64_t j) const {
     return const_cast<uint64_t*>(j < R ? dev + j : host_off + j);
@@ -2798,10 +2803,11 @@ __global__ void k_cache_redirect(Bins F, const unsigned long long* __restrict__ 
                                  const uint32_t* __restrict__ bits, int64_t u_first, int64_t M0,
                                  int64_t vbase, unsigned long long* cnt,
                                  uint64_t* __restrict__ rescan = nullptr,
-                                 unsigned long long* nrescan = nullptr) {
+                                 unsigned long long* nrescan = nullptr,
+                                 const int64_t* __restrict__ roff = nullptr, int64_t M2 = 0) {
   const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  unsigned long long served = 0, left = 0;
+  unsigned long long served = 0, left = 0, resid = 0;
   for (int bb = 0; bb < kDegBins; ++bb) {
     const int64_t c = (int64_t)cntF[bb];
     for (int64_t i = tid; i < c; i += stride) {
@@ -2830,6 +2836,13 @@ __global__ void k_cache_redirect(Bins F, const unsigned long long* __restrict__ 
         e.y = (1ull << 40) | (uint64_t)(M0 + slot + hit);
       } else if (en - s <= K) {
         e.y = (uint64_t)(M0 + slot);
+      } else if (roff && roff[u - u_first] >= 0) {
+        // a residual row: its copy in HBM is scanned by the pointer kernels (no host read)
+        const int64_t d = en - s;
+        e.y = (uint64_t)(M2 + roff[u - u_first]) | ((uint64_t)(d < (int64_t)kBigDeg ? d : (int64_t)kBigDeg) << 40);
+        F.list[bb][i].y = e.y;
+        ++resid;
+        continue;
       } else {
         left += (unsigned long long)(en - s);
         // refill path: k_host_rescan reads the row once, refills the cache with its K largest
@@ -2844,10 +2857,12 @@ __global__ void k_cache_redirect(Bins F, const unsigned long long* __restrict__ 
   for (int o = 16; o; o >>= 1) {
     served += __shfl_xor_sync(0xffffffffu, served, o);
     left += __shfl_xor_sync(0xffffffffu, left, o);
+    resid += __shfl_xor_sync(0xffffffffu, resid, o);
   }
   if ((threadIdx.x & 31) == 0) {
     if (served) atomicAdd(&cnt[0], served);
     if (left) atomicAdd(&cnt[1], left);
+    if (resid) atomicAdd(&cnt[2], resid);
   }
 }
 
@@ -2863,7 +2878,11 @@ __global__ void __launch_bounds__(256) k_host_rescan(Bins F, const uint64_t* __r
                                                      const int64_t* __restrict__ offs, AdjView adj,
                                                      const uint32_t* __restrict__ bits,
                                                      uint64_t* __restrict__ cache, int64_t u_first,
-                                                     int64_t M0, int64_t vbase) {
+                                                     int64_t M0, int64_t vbase,
+                                                     uint64_t* __restrict__ res = nullptr,
+                                                     int64_t res_cap = 0,
+                                                     unsigned long long* res_used = nullptr,
+                                                     int64_t* __restrict__ roff = nullptr) {
   const int lane = threadIdx.x & 31;
   const int64_t c = (int64_t)*nrescan;
   const int64_t wid = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -2879,10 +2898,20 @@ __global__ void __launch_bounds__(256) k_host_rescan(Bins F, const uint64_t* __r
     uint64_t t[K];
 #pragma unroll
     for (int q = 0; q < K; ++q) t[q] = 0ull;
+    // residual rows (NEXT-1): the row is read over PCIe here anyway, so it is also copied into
+    // the HBM residual buffer while space lasts; later rescans of it read HBM instead
+    unsigned long long base = ~0ull;
+    if (res && lane == 0) {
+      const unsigned long long b0 = atomicAdd(res_used, (unsigned long long)(en - s));
+      if ((int64_t)b0 + (en - s) <= res_cap) base = b0;
+    }
+    base = __shfl_sync(0xffffffffu, base, 0);
     for (int64_t j = s + lane; j < en; j += 32) {
       const uint64_t k = adj.at(j);
+      if (base != ~0ull) res[base + (j - s)] = k;
       if (k && !bit_test(bits, (uint32_t)k)) topk_insert<K>(t, k);
     }
+    if (base != ~0ull && lane == 0) roff[u - u_first] = (int64_t)base;
     const uint64_t mine = warp_topk_pop<K>(t);
     const int64_t slot = (u - u_first) * K;
     if (lane < K) cache[slot + lane] = mine;

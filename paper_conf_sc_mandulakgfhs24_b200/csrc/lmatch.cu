@@ -281,6 +281,14 @@ struct lmatch_graph {
   int64_t cap_rescan = -1;
   int64_t* cache_big = nullptr;      // device [1 + cap]: count, then rows listed for the CTA fill
   int64_t cap_cache_big = -1;
+  // residual rows (opts.residual_mb): HBM copies of rescanned host rows, roff[u - u_first] = their
+  // start in `res` (-1 = not copied), addressed through AdjView as indices >= M2
+  int residual_mb = 0;
+  uint64_t* res = nullptr;
+  int64_t cap_res = -1, M2 = INT64_MAX;
+  unsigned long long* res_used = nullptr;
+  int64_t* roff = nullptr;
+  int64_t cap_roff = -1;
   bool use_cache() const { return streaming && cache != nullptr; }
   cudaEvent_t ev_full[2] = {}, ev_free[2] = {};
   int sweep_grid = 0;
@@ -322,6 +330,9 @@ struct lmatch_graph {
   cudaEvent_t ev[8] = {};
   int64_t device_bytes = 0;
   std::vector<int64_t> round_log;  // per round: |F_r|, |L_r|, E(F_r) (directed entries scanned)
+  // (timing=1) per-round events of the host-driven rounds >= 2 of the last run (lmatch_round_ms)
+  std::vector<cudaEvent_t> rev;
+  int64_t n_rev = 0, tail_rounds_from = -1;
   // device-side round loop
   lm::RoundState* rstate = nullptr;
   lm::RoundArgs* d_rargs = nullptr;    // device copy of rargs() (kernels read it by pointer)
@@ -337,6 +348,7 @@ struct lmatch_graph {
   lm::AdjView view() const {
     lm::AdjView v{adj, host_adj_dev - R, R};
     if (use_cache()) { v.cache_off = cache - M0; v.M0 = M0; }
+    if (use_cache() && res) { v.res_off = res - M2; v.M2 = M2; }
     return v;
   }
   const lm::RoundArgs* ra() const { return d_rargs; }
@@ -858,6 +870,24 @@ int build_cache_index(lmatch_graph* g, cudaStream_t st) {
   // a window holds at most (entries / kCacheBigRow) rows longer than kCacheBigRow
   TRY(ensure(g, &g->cache_big, &g->cap_cache_big, std::max(C, g->R) / lm::kCacheBigRow + 8));
   g->M0 = g->m + 64;  // past the host part and its padding
+  // residual rows: a buffer of up to residual_mb MiB (leaving 1 GiB of free memory), reset per
+  // loaded graph; the copies persist across runs on the same graph
+  if (g->residual_mb > 0) {
+    size_t fr = 0, tot = 0;
+    CK(cudaMemGetInfo(&fr, &tot));
+    int64_t want = (int64_t)g->residual_mb * (1ll << 20) / 8;
+    if (g->res && g->cap_res >= want) want = g->cap_res;
+    const int64_t room = ((int64_t)fr - (1ll << 30)) / 8 + (g->res ? g->cap_res : 0);
+    want = std::min(want, room);
+    if (want > 0) {
+      TRY(ensure(g, &g->res, &g->cap_res, want));
+      TRY(ensure(g, &g->roff, &g->cap_roff, g->n - uf + 1));
+      if (!g->res_used) TRY(dmalloc(g, &g->res_used, 1));
+      CK(cudaMemsetAsync(g->res_used, 0, 8, st));
+      CK(cudaMemsetAsync(g->roff, 0xff, (size_t)(g->n - uf + 1) * 8, st));
+      g->M2 = g->M0 + g->cap_cache;
+    }
+  }
   return LMATCH_OK;
 }
 
@@ -1020,6 +1050,7 @@ int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** 
     g->batches = opts->batches;
     g->algorithm = opts->algorithm;
     g->key_cache = opts->key_cache > 0;
+    g->residual_mb = opts->residual_mb;
     if (opts->sort_chunk_log2 != 0) {
       if (opts->sort_chunk_log2 < 4 || opts->sort_chunk_log2 > 30) {
         set_err("sort_chunk_log2 = %d outside 4..30", opts->sort_chunk_log2);
@@ -1194,12 +1225,13 @@ void lmatch_destroy(lmatch_graph* g) {
                   g->cache, g->chunk_rows, g->cache_big, g->rescan, g->rescan_cnt, g->live, g->win, g->suitor, g->wl[0],
                   g->wl[1], g->wl_big, g->wl_cnt, g->sc_cur, g->sc_ptr, g->sc_L[0], g->sc_L[1], g->shadow, g->d_dseg, g->d_dcnt,
                   g->d_dbits, g->d_dnf, g->d_dflag, g->d_dresw, g->d_dresc, g->d_berr,
-                  g->kc_buf, g->xpart, g->xrows, g->nx};
+                  g->kc_buf, g->xpart, g->xrows, g->nx, g->res, g->res_used, g->roff};
   for (void* p : pdev) if (p) cudaFree(p);
   if (g->h_claim_cnt) cudaFreeHost(g->h_claim_cnt);
   if (g->h_res) cudaFreeHost(g->h_res);
   if (g->h_resc) cudaFreeHost(g->h_resc);
   for (auto e : g->ev) if (e) cudaEventDestroy(e);
+  for (auto e : g->rev) if (e) cudaEventDestroy(e);
   if (g->stream) cudaStreamDestroy(g->stream);
   for (auto s : g->up) if (s) cudaStreamDestroy(s);
   for (auto s : g->bs) if (s) cudaStreamDestroy(s);
@@ -1270,6 +1302,20 @@ int lmatch_round_log(const lmatch_graph* g, int64_t* out, int64_t cap, int64_t* 
   if (nrounds) *nrounds = r;
   if (out)
     for (int64_t i = 0; i < std::min<int64_t>(3 * r, 3 * cap); ++i) out[i] = g->round_log[(size_t)i];
+  return LMATCH_OK;
+}
+
+int lmatch_round_ms(const lmatch_graph* g, double* ms, int64_t cap, int64_t* nrounds,
+                    int64_t* tail_from) {
+  if (!g) { set_err("NULL handle"); return LMATCH_ESTATE; }
+  const int64_t r = g->n_rev > 1 ? g->n_rev - 1 : 0;
+  if (nrounds) *nrounds = r;
+  if (tail_from) *tail_from = g->tail_rounds_from;
+  for (int64_t i = 0; ms && i < std::min(r, cap); ++i) {
+    float x = 0.f;
+    CK(cudaEventElapsedTime(&x, g->rev[(size_t)i], g->rev[(size_t)i + 1]));
+    ms[i] = x;
+  }
   return LMATCH_OK;
 }
 
@@ -1360,13 +1406,13 @@ static int seq_body(lmatch_graph* g, cudaStream_t st, int cur, const int64_t* nF
     if (refill) CK(cudaMemsetAsync(g->rescan_cnt, 0, 8, st));
     lm::k_cache_redirect<lm::kCacheK><<<grid_for(nF, 256, 65536), 256, 0, st>>>(
         Fb, cF, g->offs, g->cache, g->bits, g->u_first, g->M0, g->v0, g->counters + lm::kCntCache,
-        refill ? g->rescan : nullptr, refill ? g->rescan_cnt : nullptr);
+        refill ? g->rescan : nullptr, refill ? g->rescan_cnt : nullptr, g->res ? g->roff : nullptr, g->M2);
     CKL();
     ++*launches;
     if (refill) {
       lm::k_host_rescan<lm::kCacheK><<<(unsigned)(8 * g->num_sms), 256, 0, st>>>(
           Fb, g->rescan, g->rescan_cnt, g->offs, g->view(), g->bits, g->cache, g->u_first, g->M0,
-          g->v0);
+          g->v0, g->res, g->cap_res, g->res_used, g->roff);
       CKL();
       ++*launches;
     }
@@ -1864,6 +1910,8 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
   int64_t launches = 0, sweep_launches = 0, bytes_streamed = 0;
 
   if (tm) CK(cudaEventRecord(g->ev[0], st));
+  g->n_rev = 0;
+  g->tail_rounds_from = -1;
   if (use_graph) {
     if (!g->gexec) TRY(build_graph_persistent(g));
     CK(cudaGraphLaunch(g->gexec, st));
@@ -1872,6 +1920,20 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
     if (g->ntiles > 0 && n > 0) TRY(launch_persistent(g, st, &launches));
   } else {
     TRY(seq_prefix(g, st, 0, 0, &launches, &sweep_launches, &bytes_streamed));
+    // (timing=1) an event at the start of every host-driven round and at the end of the loop:
+    // per-round device times for lmatch_round_ms
+    size_t nre = 0;
+    auto round_mark = [&]() -> int {
+      if (!tm) return LMATCH_OK;
+      if (nre == g->rev.size()) {
+        cudaEvent_t e;
+        CK(cudaEventCreate(&e));
+        g->rev.push_back(e);
+      }
+      CK(cudaEventRecord(g->rev[nre++], st));
+      return LMATCH_OK;
+    };
+    g->tail_rounds_from = -1;
     for (;;) {
       CK(cudaMemcpyAsync(g->h_rstate, g->rstate, sizeof(lm::RoundState), cudaMemcpyDeviceToHost, st));
       CK(cudaMemcpyAsync(g->h_counters, g->counters, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
@@ -1881,12 +1943,16 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
       int64_t nFb[lm::kBins], nF = 0;
       for (int b = 0; b < lm::kBins; ++b) { nFb[b] = (int64_t)g->h_counters[lm::cnt_F(cur, b)]; nF += nFb[b]; }
       const int64_t nS = (int64_t)g->h_counters[lm::cnt_S(cur)];
+      TRY(round_mark());
       if (mode == 0 && nF <= kPersistentBelow) {  // the tail: every remaining round on the device
+        g->tail_rounds_from = (int64_t)nre - 1;
         TRY(launch_persistent(g, st, &launches));
         break;
       }
       TRY(seq_body(g, st, cur, nFb, nS, &launches));
     }
+    TRY(round_mark());
+    g->n_rev = (int64_t)nre;
   }
   // ---- hybrid: a frontier left after kHandoffRounds phases goes to Suitor on the residual graph
   int64_t tail_passes = 0;
@@ -1977,6 +2043,7 @@ int lmatch_run_device(lmatch_graph* g, int32_t* d_mate, void* stream, lmatch_sta
     stats->tail_passes = tail_passes;
     if (g->kcache) stats->cache_rows = (int64_t)g->h_counters[lm::kCntCache];
     if (g->use_cache()) {
+      stats->residual_rows = (int64_t)g->h_counters[lm::kCntCache + 2];
       stats->cache_rows = (int64_t)g->h_counters[lm::kCntCache];
       stats->host_entries_read = (int64_t)g->h_counters[lm::kCntCache + 1];
       stats->cache_bytes = g->cap_cache * 8;
@@ -2305,12 +2372,12 @@ static int part_point_impl(lmatch_graph* g, cudaStream_t st, int64_t* claim_coun
     if (refill) CK(cudaMemsetAsync(g->rescan_cnt, 0, 8, st));
     lm::k_cache_redirect<lm::kCacheK><<<grid_for(nF, 256, 65536), 256, 0, st>>>(
         Fb, cF, g->offs, g->cache, g->bits, g->u_first, g->M0, g->v0, g->counters + lm::kCntCache,
-        refill ? g->rescan : nullptr, refill ? g->rescan_cnt : nullptr);
+        refill ? g->rescan : nullptr, refill ? g->rescan_cnt : nullptr, g->res ? g->roff : nullptr, g->M2);
     CKL();
     if (refill) {
       lm::k_host_rescan<lm::kCacheK><<<(unsigned)(8 * g->num_sms), 256, 0, st>>>(
           Fb, g->rescan, g->rescan_cnt, g->offs, g->view(), g->bits, g->cache, g->u_first, g->M0,
-          g->v0);
+          g->v0, g->res, g->cap_res, g->res_used, g->roff);
       CKL();
     }
   }

@@ -270,3 +270,34 @@ def test_key_cache_identity(lm, maker, round_loop):
         assert out[True]["cache_rows"] > 0
         assert out[True]["entries_swept"] <= out[False]["entries_swept"]
     assert out[False]["cache_rows"] == 0
+
+
+@pytest.mark.parametrize("maker,frac", [
+    (lambda: graphgen.rmat(16, 16, seed=5), 0.2),
+    (lambda: graphgen.er(1 << 15, 24.0, seed=2, weights="paper"), 0.1),
+    (lambda: graphgen.from_edges(4000, [(0, v, float(np.float32(1.0 / (1 + v % 97)))) for v in range(1, 4000)]
+                                 + [(v, v + 1, 0.5) for v in range(1, 3999)]), 0.0),
+])
+def test_out_of_core_residual_rows(lm, maker, frac):
+    """NEXT-1 residual rows (opts.residual_mb): host rows that are rescanned are also copied into
+    HBM, and later rounds and runs scan that copy.  Bit-identical across repeated runs (the copies
+    persist) and a reload (they are dropped), fewer host entries read once rows are resident."""
+    g = maker()
+    ref = oracle.greedy(g)
+    _, ph, _ = oracle.ld_frontier(g)
+    chunk = 1024
+    budget = int(8 * g.m * frac) + 2 * 8 * chunk
+    with lm.Matcher(g, hbm_budget_bytes=budget, stream_chunk=chunk, residual_mb=4) as M:
+        stats = []
+        for _ in range(3):
+            mate, st = M.run()
+            np.testing.assert_array_equal(mate, ref.mate)
+            assert st["rounds"] == ph
+            assert math.isclose(st["weight"], ref.weight, rel_tol=WTOL)
+            stats.append(st)
+        M.reload(g.offsets, g.col, g.w)
+        mate, st = M.run()
+        np.testing.assert_array_equal(mate, ref.mate)
+    if stats[0]["host_entries_read"] > 0:
+        assert stats[2]["residual_rows"] > 0
+        assert stats[2]["host_entries_read"] < stats[0]["host_entries_read"]
