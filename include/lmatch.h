@@ -177,7 +177,14 @@ typedef struct lmatch_opts {
                                  while space lasts, and later rounds -- and later runs on the same
                                  graph -- scan the HBM copy instead (no extra PCIe traffic).
                                  lmatch_stats.residual_rows counts the rows scanned from it */
-  int32_t reserved[4];
+  int32_t frontier;           /* A6 next-frontier construction in the persistent-kernel rounds
+                                 (round_loop 0, 2, 3): 0 = default, pull (compaction of the live
+                                 list) switching to push once the live list is 8x the frontier
+                                 (the vertices newly matched in a round push their row neighbours
+                                 that pointed at them: O(m) over the run instead of O(|L| x
+                                 rounds) -- many-round graphs); 1 = pull only.  Not with prune or
+                                 algorithm 2.  Same result and pointing phases */
+  int32_t reserved[3];
 } lmatch_opts;
 
 /* Filled by lmatch_run / lmatch_run_device when non-NULL. */
@@ -274,6 +281,9 @@ LMATCH_API int lmatch_round_log(const lmatch_graph* g, int64_t* out, int64_t cap
  * is that whole tail and *tail_from = its index (else -1).  0 rounds without timing. */
 LMATCH_API int lmatch_round_ms(const lmatch_graph* g, double* ms, int64_t cap, int64_t* nrounds,
                                int64_t* tail_from);
+
+/* Rounds of the last lmatch_run* whose next frontier was pushed (opts.frontier; 0 = all pulled). */
+LMATCH_API int lmatch_push_rounds(const lmatch_graph* g, int64_t* push_rounds);
 
 /* ---------------------------------------------------------------------------------------------
  * Partitioned mode (multi-GPU, one process or thread per GPU).

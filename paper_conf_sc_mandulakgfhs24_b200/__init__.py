@@ -48,7 +48,7 @@ class Opts(ctypes.Structure):
         ("host_cache", ctypes.c_int32), ("batches", ctypes.c_int32),
         ("algorithm", ctypes.c_int32), ("sort_chunk_log2", ctypes.c_int32),
         ("key_cache", ctypes.c_int32), ("residual_mb", ctypes.c_int32),
-        ("reserved", ctypes.c_int32 * 4),
+        ("frontier", ctypes.c_int32), ("reserved", ctypes.c_int32 * 3),
     ]
 
 
@@ -88,6 +88,7 @@ _sig = {
                      ctypes.POINTER(_I64)], ctypes.c_int),
     "lmatch_round_log": ([_P, _P, _I64, ctypes.POINTER(_I64)], ctypes.c_int),
     "lmatch_round_ms": ([_P, _P, _I64, ctypes.POINTER(_I64), ctypes.POINTER(_I64)], ctypes.c_int),
+    "lmatch_push_rounds": ([_P, ctypes.POINTER(_I64)], ctypes.c_int),
     "lmatch_destroy": ([_P], None),
     "lmatch_strerror": ([ctypes.c_int], ctypes.c_char_p),
     "lmatch_last_error": ([], ctypes.c_char_p),
@@ -246,6 +247,13 @@ def lmatch_round_ms(h: int):
     return out[: nr.value], int(tf.value)
 
 
+def lmatch_push_rounds(h: int) -> int:
+    """Rounds of the last run whose next frontier was pushed (A6 push frontier)."""
+    r = _I64()
+    _check(_lib.lmatch_push_rounds(h, ctypes.byref(r)), "lmatch_push_rounds")
+    return int(r.value)
+
+
 def lmatch_destroy(h: int | None) -> None:
     _lib.lmatch_destroy(h)
 
@@ -260,7 +268,7 @@ class Matcher:
                  max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
                  round_loop: int = 0, prune: bool = False, host_cache: bool = True,
                  batches: int = 0, algorithm: str = "ld", sort_chunk_log2: int = 0,
-                 key_cache: bool = False, residual_mb: int = 0):
+                 key_cache: bool = False, residual_mb: int = 0, frontier: str = "auto"):
         self.h = None
         if handle is not None:
             self.h = handle
@@ -272,7 +280,7 @@ class Matcher:
                                                      max_rounds, hbm_budget_bytes, stream_chunk,
                                                      round_loop, prune, host_cache, batches,
                                                      algorithm, sort_chunk_log2, key_cache,
-                                                     residual_mb))
+                                                     residual_mb, frontier))
         self.info = lmatch_info(self.h)
 
     @classmethod
@@ -292,6 +300,9 @@ class Matcher:
 
     def weight(self, mate) -> float:
         return lmatch_weight(self.h, mate)
+
+    def push_rounds(self) -> int:
+        return lmatch_push_rounds(self.h)
 
     def reload(self, offsets, col, w) -> None:
         lmatch_reload(self.h, offsets, col, w)
@@ -318,7 +329,7 @@ def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int =
               max_rounds: int = 0, hbm_budget_bytes: int = 0, stream_chunk: int = 0,
               round_loop: int = 0, prune: bool = False, host_cache: bool = True,
               batches: int = 0, algorithm: str = "ld", sort_chunk_log2: int = 0,
-              key_cache: bool = False, residual_mb: int = 0) -> Opts:
+              key_cache: bool = False, residual_mb: int = 0, frontier: str = "auto") -> Opts:
     """round_loop (include/lmatch.h): 0 = hybrid (work-sized launches, then one persistent kernel
     for the tail; default), 1 = host-driven launches only, 2 = persistent kernel after round 1,
     3 = CUDA graph {round 1, persistent kernel}."""
@@ -331,6 +342,7 @@ def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int =
     o.sort_chunk_log2 = int(sort_chunk_log2)
     o.key_cache = 1 if key_cache else 0
     o.residual_mb = int(residual_mb)
+    o.frontier = {"auto": 0, "pull": 1}[frontier]
     o.hbm_budget_bytes = int(hbm_budget_bytes)
     o.stream_chunk = int(stream_chunk)
     o.validate_level = int(validate_level)

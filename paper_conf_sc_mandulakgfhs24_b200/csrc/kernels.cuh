@@ -1086,6 +1086,8 @@ __global__ void k_low32(const int64_t* __restrict__ noffs, int64_t cnt, uint32_t
 constexpr int kNumCounters = 24;
 constexpr int kCntSwept = 16;
 constexpr int kCntCache = 17;  // [17] rows served by the out-of-core cache, [18] host entries read
+constexpr int kCntN = 20;      // A6 push frontier: |N_r|, the vertices newly matched this round
+constexpr int kCntPushRounds = 21;  // rounds whose next frontier the push step built
 __host__ __device__ constexpr int cnt_S(int set) { return 8 * set; }
 __host__ __device__ constexpr int cnt_F(int set, int b) { return 8 * set + 1 + b; }
 constexpr uint32_t kNoPtr = 0xffffffffu;
@@ -1117,7 +1119,7 @@ struct RoundState {
   long long log_cap;
   unsigned long long swept_prev;
   uint32_t tag;          // per-run tag of the A7 live counts (1..65535, advanced by k_round_init)
-  uint32_t pad;
+  uint32_t push;         // A6 push frontier active (persistent kernel; set by end_round_body)
 };
 __device__ __forceinline__ uint32_t round_tag(const RoundState* st) {
   return *reinterpret_cast<const volatile uint32_t*>(&st->tag);
@@ -1131,6 +1133,7 @@ struct RoundArgs {
   uint32_t* live;           // A7 pruning: per-vertex live counts (nullptr = pruning off)
   const uint64_t* kc;       // resident key cache [n][kKC] (nullptr = off)
   uint64_t* best;           // per-vertex pointers (the compaction writes the cache-decided ones)
+  uint32_t* N;              // A6 push frontier: vertices newly matched this round (nullptr = off)
 };
 
 // A2 pointer phase on the frontier (rounds >= 2): G lanes per vertex (degree-binned).
@@ -2218,10 +2221,16 @@ __global__ void k_round_init(RoundState* st, long long max_rounds, long long log
   st->log_cap = log_cap;
   st->swept_prev = 0;
   st->tag = st->tag >= 0xffffu ? 1u : st->tag + 1u;
+  st->push = 0;
 }
 // After a compaction: the output set becomes current; decide whether another round runs.
 // `graph_handle` != 0: running inside a CUDA graph -> set the WHILE node's condition.
-__device__ __forceinline__ int end_round_body(const RoundArgs* __restrict__ ra, long long first_log_rows) {
+#ifndef LM_PUSH_RATIO
+#define LM_PUSH_RATIO 8
+#endif
+constexpr unsigned long long kPushRatio = LM_PUSH_RATIO;
+__device__ __forceinline__ int end_round_body(const RoundArgs* __restrict__ ra, long long first_log_rows,
+                                              bool push_ok = false) {
   RoundState* st = ra->st;
   const int cur = st->cur ^ 1;
   st->cur = cur;
@@ -2230,6 +2239,11 @@ __device__ __forceinline__ int end_round_body(const RoundArgs* __restrict__ ra, 
   for (int b = 0; b < kBins; ++b) nF += ra->cnt[cnt_F(cur, b)];
   const unsigned long long nS = ra->cnt[cnt_S(cur)];
   const int cont = nF > 0 && st->rounds < st->max_rounds;
+  // A6: once the live list is much longer than the frontier (many-round graphs), the next
+  // frontier is pushed from the newly matched vertices instead of pulled from the live list
+  // (only the persistent kernel runs push rounds; it passes push_ok)
+  if (push_ok && ra->N && !st->push && nS + nF > kPushRatio * nF) st->push = 1;
+  ra->cnt[kCntN] = 0ull;
   // zero the counters of the set the next compaction writes
 #pragma unroll
   for (int q = 0; q < 1 + kBins; ++q) ra->cnt[cnt_S(cur ^ 1) + q] = 0ull;
@@ -2254,6 +2268,74 @@ __global__ void k_end_round(const RoundArgs* __restrict__ ra, cudaGraphCondition
   if (threadIdx.x != 0 || blockIdx.x != 0) return;
   const int cont = end_round_body(ra, first_log_rows);
   if (in_graph) cudaGraphSetConditional(handle, (unsigned)cont);
+}
+
+// ---- A6 push-style frontier (SURVEY 8(a) A6 "push alternative"; not in the paper, whose Alg. 3
+// rescans every unmatched vertex).  The pull compaction reads the whole live list every
+// round, O(|L| x rounds): quadratic on many-round graphs (a weight gradient along paths).  In a
+// push round the match records the vertices it newly matched (N_r, deduplicated by the atomicOr's
+// old value), and the next frontier is built from their rows: u joins F_{r+1} iff u is unmatched
+// and its pointer is a vertex of N_r -- exactly the pull rule, since a live u's target was
+// unmatched when the round began.  Each vertex is matched once, so the whole run pushes O(m)
+// entries.  A frontier vertex is claimed by a CAS of its pointer to 0 (its pointer is recomputed
+// next round anyway), so repeated (u,v) entries cannot list it twice.
+__device__ __forceinline__ void match_push_body(const Bins& F, const unsigned long long* cntF,
+                                                const uint64_t* __restrict__ best, uint32_t* bits,
+                                                uint32_t* N, unsigned long long* cntN, int64_t tid,
+                                                int64_t stride) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll 1
+  for (int bb = 0; bb < kBins; ++bb) {
+    const int64_t c = (int64_t)cntF[bb];
+    for (int64_t i0 = tid - lane; i0 < c; i0 += stride) {  // warp-uniform trip count
+      const int64_t i = i0 + lane;
+      const uint64_t p = i < c ? F.list[bb][i].x : ((uint64_t)kNoPtr << 32);
+      const uint32_t u = (uint32_t)p, v = (uint32_t)(p >> 32);
+      bool nu = false, nv = false;
+      if (v != kNoPtr) {
+        const uint64_t kv = best[v];
+        if (kv != 0 && (uint32_t)kv == u) {
+          const uint32_t mu = 1u << (u & 31), mv = 1u << (v & 31);
+          nu = !(atomicOr(&bits[u >> 5], mu) & mu);
+          nv = !(atomicOr(&bits[v >> 5], mv) & mv);
+        }
+      }
+      warp_append(nu, (int32_t)u, reinterpret_cast<int32_t*>(N), cntN);
+      warp_append(nv, (int32_t)v, reinterpret_cast<int32_t*>(N), cntN);
+    }
+  }
+}
+// F_{r+1} from the rows of N_r (a lane per newly matched vertex; its row is short on the graphs
+// that reach push mode); appends into the degree bins of the output set
+__device__ __forceinline__ void push_body(const uint32_t* __restrict__ N, int64_t nN,
+                                          const int64_t* __restrict__ offs, const AdjView adj,
+                                          const uint32_t* __restrict__ bits, uint64_t* best,
+                                          const Bins& Fout, unsigned long long* cntFout,
+                                          unsigned long long* swept, int64_t vbase, int64_t tid,
+                                          int64_t stride) {
+  unsigned long long degsum = 0;
+  for (int64_t i = tid; i < nN; i += stride) {
+    const uint32_t v = N[i];
+    const int64_t lv = (int64_t)v - vbase;
+    for (int64_t j = offs[lv], e = offs[lv + 1]; j < e; ++j) {
+      const uint64_t k = adj.at(j);
+      const uint32_t u = (uint32_t)k;
+      if (k == 0 || bit_test(bits, u)) continue;
+      const int64_t lu = (int64_t)u - vbase;
+      const uint64_t bu = *reinterpret_cast<volatile const uint64_t*>(best + lu);
+      if (bu == 0 || (uint32_t)bu != v) continue;
+      if (atomicCAS(reinterpret_cast<unsigned long long*>(best + lu), (unsigned long long)bu, 0ull) != bu)
+        continue;
+      const int64_t os = offs[lu], d = offs[lu + 1] - os;
+      const int b = bin_of(d);
+      const unsigned long long pos = atomicAdd(&cntFout[b], 1ull);
+      Fout.list[b][pos] = make_ulonglong2(make_pair(u, v),
+                                          (uint64_t)os | ((uint64_t)(d < (int64_t)kBigDeg ? d : (int64_t)kBigDeg) << 40));
+      degsum += (unsigned long long)d;
+    }
+  }
+  for (int o = 16; o; o >>= 1) degsum += __shfl_xor_sync(0xffffffffu, degsum, o);
+  if ((threadIdx.x & 31) == 0 && degsum) atomicAdd(swept, degsum);
 }
 
 // All rounds >= 2 in ONE cooperative launch (grid = co-resident blocks): pointer phase (every
@@ -2284,14 +2366,25 @@ __global__ void __launch_bounds__(256)
                                  gridDim.x);
     }
     grid.sync();
-    match_bins_body(ra->F[cur], ra->cnt + cnt_F(cur, 0), best, bits, gtid, gthreads);
+    const bool push = *reinterpret_cast<volatile uint32_t*>(&ra->st->push) != 0u;
+    if (push)
+      match_push_body(ra->F[cur], ra->cnt + cnt_F(cur, 0), best, bits, ra->N, ra->cnt + kCntN, gtid, gthreads);
+    else
+      match_bins_body(ra->F[cur], ra->cnt + cnt_F(cur, 0), best, bits, gtid, gthreads);
     grid.sync();
-    {
+    if (push) {
+      push_body(ra->N, (int64_t)*reinterpret_cast<volatile unsigned long long*>(ra->cnt + kCntN), offs, adj,
+                bits, best, ra->F[cur ^ 1], ra->cnt + cnt_F(cur ^ 1, 0), ra->cnt + kCntSwept, vbase, gtid,
+                gthreads);
+    } else {
       const CompactIO io = compact_io(*ra, cur);
       compact_body<false, K, KC>(io, n, best, bits, offs, vbase, blockIdx.x, gridDim.x);
     }
     grid.sync();
-    if (gtid == 0) end_round_body(ra, 0);
+    if (gtid == 0) {
+      if (push) ++ra->cnt[kCntPushRounds];
+      end_round_body(ra, 0, !PRUNE);
+    }
     grid.sync();
   }
 }

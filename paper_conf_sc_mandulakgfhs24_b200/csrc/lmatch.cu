@@ -248,6 +248,10 @@ struct lmatch_graph {
   // resident key cache (opts.key_cache): the 4 largest keys of every row, filled by the sweep
   int key_cache = 0;
   int kc_attr = 0;
+  // A6 push frontier (persistent-kernel rounds; opts.frontier): newly matched vertices [n_nz + 1]
+  int push_ok = 1;
+  uint32_t* pushN = nullptr;
+  int64_t cap_pushN = -1;
   uint64_t* kcache = nullptr;        // the active cache: kc_buf, or nullptr = off for this graph
   uint64_t* kc_buf = nullptr;        // [n + 1][kKC]
   uint64_t* xpart = nullptr;         // [ntiles][2][kKC] partial lists of tile-crossing rows
@@ -364,6 +368,7 @@ struct lmatch_graph {
     a.live = prune ? live : nullptr;
     a.kc = kcache;
     a.best = best;
+    a.N = (push_ok && !prune && algorithm != 2) ? pushN : nullptr;
     return a;
   }
 };
@@ -833,6 +838,7 @@ int alloc_bins(lmatch_graph* g, cudaStream_t st) {
   g->device_bytes -= 16;
   // A7 pruning moves rows to LOWER bins (live degrees only shrink): bin b must then hold every
   // row whose full degree is in bin b or above
+  if (g->push_ok) TRY(ensure(g, &g->pushN, &g->cap_pushN, g->n_nz + 1));
   // the decided list (key cache) can hold any non-empty row
   h[lm::kDecided] = 0;
   for (int b = 0; b < lm::kDegBins; ++b) h[lm::kDecided] += h[b];
@@ -1051,6 +1057,7 @@ int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** 
     g->algorithm = opts->algorithm;
     g->key_cache = opts->key_cache > 0;
     g->residual_mb = opts->residual_mb;
+    g->push_ok = opts->frontier != 1;
     if (opts->sort_chunk_log2 != 0) {
       if (opts->sort_chunk_log2 < 4 || opts->sort_chunk_log2 > 30) {
         set_err("sort_chunk_log2 = %d outside 4..30", opts->sort_chunk_log2);
@@ -1225,7 +1232,7 @@ void lmatch_destroy(lmatch_graph* g) {
                   g->cache, g->chunk_rows, g->cache_big, g->rescan, g->rescan_cnt, g->live, g->win, g->suitor, g->wl[0],
                   g->wl[1], g->wl_big, g->wl_cnt, g->sc_cur, g->sc_ptr, g->sc_L[0], g->sc_L[1], g->shadow, g->d_dseg, g->d_dcnt,
                   g->d_dbits, g->d_dnf, g->d_dflag, g->d_dresw, g->d_dresc, g->d_berr,
-                  g->kc_buf, g->xpart, g->xrows, g->nx, g->res, g->res_used, g->roff};
+                  g->kc_buf, g->xpart, g->xrows, g->nx, g->res, g->res_used, g->roff, g->pushN};
   for (void* p : pdev) if (p) cudaFree(p);
   if (g->h_claim_cnt) cudaFreeHost(g->h_claim_cnt);
   if (g->h_res) cudaFreeHost(g->h_res);
@@ -1302,6 +1309,12 @@ int lmatch_round_log(const lmatch_graph* g, int64_t* out, int64_t cap, int64_t* 
   if (nrounds) *nrounds = r;
   if (out)
     for (int64_t i = 0; i < std::min<int64_t>(3 * r, 3 * cap); ++i) out[i] = g->round_log[(size_t)i];
+  return LMATCH_OK;
+}
+
+int lmatch_push_rounds(const lmatch_graph* g, int64_t* push_rounds) {
+  if (!g || !push_rounds) { set_err("NULL argument"); return LMATCH_ESTATE; }
+  *push_rounds = g->h_counters ? (int64_t)g->h_counters[lm::kCntPushRounds] : 0;
   return LMATCH_OK;
 }
 

@@ -301,3 +301,34 @@ def test_out_of_core_residual_rows(lm, maker, frac):
     if stats[0]["host_entries_read"] > 0:
         assert stats[2]["residual_rows"] > 0
         assert stats[2]["host_entries_read"] < stats[0]["host_entries_read"]
+
+
+@pytest.mark.parametrize("round_loop", [0, 2, 3])
+@pytest.mark.parametrize("maker", [
+    lambda: graphgen.mesh(96, seed=1, weights="gradient"),           # ~2*side phases
+    lambda: graphgen.mesh(120, keep=0.6, seed=2, weights="gradient"),
+    lambda: graphgen.from_edges(3001, [(i, i + 1, float(i + 1)) for i in range(3000)]),  # 1500 phases
+    lambda: graphgen.rmat(15, 16, seed=8),
+    lambda: graphgen.from_edges(600, [(i, i + 1, float(i + 1)) for i in range(599)] + [(i, i + 1, float(i + 1)) for i in range(599)]),
+])
+def test_push_frontier(lm, maker, round_loop):
+    """A6 push frontier (opts.frontier): in the persistent-kernel rounds the next frontier is built
+    from the rows of the newly matched vertices once the live list is much longer than the
+    frontier.  Same mate[] and the same pointing phases as Alg. 1 and as pull-only; many-round
+    graphs actually switch to push.  (The last graph lists every edge twice: a pushed vertex is
+    claimed once.)"""
+    g = maker()
+    ref = oracle.greedy(g)
+    _, ph, _ = oracle.ld_frontier(g)
+    res = {}
+    for fr in ("auto", "pull"):
+        with lm.Matcher(g, round_loop=round_loop, frontier=fr) as M:
+            for _ in range(2):
+                mate, st = M.run()
+                np.testing.assert_array_equal(mate, ref.mate)
+                assert st["rounds"] == ph
+                assert math.isclose(st["weight"], ref.weight, rel_tol=WTOL)
+            res[fr] = M.push_rounds()
+    assert res["pull"] == 0
+    if ph > 100:
+        assert res["auto"] > 0

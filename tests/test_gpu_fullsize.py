@@ -113,3 +113,21 @@ def test_rmat_s29_resident(lm):
     with lm.Matcher(g) as M:
         mate, st = M.run()
     _certify(g, mate, st)
+
+
+def test_gradient_mesh_8192_ld_push(lm):
+    """configs[2]'s many-round variant at full size on the LD path (SURVEY 8(d) C3 gradient:
+    ~2 x 8192 pointing phases): the A6 push frontier keeps every round O(new matches) instead of
+    O(live list), so the 16K-round run finishes in about a second; certificate + oracle weight."""
+    import torch
+    import graphgen.gpu as gg
+    dg = gg.mesh(8192, seed=1, weights="gradient", device=torch.device("cuda"))
+    g = graphgen.Graph(dg.offsets.cpu().numpy(), dg.col.cpu().numpy(), dg.w.cpu().numpy())
+    M = lm.Matcher.from_device(dg.offsets, dg.col, dg.w, dg.n, dg.m, stream=torch.cuda.current_stream())
+    del dg
+    torch.cuda.empty_cache()
+    mate, st = M.run()
+    pushed = M.push_rounds()
+    M.close()
+    assert st["rounds"] > 8000 and pushed > 8000
+    _certify(g, mate, st)
