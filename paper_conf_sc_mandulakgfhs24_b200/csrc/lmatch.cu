@@ -234,6 +234,8 @@ struct lmatch_graph {
   std::vector<void*> ipc_opened;     // peer allocations opened with cudaIpcOpenMemHandle
   unsigned long long* h_nf = nullptr;  // pinned [P]
   float part_sweep_ms = 0.f;  // (timing=1) last lmatch_part_begin's round-1 sweep
+  bool sweep_ms_pending = false;  // its events are recorded, the time not read yet
+  bool counts_on_host = false;    // peer-memory round: h_counters holds this set's bin sizes
   int validate_level = 1;
   int timing = 0;
   int64_t max_rounds = 0;
@@ -2223,24 +2225,26 @@ static int part_begin_impl(lmatch_graph* g, cudaStream_t st, int64_t* claim_coun
   CKL();
   lm::k_round_init<<<1, 1, 0, st>>>(g->rstate, g->max_rounds, kLogCap, 1);
   CKL();
-  CK(cudaMemsetAsync(g->ghost, 0xff, ((size_t)g->n_global + 1) * 4, st));
+  // one part: nothing is remote, so there are no ghosts and no claims
+  if (g->P > 1) CK(cudaMemsetAsync(g->ghost, 0xff, ((size_t)g->n_global + 1) * 4, st));
   CK(cudaMemsetAsync(g->claim_cnt, 0, (size_t)g->P * 8, st));
   int64_t l = 0, sl = 0, bs = 0;
   if (g->timing) CK(cudaEventRecord(g->ev[1], st));
   if (g->ntiles > 0 && g->n > 0) TRY(round1_sweep(g, st, &l, &sl, &bs));
   if (g->timing) CK(cudaEventRecord(g->ev[2], st));
   const lm::Claims Cl = part_claims_desc(g);
-  if (g->n > 0) {
+  if (g->n > 0 && g->P > 1) {
     lm::k_claims_all<<<grid_for(g->n, 256, 65536), 256, 0, st>>>(g->best, g->n, g->v0,
                                                                    g->v0 + g->n, Cl);
     CKL();
   }
   g->part_round = 1;
   g->round_log.clear();
+  g->sweep_ms_pending = g->timing != 0;  // read when the stream next synchronises
   const int rc = g->p2p ? LMATCH_OK : part_claims_out(g, st, claim_counts);
-  if (!rc && g->timing) {
-    CK(cudaStreamSynchronize(st));
+  if (!rc && g->timing && !g->p2p) {
     CK(cudaEventElapsedTime(&g->part_sweep_ms, g->ev[1], g->ev[2]));
+    g->sweep_ms_pending = false;
   }
   return rc;
 }
@@ -2295,6 +2299,12 @@ int lmatch_part_apply(lmatch_graph* g, const uint64_t* d_recv, int64_t nrecv, vo
 
 int lmatch_part_info(const lmatch_graph* g, int64_t* rounds, double* sweep_ms) {
   if (!g || !g->ghost) { set_err("not a partition handle"); return LMATCH_ESTATE; }
+  if (g->sweep_ms_pending) {
+    lmatch_graph* gm = const_cast<lmatch_graph*>(g);
+    CK(cudaEventSynchronize(g->ev[2]));
+    CK(cudaEventElapsedTime(&gm->part_sweep_ms, g->ev[1], g->ev[2]));
+    gm->sweep_ms_pending = false;
+  }
   if (rounds) *rounds = g->part_round;
   if (sweep_ms) *sweep_ms = g->part_sweep_ms;
   return LMATCH_OK;
@@ -2318,12 +2328,14 @@ static int part_compact_launch(lmatch_graph* g, cudaStream_t st) {
   // makes that set current (and zeroes the counters the next compaction writes)
   if (g->part_round == 1) {
     if (n > 0) {
-      const unsigned grid = grid_for((n + 31) / 32, 8 * kCompactK, 65536);
-      const lm::CompactIO io = lm::compact_io(g->rargs(), 1);
+      // items are the non-empty rows (nzr): empty rows never hold a pointer
+      const unsigned grid = grid_for((g->n_nz + 31) / 32, 8 * kCompactK, 65536);
+      lm::CompactIO io = lm::compact_io(g->rargs(), 1);
+      io.nzr = g->nzr;
       if (g->kcache)
-        lm::k_compact<true, kCompactK, true><<<grid, 256, 0, st>>>(io, n, g->best, g->bits, g->offs, g->v0);
+        lm::k_compact<true, kCompactK, true><<<grid, 256, 0, st>>>(io, g->n_nz, g->best, g->bits, g->offs, g->v0);
       else
-        lm::k_compact<true, kCompactK, false><<<grid, 256, 0, st>>>(io, n, g->best, g->bits, g->offs, g->v0);
+        lm::k_compact<true, kCompactK, false><<<grid, 256, 0, st>>>(io, g->n_nz, g->best, g->bits, g->offs, g->v0);
       CKL();
     }
     g->part_cur = 0;
@@ -2368,13 +2380,14 @@ static int part_point_impl(lmatch_graph* g, cudaStream_t st, int64_t* claim_coun
   const int cur = g->part_cur;
   int64_t nFb[lm::kBins], nF = 0;
   for (int b = 0; b < lm::kBins; ++b) { nFb[b] = (int64_t)g->h_counters[lm::cnt_F(cur, b)]; nF += nFb[b]; }
-  if (g->p2p) {
+  if (g->p2p && !g->counts_on_host) {
     // peer-memory rounds do not read the bin sizes back: every kernel below loops over the
     // device-resident count, so launch each bin with a full resident wave (an empty bin exits)
     const int64_t wave = 8ll * g->num_sms;
     for (int b = 0; b < lm::kBins; ++b) nFb[b] = wave * 256;
     nF = wave * 256;
   }
+  g->counts_on_host = false;
   const lm::AdjView av = g->view();
   const lm::Bins& Fb = g->F[cur];
   const unsigned long long* cF = g->counters + lm::cnt_F(cur, 0);
@@ -2415,7 +2428,7 @@ static int part_point_impl(lmatch_graph* g, cudaStream_t st, int64_t* claim_coun
   if (nFb[2]) { lm::k_point_bin<LM_B2_G, LM_B2_U><<<grid_for(nFb[2] * LM_B2_G, 256, 65536), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, av, g->bits, g->best, g->v0); CKL(); }
   if (nFb[3]) { lm::k_point_bin_cta<256, LM_CTA_U><<<(unsigned)std::min<int64_t>(nFb[3], g->p2p ? 8ll * g->num_sms : 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); }
   if (!g->p2p) CK(cudaMemsetAsync(g->claim_cnt, 0, (size_t)g->P * 8, st));
-  if (nF > 0) {
+  if (nF > 0 && g->P > 1) {
     const lm::Claims Cl = part_claims_desc(g);
     lm::k_claims_bins<<<grid_for(nF, 256, 65536), 256, 0, st>>>(Fb, cF, g->v0, g->v0 + g->n, Cl);
     CKL();
@@ -2625,8 +2638,10 @@ int lmatch_p2p_match(lmatch_graph* g, void* stream) {
   unsigned long long* icnt = reinterpret_cast<unsigned long long*>(g->win + (size_t)P * g->win_cap);
   const int64_t grid = std::max<int64_t>(1, std::min<int64_t>((g->win_cap + 255) / 256, 4 * g->num_sms));
   // received claims (v owned, u remote): ghost pointers, then the owned mutual checks
-  lm::k_apply_inbox<<<(unsigned)grid, 256, 0, st>>>(g->win, g->win_cap, icnt, P, g->ghost);
-  CKL();
+  if (P > 1) {
+    lm::k_apply_inbox<<<(unsigned)grid, 256, 0, st>>>(g->win, g->win_cap, icnt, P, g->ghost);
+    CKL();
+  }
   if (g->part_round == 1) {
     if (g->n > 0) {
       lm::k_match_part_all<<<grid_for(((g->n + 31) / 32) * 32, 256, 65536), 256, 0, st>>>(
@@ -2640,6 +2655,7 @@ int lmatch_p2p_match(lmatch_graph* g, void* stream) {
         g->ghost, g->bits);
     CKL();
   }
+  if (P == 1) return LMATCH_OK;  // one part: no inbox, no replicas to update
   lm::k_match_inbox<<<(unsigned)grid, 256, 0, st>>>(g->win, g->win_cap, icnt, P, g->best, g->v0,
                                                      g->bits);
   CKL();
@@ -3048,7 +3064,38 @@ int lmatch_run_dist_device(lmatch_graph* g, int32_t* d_mate_local, void* stream,
   TRY(phase("begin"));
   int64_t rounds = 1;
   bool compacted = false, capped = false;
-  for (;;) {
+  if (P == 1) {
+    // one rank: nothing to exchange, so the round loop is the single-GPU one -- the frontier
+    // size read after each compaction sizes the next pointer launches exactly, and the small
+    // tail runs in the persistent cooperative kernel (no host round trips)
+    for (;;) {
+      TRY(lmatch_p2p_match(g, st));
+      TRY(lmatch_p2p_compact(g, st, nullptr));
+      CK(cudaMemcpyAsync(g->h_counters, g->counters, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
+      CK(cudaStreamSynchronize(st));
+      int64_t nF = 0;
+      for (int b = 0; b < lm::kBins; ++b) nF += (int64_t)g->h_counters[lm::cnt_F(g->part_cur, b)];
+      if (nF == 0) break;
+      if (rounds >= g->max_rounds) { capped = true; break; }
+      ++rounds;
+      if (g->round_loop == 0 && nF <= kPersistentBelow) {
+        // k_end_round left the state of the next round in rstate (same cur as part_cur)
+        int64_t l = 0;
+        TRY(launch_persistent(g, st, &l));
+        CK(cudaMemcpyAsync(g->h_rstate, g->rstate, sizeof(lm::RoundState), cudaMemcpyDeviceToHost, st));
+        CK(cudaMemcpyAsync(g->h_counters, g->counters, lm::kNumCounters * 8, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        rounds = g->h_rstate->rounds;  // pointing phases begun, as counted by k_end_round
+        int64_t left = 0;
+        for (int b = 0; b < lm::kBins; ++b) left += (int64_t)g->h_counters[lm::cnt_F(g->h_rstate->cur, b)];
+        capped = left > 0;
+        break;
+      }
+      g->counts_on_host = true;
+      TRY(part_point_impl(g, st, nullptr));
+    }
+  }
+  for (; P > 1;) {
     TRY(barrier());  // claims are in the owners' inboxes; frontier sizes in every slot
     if (compacted) {
       int64_t total = 0;
@@ -3115,7 +3162,9 @@ int lmatch_run_dist_device(lmatch_graph* g, int32_t* d_mate_local, void* stream,
       CK(cudaEventSynchronize(g->ev[5]));
       CK(cudaEventElapsedTime(&a, g->ev[0], g->ev[5]));
       stats->ms_total = a;
-      stats->ms_sweep = g->part_sweep_ms;
+      double sw = 0;
+      TRY(lmatch_part_info(g, nullptr, &sw));
+      stats->ms_sweep = sw;
     }
   }
   if (capped) {

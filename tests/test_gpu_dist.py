@@ -275,3 +275,13 @@ def test_out_of_core_parts(D, P, kw):
         assert res.rounds == ph
     mate, st, _ = D.match_dist_threads(g.offsets, g.col, g.w, P, **kw)
     check(g, mate, st)
+
+
+def test_dist_single_rank_uses_the_device_round_loop(D):
+    """A one-rank lmatch_create_dist group exchanges nothing: it sizes the pointer launches from the
+    frontier it reads after each compaction and runs the small tail in the persistent kernel, as
+    the single-graph path does.  Same result and phases (incl. a many-round graph, whose tail
+    switches to the push frontier)."""
+    for g in (graphgen.rmat(15, 16, seed=4), graphgen.mesh(64, seed=1, weights="gradient")):
+        mate, st, _ = D.match_dist_threads(g.offsets, g.col, g.w, 1)
+        check(g, mate, st)
