@@ -723,6 +723,7 @@ def main():
                "note": "sweep = resident HBM tiles + host chunks over PCIe (2-slot ring); later "
                        "rounds read host rows zero-copy, except rows whose pointer the top-8 "
                        "host-row key cache decides (filled in round 1; NEXT-1)"}
+    mate_last = d_mate.cpu().numpy() if (g is not None and not a.no_cpu and world == 1) else None
     round_log = lm.lmatch_round_log(h)
     rounds_roofline = per_round_roofline(round_log, *lm.lmatch_round_ms(h), load_peaks()[0])
     lm.lmatch_destroy(h)
@@ -732,6 +733,19 @@ def main():
     cpu = None
     if rank == 0 and world == 1 and not a.no_cpu:
         cpu = cpu_baseline(a, cpu_sample_scale(a))
+        if g is not None and mate_last is not None:
+            # the O(m) certificate (oracle/, all host cores) on THIS line's graph and result: a
+            # verifier, not a baseline -- it checks the GPU's mate[] at full size and shows what
+            # the host needs for one pass over the same adjacency
+            import oracle
+            oracle.threads(0)
+            t0 = time.perf_counter()
+            code, _ = oracle.certificate(g, mate_last)
+            cert_s = time.perf_counter() - t0
+            cpu["certificate_on_this_graph"] = {
+                "ok": code == 0, "seconds": cert_s, "cores": os.cpu_count(),
+                "gteps_equivalent": m_u / cert_s / 1e9,
+                "kind": "verifier (C(M) holds iff mate[] is the unique LD matching), not a matcher"}
 
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": a.steps,

@@ -432,7 +432,8 @@ LMATCH_API int lmatch_dist_id_new(lmatch_dist_id* id);
  * n_global vertices, given as a HOST local CSR whose col_idx are GLOBAL ids (cut edges appear in
  * both owners' rows); part_bounds: HOST int64[world+1] as lmatch_partition returns (every
  * rank passes the same bounds; v_begin must be part_bounds[rank]).  Blocks until all `world`
- * ranks of `id` have joined (ENCCL after 60 s), then opens every peer's exchange window: plain
+ * ranks of `id` have joined (ENCCL after 60 s; environment LMATCH_DIST_TIMEOUT_S overrides the
+ * wait here and at the device barriers), then opens every peer's exchange window: plain
  * device pointers for ranks in the same process (peer access enabled across devices), CUDA IPC
  * for other processes.  opts: as for lmatch_create_ex (hbm_budget_bytes / batches stream this
  * rank's rows: the paper's per-device batches N_i), except validate_level 2 and

@@ -2769,7 +2769,16 @@ bool dist_trace() { return dist_trace_level() >= 1; }
     }                                                                                    \
   } while (0)
 constexpr uint32_t kShmMagic = 0x4c4d4431u;  // "LMD1"
-constexpr unsigned long long kDistTimeoutNs = 60ull * 1000000000ull;
+// how long a rank waits for its peers (rendezvous, barriers): LMATCH_DIST_TIMEOUT_S, default 60 s
+unsigned long long dist_timeout_ns() {
+  static const unsigned long long t = [] {
+    const char* e = getenv("LMATCH_DIST_TIMEOUT_S");
+    const long long v = e ? atoll(e) : 0;
+    return (unsigned long long)(v > 0 ? v : 60) * 1000000000ull;
+  }();
+  return t;
+}
+#define kDistTimeoutNs dist_timeout_ns()
 struct DistSlot {
   uint32_t valid;
   int32_t pid;
@@ -2905,7 +2914,9 @@ int dist_bootstrap(lmatch_graph* g, const lmatch_dist_id* id, int rank, int worl
   bool local = true;
   for (int q = 0; q < world; ++q) local = local && h->slot[q].pid == (int32_t)getpid();
   DTRACE(g, "peers attached (rc %d, %s)", rc, local ? "in-process event barriers" : "device flag barriers");
-  if (__atomic_add_fetch(&h->attached, 1, __ATOMIC_ACQ_REL) == world) shm_unlink(name);
+  // the last rank to attach removes the rendezvous; a rank that gave up waiting removes it too
+  // (the group cannot complete), so no segment is left behind in /dev/shm
+  if (__atomic_add_fetch(&h->attached, 1, __ATOMIC_ACQ_REL) == world || rc == LMATCH_ENCCL) shm_unlink(name);
   if (!rc && local) {
     g->dist_local = 1;
     g->dist_shm = mp;

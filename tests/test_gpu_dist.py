@@ -285,3 +285,36 @@ def test_dist_single_rank_uses_the_device_round_loop(D):
     for g in (graphgen.rmat(15, 16, seed=4), graphgen.mesh(64, seed=1, weights="gradient")):
         mate, st, _ = D.match_dist_threads(g.offsets, g.col, g.w, 1)
         check(g, mate, st)
+
+
+def _lonely_rank(q):
+    import paper_conf_sc_mandulakgfhs24_b200 as lm
+    import paper_conf_sc_mandulakgfhs24_b200.dist as Dm
+    g = graphgen.rmat(10, 8, seed=1)
+    b = Dm.edge_balanced_bounds(g.offsets, 2)
+    lo, lc, lw = Dm.local_csr(g.offsets, g.col, g.w, int(b[0]), int(b[1]))
+    try:
+        Dm.DistMatcher(lo, lc, lw, 0, g.n, 0, 2, b, Dm.dist_id_new())
+        q.put(0)
+    except lm.LMatchError as e:
+        q.put(e.status)
+
+
+def test_dist_missing_peer_times_out(D):
+    """Rank 0 of a 2-rank group whose peer never joins gets ENCCL after the rendezvous timeout
+    (LMATCH_DIST_TIMEOUT_S=3) instead of hanging, and leaves no segment in /dev/shm."""
+    import torch.multiprocessing as mp
+    before = set(os.listdir("/dev/shm")) if os.path.isdir("/dev/shm") else set()
+    os.environ["LMATCH_DIST_TIMEOUT_S"] = "3"
+    try:
+        ctx = mp.get_context("spawn")
+        q = ctx.Queue()
+        p = ctx.Process(target=_lonely_rank, args=(q,))
+        p.start()
+        p.join(timeout=120)
+        assert p.exitcode == 0
+        assert q.get(timeout=5) == -5  # LMATCH_ENCCL
+    finally:
+        del os.environ["LMATCH_DIST_TIMEOUT_S"]
+    after = set(os.listdir("/dev/shm")) if os.path.isdir("/dev/shm") else set()
+    assert not [x for x in after - before if x.startswith("lmatch-")]
