@@ -1161,6 +1161,12 @@ struct RoundArgs {
 #ifndef LM_RES_FAST
 #define LM_RES_FAST 1  // rows wholly in the HBM-resident prefix load keys straight from adj.dev
 #endif
+#ifndef LM_UB_FILTER
+#define LM_UB_FILTER 0  // 1 = keys at or above the vertex's previous pointer are skipped (R3)
+#endif
+#ifndef LM_LIST_PF
+#define LM_LIST_PF 0  // 1 = binned pointer kernels prefetch the group's next frontier entry
+#endif
 #ifndef LM_QEXIT
 #define LM_QEXIT 0  // 1 = sub-warp groups skip the key columns past the row end (group-uniform)
 #endif
@@ -1170,7 +1176,8 @@ template <int G, int U, bool RES>
 __device__ __forceinline__ uint64_t scan_row_available_t(const AdjView adj,
                                                          const uint32_t* __restrict__ bits,
                                                          int64_t s, int64_t e, int gl,
-                                                         unsigned rmask) {
+                                                         unsigned rmask, uint64_t ub = ~0ull) {
+  (void)ub;
   uint64_t b = 0;
   (void)rmask;
 #if LM_IDX32
@@ -1192,6 +1199,9 @@ __device__ __forceinline__ uint64_t scan_row_available_t(const AdjView adj,
         if ((int64_t)q * G >= rest) break;
         const int64_t j = j0 + (int64_t)q * G;
         if (j < e) k[q] = RES ? ld_stream_u64(adj.dev + j) : adj.at(j);
+#if LM_UB_FILTER
+        if (k[q] >= ub) k[q] = 0ull;
+#endif
       }
       uint32_t wd[U];
 #pragma unroll
@@ -1229,6 +1239,9 @@ __device__ __forceinline__ uint64_t scan_row_available_t(const AdjView adj,
     for (int q = 0; q < U; ++q) {
       const int64_t j = j0 + (int64_t)q * G;
       k[q] = j < e ? (RES ? ld_stream_u64(adj.dev + j) : adj.at(j)) : 0ull;
+#if LM_UB_FILTER
+      if (k[q] >= ub) k[q] = 0ull;
+#endif
     }
     }
 #if LM_PROBE == 3
@@ -1326,15 +1339,18 @@ __device__ __forceinline__ uint64_t scan_row_available_t(const AdjView adj,
   }
   return b;
 }
+// ub: an exclusive upper bound on the available keys of the row (LM_UB_FILTER): the vertex's
+// previous pointer, since every key above it was unavailable when it was computed and stays so
+// (R3) and the pointer's own target was matched; keys >= ub are neither compared nor probed
 template <int G, int U>
 __device__ __forceinline__ uint64_t scan_row_available(const AdjView adj,
                                                        const uint32_t* __restrict__ bits,
                                                        int64_t s, int64_t e, int gl,
-                                                       unsigned rmask) {
+                                                       unsigned rmask, uint64_t ub = ~0ull) {
 #if LM_RES_FAST
-  if (e <= adj.R) return scan_row_available_t<G, U, true>(adj, bits, s, e, gl, rmask);
+  if (e <= adj.R) return scan_row_available_t<G, U, true>(adj, bits, s, e, gl, rmask, ub);
 #endif
-  return scan_row_available_t<G, U, false>(adj, bits, s, e, gl, rmask);
+  return scan_row_available_t<G, U, false>(adj, bits, s, e, gl, rmask, ub);
 }
 
 // A7 in-place pruning (opt-in, lmatch_opts.prune) of a row that fits ONE batch
@@ -1408,15 +1424,32 @@ __device__ __forceinline__ void point_bin_body(ulonglong2* __restrict__ list, in
   const int gl = lane & (G - 1);
   const unsigned gmask = (G == 32) ? 0xffffffffu : (((1u << G) - 1u) << (lane & ~(G - 1)));
   const int64_t ng = gthreads / G;
+#if LM_LIST_PF
+  // the group's next list entry is loaded one row ahead, so a row's key loads do not wait for
+  // its entry (one dependent DRAM trip less per row)
+  ulonglong2 enx = gtid / G < cnt ? list[gtid / G] : make_ulonglong2(0ull, 0ull);
+#endif
   for (int64_t i = gtid / G; i < cnt; i += ng) {
+#if LM_LIST_PF
+    const ulonglong2 e = enx;
+    enx = i + ng < cnt ? list[i + ng] : make_ulonglong2(0ull, 0ull);
+#else
     const ulonglong2 e = list[i];
+#endif
     int64_t s, en;
     row_range(e, offs, vbase, &s, &en);
+    uint64_t ub = ~0ull;
+#if LM_UB_FILTER
+    {
+      const uint64_t old = best[(int64_t)(uint32_t)e.x - vbase];
+      if (old) ub = old;  // 0: unknown (a pushed vertex's pointer was cleared)
+    }
+#endif
     uint64_t b;
     if (PRUNE && en - s <= (int64_t)G * U)
       b = prune_row<G, U>(adj, bits, s, en, gl, gmask, live, tag, (int64_t)(uint32_t)e.x - vbase);
     else
-      b = group_max_key(scan_row_available<G, U>(adj, bits, s, en, gl, gmask), gmask);
+      b = group_max_key(scan_row_available<G, U>(adj, bits, s, en, gl, gmask, ub), gmask);
     if (gl == 0) {
       const uint32_t u = (uint32_t)e.x;
       best[u - vbase] = b;
@@ -1709,7 +1742,14 @@ __device__ __forceinline__ void point_bin_cta_body(ulonglong2* __restrict__ list
     const ulonglong2 e = list[i];
     int64_t s, en;
     row_range(e, offs, vbase, &s, &en);
-    uint64_t b = scan_row_available<THREADS, U>(adj, bits, s, en, threadIdx.x, 0xffffffffu);
+    uint64_t ub = ~0ull;
+#if LM_UB_FILTER
+    {
+      const uint64_t old = best[(int64_t)(uint32_t)e.x - vbase];
+      if (old) ub = old;
+    }
+#endif
+    uint64_t b = scan_row_available<THREADS, U>(adj, bits, s, en, threadIdx.x, 0xffffffffu, ub);
     b = group_max_key(b, 0xffffffffu);
     if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = b;
     __syncthreads();

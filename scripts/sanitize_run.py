@@ -8,7 +8,8 @@ driver is not run here: its device-barrier kernel spins on peers' flags, which t
 kernel serialisation would turn into a timeout; its in-process form, threads with event
 barriers, is run.)
 
-usage: compute-sanitizer --tool memcheck python scripts/sanitize_run.py [--quick]
+usage: compute-sanitizer --tool memcheck python scripts/sanitize_run.py [--quick] [--single]
+(--single: single-graph handles only)
 """
 import os
 import sys
@@ -36,13 +37,17 @@ for g in graphs:
         dict(hbm_budget_bytes=8 * g.m // 3, stream_chunk=4096, host_cache=False),
         dict(batches=3)]
     for kw in configs:
+        print(f"{g.name} {kw}", flush=True)
         with lm.Matcher(g, **kw) as M:
             mate, st = M.run()
             assert np.array_equal(mate, ref), (g.name, kw)
             w = M.weight(mate)
             assert abs(w - st["weight"]) <= 1e-9 * max(1.0, abs(w))
         runs += 1
+    if "--single" in sys.argv:
+        continue
     for ex in ("transport", "p2p", "p2p_sync"):
+        print(f"{g.name} partitioned {ex}", flush=True)
         mate, _ = D.match_partitioned_local(g.offsets, g.col, g.w, 3, exchange=ex)
         assert np.array_equal(mate, ref), (g.name, ex)
         runs += 1
