@@ -317,9 +317,13 @@ def gen_rank_rows(a, scale, rank, world, dev):
         offs_h = offs.cpu().numpy()
         bounds = D.edge_balanced_bounds(offs_h, world)
         v0, v1 = int(bounds[rank]), int(bounds[rank + 1])
+        m_loc = int(offs_h[v1] - offs_h[v0])
+        # the rank's device CSR (8 B/entry) next to the matcher's packed keys (8 B/entry) and
+        # per-vertex state must fit in HBM; else the rows are assembled in pinned host memory
+        host_out = 16 * m_loc + 48 * (v1 - v0) > 0.85 * torch.cuda.get_device_properties(dev).total_memory
         if a.workload == "rmat":
             dg = gg.rmat_rows(scale, v0, v1, offs, a.edgefactor, seed=a.seed, weights=a.weights or "uniform",
-                              device=dev)
+                              device=dev, host_out=host_out)
         else:
             dg = gg.er_rows(1 << scale, v0, v1, offs, float(a.edgefactor), seed=a.seed,
                             weights=a.weights or "uniform", device=dev)
@@ -356,8 +360,10 @@ def run_partitioned(a, rank, world, local, dev):
     lo, lc, lw, v0, v1, bounds, n, m, offs_h = gen_rank_rows(a, scale, rank, world, dev)
     m_u = m // 2
     host = None
+    if not lo.is_cuda:  # assembled in pinned host memory: create from host arrays
+        lo, lc, lw = lo.numpy(), lc.numpy(), lw.numpy()
     if not a.no_e2e:
-        host = (lo.cpu().numpy(), lc.cpu().numpy(), lw.cpu().numpy())
+        host = tuple(x.cpu().numpy() if hasattr(x, "is_cuda") else x for x in (lo, lc, lw))
     n_nz_loc = int(np.count_nonzero(np.diff(offs_h[v0:v1 + 1])))
     del offs_h
     gen_s = time.time() - t0

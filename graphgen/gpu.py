@@ -152,12 +152,14 @@ def _edge_graph(kind, n, scale, M, seed, a, b, c, weights, wseed, device, bucket
 
 
 def _edge_graph_rows(kind, n, scale, M, seed, a, b, c, weights, wseed, device, bucket_entries, name,
-                     rows=None, offsets=None):
+                     rows=None, offsets=None, host_out=False):
     """Row-range generation for one rank of a partitioned run (each rank holds only its rows):
     rows=None -> pass 1: the graph's full CSR offsets (torch int64[n+1] on `device`; col/w of each
     bucket go to scratch and are dropped); rows=(v0, v1) with the pass-1 offsets -> pass 2: the
     local CSR of rows [v0, v1) (offsets rebased to 0, GLOBAL column ids), generating only the
-    buckets that hold those rows.  Same edges and weights as _edge_graph (same kernels)."""
+    buckets that hold those rows.  Same edges and weights as _edge_graph (same kernels).
+    host_out (pass 2): the local CSR is assembled in pinned host memory (a rank whose rows and
+    the matcher's packed keys would not fit in HBM together)."""
     import torch
     L = _load()
     dev = torch.device(device)
@@ -186,8 +188,9 @@ def _edge_graph_rows(kind, n, scale, M, seed, a, b, c, weights, wseed, device, b
         v0, v1 = int(rows[0]), int(rows[1])
         offs_h = offsets.cpu() if offsets.is_cuda else offsets
         S, E = int(offs_h[v0]), int(offs_h[v1])
-        col = torch.empty(max(E - S, 1), dtype=torch.int32, device=dev)
-        w = torch.empty(max(E - S, 1), dtype=torch.float32, device=dev)
+        odev = "cpu" if host_out else dev
+        col = torch.empty(max(E - S, 1), dtype=torch.int32, device=odev, pin_memory=host_out)
+        w = torch.empty(max(E - S, 1), dtype=torch.float32, device=odev, pin_memory=host_out)
     base = 0
     for bkt in range(nb):
         if counts_h[bkt] == 0:
@@ -221,7 +224,7 @@ def _edge_graph_rows(kind, n, scale, M, seed, a, b, c, weights, wseed, device, b
         torch.cuda.synchronize(dev)
         return offsets
     del first
-    loff = (offsets[v0:v1 + 1].to(dev) - S).contiguous()
+    loff = (offsets[v0:v1 + 1].to("cpu" if host_out else dev) - S).contiguous()
     torch.cuda.synchronize(dev)
     return DeviceGraph(loff, col[:E - S], w[:E - S], v1 - v0, E - S, name + f"_rows{v0}-{v1}")
 
@@ -236,12 +239,15 @@ def rmat_offsets(scale: int, edgefactor: int = 16, seed: int = 1, a: float = 0.5
 
 def rmat_rows(scale: int, v0: int, v1: int, offsets, edgefactor: int = 16, seed: int = 1,
               a: float = 0.57, b: float = 0.19, c: float = 0.19, weights: str = "uniform",
-              wseed: int | None = None, device="cuda", bucket_entries: int = 1 << 28) -> DeviceGraph:
+              wseed: int | None = None, device="cuda", bucket_entries: int = 1 << 28,
+              host_out: bool = False) -> DeviceGraph:
     """Rows [v0, v1) of rmat(scale, ...) as a local CSR (global column ids); `offsets` from
-    rmat_offsets.  n / m of the result are the LOCAL row and entry counts."""
+    rmat_offsets.  n / m of the result are the LOCAL row and entry counts.  host_out: pinned CPU
+    tensors (built on the GPU)."""
     n = 1 << scale
     return _edge_graph_rows(1, n, scale, edgefactor * n, seed, a, b, c, weights, wseed, device,
-                            bucket_entries, f"rmat_s{scale}_ef{edgefactor}", (v0, v1), offsets)
+                            bucket_entries, f"rmat_s{scale}_ef{edgefactor}", (v0, v1), offsets,
+                            host_out)
 
 
 def er_offsets(n: int, avg_degree: float = 16.0, seed: int = 1, device="cuda",

@@ -11,8 +11,8 @@ want = ['Kernel Name', 'gpu__time_duration.sum', 'dram__bytes_read.sum', 'dram__
         'lts__t_sector_hit_rate.pct', 'lts__throughput.avg.pct_of_peak_sustained_elapsed',
         'smsp__inst_executed.sum', 'launch__shared_mem_per_block_dynamic',
         'l1tex__data_bank_conflicts_pipe_lsu_mem_shared.sum', 'smsp__issue_active.avg.pct_of_peak_sustained_active',
-        'smsp__sass_average_data_bytes_per_sector_mem_global_op_ld.pct',
-        'smsp__sass_average_data_bytes_per_sector_mem_global_op_st.pct',
+        'smsp__sass_average_data_bytes_per_sector_mem_global_op_ld.ratio',
+        'smsp__sass_average_data_bytes_per_sector_mem_global_op_st.ratio',
         'lts__t_sectors_srcunit_tex_op_read.sum', 'l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum']
 for row in r[2:]:
     for i, k in enumerate(h):
