@@ -63,6 +63,9 @@ def parse():
                         "adjacency from pinned host memory as B batches in round 1")
     p.add_argument("--key-cache", action="store_true",
                    help="resident: the round-1 top-4 key cache (lmatch_opts.key_cache = 1; off by default)")
+    p.add_argument("--frontier", default="auto", choices=["auto", "pull", "push"],
+                   help="A6 next frontier in the persistent-kernel rounds: auto = pull, switching to "
+                        "push on many-round graphs (lmatch_opts.frontier = 0); pull = pull only")
     p.add_argument("--residual-mb", type=int, default=0,
                    help="out of core: MiB of HBM for copies of rescanned host rows (lmatch_opts.residual_mb)")
     p.add_argument("--no-host-cache", action="store_true",
@@ -145,6 +148,8 @@ def workload_config(a, scale, n, m):
         cfg["prune"] = True
     if getattr(a, "algorithm", "ld") != "ld":
         cfg["algorithm"] = a.algorithm
+    if getattr(a, "frontier", "auto") != "auto":
+        cfg["frontier"] = a.frontier
     return cfg
 
 
@@ -590,7 +595,8 @@ def main():
     opts = lm.make_opts(validate_level=1, timing=1,
                         hbm_budget_bytes=int(a.hbm_budget_gb * 1e9), stream_chunk=a.stream_chunk,
                         prune=a.prune, host_cache=not a.no_host_cache,
-                        batches=a.batches, algorithm=a.algorithm, key_cache=a.key_cache, residual_mb=a.residual_mb)
+                        batches=a.batches, algorithm=a.algorithm, key_cache=a.key_cache, residual_mb=a.residual_mb,
+                        frontier=a.frontier)
     pinned_host = d_off is None
     if pinned_host:
         h = lm.lmatch_create_ex(g.offsets, g.col, g.w, n, m, opts)

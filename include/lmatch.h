@@ -180,10 +180,12 @@ typedef struct lmatch_opts {
   int32_t frontier;           /* A6 next-frontier construction in the persistent-kernel rounds
                                  (round_loop 0, 2, 3): 0 = default, pull (compaction of the live
                                  list) switching to push once the live list is 8x the frontier
-                                 (the vertices newly matched in a round push their row neighbours
-                                 that pointed at them: O(m) over the run instead of O(|L| x
-                                 rounds) -- many-round graphs); 1 = pull only.  Not with prune or
-                                 algorithm 2.  Same result and pointing phases */
+                                 and at least 2^20 vertices long (the vertices newly matched in a
+                                 round push their row neighbours that pointed at them: O(m) over
+                                 the run instead of O(|L| x rounds) -- many-round graphs);
+                                 1 = pull only; 2 = push as soon as the live list is 8x the
+                                 frontier, whatever its length.  Not with prune or algorithm 2.
+                                 Same result and pointing phases */
   int32_t reserved[3];
 } lmatch_opts;
 

@@ -342,7 +342,7 @@ def make_opts(validate_level: int = 1, timing: bool = False, upload_chunk: int =
     o.sort_chunk_log2 = int(sort_chunk_log2)
     o.key_cache = 1 if key_cache else 0
     o.residual_mb = int(residual_mb)
-    o.frontier = {"auto": 0, "pull": 1}[frontier]
+    o.frontier = {"auto": 0, "pull": 1, "push": 2}[frontier]
     o.hbm_budget_bytes = int(hbm_budget_bytes)
     o.stream_chunk = int(stream_chunk)
     o.validate_level = int(validate_level)

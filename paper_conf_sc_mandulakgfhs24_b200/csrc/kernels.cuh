@@ -1134,6 +1134,7 @@ struct RoundArgs {
   const uint64_t* kc;       // resident key cache [n][kKC] (nullptr = off)
   uint64_t* best;           // per-vertex pointers (the compaction writes the cache-decided ones)
   uint32_t* N;              // A6 push frontier: vertices newly matched this round (nullptr = off)
+  unsigned long long push_min_live;  // ... used once the live list is at least this long
 };
 
 // A2 pointer phase on the frontier (rounds >= 2): G lanes per vertex (degree-binned).
@@ -2269,6 +2270,13 @@ __global__ void k_round_init(RoundState* st, long long max_rounds, long long log
 #define LM_PUSH_RATIO 8
 #endif
 constexpr unsigned long long kPushRatio = LM_PUSH_RATIO;
+// ... and only once the live list is long enough for its per-round pass to cost more than the
+// push step's fixed work (gradient meshes: pull wins at 1024^2 -- 45 vs 57 ms -- push at 2048^2
+// and 4096^2 -- 123 vs 135 ms, 222 vs 720 ms)
+#ifndef LM_PUSH_MIN_LIVE
+#define LM_PUSH_MIN_LIVE (1ull << 20)
+#endif
+constexpr unsigned long long kPushMinLive = LM_PUSH_MIN_LIVE;
 __device__ __forceinline__ int end_round_body(const RoundArgs* __restrict__ ra, long long first_log_rows,
                                               bool push_ok = false) {
   RoundState* st = ra->st;
@@ -2282,7 +2290,8 @@ __device__ __forceinline__ int end_round_body(const RoundArgs* __restrict__ ra, 
   // A6: once the live list is much longer than the frontier (many-round graphs), the next
   // frontier is pushed from the newly matched vertices instead of pulled from the live list
   // (only the persistent kernel runs push rounds; it passes push_ok)
-  if (push_ok && ra->N && !st->push && nS + nF > kPushRatio * nF) st->push = 1;
+  if (push_ok && ra->N && !st->push && nS + nF > kPushRatio * nF && nS + nF >= ra->push_min_live)
+    st->push = 1;
   ra->cnt[kCntN] = 0ull;
   // zero the counters of the set the next compaction writes
 #pragma unroll

@@ -371,6 +371,7 @@ struct lmatch_graph {
     a.kc = kcache;
     a.best = best;
     a.N = (push_ok && !prune && algorithm != 2) ? pushN : nullptr;
+    a.push_min_live = push_ok == 2 ? 0ull : lm::kPushMinLive;
     return a;
   }
 };
@@ -1059,7 +1060,7 @@ int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** 
     g->algorithm = opts->algorithm;
     g->key_cache = opts->key_cache > 0;
     g->residual_mb = opts->residual_mb;
-    g->push_ok = opts->frontier != 1;
+    g->push_ok = opts->frontier == 1 ? 0 : (opts->frontier == 2 ? 2 : 1);
     if (opts->sort_chunk_log2 != 0) {
       if (opts->sort_chunk_log2 < 4 || opts->sort_chunk_log2 > 30) {
         set_err("sort_chunk_log2 = %d outside 4..30", opts->sort_chunk_log2);
@@ -1088,8 +1089,10 @@ int create_common(int64_t n, int64_t m, const lmatch_opts* opts, lmatch_graph** 
   if (part) {
     TRY(dmalloc(g, &g->bounds, (size_t)g->P + 1));
     CK(cudaMemcpy(g->bounds, part->bounds, ((size_t)g->P + 1) * 8, cudaMemcpyHostToDevice));
-    TRY(dmalloc(g, &g->ghost, (size_t)g->n_global + 1));
-    g->claim_cap = std::max<int64_t>(n, 1);
+    // one part: nothing is remote, so no ghosts and no claims are ever stored (minimal buffers;
+    // the handle still counts as a partition handle)
+    TRY(dmalloc(g, &g->ghost, g->P > 1 ? (size_t)g->n_global + 1 : 2));
+    g->claim_cap = g->P > 1 ? std::max<int64_t>(n, 1) : 1;
     TRY(dmalloc(g, &g->claims, (size_t)g->P * (size_t)g->claim_cap));
     TRY(dmalloc(g, &g->claim_cnt, (size_t)g->P));
     CK(cudaHostAlloc(reinterpret_cast<void**>(&g->h_claim_cnt), (size_t)g->P * 8, cudaHostAllocDefault));
@@ -2517,8 +2520,8 @@ int lmatch_p2p_enable(lmatch_graph* g, int32_t me) {
   if (g->p2p) return LMATCH_OK;
   CK(cudaSetDevice(g->device));
   const int P = g->P;
-  int64_t cap = 1;
-  for (int p = 0; p < P; ++p) cap = std::max(cap, g->hbounds[p + 1] - g->hbounds[p]);
+  int64_t cap = 1;  // inbox segment: the largest part (one part receives no claims)
+  for (int p = 0; P > 1 && p < P; ++p) cap = std::max(cap, g->hbounds[p + 1] - g->hbounds[p]);
   g->me = me;
   g->win_cap = cap;
   TRY(dmalloc(g, &g->win, (size_t)P * cap + 6 * (size_t)P));
