@@ -138,7 +138,8 @@ constexpr int64_t kHandoffRounds = 32;  // hybrid (algorithm 2): LD pointing pha
 // host-driven rounds: software-pipelined pointer kernels (one resident wave) per bin: bit b of
 // LM_PIPE set = bin b uses k_point_pipe<LM_Pb_G, LM_Pb_U>
 #ifndef LM_PIPE
-#define LM_PIPE 1  // measured (R-MAT s26): pipelining helps the thread-per-row bin only (-10 to -20%)
+#define LM_PIPE 3  // bins 0 and 1 software-pipelined (k_point_pipe<1,8>, <8,4>); round 2, R-MAT s26, one box:
+                   // 12.06 -> 11.89 ms against the 16 x 4 bin kernel (4 x 4: 11.89, 4 x 8: 11.95, 2 x 8: 11.97)
 #endif
 #ifndef LM_P0_G
 #define LM_P0_G 1
@@ -841,10 +842,12 @@ int alloc_bins(lmatch_graph* g, cudaStream_t st) {
   g->device_bytes -= 16;
   // A7 pruning moves rows to LOWER bins (live degrees only shrink): bin b must then hold every
   // row whose full degree is in bin b or above
-  if (g->push_ok) TRY(ensure(g, &g->pushN, &g->cap_pushN, g->n_nz + 1));
-  // the decided list (key cache) can hold any non-empty row
+  // the push frontier runs in the persistent kernel only (single graph or a one-rank partition)
+  if (g->push_ok && !g->prune && g->algorithm != 2 && g->round_loop != 1 && !g->streaming && g->P == 1)
+    TRY(ensure(g, &g->pushN, &g->cap_pushN, g->n_nz + 1));
+  // the decided list (key cache only) can hold any non-empty row
   h[lm::kDecided] = 0;
-  for (int b = 0; b < lm::kDegBins; ++b) h[lm::kDecided] += h[b];
+  for (int b = 0; g->kcache && b < lm::kDegBins; ++b) h[lm::kDecided] += h[b];
   if (g->prune)
     for (int b = lm::kDegBins - 2; b >= 0; --b) h[b] += h[b + 1];
   for (int i = 0; i < 2; ++i)
