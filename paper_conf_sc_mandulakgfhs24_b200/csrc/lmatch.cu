@@ -2430,7 +2430,21 @@ static int part_point_impl(lmatch_graph* g, cudaStream_t st, int64_t* claim_coun
 #endif
     CKL();
   }
-  if (nFb[1]) { lm::k_point_bin<LM_B1_G, LM_B1_U><<<grid_for(nFb[1] * LM_B1_G, 256, 65536), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, av, g->bits, g->best, g->v0); CKL(); }
+  if (nFb[1]) {
+#if LM_PIPE & 2
+    static int occ1 = 0;
+    if (!occ1) {
+      CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ1, lm::k_point_pipe<LM_P1_G, LM_P1_U>, 256, 0));
+      if (occ1 < 1) occ1 = 1;
+    }
+    const int64_t wave1 = (int64_t)occ1 * g->num_sms * LM_PIPE_WAVES;
+    lm::k_point_pipe<LM_P1_G, LM_P1_U><<<(unsigned)std::min<int64_t>(wave1, (nFb[1] * LM_P1_G + 255) / 256), 256, 0, st>>>(
+        Fb.list[1], cF + 1, g->offs, av, g->bits, g->best, g->v0);
+#else
+    lm::k_point_bin<LM_B1_G, LM_B1_U><<<grid_for(nFb[1] * LM_B1_G, 256, 65536), 256, 0, st>>>(Fb.list[1], cF + 1, g->offs, av, g->bits, g->best, g->v0);
+#endif
+    CKL();
+  }
   if (nFb[2]) { lm::k_point_bin<LM_B2_G, LM_B2_U><<<grid_for(nFb[2] * LM_B2_G, 256, 65536), 256, 0, st>>>(Fb.list[2], cF + 2, g->offs, av, g->bits, g->best, g->v0); CKL(); }
   if (nFb[3]) { lm::k_point_bin_cta<256, LM_CTA_U><<<(unsigned)std::min<int64_t>(nFb[3], g->p2p ? 8ll * g->num_sms : 65536), 256, 0, st>>>(Fb.list[3], cF + 3, g->offs, av, g->bits, g->best, g->v0); CKL(); }
   if (!g->p2p) CK(cudaMemsetAsync(g->claim_cnt, 0, (size_t)g->P * 8, st));
