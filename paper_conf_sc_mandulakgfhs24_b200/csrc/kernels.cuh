@@ -1103,8 +1103,20 @@ __device__ __forceinline__ void row_range(const ulonglong2& e, const int64_t* __
   *en = d == kBigDeg ? offs[(int64_t)(uint32_t)e.x - vbase + 1] : *s + (int64_t)d;
 }
 
+// One frontier list, structure of arrays (round 2): p[i] = u | ptr << 32 (the pair the match and
+// the compaction read: 8 B per entry instead of 16), r[i] = row start | degree << 40 (read by the
+// pointer kernels with it).  list[i] returns both as a ulonglong2 (.x = p, .y = r).
+struct FL {
+  uint64_t* p;
+  uint64_t* r;
+  __device__ __forceinline__ ulonglong2 operator[](int64_t i) const { return make_ulonglong2(p[i], r[i]); }
+  __device__ __forceinline__ void put(int64_t i, const ulonglong2& e) const {
+    p[i] = e.x;
+    r[i] = e.y;
+  }
+};
 struct Bins {
-  ulonglong2* list[kBins];
+  FL list[kBins];
 };
 
 // Device-resident round bookkeeping, so the round loop needs no host decision: the same launch
@@ -1414,7 +1426,7 @@ __device__ __forceinline__ uint64_t prune_row(const AdjView adj, const uint32_t*
 }
 
 template <int G, int U, bool PRUNE = false>
-__device__ __forceinline__ void point_bin_body(ulonglong2* __restrict__ list, int64_t cnt,
+__device__ __forceinline__ void point_bin_body(const FL list, int64_t cnt,
                                                const int64_t* __restrict__ offs, const AdjView adj,
                                                const uint32_t* __restrict__ bits,
                                                uint64_t* __restrict__ best, int64_t vbase,
@@ -1454,7 +1466,7 @@ __device__ __forceinline__ void point_bin_body(ulonglong2* __restrict__ list, in
     if (gl == 0) {
       const uint32_t u = (uint32_t)e.x;
       best[u - vbase] = b;
-      list[i].x = make_pair(u, b ? (uint32_t)b : kNoPtr);
+      list.p[i] = make_pair(u, b ? (uint32_t)b : kNoPtr);
     }
   }
 }
@@ -1462,7 +1474,7 @@ __device__ __forceinline__ void point_bin_body(ulonglong2* __restrict__ list, in
 #define LM_BIN_MINB 8  // 32-register cap, full occupancy (6 -> 8 with the 16x4 / 32x8 bins: rounds 8.09 -> 7.74 ms)
 #endif
 template <int G, int U, bool PRUNE = false>
-__global__ void __launch_bounds__(256, LM_BIN_MINB) k_point_bin(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
+__global__ void __launch_bounds__(256, LM_BIN_MINB) k_point_bin(const FL list, const unsigned long long* cnt_ptr,
                             const int64_t* __restrict__ offs, const AdjView adj,
                             const uint32_t* __restrict__ bits, uint64_t* __restrict__ best,
                             int64_t vbase, uint32_t* __restrict__ live = nullptr,
@@ -1548,7 +1560,7 @@ __device__ __forceinline__ uint64_t probe_batch2(const uint32_t* __restrict__ bi
 }
 
 template <int G, int U>
-__device__ __forceinline__ void point_pipe_body(ulonglong2* __restrict__ list, int64_t cnt,
+__device__ __forceinline__ void point_pipe_body(const FL list, int64_t cnt,
                                                 const int64_t* __restrict__ offs, const AdjView adj,
                                                 const uint32_t* __restrict__ bits,
                                                 uint64_t* __restrict__ best, int64_t vbase,
@@ -1604,7 +1616,7 @@ __device__ __forceinline__ void point_pipe_body(ulonglong2* __restrict__ list, i
 #endif
       if (gl == 0) {
         best[cu - vbase] = r;
-        list[ci].x = make_pair(cu, r ? (uint32_t)r : kNoPtr);
+        list.p[ci] = make_pair(cu, r ? (uint32_t)r : kNoPtr);
       }
       b = 0;
     }
@@ -1621,7 +1633,7 @@ __device__ __forceinline__ void point_pipe_body(ulonglong2* __restrict__ list, i
 #endif
 template <int G, int U>
 __global__ void __launch_bounds__(256, LM_PIPE_MINB)
-    k_point_pipe(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
+    k_point_pipe(const FL list, const unsigned long long* cnt_ptr,
                  const int64_t* __restrict__ offs, const AdjView adj,
                  const uint32_t* __restrict__ bits, uint64_t* __restrict__ best, int64_t vbase) {
   point_pipe_body<G, U>(list, (int64_t)*cnt_ptr, offs, adj, bits, best, vbase,
@@ -1648,7 +1660,7 @@ __device__ __forceinline__ void cp_async_wait() {
 }
 template <int G, int U, int S>
 __global__ void __launch_bounds__(256)
-    k_point_async(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
+    k_point_async(const FL list, const unsigned long long* cnt_ptr,
                   const int64_t* __restrict__ offs, const uint64_t* __restrict__ adj,
                   const uint32_t* __restrict__ bits, uint64_t* __restrict__ best, int64_t vbase) {
   extern __shared__ __align__(16) uint64_t sk[];  // [S][U][256]
@@ -1721,7 +1733,7 @@ __global__ void __launch_bounds__(256)
         const uint64_t r = G > 1 ? group_max_key(b, gmask) : b;
         if (gl == 0) {
           best[tu[st] - vbase] = r;
-          list[tci[st]].x = make_pair(tu[st], r ? (uint32_t)r : kNoPtr);
+          list.p[tci[st]] = make_pair(tu[st], r ? (uint32_t)r : kNoPtr);
         }
         b = 0;
       }
@@ -1732,7 +1744,7 @@ done:
 }
 
 template <int THREADS, int U>
-__device__ __forceinline__ void point_bin_cta_body(ulonglong2* __restrict__ list, int64_t cnt,
+__device__ __forceinline__ void point_bin_cta_body(const FL list, int64_t cnt,
                                                    const int64_t* __restrict__ offs,
                                                    const AdjView adj,
                                                    const uint32_t* __restrict__ bits,
@@ -1760,7 +1772,7 @@ __device__ __forceinline__ void point_bin_cta_body(ulonglong2* __restrict__ list
       if (threadIdx.x == 0) {
         const uint32_t u = (uint32_t)e.x;
         best[u - vbase] = x;
-        list[i].x = make_pair(u, x ? (uint32_t)x : kNoPtr);
+        list.p[i] = make_pair(u, x ? (uint32_t)x : kNoPtr);
       }
     }
     __syncthreads();
@@ -1768,7 +1780,7 @@ __device__ __forceinline__ void point_bin_cta_body(ulonglong2* __restrict__ list
 }
 template <int THREADS, int U>
 __global__ void __launch_bounds__(THREADS)
-    k_point_bin_cta(ulonglong2* __restrict__ list, const unsigned long long* cnt_ptr,
+    k_point_bin_cta(const FL list, const unsigned long long* cnt_ptr,
                     const int64_t* __restrict__ offs, const AdjView adj,
                     const uint32_t* __restrict__ bits, uint64_t* __restrict__ best, int64_t vbase) {
   point_bin_cta_body<THREADS, U>(list, (int64_t)*cnt_ptr, offs, adj, bits, best, vbase, blockIdx.x,
@@ -1823,7 +1835,7 @@ __device__ __forceinline__ void match_bins_body(const Bins& F, const unsigned lo
 #pragma unroll
       for (int q = 0; q < V; ++q) {
         const int64_t i = i0 + q * stride;
-        p[q] = i < c ? F.list[bb][i].x : ((uint64_t)kNoPtr << 32);
+        p[q] = i < c ? F.list[bb].p[i] : ((uint64_t)kNoPtr << 32);
       }
 #pragma unroll
       for (int q = 0; q < V; ++q) {
@@ -1845,7 +1857,7 @@ __device__ __forceinline__ void match_bins_body(const Bins& F, const unsigned lo
   for (int bb = 0; bb < kBins; ++bb) {
     const int64_t c = (int64_t)cntF[bb];
     for (int64_t i = tid; i < c; i += stride) {
-      const uint64_t p = F.list[bb][i].x;
+      const uint64_t p = F.list[bb].p[i];
       const uint32_t u = (uint32_t)p, v = (uint32_t)(p >> 32);
       if (v == kNoPtr) continue;
       const uint64_t kv = best[v];
@@ -1973,10 +1985,10 @@ __device__ __forceinline__ void compact_body_plain(const CompactIO& io, int64_t 
           p = make_pair((uint32_t)(r + vbase), bb ? (uint32_t)bb : kNoPtr);
         } else {
           p = i < p0 ? S[i]
-              : i < p1 ? Fin.list[0][i - p0].x
-              : i < p2 ? Fin.list[1][i - p1].x
-              : i < p3 ? Fin.list[2][i - p2].x
-                       : Fin.list[3][i - p3].x;
+              : i < p1 ? Fin.list[0].p[i - p0]
+              : i < p2 ? Fin.list[1].p[i - p1]
+              : i < p3 ? Fin.list[2].p[i - p2]
+                       : Fin.list[3].p[i - p3];
         }
       }
       pr[k] = p;
@@ -2054,16 +2066,16 @@ __device__ __forceinline__ void compact_body_plain(const CompactIO& io, int64_t 
       bs += __popc(bls);
       const ulonglong2 ent = make_ulonglong2(pr[k], rr[k]);
       unsigned bb = __ballot_sync(0xffffffffu, (fb0 & m) != 0);
-      if (fb0 & m) Fout.list[0][bf0 + __popc(bb & lt)] = ent;
+      if (fb0 & m) Fout.list[0].put(bf0 + __popc(bb & lt), ent);
       bf0 += __popc(bb);
       bb = __ballot_sync(0xffffffffu, (fb1 & m) != 0);
-      if (fb1 & m) Fout.list[1][bf1 + __popc(bb & lt)] = ent;
+      if (fb1 & m) Fout.list[1].put(bf1 + __popc(bb & lt), ent);
       bf1 += __popc(bb);
       bb = __ballot_sync(0xffffffffu, (fb2 & m) != 0);
-      if (fb2 & m) Fout.list[2][bf2 + __popc(bb & lt)] = ent;
+      if (fb2 & m) Fout.list[2].put(bf2 + __popc(bb & lt), ent);
       bf2 += __popc(bb);
       bb = __ballot_sync(0xffffffffu, (fb3 & m) != 0);
-      if (fb3 & m) Fout.list[3][bf3 + __popc(bb & lt)] = ent;
+      if (fb3 & m) Fout.list[3].put(bf3 + __popc(bb & lt), ent);
       bf3 += __popc(bb);
     }
   }
@@ -2122,11 +2134,11 @@ __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
           p = make_pair((uint32_t)(r + vbase), bb ? (uint32_t)bb : kNoPtr);
         } else {
           p = i < pe[0] ? S[i]
-              : i < pe[1] ? Fin.list[0][i - pe[0]].x
-              : i < pe[2] ? Fin.list[1][i - pe[1]].x
-              : i < pe[3] ? Fin.list[2][i - pe[2]].x
-              : i < pe[4] ? Fin.list[3][i - pe[3]].x
-                          : Fin.list[4][i - pe[4]].x;
+              : i < pe[1] ? Fin.list[0].p[i - pe[0]]
+              : i < pe[2] ? Fin.list[1].p[i - pe[1]]
+              : i < pe[3] ? Fin.list[2].p[i - pe[2]]
+              : i < pe[4] ? Fin.list[3].p[i - pe[3]]
+                          : Fin.list[4].p[i - pe[4]];
         }
       }
       pr[k] = p;
@@ -2226,7 +2238,7 @@ __device__ __forceinline__ void compact_body(const CompactIO& io, int64_t n,
 #pragma unroll
       for (int q = 0; q < NOUT; ++q) {
         const unsigned bb = __ballot_sync(0xffffffffu, (fb[q] & m) != 0);
-        if (fb[q] & m) Fout.list[q][bf[q] + __popc(bb & lt)] = ent;
+        if (fb[q] & m) Fout.list[q].put(bf[q] + __popc(bb & lt), ent);
         bf[q] += __popc(bb);
       }
     }
@@ -2338,7 +2350,7 @@ __device__ __forceinline__ void match_push_body(const Bins& F, const unsigned lo
     const int64_t c = (int64_t)cntF[bb];
     for (int64_t i0 = tid - lane; i0 < c; i0 += stride) {  // warp-uniform trip count
       const int64_t i = i0 + lane;
-      const uint64_t p = i < c ? F.list[bb][i].x : ((uint64_t)kNoPtr << 32);
+      const uint64_t p = i < c ? F.list[bb].p[i] : ((uint64_t)kNoPtr << 32);
       const uint32_t u = (uint32_t)p, v = (uint32_t)(p >> 32);
       bool nu = false, nv = false;
       if (v != kNoPtr) {
@@ -2378,8 +2390,8 @@ __device__ __forceinline__ void push_body(const uint32_t* __restrict__ N, int64_
       const int64_t os = offs[lu], d = offs[lu + 1] - os;
       const int b = bin_of(d);
       const unsigned long long pos = atomicAdd(&cntFout[b], 1ull);
-      Fout.list[b][pos] = make_ulonglong2(make_pair(u, v),
-                                          (uint64_t)os | ((uint64_t)(d < (int64_t)kBigDeg ? d : (int64_t)kBigDeg) << 40));
+      Fout.list[b].put(pos, make_ulonglong2(make_pair(u, v),
+                                            (uint64_t)os | ((uint64_t)(d < (int64_t)kBigDeg ? d : (int64_t)kBigDeg) << 40)));
       degsum += (unsigned long long)d;
     }
   }
@@ -2511,7 +2523,7 @@ __global__ void k_claims_bins(Bins F, const unsigned long long* cntF, int64_t vb
     const int64_t c = (int64_t)cntF[bb];
     const int64_t c32 = (c + 31) & ~31ll;
     for (int64_t i = tid; i < c32; i += stride) {
-      const uint64_t p = i < c ? F.list[bb][i].x : ((uint64_t)kNoPtr << 32);
+      const uint64_t p = i < c ? F.list[bb].p[i] : ((uint64_t)kNoPtr << 32);
       const uint32_t u = (uint32_t)p, v = (uint32_t)(p >> 32);
       claim_append(C, v != kNoPtr && ((int64_t)v < vbase || (int64_t)v >= vend), v, u);
     }
@@ -2674,7 +2686,7 @@ __global__ void k_match_part_bins(Bins F, const unsigned long long* cntF,
   for (int bb = 0; bb < kBins; ++bb) {
     const int64_t c = (int64_t)cntF[bb];
     for (int64_t i = tid; i < c; i += stride) {
-      const uint64_t p = F.list[bb][i].x;
+      const uint64_t p = F.list[bb].p[i];
       const uint32_t u = (uint32_t)p, v = (uint32_t)(p >> 32);
       if (v == kNoPtr) continue;
       if (ptr_of(best, ghost, vbase, vend, v) == u) {
@@ -2982,7 +2994,7 @@ __global__ void k_cache_redirect(Bins F, const unsigned long long* __restrict__ 
         // a residual row: its copy in HBM is scanned by the pointer kernels (no host read)
         const int64_t d = en - s;
         e.y = (uint64_t)(M2 + roff[u - u_first]) | ((uint64_t)(d < (int64_t)kBigDeg ? d : (int64_t)kBigDeg) << 40);
-        F.list[bb][i].y = e.y;
+        F.list[bb].r[i] = e.y;
         ++resid;
         continue;
       } else {
@@ -2992,7 +3004,7 @@ __global__ void k_cache_redirect(Bins F, const unsigned long long* __restrict__ 
         if (rescan) rescan[atomicAdd(nrescan, 1ull)] = ((uint64_t)bb << 40) | (uint64_t)i;
         continue;
       }
-      F.list[bb][i].y = e.y;
+      F.list[bb].r[i] = e.y;
       ++served;
     }
   }
@@ -3059,7 +3071,7 @@ __global__ void __launch_bounds__(256) k_host_rescan(Bins F, const uint64_t* __r
     if (lane < K) cache[slot + lane] = mine;
     const uint64_t top = __shfl_sync(0xffffffffu, mine, 0);
     if (lane == 0)
-      F.list[bb][i].y = top ? ((1ull << 40) | (uint64_t)(M0 + slot)) : (uint64_t)(M0 + slot);
+      F.list[bb].r[i] = top ? ((1ull << 40) | (uint64_t)(M0 + slot)) : (uint64_t)(M0 + slot);
   }
 }
 
@@ -3252,7 +3264,7 @@ __global__ void k_suitor_tail_list(const uint64_t* __restrict__ S, const unsigne
     const int64_t c = (int64_t)cntF[bb];
     for (int64_t i0 = tid - (threadIdx.x & 31); i0 < c; i0 += stride) {
       const int64_t i = i0 + (threadIdx.x & 31);
-      suitor_push(i < c ? (uint32_t)F.list[bb][i].x : kNoPtr, wl, wcnt);
+      suitor_push(i < c ? (uint32_t)F.list[bb].p[i] : kNoPtr, wl, wcnt);
     }
   }
 }

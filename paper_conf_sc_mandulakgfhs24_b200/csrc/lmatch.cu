@@ -314,7 +314,8 @@ struct lmatch_graph {
   // capacities of the buffers sized by the graph's shape (non-empty rows, bins); a reload with a
   // different degree mix grows them and drops the captured CUDA graph
   int64_t cap_noffs = -1, cap_nzr = -1, cap_nlo = -1, cap_S[2] = {-1, -1};
-  int64_t cap_bin[2][lm::kBins] = {{-1, -1, -1, -1, -1}, {-1, -1, -1, -1, -1}};
+  int64_t cap_bin[2][lm::kBins] = {{-1, -1, -1, -1, -1}, {-1, -1, -1, -1, -1}};   // .p arrays
+  int64_t cap_binr[2][lm::kBins] = {{-1, -1, -1, -1, -1}, {-1, -1, -1, -1, -1}};  // .r arrays
   // state
   uint64_t* best = nullptr;
   uint32_t* bits = nullptr;
@@ -852,7 +853,10 @@ int alloc_bins(lmatch_graph* g, cudaStream_t st) {
     for (int b = lm::kDegBins - 2; b >= 0; --b) h[b] += h[b + 1];
   for (int i = 0; i < 2; ++i)
     for (int b = 0; b < lm::kBins; ++b)
-      TRY(ensure(g, &g->F[i].list[b], &g->cap_bin[i][b], (int64_t)h[b] + 1));
+    {
+      TRY(ensure(g, &g->F[i].list[b].p, &g->cap_bin[i][b], (int64_t)h[b] + 1));
+      TRY(ensure(g, &g->F[i].list[b].r, &g->cap_binr[i][b], (int64_t)h[b] + 1));
+    }
   const lm::RoundArgs a = g->rargs();
   CK(cudaMemcpy(g->d_rargs, &a, sizeof a, cudaMemcpyHostToDevice));
   return LMATCH_OK;
@@ -1218,7 +1222,10 @@ void lmatch_destroy(lmatch_graph* g) {
                  g->st_col[0], g->st_col[1], g->st_w[0], g->st_w[1]};
   for (void* p : dev) if (p) cudaFree(p);
   for (auto& F : g->F)
-    for (auto p : F.list) if (p) cudaFree(p);
+    for (auto& l : F.list) {
+      if (l.p) cudaFree(l.p);
+      if (l.r) cudaFree(l.r);
+    }
   if (g->h_counters) cudaFreeHost(g->h_counters);
   if (g->host_adj) cudaFreeHost(g->host_adj);
   for (int i = 0; i < 2; ++i) {
