@@ -513,7 +513,24 @@ __device__ __forceinline__ uint64_t umax_skip(uint64_t b, uint64_t key, uint32_t
 // cached keys) are scanned again.  A row crossing a sweep tile writes its per-tile top-kKC into
 // xpart[tile][slot] (slot 0: the row began before the tile; 1: it continues after it), merged by
 // k_kc_merge.
-constexpr int kKC = 4;
+#ifndef LM_KC
+#define LM_KC 4  // keys per row in the resident key cache (2 or 4; 2 = the row maximum and the next key)
+#endif
+constexpr int kKC = LM_KC;
+static_assert(kKC == 2 || kKC == 4, "key cache width must be 2 or 4");
+// top-2 update of a descending pair (t0 >= t1): branch-free, two u64 max and one u64 min
+__device__ __forceinline__ void top2_insert(uint64_t& t0, uint64_t& t1, uint64_t k) {
+  const uint64_t lo = k < t0 ? k : t0;
+  t1 = lo > t1 ? lo : t1;
+  t0 = k > t0 ? k : t0;
+}
+// merge two descending pairs into the descending top-2 of their union
+__device__ __forceinline__ void top2_merge(uint64_t& t0, uint64_t& t1, uint64_t o0, uint64_t o1) {
+  const uint64_t lo = o0 < t0 ? o0 : t0;
+  const uint64_t hi1 = o1 > t1 ? o1 : t1;
+  t1 = lo > hi1 ? lo : hi1;
+  t0 = o0 > t0 ? o0 : t0;
+}
 // insert key k into the descending list t0 >= t1 >= t2 >= t3 (keeps the kKC largest)
 __device__ __forceinline__ void top4_insert(uint64_t& t0, uint64_t& t1, uint64_t& t2, uint64_t& t3,
                                             uint64_t k) {
@@ -707,17 +724,25 @@ __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
       if (KC && L > 0 && L < LM_SWEEP_LONG) {
         // the row's 4 largest keys (descending); rows wholly in the tile store them in the cache
         uint64_t t0 = 0, t1 = 0, t2 = 0, t3 = 0;
-        for (int j = max(rs, 0), je = min(re, len); j < je; ++j) top4_insert(t0, t1, t2, t3, K[j]);
-        if (inside) {
-          A.best[vid] = t0;
-          ulonglong2* c = reinterpret_cast<ulonglong2*>(A.kc + (size_t)vid * kKC);
-          c[0] = make_ulonglong2(t0, t1);
-          c[1] = make_ulonglong2(t2, t3);
+        if constexpr (kKC == 2) {
+          // two independent top-2 chains, merged
+          uint64_t u0 = 0, u1 = 0;
+          int j = max(rs, 0);
+          const int je = min(re, len);
+          for (; j + 1 < je; j += 2) {
+            top2_insert(t0, t1, K[j]);
+            top2_insert(u0, u1, K[j + 1]);
+          }
+          if (j < je) top2_insert(t0, t1, K[j]);
+          top2_merge(t0, t1, u0, u1);
         } else {
-          ulonglong2* c = reinterpret_cast<ulonglong2*>(A.xpart + ((size_t)t * 2 + (rs < 0 ? 0 : 1)) * kKC);
-          c[0] = make_ulonglong2(t0, t1);
-          c[1] = make_ulonglong2(t2, t3);
+          for (int j = max(rs, 0), je = min(re, len); j < je; ++j) top4_insert(t0, t1, t2, t3, K[j]);
         }
+        ulonglong2* c = inside ? reinterpret_cast<ulonglong2*>(A.kc + (size_t)vid * kKC)
+                               : reinterpret_cast<ulonglong2*>(A.xpart + ((size_t)t * 2 + (rs < 0 ? 0 : 1)) * kKC);
+        if (inside) A.best[vid] = t0;
+        c[0] = make_ulonglong2(t0, t1);
+        if constexpr (kKC == 4) c[1] = make_ulonglong2(t2, t3);
       }
       if (!KC && L > 0 && L < LM_SWEEP_LONG) {
 #endif
@@ -749,9 +774,29 @@ __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
         if (KC) {
           // per-lane top 4 over the lane's keys, then 4 warp-wide pops: lane q < 4 holds the
           // row segment's q-th largest key
-          uint64_t tt[kKC] = {0, 0, 0, 0};
-          for (int j = ja + lane; j < jb; j += 32) top4_insert(tt[0], tt[1], tt[2], tt[3], K[j]);
-          const uint64_t mine = warp_topk_pop<kKC>(tt);
+          uint64_t tt[kKC] = {};
+          uint64_t mine;
+          if constexpr (kKC == 2) {
+            // per-lane top-2 over two chains, then a butterfly top-2 merge; lane q < 2 takes key q
+            uint64_t u0 = 0, u1 = 0;
+            int j = ja + lane;
+            for (; j + 32 < jb; j += 64) {
+              top2_insert(tt[0], tt[1], K[j]);
+              top2_insert(u0, u1, K[j + 32]);
+            }
+            if (j < jb) top2_insert(tt[0], tt[1], K[j]);
+            top2_merge(tt[0], tt[1], u0, u1);
+#pragma unroll
+            for (int o = 16; o; o >>= 1) {
+              const uint64_t o0 = __shfl_xor_sync(0xffffffffu, tt[0], o);
+              const uint64_t o1 = __shfl_xor_sync(0xffffffffu, tt[1], o);
+              top2_merge(tt[0], tt[1], o0, o1);
+            }
+            mine = lane == 0 ? tt[0] : tt[1];
+          } else {
+            for (int j = ja + lane; j < jb; j += 32) top4_insert(tt[0], tt[1], tt[2], tt[3], K[j]);
+            mine = warp_topk_pop<kKC>(tt);
+          }
           const bool rs_neg = __shfl_sync(0xffffffffu, (int)(rs < 0), l) != 0;
           uint64_t* dst = ins ? A.kc + (size_t)v * kKC : A.xpart + ((size_t)t * 2 + (rs_neg ? 0 : 1)) * kKC;
           if (lane < kKC) dst[lane] = mine;
@@ -1051,14 +1096,15 @@ __global__ void k_kc_merge(const int32_t* __restrict__ xrows, const unsigned lon
   for (int64_t i = w0; i < cnt; i += ws) {
     const int64_t r = xrows[i];
     const int64_t tf = noffs[r] / tile, tl = (noffs[r + 1] - 1) / tile;
-    uint64_t t[kKC] = {0, 0, 0, 0};
+    uint64_t t[kKC] = {};
     for (int64_t tt = tf + lane; tt <= tl; tt += 32) {
       const ulonglong2* p = reinterpret_cast<const ulonglong2*>(xpart + ((size_t)tt * 2 + (tt == tf ? 1 : 0)) * kKC);
-      const ulonglong2 a = p[0], b = p[1];
-      topk_insert<kKC>(t, a.x);
-      topk_insert<kKC>(t, a.y);
-      topk_insert<kKC>(t, b.x);
-      topk_insert<kKC>(t, b.y);
+#pragma unroll
+      for (int h = 0; h < kKC / 2; ++h) {
+        const ulonglong2 a = p[h];
+        topk_insert<kKC>(t, a.x);
+        topk_insert<kKC>(t, a.y);
+      }
     }
     const uint64_t mine = warp_topk_pop<kKC>(t);
     const uint32_t u = (uint32_t)nzr[r];
@@ -1523,6 +1569,9 @@ __device__ __forceinline__ uint64_t probe_batch(const uint32_t* __restrict__ bit
 }
 // Two-phase probe of one batch (group-uniform b): lanes probe their top candidate; only keys
 // above the group's best available top are probed in a second step.
+#ifndef LM_PIPE_PROBE3_MIN_G
+#define LM_PIPE_PROBE3_MIN_G 1
+#endif
 #ifndef LM_PIPE_PROBE
 #define LM_PIPE_PROBE 0
 #endif
@@ -1605,15 +1654,15 @@ __device__ __forceinline__ void point_pipe_body(const FL list, int64_t cnt,
       nlast = ls + B >= lend;
       ljb = ls + B;
     }
-#if LM_PIPE_PROBE == 3
-    b = probe_batch2<G, U>(bits, kc, b, gmask);  // group-uniform
+    // LM_PIPE_PROBE == 3: two-phase probing (probe_batch2, group-uniform b) for groups of at
+    // least LM_PIPE_PROBE3_MIN_G lanes; else every candidate of the batch at once
+    constexpr bool two_phase = LM_PIPE_PROBE == 3 && G >= LM_PIPE_PROBE3_MIN_G;
+    if (two_phase)
+      b = probe_batch2<G, U>(bits, kc, b, gmask);
+    else
+      b = probe_batch<U>(bits, kc, b);
     if (clast) {
-      const uint64_t r = b;
-#else
-    b = probe_batch<U>(bits, kc, b);
-    if (clast) {
-      const uint64_t r = G > 1 ? group_max_key(b, gmask) : b;
-#endif
+      const uint64_t r = (G > 1 && !two_phase) ? group_max_key(b, gmask) : b;
       if (gl == 0) {
         best[cu - vbase] = r;
         list.p[ci] = make_pair(cu, r ? (uint32_t)r : kNoPtr);
@@ -1924,8 +1973,13 @@ __host__ __device__ inline CompactIO compact_io(const RoundArgs& a, int cur) {
 __device__ __forceinline__ bool kc_decide(const uint64_t* __restrict__ kc, const uint32_t* __restrict__ bits,
                                           int64_t lu, uint64_t* key) {
   const ulonglong2* c = reinterpret_cast<const ulonglong2*>(kc + (size_t)lu * kKC);
-  const ulonglong2 c01 = c[0], c23 = c[1];
-  const uint64_t k[kKC] = {c01.x, c01.y, c23.x, c23.y};
+  uint64_t k[kKC];
+#pragma unroll
+  for (int h = 0; h < kKC / 2; ++h) {
+    const ulonglong2 a = c[h];
+    k[2 * h] = a.x;
+    k[2 * h + 1] = a.y;
+  }
   uint32_t wd[kKC];
 #pragma unroll
   for (int q = 0; q < kKC; ++q) wd[q] = k[q] ? bits[(uint32_t)k[q] >> 5] : 0xffffffffu;

@@ -13,6 +13,7 @@ p.add_argument("--workload", default="rmat")
 p.add_argument("--scale", type=int, default=26)
 p.add_argument("--runs", type=int, default=1)
 p.add_argument("--round-loop", type=int, default=0)
+p.add_argument("--key-cache", action="store_true")
 a = p.parse_args()
 dev = torch.device("cuda:0")
 torch.cuda.set_device(dev)
@@ -25,7 +26,7 @@ else:
     dg = gg.mesh(side, keep=0.6 if a.workload == "road" else 1.0, seed=1,
                  weights="gradient" if a.workload == "gradient" else "uniform", device=dev)
 stream = torch.cuda.current_stream(dev).cuda_stream
-opts = lm.make_opts(validate_level=1, timing=1, round_loop=a.round_loop)
+opts = lm.make_opts(validate_level=1, timing=1, round_loop=a.round_loop, key_cache=int(a.key_cache))
 h = lm.lmatch_create_device(dg.offsets, dg.col, dg.w, dg.n, dg.m, opts, stream)
 n = dg.n
 dg = None
