@@ -499,6 +499,22 @@ __global__ void k_reset(uint32_t* bits, int64_t nwords, uint64_t* best,
 #define LM_SWEEP_MID 0  // 1 = rows of 8..31 in-tile entries by 8-lane groups (build knob)
 #endif
 __device__ __forceinline__ uint64_t umax64(uint64_t a, uint64_t b) { return a > b ? a : b; }
+// The sweep's key max on the FP64 pipe (LM_SWEEP_DMAX): a packed key float_bits(w) << 32 | col
+// with w > 0 finite (validated at ingest) or 0 is the bit pattern of a non-negative, finite,
+// non-NaN double (exponent field <= 0x7F7), and for such doubles the IEEE order is the unsigned
+// integer order of the bit patterns -- so DSETP + 2 FSEL computes exactly the u64 max, off the
+// integer ALU pipe that bounds the sweep (2 ISETP + 2 SEL per key otherwise).
+#ifndef LM_SWEEP_DMAX
+#define LM_SWEEP_DMAX 1
+#endif
+__device__ __forceinline__ uint64_t kmax64(uint64_t a, uint64_t b) {
+#if LM_SWEEP_DMAX
+  const double x = __longlong_as_double((long long)a), y = __longlong_as_double((long long)b);
+  return (uint64_t)__double_as_longlong(y > x ? y : x);
+#else
+  return a > b ? a : b;
+#endif
+}
 // max(b, key) unless key is the self-loop entry of vertex `self`
 __device__ __forceinline__ uint64_t umax_skip(uint64_t b, uint64_t key, uint32_t self) {
   return ((uint32_t)key != self && key > b) ? key : b;
@@ -708,12 +724,12 @@ __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
         uint64_t b0 = 0, b1 = 0;
         int j = ja + gl;
         for (; j + 8 < jb; j += 16) {
-          b0 = umax64(b0, K[j]);
-          b1 = umax64(b1, K[j + 8]);
+          b0 = kmax64(b0, K[j]);
+          b1 = kmax64(b1, K[j + 8]);
         }
-        if (j < jb) b0 = umax64(b0, K[j]);
+        if (j < jb) b0 = kmax64(b0, K[j]);
         const unsigned gmask = 0xffu << (q * 8);
-        const uint64_t b = group_max_key(umax64(b0, b1), gmask);
+        const uint64_t b = group_max_key(kmax64(b0, b1), gmask);
         if (has && gl == 0) {
           if (ins) A.best[v] = b;
           else if (b) atomicMax(reinterpret_cast<unsigned long long*>(&A.best[v]), (unsigned long long)b);
@@ -750,15 +766,15 @@ __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
         int j = max(rs, 0);
         const int je = min(re, len);
         for (; j + 3 < je; j += 4) {
-          b0 = umax64(b0, K[j]);
-          b1 = umax64(b1, K[j + 1]);
-          b2 = umax64(b2, K[j + 2]);
-          b3 = umax64(b3, K[j + 3]);
+          b0 = kmax64(b0, K[j]);
+          b1 = kmax64(b1, K[j + 1]);
+          b2 = kmax64(b2, K[j + 2]);
+          b3 = kmax64(b3, K[j + 3]);
         }
-        if (j < je) b0 = umax64(b0, K[j]);  // <= 3 left: independent, predicated
-        if (j + 1 < je) b1 = umax64(b1, K[j + 1]);
-        if (j + 2 < je) b2 = umax64(b2, K[j + 2]);
-        const uint64_t b = umax64(umax64(b0, b1), umax64(b2, b3));
+        if (j < je) b0 = kmax64(b0, K[j]);  // <= 3 left: independent, predicated
+        if (j + 1 < je) b1 = kmax64(b1, K[j + 1]);
+        if (j + 2 < je) b2 = kmax64(b2, K[j + 2]);
+        const uint64_t b = kmax64(kmax64(b0, b1), kmax64(b2, b3));
         if (inside) A.best[vid] = b;
         else if (b) atomicMax(reinterpret_cast<unsigned long long*>(&A.best[vid]), (unsigned long long)b);
       }
@@ -806,15 +822,15 @@ __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
         uint64_t b0 = 0, b1 = 0, b2 = 0, b3 = 0;  // 4 independent max chains
         int j = ja + lane;
         for (; j + 96 < jb; j += 128) {
-          b0 = umax64(b0, K[j]);
-          b1 = umax64(b1, K[j + 32]);
-          b2 = umax64(b2, K[j + 64]);
-          b3 = umax64(b3, K[j + 96]);
+          b0 = kmax64(b0, K[j]);
+          b1 = kmax64(b1, K[j + 32]);
+          b2 = kmax64(b2, K[j + 64]);
+          b3 = kmax64(b3, K[j + 96]);
         }
-        if (j < jb) b0 = umax64(b0, K[j]);  // <= 3 steps left: independent, predicated
-        if (j + 32 < jb) b1 = umax64(b1, K[j + 32]);
-        if (j + 64 < jb) b2 = umax64(b2, K[j + 64]);
-        const uint64_t b = group_max_key(umax64(umax64(b0, b1), umax64(b2, b3)), 0xffffffffu);
+        if (j < jb) b0 = kmax64(b0, K[j]);  // <= 3 steps left: independent, predicated
+        if (j + 32 < jb) b1 = kmax64(b1, K[j + 32]);
+        if (j + 64 < jb) b2 = kmax64(b2, K[j + 64]);
+        const uint64_t b = group_max_key(kmax64(kmax64(b0, b1), kmax64(b2, b3)), 0xffffffffu);
         if (lane == 0) {
           if (ins) A.best[v] = b;
           else if (b) atomicMax(reinterpret_cast<unsigned long long*>(&A.best[v]), (unsigned long long)b);
