@@ -515,6 +515,13 @@ __device__ __forceinline__ uint64_t kmax64(uint64_t a, uint64_t b) {
   return a > b ? a : b;
 #endif
 }
+// the same order for the frontier kernels' key compares and selects (LM_FRONT_DMAX): keys held as
+// doubles compare with DSETP and select with FSEL, off the integer ALU pipe
+#ifndef LM_FRONT_DMAX
+#define LM_FRONT_DMAX 0  // measured neutral (the frontier kernels are latency-bound): 11.48 vs 11.48 ms
+#endif
+__device__ __forceinline__ double kd_of(uint64_t k) { return __longlong_as_double((long long)k); }
+__device__ __forceinline__ uint64_t ku_of(double d) { return (uint64_t)__double_as_longlong(d); }
 // max(b, key) unless key is the self-loop entry of vertex `self`
 __device__ __forceinline__ uint64_t umax_skip(uint64_t b, uint64_t key, uint32_t self) {
   return ((uint32_t)key != self && key > b) ? key : b;
@@ -1329,7 +1336,13 @@ __device__ __forceinline__ uint64_t scan_row_available_t(const AdjView adj,
     {
       uint64_t mx = 0;
 #pragma unroll
-#if LM_MAX1
+#if LM_FRONT_DMAX
+      {
+        double m = 0.0;
+        for (int q = 0; q < U; ++q) m = kd_of(k[q]) > m ? kd_of(k[q]) : m;
+        mx = m > kd_of(b) ? ku_of(m) : 0ull;
+      }
+#elif LM_MAX1
       for (int q = 0; q < U; ++q) mx = umax64(mx, k[q]);
       if (mx <= b) mx = 0;
 #else
@@ -1364,6 +1377,18 @@ __device__ __forceinline__ uint64_t scan_row_available_t(const AdjView adj,
     }
     } else {
       uint32_t wd[U];
+#if LM_FRONT_DMAX
+      double bd = kd_of(b);
+#pragma unroll
+      for (int q = 0; q < U; ++q) wd[q] = kd_of(k[q]) > bd ? probe_word(bits, (uint32_t)k[q]) : 0xffffffffu;
+#pragma unroll
+      for (int q = 0; q < U; ++q) {
+        const uint32_t v = (uint32_t)k[q];
+        const double kd = kd_of(k[q]);
+        bd = (!((wd[q] >> (v & 31)) & 1u) && kd > bd) ? kd : bd;
+      }
+      b = ku_of(bd);
+#else
 #pragma unroll
       for (int q = 0; q < U; ++q) wd[q] = k[q] > b ? probe_word(bits, (uint32_t)k[q]) : 0xffffffffu;
 #pragma unroll
@@ -1371,6 +1396,7 @@ __device__ __forceinline__ uint64_t scan_row_available_t(const AdjView adj,
         const uint32_t v = (uint32_t)k[q];
         if (!((wd[q] >> (v & 31)) & 1u) && k[q] > b) b = k[q];
       }
+#endif
     }
 #elif LM_PROBE == 1
     // descending: probe the lane's largest candidate, drop it if matched, repeat
@@ -1574,6 +1600,18 @@ template <int U>
 __device__ __forceinline__ uint64_t probe_batch(const uint32_t* __restrict__ bits,
                                                 const uint64_t (&k)[U], uint64_t b) {
   uint32_t wd[U];
+#if LM_FRONT_DMAX
+  double bd = kd_of(b);
+#pragma unroll
+  for (int q = 0; q < U; ++q) wd[q] = kd_of(k[q]) > bd ? probe_word(bits, (uint32_t)k[q]) : 0xffffffffu;
+#pragma unroll
+  for (int q = 0; q < U; ++q) {
+    const uint32_t v = (uint32_t)k[q];
+    const double kd = kd_of(k[q]);
+    bd = (!((wd[q] >> (v & 31)) & 1u) && kd > bd) ? kd : bd;
+  }
+  return ku_of(bd);
+#else
 #pragma unroll
   for (int q = 0; q < U; ++q) wd[q] = k[q] > b ? probe_word(bits, (uint32_t)k[q]) : 0xffffffffu;
 #pragma unroll
@@ -1582,6 +1620,7 @@ __device__ __forceinline__ uint64_t probe_batch(const uint32_t* __restrict__ bit
     if (!((wd[q] >> (v & 31)) & 1u) && k[q] > b) b = k[q];
   }
   return b;
+#endif
 }
 // Two-phase probe of one batch (group-uniform b): lanes probe their top candidate; only keys
 // above the group's best available top are probed in a second step.

@@ -1,6 +1,7 @@
 # Round-2 final measurements (builder tooling; GPU box).  Everything lands in gpurun_out/r02f/.
 set -x
 O=gpurun_out/r02f; mkdir -p $O
+timeout 2400 python -m pytest tests -m gpu -q 2>&1 | tail -5 > $O/gpu_tests.txt
 python bench.py > $O/bench_rmat_s26.json 2> $O/bench_rmat_s26.err
 python bench.py --impl reference > $O/bench_reference.json 2> $O/bench_reference.err
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $O/launches_rmat_s26.csv \
