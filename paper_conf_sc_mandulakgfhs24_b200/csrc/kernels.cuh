@@ -1896,8 +1896,14 @@ __global__ void __launch_bounds__(THREADS)
 // =============================================================================================
 // Round 1: every vertex; the warp owning 32 consecutive vertices writes their bitmap word.
 // Each warp owns 4 bitmap words per step and issues the 4 random best[ptr u] reads together.
+#ifndef LM_MATCHALL_HALF
+#define LM_MATCHALL_HALF 1  // round-1 match: mutual pairs checked from their smaller endpoint only
+#endif
+#ifndef LM_MATCHALL_V
+#define LM_MATCHALL_V 4  // bitmap words per warp step (independent best[ptr u] gathers per lane)
+#endif
 __global__ void k_match_all(const uint64_t* __restrict__ best, int64_t n, uint32_t* bits) {
-  constexpr int V = 4;
+  constexpr int V = LM_MATCHALL_V;
   const int64_t nwords = (n + 31) >> 5;
   const int lane = threadIdx.x & 31;
   const int64_t w0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -1909,6 +1915,28 @@ __global__ void k_match_all(const uint64_t* __restrict__ best, int64_t n, uint32
       const int64_t u = ((wb + q * ws) << 5) + lane;
       b[q] = (wb + q * ws < nwords && u < n) ? best[u] : 0ull;
     }
+#if LM_MATCHALL_HALF
+    // a mutual pair is found by its smaller endpoint only: u reads best[v] only when v > u, so
+    // the random gathers (the kernel's cost) halve; that endpoint marks both (bits zeroed by
+    // k_reset, so every mark is an atomicOr)
+#pragma unroll
+    for (int q = 0; q < V; ++q) {
+      const int64_t u = ((wb + q * ws) << 5) + lane;
+      bv[q] = (b[q] && (int64_t)(uint32_t)b[q] > u) ? best[(uint32_t)b[q]] : 0ull;
+    }
+#pragma unroll
+    for (int q = 0; q < V; ++q) {
+      const int64_t wi = wb + q * ws;
+      const int64_t u = (wi << 5) + lane;
+      const bool mutual = bv[q] != 0 && (uint32_t)bv[q] == (uint32_t)u;
+      const unsigned word = __ballot_sync(0xffffffffu, mutual);
+      if (lane == 0 && wi < nwords && word) atomicOr(&bits[wi], word);
+      if (mutual) {
+        const uint32_t v = (uint32_t)b[q];
+        atomicOr(&bits[v >> 5], 1u << (v & 31));
+      }
+    }
+#else
 #pragma unroll
     for (int q = 0; q < V; ++q) bv[q] = b[q] ? best[(uint32_t)b[q]] : 0ull;
 #pragma unroll
@@ -1919,6 +1947,7 @@ __global__ void k_match_all(const uint64_t* __restrict__ best, int64_t n, uint32
       const unsigned word = __ballot_sync(0xffffffffu, mutual);
       if (lane == 0 && wi < nwords) bits[wi] = word;
     }
+#endif
   }
 }
 

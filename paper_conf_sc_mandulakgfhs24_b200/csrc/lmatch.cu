@@ -1399,7 +1399,7 @@ static int seq_prefix(lmatch_graph* g, cudaStream_t st, cudaGraphConditionalHand
   // round 1: A2 full sweep (no bitmap test), A4 match-all, A6 compact-all
   TRY(round1_sweep(g, st, launches, sweep_launches, bytes_streamed));
   TRY(mark(2));
-  lm::k_match_all<<<grid_for(nwords * 32, 256, 65536), 256, 0, st>>>(g->best, n, g->bits);
+  lm::k_match_all<<<grid_for((nwords + LM_MATCHALL_V - 1) / LM_MATCHALL_V * 32, 256, 65536), 256, 0, st>>>(g->best, n, g->bits);
   CKL();
   // round-1 compaction: input set 1 (unused), output set 0; k_end_round makes set 0 current.
   // Items are the non-empty rows (nzr): empty rows never hold a pointer.
