@@ -2806,12 +2806,29 @@ __global__ void k_match_part_all(const uint64_t* __restrict__ best, int64_t n_lo
   for (int64_t wi = w0; wi < nwords; wi += ws) {
     const int64_t i = (wi << 5) + lane;
     bool mutual = false;
+#if LM_MATCHALL_HALF
+    // as k_match_all: a pair with both ends in this part is checked from its smaller end, which
+    // marks both (atomicOr; the owned words were zeroed by k_reset); a remote target is checked
+    // here, its own part marks it
+    uint32_t v = 0;
+    if (i < n_loc) {
+      const uint64_t b = best[i];
+      v = (uint32_t)b;
+      const bool local = (int64_t)v >= vbase && (int64_t)v < vend;
+      if (b && (!local || (int64_t)v > i + vbase))
+        mutual = ptr_of(best, ghost, vbase, vend, v) == (uint32_t)(i + vbase);
+    }
+    const unsigned word = __ballot_sync(0xffffffffu, mutual);
+    if (lane == 0 && word) atomicOr(&bits[(vbase >> 5) + wi], word);
+    if (mutual && (int64_t)v >= vbase && (int64_t)v < vend) atomicOr(&bits[v >> 5], 1u << (v & 31));
+#else
     if (i < n_loc) {
       const uint64_t b = best[i];
       if (b) mutual = ptr_of(best, ghost, vbase, vend, (uint32_t)b) == (uint32_t)(i + vbase);
     }
     const unsigned word = __ballot_sync(0xffffffffu, mutual);
     if (lane == 0) bits[(vbase >> 5) + wi] = word;
+#endif
   }
 }
 // rounds >= 2 match over the re-pointed frontier
