@@ -237,6 +237,8 @@ struct lmatch_graph {
   float part_sweep_ms = 0.f;  // (timing=1) last lmatch_part_begin's round-1 sweep
   bool sweep_ms_pending = false;  // its events are recorded, the time not read yet
   bool counts_on_host = false;    // peer-memory round: h_counters holds this set's bin sizes
+  bool one_rank_loop = false;     // lmatch_run_dist with P = 1: h_counters is read back after every
+                                  // compaction, so match and compaction launches are sized from it
   int validate_level = 1;
   int timing = 0;
   int64_t max_rounds = 0;
@@ -2359,7 +2361,7 @@ static int part_compact_launch(lmatch_graph* g, cudaStream_t st) {
     int64_t nF = 0;
     for (int b = 0; b < lm::kBins; ++b) nF += (int64_t)g->h_counters[lm::cnt_F(cur, b)];
     if (g->p2p || nS + nF > 0) {
-      const unsigned grid = g->p2p ? (unsigned)(4 * g->num_sms)
+      const unsigned grid = (g->p2p && !g->one_rank_loop) ? (unsigned)(4 * g->num_sms)
                                    : grid_for((nS + nF + 31) / 32, 8 * kCompactK, 65536);
       const lm::CompactIO io = lm::compact_io(g->rargs(), cur);
       if (g->kcache)
@@ -2669,7 +2671,25 @@ int lmatch_p2p_match(lmatch_graph* g, void* stream) {
     lm::k_apply_inbox<<<(unsigned)grid, 256, 0, st>>>(g->win, g->win_cap, icnt, P, g->ghost);
     CKL();
   }
-  if (g->part_round == 1) {
+  if (g->one_rank_loop) {
+    // one part (v0 = 0, no ghosts): the single-graph match kernels, sized from the host counts
+    if (g->part_round == 1) {
+      const int64_t nwords = (g->n + 31) / 32;
+      if (g->n > 0) {
+        lm::k_match_all<<<grid_for((nwords + LM_MATCHALL_V - 1) / LM_MATCHALL_V * 32, 256, 65536), 256, 0, st>>>(
+            g->best, g->n, g->bits);
+        CKL();
+      }
+    } else {
+      int64_t nF = 0;
+      for (int b = 0; b < lm::kBins; ++b) nF += (int64_t)g->h_counters[lm::cnt_F(g->part_cur, b)];
+      if (nF > 0) {
+        lm::k_match_bins<<<grid_for((nF + LM_MATCH_V - 1) / LM_MATCH_V, 256, 65536), 256, 0, st>>>(
+            g->F[g->part_cur], g->counters + lm::cnt_F(g->part_cur, 0), g->best, g->bits);
+        CKL();
+      }
+    }
+  } else if (g->part_round == 1) {
     if (g->n > 0) {
       lm::k_match_part_all<<<grid_for(((g->n + 31) / 32) * 32, 256, 65536), 256, 0, st>>>(
           g->best, g->n, g->v0, g->v0 + g->n, g->ghost, g->bits);
@@ -3104,8 +3124,13 @@ int lmatch_run_dist_device(lmatch_graph* g, int32_t* d_mate_local, void* stream,
   bool compacted = false, capped = false;
   if (P == 1) {
     // one rank: nothing to exchange, so the round loop is the single-GPU one -- the frontier
-    // size read after each compaction sizes the next pointer launches exactly, and the small
-    // tail runs in the persistent cooperative kernel (no host round trips)
+    // size read after each compaction sizes the next match, compaction and pointer launches
+    // exactly, and the small tail runs in the persistent cooperative kernel (no host round trips)
+    g->one_rank_loop = g->v0 == 0 && g->n_global == g->n;
+    struct Off {
+      lmatch_graph* g;
+      ~Off() { g->one_rank_loop = false; }
+    } off{g};
     for (;;) {
       TRY(lmatch_p2p_match(g, st));
       TRY(lmatch_p2p_compact(g, st, nullptr));
