@@ -2837,16 +2837,31 @@ __global__ void k_match_part_bins(Bins F, const unsigned long long* cntF,
                                   const uint32_t* __restrict__ ghost, uint32_t* bits) {
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  // LM_MATCH_V entries per thread step with their dependent loads batched, as match_bins_body
+  constexpr int V = LM_MATCH_V;
 #pragma unroll
   for (int bb = 0; bb < kBins; ++bb) {
     const int64_t c = (int64_t)cntF[bb];
-    for (int64_t i = tid; i < c; i += stride) {
-      const uint64_t p = F.list[bb].p[i];
-      const uint32_t u = (uint32_t)p, v = (uint32_t)(p >> 32);
-      if (v == kNoPtr) continue;
-      if (ptr_of(best, ghost, vbase, vend, v) == u) {
-        atomicOr(&bits[u >> 5], 1u << (u & 31));
-        if ((int64_t)v >= vbase && (int64_t)v < vend) atomicOr(&bits[v >> 5], 1u << (v & 31));
+    for (int64_t i0 = tid; i0 < c; i0 += V * stride) {
+      uint64_t p[V];
+      uint32_t pv[V];
+#pragma unroll
+      for (int q = 0; q < V; ++q) {
+        const int64_t i = i0 + q * stride;
+        p[q] = i < c ? F.list[bb].p[i] : ((uint64_t)kNoPtr << 32);
+      }
+#pragma unroll
+      for (int q = 0; q < V; ++q) {
+        const uint32_t v = (uint32_t)(p[q] >> 32);
+        pv[q] = v != kNoPtr ? ptr_of(best, ghost, vbase, vend, v) : kNoPtr;
+      }
+#pragma unroll
+      for (int q = 0; q < V; ++q) {
+        const uint32_t u = (uint32_t)p[q], v = (uint32_t)(p[q] >> 32);
+        if (v != kNoPtr && pv[q] == u) {
+          atomicOr(&bits[u >> 5], 1u << (u & 31));
+          if ((int64_t)v >= vbase && (int64_t)v < vend) atomicOr(&bits[v >> 5], 1u << (v & 31));
+        }
       }
     }
   }

@@ -696,3 +696,28 @@ def test_sorted_rejects_out_of_core(lm):
     with lm.Matcher(g, algorithm="sorted", hbm_budget_bytes=8 * g.m // 2, stream_chunk=1024) as M:
         with pytest.raises(lm.LMatchError):
             M.run()
+
+
+def test_extreme_weights_key_order(lm):
+    """Float subnormal, smallest-normal and near-FLT_MAX weights mixed with ordinary ones, in a
+    hub row that spans several sweep tiles, warp-reduced rows and lane-reduced rows: the sweep's
+    FP64-pipe key max (kmax64) must order them exactly as the u64 keys."""
+    rng = np.random.default_rng(17)
+    fi = np.finfo(np.float32)
+    pool = np.array([fi.smallest_subnormal, 3 * fi.smallest_subnormal, 1e-40, fi.tiny, 2 * fi.tiny,
+                     1e-30, 0.001, 0.5, 0.999, 1.0, 7.0, 1e30, fi.max / 2, fi.max], dtype=np.float32)
+    n = 4000
+    edges = [(0, v, float(pool[v % len(pool)])) for v in range(1, 1800)]       # hub: > 3 tiles
+    for u in range(1800, 2400):                                                 # 40-entry rows
+        for d in range(1, 21):
+            edges.append((u, 1800 + (u - 1800 + 37 * d) % 600, float(pool[rng.integers(len(pool))])))
+    for _ in range(6000):                                                       # short rows
+        u, v = rng.integers(2400, n, size=2)
+        edges.append((int(u), int(v), float(pool[rng.integers(len(pool))])))
+    uniq = {}
+    for u, v, w in edges:
+        if u != v:
+            uniq.setdefault((min(u, v), max(u, v)), w)   # a simple graph: one weight per edge
+    g = graphgen.from_edges(n, [(u, v, w) for (u, v), w in uniq.items()])
+    check_parity(lm, g)
+    check_parity(lm, g, round_loop=1)
