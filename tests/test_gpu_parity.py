@@ -721,3 +721,33 @@ def test_extreme_weights_key_order(lm):
     g = graphgen.from_edges(n, [(u, v, w) for (u, v), w in uniq.items()])
     check_parity(lm, g)
     check_parity(lm, g, round_loop=1)
+
+
+@pytest.mark.parametrize("kw", [dict(), dict(round_loop=1), dict(round_loop=2), dict(algorithm="hybrid"),
+                                dict(algorithm="suitor")])
+def test_crossing_rows_repeat_runs(lm, kw):
+    """Tile-crossing rows merge their partial maxima into best[] with atomicMax, and best[] is not
+    re-zeroed between runs (LM_XROW_RESET = 0): a run starts from the previous run's final
+    pointers, each 0 or a key of the vertex's own row.  Overlapping hubs spanning several tiles
+    (their final pointers far below their maxima) and random short rows, every round-loop mode and
+    algorithm that runs the sweep: every one of three runs on one handle equals the oracle."""
+    rng = np.random.default_rng(21)
+    n = 12000
+    edges = []
+    for h, (lo, hi) in enumerate([(50, 4050), (2000, 7000), (6000, 11990)]):
+        for v in range(lo, hi):
+            edges.append((h, v, float(np.float32(rng.random() * 0.9 + 0.05))))
+    for _ in range(20000):
+        u, v = rng.integers(3, n, size=2)
+        if u != v:
+            edges.append((int(u), int(v), float(np.float32(rng.random()))))
+    uniq = {}
+    for u, v, w in edges:
+        uniq.setdefault((min(u, v), max(u, v)), w)
+    g = graphgen.from_edges(n, [(u, v, w) for (u, v), w in uniq.items()])
+    ref = oracle.greedy(g)
+    with lm.Matcher(g, **kw) as M:
+        for _ in range(3):
+            mate, st = M.run()
+            np.testing.assert_array_equal(mate, ref.mate)
+            assert math.isclose(st["weight"], ref.weight, rel_tol=WTOL)
