@@ -1231,6 +1231,9 @@ struct RoundArgs {
 #define LM_PROBE 3  // bitmap probes per batch: 0 = all candidates in parallel, 1 = descending, 2 = top first,
                     // 3 = two-phase (lane tops, then only keys above the group's best)
 #endif
+#ifndef LM_R1_NOFFS
+#define LM_R1_NOFFS 1  // round-1 compaction reads frontier rows' ranges from noffs (item order)
+#endif
 #ifndef LM_MATCH_V
 #define LM_MATCH_V 4  // frontier entries per thread step in the match, loads batched (1 -> 4: -0.4%)
 #endif
@@ -2030,6 +2033,7 @@ struct CompactIO {
   const uint32_t* live;           // A7: live counts (nullptr = pruning off)
   const RoundState* st;
   const int32_t* nzr;             // ALL mode: iterate the non-empty rows only (nullptr = all n)
+  const int64_t* noffs = nullptr; // ALL mode with nzr: the non-empty rows' offsets (LM_R1_NOFFS)
   const uint64_t* kc;             // key cache [n][kKC] (nullptr = off)
   uint64_t* best_w;               // key cache: pointers decided by the compaction (= best)
 };
@@ -2045,6 +2049,7 @@ __host__ __device__ inline CompactIO compact_io(const RoundArgs& a, int cur) {
   io.live = a.live;
   io.st = a.st;
   io.nzr = nullptr;
+  io.noffs = nullptr;
   io.kc = a.kc;
   io.best_w = a.best;
   return io;
@@ -2149,8 +2154,18 @@ __device__ __forceinline__ void compact_body_plain(const CompactIO& io, int64_t 
       const bool tgt = (wv[k] >> (v & 31)) & 1u;
       if (live && !tgt) sbits |= 1u << k;
       const bool fr = live && tgt;
-      os[k] = fr ? offs[u - vbase] : 0;
-      oe[k] = fr ? offs[u - vbase + 1] : -1;
+#if LM_R1_NOFFS
+      // round 1 over the non-empty rows: row i's range is noffs[i], noffs[i+1] (item order)
+      if (ALL && io.noffs) {
+        const int64_t i = c0 + 32 * k + lane;
+        os[k] = fr ? io.noffs[i] : 0;
+        oe[k] = fr ? io.noffs[i + 1] : -1;
+      } else
+#endif
+      {
+        os[k] = fr ? offs[u - vbase] : 0;
+        oe[k] = fr ? offs[u - vbase + 1] : -1;
+      }
       if (lcnt && fr) {  // A7: a row pruned earlier in this run is scanned over its live prefix
         const uint32_t x = lcnt[u - vbase];
         if ((x >> 16) == tag) oe[k] = os[k] + (int64_t)(x & 0xffffu);

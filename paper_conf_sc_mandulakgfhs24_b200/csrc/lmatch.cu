@@ -102,7 +102,10 @@ using Sweep = lm::SweepCfg<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap>;
 #define SWEEP_KERNEL_KC lm::k_sweep<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap, false, true>
 constexpr int kSweepThreads = Sweep::kThreads;
 constexpr int64_t kTile = Sweep::kTile;
-constexpr int kCompactK = 8;  // items per lane per compaction chunk
+#ifndef LM_COMPACT_K
+#define LM_COMPACT_K 8
+#endif
+constexpr int kCompactK = LM_COMPACT_K;  // items per lane per compaction chunk
 constexpr long long kLogCap = 1 << 16;  // per-round log rows kept on the device
 // hybrid round loop: frontiers up to this size run in the persistent kernel
 #ifndef LM_PERSIST_BELOW
@@ -1418,6 +1421,7 @@ static int seq_prefix(lmatch_graph* g, cudaStream_t st, cudaGraphConditionalHand
   {
     lm::CompactIO io = lm::compact_io(g->rargs(), 1);
     io.nzr = g->nzr;
+    io.noffs = g->noffs;
     const unsigned grid = grid_for((g->n_nz + 31) / 32, 8 * kCompactK, 65536);
     if (g->kcache)
       lm::k_compact<true, kCompactK, true><<<grid, 256, 0, st>>>(io, g->n_nz, g->best, g->bits, g->offs, g->v0);
@@ -2357,6 +2361,7 @@ static int part_compact_launch(lmatch_graph* g, cudaStream_t st) {
       const unsigned grid = grid_for((g->n_nz + 31) / 32, 8 * kCompactK, 65536);
       lm::CompactIO io = lm::compact_io(g->rargs(), 1);
       io.nzr = g->nzr;
+      io.noffs = g->noffs;
       if (g->kcache)
         lm::k_compact<true, kCompactK, true><<<grid, 256, 0, st>>>(io, g->n_nz, g->best, g->bits, g->offs, g->v0);
       else
