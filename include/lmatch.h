@@ -85,7 +85,8 @@ typedef struct lmatch_opts {
                               must repeat the same weight (exact: every row is sorted by
                               (v, weight bits) in scratch memory, in chunks of <= 2^27 entries,
                               and neighbouring entries are compared);
-                              -1 = skip validation (caller guarantees a valid CSR) */
+                              -1 = skip validation (caller guarantees a valid CSR, including
+                              weights finite and > 0: the sweep's key max relies on it) */
   int32_t timing;          /* 1 = record CUDA events per phase into lmatch_stats */
   int64_t max_rounds;      /* 0 = default: n/2 + 2 (the strict order bounds rounds by n/2+1).
                               A smaller cap that stops the iteration with a non-empty frontier
