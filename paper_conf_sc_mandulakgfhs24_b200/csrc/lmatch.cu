@@ -106,6 +106,10 @@ constexpr int64_t kTile = Sweep::kTile;
 #define LM_COMPACT_K 8
 #endif
 constexpr int kCompactK = LM_COMPACT_K;  // items per lane per compaction chunk
+#ifndef LM_COMPACT_K1
+#define LM_COMPACT_K1 4  // the round-1 compaction (every non-empty row): 4 items per lane measured
+#endif               // 0.646 vs 0.665 ms for round-1 match + compaction; later rounds keep 8
+constexpr int kCompactK1 = LM_COMPACT_K1;
 constexpr long long kLogCap = 1 << 16;  // per-round log rows kept on the device
 // hybrid round loop: frontiers up to this size run in the persistent kernel
 #ifndef LM_PERSIST_BELOW
@@ -1422,11 +1426,11 @@ static int seq_prefix(lmatch_graph* g, cudaStream_t st, cudaGraphConditionalHand
     lm::CompactIO io = lm::compact_io(g->rargs(), 1);
     io.nzr = g->nzr;
     io.noffs = g->noffs;
-    const unsigned grid = grid_for((g->n_nz + 31) / 32, 8 * kCompactK, 65536);
+    const unsigned grid = grid_for((g->n_nz + 31) / 32, 8 * kCompactK1, 65536);
     if (g->kcache)
-      lm::k_compact<true, kCompactK, true><<<grid, 256, 0, st>>>(io, g->n_nz, g->best, g->bits, g->offs, g->v0);
+      lm::k_compact<true, kCompactK1, true><<<grid, 256, 0, st>>>(io, g->n_nz, g->best, g->bits, g->offs, g->v0);
     else
-      lm::k_compact<true, kCompactK, false><<<grid, 256, 0, st>>>(io, g->n_nz, g->best, g->bits, g->offs, g->v0);
+      lm::k_compact<true, kCompactK1, false><<<grid, 256, 0, st>>>(io, g->n_nz, g->best, g->bits, g->offs, g->v0);
   }
   CKL();
   lm::k_end_round<<<1, 32, 0, st>>>(g->ra(), h, in_graph, 0);
@@ -2358,14 +2362,14 @@ static int part_compact_launch(lmatch_graph* g, cudaStream_t st) {
   if (g->part_round == 1) {
     if (n > 0) {
       // items are the non-empty rows (nzr): empty rows never hold a pointer
-      const unsigned grid = grid_for((g->n_nz + 31) / 32, 8 * kCompactK, 65536);
+      const unsigned grid = grid_for((g->n_nz + 31) / 32, 8 * kCompactK1, 65536);
       lm::CompactIO io = lm::compact_io(g->rargs(), 1);
       io.nzr = g->nzr;
       io.noffs = g->noffs;
       if (g->kcache)
-        lm::k_compact<true, kCompactK, true><<<grid, 256, 0, st>>>(io, g->n_nz, g->best, g->bits, g->offs, g->v0);
+        lm::k_compact<true, kCompactK1, true><<<grid, 256, 0, st>>>(io, g->n_nz, g->best, g->bits, g->offs, g->v0);
       else
-        lm::k_compact<true, kCompactK, false><<<grid, 256, 0, st>>>(io, g->n_nz, g->best, g->bits, g->offs, g->v0);
+        lm::k_compact<true, kCompactK1, false><<<grid, 256, 0, st>>>(io, g->n_nz, g->best, g->bits, g->offs, g->v0);
       CKL();
     }
     g->part_cur = 0;
