@@ -495,6 +495,12 @@ __global__ void k_reset(uint32_t* bits, int64_t nwords, uint64_t* best,
 #ifndef LM_SWEEP_LONG
 #define LM_SWEEP_LONG 32  // in-tile rows with at least this many entries are reduced by the warp
 #endif
+#ifndef LM_SWEEP_WCHAINS
+#define LM_SWEEP_WCHAINS 4  // independent max chains per lane of a warp-reduced (long) row: 4 or 2
+#endif
+#ifndef LM_SWEEP_LCHAINS
+#define LM_SWEEP_LCHAINS 2  // independent max chains of a lane-reduced (short) row: 2 (measured 2.98 vs 3.00 ms) or 4
+#endif
 #ifndef LM_SWEEP_MID
 #define LM_SWEEP_MID 0  // 1 = rows of 8..31 in-tile entries by 8-lane groups (build knob)
 #endif
@@ -769,6 +775,17 @@ __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
       }
       if (!KC && L > 0 && L < LM_SWEEP_LONG) {
 #endif
+#if LM_SWEEP_LCHAINS == 2
+        uint64_t b0 = 0, b1 = 0;  // 2 independent max chains (short rows: less tail and combine)
+        int j = max(rs, 0);
+        const int je = min(re, len);
+        for (; j + 1 < je; j += 2) {
+          b0 = kmax64(b0, K[j]);
+          b1 = kmax64(b1, K[j + 1]);
+        }
+        if (j < je) b0 = kmax64(b0, K[j]);
+        const uint64_t b = kmax64(b0, b1);
+#else
         uint64_t b0 = 0, b1 = 0, b2 = 0, b3 = 0;  // 4 independent max chains
         int j = max(rs, 0);
         const int je = min(re, len);
@@ -782,6 +799,7 @@ __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
         if (j + 1 < je) b1 = kmax64(b1, K[j + 1]);
         if (j + 2 < je) b2 = kmax64(b2, K[j + 2]);
         const uint64_t b = kmax64(kmax64(b0, b1), kmax64(b2, b3));
+#endif
         if (inside) A.best[vid] = b;
         else if (b) atomicMax(reinterpret_cast<unsigned long long*>(&A.best[vid]), (unsigned long long)b);
       }
@@ -826,6 +844,16 @@ __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
           if (ins && lane == 0) A.best[v] = mine;
           continue;
         }
+#if LM_SWEEP_WCHAINS == 2
+        uint64_t b0 = 0, b1 = 0;  // 2 independent max chains per lane
+        int j = ja + lane;
+        for (; j + 32 < jb; j += 64) {
+          b0 = kmax64(b0, K[j]);
+          b1 = kmax64(b1, K[j + 32]);
+        }
+        if (j < jb) b0 = kmax64(b0, K[j]);
+        const uint64_t b = group_max_key(kmax64(b0, b1), 0xffffffffu);
+#else
         uint64_t b0 = 0, b1 = 0, b2 = 0, b3 = 0;  // 4 independent max chains
         int j = ja + lane;
         for (; j + 96 < jb; j += 128) {
@@ -838,6 +866,7 @@ __global__ void __launch_bounds__(32 * WARPS) k_sweep(SweepArgs A) {
         if (j + 32 < jb) b1 = kmax64(b1, K[j + 32]);
         if (j + 64 < jb) b2 = kmax64(b2, K[j + 64]);
         const uint64_t b = group_max_key(kmax64(kmax64(b0, b1), kmax64(b2, b3)), 0xffffffffu);
+#endif
         if (lane == 0) {
           if (ins) A.best[v] = b;
           else if (b) atomicMax(reinterpret_cast<unsigned long long*>(&A.best[v]), (unsigned long long)b);
