@@ -480,7 +480,9 @@ def run_partitioned(a, rank, world, local, dev):
     allr = allgather(mine)
     worst = max(allr, key=lambda x: x[0])
     peak, peak_src = load_peaks()
-    ntiles_w = (worst[1] + 511) // 512
+    mine_tile = lm.lmatch_sweep_tile(getattr(part, "h", None))
+    tile_w = int(allgather([mine_tile])[allr.index(worst)][0])
+    ntiles_w = (worst[1] + tile_w - 1) // tile_w
     sweep_bytes = 8 * worst[1] + 16 * worst[2] + 4 * (ntiles_w + 1)
     achieved = sweep_bytes / (worst[0] / 1e3) / 1e9 if worst[0] > 0 else None
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",

@@ -229,6 +229,10 @@ LMATCH_API int lmatch_abi_version(void);
 /* Kernels this library has launched in this process so far (all handles; a captured CUDA graph
  * counts its launches once, at capture).  Callers take differences around a region. */
 LMATCH_API int64_t lmatch_kernel_launch_count(void);
+/* Adjacency entries per round-1 sweep tile of handle g (the configuration follows the average
+ * degree; NULL: the dense configuration's tile).  The sweep reads one 4-byte tile index entry per
+ * tile: the tile term of its algorithmic bytes, DESIGN.md section 7. */
+LMATCH_API int32_t lmatch_sweep_tile(const lmatch_graph* g);
 
 /* Build a handle from HOST CSR arrays (copied to the device in chunks, packed into 64-bit
  * (weight-bits << 32 | neighbour) keys, validated, and indexed for the round-1 sweep).

@@ -21,7 +21,7 @@ __all__ = [
     "lmatch_abi_version", "lmatch_create", "lmatch_create_ex", "lmatch_create_device",
     "lmatch_reload", "lmatch_run", "lmatch_run_device", "lmatch_weight", "lmatch_weight_device",
     "lmatch_info", "lmatch_round_log", "lmatch_round_ms", "lmatch_destroy", "lmatch_strerror",
-    "lmatch_last_error",
+    "lmatch_last_error", "lmatch_sweep_tile",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -90,6 +90,7 @@ _sig = {
     "lmatch_round_ms": ([_P, _P, _I64, ctypes.POINTER(_I64), ctypes.POINTER(_I64)], ctypes.c_int),
     "lmatch_push_rounds": ([_P, ctypes.POINTER(_I64)], ctypes.c_int),
     "lmatch_destroy": ([_P], None),
+    "lmatch_sweep_tile": ([_P], ctypes.c_int32),
     "lmatch_strerror": ([ctypes.c_int], ctypes.c_char_p),
     "lmatch_last_error": ([], ctypes.c_char_p),
 }
@@ -137,6 +138,11 @@ def _stream_ptr(stream):
 # ------------------------------------------------------------------------ C-named wrappers
 def lmatch_abi_version() -> int:
     return int(_lib.lmatch_abi_version())
+
+
+def lmatch_sweep_tile(h=None) -> int:
+    """Adjacency entries per round-1 sweep tile of handle h (None: the dense configuration's)."""
+    return int(_lib.lmatch_sweep_tile(h))
 
 
 def lmatch_strerror(status: int) -> str:
@@ -224,7 +230,8 @@ def lmatch_info(h: int) -> dict:
     n, m, nz, db = _I64(), _I64(), _I64(), _I64()
     _check(_lib.lmatch_info(h, ctypes.byref(n), ctypes.byref(m), ctypes.byref(nz),
                             ctypes.byref(db)), "lmatch_info")
-    return dict(n=n.value, m=m.value, nonempty_rows=nz.value, device_bytes=db.value)
+    return dict(n=n.value, m=m.value, nonempty_rows=nz.value, device_bytes=db.value,
+                sweep_tile=int(_lib.lmatch_sweep_tile(h)))
 
 
 def lmatch_round_log(h: int) -> np.ndarray:

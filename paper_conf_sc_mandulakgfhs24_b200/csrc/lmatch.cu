@@ -71,18 +71,36 @@ static inline void count_launches(long long k) {
     if (s_ != LMATCH_OK) return s_; \
   } while (0)
 
-// Round-1 sweep configuration (tuned on B200).
+// Round-1 sweep configurations (tuned on B200), chosen per handle by the
+// average degree.  Round 2, after the key max moved to the FP64 pipe, the per-tile TMA issue and
+// row-window work became the larger share of the sweep's instructions: for graphs with average
+// degree >= LM_SWEEP_DENSE_DEG, 1024-entry tiles, 6 warps per CTA (2 CTAs = 12 warps per SM) and a
+// 104-row window measured 2.88 ms against 2.99 ms for 512 / 8 / 72 on R-MAT s26 (ER 1.51 vs
+// 1.60 ms); sparse graphs (meshes, road-like) keep 512 / 8 / 72, whose row window holds their
+// many short rows (2-D mesh 0.64 vs 0.90 ms, road-like 0.58 vs 0.95 ms with 1024-entry tiles).
+#ifndef LM_SWEEP_DENSE_DEG
+#define LM_SWEEP_DENSE_DEG 10
+#endif
+#ifndef LM_SWEEP_S_TILE
+#define LM_SWEEP_S_TILE 512
+#endif
+#ifndef LM_SWEEP_S_WARPS
+#define LM_SWEEP_S_WARPS 8
+#endif
+#ifndef LM_SWEEP_S_WCAP
+#define LM_SWEEP_S_WCAP 72
+#endif
 #ifndef LM_SWEEP_TILE
-#define LM_SWEEP_TILE 512
+#define LM_SWEEP_TILE 1024
 #endif
 #ifndef LM_SWEEP_RING
 #define LM_SWEEP_RING 2
 #endif
 #ifndef LM_SWEEP_WARPS
-#define LM_SWEEP_WARPS 8
+#define LM_SWEEP_WARPS 6
 #endif
 #ifndef LM_SWEEP_WCAP
-#define LM_SWEEP_WCAP 72
+#define LM_SWEEP_WCAP 104
 #endif
 constexpr int kSweepTile = LM_SWEEP_TILE;    // entries per warp tile
 constexpr int kSweepRing = LM_SWEEP_RING;    // TMA stages per warp
@@ -99,9 +117,9 @@ using Sweep = lm::SweepCfg<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap>;
 #define SWEEP_KERNEL lm::k_sweep<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap>
 #endif
 // the round-1 sweep that also fills the resident key cache (opts.key_cache)
-#define SWEEP_KERNEL_KC lm::k_sweep<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap, false, true>
 constexpr int kSweepThreads = Sweep::kThreads;
-constexpr int64_t kTile = Sweep::kTile;
+using SweepD = lm::SweepCfg<LM_SWEEP_TILE, LM_SWEEP_RING, LM_SWEEP_WARPS, LM_SWEEP_WCAP>;      // dense
+using SweepS = lm::SweepCfg<LM_SWEEP_S_TILE, LM_SWEEP_RING, LM_SWEEP_S_WARPS, LM_SWEEP_S_WCAP>; // sparse
 #ifndef LM_COMPACT_K
 #define LM_COMPACT_K 8
 #endif
@@ -308,6 +326,8 @@ struct lmatch_graph {
   bool use_cache() const { return streaming && cache != nullptr; }
   cudaEvent_t ev_full[2] = {}, ev_free[2] = {};
   int sweep_grid = 0;
+  bool sweep_dense = true;   // round-1 sweep configuration: SweepD (true) or SweepS
+  int64_t tile = 1024;       // its entries per tile
   alignas(64) CUtensorMap tmap;  // adjacency as a [ceil(m/16)][16] u64 tensor, 128B swizzle
   int num_sms = 148;
   cudaAccessPolicyWindow bits_window = {};  // LM_L2_WINDOW: the matched bitmap, persisting
@@ -437,6 +457,44 @@ void drop_graph(lmatch_graph* g) {
 #endif
 static int64_t xrow_resets(const lmatch_graph* g) { return LM_XROW_RESET ? g->n_atomic : 0; }
 
+// ---- round-1 sweep launches in the handle's configuration (SweepD or SweepS)
+template <class C, bool ZAP, bool KC>
+static void sweep_launch_cfg(unsigned grid, cudaStream_t st, const lm::SweepArgs& A) {
+  lm::k_sweep<C::kTile, C::kRing, C::kWarps, C::kWin, ZAP, KC><<<grid, C::kThreads, C::kSmem, st>>>(A);
+}
+template <bool ZAP, bool KC>
+static void sweep_launch_any(const lmatch_graph* g, unsigned grid, cudaStream_t st, const lm::SweepArgs& A) {
+  if (g->sweep_dense) sweep_launch_cfg<SweepD, ZAP, KC>(grid, st, A);
+  else sweep_launch_cfg<SweepS, ZAP, KC>(grid, st, A);
+}
+static int sweep_warps(const lmatch_graph* g) { return g->sweep_dense ? SweepD::kWarps : SweepS::kWarps; }
+// dynamic shared memory opt-in of every sweep instantiation (once per process)
+template <class C>
+static cudaError_t sweep_attrs_cfg() {
+  cudaError_t e = cudaFuncSetAttribute(lm::k_sweep<C::kTile, C::kRing, C::kWarps, C::kWin, false, false>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::kSmem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(lm::k_sweep<C::kTile, C::kRing, C::kWarps, C::kWin, true, false>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::kSmem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(lm::k_sweep<C::kTile, C::kRing, C::kWarps, C::kWin, false, true>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::kSmem);
+  return e;
+}
+static cudaError_t sweep_attrs() {
+  cudaError_t e = sweep_attrs_cfg<SweepD>();
+  return e == cudaSuccess ? sweep_attrs_cfg<SweepS>() : e;
+}
+static cudaError_t sweep_occupancy(const lmatch_graph* g, int* occ) {
+  return g->sweep_dense
+             ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+                   occ, lm::k_sweep<SweepD::kTile, SweepD::kRing, SweepD::kWarps, SweepD::kWin, false, false>,
+                   SweepD::kThreads, SweepD::kSmem)
+             : cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+                   occ, lm::k_sweep<SweepS::kTile, SweepS::kRing, SweepS::kWarps, SweepS::kWin, false, false>,
+                   SweepS::kThreads, SweepS::kSmem);
+}
+
 int grid_for(int64_t work, int threads, int max_blocks) {
   int64_t b = (work + threads - 1) / threads;
   if (b < 1) b = 1;
@@ -476,6 +534,16 @@ int check_args(const void* a, const void* b, const void* c, int64_t n, int64_t m
 
 int alloc_all(lmatch_graph* g) {
   const int64_t n = g->n, m = g->m;
+#if LM_SWEEP_IMPL == 2
+  g->sweep_dense = true;
+  g->tile = kSweepTile;
+#else
+  // dense configuration when the average degree reaches LM_SWEEP_DENSE_DEG (rows per tile stay
+  // within its row window); the local part of a partition handle decides for itself
+  g->sweep_dense = n > 0 && m >= (int64_t)LM_SWEEP_DENSE_DEG * n;
+  g->tile = g->sweep_dense ? SweepD::kTile : SweepS::kTile;
+#endif
+  const int64_t kTile = g->tile;
   TRY(dmalloc(g, &g->offs, (size_t)n + 1));
   // out-of-core split: keep a prefix of R entries (multiple of the stream chunk) in HBM
   g->R = m;
@@ -569,7 +637,7 @@ int build_index(lmatch_graph* g, cudaStream_t st) {
   CK(cudaStreamSynchronize(st));
   if (g->ntiles > 0) {
     lm::k_tile_rows<<<grid_for(g->ntiles + 1, 256, 4096), 256, 0, st>>>(g->noffs, g->n_nz, g->ntiles,
-                                                                        kTile, g->tile_nz);
+                                                                        g->tile, g->tile_nz);
     CKL();
     lm::k_low32<<<grid_for(g->n_nz + 1, 256, 4096), 256, 0, st>>>(g->noffs, g->n_nz + 1, g->noffs_lo);
     CKL();
@@ -577,7 +645,7 @@ int build_index(lmatch_graph* g, cudaStream_t st) {
     TRY(dmalloc(g, &cnt, 1));
     CK(cudaMemsetAsync(cnt, 0, 8, st));
     lm::k_atomic_rows<<<grid_for(g->ntiles, 256, 4096), 256, 0, st>>>(
-        g->noffs, g->nzr, g->tile_nz, g->ntiles, kTile, g->atomic_rows, cnt);
+        g->noffs, g->nzr, g->tile_nz, g->ntiles, g->tile, g->atomic_rows, cnt);
     CKL();
     unsigned long long h_cnt = 0;
     CK(cudaMemcpyAsync(&h_cnt, cnt, 8, cudaMemcpyDeviceToHost, st));
@@ -833,7 +901,7 @@ int make_tensor_map(lmatch_graph* g) {
   }
   const cuuint64_t dims[2] = {16, (cuuint64_t)((g->m + 15) / 16)};
   const cuuint64_t strides[1] = {128};
-  const cuuint32_t box[2] = {16, (cuuint32_t)(kTile / 16)};
+  const cuuint32_t box[2] = {16, (cuuint32_t)(kSweepTile / 16)};
   const cuuint32_t es[2] = {1, 1};
   const CUresult r = encode(&g->tmap, CU_TENSOR_MAP_DATA_TYPE_UINT64, 2, g->adj, dims, strides, box,
                             es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
@@ -965,11 +1033,11 @@ int setup_key_cache(lmatch_graph* g, cudaStream_t st) {
   TRY(ensure(g, &g->xrows, &g->cap_xrows, g->ntiles + 1));
   if (!g->nx) TRY(dmalloc(g, &g->nx, 1));
   CK(cudaMemsetAsync(g->nx, 0, 8, st));
-  lm::k_kc_xrows<<<grid_for((g->n_nz + 31) & ~31ll, 256, 8192), 256, 0, st>>>(g->noffs, g->n_nz, kTile,
+  lm::k_kc_xrows<<<grid_for((g->n_nz + 31) & ~31ll, 256, 8192), 256, 0, st>>>(g->noffs, g->n_nz, g->tile,
                                                                               g->xrows, g->nx);
   CKL();
   if (!g->kc_attr) {
-    CK(cudaFuncSetAttribute(SWEEP_KERNEL_KC, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Sweep::kSmem));
+    CK(sweep_attrs());
     g->kc_attr = 1;
   }
   return LMATCH_OK;
@@ -1017,15 +1085,11 @@ int finish_create(lmatch_graph* g, cudaStream_t st) {
     CK(cudaMemsetAsync(g->werr, 0, 8, st));
     unsigned long long* zc = reinterpret_cast<unsigned long long*>(g->werr);
     if (!g->streaming && g->ntiles > 0) {
-      CK(cudaFuncSetAttribute(lm::k_sweep<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap, true>,
-                              cudaFuncAttributeMaxDynamicSharedMemorySize,
-                              (int)lm::SweepCfg<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap>::kSmem));
-      const int64_t grid = std::max<int64_t>(1, std::min<int64_t>((g->ntiles + kSweepWarps - 1) / kSweepWarps,
+      CK(sweep_attrs());
+      const int64_t grid = std::max<int64_t>(1, std::min<int64_t>((g->ntiles + sweep_warps(g) - 1) / sweep_warps(g),
                                                                   3 * (int64_t)g->num_sms));
       lm::SweepArgs A{g->adj, g->adj, zc, (uint32_t)g->v0, g->noffs_lo, g->nzr, g->tile_nz, g->best, g->m, 0, g->ntiles};
-      lm::k_sweep<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap, true>
-          <<<(unsigned)grid, 32 * kSweepWarps,
-             lm::SweepCfg<kSweepTile, kSweepRing, kSweepWarps, kSweepWcap>::kSmem, st>>>(A);
+      sweep_launch_any<true, false>(g, (unsigned)grid, st, A);
       CKL();
     } else {
       lm::k_zap_self_loops<<<grid_for(g->n * 8, 256, 16384), 256, 0, st>>>(g->offs, g->view(), g->n,
@@ -1038,13 +1102,18 @@ int finish_create(lmatch_graph* g, cudaStream_t st) {
   if (g->ntiles > 0) TRY(make_tensor_map(g));
 #endif
   if (g->ntiles > 0) {
+    int occ = 0;
+#if LM_SWEEP_IMPL == 2
     CK(cudaFuncSetAttribute(SWEEP_KERNEL,
                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)Sweep::kSmem));
-    int occ = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(
         &occ, SWEEP_KERNEL, kSweepThreads, Sweep::kSmem));
+#else
+    CK(sweep_attrs());
+    CK(sweep_occupancy(g, &occ));
+#endif
     if (occ < 1) occ = 1;
-    g->sweep_grid = (int)std::min<int64_t>((g->ntiles + kSweepWarps - 1) / kSweepWarps,
+    g->sweep_grid = (int)std::min<int64_t>((g->ntiles + sweep_warps(g) - 1) / sweep_warps(g),
                                            (int64_t)occ * g->num_sms);
   }
   CK(cudaStreamSynchronize(st));
@@ -1142,16 +1211,16 @@ int round1_sweep(lmatch_graph* g, cudaStream_t st, int64_t* launches_out, int64_
 #else
   // resident tiles [0, R/TILE), then the streamed chunks through a 2-slot device ring:
   // the copy of chunk k+1 (copy stream) overlaps the sweep of chunk k (run stream).
-  const int64_t rt = g->streaming ? g->R / kTile : g->ntiles;
+  const int64_t rt = g->streaming ? g->R / g->tile : g->ntiles;
   auto sweep_launch = [&](const uint64_t* base, int64_t t0, int64_t t1) -> int {
-    const int64_t grid = std::min<int64_t>((t1 - t0 + kSweepWarps - 1) / kSweepWarps, g->sweep_grid);
+    const int64_t grid = std::min<int64_t>((t1 - t0 + sweep_warps(g) - 1) / sweep_warps(g), g->sweep_grid);
     lm::SweepArgs A{base, nullptr, nullptr, 0u, g->noffs_lo, g->nzr, g->tile_nz, g->best, g->m, t0, t1};
     if (g->kcache) {
       A.kc = g->kcache;
       A.xpart = g->xpart;
-      SWEEP_KERNEL_KC<<<(unsigned)std::max<int64_t>(grid, 1), kSweepThreads, Sweep::kSmem, st>>>(A);
+      sweep_launch_any<false, true>(g, (unsigned)std::max<int64_t>(grid, 1), st, A);
     } else {
-      SWEEP_KERNEL<<<(unsigned)std::max<int64_t>(grid, 1), kSweepThreads, Sweep::kSmem, st>>>(A);
+      sweep_launch_any<false, false>(g, (unsigned)std::max<int64_t>(grid, 1), st, A);
     }
     CKL();
     ++launches;
@@ -1162,7 +1231,7 @@ int round1_sweep(lmatch_graph* g, cudaStream_t st, int64_t* launches_out, int64_
   if (g->kcache && rt > 0) {
     // the rows crossing a tile boundary: merge their per-tile top-4 lists (also their pointer)
     lm::k_kc_merge<<<(unsigned)(8 * g->num_sms), 256, 0, st>>>(g->xrows, g->nx, g->noffs, g->nzr, g->xpart,
-                                                               kTile, g->kcache, g->best);
+                                                               g->tile, g->kcache, g->best);
     CKL();
     ++launches;
   }
@@ -1193,7 +1262,7 @@ int round1_sweep(lmatch_graph* g, cudaStream_t st, int64_t* launches_out, int64_
       CK(cudaEventRecord(g->ev_full[slot], g->cs));
       bytes_streamed += cnt * 8;
       CK(cudaStreamWaitEvent(st, g->ev_full[slot], 0));
-      TRY(sweep_launch(g->ring[slot], e0 / kTile, std::min(g->ntiles, (e0 + cnt + kTile - 1) / kTile)));
+      TRY(sweep_launch(g->ring[slot], e0 / g->tile, std::min(g->ntiles, (e0 + cnt + g->tile - 1) / g->tile)));
       if (g->use_cache())
         TRY(cache_fill(g->ring[slot], e0, e0, e0 + cnt, g->chunk_rows + k, g->chunk_rows + k + 1));
       CK(cudaEventRecord(g->ev_free[slot], st));
@@ -1214,6 +1283,7 @@ extern "C" {
 int lmatch_abi_version(void) { return LMATCH_ABI_VERSION; }
 
 int64_t lmatch_kernel_launch_count(void) { return (int64_t)g_launch_count.load(); }
+int32_t lmatch_sweep_tile(const lmatch_graph* g) { return g ? (int32_t)g->tile : (int32_t)SweepD::kTile; }
 
 const char* lmatch_strerror(int status) {
   switch (status) {
