@@ -21,9 +21,4 @@ python bench.py --no-cpu --no-e2e --steps 5 --scale 29 > $O/bench_rmat_s29.json 
 python bench.py --no-cpu --no-e2e --steps 5 --scale 29 --partitioned > $O/bench_rmat_s29_partitioned_n1.json 2> $O/bench_rmat_s29_partitioned_n1.err
 python bench.py --no-cpu --gpus 2 --steps 5 > $O/bench_rmat_s26_2ranks_1gpu.json 2> $O/bench_rmat_s26_2ranks_1gpu.err
 ls -la $O
-# compute-sanitizer on the final build (every code path on small graphs, each result oracle-checked)
-for tool in memcheck synccheck initcheck; do
-  timeout 1500 compute-sanitizer --tool $tool python scripts/sanitize_run.py > $O/sanitizer_$tool.log 2>&1; echo "exit=$?" >> $O/sanitizer_$tool.log
-done
-timeout 1500 compute-sanitizer --tool racecheck python scripts/sanitize_run.py --quick --single > $O/sanitizer_racecheck.log 2>&1; echo "exit=$?" >> $O/sanitizer_racecheck.log
 ls -la $O
