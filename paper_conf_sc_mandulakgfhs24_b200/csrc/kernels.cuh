@@ -549,16 +549,32 @@ constexpr int kKC = LM_KC;
 static_assert(kKC == 2 || kKC == 4, "key cache width must be 2 or 4");
 // top-2 update of a descending pair (t0 >= t1): branch-free, two u64 max and one u64 min
 __device__ __forceinline__ void top2_insert(uint64_t& t0, uint64_t& t1, uint64_t k) {
+#if LM_SWEEP_DMAX
+  // the same key order on the FP64 pipe (see kmax64)
+  const double d = kd_of(k), a0 = kd_of(t0), a1 = kd_of(t1);
+  const double lo = d < a0 ? d : a0;
+  t1 = ku_of(lo > a1 ? lo : a1);
+  t0 = ku_of(d > a0 ? d : a0);
+#else
   const uint64_t lo = k < t0 ? k : t0;
   t1 = lo > t1 ? lo : t1;
   t0 = k > t0 ? k : t0;
+#endif
 }
 // merge two descending pairs into the descending top-2 of their union
 __device__ __forceinline__ void top2_merge(uint64_t& t0, uint64_t& t1, uint64_t o0, uint64_t o1) {
+#if LM_SWEEP_DMAX
+  const double a0 = kd_of(t0), a1 = kd_of(t1), b0 = kd_of(o0), b1 = kd_of(o1);
+  const double lo = b0 < a0 ? b0 : a0;
+  const double hi1 = b1 > a1 ? b1 : a1;
+  t1 = ku_of(lo > hi1 ? lo : hi1);
+  t0 = ku_of(b0 > a0 ? b0 : a0);
+#else
   const uint64_t lo = o0 < t0 ? o0 : t0;
   const uint64_t hi1 = o1 > t1 ? o1 : t1;
   t1 = lo > hi1 ? lo : hi1;
   t0 = o0 > t0 ? o0 : t0;
+#endif
 }
 // insert key k into the descending list t0 >= t1 >= t2 >= t3 (keeps the kKC largest)
 __device__ __forceinline__ void top4_insert(uint64_t& t0, uint64_t& t1, uint64_t& t2, uint64_t& t3,
